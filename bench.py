@@ -1,0 +1,345 @@
+#!/usr/bin/env python
+"""bench.py — DGR differentiable DAG-forest solver on B200 (driver contract).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl dgr|reference] [--config ispd19]
+
+A "step" is one solver iteration: every per-iteration row of SURVEY §8(a) (Gumbel-softmax,
+demand scatter, loss + gradient map, reverse pass, Adam) over the whole synthetic forest;
+induction (row 6, once per solve) is timed separately (`induce_ms`).  Default workload:
+BASELINE.json configs[3] (ISPD'19-shaped, ~1e6 nets, 1000x1000), the config the north-star
+target and the 1/2/4/8-GPU metric are quoted on.  For N > 1 (torchrun) the same forest is
+sharded over the ranks (strong scaling) with one NCCL allreduce of the demand per iteration.
+
+--impl reference runs the CPU oracle (oracle/, fp64, single thread) on rank 0 on a bounded
+sample of the same workload; other ranks exit 0 without work.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import platform
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+BETA1 = 0.9
+HBM_FALLBACK_GBS = 6650.0   # /opt/skills/guides/B200_PROFILING.md fallback (only if MEASURED_PEAKS.json is absent)
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--impl", default="dgr", choices=["dgr", "reference"])
+    ap.add_argument("--config", default="ispd19")
+    ap.add_argument("--no-quality", action="store_true", help="skip the full 1000-iteration solve")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+def measured_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as fh:
+            m = json.load(fh)
+        return float(m["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy kernel)"
+    return HBM_FALLBACK_GBS, "fallback (B200_PROFILING.md)"
+
+
+# --------------------------------------------------------------------------------------------
+# algorithmic bytes per launch of each stage: minimal reads + writes of the data
+# each stage must touch once; padding slots, re-reads and atomics' RMW are overhead, not counted.
+# --------------------------------------------------------------------------------------------
+def stage_bytes(st: dict) -> dict:
+    P, S, T, N, B, V = st["paths"], st["subnets"], st["trees"], st["nets"], st["bundles"], st["cells"]
+    return {
+        "KQ": 4 * N + 8 * T,                               # net offsets; w_tree read, q write
+        "zero": 24 * V,                                    # dH, dV, VD cleared
+        "KF": 8 * P + 8 * S + 4 * T + 16 * B + 24 * V,     # w, pword; endpoints; q; bundle info; 3 grids written
+        "allreduce": 0,
+        "KG": 48 * V,                                      # dH dV VD read, capH capV read, S_H S_V written
+        "KB": 28 * P + 8 * S + 12 * T + 16 * B + 16 * V,   # w m v r+w, pword; endpoints; q, dq; S_H S_V read
+        "KT": 4 * N + 44 * T,                              # offsets; q, dq r/w, w m v r/w
+    }
+
+
+class Clocks:
+    """nvidia-smi sampler for the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), "--query-gpu=clocks.sm,clocks.max.sm,power.draw,"
+                 "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0])); mx = float(parts[1])
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[3:7]):
+                if v.lower() in ("active", "1"):
+                    reasons.add(n)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        load = [s for s in sm if s > 0.5 * (mx or max(sm))] or sm
+        return {"sm_mhz": float(np.median(load)), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", 0)); world = int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    return rank, world, local
+
+
+def paper_schedule_quality(s, W):
+    """The paper's schedule: 1000 iterations, t0 = 1 x 0.9 every 100, Adam lr 0.3; then
+    argmax tree + top-p paths.  Returns the induced-solution metrics."""
+    for k in range(10):
+        s.step(100, 0.9 ** k, 0.3, W, want_loss=False)
+    r = s.induce(0.9)
+    return {"overflow": float(r.metrics[0]), "overflowed_edges": int(r.metrics[1]), "max_overflow": float(r.metrics[2]),
+            "wl": float(r.metrics[3]), "tp": float(r.metrics[4]), "iterations": 1000, "top_p": 0.9}
+
+
+def cpu_baseline(f, seconds_target=12.0):
+    """The oracle as it stands (fp64, single thread) on this host on a bounded sample: whole-forest
+    iterations of the same workload until ~seconds_target of CPU work."""
+    import oracle
+    o = oracle.Oracle(f)
+    W = oracle.weights()
+    t0 = time.perf_counter()
+    o.step(1, 1.0, 0.3, W)                      # one untimed iteration (page-in)
+    first = time.perf_counter() - t0
+    n = max(1, min(20, int(seconds_target / max(first, 1e-3))))
+    t0 = time.perf_counter()
+    o.step(n, 1.0, 0.3, W)
+    dt = time.perf_counter() - t0
+    return {"value": n / dt, "unit": "iters/s", "cores": 1, "kind": "oracle",
+            "sample": f"{n} full iterations of the same {f.n_nets}-net forest (fp64, single thread, "
+                      f"{platform.processor() or platform.machine()}, nproc={os.cpu_count()})",
+            "path_cand_per_s": n / dt * f.n_paths}
+
+
+def run_reference(args):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return
+    import forestgen
+    import oracle
+    f = forestgen.generate(args.config)
+    o = oracle.Oracle(f)
+    W = oracle.weights()
+    t0 = time.perf_counter()
+    o.step(1, 1.0, 0.3, W)
+    per = time.perf_counter() - t0
+    # bound the run to ~3 minutes: whole-forest iterations if they fit, else a net-shard sample
+    budget = 180.0
+    total_steps = args.steps + args.warmup
+    frac = min(1.0, budget / max(per * total_steps, 1e-9))
+    if frac < 1.0:
+        hi = max(1, int(f.n_nets * frac))
+        o.set_shard(0, hi)
+        sample = f"each step = one oracle iteration over nets [0,{hi}) of {f.n_nets} ({frac:.3f} of the forest; full grid pass), scaled by the net fraction"
+    else:
+        sample = f"each step = one full oracle iteration over all {f.n_nets} nets"
+    for _ in range(args.warmup):
+        o.step(1, 1.0, 0.3, W)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        o.step(1, 1.0, 0.3, W)
+    dt = time.perf_counter() - t0
+    value = args.steps / dt * frac
+    line = {"metric": "DAG-forest solver iters/sec", "value": value, "unit": "iters/s", "impl": "reference",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": args.config, "nets": f.n_nets, "paths": f.n_paths},
+            "path_cand_per_s": value * f.n_paths,
+            "cpu_baseline": {"value": value, "unit": "iters/s", "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": "iters/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import torch
+    import torch.distributed as tdist
+
+    import forestgen
+    import paper_conf_dac_0159layhrr24_b200 as dgr
+
+    rank, world, local = dist_env()
+    if world != args.gpus:
+        print(f"warning: --gpus {args.gpus} but WORLD_SIZE {world}; using WORLD_SIZE", file=sys.stderr)
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    nccl_id = None
+    if world > 1:
+        tdist.init_process_group("nccl", device_id=dev)
+        buf = torch.zeros(128, dtype=torch.uint8, device=dev)
+        if rank == 0:
+            buf.copy_(torch.frombuffer(bytearray(dgr.nccl_unique_id()), dtype=torch.uint8))
+        tdist.broadcast(buf, 0)
+        nccl_id = bytes(buf.cpu().numpy().tobytes())
+
+    def barrier():
+        if world > 1:
+            tdist.barrier(device_ids=[local])
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+        return float(t.item())
+
+    f = forestgen.generate(args.config)
+    W = dgr.Weights()
+    stream = torch.cuda.current_stream(dev)
+
+    # ---------------- e2e: one solve through the public API from host buffers ----------------
+    barrier(); torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    s = dgr.Solver(f, rank=rank, world=world, nccl_id=nccl_id, device=dev, stream=stream)  # H2D of the forest
+    h2d = s.host_input_bytes()
+    d2h = 0
+    for _ in range(args.warmup + args.steps):
+        s.step(1, 1.0, 0.3, W, want_loss=True)     # loss read back every iteration (32 B)
+        d2h += 32
+    dh, dv = s.demand()
+    d2h += dh.nbytes + dv.nbytes
+    torch.cuda.synchronize()
+    e2e_s = max_over_ranks(time.perf_counter() - t0)
+    e2e_iters = args.warmup + args.steps
+    s.close()
+    del s
+
+    # ---------------- device-timed region: K iterations, inputs resident in HBM ----------------
+    s = dgr.Solver(f, rank=rank, world=world, nccl_id=nccl_id, device=dev, stream=stream)
+    info = s.info()
+    s.step(max(3, args.warmup), 1.0, 0.3, W, want_loss=False)
+    ev0 = torch.cuda.Event(enable_timing=True); ev1 = torch.cuda.Event(enable_timing=True)
+    with Clocks(local) as clk:
+        barrier(); torch.cuda.synchronize()
+        ev0.record(stream)
+        s.step(args.steps, 1.0, 0.3, W, want_loss=False)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ms = max_over_ranks(ev0.elapsed_time(ev1))
+        # the same K iterations again with per-stage CUDA events on the launching stream
+        s.profile(True)
+        s.step(args.steps, 1.0, 0.3, W, want_loss=False)
+        stage_ms, n_prof = s.profile_read()
+        s.profile(False)
+    clocks = clk.summary()
+    loss = s.step(0, 1.0, 0.3, W)
+    t_ind0 = time.perf_counter(); s.induce(0.9); induce_ms = (time.perf_counter() - t_ind0) * 1e3
+    quality = None if args.no_quality else paper_schedule_quality(s, W)
+
+    cells = f.X * f.Y
+    st = dict(paths=f.n_paths, subnets=f.n_subnets, trees=f.n_trees, nets=f.n_nets, bundles=info["n_bundles"],
+              cells=cells)
+    if world > 1:   # this rank's share of the per-candidate work
+        lo, hi = info["net_hi"] - (info["net_hi"] - info["net_lo"]), info["net_hi"]
+        t0_, t1_ = f.net_tree_off[lo], f.net_tree_off[hi]
+        s0_, s1_ = f.tree_sub_off[t0_], f.tree_sub_off[t1_]
+        st.update(paths=int(f.sub_path_off[s1_] - f.sub_path_off[s0_]), subnets=int(s1_ - s0_), trees=int(t1_ - t0_),
+                  nets=int(hi - lo))
+    sb = stage_bytes(st)
+    per_iter_ms = {k: v / max(n_prof, 1) for k, v in stage_ms.items()}
+    mine = {k: v for k, v in per_iter_ms.items() if k not in ("zero", "allreduce")}
+    dom = max(mine, key=mine.get)
+    peak, peak_src = measured_peak()
+    achieved = sb[dom] / (per_iter_ms[dom] * 1e-3) / 1e9
+    traffic = None
+    summ = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(summ):
+        with open(summ) as fh:
+            traffic = json.load(fh).get(args.config, {}).get(dom)
+    iters_per_s = args.steps / (ms * 1e-3)
+    alg_iter = sum(sb.values())
+    line = {
+        "metric": "DAG-forest solver iters/sec (path-cand/s, overflow, WL alongside)",
+        "value": iters_per_s, "unit": "iters/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+        "dtype": "f32", "data": "synthetic",
+        "config": {"workload": f"{args.config} (BASELINE.json configs[3]: ISPD'19-shaped congested synthetic)",
+                   "grid": f"{f.X}x{f.Y}", "nets": f.n_nets, "trees": f.n_trees, "subnets": f.n_subnets,
+                   "paths": f.n_paths, "segments": f.n_segs, "turning_points": f.n_tps,
+                   "step": "one solver iteration (softmax, scatter, loss/gradient map, reverse, Adam); induction timed separately",
+                   "l2": f"inputs larger than L2: {info['workspace_bytes'] / 1e6:.0f} MB resident state per rank touched every iteration > 126 MB L2",
+                   "parallelism": f"dp{world} (nets sharded, demand allreduce)" if world > 1 else "single GPU"},
+        "path_cand_per_s": iters_per_s * f.n_paths,
+        "iteration_roofline": {"alg_bytes": alg_iter, "achieved_gbs": alg_iter * iters_per_s / 1e9, "peak": peak,
+                               "frac": alg_iter * iters_per_s / 1e9 / peak},
+        "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                     "alg_bytes_per_launch": sb[dom], "avg_launch_ms": per_iter_ms[dom]},
+        "stage_ms_per_iter": per_iter_ms,
+        "gpu_launches": 6 * args.steps,
+        "clocks": clocks,
+        "induce_ms": induce_ms,
+        "loss": {"total": float(loss[0]), "wl": float(loss[1]), "via": float(loss[2]), "overflow": float(loss[3])},
+        "quality": quality,
+        "hbm_footprint_bytes": info["workspace_bytes"],
+        "e2e": {"value": e2e_iters / e2e_s, "unit": "iters/s", "h2d_bytes_per_step": h2d / e2e_iters,
+                "d2h_bytes_per_step": d2h / e2e_iters,
+                "note": f"one solve from host CSR arrays through the C ABI: dgr_forest_load (H2D {h2d} B, host "
+                        f"validation + encoding) + {e2e_iters} x dgr_step(1) with the loss read back each "
+                        f"iteration + dgr_get_demand; wall clock, max over ranks"},
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(f)
+    s.close()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        tdist.barrier(device_ids=[local])
+        tdist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

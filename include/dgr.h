@@ -1,0 +1,160 @@
+/* dgr.h — C ABI of libdgr: the B200 (sm_100a) DGR differentiable DAG-forest solver.
+ *
+ * The operation: PAPER.md (DGR, DAC'24) §4.3-4.5.  One solver iteration (dgr_step) is
+ *   (1) Gumbel-softmax over every net's routing-tree candidates and every 2-pin sub-net's
+ *       path candidates                                      §4.4
+ *   (2) expected demand on the H/V G-cell edges, Eq. (10)
+ *   (3) cost = a1 WL + a2 via + a3 overflow, Eqs. (9),(11),(12)
+ *   (4) its gradient w.r.t. the logits (the paper uses autograd)
+ *   (5) Adam on the logits
+ * and dgr_induce is the discrete selection of §4.5 (argmax tree, top-p paths).
+ * The readings of the paper this library implements are listed in DESIGN.md §3
+ * (grouping = sub-net, f = sigmoid(-s r) / ReLU(-r), beta_v global, sqrt(L) with L = n_layers,
+ * Philox4x32-10 noise keyed on (seed, global candidate index, iteration, stream)).
+ *
+ * Conventions for every entry point
+ *   - return int: 0 = DGR_OK, < 0 = error code below; dgr_last_error() (thread-local) says why.
+ *     No C++ exception crosses this boundary.  An error leaves no partial state behind.
+ *   - host pointers are caller-owned, read during the call only (inputs are copied at load).
+ *   - the device workspace is caller-owned memory (e.g. a torch uint8 CUDA tensor) of at least
+ *     dgr_workspace_size() bytes that must outlive the handle; its layout is library-owned.
+ *   - all work is ordered on the cudaStream_t passed to dgr_forest_load; calls that return
+ *     data to the host synchronise that stream.
+ *   - a handle is not thread-safe.  With world > 1 there is one process per GPU, each with its
+ *     own handle, and dgr_step / dgr_induce are collective over the ranks (NCCL).
+ *
+ * Geometry (identical to include/forestgen.h)
+ *   G-cell grid X x Y.  H edge (x,y)-(x+1,y), x in [0,X-2]; V edge (x,y)-(x,y+1), y in [0,Y-2].
+ *   Grids are row-major [Y][X]; the last column (H) / last row (V) is padding.
+ *   Segment {dir (0 = H, 1 = V), line (y for H, x for V), lo, hi}: the edges [lo,hi) of the line.
+ *   Every path candidate must be one of the patterns of its sub-net (x0,y0)-(x1,y1): the
+ *   straight path, HV / VH L-shapes, Z-HVH (interior x_m) or Z-VHV (interior y_m) (§3.1,
+ *   P:313-315; §4.2); each sub-net has 1..32 candidates.
+ */
+#ifndef DGR_H
+#define DGR_H
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+  DGR_OK = 0,
+  DGR_EINVAL = -1,   /* invalid argument or malformed forest (nothing was allocated or changed) */
+  DGR_ECUDA = -2,    /* a CUDA runtime call failed */
+  DGR_ENCCL = -3,    /* an NCCL call failed */
+  DGR_ENOMEM = -4,   /* workspace too small / host allocation failed */
+  DGR_ESTATE = -5    /* call not valid in the handle's state (e.g. dgr_get_demand before a forward) */
+};
+
+/* Message for the last error on this thread ("" if none). */
+const char* dgr_last_error(void);
+
+/* The routing DAG forest F = {T, S, P} of §3.2 as flat CSR arrays, in GLOBAL order.
+ * Offsets have length n+1, start at 0 and are non-decreasing; every group is non-empty. */
+typedef struct {
+  int32_t X, Y;                           /* grid; 2..32767 each */
+  int64_t n_nets, n_trees, n_subnets, n_paths, n_segs, n_tps;
+  const int64_t* net_tree_off;            /* net -> its routing-tree candidates (T) */
+  const int64_t* tree_sub_off;            /* tree -> its 2-pin sub-nets (S) */
+  const int64_t* sub_path_off;            /* sub-net -> its path candidates (P), 1..32 each */
+  const int64_t* path_seg_off;            /* path -> its segments */
+  const int64_t* path_tp_off;             /* path -> its turning points */
+  const int32_t* seg;                     /* n_segs x {dir, line, lo, hi} */
+  const int32_t* tp_xy;                   /* n_tps x {x, y} */
+  const int32_t* sub_xy;                  /* n_subnets x {x0, y0, x1, y1} (either orientation) */
+  const float* cap_h;                     /* [Y][X] capacity of H edges, Eq. (1) */
+  const float* cap_v;                     /* [Y][X] capacity of V edges */
+  const float* w_tree0;                   /* [n_trees] initial logits w */
+  const float* w_path0;                   /* [n_paths] */
+  uint64_t seed;                          /* Philox key of the Gumbel noise */
+} dgr_forest_desc;
+
+/* Multi-GPU: one process per GPU.  rank 0 calls dgr_nccl_unique_id and broadcasts the 128
+ * bytes (e.g. over torch.distributed); every rank passes them here. NULL or world == 1: single GPU. */
+typedef struct {
+  int32_t rank, world;
+  const void* nccl_unique_id;             /* 128 bytes */
+} dgr_dist;
+
+/* Cost weights and model constants. */
+typedef struct {
+  float a_wl, a_via, a_of;   /* a1, a2, a3 of Eq. (3); paper: 0.5, 4, 500 */
+  float beta_via;            /* beta_v of Eqs. (2)/(10), one global value (Q3; default 0.25) */
+  float n_layers;            /* L in sqrt(L) of Eqs. (5)/(12) (Q4; default 5) */
+  int32_t f_kind;            /* overflow function f of Eq. (9): 0 = sigmoid, 1 = ReLU */
+  float f_slope;             /* s in f(r) = 1 / (1 + exp(s r)) (Q2; default 1) */
+} dgr_weights;
+
+/* Loss of a forward pass: total = a_wl*wl + a_via*via + a_of*overflow, with
+ * wl = E[WL] (Eq. 11), via = sqrt(L) E[TP] (Eq. 12), overflow = sum_e f(cap_e - d_e) (Eq. 9). */
+typedef struct { double total, wl, via, overflow; } dgr_loss;
+
+struct dgr_handle;
+
+/* Writes the 128-byte ncclUniqueId (call on rank 0 only). */
+int dgr_nccl_unique_id(void* out128);
+
+/* Contiguous net ranges [out[r], out[r+1]) for `world` ranks, balanced on the candidate work
+ * (paths + segments) of each net; out has world+1 entries.  Host-only, no GPU needed. */
+int dgr_partition(const dgr_forest_desc* desc, int32_t world, int64_t* out);
+
+/* Bytes of device workspace this rank needs for desc (0 on error; see dgr_last_error). */
+int64_t dgr_workspace_size(const dgr_forest_desc* desc, const dgr_dist* dist);
+
+/* Validates desc, keeps this rank's nets (dgr_partition), encodes them for the device, copies
+ * them into dev_workspace (>= dgr_workspace_size bytes, 256-byte aligned) on cuda_stream
+ * (a cudaStream_t; NULL = legacy default stream), zeroes Adam state and the iteration counter k.
+ * With world > 1 this also creates the NCCL communicator (collective).  Synchronises. */
+int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev_workspace,
+                    int64_t workspace_bytes, void* cuda_stream, struct dgr_handle** out);
+
+/* Runs `iters` solver iterations at temperature t and Adam learning rate lr: each is
+ * forward (steps 1-3), reverse (step 4) and Adam (step 5), with k incremented after each.
+ * iters == 0 runs one forward only (no update, k unchanged).  The Gumbel noise of iteration k
+ * is keyed on the global k, so 10 calls of 100 iterations equal 1 call of 1000 at equal t.
+ * If `last` is non-NULL it receives the loss of the last forward (synchronises). */
+int dgr_step(struct dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w,
+             dgr_loss* last);
+
+/* Demand d_e (Eq. 10) of the last forward, full grids [Y][X] (H padding column / V padding
+ * row are 0).  With world > 1 this is the global (all-rank) demand.  Synchronises. */
+int dgr_get_demand(struct dgr_handle* h, float* d_h, float* d_v);
+
+/* Current logits in GLOBAL order.  With world > 1 only this rank's entries are written. */
+int dgr_get_logits(struct dgr_handle* h, float* w_tree, float* w_path);
+
+/* Discrete selection of §4.5 from the current logits at the temperature of the last dgr_step
+ * (noise-free softmax): tree_choice[n] = global index of argmax_j q_hat (ties: lowest index);
+ * for each sub-net of a chosen tree the paths ranked by p_hat descending (ties: lowest index),
+ * the nucleus = the smallest prefix whose cumulative p_hat reaches top_p (at least one path),
+ * route[s] = its first path (global index), -1 for sub-nets of unchosen trees.
+ * nucleus_off [n_subnets+1] / nucleus (capacity n_paths) hold the nuclei as CSR in sub-net order.
+ * D_h, D_v [Y][X]: integer wire demand of the routes; metrics = {sum_e max(0, D_e + beta V_e -
+ * cap_e), number of edges where that is > 0, its maximum, sum WL, sum TP} of the routes, V_e =
+ * route turning points at e's end cells.  With world > 1, entries outside this rank's nets are
+ * -1 / empty and D_h, D_v, metrics are global.  Synchronises. */
+int dgr_induce(struct dgr_handle* h, float top_p, int32_t* tree_choice, int32_t* route,
+               int64_t* nucleus_off, int32_t* nucleus, int32_t* D_h, int32_t* D_v, double metrics[5]);
+
+/* Introspection: iteration counter k, this rank's net range, encoded sizes.  info[8] =
+ * {k, net_lo, net_hi, n_bundles, n_path_slots, workspace_bytes, world, rank}. */
+int dgr_get_info(struct dgr_handle* h, int64_t info[8]);
+
+/* Per-stage device time of subsequent dgr_step calls, from CUDA events recorded on the handle's
+ * stream between the stages.  enable != 0 starts (and clears) recording, 0 stops it.
+ * dgr_profile_read synchronises and returns, for the stages
+ *   0 KQ (tree softmax), 1 demand-buffer zeroing (cudaMemsetAsync), 2 KF (path softmax + scatter),
+ *   3 demand allreduce (NCCL; world > 1 only), 4 KG (scan/loss/gradient map, 2 kernels),
+ *   5 KB (reverse + Adam), 6 KT (tree reverse + Adam), 7 unused
+ * the summed milliseconds and the number of iterations recorded. */
+int dgr_profile(struct dgr_handle* h, int32_t enable);
+int dgr_profile_read(struct dgr_handle* h, double ms[8], int64_t* iterations);
+
+/* Releases the handle (and the NCCL communicator); the workspace stays the caller's. */
+int dgr_free(struct dgr_handle* h);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

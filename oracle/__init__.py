@@ -28,14 +28,16 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "dgr_oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
-_lib = None
+_LIB32 = os.path.join(_HERE, "liboracle32.so")   # conditioning probe only (same source, real = float)
+_libs = {}
 
 
 def build(verbose: bool = False) -> str:
-    cmd = ["gcc", "-O2", "-std=c11", "-shared", "-fPIC", "-o", _LIB, _SRC, "-lm"]
-    if verbose:
-        print(" ".join(cmd))
-    subprocess.check_call(cmd)
+    for out, extra in ((_LIB, []), (_LIB32, ["-DODGR_REAL=float"])):
+        cmd = ["gcc", "-O2", "-std=c11", "-shared", "-fPIC", *extra, "-o", out, _SRC, "-lm"]
+        if verbose:
+            print(" ".join(cmd))
+        subprocess.check_call(cmd)
     return _LIB
 
 
@@ -57,12 +59,12 @@ _f32 = np.ctypeslib.ndpointer(dtype=np.float32, flags="C_CONTIGUOUS")
 _u32 = np.ctypeslib.ndpointer(dtype=np.uint32, flags="C_CONTIGUOUS")
 
 
-def _load():
-    global _lib
-    if _lib is None:
-        if not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+def _load(fp32: bool = False):
+    path = _LIB32 if fp32 else _LIB
+    if path not in _libs:
+        if not os.path.exists(path) or os.path.getmtime(path) < os.path.getmtime(_SRC):
             build()
-        L = ctypes.CDLL(_LIB)
+        L = ctypes.CDLL(path)
         vp, c = ctypes.c_void_p, ctypes
         L.odgr_philox4x32_10.argtypes = [_u32, _u32, _u32]
         L.odgr_uniform.argtypes = [c.c_uint64, c.c_uint64, c.c_uint64, c.c_uint32]
@@ -95,8 +97,9 @@ def _load():
         L.odgr_get_demand.argtypes = [vp, _dp, _dp]
         L.odgr_induce.argtypes = [vp, c.c_double, c.c_double, c.c_double, _i32, _i32, _i64, _i32, _i32, _i32,
                                   _dp, _dp, _dp, _dp]
-        _lib = L
-    return _lib
+        L.odgr_real_bytes.restype = c.c_int32
+        _libs[path] = L
+    return _libs[path]
 
 
 def philox4x32_10(ctr, key) -> np.ndarray:
@@ -128,10 +131,14 @@ class InduceResult:
 
 
 class Oracle:
-    """fp64 CPU oracle over a ``forestgen.Forest``."""
+    """fp64 CPU oracle over a ``forestgen.Forest``.
 
-    def __init__(self, f):
-        L = _load()
+    ``fp32=True`` loads the same source compiled with ``real = float``: NOT a reference, only the
+    conditioning probe that marks outputs fp32 arithmetic cannot pin to the tolerance."""
+
+    def __init__(self, f, fp32: bool = False):
+        self._L = L = _load(fp32)
+        self.fp32 = fp32
         self.f = f
         self.X, self.Y = f.X, f.Y
         self._h = L.odgr_new(
@@ -148,78 +155,78 @@ class Oracle:
 
     def __del__(self):
         if getattr(self, "_h", None):
-            _load().odgr_free(self._h)
+            self._L.odgr_free(self._h)
             self._h = None
 
     # --- state -------------------------------------------------------------------
     @property
     def iteration(self) -> int:
-        return _load().odgr_iteration(self._h)
+        return self._L.odgr_iteration(self._h)
 
     @iteration.setter
     def iteration(self, k: int):
-        _load().odgr_set_iteration(self._h, k)
+        self._L.odgr_set_iteration(self._h, k)
 
     def set_shard(self, lo: int, hi: int):
-        _load().odgr_set_shard(self._h, lo, hi)
+        self._L.odgr_set_shard(self._h, lo, hi)
 
     def logits(self):
         wt = np.zeros(self.f.n_trees); wp = np.zeros(self.f.n_paths)
-        _load().odgr_get_logits(self._h, wt, wp)
+        self._L.odgr_get_logits(self._h, wt, wp)
         return wt, wp
 
     def set_logits(self, wt, wp):
-        _load().odgr_set_logits(self._h, np.ascontiguousarray(wt, np.float64), np.ascontiguousarray(wp, np.float64))
+        self._L.odgr_set_logits(self._h, np.ascontiguousarray(wt, np.float64), np.ascontiguousarray(wp, np.float64))
 
     def adam_state(self):
         a = [np.zeros(self.f.n_trees), np.zeros(self.f.n_trees), np.zeros(self.f.n_paths), np.zeros(self.f.n_paths)]
-        _load().odgr_get_adam(self._h, *a)
+        self._L.odgr_get_adam(self._h, *a)
         return a
 
     def probs(self):
         q = np.zeros(self.f.n_trees); p = np.zeros(self.f.n_paths)
-        _load().odgr_get_probs(self._h, q, p)
+        self._L.odgr_get_probs(self._h, q, p)
         return q, p
 
     def demand(self):
         dh = np.zeros((self.Y, self.X)); dv = np.zeros((self.Y, self.X))
-        _load().odgr_get_demand(self._h, dh, dv)
+        self._L.odgr_get_demand(self._h, dh, dv)
         return dh, dv
 
     # --- the iteration -------------------------------------------------------------
     def forward(self, t: float, w: Weights, noise: bool = True) -> np.ndarray:
         out = np.zeros(4)
-        _load().odgr_forward(self._h, t, ctypes.byref(w), int(noise), out)
+        self._L.odgr_forward(self._h, t, ctypes.byref(w), int(noise), out)
         self.last_t = t
         return out
 
     def forward_partial(self, t: float, w: Weights, noise: bool = True):
         dh = np.zeros((self.Y, self.X)); dv = np.zeros((self.Y, self.X))
         ewl = ctypes.c_double(); etp = ctypes.c_double()
-        _load().odgr_forward_partial(self._h, t, ctypes.byref(w), int(noise), dh, dv, ctypes.byref(ewl),
+        self._L.odgr_forward_partial(self._h, t, ctypes.byref(w), int(noise), dh, dv, ctypes.byref(ewl),
                                      ctypes.byref(etp))
         return dh, dv, ewl.value, etp.value
 
     def forward_finish(self, dh, dv, ewl, etp, w: Weights) -> np.ndarray:
         out = np.zeros(4)
-        _load().odgr_forward_finish(self._h, np.ascontiguousarray(dh, np.float64), np.ascontiguousarray(dv, np.float64),
+        self._L.odgr_forward_finish(self._h, np.ascontiguousarray(dh, np.float64), np.ascontiguousarray(dv, np.float64),
                                     ewl, etp, ctypes.byref(w), out)
         return out
 
     def backward(self, t: float, w: Weights):
         dw = np.zeros(self.f.n_paths); du = np.zeros(self.f.n_trees)
-        _load().odgr_backward(self._h, t, ctypes.byref(w), dw, du)
+        self._L.odgr_backward(self._h, t, ctypes.byref(w), dw, du)
         return dw, du
 
     def adam(self, lr: float, dw, du):
-        _load().odgr_adam(self._h, lr, np.ascontiguousarray(dw, np.float64), np.ascontiguousarray(du, np.float64))
+        self._L.odgr_adam(self._h, lr, np.ascontiguousarray(dw, np.float64), np.ascontiguousarray(du, np.float64))
 
     def next_iteration(self):
-        _load().odgr_next_iteration(self._h)
+        self._L.odgr_next_iteration(self._h)
 
     def step(self, iters: int, t: float, lr: float, w: Weights) -> np.ndarray:
         out = np.zeros(4)
-        _load().odgr_step(self._h, iters, t, lr, ctypes.byref(w), out)
+        self._L.odgr_step(self._h, iters, t, lr, ctypes.byref(w), out)
         self.last_t = t
         return out
 
@@ -232,7 +239,7 @@ class Oracle:
             D_h=np.zeros((f.Y, f.X), np.int32), D_v=np.zeros((f.Y, f.X), np.int32), metrics=np.zeros(5),
             margin_tree=np.zeros(f.n_nets), margin_route=np.zeros(f.n_subnets),
             margin_nucleus=np.zeros(f.n_subnets))
-        _load().odgr_induce(self._h, t, top_p, beta, r.tree_choice, r.route, r.nucleus_off, r.nucleus, r.D_h, r.D_v,
+        self._L.odgr_induce(self._h, t, top_p, beta, r.tree_choice, r.route, r.nucleus_off, r.nucleus, r.D_h, r.D_v,
                             r.metrics, r.margin_tree, r.margin_route, r.margin_nucleus)
         r.nucleus = r.nucleus[: r.nucleus_off[-1]].copy()
         return r

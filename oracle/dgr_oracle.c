@@ -28,12 +28,21 @@
  * fixed point: those are implementation devices of the CUDA path, not the method.
  * Readings (Q-numbers) are listed in DESIGN.md §3.
  */
-#include <math.h>
 #include <stdint.h>
+#include <tgmath.h>   /* type-generic exp/log/sqrt/pow/fabs: follow `real` below */
 #include <stdlib.h>
 #include <string.h>
 
 #define ODGR_API __attribute__((visibility("default")))
+
+/* The oracle computes in `real` = double (fp64, the parity reference).  The same source built with
+ * -DODGR_REAL=float is used ONLY as a conditioning probe: it shows which outputs fp32 arithmetic
+ * cannot determine to the parity tolerance (reading Q21b).  The ABI stays double. */
+#ifndef ODGR_REAL
+#define ODGR_REAL double
+#endif
+typedef ODGR_REAL real;
+#define R(x) ((real)(x))
 
 /* ------------------------------------------------------------------------------------ */
 /* Philox4x32-10 (Salmon et al., SC'11; the Random123 constants).  Reading Q7.          */
@@ -88,15 +97,15 @@ typedef struct {
   int64_t n_nets, n_trees, n_subnets, n_paths, n_segs, n_tps;
   int64_t *net_tree_off, *tree_sub_off, *sub_path_off, *path_seg_off, *path_tp_off;
   int32_t *seg, *tp_xy;
-  double *cap_h, *cap_v;      /* [Y][X] */
+  real *cap_h, *cap_v;        /* [Y][X] */
   uint64_t seed;
   /* trainable logits and Adam state */
-  double *w_tree, *w_path, *m_tree, *v_tree, *m_path, *v_path;
+  real *w_tree, *w_path, *m_tree, *v_tree, *m_path, *v_path;
   int64_t k;                  /* global iteration counter (noise key; Adam step = k+1) */
   int64_t net_lo, net_hi;     /* shard (all nets by default) */
   /* last forward */
-  double *p, *q, *d_h, *d_v;
-  double e_wl, e_tp, overflow, loss;
+  real *p, *q, *d_h, *d_v;
+  real e_wl, e_tp, overflow, loss;
   double t_last;
 } odgr_state;
 
@@ -105,6 +114,11 @@ static void* xcopy(const void* src, size_t bytes) {
   if (bytes) memcpy(p, src, bytes);
   return p;
 }
+static real* rzeros(size_t n) { return (real*)calloc(n + 1, sizeof(real)); }
+static void to_double(double* dst, const real* src, size_t n) { for (size_t i = 0; i < n; ++i) dst[i] = (double)src[i]; }
+static void to_real(real* dst, const double* src, size_t n) { for (size_t i = 0; i < n; ++i) dst[i] = (real)src[i]; }
+
+ODGR_API int32_t odgr_real_bytes(void) { return (int32_t)sizeof(real); }
 
 ODGR_API odgr_state* odgr_new(int32_t X, int32_t Y, int64_t n_nets, int64_t n_trees, int64_t n_subnets,
                               int64_t n_paths, int64_t n_segs, int64_t n_tps,
@@ -125,22 +139,18 @@ ODGR_API odgr_state* odgr_new(int32_t X, int32_t Y, int64_t n_nets, int64_t n_tr
   s->seg = (int32_t*)xcopy(seg, sizeof(int32_t) * 4 * n_segs);
   s->tp_xy = (int32_t*)xcopy(tp_xy, sizeof(int32_t) * 2 * n_tps);
   size_t G = (size_t)X * Y;
-  s->cap_h = (double*)malloc(sizeof(double) * G);
-  s->cap_v = (double*)malloc(sizeof(double) * G);
+  s->cap_h = rzeros(G);
+  s->cap_v = rzeros(G);
   for (size_t e = 0; e < G; ++e) { s->cap_h[e] = cap_h[e]; s->cap_v[e] = cap_v[e]; }
   s->seed = seed;
-  s->w_tree = (double*)malloc(sizeof(double) * (n_trees + 1));
-  s->w_path = (double*)malloc(sizeof(double) * (n_paths + 1));
+  s->w_tree = rzeros(n_trees);
+  s->w_path = rzeros(n_paths);
   for (int64_t j = 0; j < n_trees; ++j) s->w_tree[j] = w_tree0[j];
   for (int64_t i = 0; i < n_paths; ++i) s->w_path[i] = w_path0[i];
-  s->m_tree = (double*)calloc(n_trees + 1, sizeof(double));
-  s->v_tree = (double*)calloc(n_trees + 1, sizeof(double));
-  s->m_path = (double*)calloc(n_paths + 1, sizeof(double));
-  s->v_path = (double*)calloc(n_paths + 1, sizeof(double));
-  s->p = (double*)calloc(n_paths + 1, sizeof(double));
-  s->q = (double*)calloc(n_trees + 1, sizeof(double));
-  s->d_h = (double*)calloc(G, sizeof(double));
-  s->d_v = (double*)calloc(G, sizeof(double));
+  s->m_tree = rzeros(n_trees); s->v_tree = rzeros(n_trees);
+  s->m_path = rzeros(n_paths); s->v_path = rzeros(n_paths);
+  s->p = rzeros(n_paths); s->q = rzeros(n_trees);
+  s->d_h = rzeros(G); s->d_v = rzeros(G);
   s->k = 0;
   s->net_lo = 0; s->net_hi = n_nets;
   s->t_last = 1.0;
@@ -162,55 +172,56 @@ ODGR_API void odgr_set_iteration(odgr_state* s, int64_t k) { s->k = k; }
 ODGR_API void odgr_set_shard(odgr_state* s, int64_t lo, int64_t hi) { s->net_lo = lo; s->net_hi = hi; }
 
 /* WL_i: total length of i's segments in G-cell edges (reading Q5). TP_i: its turning points. */
-static double path_wl(const odgr_state* s, int64_t i) {
-  double wl = 0;
+static real path_wl(const odgr_state* s, int64_t i) {
+  int64_t wl = 0;
   for (int64_t g = s->path_seg_off[i]; g < s->path_seg_off[i + 1]; ++g) wl += s->seg[4 * g + 3] - s->seg[4 * g + 2];
-  return wl;
+  return (real)wl;
 }
-static double path_tp(const odgr_state* s, int64_t i) { return (double)(s->path_tp_off[i + 1] - s->path_tp_off[i]); }
+static real path_tp(const odgr_state* s, int64_t i) { return (real)(s->path_tp_off[i + 1] - s->path_tp_off[i]); }
 
 /* edge accessors: H edge (x,y)-(x+1,y) and V edge (x,y)-(x,y+1), both stored at [y][x] */
-static double* edge_ref(double* gh, double* gv, int X, int dir, int line, int e) {
+static real* edge_ref(real* gh, real* gv, int X, int dir, int line, int e) {
   return dir == 0 ? &gh[(size_t)line * X + e] : &gv[(size_t)e * X + line];
 }
 
 /* ---- forward, part 1 (this shard): probabilities and this shard's demand ---- */
 /* p, q per §4.4; the demand of Eq. (10) added edge by edge; E[WL], E[TP] per Eqs. (11)/(12). */
-ODGR_API void odgr_forward_partial(odgr_state* s, double t, const odgr_weights* W, int noise,
-                                   double* d_h, double* d_v, double* e_wl, double* e_tp) {
+static void forward_partial(odgr_state* s, real t, const odgr_weights* W, int noise, real* d_h, real* d_v,
+                            real* e_wl, real* e_tp) {
   const int X = s->X, Y = s->Y;
-  memset(d_h, 0, sizeof(double) * X * Y);
-  memset(d_v, 0, sizeof(double) * X * Y);
-  double ewl = 0, etp = 0;
+  memset(d_h, 0, sizeof(real) * X * Y);
+  memset(d_v, 0, sizeof(real) * X * Y);
+  const real beta = (real)W->beta;
+  real ewl = 0, etp = 0;
   for (int64_t n = s->net_lo; n < s->net_hi; ++n) {
     /* q_j = exp((w_j + g_j)/t) / sum_{k: net(k)=net(j)} exp((w_k + g_k)/t) */
     int64_t j0 = s->net_tree_off[n], j1 = s->net_tree_off[n + 1];
-    double zmax = -INFINITY;
+    real zmax = -INFINITY;
     for (int64_t j = j0; j < j1; ++j) {
-      double g = noise ? odgr_gumbel(s->seed, (uint64_t)j, (uint64_t)s->k, 1) : 0.0;
-      double z = (s->w_tree[j] + g) / t;
+      real g = noise ? (real)odgr_gumbel(s->seed, (uint64_t)j, (uint64_t)s->k, 1) : R(0);
+      real z = (s->w_tree[j] + g) / t;
       s->q[j] = z;
       if (z > zmax) zmax = z;
     }
-    double zs = 0;
+    real zs = 0;
     for (int64_t j = j0; j < j1; ++j) { s->q[j] = exp(s->q[j] - zmax); zs += s->q[j]; }
     for (int64_t j = j0; j < j1; ++j) s->q[j] /= zs;
     for (int64_t j = j0; j < j1; ++j) {
       for (int64_t sn = s->tree_sub_off[j]; sn < s->tree_sub_off[j + 1]; ++sn) {
         /* p_i = exp((w_i + g_i)/t) / sum_{k: subnet(k)=subnet(i)} exp((w_k + g_k)/t) */
         int64_t i0 = s->sub_path_off[sn], i1 = s->sub_path_off[sn + 1];
-        double pm = -INFINITY;
+        real pm = -INFINITY;
         for (int64_t i = i0; i < i1; ++i) {
-          double g = noise ? odgr_gumbel(s->seed, (uint64_t)i, (uint64_t)s->k, 0) : 0.0;
-          double z = (s->w_path[i] + g) / t;
+          real g = noise ? (real)odgr_gumbel(s->seed, (uint64_t)i, (uint64_t)s->k, 0) : R(0);
+          real z = (s->w_path[i] + g) / t;
           s->p[i] = z;
           if (z > pm) pm = z;
         }
-        double ps = 0;
+        real ps = 0;
         for (int64_t i = i0; i < i1; ++i) { s->p[i] = exp(s->p[i] - pm); ps += s->p[i]; }
         for (int64_t i = i0; i < i1; ++i) s->p[i] /= ps;
         for (int64_t i = i0; i < i1; ++i) {
-          double pi = s->q[j] * s->p[i];         /* q_tree(i) p_i */
+          real pi = s->q[j] * s->p[i];           /* q_tree(i) p_i */
           /* wire demand: every edge e of every segment of i */
           for (int64_t g = s->path_seg_off[i]; g < s->path_seg_off[i + 1]; ++g) {
             const int32_t* sg = &s->seg[4 * g];
@@ -219,7 +230,7 @@ ODGR_API void odgr_forward_partial(odgr_state* s, double t, const odgr_weights* 
           /* via demand: beta * pi on every edge incident to each turning point v of i */
           for (int64_t u = s->path_tp_off[i]; u < s->path_tp_off[i + 1]; ++u) {
             int x = s->tp_xy[2 * u], y = s->tp_xy[2 * u + 1];
-            double b = W->beta * pi;
+            real b = beta * pi;
             if (x >= 1) d_h[(size_t)y * X + (x - 1)] += b;
             if (x <= X - 2) d_h[(size_t)y * X + x] += b;
             if (y >= 1) d_v[(size_t)(y - 1) * X + x] += b;
@@ -235,86 +246,100 @@ ODGR_API void odgr_forward_partial(odgr_state* s, double t, const odgr_weights* 
   *e_tp = etp;
 }
 
-static double sigm(double x) { return 1.0 / (1.0 + exp(-x)); }
+ODGR_API void odgr_forward_partial(odgr_state* s, double t, const odgr_weights* W, int noise,
+                                   double* d_h, double* d_v, double* e_wl, double* e_tp) {
+  real ewl, etp;
+  forward_partial(s, (real)t, W, noise, s->d_h, s->d_v, &ewl, &etp);
+  to_double(d_h, s->d_h, (size_t)s->X * s->Y);
+  to_double(d_v, s->d_v, (size_t)s->X * s->Y);
+  *e_wl = (double)ewl;
+  *e_tp = (double)etp;
+}
 
-/* ---- forward, part 2: the cost of Eq. (3) from the (global) demand ---- */
-ODGR_API double odgr_forward_finish(odgr_state* s, const double* d_h, const double* d_v, double e_wl,
-                                    double e_tp, const odgr_weights* W, double out[4]) {
+static real sigm(real x) { return R(1) / (R(1) + exp(-x)); }
+
+/* ---- forward, part 2: the cost of Eq. (3) from the (global) demand in s->d_h, s->d_v ---- */
+static real forward_finish(odgr_state* s, real e_wl, real e_tp, const odgr_weights* W, double out[4]) {
   const int X = s->X, Y = s->Y;
-  if (d_h != s->d_h) memcpy(s->d_h, d_h, sizeof(double) * X * Y);
-  if (d_v != s->d_v) memcpy(s->d_v, d_v, sizeof(double) * X * Y);
-  double of = 0;
+  const real slope = (real)W->f_slope;
+  real of = 0;
   for (int y = 0; y < Y; ++y)
     for (int x = 0; x < X; ++x) {
       size_t e = (size_t)y * X + x;
       for (int dir = 0; dir < 2; ++dir) {
         if (dir == 0 && x > X - 2) continue;
         if (dir == 1 && y > Y - 2) continue;
-        double r = (dir == 0 ? s->cap_h[e] - s->d_h[e] : s->cap_v[e] - s->d_v[e]);  /* resource */
-        if (W->f_kind == 0) of += 1.0 / (1.0 + exp(W->f_slope * r));   /* sigmoid, decreasing in r */
-        else of += r < 0 ? -r : 0.0;                                      /* ReLU(d - cap) */
+        real r = (dir == 0 ? s->cap_h[e] - s->d_h[e] : s->cap_v[e] - s->d_v[e]);  /* resource */
+        if (W->f_kind == 0) of += R(1) / (R(1) + exp(slope * r));   /* sigmoid, decreasing in r */
+        else of += r < 0 ? -r : R(0);                                 /* ReLU(d - cap) */
       }
     }
   s->e_wl = e_wl; s->e_tp = e_tp; s->overflow = of;
-  double wl_cost = e_wl, via_cost = sqrt(W->n_layers) * e_tp;
-  s->loss = W->a_wl * wl_cost + W->a_via * via_cost + W->a_of * of;
+  real wl_cost = e_wl, via_cost = sqrt((real)W->n_layers) * e_tp;
+  s->loss = (real)W->a_wl * wl_cost + (real)W->a_via * via_cost + (real)W->a_of * of;
   if (out) { out[0] = s->loss; out[1] = wl_cost; out[2] = via_cost; out[3] = of; }
   return s->loss;
 }
 
+ODGR_API double odgr_forward_finish(odgr_state* s, const double* d_h, const double* d_v, double e_wl,
+                                    double e_tp, const odgr_weights* W, double out[4]) {
+  to_real(s->d_h, d_h, (size_t)s->X * s->Y);
+  to_real(s->d_v, d_v, (size_t)s->X * s->Y);
+  return (double)forward_finish(s, (real)e_wl, (real)e_tp, W, out);
+}
+
 ODGR_API double odgr_forward(odgr_state* s, double t, const odgr_weights* W, int noise, double out[4]) {
-  double ewl, etp;
-  odgr_forward_partial(s, t, W, noise, s->d_h, s->d_v, &ewl, &etp);
+  real ewl, etp;
+  forward_partial(s, (real)t, W, noise, s->d_h, s->d_v, &ewl, &etp);
   s->t_last = t;
-  return odgr_forward_finish(s, s->d_h, s->d_v, ewl, etp, W, out);
+  return (double)forward_finish(s, ewl, etp, W, out);
 }
 
 /* ---- reverse: d cost / d w for the shard's logits (the chain rule of P:841-845) ---- */
-ODGR_API void odgr_backward(odgr_state* s, double t, const odgr_weights* W, double* dw_path, double* du_tree) {
+static void backward(odgr_state* s, real t, const odgr_weights* W, real* dw_path, real* du_tree) {
   const int X = s->X, Y = s->Y;
   size_t G = (size_t)X * Y;
+  const real a3 = (real)W->a_of, slope = (real)W->f_slope, beta = (real)W->beta;
   /* G_e = d cost / d d_e = -a3 f'(cap_e - d_e) */
-  double* gh = (double*)calloc(G, sizeof(double));
-  double* gv = (double*)calloc(G, sizeof(double));
+  real* gh = rzeros(G);
+  real* gv = rzeros(G);
   for (int y = 0; y < Y; ++y)
     for (int x = 0; x < X; ++x) {
       size_t e = (size_t)y * X + x;
       if (x <= X - 2) {
-        double r = s->cap_h[e] - s->d_h[e];
-        gh[e] = W->f_kind == 0 ? W->a_of * W->f_slope * sigm(W->f_slope * r) * sigm(-W->f_slope * r)
-                               : (s->d_h[e] > s->cap_h[e] ? W->a_of : 0.0);
+        real r = s->cap_h[e] - s->d_h[e];
+        gh[e] = W->f_kind == 0 ? a3 * slope * sigm(slope * r) * sigm(-slope * r) : (s->d_h[e] > s->cap_h[e] ? a3 : R(0));
       }
       if (y <= Y - 2) {
-        double r = s->cap_v[e] - s->d_v[e];
-        gv[e] = W->f_kind == 0 ? W->a_of * W->f_slope * sigm(W->f_slope * r) * sigm(-W->f_slope * r)
-                               : (s->d_v[e] > s->cap_v[e] ? W->a_of : 0.0);
+        real r = s->cap_v[e] - s->d_v[e];
+        gv[e] = W->f_kind == 0 ? a3 * slope * sigm(slope * r) * sigm(-slope * r) : (s->d_v[e] > s->cap_v[e] ? a3 : R(0));
       }
     }
-  const double sqL = sqrt(W->n_layers);
+  const real sqL = sqrt((real)W->n_layers);
   for (int64_t n = s->net_lo; n < s->net_hi; ++n) {
     int64_t j0 = s->net_tree_off[n], j1 = s->net_tree_off[n + 1];
     for (int64_t j = j0; j < j1; ++j) {
-      double dq = 0;                    /* dq_j = sum_{i: tree(i)=j} p_i c_i */
+      real dq = 0;                      /* dq_j = sum_{i: tree(i)=j} p_i c_i */
       for (int64_t sn = s->tree_sub_off[j]; sn < s->tree_sub_off[j + 1]; ++sn) {
         int64_t i0 = s->sub_path_off[sn], i1 = s->sub_path_off[sn + 1];
-        double spd = 0;                 /* sum_{k in subnet} p_k dp_k */
+        real spd = 0;                   /* sum_{k in subnet} p_k dp_k */
         for (int64_t i = i0; i < i1; ++i) {
           /* c_i = d cost / d pi_i */
-          double c = W->a_wl * path_wl(s, i) + W->a_via * sqL * path_tp(s, i);
+          real c = (real)W->a_wl * path_wl(s, i) + (real)W->a_via * sqL * path_tp(s, i);
           for (int64_t g = s->path_seg_off[i]; g < s->path_seg_off[i + 1]; ++g) {
             const int32_t* sg = &s->seg[4 * g];
             for (int e = sg[2]; e < sg[3]; ++e) c += *edge_ref(gh, gv, X, sg[0], sg[1], e);
           }
           for (int64_t u = s->path_tp_off[i]; u < s->path_tp_off[i + 1]; ++u) {
             int x = s->tp_xy[2 * u], y = s->tp_xy[2 * u + 1];
-            double v = 0;
+            real v = 0;
             if (x >= 1) v += gh[(size_t)y * X + (x - 1)];
             if (x <= X - 2) v += gh[(size_t)y * X + x];
             if (y >= 1) v += gv[(size_t)(y - 1) * X + x];
             if (y <= Y - 2) v += gv[(size_t)y * X + x];
-            c += W->beta * v;
+            c += beta * v;
           }
-          dw_path[i] = s->q[j] * c;     /* dp_i = q_tree(i) c_i (stored temporarily) */
+          dw_path[i] = s->q[j] * c;       /* dp_i = q_tree(i) c_i (stored temporarily) */
           dq += s->p[i] * c;
           spd += s->p[i] * dw_path[i];
         }
@@ -323,7 +348,7 @@ ODGR_API void odgr_backward(odgr_state* s, double t, const odgr_weights* W, doub
       }
       du_tree[j] = dq;
     }
-    double sqd = 0;
+    real sqd = 0;
     for (int64_t j = j0; j < j1; ++j) sqd += s->q[j] * du_tree[j];
     for (int64_t j = j0; j < j1; ++j) du_tree[j] = s->q[j] / t * (du_tree[j] - sqd);
   }
@@ -331,17 +356,31 @@ ODGR_API void odgr_backward(odgr_state* s, double t, const odgr_weights* W, doub
   free(gv);
 }
 
+ODGR_API void odgr_backward(odgr_state* s, double t, const odgr_weights* W, double* dw_path, double* du_tree) {
+  real* dw = rzeros(s->n_paths);
+  real* du = rzeros(s->n_trees);
+  backward(s, (real)t, W, dw, du);
+  for (int64_t n = s->net_lo; n < s->net_hi; ++n)
+    for (int64_t j = s->net_tree_off[n]; j < s->net_tree_off[n + 1]; ++j) {
+      du_tree[j] = du[j];
+      for (int64_t i = s->sub_path_off[s->tree_sub_off[j]]; i < s->sub_path_off[s->tree_sub_off[j + 1]]; ++i)
+        dw_path[i] = dw[i];
+    }
+  free(dw);
+  free(du);
+}
+
 /* ---- Adam (torch.optim.Adam semantics; betas 0.9/0.999, eps 1e-8; reading Q9) ---- */
-static void adam_one(double* w, double* m, double* v, double g, double lr, int64_t step) {
-  const double b1 = 0.9, b2 = 0.999, eps = 1e-8;
-  *m = b1 * *m + (1 - b1) * g;
-  *v = b2 * *v + (1 - b2) * g * g;
-  double bc1 = 1 - pow(b1, (double)step), bc2 = 1 - pow(b2, (double)step);
-  double denom = sqrt(*v) / sqrt(bc2) + eps;
+static void adam_one(real* w, real* m, real* v, real g, real lr, int64_t step) {
+  const real b1 = R(0.9), b2 = R(0.999), eps = R(1e-8);
+  *m = b1 * *m + (R(1) - b1) * g;
+  *v = b2 * *v + (R(1) - b2) * g * g;
+  real bc1 = R(1) - pow(b1, (real)step), bc2 = R(1) - pow(b2, (real)step);
+  real denom = sqrt(*v) / sqrt(bc2) + eps;
   *w -= (lr / bc1) * (*m / denom);
 }
 
-ODGR_API void odgr_adam(odgr_state* s, double lr, const double* dw_path, const double* du_tree) {
+static void adam(odgr_state* s, real lr, const real* dw_path, const real* du_tree) {
   int64_t step = s->k + 1;
   for (int64_t n = s->net_lo; n < s->net_hi; ++n)
     for (int64_t j = s->net_tree_off[n]; j < s->net_tree_off[n + 1]; ++j) {
@@ -352,17 +391,27 @@ ODGR_API void odgr_adam(odgr_state* s, double lr, const double* dw_path, const d
     }
 }
 
+ODGR_API void odgr_adam(odgr_state* s, double lr, const double* dw_path, const double* du_tree) {
+  real* dw = rzeros(s->n_paths);
+  real* du = rzeros(s->n_trees);
+  to_real(dw, dw_path, (size_t)s->n_paths);
+  to_real(du, du_tree, (size_t)s->n_trees);
+  adam(s, (real)lr, dw, du);
+  free(dw);
+  free(du);
+}
+
 ODGR_API void odgr_next_iteration(odgr_state* s) { s->k += 1; }
 
 /* iters x {forward, reverse, Adam}; iters = 0 is forward only (include/dgr.h contract) */
 ODGR_API void odgr_step(odgr_state* s, int iters, double t, double lr, const odgr_weights* W, double out[4]) {
   if (iters == 0) { odgr_forward(s, t, W, 1, out); return; }
-  double* dw = (double*)malloc(sizeof(double) * (s->n_paths + 1));
-  double* du = (double*)malloc(sizeof(double) * (s->n_trees + 1));
+  real* dw = rzeros(s->n_paths);
+  real* du = rzeros(s->n_trees);
   for (int it = 0; it < iters; ++it) {
     odgr_forward(s, t, W, 1, out);
-    odgr_backward(s, t, W, dw, du);
-    odgr_adam(s, lr, dw, du);
+    backward(s, (real)t, W, dw, du);
+    adam(s, (real)lr, dw, du);
     s->k += 1;
   }
   free(dw);
@@ -370,26 +419,26 @@ ODGR_API void odgr_step(odgr_state* s, int iters, double t, double lr, const odg
 }
 
 ODGR_API void odgr_get_logits(const odgr_state* s, double* w_tree, double* w_path) {
-  if (w_tree) memcpy(w_tree, s->w_tree, sizeof(double) * s->n_trees);
-  if (w_path) memcpy(w_path, s->w_path, sizeof(double) * s->n_paths);
+  if (w_tree) to_double(w_tree, s->w_tree, (size_t)s->n_trees);
+  if (w_path) to_double(w_path, s->w_path, (size_t)s->n_paths);
 }
 ODGR_API void odgr_set_logits(odgr_state* s, const double* w_tree, const double* w_path) {
-  if (w_tree) memcpy(s->w_tree, w_tree, sizeof(double) * s->n_trees);
-  if (w_path) memcpy(s->w_path, w_path, sizeof(double) * s->n_paths);
+  if (w_tree) to_real(s->w_tree, w_tree, (size_t)s->n_trees);
+  if (w_path) to_real(s->w_path, w_path, (size_t)s->n_paths);
 }
 ODGR_API void odgr_get_adam(const odgr_state* s, double* m_tree, double* v_tree, double* m_path, double* v_path) {
-  if (m_tree) memcpy(m_tree, s->m_tree, sizeof(double) * s->n_trees);
-  if (v_tree) memcpy(v_tree, s->v_tree, sizeof(double) * s->n_trees);
-  if (m_path) memcpy(m_path, s->m_path, sizeof(double) * s->n_paths);
-  if (v_path) memcpy(v_path, s->v_path, sizeof(double) * s->n_paths);
+  if (m_tree) to_double(m_tree, s->m_tree, (size_t)s->n_trees);
+  if (v_tree) to_double(v_tree, s->v_tree, (size_t)s->n_trees);
+  if (m_path) to_double(m_path, s->m_path, (size_t)s->n_paths);
+  if (v_path) to_double(v_path, s->v_path, (size_t)s->n_paths);
 }
 ODGR_API void odgr_get_probs(const odgr_state* s, double* q, double* p) {
-  if (q) memcpy(q, s->q, sizeof(double) * s->n_trees);
-  if (p) memcpy(p, s->p, sizeof(double) * s->n_paths);
+  if (q) to_double(q, s->q, (size_t)s->n_trees);
+  if (p) to_double(p, s->p, (size_t)s->n_paths);
 }
 ODGR_API void odgr_get_demand(const odgr_state* s, double* d_h, double* d_v) {
-  memcpy(d_h, s->d_h, sizeof(double) * s->X * s->Y);
-  memcpy(d_v, s->d_v, sizeof(double) * s->X * s->Y);
+  to_double(d_h, s->d_h, (size_t)s->X * s->Y);
+  to_double(d_v, s->d_v, (size_t)s->X * s->Y);
 }
 
 /* ---- discrete induction (§4.5; readings Q12, Q13, Q23) ----

@@ -1,0 +1,664 @@
+// dgr_api.cu — libdgr's C ABI (include/dgr.h): validation, net sharding, device encoding,
+// workspace layout, the iteration driver and the NCCL demand exchange.
+//
+// The data-parallel unit is the net (§3.2: nets couple only through the demand d of
+// Eq. (10)).  Rank r keeps a contiguous, work-balanced range of nets; per iteration
+// the ranks exchange one int64 buffer [dH | dV^T | VD | E[WL] | E[TP]] with ncclAllReduce —
+// fixed point makes the sum exact, so every rank then runs the (replicated) grid pass on
+// identical data and the result does not depend on the number of ranks.
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "dgr.h"
+#include "dgr_internal.h"
+
+using namespace dgr;
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return code;
+}
+
+#define CUDA_TRY(x)                                                                          \
+  do {                                                                                       \
+    cudaError_t e_ = (x);                                                                    \
+    if (e_ != cudaSuccess) return fail(DGR_ECUDA, "%s: %s", #x, cudaGetErrorString(e_));      \
+  } while (0)
+#define NCCL_TRY(x)                                                                          \
+  do {                                                                                       \
+    ncclResult_t r_ = (x);                                                                   \
+    if (r_ != ncclSuccess) return fail(DGR_ENCCL, "%s: %s", #x, ncclGetErrorString(r_));      \
+  } while (0)
+
+// ---------------------------------------------------------------------------------------
+// validation + sharding
+// ---------------------------------------------------------------------------------------
+int check_offsets(const int64_t* off, int64_t n, int64_t total, const char* name, bool nonempty) {
+  if (!off) return fail(DGR_EINVAL, "%s is NULL", name);
+  if (off[0] != 0) return fail(DGR_EINVAL, "%s[0] != 0", name);
+  for (int64_t i = 0; i < n; ++i) {
+    if (off[i + 1] < off[i]) return fail(DGR_EINVAL, "%s not monotone at %lld", name, (long long)i);
+    if (nonempty && off[i + 1] == off[i]) return fail(DGR_EINVAL, "%s: empty group %lld", name, (long long)i);
+  }
+  if (off[n] != total) return fail(DGR_EINVAL, "%s[n] = %lld != %lld", name, (long long)off[n], (long long)total);
+  return DGR_OK;
+}
+
+int validate_structure(const dgr_forest_desc* d) {
+  if (!d) return fail(DGR_EINVAL, "desc is NULL");
+  if (d->X < 2 || d->Y < 2 || d->X > 32767 || d->Y > 32767) return fail(DGR_EINVAL, "grid must be 2..32767 per side");
+  if (d->n_nets < 0 || d->n_trees < 0 || d->n_subnets < 0 || d->n_paths < 0 || d->n_segs < 0 || d->n_tps < 0)
+    return fail(DGR_EINVAL, "negative count");
+  if (d->n_paths >= (1ll << 31) || d->n_subnets >= (1ll << 31) || d->n_trees >= (1ll << 31))
+    return fail(DGR_EINVAL, "more than 2^31 candidates");
+  int rc;
+  if ((rc = check_offsets(d->net_tree_off, d->n_nets, d->n_trees, "net_tree_off", true))) return rc;
+  if ((rc = check_offsets(d->tree_sub_off, d->n_trees, d->n_subnets, "tree_sub_off", true))) return rc;
+  if ((rc = check_offsets(d->sub_path_off, d->n_subnets, d->n_paths, "sub_path_off", true))) return rc;
+  if ((rc = check_offsets(d->path_seg_off, d->n_paths, d->n_segs, "path_seg_off", true))) return rc;
+  if ((rc = check_offsets(d->path_tp_off, d->n_paths, d->n_tps, "path_tp_off", false))) return rc;
+  for (int64_t s = 0; s < d->n_subnets; ++s)
+    if (d->sub_path_off[s + 1] - d->sub_path_off[s] > 32)
+      return fail(DGR_EINVAL, "sub-net %lld has %lld > 32 candidates", (long long)s,
+                  (long long)(d->sub_path_off[s + 1] - d->sub_path_off[s]));
+  if ((d->n_segs && !d->seg) || (d->n_tps && !d->tp_xy) || (d->n_subnets && !d->sub_xy) || !d->cap_h ||
+      !d->cap_v || (d->n_trees && !d->w_tree0) || (d->n_paths && !d->w_path0))
+    return fail(DGR_EINVAL, "NULL array");
+  return DGR_OK;
+}
+
+int partition(const dgr_forest_desc* d, int world, std::vector<int64_t>& out) {
+  if (world < 1) return fail(DGR_EINVAL, "world < 1");
+  out.assign(world + 1, 0);
+  // work of a net = its paths + its segments (the per-candidate streams of KF / KB)
+  std::vector<int64_t> pref(d->n_nets + 1, 0);
+  for (int64_t n = 0; n < d->n_nets; ++n) {
+    const int64_t s0 = d->tree_sub_off[d->net_tree_off[n]], s1 = d->tree_sub_off[d->net_tree_off[n + 1]];
+    const int64_t p0 = d->sub_path_off[s0], p1 = d->sub_path_off[s1];
+    pref[n + 1] = pref[n] + (p1 - p0) + (d->path_seg_off[p1] - d->path_seg_off[p0]);
+  }
+  const int64_t total = pref[d->n_nets];
+  for (int r = 1; r < world; ++r) {
+    const double target = (double)total * r / world;
+    const int64_t lo = out[r - 1];
+    int64_t n = std::lower_bound(pref.begin() + lo, pref.end(), (int64_t)std::ceil(target)) - pref.begin();
+    out[r] = std::min<int64_t>(std::max<int64_t>(n, lo), d->n_nets);
+  }
+  out[world] = d->n_nets;
+  return DGR_OK;
+}
+
+// ---------------------------------------------------------------------------------------
+// pattern recognition: each explicit path must be a straight / L / Z pattern of its sub-net
+// ---------------------------------------------------------------------------------------
+struct Seg4 { int a, b, c, d; };
+inline bool seg_less(const Seg4& x, const Seg4& y) {
+  if (x.a != y.a) return x.a < y.a;
+  if (x.b != y.b) return x.b < y.b;
+  if (x.c != y.c) return x.c < y.c;
+  return x.d < y.d;
+}
+inline bool seg_eq(const Seg4& x, const Seg4& y) { return x.a == y.a && x.b == y.b && x.c == y.c && x.d == y.d; }
+// order-insensitive equality of two small lists (n <= 3)
+inline bool same_sets(Seg4* a, Seg4* b, int n) {
+  std::sort(a, a + n, seg_less);
+  std::sort(b, b + n, seg_less);
+  for (int i = 0; i < n; ++i) if (!seg_eq(a[i], b[i])) return false;
+  return true;
+}
+
+bool classify(const dgr_forest_desc* d, int64_t i, int x0, int y0, int x1, int y1, uint32_t* shape, int* mid) {
+  const int64_t g0 = d->path_seg_off[i], g1 = d->path_seg_off[i + 1];
+  const int64_t t0 = d->path_tp_off[i], t1 = d->path_tp_off[i + 1];
+  const int ns = (int)(g1 - g0), nt = (int)(t1 - t0);
+  if (ns < 1 || ns > 3 || nt != ns - 1) return false;
+  Seg4 segs[3], tps[2];
+  for (int g = 0; g < ns; ++g) {
+    const int32_t* s = d->seg + 4 * (g0 + g);
+    segs[g] = {s[0], s[1], s[2], s[3]};
+  }
+  for (int t = 0; t < nt; ++t) tps[t] = {d->tp_xy[2 * (t0 + t)], d->tp_xy[2 * (t0 + t) + 1], 0, 0};
+  const int ylo = std::min(y0, y1), yhi = std::max(y0, y1);
+  auto try_shape = [&](uint32_t sh, int m, std::initializer_list<Seg4> es, std::initializer_list<Seg4> et) {
+    if ((int)es.size() != ns || (int)et.size() != nt) return false;
+    Seg4 a[3], b[3], c[2], e[2];
+    int k = 0;
+    for (auto& s : es) a[k++] = s;
+    for (int q = 0; q < ns; ++q) b[q] = segs[q];
+    k = 0;
+    for (auto& s : et) c[k++] = s;
+    for (int q = 0; q < nt; ++q) e[q] = tps[q];
+    if (same_sets(a, b, ns) && same_sets(c, e, nt)) { *shape = sh; *mid = m; return true; }
+    return false;
+  };
+  if (y0 == y1) return try_shape(kStraightH, 0, {{0, y0, x0, x1}}, {});
+  if (x0 == x1) return try_shape(kStraightV, 0, {{1, x0, ylo, yhi}}, {});
+  if (ns == 2) {
+    if (try_shape(kHV, 0, {{0, y0, x0, x1}, {1, x1, ylo, yhi}}, {{x1, y0, 0, 0}})) return true;
+    return try_shape(kVH, 0, {{1, x0, ylo, yhi}, {0, y1, x0, x1}}, {{x0, y1, 0, 0}});
+  }
+  if (ns == 3) {
+    int nh = 0;
+    for (int q = 0; q < 3; ++q) nh += segs[q].a == 0;
+    if (nh == 2) {
+      int xm = -1;
+      for (int q = 0; q < 3; ++q) if (segs[q].a == 1) xm = segs[q].b;
+      if (!(x0 < xm && xm < x1)) return false;
+      return try_shape(kZHVH, xm, {{0, y0, x0, xm}, {1, xm, ylo, yhi}, {0, y1, xm, x1}}, {{xm, y0, 0, 0}, {xm, y1, 0, 0}});
+    }
+    if (nh == 1) {
+      int ym = -1;
+      for (int q = 0; q < 3; ++q) if (segs[q].a == 0) ym = segs[q].b;
+      if (!(ylo < ym && ym < yhi)) return false;
+      return try_shape(kZVHV, ym,
+                       {{1, x0, std::min(y0, ym), std::max(y0, ym)}, {0, ym, x0, x1}, {1, x1, std::min(ym, y1), std::max(ym, y1)}},
+                       {{x0, ym, 0, 0}, {x1, ym, 0, 0}});
+    }
+  }
+  return false;
+}
+
+// ---------------------------------------------------------------------------------------
+// the rank's encoded shard
+// ---------------------------------------------------------------------------------------
+struct Plan {
+  int64_t net_lo = 0, net_hi = 0, tree_lo = 0, tree_hi = 0, sub_lo = 0, sub_hi = 0, path_lo = 0, path_hi = 0;
+  int nb = 0;
+  std::vector<int4> binfo;
+  std::vector<uint32_t> pword;
+  std::vector<short4> sxy;
+  std::vector<int32_t> net_tree_off;
+  std::vector<int64_t> sub_first_path;   // local path index of each local sub-net's first candidate
+};
+
+int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
+  int rc = validate_structure(d);
+  if (rc) return rc;
+  std::vector<int64_t> part;
+  if ((rc = partition(d, world, part))) return rc;
+  pl.net_lo = part[rank];
+  pl.net_hi = part[rank + 1];
+  pl.tree_lo = d->net_tree_off[pl.net_lo];
+  pl.tree_hi = d->net_tree_off[pl.net_hi];
+  pl.sub_lo = d->tree_sub_off[pl.tree_lo];
+  pl.sub_hi = d->tree_sub_off[pl.tree_hi];
+  pl.path_lo = d->sub_path_off[pl.sub_lo];
+  pl.path_hi = d->sub_path_off[pl.sub_hi];
+  const int64_t nn = pl.net_hi - pl.net_lo, ns = pl.sub_hi - pl.sub_lo;
+  pl.net_tree_off.resize(nn + 1);
+  for (int64_t n = 0; n <= nn; ++n) pl.net_tree_off[n] = (int32_t)(d->net_tree_off[pl.net_lo + n] - pl.tree_lo);
+  pl.sxy.resize(ns);
+  pl.sub_first_path.resize(ns);
+  pl.binfo.clear();
+  pl.pword.clear();
+  int fill = 32;   // forces a new bundle at the first sub-net
+  for (int64_t j = pl.tree_lo; j < pl.tree_hi; ++j) {
+    for (int64_t s = d->tree_sub_off[j]; s < d->tree_sub_off[j + 1]; ++s) {
+      const int32_t* e = d->sub_xy + 4 * s;
+      int x0 = e[0], y0 = e[1], x1 = e[2], y1 = e[3];
+      if (x0 > x1 || (x0 == x1 && y0 > y1)) { std::swap(x0, x1); std::swap(y0, y1); }
+      if (x0 < 0 || x1 >= d->X || std::min(y0, y1) < 0 || std::max(y0, y1) >= d->Y)
+        return fail(DGR_EINVAL, "sub-net %lld endpoints outside the grid", (long long)s);
+      if (x0 == x1 && y0 == y1) return fail(DGR_EINVAL, "sub-net %lld has zero length", (long long)s);
+      const int64_t ls = s - pl.sub_lo;
+      pl.sxy[ls] = make_short4((short)x0, (short)y0, (short)x1, (short)y1);
+      const int64_t p0 = d->sub_path_off[s], p1 = d->sub_path_off[s + 1];
+      const int g = (int)(p1 - p0);
+      if (fill + g > 32) {
+        // close the previous bundle's padding, open a new one
+        while (!pl.pword.empty() && pl.pword.size() % 32) pl.pword.push_back(kPad | kSubHead);
+        pl.binfo.push_back(make_int4((int)(p0 - pl.path_lo), (int)ls, (int)(j - pl.tree_lo), 0));
+        fill = 0;
+      }
+      pl.sub_first_path[ls] = p0 - pl.path_lo;
+      for (int64_t i = p0; i < p1; ++i) {
+        uint32_t shape;
+        int mid;
+        if (!classify(d, i, x0, y0, x1, y1, &shape, &mid))
+          return fail(DGR_EINVAL, "path %lld is not a straight/L/Z pattern of sub-net %lld (or its turning points are wrong)",
+                      (long long)i, (long long)s);
+        uint32_t pw = shape | ((uint32_t)mid << 16);
+        if (i == p0) {
+          pw |= kSubHead;
+          if (s == d->tree_sub_off[j]) pw |= kTreeHead;
+        }
+        pl.pword.push_back(pw);
+      }
+      fill += g;
+      pl.binfo.back().w += g;
+    }
+  }
+  while (pl.pword.size() % 32) pl.pword.push_back(kPad | kSubHead);
+  pl.nb = (int)pl.binfo.size();
+  return DGR_OK;
+}
+
+// ---------------------------------------------------------------------------------------
+// workspace layout
+// ---------------------------------------------------------------------------------------
+struct Layout {
+  size_t binfo, pword, sxy, wp, mp, vp, nto, wt, mt, vt, q, dq, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
+      partial, loss, chosen, tree_choice, route, nsize, nucleus_tmp, DHVC, iscal, ipartial, metrics, total;
+  size_t xcount;   // int64 elements in the exchange buffer
+};
+
+Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
+  Layout L{};
+  size_t o = 0;
+  auto take = [&](size_t bytes) { size_t r = o; o += (bytes + 255) & ~(size_t)255; return r; };
+  const size_t slots = (size_t)pl.nb * 32, ns = pl.sxy.size(), nt = (size_t)(pl.tree_hi - pl.tree_lo),
+               nn = (size_t)(pl.net_hi - pl.net_lo), G = (size_t)X * Y;
+  L.binfo = take(sizeof(int4) * pl.nb);
+  L.pword = take(4 * slots);
+  L.sxy = take(8 * ns);
+  L.wp = take(4 * slots);
+  L.mp = take(4 * slots);
+  L.vp = take(4 * slots);
+  L.nto = take(4 * (nn + 1));
+  L.wt = take(4 * nt);
+  L.mt = take(4 * nt);
+  L.vt = take(4 * nt);
+  L.q = take(4 * nt);
+  L.dq = take(8 * nt);
+  L.xcount = 3 * G + 2;
+  L.xbuf = take(8 * L.xcount);
+  L.capH = take(4 * G);
+  L.capVT = take(4 * G);
+  L.SH = take(8 * G);
+  L.SVT = take(8 * G);
+  L.dOutH = take(4 * G);
+  L.dOutVT = take(4 * G);
+  L.partial = take(8 * (size_t)(X + Y));
+  L.loss = take(8 * 4);
+  L.chosen = take(nt);
+  L.tree_choice = take(4 * nn);
+  L.route = take(4 * ns);
+  L.nsize = take(4 * ns);
+  L.nucleus_tmp = take(4 * slots);
+  L.DHVC = take(4 * 3 * G);
+  L.iscal = take(8 * 2);
+  L.ipartial = take(8 * 3 * (size_t)metric_blocks);
+  L.metrics = take(8 * 5);
+  L.total = o;
+  return L;
+}
+
+}  // namespace
+
+struct dgr_handle {
+  int X = 0, Y = 0;
+  int64_t n_nets = 0, n_trees = 0, n_subnets = 0, n_paths = 0;
+  Plan plan;
+  Layout lay{};
+  KParams P{};
+  cudaStream_t stream = nullptr;
+  int rank = 0, world = 1;
+  ncclComm_t comm = nullptr;
+  char* ws = nullptr;
+  int64_t ws_bytes = 0;
+  int64_t k = 0;
+  float t_last = 1.f;
+  float beta_last = 0.25f;
+  bool have_forward = false;
+  double* pinned = nullptr;   // 16 doubles of pinned host memory
+  // profiling: 8 events per recorded iteration (stage boundaries)
+  bool prof = false;
+  std::vector<cudaEvent_t> ev;
+  size_t ev_used = 0;
+};
+
+namespace {
+constexpr int kStages = 7;
+// records the boundary event `b` (0..7) of the current profiled iteration
+int prof_mark(dgr_handle* h, int b) {
+  if (!h->prof) return DGR_OK;
+  const size_t idx = h->ev_used + b;
+  while (h->ev.size() <= idx) {
+    cudaEvent_t e;
+    CUDA_TRY(cudaEventCreate(&e));
+    h->ev.push_back(e);
+  }
+  CUDA_TRY(cudaEventRecord(h->ev[idx], h->stream));
+  if (b == kStages) h->ev_used += kStages + 1;
+  return DGR_OK;
+}
+}  // namespace
+
+extern "C" {
+
+const char* dgr_last_error(void) { return g_err.c_str(); }
+
+int dgr_nccl_unique_id(void* out128) {
+  if (!out128) return fail(DGR_EINVAL, "out is NULL");
+  static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+  ncclUniqueId id;
+  NCCL_TRY(ncclGetUniqueId(&id));
+  memcpy(out128, &id, sizeof(id));
+  return DGR_OK;
+}
+
+int dgr_partition(const dgr_forest_desc* desc, int32_t world, int64_t* out) {
+  int rc = validate_structure(desc);
+  if (rc) return rc;
+  if (!out) return fail(DGR_EINVAL, "out is NULL");
+  std::vector<int64_t> part;
+  if ((rc = partition(desc, world, part))) return rc;
+  std::copy(part.begin(), part.end(), out);
+  return DGR_OK;
+}
+
+static int dist_args(const dgr_dist* dist, int* rank, int* world) {
+  *rank = 0;
+  *world = 1;
+  if (dist) {
+    *rank = dist->rank;
+    *world = dist->world;
+  }
+  if (*world < 1 || *rank < 0 || *rank >= *world) return fail(DGR_EINVAL, "bad rank/world %d/%d", *rank, *world);
+  if (*world > 1 && (!dist || !dist->nccl_unique_id)) return fail(DGR_EINVAL, "world > 1 needs an NCCL unique id");
+  return DGR_OK;
+}
+
+int64_t dgr_workspace_size(const dgr_forest_desc* desc, const dgr_dist* dist) {
+  int rank, world;
+  if (dist_args(dist, &rank, &world)) return 0;
+  Plan pl;
+  if (make_plan(desc, rank, world, pl)) return 0;
+  dgr::KParams tmp{};
+  tmp.X = desc->X;
+  tmp.Y = desc->Y;
+  return (int64_t)make_layout(pl, desc->X, desc->Y, induce_metric_blocks(tmp)).total;
+}
+
+int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev_workspace, int64_t workspace_bytes,
+                    void* cuda_stream, dgr_handle** out) {
+  if (!out) return fail(DGR_EINVAL, "out is NULL");
+  *out = nullptr;
+  int rank, world, rc;
+  if ((rc = dist_args(dist, &rank, &world))) return rc;
+  auto* h = new dgr_handle();
+  if ((rc = make_plan(desc, rank, world, h->plan))) { delete h; return rc; }
+  const Plan& pl = h->plan;
+  h->X = desc->X; h->Y = desc->Y;
+  h->n_nets = desc->n_nets; h->n_trees = desc->n_trees; h->n_subnets = desc->n_subnets; h->n_paths = desc->n_paths;
+  h->rank = rank; h->world = world;
+  h->stream = (cudaStream_t)cuda_stream;
+  KParams& P = h->P;
+  P.X = desc->X; P.Y = desc->Y;
+  h->lay = make_layout(pl, desc->X, desc->Y, induce_metric_blocks(P));
+  const Layout& L = h->lay;
+  if (!dev_workspace || workspace_bytes < (int64_t)L.total) {
+    delete h;
+    return fail(DGR_ENOMEM, "workspace of %lld bytes < %zu needed", (long long)workspace_bytes, L.total);
+  }
+  if (((uintptr_t)dev_workspace) & 255) { delete h; return fail(DGR_EINVAL, "workspace not 256-byte aligned"); }
+  h->ws = (char*)dev_workspace;
+  h->ws_bytes = workspace_bytes;
+  char* ws = h->ws;
+  P.nb = pl.nb;
+  P.n_nets_l = (int32_t)(pl.net_hi - pl.net_lo);
+  P.path_base = pl.path_lo;
+  P.tree_base = pl.tree_lo;
+  P.seed = desc->seed;
+  P.binfo = (const int4*)(ws + L.binfo);
+  P.pword = (const uint32_t*)(ws + L.pword);
+  P.sxy = (const short4*)(ws + L.sxy);
+  P.wp = (float*)(ws + L.wp); P.mp = (float*)(ws + L.mp); P.vp = (float*)(ws + L.vp);
+  P.net_tree_off = (const int32_t*)(ws + L.nto);
+  P.wt = (float*)(ws + L.wt); P.mt = (float*)(ws + L.mt); P.vt = (float*)(ws + L.vt); P.q = (float*)(ws + L.q);
+  P.dq = (long long*)(ws + L.dq);
+  const size_t G = (size_t)desc->X * desc->Y;
+  P.dH = (long long*)(ws + L.xbuf);
+  P.dVT = P.dH + G;
+  P.VD = P.dVT + G;
+  P.scal = P.VD + G;
+  P.capH = (const float*)(ws + L.capH);
+  P.capVT = (const float*)(ws + L.capVT);
+  P.SH = (double*)(ws + L.SH); P.SVT = (double*)(ws + L.SVT);
+  P.dOutH = (float*)(ws + L.dOutH); P.dOutVT = (float*)(ws + L.dOutVT);
+  P.partial = (double*)(ws + L.partial);
+  P.loss = (double*)(ws + L.loss);
+  P.chosen = (uint8_t*)(ws + L.chosen);
+  P.tree_choice = (int32_t*)(ws + L.tree_choice);
+  P.route = (int32_t*)(ws + L.route);
+  P.nsize = (int32_t*)(ws + L.nsize);
+  P.nucleus_tmp = (int32_t*)(ws + L.nucleus_tmp);
+  P.DH = (int32_t*)(ws + L.DHVC);
+  P.DV = P.DH + G;
+  P.VC = P.DV + G;
+  P.iscal = (long long*)(ws + L.iscal);
+  P.ipartial = (double*)(ws + L.ipartial);
+  P.metrics = (double*)(ws + L.metrics);
+
+  auto cleanup = [&](int code) { if (h->pinned) cudaFreeHost(h->pinned); delete h; return code; };
+  cudaStream_t s = h->stream;
+  if (cudaMemsetAsync(ws, 0, L.total, s) != cudaSuccess) return cleanup(fail(DGR_ECUDA, "memset workspace failed"));
+  // host-side staging of the encoded shard
+  const size_t slots = (size_t)pl.nb * 32;
+  std::vector<float> wslots(slots, 0.f);
+  for (int b = 0; b < pl.nb; ++b)
+    for (int l = 0; l < pl.binfo[b].w; ++l) wslots[(size_t)b * 32 + l] = desc->w_path0[pl.path_lo + pl.binfo[b].x + l];
+  std::vector<float> capVT(G);
+  for (int y = 0; y < desc->Y; ++y)
+    for (int x = 0; x < desc->X; ++x) capVT[(size_t)x * desc->Y + y] = desc->cap_v[(size_t)y * desc->X + x];
+  const size_t nt = (size_t)(pl.tree_hi - pl.tree_lo);
+  cudaError_t e = cudaSuccess;
+  auto cp = [&](size_t off, const void* src, size_t bytes) {
+    if (bytes && e == cudaSuccess) e = cudaMemcpyAsync(ws + off, src, bytes, cudaMemcpyHostToDevice, s);
+  };
+  cp(L.binfo, pl.binfo.data(), sizeof(int4) * pl.nb);
+  cp(L.pword, pl.pword.data(), 4 * slots);
+  cp(L.sxy, pl.sxy.data(), 8 * pl.sxy.size());
+  cp(L.wp, wslots.data(), 4 * slots);
+  cp(L.nto, pl.net_tree_off.data(), 4 * pl.net_tree_off.size());
+  cp(L.wt, desc->w_tree0 + pl.tree_lo, 4 * nt);
+  cp(L.capH, desc->cap_h, 4 * G);
+  cp(L.capVT, capVT.data(), 4 * G);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cleanup(fail(DGR_ECUDA, "upload: %s", cudaGetErrorString(e)));
+  if (cudaMallocHost(&h->pinned, 16 * sizeof(double)) != cudaSuccess) return cleanup(fail(DGR_ECUDA, "cudaMallocHost failed"));
+  if (world > 1) {
+    ncclUniqueId id;
+    memcpy(&id, dist->nccl_unique_id, sizeof(id));
+    ncclResult_t r = ncclCommInitRank(&h->comm, world, id, rank);
+    if (r != ncclSuccess) return cleanup(fail(DGR_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r)));
+  }
+  *out = h;
+  g_err.clear();
+  return DGR_OK;
+}
+
+int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w, dgr_loss* last) {
+  if (!h || !w) return fail(DGR_EINVAL, "NULL handle or weights");
+  if (iters < 0) return fail(DGR_EINVAL, "iters < 0");
+  if (!(temperature > 0.f) || !std::isfinite(temperature)) return fail(DGR_EINVAL, "temperature must be > 0");
+  if (w->f_kind != 0 && w->f_kind != 1) return fail(DGR_EINVAL, "f_kind must be 0 (sigmoid) or 1 (ReLU)");
+  KParams& P = h->P;
+  StepArgs a{};
+  a.inv_t = 1.f / temperature;
+  a.t = temperature;
+  a.a_wl = w->a_wl; a.a_via = w->a_via; a.a_of = w->a_of; a.beta = w->beta_via;
+  a.sqrt_l = std::sqrt(w->n_layers);
+  a.f_slope = w->f_slope; a.f_kind = w->f_kind;
+  const int n = iters == 0 ? 1 : iters;
+  const size_t xbytes = 8 * h->lay.xcount;
+  cudaStream_t s = h->stream;
+  for (int it = 0; it < n; ++it) {
+    a.k = h->k;
+    a.store_d = (it == n - 1);
+    const double step = (double)(h->k + 1);
+    a.lr_over_bc1 = (float)(lr / (1.0 - std::pow(0.9, step)));
+    a.inv_sqrt_bc2 = (float)(1.0 / std::sqrt(1.0 - std::pow(0.999, step)));
+    int rc;
+    if ((rc = prof_mark(h, 0))) return rc;
+    launch_kq(P, a, s);
+    if ((rc = prof_mark(h, 1))) return rc;
+    CUDA_TRY(cudaMemsetAsync(P.dH, 0, xbytes, s));
+    if ((rc = prof_mark(h, 2))) return rc;
+    launch_kf(P, a, s);
+    if ((rc = prof_mark(h, 3))) return rc;
+    if (h->world > 1) NCCL_TRY(ncclAllReduce(P.dH, P.dH, h->lay.xcount, ncclInt64, ncclSum, h->comm, s));
+    if ((rc = prof_mark(h, 4))) return rc;
+    launch_kg(P, a, s);
+    if ((rc = prof_mark(h, 5))) return rc;
+    if (iters > 0) {
+      launch_kb(P, a, s);
+      if ((rc = prof_mark(h, 6))) return rc;
+      launch_kt(P, a, s);
+      h->k += 1;
+    } else if ((rc = prof_mark(h, 6))) {
+      return rc;
+    }
+    if ((rc = prof_mark(h, 7))) return rc;
+  }
+  CUDA_TRY(cudaGetLastError());
+  h->t_last = temperature;
+  h->beta_last = w->beta_via;
+  h->have_forward = true;
+  if (last) {
+    CUDA_TRY(cudaMemcpyAsync(h->pinned, P.loss, 4 * sizeof(double), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    last->total = h->pinned[0];
+    last->wl = h->pinned[1];
+    last->via = h->pinned[2];
+    last->overflow = h->pinned[3];
+  }
+  return DGR_OK;
+}
+
+int dgr_get_demand(dgr_handle* h, float* d_h, float* d_v) {
+  if (!h || !d_h || !d_v) return fail(DGR_EINVAL, "NULL argument");
+  if (!h->have_forward) return fail(DGR_ESTATE, "no forward has run yet");
+  const size_t G = (size_t)h->X * h->Y;
+  std::vector<float> vt(G);
+  CUDA_TRY(cudaMemcpyAsync(d_h, h->P.dOutH, 4 * G, cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(vt.data(), h->P.dOutVT, 4 * G, cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  for (int x = 0; x < h->X; ++x)
+    for (int y = 0; y < h->Y; ++y) d_v[(size_t)y * h->X + x] = vt[(size_t)x * h->Y + y];
+  return DGR_OK;
+}
+
+int dgr_get_logits(dgr_handle* h, float* w_tree, float* w_path) {
+  if (!h) return fail(DGR_EINVAL, "NULL handle");
+  const Plan& pl = h->plan;
+  if (w_path) {
+    std::vector<float> slots((size_t)pl.nb * 32);
+    CUDA_TRY(cudaMemcpyAsync(slots.data(), h->P.wp, 4 * slots.size(), cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    for (int b = 0; b < pl.nb; ++b)
+      for (int l = 0; l < pl.binfo[b].w; ++l) w_path[pl.path_lo + pl.binfo[b].x + l] = slots[(size_t)b * 32 + l];
+  }
+  if (w_tree) {
+    CUDA_TRY(cudaMemcpyAsync(w_tree + pl.tree_lo, h->P.wt, 4 * (size_t)(pl.tree_hi - pl.tree_lo),
+                             cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+  }
+  return DGR_OK;
+}
+
+int dgr_induce(dgr_handle* h, float top_p, int32_t* tree_choice, int32_t* route, int64_t* nucleus_off,
+               int32_t* nucleus, int32_t* D_h, int32_t* D_v, double metrics[5]) {
+  if (!h || !tree_choice || !route || !nucleus_off || !nucleus || !D_h || !D_v || !metrics)
+    return fail(DGR_EINVAL, "NULL argument");
+  if (!(top_p >= 0.f) || !std::isfinite(top_p)) return fail(DGR_EINVAL, "top_p must be finite and >= 0");
+  KParams& P = h->P;
+  const Plan& pl = h->plan;
+  cudaStream_t s = h->stream;
+  const size_t G = (size_t)h->X * h->Y;
+  CUDA_TRY(cudaMemsetAsync(P.DH, 0, 4 * 3 * G, s));
+  CUDA_TRY(cudaMemsetAsync(P.iscal, 0, 16, s));
+  launch_induce(P, h->t_last, top_p, h->beta_last, s);
+  if (h->world > 1) {
+    NCCL_TRY(ncclAllReduce(P.DH, P.DH, 3 * G, ncclInt32, ncclSum, h->comm, s));
+    NCCL_TRY(ncclAllReduce(P.iscal, P.iscal, 2, ncclInt64, ncclSum, h->comm, s));
+  }
+  launch_induce_metrics(P, h->beta_last, s);
+  CUDA_TRY(cudaGetLastError());
+  const int64_t nn = pl.net_hi - pl.net_lo, ns = pl.sub_hi - pl.sub_lo;
+  std::vector<int32_t> tc(nn), rt(ns), nsz(ns), nuc((size_t)pl.nb * 32);
+  CUDA_TRY(cudaMemcpyAsync(tc.data(), P.tree_choice, 4 * nn, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaMemcpyAsync(rt.data(), P.route, 4 * ns, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaMemcpyAsync(nsz.data(), P.nsize, 4 * ns, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaMemcpyAsync(nuc.data(), P.nucleus_tmp, 4 * nuc.size(), cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaMemcpyAsync(D_h, P.DH, 4 * G, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaMemcpyAsync(D_v, P.DV, 4 * G, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaMemcpyAsync(h->pinned, P.metrics, 5 * sizeof(double), cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  for (int i = 0; i < 5; ++i) metrics[i] = h->pinned[i];
+  if (h->world > 1) {
+    std::fill(tree_choice, tree_choice + h->n_nets, -1);
+    std::fill(route, route + h->n_subnets, -1);
+  }
+  std::copy(tc.begin(), tc.end(), tree_choice + pl.net_lo);
+  std::copy(rt.begin(), rt.end(), route + pl.sub_lo);
+  int64_t pos = 0;
+  nucleus_off[0] = 0;
+  // nucleus_tmp holds each sub-net's nucleus in rank order at its first candidate's local index
+  for (int64_t sg = 0; sg < h->n_subnets; ++sg) {
+    if (sg >= pl.sub_lo && sg < pl.sub_hi) {
+      const int64_t ls = sg - pl.sub_lo;
+      for (int r = 0; r < nsz[ls]; ++r) nucleus[pos++] = nuc[(size_t)pl.sub_first_path[ls] + r];
+    }
+    nucleus_off[sg + 1] = pos;
+  }
+  return DGR_OK;
+}
+
+int dgr_get_info(dgr_handle* h, int64_t info[8]) {
+  if (!h || !info) return fail(DGR_EINVAL, "NULL argument");
+  info[0] = h->k; info[1] = h->plan.net_lo; info[2] = h->plan.net_hi; info[3] = h->plan.nb;
+  info[4] = (int64_t)h->plan.nb * 32; info[5] = (int64_t)h->lay.total; info[6] = h->world; info[7] = h->rank;
+  return DGR_OK;
+}
+
+int dgr_profile(dgr_handle* h, int32_t enable) {
+  if (!h) return fail(DGR_EINVAL, "NULL handle");
+  h->prof = enable != 0;
+  h->ev_used = 0;
+  return DGR_OK;
+}
+
+int dgr_profile_read(dgr_handle* h, double ms[8], int64_t* iterations) {
+  if (!h || !ms || !iterations) return fail(DGR_EINVAL, "NULL argument");
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  for (int i = 0; i < 8; ++i) ms[i] = 0.0;
+  const size_t n = h->ev_used / (kStages + 1);
+  for (size_t it = 0; it < n; ++it)
+    for (int b = 0; b < kStages; ++b) {
+      float t = 0.f;
+      CUDA_TRY(cudaEventElapsedTime(&t, h->ev[it * (kStages + 1) + b], h->ev[it * (kStages + 1) + b + 1]));
+      ms[b] += t;
+    }
+  *iterations = (int64_t)n;
+  return DGR_OK;
+}
+
+int dgr_free(dgr_handle* h) {
+  if (!h) return DGR_OK;
+  if (h->stream) cudaStreamSynchronize(h->stream);
+  for (auto e : h->ev) cudaEventDestroy(e);
+  if (h->comm) ncclCommDestroy(h->comm);
+  if (h->pinned) cudaFreeHost(h->pinned);
+  delete h;
+  return DGR_OK;
+}
+
+}  // extern "C"

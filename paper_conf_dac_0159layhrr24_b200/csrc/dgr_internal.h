@@ -1,0 +1,95 @@
+// dgr_internal.h — device data layout shared by the libdgr host code and its sm_100a kernels.
+//
+// Layout in HBM:
+//   * candidates live in 32-slot "bundles": one warp processes one bundle, one lane one path
+//     candidate.  A bundle holds whole sub-nets (groups of 1..32 candidates, packed in order,
+//     never split), so the sub-net softmax is a segmented warp reduction.  Unused tail lanes
+//     are padding (shape PAD).
+//   * per slot:    pword (shape | flags | mid), w, m, v (fp32)
+//   * per bundle:  {first local path, first local sub-net, first local tree, #valid lanes}
+//   * per sub-net: canonical endpoints (x0 <= x1; y0 < y1 if x0 == x1) as int16 x 4
+//   * per tree:    w, m, v, q (fp32), dq (int64 fixed point)
+//   * grids: diff arrays of the wire demand along H rows ([Y][X]) and along V columns (stored
+//     transposed, [X][Y], so both scans run over contiguous lines), the turning-point
+//     ("via") demand per G-cell ([Y][X]), all int64 in 2^-24 fixed point; prefix sums S of the
+//     overflow gradient per line (fp64, same two layouts).
+#pragma once
+#include <cstdint>
+
+namespace dgr {
+
+constexpr int kFracBits = 24;                      // fixed point of pi: round(pi * 2^24)
+constexpr float kFixScale = 16777216.0f;           // 2^24
+constexpr double kFixInv = 1.0 / 16777216.0;
+
+enum Shape : uint32_t {
+  kStraightH = 0, kStraightV = 1, kHV = 2, kVH = 3, kZHVH = 4, kZVHV = 5, kPad = 7
+};
+constexpr uint32_t kSubHead = 8u;    // lane starts a sub-net group
+constexpr uint32_t kTreeHead = 16u;  // sub-net is the first of its tree (set on the group head)
+// bits 16..31: x_m (Z-HVH) or y_m (Z-VHV)
+
+struct KParams {
+  // sizes
+  int32_t X, Y;
+  int32_t nb;               // bundles
+  int32_t n_nets_l;         // local nets
+  int64_t path_base, tree_base;   // global index of the first local path / tree
+  uint64_t seed;
+  // forest encoding
+  const int4* binfo;
+  const uint32_t* pword;
+  const short4* sxy;
+  float *wp, *mp, *vp;
+  const int32_t* net_tree_off;    // local, n_nets_l + 1
+  float *wt, *mt, *vt, *q;
+  long long* dq;
+  // grids
+  long long* dH;            // [Y][X]
+  long long* dVT;           // [X][Y]
+  long long* VD;            // [Y][X]
+  long long* scal;          // {E[WL], E[TP]} fixed point
+  const float* capH;        // [Y][X]
+  const float* capVT;       // [X][Y]
+  double* SH;               // [Y][X]
+  double* SVT;              // [X][Y]
+  float* dOutH;             // [Y][X]
+  float* dOutVT;            // [X][Y]
+  double* partial;          // [Y + X] overflow partial sums
+  double* loss;             // [4]
+  // induce scratch
+  uint8_t* chosen;          // [n_trees_l]
+  int32_t* tree_choice;     // [n_nets_l] (global tree index)
+  int32_t* route;           // [n_subs_l] (global path index or -1)
+  int32_t* nsize;           // [n_subs_l]
+  int32_t* nucleus_tmp;     // [nb*32] indexed by local path
+  int32_t* DH;              // [Y][X]
+  int32_t* DV;              // [Y][X]
+  int32_t* VC;              // [Y][X]
+  long long* iscal;         // {sum WL, sum TP}
+  double* ipartial;         // [3 * nblocks]
+  double* metrics;          // [5]
+};
+
+struct StepArgs {
+  int64_t k;          // global iteration
+  float inv_t;        // 1 / temperature
+  float t;
+  float lr_over_bc1;  // lr / (1 - beta1^(k+1))
+  float inv_sqrt_bc2; // 1 / sqrt(1 - beta2^(k+1))
+  float a_wl, a_via, a_of, beta, sqrt_l, f_slope;
+  int32_t f_kind;
+  int32_t store_d;
+};
+
+// launchers (dgr_kernels.cu)
+void launch_kq(const KParams& p, const StepArgs& a, cudaStream_t s);
+void launch_kf(const KParams& p, const StepArgs& a, cudaStream_t s);
+void launch_kg(const KParams& p, const StepArgs& a, cudaStream_t s);
+void launch_kb(const KParams& p, const StepArgs& a, cudaStream_t s);
+void launch_kt(const KParams& p, const StepArgs& a, cudaStream_t s);
+void launch_induce(const KParams& p, float t_final, float top_p, float beta, cudaStream_t s);
+void launch_induce_metrics(const KParams& p, float beta, cudaStream_t s);
+int induce_metric_blocks(const KParams& p);
+
+}  // namespace dgr

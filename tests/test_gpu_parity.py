@@ -1,0 +1,249 @@
+"""Parity of the sm_100a path (through the C ABI) against the fp64 oracle, element by element.
+
+Tolerance (BASELINE.json north_star; reading Q21): floats |gpu - oracle| <= 1e-4 * max(|oracle|, 1)
+elementwise for demand and logits, relative 1e-4 for the scalar loss terms; integer outputs
+(one-hot demand, induced routes where the top-1/top-2 margin exceeds 1e-3) bit-exact.
+"""
+import copy
+
+import numpy as np
+import pytest
+
+import forestgen
+import oracle
+import paper_conf_dac_0159layhrr24_b200 as dgr
+from tests import _ref
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-4
+
+
+def assert_close(a, b, tol=TOL, what=""):
+    a = np.asarray(a, np.float64); b = np.asarray(b, np.float64)
+    err = np.abs(a - b) / np.maximum(np.abs(b), 1.0)
+    i = int(np.argmax(err)) if err.size else 0
+    assert err.size == 0 or err.max() <= tol, f"{what}: max scaled err {err.max():.3e} at {i}: gpu {a.flat[i]} oracle {b.flat[i]}"
+
+
+def assert_rel(a, b, tol=TOL, what=""):
+    assert abs(a - b) <= tol * max(abs(b), 1e-12), f"{what}: gpu {a} oracle {b}"
+
+
+def ow(w: dgr.Weights):
+    return oracle.weights(a_wl=w.a_wl, a_via=w.a_via, a_of=w.a_of, beta=w.beta_via, n_layers=w.n_layers,
+                          f_kind=w.f_kind, f_slope=w.f_slope)
+
+
+@pytest.fixture(scope="module")
+def forests():
+    return {n: forestgen.generate(n) for n in ("tiny", "c1e4", "ispd18")}
+
+
+def run_both(f, schedule, W=None, lr=0.3):
+    """schedule: list of (iters, t).  Returns (solver, oracle, gpu losses, oracle losses)."""
+    W = W or dgr.Weights()
+    s = dgr.Solver(f)
+    o = oracle.Oracle(f)
+    gl, ol = [], []
+    for iters, t in schedule:
+        gl.append(s.step(iters, t, lr, W))
+        ol.append(o.step(iters, t, lr, ow(W)))
+    return s, o, gl, ol
+
+
+def probes(f, schedule, W=None):
+    """Conditioning probe: the oracle source built with real = float (the paper's presumed fp32,
+    rounding everywhere), replaying the same schedule."""
+    W = ow(W or dgr.Weights())
+    o = oracle.Oracle(f, fp32=True)
+    for iters, t in schedule:
+        o.step(iters, t, 0.3, W)
+    return o
+
+
+def scaled_err(a, b):
+    a = np.asarray(a, np.float64); b = np.asarray(b, np.float64)
+    return np.abs(a - b) / np.maximum(np.abs(b), 1.0)
+
+
+def compare_state(s, o, what, probe=None, max_ill=0.01):
+    """Element-wise parity of demand and logits.  Without a probe: every element within TOL.
+    With the fp32 probe (multi-iteration runs, DESIGN.md §3 Q21b): every element within TOL, or, where
+    an fp32 evaluation of the same formulation is itself further than TOL from fp64 (Adam turns a
+    near-zero gradient's rounding into an lr-sized step), no further from fp64 than 10x that fp32
+    evaluation (one sample of fp32 rounding; the kernel rounds elsewhere); such elements must stay
+    below `max_ill` of the total."""
+    gdh, gdv = s.demand()
+    odh, odv = o.demand()
+    gwt, gwp = s.logits()
+    owt, owp = o.logits()
+    if probe is None:
+        assert_close(gdh, odh, what=what + " d_h")
+        assert_close(gdv, odv, what=what + " d_v")
+        assert_close(gwp, owp, what=what + " w_path")
+        assert_close(gwt, owt, what=what + " w_tree")
+        return
+    pdh, pdv = probe.demand()
+    pwt, pwp = probe.logits()
+    for g, r, pr, nm in ((gdh, odh, pdh, "d_h"), (gdv, odv, pdv, "d_v"), (gwp, owp, pwp, "w_path"),
+                         (gwt, owt, pwt, "w_tree")):
+        eg, e32 = scaled_err(g, r), scaled_err(pr, r)
+        strict = eg <= TOL
+        relaxed = ~strict & (eg <= 10.0 * e32)
+        bad = ~strict & ~relaxed
+        i = int(np.argmax(np.where(bad, eg, -1))) if bad.any() else 0
+        assert not bad.any(), (f"{what} {nm}: {bad.sum()} elements beyond TOL and beyond 10x the fp32 probe; "
+                               f"worst {i}: gpu {g.flat[i]} fp64 {r.flat[i]} fp32 {pr.flat[i]}")
+        assert relaxed.mean() <= max_ill, f"{what} {nm}: {relaxed.sum()} of {relaxed.size} need the fp32 clause"
+
+
+@pytest.mark.parametrize("beta", [0.0, 0.25])
+def test_one_hot_demand_is_bit_exact(forests, beta):
+    f = copy.deepcopy(forests["c1e4"])
+    rng = np.random.default_rng(0)
+    wt = np.zeros(f.n_trees, np.float32); wp = np.zeros(f.n_paths, np.float32)
+    pick = [int(rng.integers(f.sub_path_off[sn], f.sub_path_off[sn + 1])) for sn in range(f.n_subnets)]
+    wp[pick] = 1000.0                       # winner gap 1000: exact 0/1 probabilities in fp32 and fp64
+    sel = []
+    for n in range(f.n_nets):
+        j = int(rng.integers(f.net_tree_off[n], f.net_tree_off[n + 1])); wt[j] = 1000.0
+        sel += [pick[sn] for sn in range(f.tree_sub_off[j], f.tree_sub_off[j + 1])]
+    f.w_tree0, f.w_path0 = wt, wp
+    W = dgr.Weights(beta_via=beta)
+    s = dgr.Solver(f)
+    s.step(0, 1.0, 0.3, W)
+    gdh, gdv = s.demand()
+    rdh, rdv = _ref.rasterise(f, sel, beta=beta)
+    assert np.array_equal(gdh.astype(np.float64), rdh) and np.array_equal(gdv.astype(np.float64), rdv)
+    o = oracle.Oracle(f)
+    o.forward(1.0, ow(W))
+    odh, odv = o.demand()
+    assert np.array_equal(gdh.astype(np.float64), odh) and np.array_equal(gdv.astype(np.float64), odv)
+
+
+@pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18"])
+@pytest.mark.parametrize("f_kind", [0, 1])
+def test_forward_parity(forests, name, f_kind):
+    W = dgr.Weights(f_kind=f_kind)
+    f = forests[name]
+    s, o, gl, ol = run_both(f, [(0, 0.7)], W)
+    gdh, gdv = s.demand()
+    odh, odv = o.demand()
+    assert_close(gdh, odh, what="d_h"); assert_close(gdv, odv, what="d_v")
+    for i, nm in enumerate(("total", "wl", "via", "overflow")):
+        assert_rel(gl[0][i], ol[0][i], what=nm)
+    assert s.iteration == 0
+
+
+@pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18"])
+def test_one_iteration_parity(forests, name):
+    s, o, gl, ol = run_both(forests[name], [(1, 1.0)])
+    compare_state(s, o, name)
+    assert s.iteration == 1
+
+
+@pytest.mark.parametrize("name,schedule", [
+    ("tiny", [(100, 1.0), (100, 0.9)]),                  # BASELINE.json: tiny, 200 iterations
+    ("c1e4", [(100, 1.0)]),
+])
+def test_trajectory_parity(forests, name, schedule):
+    f = forests[name]
+    s, o, gl, ol = run_both(f, schedule)
+    compare_state(s, o, name, probe=probes(f, schedule))
+    for i, nm in enumerate(("total", "wl", "via", "overflow")):
+        assert_rel(gl[-1][i], ol[-1][i], what=nm)
+
+
+def test_relu_trajectory_parity(forests):
+    """ReLU's gradient is a step in d: trajectories are piecewise and chaotic, so parity
+    is checked over 5 iterations (the Table 1 objective's quality is checked by the oracle tests)."""
+    W = dgr.Weights(f_kind=1)
+    for name in ("tiny", "c1e4"):
+        sched = [(5, 1.0)]
+        s, o, gl, ol = run_both(forests[name], sched, W)
+        compare_state(s, o, "relu " + name, probe=probes(forests[name], sched, W))
+
+
+def test_split_calls_and_determinism(forests):
+    f = forests["c1e4"]
+    a = dgr.Solver(f); b = dgr.Solver(f)
+    a.step(10, 0.9, 0.3)
+    for _ in range(5):
+        b.step(2, 0.9, 0.3)
+    assert np.array_equal(a.logits()[1], b.logits()[1]) and np.array_equal(a.logits()[0], b.logits()[0])
+    assert all(np.array_equal(x, y) for x, y in zip(a.demand(), b.demand()))
+
+
+@pytest.mark.parametrize("name", ["tiny", "c1e4"])
+def test_induce_parity(forests, name):
+    f = forests[name]
+    s, o, _, _ = run_both(f, [(60, 1.0), (40, 0.9)])
+    g = s.induce(0.9)
+    r = o.induce(0.9, beta=0.25, t_final=0.9)
+    sure_tree = r.margin_tree > 1e-3
+    assert np.array_equal(g.tree_choice[sure_tree], r.tree_choice[sure_tree])
+    # routes: bit-exact where the sub-net's tree choice and top-1 / top-2 margin are clear
+    path_tree = np.repeat(np.arange(f.n_trees), np.diff(f.tree_sub_off))
+    sub_net = np.repeat(np.arange(f.n_nets), np.diff(f.net_tree_off))[path_tree]
+    sure = sure_tree[sub_net] & (r.margin_route > 1e-3)
+    assert np.array_equal(g.route[sure], r.route[sure])
+    assert sure.mean() > 0.5
+    # nuclei where the cumulative sums are clear of top_p
+    for sn in np.nonzero(sure & (r.margin_nucleus > 1e-3))[0][:2000]:
+        assert np.array_equal(g.nucleus[g.nucleus_off[sn]:g.nucleus_off[sn + 1]],
+                              r.nucleus[r.nucleus_off[sn]:r.nucleus_off[sn + 1]])
+    # the integer grids and metrics of the GPU's own routes, recomputed independently
+    routes = [int(i) for i in g.route if i >= 0]
+    dh, dv = _ref.rasterise(f, routes, beta=0.0)
+    assert np.array_equal(g.D_h, dh.astype(np.int32)) and np.array_equal(g.D_v, dv.astype(np.int32))
+    assert g.metrics[3] == dh.sum() + dv.sum()
+    if sure.all():
+        assert np.array_equal(g.D_h, r.D_h) and np.array_equal(g.D_v, r.D_v)
+        np.testing.assert_allclose(g.metrics, r.metrics, rtol=1e-9)
+
+
+def test_induce_metrics_exact_on_oracle_routes(forests):
+    """Metrics of identical routes: start from w0 (both sides read the same fp32 logits)."""
+    f = forests["c1e4"]
+    s = dgr.Solver(f); o = oracle.Oracle(f)
+    s.step(0, 1.0, 0.3)
+    g = s.induce(0.9)
+    r = o.induce(0.9, beta=0.25, t_final=1.0)
+    assert np.array_equal(g.tree_choice, r.tree_choice)
+    assert np.array_equal(g.route, r.route)
+    assert np.array_equal(g.D_h, r.D_h) and np.array_equal(g.D_v, r.D_v)
+    np.testing.assert_allclose(g.metrics, r.metrics, rtol=1e-12)
+
+
+def test_empty_and_degenerate_forests():
+    # no routed nets at all: demand 0, loss = a3 * sum_e f(cap_e)
+    f = forestgen.generate("tiny", n_nets=0)
+    s = dgr.Solver(f)
+    gl = s.step(3, 1.0, 0.3)
+    o = oracle.Oracle(f)
+    ol = o.step(3, 1.0, 0.3, ow(dgr.Weights()))
+    assert_rel(gl[0], ol[0], what="empty loss")
+    assert not s.demand()[0].any()
+    # a 2x2 grid
+    f = forestgen.generate(dict(X=2, Y=2, n_nets=6, pins_mode=0, pins_min=2, pins_max=4, box_mode=0, box_min=2,
+                                box_max=2, track=1.0, n_tree_cand=2, z_cap=0, seed=3))
+    s, o, gl, ol = run_both(f, [(20, 1.0)])
+    compare_state(s, o, "2x2", probe=probes(f, [(20, 1.0)]))
+
+
+def test_full_size_sampled_parity():
+    """BASELINE.json configs[3] (ispd19, ~1e6 nets, the bench workload) in the bench's launch
+    configuration: full demand / loss of the first forward and every logit after one iteration."""
+    f = forestgen.generate("ispd19")
+    s = dgr.Solver(f)
+    o = oracle.Oracle(f)
+    gl = s.step(0, 1.0, 0.3)
+    ol = o.step(0, 1.0, 0.3, ow(dgr.Weights()))
+    for i in range(4):
+        assert_rel(gl[i], ol[i], what="loss")
+    gdh, gdv = s.demand(); odh, odv = o.demand()
+    assert_close(gdh, odh, what="d_h"); assert_close(gdv, odv, what="d_v")
+    s.step(1, 1.0, 0.3)
+    o.step(1, 1.0, 0.3, ow(dgr.Weights()))
+    compare_state(s, o, "ispd19", probe=probes(f, [(0, 1.0), (1, 1.0)]), max_ill=1e-4)
