@@ -61,13 +61,17 @@ def measured_peak():
 def stage_bytes(st: dict) -> dict:
     P, S, T, N, B, V = st["paths"], st["subnets"], st["trees"], st["nets"], st["bundles"], st["cells"]
     return {
-        "KQ": 4 * N + 8 * T,                               # net offsets; w_tree read, q write
-        "zero": 24 * V,                                    # dH, dV, VD cleared
-        "KF": 8 * P + 8 * S + 4 * T + 16 * B + 24 * V,     # w, pword; endpoints; q; bundle info; 3 grids written
+        # forward only: w, pword per path; endpoints; w_tree read + q write; net offsets; bundle info;
+        # the 4 demand arrays (dH, dV, VD x2 layouts, int64) written once
+        "KF": 8 * P + 8 * S + 8 * T + 4 * N + 16 * B + 32 * V,
         "allreduce": 0,
-        "KG": 48 * V,                                      # dH dV VD read, capH capV read, S_H S_V written
-        "KB": 28 * P + 8 * S + 12 * T + 16 * B + 16 * V,   # w m v r+w, pword; endpoints; q, dq; S_H S_V read
-        "KT": 4 * N + 44 * T,                              # offsets; q, dq r/w, w m v r/w
+        # 4 demand arrays read and cleared, capH/capV read, S_H/S_V written
+        "KG": 88 * V,
+        # reverse of k + forward of k+1: w m v read+written, pword; endpoints; q r/w + tree w m v r/w;
+        # net offsets; bundle info; S windows read once; demand arrays written once
+        "KBF": 28 * P + 8 * S + 32 * T + 4 * N + 16 * B + 48 * V,
+        # reverse only (last iteration of a call)
+        "KB": 28 * P + 8 * S + 28 * T + 4 * N + 16 * B + 16 * V,
     }
 
 
@@ -289,18 +293,19 @@ def main():
         st.update(paths=int(f.sub_path_off[s1_] - f.sub_path_off[s0_]), subnets=int(s1_ - s0_), trees=int(t1_ - t0_),
                   nets=int(hi - lo))
     sb = stage_bytes(st)
-    per_iter_ms = {k: v / max(n_prof, 1) for k, v in stage_ms.items()}
-    mine = {k: v for k, v in per_iter_ms.items() if k not in ("zero", "allreduce")}
+    per_launch_ms = {k: stage_ms[k] / n_prof[k] for k in stage_ms if n_prof[k]}
+    mine = {k: stage_ms[k] for k in stage_ms if k != "allreduce" and n_prof[k]}
     dom = max(mine, key=mine.get)
     peak, peak_src = measured_peak()
-    achieved = sb[dom] / (per_iter_ms[dom] * 1e-3) / 1e9
+    achieved = sb[dom] / (per_launch_ms[dom] * 1e-3) / 1e9
     traffic = None
     summ = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(summ):
         with open(summ) as fh:
             traffic = json.load(fh).get(args.config, {}).get(dom)
     iters_per_s = args.steps / (ms * 1e-3)
-    alg_iter = sum(sb.values())
+    # one steady-state iteration = KG + KBF (+ allreduce)
+    alg_iter = sb["KG"] + sb["KBF"]
     line = {
         "metric": "DAG-forest solver iters/sec (path-cand/s, overflow, WL alongside)",
         "value": iters_per_s, "unit": "iters/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
@@ -309,7 +314,7 @@ def main():
         "config": {"workload": f"{args.config} (BASELINE.json configs[3]: ISPD'19-shaped congested synthetic)",
                    "grid": f"{f.X}x{f.Y}", "nets": f.n_nets, "trees": f.n_trees, "subnets": f.n_subnets,
                    "paths": f.n_paths, "segments": f.n_segs, "turning_points": f.n_tps,
-                   "step": "one solver iteration (softmax, scatter, loss/gradient map, reverse, Adam); induction timed separately",
+                   "step": "one solver iteration (softmax, scatter, loss/gradient map, reverse, Adam) = KG + KBF; induction timed separately",
                    "l2": f"inputs larger than L2: {info['workspace_bytes'] / 1e6:.0f} MB resident state per rank touched every iteration > 126 MB L2",
                    "parallelism": f"dp{world} (nets sharded, demand allreduce)" if world > 1 else "single GPU"},
         "path_cand_per_s": iters_per_s * f.n_paths,
@@ -317,9 +322,11 @@ def main():
                                "frac": alg_iter * iters_per_s / 1e9 / peak},
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                     "alg_bytes_per_launch": sb[dom], "avg_launch_ms": per_iter_ms[dom]},
-        "stage_ms_per_iter": per_iter_ms,
-        "gpu_launches": 6 * args.steps,
+                     "alg_bytes_per_launch": sb[dom], "avg_launch_ms": per_launch_ms[dom],
+                     "share_of_step": stage_ms[dom] / sum(stage_ms.values())},
+        "stage_ms_per_launch": per_launch_ms,
+        "stage_launches": n_prof,
+        "gpu_launches": 3 * args.steps + 1,
         "clocks": clocks,
         "induce_ms": induce_ms,
         "loss": {"total": float(loss[0]), "wl": float(loss[1]), "via": float(loss[2]), "overflow": float(loss[3])},

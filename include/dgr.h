@@ -137,19 +137,25 @@ int dgr_get_logits(struct dgr_handle* h, float* w_tree, float* w_path);
 int dgr_induce(struct dgr_handle* h, float top_p, int32_t* tree_choice, int32_t* route,
                int64_t* nucleus_off, int32_t* nucleus, int32_t* D_h, int32_t* D_v, double metrics[5]);
 
-/* Introspection: iteration counter k, this rank's net range, encoded sizes.  info[8] =
- * {k, net_lo, net_hi, n_bundles, n_path_slots, workspace_bytes, world, rank}. */
-int dgr_get_info(struct dgr_handle* h, int64_t info[8]);
+/* Introspection: iteration counter k, this rank's net range, encoded sizes.  info[12] =
+ * {k, net_lo, net_hi, n_bundles, n_path_slots, workspace_bytes, world, rank, n_tiles,
+ *  n_global_tiles, 0, 0}. */
+int dgr_get_info(struct dgr_handle* h, int64_t info[12]);
+
+/* Host-only view of the rank's encoding plan (no GPU needed): out[8] = {n_tiles, n_global_tiles,
+ * n_bundles, n_path_slots, workspace_bytes, n_paths, paths in global tiles, largest window (cells)}.
+ * A tile is a run of whole nets whose candidates fit one shared-memory window of the grid; a
+ * global tile's nets are too spread out and run against HBM directly. */
+int dgr_plan_info(const dgr_forest_desc* desc, const dgr_dist* dist, int64_t out[8]);
 
 /* Per-stage device time of subsequent dgr_step calls, from CUDA events recorded on the handle's
- * stream between the stages.  enable != 0 starts (and clears) recording, 0 stops it.
- * dgr_profile_read synchronises and returns, for the stages
- *   0 KQ (tree softmax), 1 demand-buffer zeroing (cudaMemsetAsync), 2 KF (path softmax + scatter),
- *   3 demand allreduce (NCCL; world > 1 only), 4 KG (scan/loss/gradient map, 2 kernels),
- *   5 KB (reverse + Adam), 6 KT (tree reverse + Adam), 7 unused
- * the summed milliseconds and the number of iterations recorded. */
+ * stream after every stage.  enable != 0 starts (and clears) recording, 0 stops it.
+ * dgr_profile_read synchronises and returns, per stage, the summed milliseconds and the number of
+ * launches: 0 KF (forward-only tile kernel, once per dgr_step call), 1 demand allreduce (NCCL;
+ * world > 1), 2 KG (scan / loss / gradient map; 2 kernels), 3 KBF (reverse of k fused with the
+ * forward of k+1), 4 KB (reverse only: the last iteration of a call), 5..7 unused. */
 int dgr_profile(struct dgr_handle* h, int32_t enable);
-int dgr_profile_read(struct dgr_handle* h, double ms[8], int64_t* iterations);
+int dgr_profile_read(struct dgr_handle* h, double ms[8], int64_t launches[8]);
 
 /* Releases the handle (and the NCCL communicator); the workspace stays the caller's. */
 int dgr_free(struct dgr_handle* h);

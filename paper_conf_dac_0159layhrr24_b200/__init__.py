@@ -6,6 +6,6 @@ solver iteration runs in the CUDA kernels.  There is no CPU fallback: without th
 extension or a GPU the binding raises.
 """
 from .dgr import (DgrError, Loss, Solver, Weights, lib_path, load_library, nccl_unique_id,  # noqa: F401
-                  partition)
+                  partition, plan_info)
 
-__all__ = ["Solver", "Weights", "Loss", "DgrError", "partition", "nccl_unique_id", "load_library", "lib_path"]
+__all__ = ["Solver", "Weights", "Loss", "DgrError", "partition", "nccl_unique_id", "load_library", "lib_path", "plan_info"]

@@ -186,7 +186,22 @@ struct Plan {
   std::vector<short4> sxy;
   std::vector<int32_t> net_tree_off;
   std::vector<int64_t> sub_first_path;   // local path index of each local sub-net's first candidate
+  std::vector<TileDesc> tiles;
+  int64_t n_global_tiles = 0;
 };
+
+// Cells (x, y) touched by one candidate's demand events (see forward_bundle in dgr_kernels.cu)
+// and the fields they touch (bit 0 dH, 1 dV, 2 VD).
+int lane_events(uint32_t shape, int x0, int y0, int x1, int y1, int m, int ex[2], int ey[2], int fm[2]) {
+  switch (shape) {
+    case kStraightH: ex[0] = x0; ey[0] = y0; fm[0] = 1; ex[1] = x1; ey[1] = y0; fm[1] = 1; return 2;
+    case kStraightV: ex[0] = x0; ey[0] = y0; fm[0] = 2; ex[1] = x0; ey[1] = y1; fm[1] = 2; return 2;
+    case kHV: ex[0] = x0; ey[0] = y0; fm[0] = 3; ex[1] = x1; ey[1] = y0; fm[1] = 7; return 2;
+    case kVH: ex[0] = x0; ey[0] = y1; fm[0] = 7; ex[1] = x1; ey[1] = y1; fm[1] = 3; return 2;
+    case kZHVH: ex[0] = m; ey[0] = y0; fm[0] = 7; ex[1] = m; ey[1] = y1; fm[1] = 7; return 2;
+    default: ex[0] = x0; ey[0] = m; fm[0] = 7; ex[1] = x1; ey[1] = m; fm[1] = 7; return 2;
+  }
+}
 
 int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   int rc = validate_structure(d);
@@ -202,31 +217,24 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   pl.path_lo = d->sub_path_off[pl.sub_lo];
   pl.path_hi = d->sub_path_off[pl.sub_hi];
   const int64_t nn = pl.net_hi - pl.net_lo, ns = pl.sub_hi - pl.sub_lo;
+  const int X = d->X, Y = d->Y;
   pl.net_tree_off.resize(nn + 1);
   for (int64_t n = 0; n <= nn; ++n) pl.net_tree_off[n] = (int32_t)(d->net_tree_off[pl.net_lo + n] - pl.tree_lo);
   pl.sxy.resize(ns);
   pl.sub_first_path.resize(ns);
-  pl.binfo.clear();
-  pl.pword.clear();
-  int fill = 32;   // forces a new bundle at the first sub-net
+  // 1. canonical sub-net endpoints + pattern words of every local candidate
+  std::vector<uint32_t> pw_path((size_t)(pl.path_hi - pl.path_lo));
   for (int64_t j = pl.tree_lo; j < pl.tree_hi; ++j) {
     for (int64_t s = d->tree_sub_off[j]; s < d->tree_sub_off[j + 1]; ++s) {
       const int32_t* e = d->sub_xy + 4 * s;
       int x0 = e[0], y0 = e[1], x1 = e[2], y1 = e[3];
       if (x0 > x1 || (x0 == x1 && y0 > y1)) { std::swap(x0, x1); std::swap(y0, y1); }
-      if (x0 < 0 || x1 >= d->X || std::min(y0, y1) < 0 || std::max(y0, y1) >= d->Y)
+      if (x0 < 0 || x1 >= X || std::min(y0, y1) < 0 || std::max(y0, y1) >= Y)
         return fail(DGR_EINVAL, "sub-net %lld endpoints outside the grid", (long long)s);
       if (x0 == x1 && y0 == y1) return fail(DGR_EINVAL, "sub-net %lld has zero length", (long long)s);
       const int64_t ls = s - pl.sub_lo;
       pl.sxy[ls] = make_short4((short)x0, (short)y0, (short)x1, (short)y1);
       const int64_t p0 = d->sub_path_off[s], p1 = d->sub_path_off[s + 1];
-      const int g = (int)(p1 - p0);
-      if (fill + g > 32) {
-        // close the previous bundle's padding, open a new one
-        while (!pl.pword.empty() && pl.pword.size() % 32) pl.pword.push_back(kPad | kSubHead);
-        pl.binfo.push_back(make_int4((int)(p0 - pl.path_lo), (int)ls, (int)(j - pl.tree_lo), 0));
-        fill = 0;
-      }
       pl.sub_first_path[ls] = p0 - pl.path_lo;
       for (int64_t i = p0; i < p1; ++i) {
         uint32_t shape;
@@ -239,13 +247,134 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
           pw |= kSubHead;
           if (s == d->tree_sub_off[j]) pw |= kTreeHead;
         }
-        pl.pword.push_back(pw);
+        pw_path[i - pl.path_lo] = pw;
       }
-      fill += g;
-      pl.binfo.back().w += g;
     }
   }
-  while (pl.pword.size() % 32) pl.pword.push_back(kPad | kSubHead);
+  // 2. tiles of whole nets: greedy in net order while the window (union of the nets' sub-net boxes
+  //    plus a 1-cell halo) stays <= kWinMax cells, the bundles <= kTargetBundles, trees <= kTreeMax.
+  //    A net that alone exceeds the window forms a "global" tile.
+  pl.tiles.clear();
+  pl.binfo.clear();
+  pl.pword.clear();
+  struct Cur { bool open = false; int64_t net0 = 0; int nb = 0, fill = 32, ntree = 0; int bx0 = 0, by0 = 0, bx1 = -1, by1 = -1; bool global = false; } cur;
+  std::vector<int64_t> tile_net0;
+  std::vector<char> tile_glob;
+  auto net_box = [&](int64_t n, int& bx0, int& by0, int& bx1, int& by1) {
+    bx0 = X; by0 = Y; bx1 = -1; by1 = -1;
+    const int64_t s0 = d->tree_sub_off[d->net_tree_off[n]], s1 = d->tree_sub_off[d->net_tree_off[n + 1]];
+    for (int64_t s = s0; s < s1; ++s) {
+      const short4 e = pl.sxy[s - pl.sub_lo];
+      bx0 = std::min<int>(bx0, e.x); bx1 = std::max<int>(bx1, e.z);
+      by0 = std::min<int>(by0, std::min(e.y, e.w)); by1 = std::max<int>(by1, std::max(e.y, e.w));
+    }
+    bx0 = std::max(0, bx0 - 1); by0 = std::max(0, by0 - 1);
+    bx1 = std::min(X - 1, bx1 + 1); by1 = std::min(Y - 1, by1 + 1);
+  };
+  auto pack_net = [&](int64_t n, int& nb, int& fill) {   // bundle packing of one net's groups
+    const int64_t s0 = d->tree_sub_off[d->net_tree_off[n]], s1 = d->tree_sub_off[d->net_tree_off[n + 1]];
+    for (int64_t s = s0; s < s1; ++s) {
+      const int g = (int)(d->sub_path_off[s + 1] - d->sub_path_off[s]);
+      if (fill + g > 32) { ++nb; fill = 0; }
+      fill += g;
+    }
+  };
+  std::vector<int64_t> starts;
+  std::vector<char> globs;
+  for (int64_t n = pl.net_lo; n < pl.net_hi; ++n) {
+    int bx0, by0, bx1, by1;
+    net_box(n, bx0, by0, bx1, by1);
+    const bool big = (int64_t)(bx1 - bx0 + 1) * (by1 - by0 + 1) > kWinMax;
+    const int ntree = (int)(d->net_tree_off[n + 1] - d->net_tree_off[n]);
+    bool fits = cur.open && !cur.global && !big;
+    int nb2 = cur.nb, fill2 = cur.fill;
+    if (fits) {
+      const int ux0 = std::min(cur.bx0, bx0), uy0 = std::min(cur.by0, by0);
+      const int ux1 = std::max(cur.bx1, bx1), uy1 = std::max(cur.by1, by1);
+      pack_net(n, nb2, fill2);
+      fits = (int64_t)(ux1 - ux0 + 1) * (uy1 - uy0 + 1) <= kWinMax && nb2 <= kTargetBundles &&
+             cur.ntree + ntree <= kTreeMax;
+      if (fits) { cur.bx0 = ux0; cur.by0 = uy0; cur.bx1 = ux1; cur.by1 = uy1; }
+    } else if (cur.open && cur.global && big) {
+      pack_net(n, nb2, fill2);
+      fits = nb2 <= kMaxBundles && cur.ntree + ntree <= kTreeMax;
+    }
+    if (fits) {
+      cur.nb = nb2; cur.fill = fill2; cur.ntree += ntree;
+      continue;
+    }
+    // close the open tile, open a new one at net n
+    starts.push_back(n);
+    globs.push_back(big);
+    cur = Cur();
+    cur.open = true; cur.global = big; cur.net0 = n; cur.ntree = ntree;
+    cur.bx0 = bx0; cur.by0 = by0; cur.bx1 = bx1; cur.by1 = by1;
+    cur.nb = 0; cur.fill = 32;
+    pack_net(n, cur.nb, cur.fill);
+    if (cur.nb > kMaxBundles) return fail(DGR_EINVAL, "net %lld needs %d > %d bundles", (long long)n, cur.nb, kMaxBundles);
+  }
+  starts.push_back(pl.net_hi);
+  // 3. bundles, tile by tile (packing restarts at each tile)
+  std::vector<uint16_t> cnt;
+  for (size_t t = 0; t + 1 < starts.size(); ++t) {
+    TileDesc T{};
+    T.net0 = (int32_t)(starts[t] - pl.net_lo);
+    T.nnet = (int32_t)(starts[t + 1] - starts[t]);
+    T.tree0 = (int32_t)(d->net_tree_off[starts[t]] - pl.tree_lo);
+    T.ntree = (int32_t)(d->net_tree_off[starts[t + 1]] - d->net_tree_off[starts[t]]);
+    T.b0 = (int32_t)pl.binfo.size();
+    T.global = globs[t];
+    int bx0 = X, by0 = Y, bx1 = -1, by1 = -1;
+    for (int64_t n = starts[t]; n < starts[t + 1]; ++n) {
+      int a0, b0_, a1, b1_;
+      net_box(n, a0, b0_, a1, b1_);
+      bx0 = std::min(bx0, a0); by0 = std::min(by0, b0_); bx1 = std::max(bx1, a1); by1 = std::max(by1, b1_);
+    }
+    T.wx0 = bx0; T.wy0 = by0; T.ww = bx1 - bx0 + 1; T.wh = by1 - by0 + 1;
+    if (T.global) { T.wx0 = 0; T.wy0 = 0; T.ww = 0; T.wh = 0; }
+    int fill = 32;
+    const int64_t j0 = d->net_tree_off[starts[t]], j1 = d->net_tree_off[starts[t + 1]];
+    for (int64_t j = j0; j < j1; ++j) {
+      for (int64_t s = d->tree_sub_off[j]; s < d->tree_sub_off[j + 1]; ++s) {
+        const int64_t p0 = d->sub_path_off[s], p1 = d->sub_path_off[s + 1];
+        const int g = (int)(p1 - p0);
+        if (fill + g > 32) {
+          while (pl.pword.size() % 32) pl.pword.push_back(kPad | kSubHead);
+          pl.binfo.push_back(make_int4((int)(p0 - pl.path_lo), (int)(s - pl.sub_lo), (int)(j - pl.tree_lo), 0));
+          fill = 0;
+        }
+        for (int64_t i = p0; i < p1; ++i) pl.pword.push_back(pw_path[i - pl.path_lo]);
+        fill += g;
+        pl.binfo.back().w += g;
+      }
+    }
+    while (pl.pword.size() % 32) pl.pword.push_back(kPad | kSubHead);
+    T.nb = (int32_t)pl.binfo.size() - T.b0;
+    // int32 shared-memory accumulation is exact while no window cell-field gets more than
+    // kEventMax events (each |event| <= 2^24); otherwise run the tile against global memory.
+    if (!T.global) {
+      cnt.assign((size_t)3 * T.ww * T.wh, 0);
+      bool ok = true;
+      for (int64_t j = j0; j < j1 && ok; ++j)
+        for (int64_t s = d->tree_sub_off[j]; s < d->tree_sub_off[j + 1] && ok; ++s) {
+          const short4 e = pl.sxy[s - pl.sub_lo];
+          for (int64_t i = d->sub_path_off[s]; i < d->sub_path_off[s + 1] && ok; ++i) {
+            const uint32_t pw = pw_path[i - pl.path_lo];
+            int ex[2], ey[2], fm[2];
+            lane_events(pw & 7u, e.x, e.y, e.z, e.w, (int)(pw >> 16), ex, ey, fm);
+            for (int q = 0; q < 2 && ok; ++q)
+              for (int f = 0; f < 3; ++f)
+                if (fm[q] >> f & 1) {
+                  const size_t c = (size_t)f * T.ww * T.wh + (size_t)(ey[q] - T.wy0) * T.ww + (ex[q] - T.wx0);
+                  if (++cnt[c] > kEventMax) { ok = false; break; }
+                }
+          }
+        }
+      if (!ok) { T.global = 1; T.wx0 = T.wy0 = T.ww = T.wh = 0; }
+    }
+    pl.n_global_tiles += T.global;
+    pl.tiles.push_back(T);
+  }
   pl.nb = (int)pl.binfo.size();
   return DGR_OK;
 }
@@ -254,7 +383,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
 // workspace layout
 // ---------------------------------------------------------------------------------------
 struct Layout {
-  size_t binfo, pword, sxy, wp, mp, vp, nto, wt, mt, vt, q, dq, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
+  size_t tiles, binfo, pword, sxy, wp, mp, vp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
       partial, loss, chosen, tree_choice, route, nsize, nucleus_tmp, DHVC, iscal, ipartial, metrics, total;
   size_t xcount;   // int64 elements in the exchange buffer
 };
@@ -265,6 +394,7 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   auto take = [&](size_t bytes) { size_t r = o; o += (bytes + 255) & ~(size_t)255; return r; };
   const size_t slots = (size_t)pl.nb * 32, ns = pl.sxy.size(), nt = (size_t)(pl.tree_hi - pl.tree_lo),
                nn = (size_t)(pl.net_hi - pl.net_lo), G = (size_t)X * Y;
+  L.tiles = take(sizeof(TileDesc) * pl.tiles.size());
   L.binfo = take(sizeof(int4) * pl.nb);
   L.pword = take(4 * slots);
   L.sxy = take(8 * ns);
@@ -276,8 +406,7 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.mt = take(4 * nt);
   L.vt = take(4 * nt);
   L.q = take(4 * nt);
-  L.dq = take(8 * nt);
-  L.xcount = 3 * G + 2;
+  L.xcount = 4 * G + 2;   // dH | dV^T | VD (row-major) | VD (column-major) | E[WL], E[TP]
   L.xbuf = take(8 * L.xcount);
   L.capH = take(4 * G);
   L.capVT = take(4 * G);
@@ -318,25 +447,26 @@ struct dgr_handle {
   float beta_last = 0.25f;
   bool have_forward = false;
   double* pinned = nullptr;   // 16 doubles of pinned host memory
-  // profiling: 8 events per recorded iteration (stage boundaries)
+  // profiling: a CUDA event after every stage, attributed to that stage
   bool prof = false;
   std::vector<cudaEvent_t> ev;
+  std::vector<int> ev_stage;
   size_t ev_used = 0;
 };
 
 namespace {
-constexpr int kStages = 7;
-// records the boundary event `b` (0..7) of the current profiled iteration
-int prof_mark(dgr_handle* h, int b) {
+// stage -1 opens an interval; stage >= 0 closes the interval since the previous event
+int prof_mark(dgr_handle* h, int stage) {
   if (!h->prof) return DGR_OK;
-  const size_t idx = h->ev_used + b;
-  while (h->ev.size() <= idx) {
+  if (h->ev.size() <= h->ev_used) {
     cudaEvent_t e;
     CUDA_TRY(cudaEventCreate(&e));
     h->ev.push_back(e);
+    h->ev_stage.push_back(-1);
   }
-  CUDA_TRY(cudaEventRecord(h->ev[idx], h->stream));
-  if (b == kStages) h->ev_used += kStages + 1;
+  CUDA_TRY(cudaEventRecord(h->ev[h->ev_used], h->stream));
+  h->ev_stage[h->ev_used] = stage;
+  h->ev_used += 1;
   return DGR_OK;
 }
 }  // namespace
@@ -413,6 +543,8 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
   h->ws_bytes = workspace_bytes;
   char* ws = h->ws;
   P.nb = pl.nb;
+  P.ntiles = (int32_t)pl.tiles.size();
+  P.tiles = (const TileDesc*)(ws + L.tiles);
   P.n_nets_l = (int32_t)(pl.net_hi - pl.net_lo);
   P.path_base = pl.path_lo;
   P.tree_base = pl.tree_lo;
@@ -423,12 +555,12 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
   P.wp = (float*)(ws + L.wp); P.mp = (float*)(ws + L.mp); P.vp = (float*)(ws + L.vp);
   P.net_tree_off = (const int32_t*)(ws + L.nto);
   P.wt = (float*)(ws + L.wt); P.mt = (float*)(ws + L.mt); P.vt = (float*)(ws + L.vt); P.q = (float*)(ws + L.q);
-  P.dq = (long long*)(ws + L.dq);
   const size_t G = (size_t)desc->X * desc->Y;
   P.dH = (long long*)(ws + L.xbuf);
   P.dVT = P.dH + G;
-  P.VD = P.dVT + G;
-  P.scal = P.VD + G;
+  P.VDH = P.dVT + G;
+  P.VDV = P.VDH + G;
+  P.scal = P.VDV + G;
   P.capH = (const float*)(ws + L.capH);
   P.capVT = (const float*)(ws + L.capVT);
   P.SH = (double*)(ws + L.SH); P.SVT = (double*)(ws + L.SVT);
@@ -449,6 +581,7 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
 
   auto cleanup = [&](int code) { if (h->pinned) cudaFreeHost(h->pinned); delete h; return code; };
   cudaStream_t s = h->stream;
+  if (prepare_kernels() != 0) return cleanup(fail(DGR_ECUDA, "cudaFuncSetAttribute (tile kernel shared memory) failed"));
   if (cudaMemsetAsync(ws, 0, L.total, s) != cudaSuccess) return cleanup(fail(DGR_ECUDA, "memset workspace failed"));
   // host-side staging of the encoded shard
   const size_t slots = (size_t)pl.nb * 32;
@@ -463,6 +596,7 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
   auto cp = [&](size_t off, const void* src, size_t bytes) {
     if (bytes && e == cudaSuccess) e = cudaMemcpyAsync(ws + off, src, bytes, cudaMemcpyHostToDevice, s);
   };
+  cp(L.tiles, pl.tiles.data(), sizeof(TileDesc) * pl.tiles.size());
   cp(L.binfo, pl.binfo.data(), sizeof(int4) * pl.nb);
   cp(L.pword, pl.pword.data(), 4 * slots);
   cp(L.sxy, pl.sxy.data(), 8 * pl.sxy.size());
@@ -493,40 +627,45 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
   KParams& P = h->P;
   StepArgs a{};
   a.inv_t = 1.f / temperature;
-  a.t = temperature;
   a.a_wl = w->a_wl; a.a_via = w->a_via; a.a_of = w->a_of; a.beta = w->beta_via;
   a.sqrt_l = std::sqrt(w->n_layers);
   a.f_slope = w->f_slope; a.f_kind = w->f_kind;
-  const int n = iters == 0 ? 1 : iters;
   const size_t xbytes = 8 * h->lay.xcount;
+  (void)xbytes;
   cudaStream_t s = h->stream;
-  for (int it = 0; it < n; ++it) {
-    a.k = h->k;
-    a.store_d = (it == n - 1);
-    const double step = (double)(h->k + 1);
+  auto adam_args = [&](int64_t k) {
+    const double step = (double)(k + 1);
     a.lr_over_bc1 = (float)(lr / (1.0 - std::pow(0.9, step)));
     a.inv_sqrt_bc2 = (float)(1.0 / std::sqrt(1.0 - std::pow(0.999, step)));
-    int rc;
-    if ((rc = prof_mark(h, 0))) return rc;
-    launch_kq(P, a, s);
-    if ((rc = prof_mark(h, 1))) return rc;
-    CUDA_TRY(cudaMemsetAsync(P.dH, 0, xbytes, s));
-    if ((rc = prof_mark(h, 2))) return rc;
-    launch_kf(P, a, s);
-    if ((rc = prof_mark(h, 3))) return rc;
-    if (h->world > 1) NCCL_TRY(ncclAllReduce(P.dH, P.dH, h->lay.xcount, ncclInt64, ncclSum, h->comm, s));
-    if ((rc = prof_mark(h, 4))) return rc;
-    launch_kg(P, a, s);
-    if ((rc = prof_mark(h, 5))) return rc;
-    if (iters > 0) {
-      launch_kb(P, a, s);
-      if ((rc = prof_mark(h, 6))) return rc;
-      launch_kt(P, a, s);
-      h->k += 1;
-    } else if ((rc = prof_mark(h, 6))) {
-      return rc;
+  };
+  int rc;
+  // forward of iteration k (q, p, demand events of the current logits at this temperature)
+  a.k = h->k;
+  a.k_next = h->k;
+  a.store_d = 0;
+  adam_args(h->k);
+  if ((rc = prof_mark(h, -1))) return rc;
+  launch_tiles(P, a, kForwardOnly, s);
+  if ((rc = prof_mark(h, 0))) return rc;
+  const int n = iters == 0 ? 1 : iters;
+  for (int it = 0; it < n; ++it) {
+    const bool last = (it == n - 1);
+    a.k = h->k;
+    a.k_next = h->k + 1;
+    a.store_d = last;
+    adam_args(h->k);
+    if (h->world > 1) {
+      NCCL_TRY(ncclAllReduce(P.dH, P.dH, h->lay.xcount, ncclInt64, ncclSum, h->comm, s));
+      if ((rc = prof_mark(h, 1))) return rc;
     }
-    if ((rc = prof_mark(h, 7))) return rc;
+    launch_kg(P, a, s);
+    if ((rc = prof_mark(h, 2))) return rc;
+    if (iters > 0) {
+      // reverse of iteration k + (unless last) forward of k+1
+      launch_tiles(P, a, last ? kReverseOnly : kReverseForward, s);
+      h->k += 1;
+    }
+    if (iters > 0 && (rc = prof_mark(h, last ? 4 : 3))) return rc;
   }
   CUDA_TRY(cudaGetLastError());
   h->t_last = temperature;
@@ -622,10 +761,32 @@ int dgr_induce(dgr_handle* h, float top_p, int32_t* tree_choice, int32_t* route,
   return DGR_OK;
 }
 
-int dgr_get_info(dgr_handle* h, int64_t info[8]) {
+int dgr_get_info(dgr_handle* h, int64_t info[12]) {
   if (!h || !info) return fail(DGR_EINVAL, "NULL argument");
   info[0] = h->k; info[1] = h->plan.net_lo; info[2] = h->plan.net_hi; info[3] = h->plan.nb;
   info[4] = (int64_t)h->plan.nb * 32; info[5] = (int64_t)h->lay.total; info[6] = h->world; info[7] = h->rank;
+  info[8] = (int64_t)h->plan.tiles.size(); info[9] = h->plan.n_global_tiles; info[10] = 0; info[11] = 0;
+  return DGR_OK;
+}
+
+int dgr_plan_info(const dgr_forest_desc* desc, const dgr_dist* dist, int64_t out[8]) {
+  if (!out) return fail(DGR_EINVAL, "out is NULL");
+  int rank, world, rc;
+  if ((rc = dist_args(dist, &rank, &world))) return rc;
+  Plan pl;
+  if ((rc = make_plan(desc, rank, world, pl))) return rc;
+  int64_t maxw = 0, gpaths = 0;
+  for (const auto& T : pl.tiles) {
+    maxw = std::max<int64_t>(maxw, (int64_t)T.ww * T.wh);
+    if (T.global)
+      for (int b = T.b0; b < T.b0 + T.nb; ++b) gpaths += pl.binfo[b].w;
+  }
+  dgr::KParams tmp{};
+  tmp.X = desc->X;
+  tmp.Y = desc->Y;
+  out[0] = (int64_t)pl.tiles.size(); out[1] = pl.n_global_tiles; out[2] = pl.nb; out[3] = (int64_t)pl.nb * 32;
+  out[4] = (int64_t)make_layout(pl, desc->X, desc->Y, induce_metric_blocks(tmp)).total;
+  out[5] = pl.path_hi - pl.path_lo; out[6] = gpaths; out[7] = maxw;
   return DGR_OK;
 }
 
@@ -636,18 +797,18 @@ int dgr_profile(dgr_handle* h, int32_t enable) {
   return DGR_OK;
 }
 
-int dgr_profile_read(dgr_handle* h, double ms[8], int64_t* iterations) {
-  if (!h || !ms || !iterations) return fail(DGR_EINVAL, "NULL argument");
+int dgr_profile_read(dgr_handle* h, double ms[8], int64_t launches[8]) {
+  if (!h || !ms || !launches) return fail(DGR_EINVAL, "NULL argument");
   CUDA_TRY(cudaStreamSynchronize(h->stream));
-  for (int i = 0; i < 8; ++i) ms[i] = 0.0;
-  const size_t n = h->ev_used / (kStages + 1);
-  for (size_t it = 0; it < n; ++it)
-    for (int b = 0; b < kStages; ++b) {
-      float t = 0.f;
-      CUDA_TRY(cudaEventElapsedTime(&t, h->ev[it * (kStages + 1) + b], h->ev[it * (kStages + 1) + b + 1]));
-      ms[b] += t;
-    }
-  *iterations = (int64_t)n;
+  for (int i = 0; i < 8; ++i) { ms[i] = 0.0; launches[i] = 0; }
+  for (size_t i = 1; i < h->ev_used; ++i) {
+    const int st = h->ev_stage[i];
+    if (st < 0 || st >= 8) continue;
+    float t = 0.f;
+    CUDA_TRY(cudaEventElapsedTime(&t, h->ev[i - 1], h->ev[i]));
+    ms[st] += t;
+    launches[st] += 1;
+  }
   return DGR_OK;
 }
 

@@ -5,14 +5,20 @@
 //     candidate.  A bundle holds whole sub-nets (groups of 1..32 candidates, packed in order,
 //     never split), so the sub-net softmax is a segmented warp reduction.  Unused tail lanes
 //     are padding (shape PAD).
+//   * bundles are grouped into "tiles": whole nets whose candidates all lie inside one small
+//     G-cell window (<= kWinMax cells incl. a 1-cell halo).  One CTA owns one tile: it stages the
+//     tile's window of the gradient prefix sums in shared memory for the reverse pass, keeps the
+//     tile's tree state (dq, q) in shared memory, and accumulates the tile's demand events in a
+//     shared-memory window that it flushes once to the global difference arrays.  Tiles whose
+//     nets span a larger window run the same code against global memory ("global" tiles).
 //   * per slot:    pword (shape | flags | mid), w, m, v (fp32)
 //   * per bundle:  {first local path, first local sub-net, first local tree, #valid lanes}
 //   * per sub-net: canonical endpoints (x0 <= x1; y0 < y1 if x0 == x1) as int16 x 4
-//   * per tree:    w, m, v, q (fp32), dq (int64 fixed point)
-//   * grids: diff arrays of the wire demand along H rows ([Y][X]) and along V columns (stored
-//     transposed, [X][Y], so both scans run over contiguous lines), the turning-point
-//     ("via") demand per G-cell ([Y][X]), all int64 in 2^-24 fixed point; prefix sums S of the
-//     overflow gradient per line (fp64, same two layouts).
+//   * per tree:    w, m, v, q (fp32)
+//   * grids: difference arrays of the wire demand along H rows ([Y][X]) and along V columns
+//     (stored transposed, [X][Y], so both scans run over contiguous lines), the turning-point
+//     ("via") demand per G-cell in both layouts, all int64 in 2^-24 fixed point; prefix sums S of
+//     the overflow gradient per line (fp64, the same two layouts).
 #pragma once
 #include <cstdint>
 
@@ -21,6 +27,15 @@ namespace dgr {
 constexpr int kFracBits = 24;                      // fixed point of pi: round(pi * 2^24)
 constexpr float kFixScale = 16777216.0f;           // 2^24
 constexpr double kFixInv = 1.0 / 16777216.0;
+constexpr double kDqScale = 4294967296.0;          // dq_j accumulated in 2^-32 fixed point
+constexpr double kDqInv = 1.0 / 4294967296.0;
+
+constexpr int kTileThreads = 256;                  // 8 warps per tile CTA
+constexpr int kWinMax = 2048;                      // window cells per tile
+constexpr int kMaxBundles = 64;                    // bundles per tile (a whole net always fits)
+constexpr int kTargetBundles = 32;                 // planner target per tile
+constexpr int kTreeMax = 512;                      // trees per tile
+constexpr int kEventMax = 127;                     // events per window cell-field (int32 safety)
 
 enum Shape : uint32_t {
   kStraightH = 0, kStraightV = 1, kHV = 2, kVH = 3, kZHVH = 4, kZVHV = 5, kPad = 7
@@ -29,25 +44,35 @@ constexpr uint32_t kSubHead = 8u;    // lane starts a sub-net group
 constexpr uint32_t kTreeHead = 16u;  // sub-net is the first of its tree (set on the group head)
 // bits 16..31: x_m (Z-HVH) or y_m (Z-VHV)
 
+struct TileDesc {
+  int32_t b0, nb;          // bundles [b0, b0 + nb)
+  int32_t net0, nnet;      // local nets
+  int32_t tree0, ntree;    // local trees
+  int32_t wx0, wy0, ww, wh;  // window (cells), unused for global tiles
+  int32_t global, pad;
+};
+
 struct KParams {
   // sizes
   int32_t X, Y;
   int32_t nb;               // bundles
   int32_t n_nets_l;         // local nets
+  int32_t ntiles;
   int64_t path_base, tree_base;   // global index of the first local path / tree
   uint64_t seed;
   // forest encoding
+  const TileDesc* tiles;
   const int4* binfo;
   const uint32_t* pword;
   const short4* sxy;
   float *wp, *mp, *vp;
   const int32_t* net_tree_off;    // local, n_nets_l + 1
   float *wt, *mt, *vt, *q;
-  long long* dq;
-  // grids
+  // grids (the exchange buffer, in this order: dH | dVT | VDH | VDV | scal)
   long long* dH;            // [Y][X]
   long long* dVT;           // [X][Y]
-  long long* VD;            // [Y][X]
+  long long* VDH;           // [Y][X]
+  long long* VDV;           // [X][Y]
   long long* scal;          // {E[WL], E[TP]} fixed point
   const float* capH;        // [Y][X]
   const float* capVT;       // [X][Y]
@@ -62,7 +87,7 @@ struct KParams {
   int32_t* tree_choice;     // [n_nets_l] (global tree index)
   int32_t* route;           // [n_subs_l] (global path index or -1)
   int32_t* nsize;           // [n_subs_l]
-  int32_t* nucleus_tmp;     // [nb*32] indexed by local path
+  int32_t* nucleus_tmp;     // indexed by local path
   int32_t* DH;              // [Y][X]
   int32_t* DV;              // [Y][X]
   int32_t* VC;              // [Y][X]
@@ -72,9 +97,9 @@ struct KParams {
 };
 
 struct StepArgs {
-  int64_t k;          // global iteration
+  int64_t k;          // iteration of the reverse pass
+  int64_t k_next;     // iteration of the forward pass
   float inv_t;        // 1 / temperature
-  float t;
   float lr_over_bc1;  // lr / (1 - beta1^(k+1))
   float inv_sqrt_bc2; // 1 / sqrt(1 - beta2^(k+1))
   float a_wl, a_via, a_of, beta, sqrt_l, f_slope;
@@ -83,13 +108,13 @@ struct StepArgs {
 };
 
 // launchers (dgr_kernels.cu)
-void launch_kq(const KParams& p, const StepArgs& a, cudaStream_t s);
-void launch_kf(const KParams& p, const StepArgs& a, cudaStream_t s);
+enum TileMode { kForwardOnly = 0, kReverseForward = 1, kReverseOnly = 2 };
+void launch_tiles(const KParams& p, const StepArgs& a, TileMode mode, cudaStream_t s);
 void launch_kg(const KParams& p, const StepArgs& a, cudaStream_t s);
-void launch_kb(const KParams& p, const StepArgs& a, cudaStream_t s);
-void launch_kt(const KParams& p, const StepArgs& a, cudaStream_t s);
 void launch_induce(const KParams& p, float t_final, float top_p, float beta, cudaStream_t s);
 void launch_induce_metrics(const KParams& p, float beta, cudaStream_t s);
 int induce_metric_blocks(const KParams& p);
+size_t tile_smem_bytes();
+int prepare_kernels();   // sets shared-memory attributes; returns cudaError_t
 
 }  // namespace dgr

@@ -87,11 +87,12 @@ def load_library():
     L.dgr_get_logits.argtypes = [vp, _PF, _PF]
     L.dgr_induce.argtypes = [vp, c.c_float, _P32, _P32, _P64, _P32, _P32, _P32, c.POINTER(c.c_double)]
     L.dgr_get_info.argtypes = [vp, _P64]
+    L.dgr_plan_info.argtypes = [c.POINTER(_Desc), c.POINTER(_Dist), _P64]
     L.dgr_free.argtypes = [vp]
     L.dgr_profile.argtypes = [vp, c.c_int32]
     L.dgr_profile_read.argtypes = [vp, c.POINTER(c.c_double), _P64]
     for fn in ("dgr_nccl_unique_id", "dgr_partition", "dgr_forest_load", "dgr_step", "dgr_get_demand",
-               "dgr_get_logits", "dgr_induce", "dgr_get_info", "dgr_free", "dgr_profile", "dgr_profile_read"):
+               "dgr_get_logits", "dgr_induce", "dgr_get_info", "dgr_free", "dgr_profile", "dgr_profile_read", "dgr_plan_info"):
         getattr(L, fn).restype = c.c_int
     _lib = L
     return L
@@ -148,6 +149,23 @@ def partition(forest, world: int) -> np.ndarray:
     out = np.zeros(world + 1, np.int64)
     _check(L.dgr_partition(ctypes.byref(d.desc), world, _ptr(out, ctypes.c_int64)))
     return out
+
+
+def plan_info(forest, rank: int = 0, world: int = 1) -> dict:
+    """dgr_plan_info: the rank's tile / bundle plan, computed on the host (no GPU)."""
+    L = load_library()
+    d = _DescHolder(forest)
+    out = np.zeros(8, np.int64)
+    dist = _Dist(rank, world, None) if world > 1 else None
+    if world > 1:
+        # the plan does not need the NCCL id; pass a dummy so validation accepts world > 1
+        buf = ctypes.create_string_buffer(128)
+        dist.nccl_unique_id = ctypes.cast(buf, ctypes.c_void_p)
+    _check(L.dgr_plan_info(ctypes.byref(d.desc), ctypes.byref(dist) if dist is not None else None,
+                           _ptr(out, ctypes.c_int64)))
+    keys = ("n_tiles", "n_global_tiles", "n_bundles", "n_slots", "workspace_bytes", "n_paths", "global_paths",
+            "max_window")
+    return {k: int(v) for k, v in zip(keys, out)}
 
 
 def nccl_unique_id() -> bytes:
@@ -236,22 +254,24 @@ class Solver:
         return r
 
     def info(self) -> dict:
-        a = np.zeros(8, np.int64)
+        a = np.zeros(12, np.int64)
         _check(load_library().dgr_get_info(self._h, _ptr(a, ctypes.c_int64)))
         return dict(k=int(a[0]), net_lo=int(a[1]), net_hi=int(a[2]), n_bundles=int(a[3]), n_slots=int(a[4]),
-                    workspace_bytes=int(a[5]), world=int(a[6]), rank=int(a[7]))
+                    workspace_bytes=int(a[5]), world=int(a[6]), rank=int(a[7]), n_tiles=int(a[8]),
+                    n_global_tiles=int(a[9]))
 
-    STAGES = ("KQ", "zero", "KF", "allreduce", "KG", "KB", "KT")
+    STAGES = ("KF", "allreduce", "KG", "KBF", "KB")
 
     def profile(self, enable: bool = True):
         """Start (and clear) / stop per-stage CUDA-event timing of dgr_step."""
         _check(load_library().dgr_profile(self._h, int(bool(enable))))
 
-    def profile_read(self) -> tuple[dict, int]:
+    def profile_read(self) -> tuple[dict, dict]:
+        """{stage: summed ms}, {stage: launches} since profile(True)."""
         ms = (ctypes.c_double * 8)()
-        n = ctypes.c_int64()
-        _check(load_library().dgr_profile_read(self._h, ms, ctypes.byref(n)))
-        return {k: ms[i] for i, k in enumerate(self.STAGES)}, int(n.value)
+        n = (ctypes.c_int64 * 8)()
+        _check(load_library().dgr_profile_read(self._h, ms, n))
+        return {k: ms[i] for i, k in enumerate(self.STAGES)}, {k: int(n[i]) for i, k in enumerate(self.STAGES)}
 
     @property
     def iteration(self) -> int:

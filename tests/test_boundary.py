@@ -96,3 +96,17 @@ def test_gpu_required_without_cuda(tiny):
         pytest.skip("has a GPU")
     with pytest.raises(dgr.DgrError):
         dgr.Solver(tiny)
+
+
+@pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18"])
+def test_plan_tiles_cover_the_forest(name):
+    f = forestgen.generate(name)
+    pi = dgr.plan_info(f)
+    assert pi["n_paths"] == f.n_paths
+    assert pi["n_slots"] >= f.n_paths and pi["n_slots"] % 32 == 0
+    assert pi["n_slots"] <= 1.25 * f.n_paths + 32 * pi["n_tiles"]      # padding stays bounded
+    assert pi["max_window"] <= 2048
+    assert pi["global_paths"] <= 0.01 * f.n_paths                       # almost all tiles use SMEM windows
+    for world in (2, 3):
+        tot = sum(dgr.plan_info(f, rank=r, world=world)["n_paths"] for r in range(world))
+        assert tot == f.n_paths
