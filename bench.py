@@ -76,12 +76,14 @@ def stage_bytes(st: dict) -> dict:
 
 
 class Clocks:
-    """nvidia-smi sampler for the timed region (B200_PROFILING.md clocks line)."""
+    """nvidia-smi sampler for the timed region (B200_PROFILING.md clocks line), logging to a file
+    (a pipe would be block-buffered and lose the samples at termination)."""
 
     def __init__(self, gpu_index: int):
+        import tempfile
         self.gpu = gpu_index
         self.proc = None
-        self.lines = []
+        self.path = tempfile.mktemp(prefix="dgr_clocks_", suffix=".csv")
 
     def __enter__(self):
         try:
@@ -89,20 +91,16 @@ class Clocks:
                 ["nvidia-smi", "-i", str(self.gpu), "--query-gpu=clocks.sm,clocks.max.sm,power.draw,"
                  "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
                  "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
-                 "--format=csv,noheader,nounits", "-lms", "100"],
-                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-            self.t = threading.Thread(target=self._read, daemon=True)
-            self.t.start()
+                 "--format=csv,noheader,nounits", "-lms", "100", "-f", self.path],
+                stdout=subprocess.DEVNULL, stderr=subprocess.DEVNULL)
+            time.sleep(0.3)
         except OSError:
             self.proc = None
         return self
 
-    def _read(self):
-        for line in self.proc.stdout:
-            self.lines.append(line.strip())
-
     def __exit__(self, *a):
         if self.proc:
+            time.sleep(0.2)
             self.proc.terminate()
             try:
                 self.proc.wait(timeout=5)
@@ -112,7 +110,12 @@ class Clocks:
     def summary(self):
         sm, mx, reasons = [], None, set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
+        try:
+            lines = open(self.path).read().splitlines()
+            os.unlink(self.path)
+        except OSError:
+            lines = []
+        for ln in lines:
             parts = [p.strip() for p in ln.split(",")]
             if len(parts) < 7:
                 continue

@@ -383,7 +383,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
 // workspace layout
 // ---------------------------------------------------------------------------------------
 struct Layout {
-  size_t tiles, binfo, pword, sxy, wp, mp, vp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
+  size_t tiles, binfo, pword, sxy, wp, mp, vp, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
       partial, loss, chosen, tree_choice, route, nsize, nucleus_tmp, DHVC, iscal, ipartial, metrics, total;
   size_t xcount;   // int64 elements in the exchange buffer
 };
@@ -401,6 +401,7 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.wp = take(4 * slots);
   L.mp = take(4 * slots);
   L.vp = take(4 * slots);
+  L.pp = take(4 * slots);   // p of the last forward (read by the next reverse)
   L.nto = take(4 * (nn + 1));
   L.wt = take(4 * nt);
   L.mt = take(4 * nt);
@@ -410,8 +411,8 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.xbuf = take(8 * L.xcount);
   L.capH = take(4 * G);
   L.capVT = take(4 * G);
-  L.SH = take(8 * G);
-  L.SVT = take(8 * G);
+  L.SH = take(16 * G);   // S_H then S_V^T, contiguous (one base pointer in the kernels)
+  L.SVT = L.SH + 8 * G;
   L.dOutH = take(4 * G);
   L.dOutVT = take(4 * G);
   L.partial = take(8 * (size_t)(X + Y));
@@ -553,6 +554,7 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
   P.pword = (const uint32_t*)(ws + L.pword);
   P.sxy = (const short4*)(ws + L.sxy);
   P.wp = (float*)(ws + L.wp); P.mp = (float*)(ws + L.mp); P.vp = (float*)(ws + L.vp);
+  P.pp = (float*)(ws + L.pp);
   P.net_tree_off = (const int32_t*)(ws + L.nto);
   P.wt = (float*)(ws + L.wt); P.mt = (float*)(ws + L.mt); P.vt = (float*)(ws + L.vt); P.q = (float*)(ws + L.q);
   const size_t G = (size_t)desc->X * desc->Y;

@@ -11,7 +11,7 @@
 //     tile's tree state (dq, q) in shared memory, and accumulates the tile's demand events in a
 //     shared-memory window that it flushes once to the global difference arrays.  Tiles whose
 //     nets span a larger window run the same code against global memory ("global" tiles).
-//   * per slot:    pword (shape | flags | mid), w, m, v (fp32)
+//   * per slot:    pword (shape | flags | mid), w, m, v (fp32), p of the last forward (fp32)
 //   * per bundle:  {first local path, first local sub-net, first local tree, #valid lanes}
 //   * per sub-net: canonical endpoints (x0 <= x1; y0 < y1 if x0 == x1) as int16 x 4
 //   * per tree:    w, m, v, q (fp32)
@@ -66,6 +66,7 @@ struct KParams {
   const uint32_t* pword;
   const short4* sxy;
   float *wp, *mp, *vp;
+  float* pp;                // p_i of the last forward (the reverse of that iteration reads it)
   const int32_t* net_tree_off;    // local, n_nets_l + 1
   float *wt, *mt, *vt, *q;
   // grids (the exchange buffer, in this order: dH | dVT | VDH | VDV | scal)

@@ -124,107 +124,197 @@ __device__ __forceinline__ void adam_update(float& w, float& m, float& v, float 
 
 // ------------------------------------------------------------------------------------------
 // Grid accessors: the same code runs against the tile's shared-memory window or, for global
-// tiles, against the whole grid in HBM.  H-type arrays are row-major in the window/grid,
-// V-type arrays column-major (x-major), matching the line layouts of KG.
+// tiles, against the whole grid in HBM.  One base pointer: S_H (row-major) at [0, hv) and
+// S_V (column-major) at [hv, 2 hv); the same for the H / V demand-event windows.
 // ------------------------------------------------------------------------------------------
 struct Win {
-  int ox, oy, hs, vs;   // origin; row stride of H arrays (= width), column stride of V arrays (= height)
+  int ox, oy, hs, vs, hv;   // origin; row stride of H (= width); column stride of V (= height); V offset
   __device__ __forceinline__ int h(int x, int y) const { return (y - oy) * hs + (x - ox); }
-  __device__ __forceinline__ int v(int x, int y) const { return (x - ox) * vs + (y - oy); }
+  __device__ __forceinline__ int v(int x, int y) const { return hv + (x - ox) * vs + (y - oy); }
+};
+
+struct Shape6 {
+  bool sh, sv, hv, vh, zh, zv;
+  __device__ __forceinline__ explicit Shape6(uint32_t s)
+      : sh(s == kStraightH), sv(s == kStraightV), hv(s == kHV), vh(s == kVH), zh(s == kZHVH), zv(s == kZVHV) {}
 };
 
 // c_i = a1 WL + a2 sqrt(L) TP + sum over the path's edges of G + beta sum over its turning points of
-// the G of the incident edges; a segment's sum is S[hi] - S[lo]; path geometry from the canonical
-// sub-net endpoints and the pattern word (straight, HV, VH, Z-HVH(x_m), Z-VHV(y_m)).
-__device__ __forceinline__ double path_cost(const double* SH, const double* SV, const Win& W, int X, int Y,
-                                            uint32_t shape, int x0, int y0, int x1, int y1, int m,
-                                            const StepArgs& A) {
+// the G of the incident edges; a segment's sum is S[hi] - S[lo].  Branch-free: the pattern selects
+// up to three segments and two turning points (straight, HV, VH, Z-HVH(x_m), Z-VHV(y_m)); unused
+// slots read valid cells and are weighted by 0.
+__device__ __forceinline__ double path_cost(const double* S, const Win& W, int X, int Y, uint32_t shape, int x0,
+                                            int y0, int x1, int y1, int m, const StepArgs& A) {
+  const Shape6 k(shape);
   const int ylo = min(y0, y1), yhi = max(y0, y1);
-  // up to three segments: (is_v, line, lo, hi); inactive when lo == hi
-  int v1 = 0, l1 = y0, a1 = x0, b1 = x1;
-  int v2 = 0, l2 = 0, a2 = 0, b2 = 0;
-  int v3 = 0, l3 = 0, a3 = 0, b3 = 0;
-  int ntp = 0, tx0 = 0, ty0 = 0, tx1 = 0, ty1 = 0;
-  switch (shape) {
-    case kStraightH: break;
-    case kStraightV: v1 = 1; l1 = x0; a1 = y0; b1 = y1; break;
-    case kHV: v2 = 1; l2 = x1; a2 = ylo; b2 = yhi; ntp = 1; tx0 = x1; ty0 = y0; break;
-    case kVH: v1 = 1; l1 = x0; a1 = ylo; b1 = yhi; l2 = y1; a2 = x0; b2 = x1; ntp = 1; tx0 = x0; ty0 = y1; break;
-    case kZHVH:
-      b1 = m; v2 = 1; l2 = m; a2 = ylo; b2 = yhi; l3 = y1; a3 = m; b3 = x1;
-      ntp = 2; tx0 = m; ty0 = y0; tx1 = m; ty1 = y1; break;
-    default:  // kZVHV
-      v1 = 1; l1 = x0; a1 = min(y0, m); b1 = max(y0, m); l2 = m; a2 = x0; b2 = x1;
-      v3 = 1; l3 = x1; a3 = min(m, y1); b3 = max(m, y1);
-      ntp = 2; tx0 = x0; ty0 = m; tx1 = x1; ty1 = m; break;
-  }
-  auto seg = [&](int isv, int line, int lo, int hi) -> double {
-    if (lo == hi) return 0.0;
-    return isv ? SV[W.v(line, hi)] - SV[W.v(line, lo)] : SH[W.h(hi, line)] - SH[W.h(lo, line)];
-  };
+  // segment 1 (always)
+  const bool v1 = k.sv | k.vh | k.zv;
+  const int l1 = v1 ? x0 : y0;
+  const int a1 = v1 ? (k.zv ? min(y0, m) : ylo) : x0;
+  const int b1 = v1 ? (k.zv ? max(y0, m) : yhi) : (k.zh ? m : x1);
+  // segment 2 (L and Z)
+  const bool v2 = k.hv | k.zh;
+  const int l2 = k.hv ? x1 : (k.vh ? y1 : m);
+  const int a2 = v2 ? ylo : x0;
+  const int b2 = v2 ? yhi : x1;
+  // segment 3 (Z)
+  const int l3 = k.zh ? y1 : x1;
+  const int a3 = k.zh ? m : min(m, y1);
+  const int b3 = k.zh ? x1 : max(m, y1);
+  const bool s2 = !(k.sh | k.sv), s3 = k.zh | k.zv;
+  // turning points (default cell (x0, y0) when unused)
+  const int tx0 = k.hv ? x1 : (k.zh ? m : x0);
+  const int ty0 = k.hv ? y0 : (k.vh ? y1 : (k.zv ? m : y0));
+  const int tx1 = k.zh ? m : (k.zv ? x1 : x0);
+  const int ty1 = k.zh ? y1 : (k.zv ? m : y0);
+  const int ntp = (k.hv | k.vh) ? 1 : (s3 ? 2 : 0);
+  auto sidx = [&](bool isv, int line, int pos) { return isv ? W.v(line, pos) : W.h(pos, line); };
+  const int i1b = sidx(v1, l1, b1), i1a = sidx(v1, l1, a1);
+  const int i2b = s2 ? sidx(v2, l2, b2) : i1b, i2a = s2 ? sidx(v2, l2, a2) : i1b;
+  const int i3b = s3 ? sidx(k.zv, l3, b3) : i1b, i3a = s3 ? sidx(k.zv, l3, a3) : i1b;
+  const double seg = (S[i1b] - S[i1a]) + (S[i2b] - S[i2a]) + (S[i3b] - S[i3a]);
   auto tp = [&](int x, int y) -> double {
-    return SH[W.h(min(x + 1, X - 1), y)] - SH[W.h(max(x - 1, 0), y)] + SV[W.v(x, min(y + 1, Y - 1))] -
-           SV[W.v(x, max(y - 1, 0))];
+    return S[W.h(min(x + 1, X - 1), y)] - S[W.h(max(x - 1, 0), y)] + S[W.v(x, min(y + 1, Y - 1))] -
+           S[W.v(x, max(y - 1, 0))];
   };
-  double c = seg(v1, l1, a1, b1) + seg(v2, l2, a2, b2) + seg(v3, l3, a3, b3);
-  if (ntp >= 1) c += (double)A.beta * tp(tx0, ty0);
-  if (ntp >= 2) c += (double)A.beta * tp(tx1, ty1);
-  c += (double)A.a_wl * (double)((x1 - x0) + (yhi - ylo)) + (double)A.a_via * (double)A.sqrt_l * ntp;
-  return c;
+  const double t0 = tp(tx0, ty0), t1 = tp(tx1, ty1);
+  const double tps = (ntp >= 1 ? t0 : 0.0) + (ntp >= 2 ? t1 : 0.0);
+  return seg + (double)A.beta * tps + (double)A.a_wl * (double)((x1 - x0) + (yhi - ylo)) +
+         (double)A.a_via * (double)A.sqrt_l * ntp;
+}
+
+__device__ __forceinline__ void red_shared_add(uint32_t saddr, int v) {
+  asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.s32 p, %1, 0;\n\t@p red.shared.add.s32 [%0], %1;\n\t}" ::"r"(saddr), "r"(v)
+               : "memory");
+}
+
+// g = -ln(-ln u) from one Philox word
+__device__ __forceinline__ float gumbel_word(uint32_t w) {
+  const float u = ((float)(w >> 9) + 0.5f) * (1.0f / 8388608.0f);
+  return -logf(-logf(u));
+}
+
+// Gumbel noise of a warp's contiguous candidates gid0 .. gid0+n-1 into g[0..n): one Philox4x32-10
+// call per 4 consecutive candidates (counter gid >> 2), spread over the lanes.
+__device__ __forceinline__ void warp_noise(float* g, uint64_t seed, int64_t gid0, int n, uint32_t k, int lane) {
+  const int64_t c0 = gid0 >> 2, c1 = (gid0 + n - 1) >> 2;
+  const uint2 key = make_uint2((uint32_t)seed, (uint32_t)(seed >> 32));
+  for (int64_t c = c0 + lane; c <= c1; c += 32) {
+    const uint4 r = philox4x32_10(make_uint4((uint32_t)c, (uint32_t)(c >> 32), k, 0u), key);
+    const int64_t i0 = c * 4 - gid0;
+    if (i0 >= 0 && i0 < n) g[i0] = gumbel_word(r.x);
+    if (i0 + 1 >= 0 && i0 + 1 < n) g[i0 + 1] = gumbel_word(r.y);
+    if (i0 + 2 >= 0 && i0 + 2 < n) g[i0 + 2] = gumbel_word(r.z);
+    if (i0 + 3 >= 0 && i0 + 3 < n) g[i0 + 3] = gumbel_word(r.w);
+  }
+  __syncwarp();
+}
+
+// Lane view built from already-loaded bundle info and pattern word (no memory access).
+__device__ __forceinline__ void lane_from(int4 bi, uint32_t pw, const KParams& P, Lane& L) {
+  L.lane = threadIdx.x & 31;
+  L.pw = pw;
+  L.shape = pw & 7u;
+  L.valid = L.shape != kPad;
+  L.hm = __ballot_sync(kFull, pw & kSubHead);
+  L.tm = __ballot_sync(kFull, pw & kTreeHead);
+  L.le = kFull >> (31 - L.lane);
+  L.head = 31 - __clz(L.hm & L.le);
+  const uint32_t rest = L.hm & ~L.le;
+  L.end = rest ? (__ffs(rest) - 2) : 31;
+  L.gmask = (kFull >> (31 - L.end)) & ~((1u << L.head) - 1u);
+  L.sub = bi.y + __popc(L.hm & L.le) - 1;
+  L.tree = bi.z + __popc(L.tm & L.le & ~1u);
+  L.lpath = (int64_t)bi.x + L.lane;
+  L.gid = P.path_base + L.lpath;
+}
+
+__device__ __forceinline__ float softmax_from_noise(const Lane& L, float w, float g, float inv_t) {
+  const float z = L.valid ? (w + g) * inv_t : -INFINITY;
+  float m = seg_reduce(z, L.lane, L.end, Max());
+  m = __shfl_sync(kFull, m, L.head);
+  const float e = L.valid ? __expf(z - m) : 0.f;
+  float s = seg_reduce(e, L.lane, L.end, Sum());
+  s = __shfl_sync(kFull, s, L.head);
+  return L.valid ? __fdividef(e, s) : 0.f;
 }
 
 // ------------------------------------------------------------------------------------------
-// The tile kernel.  Shared memory (dynamic):
-//   SH_s, SV_s   double[kWinMax]   S window (reverse)
-//   dH_s, dV_s, VD_s int[kWinMax]  demand-event window (forward), 2^-24 fixed point
-//   wst          float[kMaxBundles*32]  new logits of the tile (reverse -> forward)
-//   dq_s         long long[kTreeMax]    dq_j in 2^-32 fixed point
-//   q_s          float[kTreeMax]        q_j of the forward iteration
-//   red_s        long long[2]           E[WL], E[TP] partial sums
+// The tile kernel.  Shared memory (dynamic), region A is reused between the two halves:
+//   A, reverse:  S_s   double[2 kWinMax]          S window: H part, then V part
+//   A, forward:  ev_s  int[3 kWinMax]             demand-event window dH | dV | VD, 2^-24 fixed point
+//                g_s   float[kWarps][kWarpCand]   Gumbel noise of each warp's candidates
+//   wst    float[kMaxBundles * 32]    new logits of the tile (reverse -> forward)
+//   dq_s   long long[kTreeMax]        dq_j in 2^-32 fixed point
+//   q_s    float[kTreeMax]            q_j (iteration k in the reverse, k_next in the forward)
+//   red_s  long long[2]               E[WL], E[TP] partial sums
+// Each warp owns a contiguous range of the tile's bundles, so its candidates are contiguous.
 // ------------------------------------------------------------------------------------------
-constexpr size_t kSmemBytes = 2 * sizeof(double) * kWinMax + 3 * sizeof(int) * kWinMax +
-                              sizeof(float) * kMaxBundles * 32 + sizeof(long long) * kTreeMax +
+constexpr int kWarps = kTileThreads / 32;
+constexpr int kWarpBundles = (kMaxBundles + kWarps - 1) / kWarps;
+constexpr int kWarpCand = kWarpBundles * 32;
+constexpr size_t kRegionA = 2 * sizeof(double) * kWinMax;
+static_assert(3 * sizeof(int) * kWinMax + sizeof(float) * kWarps * kWarpCand <= kRegionA, "region A too small");
+constexpr size_t kSmemBytes = kRegionA + sizeof(float) * kMaxBundles * 32 + sizeof(long long) * kTreeMax +
                               sizeof(float) * kTreeMax + 2 * sizeof(long long);
 
 template <bool GLOBAL>
-__device__ __forceinline__ void reverse_bundle(const KParams& P, const StepArgs& A, const TileDesc& T, int b,
-                                               const double* SH, const double* SV, const Win& W,
-                                               long long* dq_s, float* wst) {
+__device__ __forceinline__ void reverse_warp(const KParams& P, const StepArgs& A, const TileDesc& T, int bw0,
+                                             int bw1, const double* S, const Win& W, long long* dq_s,
+                                             const float* q_s, float* wst) {
+  const int lane = threadIdx.x & 31;
+  // software pipeline: bundle b computes while b+1's operands (incl. its sub-net endpoints, which
+  // depend on b+1's ballots) and b+2's bundle info / pattern word are in flight
+  size_t slot = (size_t)bw0 * 32 + lane;
   Lane L;
-  lane_setup(P, b, L);
-  const size_t slot = (size_t)b * 32 + L.lane;
-  float w = P.wp[slot];
-  const float p = group_softmax(P, A.inv_t, (uint32_t)A.k, L, w);
-  const float q = L.valid ? P.q[L.tree] : 0.f;
-  double c = 0.0;
-  if (L.valid) {
-    const short4 e = __ldg(&P.sxy[L.sub]);
-    c = path_cost(SH, SV, W, P.X, P.Y, L.shape, e.x, e.y, e.z, e.w, (int)(L.pw >> 16), A);
+  lane_from(__ldg(&P.binfo[bw0]), __ldg(&P.pword[slot]), P, L);
+  short4 e = L.valid ? __ldg(&P.sxy[L.sub]) : make_short4(0, 0, 0, 0);
+  float w = P.wp[slot], m = P.mp[slot], v = P.vp[slot], p = P.pp[slot];
+  int4 bi1 = make_int4(0, 0, 0, 0);
+  uint32_t pw1 = kPad | kSubHead;
+  if (bw0 + 1 < bw1) { bi1 = __ldg(&P.binfo[bw0 + 1]); pw1 = __ldg(&P.pword[slot + 32]); }
+  for (int b = bw0; b < bw1; ++b) {
+    Lane Ln = L;
+    short4 en = e;
+    float wn = w, mn = m, vn = v, pn = p;
+    if (b + 1 < bw1) {
+      lane_from(bi1, pw1, P, Ln);
+      if (Ln.valid) en = __ldg(&P.sxy[Ln.sub]);
+      wn = P.wp[slot + 32]; mn = P.mp[slot + 32]; vn = P.vp[slot + 32]; pn = P.pp[slot + 32];
+      if (b + 2 < bw1) { bi1 = __ldg(&P.binfo[b + 2]); pw1 = __ldg(&P.pword[slot + 64]); }
+    }
+    const float q = L.valid ? q_s[L.tree - T.tree0] : 0.f;
+    const double c = L.valid ? path_cost(S, W, P.X, P.Y, L.shape, e.x, e.y, e.z, e.w, (int)(L.pw >> 16), A) : 0.0;
+    // softmax backward dw_i = (p_i/t)(dp_i - sum_k p_k dp_k / sum_k p_k): differences to the group
+    // head's dp are formed in fp64 and reduced in fp32, so neither the magnitude of c nor
+    // sum_k p_k != 1 (rounding) leaks into dw.
+    const double dp = (double)q * c;
+    const double dref = __shfl_sync(kFull, dp, L.head);
+    const float dd = (float)(dp - dref);
+    float sa = seg_reduce(p * dd, L.lane, L.end, Sum());
+    float sb = seg_reduce(p, L.lane, L.end, Sum());
+    sa = __shfl_sync(kFull, sa, L.head);
+    sb = __shfl_sync(kFull, sb, L.head);
+    const float dw = L.valid ? p * A.inv_t * (dd - __fdividef(sa, sb)) : 0.f;
+    // dq_j = sum_{i in tree j} p_i c_i: reduce over this warp's lanes of each tree (fp64: the tree
+    // gradient is a difference of such sums)
+    const uint32_t th = L.tm | __ballot_sync(kFull, !L.valid) | 1u;
+    const uint32_t trest = th & ~L.le;
+    const int tend = trest ? (__ffs(trest) - 2) : 31;
+    const double pc = seg_reduce(L.valid ? (double)p * c : 0.0, L.lane, tend, Sum());
+    if (L.valid && ((th >> L.lane) & 1u))
+      atomicAdd(reinterpret_cast<unsigned long long*>(&dq_s[L.tree - T.tree0]),
+                static_cast<unsigned long long>(__double2ll_rn(pc * kDqScale)));
+    if (L.valid) {
+      adam_update(w, m, v, dw, A);
+      P.wp[slot] = w;
+      P.mp[slot] = m;
+      P.vp[slot] = v;
+    }
+    wst[(b - T.b0) * 32 + lane] = w;
+    L = Ln; e = en; w = wn; m = mn; v = vn; p = pn;
+    slot += 32;
   }
-  // softmax backward dw_i = (p_i/t)(dp_i - sum_k p_k dp_k).  The weighted mean is divided by the
-  // fp32 probabilities' own sum so that sum_k p_k != 1 (rounding) cannot leak c's magnitude into dw.
-  const double dp = (double)q * c;
-  double spd = seg_reduce((double)p * dp, L.lane, L.end, Sum());
-  double sp = seg_reduce((double)p, L.lane, L.end, Sum());
-  spd = __shfl_sync(kFull, spd, L.head);
-  sp = __shfl_sync(kFull, sp, L.head);
-  const double dw = L.valid ? (double)p * (double)A.inv_t * (dp - spd / sp) : 0.0;
-  // dq_j = sum_{i in tree j} p_i c_i: reduce over this warp's lanes of each tree
-  const uint32_t th = L.tm | __ballot_sync(kFull, !L.valid) | 1u;
-  const uint32_t trest = th & ~L.le;
-  const int tend = trest ? (__ffs(trest) - 2) : 31;
-  const double pc = seg_reduce(L.valid ? (double)p * c : 0.0, L.lane, tend, Sum());
-  if (L.valid && ((th >> L.lane) & 1u))
-    atomicAdd(reinterpret_cast<unsigned long long*>(&dq_s[L.tree - T.tree0]),
-              static_cast<unsigned long long>(__double2ll_rn(pc * kDqScale)));
-  if (L.valid) {
-    float m = P.mp[slot], v = P.vp[slot];
-    adam_update(w, m, v, (float)dw, A);
-    P.wp[slot] = w;
-    P.mp[slot] = m;
-    P.vp[slot] = v;
-  }
-  wst[(b - T.b0) * 32 + L.lane] = w;
 }
 
 // Forward events of one lane.  For a canonical sub-net (x0 < x1), s = sgn(y1 - y0), the +-pi events
@@ -234,119 +324,141 @@ __device__ __forceinline__ void reverse_bundle(const KParams& P, const StepArgs&
 //   Z-HVH(xm): (xm,y0): -pi, +s pi, +pi   (xm,y1): +pi, -s pi, +pi        [dH, dV, VD]
 //   Z-VHV(ym): (x0,ym): +pi, -s pi, +pi   (x1,ym): -pi, +s pi, +pi
 // with A = pi_HV, B = pi_VH, Hs = sum pi over Z-HVH, Vs = sum pi over Z-VHV.  dH is the difference
-// array of the H wire demand along rows, dV along columns, VD the turning points.
+// array of the H wire demand along rows, dV along columns, VD the turning points.  Written as
+// 0/1-flag arithmetic so the warp never diverges on the pattern.
 template <bool GLOBAL>
-__device__ __forceinline__ void forward_bundle(const KParams& P, const StepArgs& A, const TileDesc& T, int b,
-                                               bool have_w, const float* wst, const float* q_s, const Win& W,
-                                               int* dH_s, int* dV_s, int* VD_s, long long* red_s) {
-  Lane L;
-  lane_setup(P, b, L);
-  const size_t slot = (size_t)b * 32 + L.lane;
-  const float w = have_w ? wst[(b - T.b0) * 32 + L.lane] : P.wp[slot];
-  const float p = group_softmax(P, A.inv_t, (uint32_t)A.k_next, L, w);
-  const float q = L.valid ? q_s[L.tree - T.tree0] : 0.f;
-  const int vq = L.valid ? __float2int_rn(q * p * kFixScale) : 0;   // pi in 2^-24 fixed point
-  int sc = vq;                                                       // inclusive scan within the group
-#pragma unroll
-  for (int off = 1; off < 32; off <<= 1) {
-    const int o = __shfl_up_sync(kFull, sc, off);
-    if (L.lane - off >= L.head) sc += o;
-  }
-  const int nh = __popc(__ballot_sync(kFull, L.shape == kZHVH) & L.gmask);
-  const int h1 = min(L.head + 1, 31), h2 = min(L.head + 1 + nh, 31);
-  const int Av = __shfl_sync(kFull, vq, L.head);
-  const int Bv = __shfl_sync(kFull, vq, h1);
-  const int S1 = __shfl_sync(kFull, sc, h1);
-  const int S2 = __shfl_sync(kFull, sc, h2);
-  const int Se = __shfl_sync(kFull, sc, L.end);
-  int xa = 0, ya = 0, xb = 0, yb = 0;
-  int ah = 0, av = 0, ad = 0, bh = 0, bv = 0, bd = 0;
+__device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A, const TileDesc& T, int bw0,
+                                             int bw1, bool have_w, const float* wst, const float* q_s, float* g_s,
+                                             const Win& W, int* ev_s, long long* red_s) {
+  const int lane = threadIdx.x & 31;
+  const int4 bfirst = __ldg(&P.binfo[bw0]);
+  const int4 blast = __ldg(&P.binfo[bw1 - 1]);
+  warp_noise(g_s, P.seed, P.path_base + bfirst.x, blast.x + blast.w - bfirst.x, (uint32_t)A.k_next, lane);
+  const uint32_t ev_base = (uint32_t)__cvta_generic_to_shared(ev_s);
   long long wl = 0, tpc = 0;
-  if (L.valid) {
-    const short4 e = __ldg(&P.sxy[L.sub]);
+  size_t slot = (size_t)bw0 * 32 + lane;
+  Lane L;
+  lane_from(bfirst, __ldg(&P.pword[slot]), P, L);
+  short4 e = L.valid ? __ldg(&P.sxy[L.sub]) : make_short4(0, 0, 0, 0);
+  int4 bi1 = make_int4(0, 0, 0, 0);
+  uint32_t pw1 = kPad | kSubHead;
+  if (bw0 + 1 < bw1) { bi1 = __ldg(&P.binfo[bw0 + 1]); pw1 = __ldg(&P.pword[slot + 32]); }
+  for (int b = bw0; b < bw1; ++b) {
+    Lane Ln = L;
+    short4 en = e;
+    if (b + 1 < bw1) {
+      lane_from(bi1, pw1, P, Ln);
+      if (Ln.valid) en = __ldg(&P.sxy[Ln.sub]);
+      if (b + 2 < bw1) { bi1 = __ldg(&P.binfo[b + 2]); pw1 = __ldg(&P.pword[slot + 64]); }
+    }
+    const float w = have_w ? wst[(b - T.b0) * 32 + lane] : P.wp[slot];
+    const float g = L.valid ? g_s[L.lpath - bfirst.x] : 0.f;
+    const float p = softmax_from_noise(L, w, g, A.inv_t);
+    P.pp[slot] = p;
+    const float q = L.valid ? q_s[L.tree - T.tree0] : 0.f;
+    const int vq = L.valid ? __float2int_rn(q * p * kFixScale) : 0;   // pi in 2^-24 fixed point
+    int sc = vq;                                                       // inclusive scan within the group
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+      const int o = __shfl_up_sync(kFull, sc, off);
+      if (L.lane - off >= L.head) sc += o;
+    }
+    const int nh = __popc(__ballot_sync(kFull, L.shape == kZHVH) & L.gmask);
+    const int h1 = min(L.head + 1, 31), h2 = min(L.head + 1 + nh, 31);
+    const int a = __shfl_sync(kFull, vq, L.head);
+    const int bb = __shfl_sync(kFull, vq, h1);
+    const int S1 = __shfl_sync(kFull, sc, h1);
+    const int S2 = __shfl_sync(kFull, sc, h2);
+    const int Se = __shfl_sync(kFull, sc, L.end);
     const int x0 = e.x, y0 = e.y, x1 = e.z, y1 = e.w;
     const int s = (y1 > y0) ? 1 : -1;
-    const int a = Av, bb = Bv, hs = S2 - S1, vs = Se - S2, v = vq;
-    const int m = (int)(L.pw >> 16);
-    int ntp = 0;
-    switch (L.shape) {
-      case kStraightH: xa = x0; ya = y0; ah = v; xb = x1; yb = y0; bh = -v; break;
-      case kStraightV: xa = x0; ya = y0; av = v; xb = x0; yb = y1; bv = -v; break;
-      case kHV:
-        xa = x0; ya = y0; ah = a + hs; av = s * (bb + vs);
-        xb = x1; yb = y0; bh = -a; bv = s * a; bd = a; ntp = 1; break;
-      case kVH:
-        xa = x0; ya = y1; ah = bb; av = -s * bb; ad = bb;
-        xb = x1; yb = y1; bh = -(bb + hs); bv = -s * (a + vs); ntp = 1; break;
-      case kZHVH:
-        xa = m; ya = y0; ah = -v; av = s * v; ad = v;
-        xb = m; yb = y1; bh = v; bv = -s * v; bd = v; ntp = 2; break;
-      default:
-        xa = x0; ya = m; ah = v; av = -s * v; ad = v;
-        xb = x1; yb = m; bh = -v; bv = s * v; bd = v; ntp = 2; break;
+    const int hs = S2 - S1, vs = Se - S2, v = vq;
+    const int mm = (int)(L.pw >> 16);
+    const int fSH = L.shape == kStraightH, fSV = L.shape == kStraightV, fHV = L.shape == kHV;
+    const int fVH = L.shape == kVH, fZH = L.shape == kZHVH, fZV = L.shape == kZVHV;
+    const int fZ = fZH + fZV;
+    const int xa = x0 + fZH * (mm - x0);
+    const int ya = y0 + fVH * (y1 - y0) + fZV * (mm - y0);
+    const int xb = x1 + fSV * (x0 - x1) + fZH * (mm - x1);
+    const int yb = y1 + (fSH + fHV) * (y0 - y1) + fZV * (mm - y1);
+    const int ah = fSH * v + fHV * (a + hs) + fVH * bb + (fZV - fZH) * v;
+    const int av = fSV * v + s * (fHV * (bb + vs) - fVH * bb + (fZH - fZV) * v);
+    const int ad = fVH * bb + fZ * v;
+    const int bh = -fSH * v - fHV * a - fVH * (bb + hs) + (fZH - fZV) * v;
+    const int bv = -fSV * v + s * (fHV * a - fVH * (a + vs) + (fZV - fZH) * v);
+    const int bd = fHV * a + fZ * v;
+    if (L.valid) {
+      if (GLOBAL) {
+        const int X = P.X, Y = P.Y;
+        red64(P.dH + (size_t)ya * X + xa, ah); red64(P.dVT + (size_t)xa * Y + ya, av);
+        red64(P.VDH + (size_t)ya * X + xa, ad); red64(P.VDV + (size_t)xa * Y + ya, ad);
+        red64(P.dH + (size_t)yb * X + xb, bh); red64(P.dVT + (size_t)xb * Y + yb, bv);
+        red64(P.VDH + (size_t)yb * X + xb, bd); red64(P.VDV + (size_t)xb * Y + yb, bd);
+      }
+      const int ntp = fHV + fVH + 2 * fZ;
+      wl += (long long)vq * ((x1 - x0) + abs(y1 - y0));
+      tpc += (long long)vq * ntp;
     }
-    wl = (long long)vq * ((x1 - x0) + abs(y1 - y0));
-    tpc = (long long)vq * ntp;
+    if (!GLOBAL) {
+      const int hv2 = 2 * W.hv;   // VD part of the event window
+      const int ia_h = W.h(xa, ya), ib_h = W.h(xb, yb);
+      red_shared_add(ev_base + 4u * ia_h, ah);
+      red_shared_add(ev_base + 4u * W.v(xa, ya), av);
+      red_shared_add(ev_base + 4u * (hv2 + ia_h), ad);
+      red_shared_add(ev_base + 4u * ib_h, bh);
+      red_shared_add(ev_base + 4u * W.v(xb, yb), bv);
+      red_shared_add(ev_base + 4u * (hv2 + ib_h), bd);
+    }
+    L = Ln; e = en;
+    slot += 32;
   }
-  if (GLOBAL) {
-    const int X = P.X, Y = P.Y;
-    red64(P.dH + (size_t)ya * X + xa, ah); red64(P.dVT + (size_t)xa * Y + ya, av);
-    red64(P.VDH + (size_t)ya * X + xa, ad); red64(P.VDV + (size_t)xa * Y + ya, ad);
-    red64(P.dH + (size_t)yb * X + xb, bh); red64(P.dVT + (size_t)xb * Y + yb, bv);
-    red64(P.VDH + (size_t)yb * X + xb, bd); red64(P.VDV + (size_t)xb * Y + yb, bd);
-  } else {
-    if (ah) atomicAdd(&dH_s[W.h(xa, ya)], ah);
-    if (av) atomicAdd(&dV_s[W.v(xa, ya)], av);
-    if (ad) atomicAdd(&VD_s[W.h(xa, ya)], ad);
-    if (bh) atomicAdd(&dH_s[W.h(xb, yb)], bh);
-    if (bv) atomicAdd(&dV_s[W.v(xb, yb)], bv);
-    if (bd) atomicAdd(&VD_s[W.h(xb, yb)], bd);
-  }
-  wl = seg_reduce(wl, L.lane, 31, Sum());
-  tpc = seg_reduce(tpc, L.lane, 31, Sum());
-  if (L.lane == 0) {
+  wl = seg_reduce(wl, lane, 31, Sum());
+  tpc = seg_reduce(tpc, lane, 31, Sum());
+  if (lane == 0) {
     atomicAdd(reinterpret_cast<unsigned long long*>(&red_s[0]), static_cast<unsigned long long>(wl));
     atomicAdd(reinterpret_cast<unsigned long long*>(&red_s[1]), static_cast<unsigned long long>(tpc));
   }
 }
 
 template <bool REV, bool FWD>
-__global__ void __launch_bounds__(kTileThreads) tile_kernel(KParams P, StepArgs A) {
+__global__ void __launch_bounds__(kTileThreads, 3) tile_kernel(KParams P, StepArgs A) {
   extern __shared__ __align__(16) unsigned char smem[];
-  double* SH_s = reinterpret_cast<double*>(smem);
-  double* SV_s = SH_s + kWinMax;
-  int* dH_s = reinterpret_cast<int*>(SV_s + kWinMax);
-  int* dV_s = dH_s + kWinMax;
-  int* VD_s = dV_s + kWinMax;
-  float* wst = reinterpret_cast<float*>(VD_s + kWinMax);
+  double* S_s = reinterpret_cast<double*>(smem);                 // region A (reverse)
+  int* ev_s = reinterpret_cast<int*>(smem);                      // region A (forward)
+  float* g_all = reinterpret_cast<float*>(ev_s + 3 * kWinMax);   // region A (forward)
+  float* wst = reinterpret_cast<float*>(smem + kRegionA);
   long long* dq_s = reinterpret_cast<long long*>(wst + kMaxBundles * 32);
   float* q_s = reinterpret_cast<float*>(dq_s + kTreeMax);
   long long* red_s = reinterpret_cast<long long*>(q_s + kTreeMax);
 
   const TileDesc T = P.tiles[blockIdx.x];
-  const int tid = threadIdx.x, warp = tid >> 5, nwarp = kTileThreads / 32;
+  const int tid = threadIdx.x, warp = tid >> 5;
   const int ncell = T.ww * T.wh;
   const int X = P.X, Y = P.Y;
-  const Win Wg{0, 0, X, Y};
-  const Win Ws{T.wx0, T.wy0, T.ww, T.wh};
+  const Win Wg{0, 0, X, Y, X * Y};
+  const Win Ws{T.wx0, T.wy0, T.ww, T.wh, ncell};
+  float* g_s = g_all + warp * kWarpCand;
+  // this warp's contiguous bundle range
+  const int per = (T.nb + kWarps - 1) / kWarps;
+  const int bw0 = T.b0 + min(warp * per, T.nb), bw1 = T.b0 + min((warp + 1) * per, T.nb);
 
   // ---------------- reverse of iteration k ----------------
   if (REV) {
     if (!T.global) {
       for (int i = tid; i < ncell; i += kTileThreads) {
         const int yi = i / T.ww, xi = i - yi * T.ww;
-        SH_s[i] = P.SH[(size_t)(T.wy0 + yi) * X + T.wx0 + xi];
+        S_s[i] = P.SH[(size_t)(T.wy0 + yi) * X + T.wx0 + xi];
       }
       for (int i = tid; i < ncell; i += kTileThreads) {
         const int xi = i / T.wh, yi = i - xi * T.wh;
-        SV_s[i] = P.SVT[(size_t)(T.wx0 + xi) * Y + T.wy0 + yi];
+        S_s[ncell + i] = P.SVT[(size_t)(T.wx0 + xi) * Y + T.wy0 + yi];
       }
     }
-    for (int i = tid; i < T.ntree; i += kTileThreads) dq_s[i] = 0;
+    for (int i = tid; i < T.ntree; i += kTileThreads) { dq_s[i] = 0; q_s[i] = P.q[T.tree0 + i]; }
     __syncthreads();
-    for (int b = T.b0 + warp; b < T.b0 + T.nb; b += nwarp) {
-      if (T.global) reverse_bundle<true>(P, A, T, b, P.SH, P.SVT, Wg, dq_s, wst);
-      else reverse_bundle<false>(P, A, T, b, SH_s, SV_s, Ws, dq_s, wst);
+    if (bw0 < bw1) {
+      if (T.global) reverse_warp<true>(P, A, T, bw0, bw1, P.SH, Wg, dq_s, q_s, wst);
+      else reverse_warp<false>(P, A, T, bw0, bw1, S_s, Ws, dq_s, q_s, wst);
     }
     __syncthreads();
   }
@@ -359,14 +471,14 @@ __global__ void __launch_bounds__(kTileThreads) tile_kernel(KParams P, StepArgs 
       // du_j = (q_j/t)(dq_j - sum_l q_l dq_l / sum_l q_l); Adam on w_tree (iteration k)
       double sq = 0.0, sw = 0.0;
       for (int j = a; j < b; ++j) {
-        const double qj = (double)P.q[j];
+        const double qj = (double)q_s[j - T.tree0];
         sq += qj * ((double)dq_s[j - T.tree0] * kDqInv);
         sw += qj;
       }
       sq /= sw;
       for (int j = a; j < b; ++j) {
         const double du = (b - a == 1) ? 0.0
-                                       : (double)P.q[j] * (double)A.inv_t * ((double)dq_s[j - T.tree0] * kDqInv - sq);
+                                       : (double)q_s[j - T.tree0] * (double)A.inv_t * ((double)dq_s[j - T.tree0] * kDqInv - sq);
         float w = P.wt[j], m = P.mt[j], v = P.vt[j];
         adam_update(w, m, v, (float)du, A);
         P.wt[j] = w; P.mt[j] = m; P.vt[j] = v;
@@ -395,12 +507,12 @@ __global__ void __launch_bounds__(kTileThreads) tile_kernel(KParams P, StepArgs 
   // ---------------- forward of iteration k_next ----------------
   if (FWD) {
     if (!T.global)
-      for (int i = tid; i < ncell; i += kTileThreads) { dH_s[i] = 0; dV_s[i] = 0; VD_s[i] = 0; }
+      for (int i = tid; i < 3 * ncell; i += kTileThreads) ev_s[i] = 0;
     if (tid < 2) red_s[tid] = 0;
     __syncthreads();
-    for (int b = T.b0 + warp; b < T.b0 + T.nb; b += nwarp) {
-      if (T.global) forward_bundle<true>(P, A, T, b, REV, wst, q_s, Wg, dH_s, dV_s, VD_s, red_s);
-      else forward_bundle<false>(P, A, T, b, REV, wst, q_s, Ws, dH_s, dV_s, VD_s, red_s);
+    if (bw0 < bw1) {
+      if (T.global) forward_warp<true>(P, A, T, bw0, bw1, REV, wst, q_s, g_s, Wg, ev_s, red_s);
+      else forward_warp<false>(P, A, T, bw0, bw1, REV, wst, q_s, g_s, Ws, ev_s, red_s);
     }
     __syncthreads();
     if (!T.global) {
@@ -408,14 +520,14 @@ __global__ void __launch_bounds__(kTileThreads) tile_kernel(KParams P, StepArgs 
       for (int i = tid; i < ncell; i += kTileThreads) {
         const int yi = i / T.ww, xi = i - yi * T.ww;
         const size_t g = (size_t)(T.wy0 + yi) * X + T.wx0 + xi;
-        red64(P.dH + g, dH_s[i]);
-        red64(P.VDH + g, VD_s[i]);
+        red64(P.dH + g, ev_s[i]);
+        red64(P.VDH + g, ev_s[2 * ncell + i]);
       }
       for (int i = tid; i < ncell; i += kTileThreads) {
         const int xi = i / T.wh, yi = i - xi * T.wh;
         const size_t g = (size_t)(T.wx0 + xi) * Y + T.wy0 + yi;
-        red64(P.dVT + g, dV_s[i]);
-        red64(P.VDV + g, VD_s[yi * T.ww + xi]);
+        red64(P.dVT + g, ev_s[ncell + i]);
+        red64(P.VDV + g, ev_s[2 * ncell + yi * T.ww + xi]);
       }
     }
     if (tid == 0) { red64(P.scal, red_s[0]); red64(P.scal + 1, red_s[1]); }

@@ -138,8 +138,10 @@ def test_forward_parity(forests, name, f_kind):
 
 @pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18"])
 def test_one_iteration_parity(forests, name):
+    """After one Adam step the update of a coordinate whose gradient is ~eps depends on that
+    gradient's last bits (Q21b), so the fp32 probe applies from the first step on."""
     s, o, gl, ol = run_both(forests[name], [(1, 1.0)])
-    compare_state(s, o, name)
+    compare_state(s, o, name, probe=probes(forests[name], [(1, 1.0)]), max_ill=1e-3)
     assert s.iteration == 1
 
 
