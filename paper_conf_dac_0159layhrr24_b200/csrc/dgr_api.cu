@@ -186,8 +186,9 @@ struct Plan {
   std::vector<short4> sxy;
   std::vector<int32_t> net_tree_off;
   std::vector<int64_t> sub_first_path;   // local path index of each local sub-net's first candidate
-  std::vector<TileDesc> tiles;
+  std::vector<TileDesc> tiles;          // pipelined tiles first (see make_plan)
   int64_t n_global_tiles = 0;
+  int64_t n_pipe_tiles = 0;
 };
 
 // Cells (x, y) touched by one candidate's demand events (see forward_bundle in dgr_kernels.cu)
@@ -257,7 +258,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   pl.tiles.clear();
   pl.binfo.clear();
   pl.pword.clear();
-  struct Cur { bool open = false; int64_t net0 = 0; int nb = 0, fill = 32, ntree = 0; int bx0 = 0, by0 = 0, bx1 = -1, by1 = -1; bool global = false; } cur;
+  struct Cur { bool open = false; int64_t net0 = 0; int nb = 0, fill = 32, ntree = 0, nsub = 0; int bx0 = 0, by0 = 0, bx1 = -1, by1 = -1; bool global = false; } cur;
   std::vector<int64_t> tile_net0;
   std::vector<char> tile_glob;
   auto net_box = [&](int64_t n, int& bx0, int& by0, int& bx1, int& by1) {
@@ -279,35 +280,43 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       fill += g;
     }
   };
+  // windows start on even cells and have even extents so their S rows / columns are 16-byte
+  // aligned for the bulk (TMA) copies (the S arrays have an even pitch)
+  auto aligned_area = [](int bx0, int by0, int bx1, int by1) -> int64_t {
+    const int x0 = bx0 & ~1, y0 = by0 & ~1;
+    const int w = (bx1 + 1 - x0 + 1) & ~1, h = (by1 + 1 - y0 + 1) & ~1;
+    return (int64_t)w * h;
+  };
   std::vector<int64_t> starts;
   std::vector<char> globs;
   for (int64_t n = pl.net_lo; n < pl.net_hi; ++n) {
     int bx0, by0, bx1, by1;
     net_box(n, bx0, by0, bx1, by1);
-    const bool big = (int64_t)(bx1 - bx0 + 1) * (by1 - by0 + 1) > kWinMax;
+    const bool big = aligned_area(bx0, by0, bx1, by1) > kWinMax;
     const int ntree = (int)(d->net_tree_off[n + 1] - d->net_tree_off[n]);
+    const int nsub = (int)(d->tree_sub_off[d->net_tree_off[n + 1]] - d->tree_sub_off[d->net_tree_off[n]]);
     bool fits = cur.open && !cur.global && !big;
     int nb2 = cur.nb, fill2 = cur.fill;
     if (fits) {
       const int ux0 = std::min(cur.bx0, bx0), uy0 = std::min(cur.by0, by0);
       const int ux1 = std::max(cur.bx1, bx1), uy1 = std::max(cur.by1, by1);
       pack_net(n, nb2, fill2);
-      fits = (int64_t)(ux1 - ux0 + 1) * (uy1 - uy0 + 1) <= kWinMax && nb2 <= kTargetBundles &&
-             cur.ntree + ntree <= kTreeMax;
+      fits = aligned_area(ux0, uy0, ux1, uy1) <= kWinMax && nb2 <= kTargetBundles &&
+             cur.ntree + ntree <= kPipeTrees && cur.nsub + nsub <= kPipeSubs;
       if (fits) { cur.bx0 = ux0; cur.by0 = uy0; cur.bx1 = ux1; cur.by1 = uy1; }
     } else if (cur.open && cur.global && big) {
       pack_net(n, nb2, fill2);
       fits = nb2 <= kMaxBundles && cur.ntree + ntree <= kTreeMax;
     }
     if (fits) {
-      cur.nb = nb2; cur.fill = fill2; cur.ntree += ntree;
+      cur.nb = nb2; cur.fill = fill2; cur.ntree += ntree; cur.nsub += nsub;
       continue;
     }
     // close the open tile, open a new one at net n
     starts.push_back(n);
     globs.push_back(big);
     cur = Cur();
-    cur.open = true; cur.global = big; cur.net0 = n; cur.ntree = ntree;
+    cur.open = true; cur.global = big; cur.net0 = n; cur.ntree = ntree; cur.nsub = nsub;
     cur.bx0 = bx0; cur.by0 = by0; cur.bx1 = bx1; cur.by1 = by1;
     cur.nb = 0; cur.fill = 32;
     pack_net(n, cur.nb, cur.fill);
@@ -330,8 +339,11 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       net_box(n, a0, b0_, a1, b1_);
       bx0 = std::min(bx0, a0); by0 = std::min(by0, b0_); bx1 = std::max(bx1, a1); by1 = std::max(by1, b1_);
     }
-    T.wx0 = bx0; T.wy0 = by0; T.ww = bx1 - bx0 + 1; T.wh = by1 - by0 + 1;
+    T.wx0 = bx0 & ~1; T.wy0 = by0 & ~1;
+    T.ww = (bx1 + 1 - T.wx0 + 1) & ~1; T.wh = (by1 + 1 - T.wy0 + 1) & ~1;
     if (T.global) { T.wx0 = 0; T.wy0 = 0; T.ww = 0; T.wh = 0; }
+    T.sub0 = (int32_t)(d->tree_sub_off[d->net_tree_off[starts[t]]] - pl.sub_lo);
+    T.nsub = (int32_t)(d->tree_sub_off[d->net_tree_off[starts[t + 1]]] - pl.sub_lo) - T.sub0;
     int fill = 32;
     const int64_t j0 = d->net_tree_off[starts[t]], j1 = d->net_tree_off[starts[t + 1]];
     for (int64_t j = j0; j < j1; ++j) {
@@ -376,6 +388,13 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     pl.tiles.push_back(T);
   }
   pl.nb = (int)pl.binfo.size();
+  // pipelined tiles (shared-memory window, <= kTargetBundles bundles) first, then the rest
+  auto pipelined = [](const TileDesc& T) {
+    return !T.global && T.nb <= kTargetBundles && T.ntree <= kPipeTrees && T.nsub <= kPipeSubs;
+  };
+  std::stable_partition(pl.tiles.begin(), pl.tiles.end(), pipelined);
+  pl.n_pipe_tiles = 0;
+  for (const auto& T : pl.tiles) pl.n_pipe_tiles += pipelined(T);
   return DGR_OK;
 }
 
@@ -397,22 +416,25 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.tiles = take(sizeof(TileDesc) * pl.tiles.size());
   L.binfo = take(sizeof(int4) * pl.nb);
   L.pword = take(4 * slots);
-  L.sxy = take(8 * ns);
+  L.sxy = take(8 * ns + 16);
   L.wp = take(4 * slots);
   L.mp = take(4 * slots);
   L.vp = take(4 * slots);
   L.pp = take(4 * slots);   // p of the last forward (read by the next reverse)
-  L.nto = take(4 * (nn + 1));
-  L.wt = take(4 * nt);
-  L.mt = take(4 * nt);
-  L.vt = take(4 * nt);
-  L.q = take(4 * nt);
+  L.nto = take(4 * (nn + 1) + 16);   // +16 B: 16-byte aligned bulk reads may run past the end
+  L.wt = take(4 * nt + 16);
+  L.mt = take(4 * nt + 16);
+  L.vt = take(4 * nt + 16);
+  L.q = take(4 * nt + 16);
   L.xcount = 4 * G + 2;   // dH | dV^T | VD (row-major) | VD (column-major) | E[WL], E[TP]
   L.xbuf = take(8 * L.xcount);
   L.capH = take(4 * G);
   L.capVT = take(4 * G);
-  L.SH = take(16 * G);   // S_H then S_V^T, contiguous (one base pointer in the kernels)
-  L.SVT = L.SH + 8 * G;
+  // S_H [Y][XP] then S_V^T [X][YP] (even pitches, contiguous: one base pointer in the kernels),
+  // plus padding for window rows / columns that run one cell past the grid
+  const size_t XP = (size_t)(X + (X & 1)), YP = (size_t)(Y + (Y & 1));
+  L.SH = take(8 * (Y * XP + X * YP) + 256);
+  L.SVT = L.SH + 8 * Y * XP;
   L.dOutH = take(4 * G);
   L.dOutVT = take(4 * G);
   L.partial = take(8 * (size_t)(X + Y));
@@ -544,8 +566,12 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
   h->ws_bytes = workspace_bytes;
   char* ws = h->ws;
   P.nb = pl.nb;
-  P.ntiles = (int32_t)pl.tiles.size();
+  P.ntiles = (int32_t)pl.n_pipe_tiles;
   P.tiles = (const TileDesc*)(ws + L.tiles);
+  P.ntiles_slow = (int32_t)(pl.tiles.size() - pl.n_pipe_tiles);
+  P.tiles_slow = P.tiles + pl.n_pipe_tiles;
+  P.XP = desc->X + (desc->X & 1);
+  P.YP = desc->Y + (desc->Y & 1);
   P.n_nets_l = (int32_t)(pl.net_hi - pl.net_lo);
   P.path_base = pl.path_lo;
   P.tree_base = pl.tree_lo;
@@ -767,7 +793,7 @@ int dgr_get_info(dgr_handle* h, int64_t info[12]) {
   if (!h || !info) return fail(DGR_EINVAL, "NULL argument");
   info[0] = h->k; info[1] = h->plan.net_lo; info[2] = h->plan.net_hi; info[3] = h->plan.nb;
   info[4] = (int64_t)h->plan.nb * 32; info[5] = (int64_t)h->lay.total; info[6] = h->world; info[7] = h->rank;
-  info[8] = (int64_t)h->plan.tiles.size(); info[9] = h->plan.n_global_tiles; info[10] = 0; info[11] = 0;
+  info[8] = (int64_t)h->plan.tiles.size(); info[9] = h->plan.n_global_tiles; info[10] = h->plan.n_pipe_tiles; info[11] = 0;
   return DGR_OK;
 }
 

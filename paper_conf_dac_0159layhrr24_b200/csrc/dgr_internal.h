@@ -35,6 +35,8 @@ constexpr int kWinMax = 2048;                      // window cells per tile
 constexpr int kMaxBundles = 64;                    // bundles per tile (a whole net always fits)
 constexpr int kTargetBundles = 32;                 // planner target per tile
 constexpr int kTreeMax = 512;                      // trees per tile
+constexpr int kPipeTrees = 256;                    // trees per pipelined tile
+constexpr int kPipeSubs = 512;                     // sub-nets per pipelined tile
 constexpr int kEventMax = 127;                     // events per window cell-field (int32 safety)
 
 enum Shape : uint32_t {
@@ -48,8 +50,10 @@ struct TileDesc {
   int32_t b0, nb;          // bundles [b0, b0 + nb)
   int32_t net0, nnet;      // local nets
   int32_t tree0, ntree;    // local trees
-  int32_t wx0, wy0, ww, wh;  // window (cells), unused for global tiles
+  int32_t wx0, wy0, ww, wh;  // window (cells; even origin and extents), unused for global tiles
   int32_t global, pad;
+  int32_t sub0, nsub;      // local sub-nets
+  int32_t pad2, pad3;
 };
 
 struct KParams {
@@ -57,11 +61,14 @@ struct KParams {
   int32_t X, Y;
   int32_t nb;               // bundles
   int32_t n_nets_l;         // local nets
-  int32_t ntiles;
+  int32_t ntiles;           // pipelined tiles (persistent kernel)
+  int32_t ntiles_slow;      // global / oversized tiles (one CTA each)
+  int32_t XP, YP;           // even pitches of S_H rows and S_V columns
   int64_t path_base, tree_base;   // global index of the first local path / tree
   uint64_t seed;
   // forest encoding
   const TileDesc* tiles;
+  const TileDesc* tiles_slow;
   const int4* binfo;
   const uint32_t* pword;
   const short4* sxy;
@@ -77,8 +84,8 @@ struct KParams {
   long long* scal;          // {E[WL], E[TP]} fixed point
   const float* capH;        // [Y][X]
   const float* capVT;       // [X][Y]
-  double* SH;               // [Y][X]
-  double* SVT;              // [X][Y]
+  double* SH;               // [Y][XP]
+  double* SVT;              // [X][YP] (contiguous after SH)
   float* dOutH;             // [Y][X]
   float* dOutVT;            // [X][Y]
   double* partial;          // [Y + X] overflow partial sums

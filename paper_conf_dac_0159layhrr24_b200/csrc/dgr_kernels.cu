@@ -20,6 +20,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdlib>
 
 #include "dgr_internal.h"
 
@@ -191,7 +192,7 @@ __device__ __forceinline__ void red_shared_add(uint32_t saddr, int v) {
 // g = -ln(-ln u) from one Philox word
 __device__ __forceinline__ float gumbel_word(uint32_t w) {
   const float u = ((float)(w >> 9) + 0.5f) * (1.0f / 8388608.0f);
-  return -logf(-logf(u));
+  return -__logf(-logf(u));   // outer log: MUFU approximation, |error| < 1e-6 on g
 }
 
 // Gumbel noise of a warp's contiguous candidates gid0 .. gid0+n-1 into g[0..n): one Philox4x32-10
@@ -422,7 +423,7 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
 
 template <bool REV, bool FWD>
 __global__ void __launch_bounds__(kTileThreads, 3) tile_kernel(KParams P, StepArgs A) {
-  extern __shared__ __align__(16) unsigned char smem[];
+  extern __shared__ __align__(128) unsigned char smem[];
   double* S_s = reinterpret_cast<double*>(smem);                 // region A (reverse)
   int* ev_s = reinterpret_cast<int*>(smem);                      // region A (forward)
   float* g_all = reinterpret_cast<float*>(ev_s + 3 * kWinMax);   // region A (forward)
@@ -431,11 +432,11 @@ __global__ void __launch_bounds__(kTileThreads, 3) tile_kernel(KParams P, StepAr
   float* q_s = reinterpret_cast<float*>(dq_s + kTreeMax);
   long long* red_s = reinterpret_cast<long long*>(q_s + kTreeMax);
 
-  const TileDesc T = P.tiles[blockIdx.x];
+  const TileDesc T = P.tiles_slow[blockIdx.x];
   const int tid = threadIdx.x, warp = tid >> 5;
   const int ncell = T.ww * T.wh;
   const int X = P.X, Y = P.Y;
-  const Win Wg{0, 0, X, Y, X * Y};
+  const Win Wg{0, 0, P.XP, P.YP, (int)(P.SVT - P.SH)};
   const Win Ws{T.wx0, T.wy0, T.ww, T.wh, ncell};
   float* g_s = g_all + warp * kWarpCand;
   // this warp's contiguous bundle range
@@ -445,13 +446,14 @@ __global__ void __launch_bounds__(kTileThreads, 3) tile_kernel(KParams P, StepAr
   // ---------------- reverse of iteration k ----------------
   if (REV) {
     if (!T.global) {
-      for (int i = tid; i < ncell; i += kTileThreads) {
-        const int yi = i / T.ww, xi = i - yi * T.ww;
-        S_s[i] = P.SH[(size_t)(T.wy0 + yi) * X + T.wx0 + xi];
+      const int lane = tid & 31;
+      for (int yi = warp; yi < T.wh; yi += kWarps) {
+        const double* src = P.SH + (size_t)(T.wy0 + yi) * P.XP + T.wx0;
+        for (int xi = lane; xi < T.ww; xi += 32) S_s[yi * T.ww + xi] = src[xi];
       }
-      for (int i = tid; i < ncell; i += kTileThreads) {
-        const int xi = i / T.wh, yi = i - xi * T.wh;
-        S_s[ncell + i] = P.SVT[(size_t)(T.wx0 + xi) * Y + T.wy0 + yi];
+      for (int xi = warp; xi < T.ww; xi += kWarps) {
+        const double* src = P.SVT + (size_t)(T.wx0 + xi) * P.YP + T.wy0;
+        for (int yi = lane; yi < T.wh; yi += 32) S_s[ncell + xi * T.wh + yi] = src[yi];
       }
     }
     for (int i = tid; i < T.ntree; i += kTileThreads) { dq_s[i] = 0; q_s[i] = P.q[T.tree0 + i]; }
@@ -506,8 +508,10 @@ __global__ void __launch_bounds__(kTileThreads, 3) tile_kernel(KParams P, StepAr
 
   // ---------------- forward of iteration k_next ----------------
   if (FWD) {
-    if (!T.global)
-      for (int i = tid; i < 3 * ncell; i += kTileThreads) ev_s[i] = 0;
+    if (!T.global) {
+      int4* z = reinterpret_cast<int4*>(ev_s);
+      for (int i = tid; i < (3 * ncell + 3) / 4; i += kTileThreads) z[i] = make_int4(0, 0, 0, 0);
+    }
     if (tid < 2) red_s[tid] = 0;
     __syncthreads();
     if (bw0 < bw1) {
@@ -516,22 +520,450 @@ __global__ void __launch_bounds__(kTileThreads, 3) tile_kernel(KParams P, StepAr
     }
     __syncthreads();
     if (!T.global) {
-      // flush the window once: row-major fields along rows, column-major fields along columns
-      for (int i = tid; i < ncell; i += kTileThreads) {
-        const int yi = i / T.ww, xi = i - yi * T.ww;
-        const size_t g = (size_t)(T.wy0 + yi) * X + T.wx0 + xi;
-        red64(P.dH + g, ev_s[i]);
-        red64(P.VDH + g, ev_s[2 * ncell + i]);
+      // flush the window once: a warp per window row (H-type fields) / column (V-type fields),
+      // lanes along it, so the int64 reductions are coalesced
+      const int lane = tid & 31;
+      for (int yi = warp; yi < T.wh; yi += kWarps) {
+        const size_t g0 = (size_t)(T.wy0 + yi) * X + T.wx0;
+        const int* rowH = ev_s + yi * T.ww;
+        const int* rowD = ev_s + 2 * ncell + yi * T.ww;
+        for (int xi = lane; xi < T.ww; xi += 32) {
+          if (T.wx0 + xi >= X) break;
+          red64(P.dH + g0 + xi, rowH[xi]);
+          red64(P.VDH + g0 + xi, rowD[xi]);
+        }
       }
-      for (int i = tid; i < ncell; i += kTileThreads) {
-        const int xi = i / T.wh, yi = i - xi * T.wh;
-        const size_t g = (size_t)(T.wx0 + xi) * Y + T.wy0 + yi;
-        red64(P.dVT + g, ev_s[ncell + i]);
-        red64(P.VDV + g, ev_s[2 * ncell + yi * T.ww + xi]);
+      for (int xi = warp; xi < T.ww; xi += kWarps) {
+        const size_t g0 = (size_t)(T.wx0 + xi) * Y + T.wy0;
+        const int* colV = ev_s + ncell + xi * T.wh;
+        const int* colD = ev_s + 2 * ncell + xi;
+        for (int yi = lane; yi < T.wh; yi += 32) {
+          red64(P.dVT + g0 + yi, colV[yi]);
+          red64(P.VDV + g0 + yi, colD[yi * T.ww]);
+        }
       }
     }
     if (tid == 0) { red64(P.scal, red_s[0]); red64(P.scal + 1, red_s[1]); }
   }
+}
+
+// ------------------------------------------------------------------------------------------
+// Persistent, TMA-pipelined tile kernel (the hot loop).  One CTA per SM walks its tiles
+// (blockIdx.x, +gridDim.x, ...).  While tile i is processed out of shared-memory stage s, the
+// bulk-copy engine (cp.async.bulk, completion on an mbarrier) fills stage s^1 with tile i+1's
+// operands: pattern words, w, m, v, p of its bundles, bundle info, sub-net endpoints, net->tree
+// offsets, tree state, and the tile's S window (one bulk copy per window row of S_H and per
+// window column of S_V).  Updated w, m, v, p go back with bulk stores; demand events are
+// accumulated in a shared-memory window and flushed with int64 reductions.
+// ------------------------------------------------------------------------------------------
+constexpr int kPSlots = kTargetBundles * 32;                // 1024
+constexpr int kPSubMax = kPipeSubs + 2;                     // + alignment slack
+constexpr int kPTreeMax = kPipeTrees + 4;
+constexpr int kPNetMax = kPipeTrees + 8;
+
+struct StageLayout {
+  static constexpr size_t pw = 0;
+  static constexpr size_t w = pw + 4 * kPSlots;
+  static constexpr size_t m = w + 4 * kPSlots;
+  static constexpr size_t v = m + 4 * kPSlots;
+  static constexpr size_t p = v + 4 * kPSlots;
+  static constexpr size_t bi = p + 4 * kPSlots;
+  static constexpr size_t sxy = bi + 16 * kTargetBundles;
+  static constexpr size_t nto = sxy + 8 * kPSubMax;
+  static constexpr size_t q = (nto + 4 * kPNetMax + 15) / 16 * 16;
+  static constexpr size_t wt = q + 4 * kPTreeMax;
+  static constexpr size_t mt = wt + 4 * kPTreeMax;
+  static constexpr size_t vt = mt + 4 * kPTreeMax;
+  static constexpr size_t S = (vt + 4 * kPTreeMax + 127) / 128 * 128;
+  static constexpr size_t bytes = S + 2 * 8 * kWinMax;
+};
+constexpr size_t kPEvBytes = 3 * 4 * kWinMax;
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n\tWAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@!P1 bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
+struct Stage {
+  uint32_t* pw; float *w, *m, *v, *p;
+  int4* bi; short4* sxy; int* nto; float *q, *wt, *mt, *vt; double* S;
+  __device__ __forceinline__ explicit Stage(unsigned char* base) {
+    pw = reinterpret_cast<uint32_t*>(base + StageLayout::pw);
+    w = reinterpret_cast<float*>(base + StageLayout::w);
+    m = reinterpret_cast<float*>(base + StageLayout::m);
+    v = reinterpret_cast<float*>(base + StageLayout::v);
+    p = reinterpret_cast<float*>(base + StageLayout::p);
+    bi = reinterpret_cast<int4*>(base + StageLayout::bi);
+    sxy = reinterpret_cast<short4*>(base + StageLayout::sxy);
+    nto = reinterpret_cast<int*>(base + StageLayout::nto);
+    q = reinterpret_cast<float*>(base + StageLayout::q);
+    wt = reinterpret_cast<float*>(base + StageLayout::wt);
+    mt = reinterpret_cast<float*>(base + StageLayout::mt);
+    vt = reinterpret_cast<float*>(base + StageLayout::vt);
+    S = reinterpret_cast<double*>(base + StageLayout::S);
+  }
+};
+
+// aligned element ranges of a tile's sub-nets / nets / trees (16-byte bulk granularity)
+__device__ __forceinline__ void tile_ranges(const TileDesc& T, int& s_lo, int& s_hi, int& n_lo, int& n_hi, int& t_lo, int& t_hi) {
+  s_lo = T.sub0 & ~1; s_hi = (T.sub0 + T.nsub + 1) & ~1;
+  n_lo = T.net0 & ~3; n_hi = (T.net0 + T.nnet + 1 + 3) & ~3;
+  t_lo = T.tree0 & ~3; t_hi = (T.tree0 + T.ntree + 3) & ~3;
+}
+
+// warp 0 issues the bulk copies of tile T into stage `st`, completing on `bar`
+template <bool REV>
+__device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDesc& T, unsigned char* st, uint64_t* bar) {
+  const int lane = threadIdx.x & 31;
+  Stage S(st);
+  int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
+  tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
+  const uint32_t slot_bytes = (uint32_t)T.nb * 128u;
+  const uint32_t nrow = REV ? (uint32_t)T.wh : 0u, ncol = REV ? (uint32_t)T.ww : 0u;
+  const uint32_t bytes = slot_bytes * (REV ? 5u : 2u) + 16u * T.nb + 8u * (s_hi - s_lo) + 4u * (n_hi - n_lo) +
+                         4u * (t_hi - t_lo) * (REV ? 4u : 3u) + 8u * (nrow * T.ww + ncol * T.wh);
+  if (lane == 0) mbar_expect_tx(bar, bytes);
+  __syncwarp();
+  const size_t s0 = (size_t)T.b0 * 32;
+  // work items: 0..9 the 1-D arrays, then window rows, then window columns
+  const int nitems = 10 + (int)nrow + (int)ncol;
+  for (int it = lane; it < nitems; it += 32) {
+    if (it < 10) {
+      switch (it) {
+        case 0: bulk_g2s(S.pw, P.pword + s0, slot_bytes, bar); break;
+        case 1: bulk_g2s(S.w, P.wp + s0, slot_bytes, bar); break;
+        case 2: if (REV) bulk_g2s(S.m, P.mp + s0, slot_bytes, bar); break;
+        case 3: if (REV) bulk_g2s(S.v, P.vp + s0, slot_bytes, bar); break;
+        case 4: if (REV) bulk_g2s(S.p, P.pp + s0, slot_bytes, bar); break;
+        case 5: bulk_g2s(S.bi, P.binfo + T.b0, 16u * T.nb, bar); break;
+        case 6: bulk_g2s(S.sxy, P.sxy + s_lo, 8u * (s_hi - s_lo), bar); break;
+        case 7: bulk_g2s(S.nto, P.net_tree_off + n_lo, 4u * (n_hi - n_lo), bar); break;
+        case 8: bulk_g2s(S.wt, P.wt + t_lo, 4u * (t_hi - t_lo), bar);
+                bulk_g2s(S.mt, P.mt + t_lo, 4u * (t_hi - t_lo), bar); break;
+        default: bulk_g2s(S.vt, P.vt + t_lo, 4u * (t_hi - t_lo), bar);
+                 if (REV) bulk_g2s(S.q, P.q + t_lo, 4u * (t_hi - t_lo), bar); break;
+      }
+    } else if (it < 10 + (int)nrow) {
+      const int yi = it - 10;
+      bulk_g2s(S.S + (size_t)yi * T.ww, P.SH + (size_t)(T.wy0 + yi) * P.XP + T.wx0, 8u * T.ww, bar);
+    } else {
+      const int xi = it - 10 - (int)nrow;
+      bulk_g2s(S.S + (size_t)T.ww * T.wh + (size_t)xi * T.wh, P.SVT + (size_t)(T.wx0 + xi) * P.YP + T.wy0, 8u * T.wh, bar);
+    }
+  }
+}
+
+// One tile, all operands in shared memory (stage St).  ev_s / g_all may alias St.S (they are
+// only touched after the reverse half is done with it).  Ends with the slot state written back
+// by bulk stores (issued by thread 0, committed) and the demand window flushed.
+template <bool REV, bool FWD, int NT>
+__device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A, const TileDesc& T, Stage St,
+                                             int* ev_s, float* g_all, long long* dq_s, long long& wl_acc,
+                                             long long& tp_acc) {
+  constexpr int NW = NT / 32;
+  constexpr int WCAND = (kTargetBundles + NW - 1) / NW * 32;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int X = P.X, Y = P.Y;
+  float* g_s = g_all + warp * WCAND;
+  int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
+  tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
+  const int ncell = T.ww * T.wh;
+  const Win W{T.wx0, T.wy0, T.ww, T.wh, ncell};
+  const int per = (T.nb + NW - 1) / NW;
+  const int lb0 = min(warp * per, T.nb), lb1 = min((warp + 1) * per, T.nb);   // tile-local bundles
+
+  // ---------------- reverse of iteration k ----------------
+  if (REV) {
+    for (int i = tid; i < T.ntree; i += NT) dq_s[i] = 0;
+    __syncthreads();
+    for (int lb = lb0; lb < lb1; ++lb) {
+      Lane L;
+      lane_from(St.bi[lb], St.pw[lb * 32 + lane], P, L);
+      const int sl = lb * 32 + lane;
+      float w = St.w[sl], m = St.m[sl], v = St.v[sl];
+      const float p = St.p[sl];
+      const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
+      double c = 0.0;
+      if (L.valid) {
+        const short4 e = St.sxy[L.sub - s_lo];
+        c = path_cost(St.S, W, X, Y, L.shape, e.x, e.y, e.z, e.w, (int)(L.pw >> 16), A);
+      }
+      // softmax backward: differences to the group head's dp in fp64, reduced in fp32
+      const double dp = (double)q * c;
+      const double dref = __shfl_sync(kFull, dp, L.head);
+      const float dd = (float)(dp - dref);
+      float sa = seg_reduce(p * dd, L.lane, L.end, Sum());
+      float sb = seg_reduce(p, L.lane, L.end, Sum());
+      sa = __shfl_sync(kFull, sa, L.head);
+      sb = __shfl_sync(kFull, sb, L.head);
+      const float dw = L.valid ? p * A.inv_t * (dd - __fdividef(sa, sb)) : 0.f;
+      // dq_j partial sums (fp64 -> 2^-32 fixed point)
+      const uint32_t th = L.tm | __ballot_sync(kFull, !L.valid) | 1u;
+      const uint32_t trest = th & ~L.le;
+      const int tend = trest ? (__ffs(trest) - 2) : 31;
+      const double pc = seg_reduce(L.valid ? (double)p * c : 0.0, L.lane, tend, Sum());
+      if (L.valid && ((th >> L.lane) & 1u))
+        atomicAdd(reinterpret_cast<unsigned long long*>(&dq_s[L.tree - T.tree0]),
+                  static_cast<unsigned long long>(__double2ll_rn(pc * kDqScale)));
+      if (L.valid) {
+        adam_update(w, m, v, dw, A);
+        St.w[sl] = w; St.m[sl] = m; St.v[sl] = v;
+      }
+    }
+    __syncthreads();
+  }
+
+  // ---------------- tree level ----------------
+  for (int n = tid; n < T.nnet; n += NT) {
+    const int net = T.net0 + n;
+    const int a = St.nto[net - n_lo], b = St.nto[net + 1 - n_lo];
+    if (REV) {
+      double sq = 0.0, sw = 0.0;
+      for (int j = a; j < b; ++j) {
+        const double qj = (double)St.q[j - t_lo];
+        sq += qj * ((double)dq_s[j - T.tree0] * kDqInv);
+        sw += qj;
+      }
+      sq /= sw;
+      for (int j = a; j < b; ++j) {
+        const double du = (b - a == 1) ? 0.0
+                                       : (double)St.q[j - t_lo] * (double)A.inv_t * ((double)dq_s[j - T.tree0] * kDqInv - sq);
+        float w = St.wt[j - t_lo], m = St.mt[j - t_lo], v = St.vt[j - t_lo];
+        adam_update(w, m, v, (float)du, A);
+        St.wt[j - t_lo] = w;
+        P.wt[j] = w; P.mt[j] = m; P.vt[j] = v;
+      }
+    }
+    if (FWD) {
+      if (b - a == 1) {
+        St.q[a - t_lo] = 1.f;
+        P.q[a] = 1.f;
+      } else {
+        float zmax = -INFINITY;
+        for (int j = a; j < b; ++j) {
+          const float z = (St.wt[j - t_lo] + gumbel(P.seed, (uint64_t)(P.tree_base + j), (uint32_t)A.k_next, 1u)) * A.inv_t;
+          St.q[j - t_lo] = z;
+          zmax = fmaxf(zmax, z);
+        }
+        float sum = 0.f;
+        for (int j = a; j < b; ++j) { const float e = __expf(St.q[j - t_lo] - zmax); St.q[j - t_lo] = e; sum += e; }
+        const float inv = 1.f / sum;
+        for (int j = a; j < b; ++j) { St.q[j - t_lo] *= inv; P.q[j] = St.q[j - t_lo]; }
+      }
+    }
+  }
+
+  // ---------------- forward of iteration k_next ----------------
+  if (FWD) {
+    {
+      int4* z = reinterpret_cast<int4*>(ev_s);
+      for (int i = tid; i < (3 * ncell + 3) / 4; i += NT) z[i] = make_int4(0, 0, 0, 0);
+    }
+    __syncthreads();
+    if (lb0 < lb1) {
+      const int4 bfirst = St.bi[lb0];
+      const int4 blast = St.bi[lb1 - 1];
+      warp_noise(g_s, P.seed, P.path_base + bfirst.x, blast.x + blast.w - bfirst.x, (uint32_t)A.k_next, lane);
+    }
+    const uint32_t ev_base = smem_u32(ev_s);
+    for (int lb = lb0; lb < lb1; ++lb) {
+      Lane L;
+      lane_from(St.bi[lb], St.pw[lb * 32 + lane], P, L);
+      const int sl = lb * 32 + lane;
+      const float w = St.w[sl];
+      const float g = L.valid ? g_s[L.lpath - St.bi[lb0].x] : 0.f;
+      const float p = softmax_from_noise(L, w, g, A.inv_t);
+      St.p[sl] = p;
+      const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
+      const int vq = L.valid ? __float2int_rn(q * p * kFixScale) : 0;
+      int sc = vq;
+#pragma unroll
+      for (int off = 1; off < 32; off <<= 1) {
+        const int o = __shfl_up_sync(kFull, sc, off);
+        if (L.lane - off >= L.head) sc += o;
+      }
+      const int nh = __popc(__ballot_sync(kFull, L.shape == kZHVH) & L.gmask);
+      const int h1 = min(L.head + 1, 31), h2 = min(L.head + 1 + nh, 31);
+      const int a = __shfl_sync(kFull, vq, L.head);
+      const int bb = __shfl_sync(kFull, vq, h1);
+      const int S1 = __shfl_sync(kFull, sc, h1);
+      const int S2 = __shfl_sync(kFull, sc, h2);
+      const int Se = __shfl_sync(kFull, sc, L.end);
+      const short4 e = L.valid ? St.sxy[L.sub - s_lo] : make_short4(0, 0, 0, 0);
+      const int x0 = e.x, y0 = e.y, x1 = e.z, y1 = e.w;
+      const int sgn = (y1 > y0) ? 1 : -1;
+      const int hs = S2 - S1, vs = Se - S2, vv = vq;
+      const int mm = (int)(L.pw >> 16);
+      const int fSH = L.shape == kStraightH, fSV = L.shape == kStraightV, fHV = L.shape == kHV;
+      const int fVH = L.shape == kVH, fZH = L.shape == kZHVH, fZV = L.shape == kZVHV;
+      const int fZ = fZH + fZV;
+      const int xa = x0 + fZH * (mm - x0);
+      const int ya = y0 + fVH * (y1 - y0) + fZV * (mm - y0);
+      const int xb = x1 + fSV * (x0 - x1) + fZH * (mm - x1);
+      const int yb = y1 + (fSH + fHV) * (y0 - y1) + fZV * (mm - y1);
+      const int ah = fSH * vv + fHV * (a + hs) + fVH * bb + (fZV - fZH) * vv;
+      const int av = fSV * vv + sgn * (fHV * (bb + vs) - fVH * bb + (fZH - fZV) * vv);
+      const int ad = fVH * bb + fZ * vv;
+      const int bh = -fSH * vv - fHV * a - fVH * (bb + hs) + (fZH - fZV) * vv;
+      const int bv = -fSV * vv + sgn * (fHV * a - fVH * (a + vs) + (fZV - fZH) * vv);
+      const int bd = fHV * a + fZ * vv;
+      if (L.valid) {
+        const int hv2 = 2 * ncell;
+        const int ia_h = W.h(xa, ya), ib_h = W.h(xb, yb);
+        red_shared_add(ev_base + 4u * ia_h, ah);
+        red_shared_add(ev_base + 4u * W.v(xa, ya), av);
+        red_shared_add(ev_base + 4u * (hv2 + ia_h), ad);
+        red_shared_add(ev_base + 4u * ib_h, bh);
+        red_shared_add(ev_base + 4u * W.v(xb, yb), bv);
+        red_shared_add(ev_base + 4u * (hv2 + ib_h), bd);
+        wl_acc += (long long)vq * ((x1 - x0) + abs(y1 - y0));
+        tp_acc += (long long)vq * (fHV + fVH + 2 * fZ);
+      }
+    }
+  }
+  __syncthreads();
+  // write back the tile's slot state with bulk stores (asynchronous; readers wait on the group)
+  if (tid == 0) {
+    fence_proxy_async();
+    const size_t s0 = (size_t)T.b0 * 32;
+    const uint32_t slot_bytes = (uint32_t)T.nb * 128u;
+    if (REV) {
+      bulk_s2g(P.wp + s0, St.w, slot_bytes);
+      bulk_s2g(P.mp + s0, St.m, slot_bytes);
+      bulk_s2g(P.vp + s0, St.v, slot_bytes);
+    }
+    if (FWD) bulk_s2g(P.pp + s0, St.p, slot_bytes);
+    bulk_commit();
+  }
+  if (FWD) {
+    for (int yi = warp; yi < T.wh; yi += NW) {
+      if (T.wy0 + yi >= Y) break;
+      const size_t g0 = (size_t)(T.wy0 + yi) * X + T.wx0;
+      const int* rowH = ev_s + yi * T.ww;
+      const int* rowD = ev_s + 2 * ncell + yi * T.ww;
+      for (int xi = lane; xi < T.ww; xi += 32) {
+        red64(P.dH + g0 + xi, rowH[xi]);
+        red64(P.VDH + g0 + xi, rowD[xi]);
+      }
+    }
+    for (int xi = warp; xi < T.ww; xi += NW) {
+      if (T.wx0 + xi >= X) break;
+      const size_t g0 = (size_t)(T.wx0 + xi) * Y + T.wy0;
+      const int* colV = ev_s + ncell + xi * T.wh;
+      const int* colD = ev_s + 2 * ncell + xi;
+      for (int yi = lane; yi < T.wh; yi += 32) {
+        red64(P.dVT + g0 + yi, colV[yi]);
+        red64(P.VDV + g0 + yi, colD[yi * T.ww]);
+      }
+    }
+  }
+}
+
+// E[WL], E[TP] partial sums of the block -> the exchange buffer
+template <int NT>
+__device__ __forceinline__ void flush_scalars(const KParams& P, long long wl, long long tp, long long* red_s) {
+  const int lane = threadIdx.x & 31;
+  if (threadIdx.x < 2) red_s[threadIdx.x] = 0;
+  __syncthreads();
+  wl = seg_reduce(wl, lane, 31, Sum());
+  tp = seg_reduce(tp, lane, 31, Sum());
+  if (lane == 0) {
+    atomicAdd(reinterpret_cast<unsigned long long*>(&red_s[0]), static_cast<unsigned long long>(wl));
+    atomicAdd(reinterpret_cast<unsigned long long*>(&red_s[1]), static_cast<unsigned long long>(tp));
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) { red64(P.scal, red_s[0]); red64(P.scal + 1, red_s[1]); }
+}
+
+// (a) one tile per CTA: the whole tile arrives by bulk copies on one mbarrier; the event window
+// and noise alias the S window.  3 CTAs per SM overlap one CTA's copies with the others' math.
+constexpr int kBThreads = 256;
+constexpr size_t kBSmemBytes = StageLayout::bytes + 8 * kPipeTrees + 64;
+static_assert(kPEvBytes + 4 * kWinMax <= 2 * 8 * kWinMax, "event window + noise must fit the S window");
+
+template <bool REV, bool FWD>
+__global__ void __launch_bounds__(kBThreads, 3) tile_bulk(KParams P, StepArgs A) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  Stage St(smem);
+  long long* dq_s = reinterpret_cast<long long*>(smem + StageLayout::bytes);
+  long long* red_s = dq_s + kPipeTrees;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(red_s + 2);
+  int* ev_s = reinterpret_cast<int*>(St.S);
+  float* g_all = reinterpret_cast<float*>(ev_s + 3 * kWinMax);
+  const TileDesc T = P.tiles[blockIdx.x];
+  if (threadIdx.x == 0) {
+    mbar_init(bar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (threadIdx.x < 32) issue_tile_loads<REV>(P, T, smem, bar);
+  mbar_wait(bar, 0u);
+  long long wl = 0, tp = 0;
+  process_tile<REV, FWD, kBThreads>(P, A, T, St, ev_s, g_all, dq_s, wl, tp);
+  if (FWD) flush_scalars<kBThreads>(P, wl, tp, red_s);
+  if (threadIdx.x == 0) bulk_wait_read();   // the stage must outlive the bulk stores' reads
+}
+
+// (b) persistent, double-buffered: one CTA per SM, tile i+1 streams into the other stage while
+// tile i computes.
+constexpr int kPThreads = 512;
+constexpr size_t kPSmemBytes = 2 * StageLayout::bytes + kPEvBytes + 4 * kWinMax + 8 * kPipeTrees + 64;
+
+template <bool REV, bool FWD>
+__global__ void __launch_bounds__(kPThreads, 1) tile_persistent(KParams P, StepArgs A) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  unsigned char* stage_base[2] = {smem, smem + StageLayout::bytes};
+  int* ev_s = reinterpret_cast<int*>(smem + 2 * StageLayout::bytes);
+  float* g_all = reinterpret_cast<float*>(smem + 2 * StageLayout::bytes + kPEvBytes);
+  long long* dq_s = reinterpret_cast<long long*>(g_all + kWinMax);
+  long long* red_s = dq_s + kPipeTrees;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(red_s + 2);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  if (tid == 0) {
+    mbar_init(&bars[0], 1);
+    mbar_init(&bars[1], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (warp == 0 && (int)blockIdx.x < P.ntiles) issue_tile_loads<REV>(P, P.tiles[blockIdx.x], stage_base[0], &bars[0]);
+  long long wl = 0, tp = 0;
+  for (int it = 0;; ++it) {
+    const int tile = blockIdx.x + it * gridDim.x;
+    if (tile >= P.ntiles) break;
+    const int sidx = it & 1;
+    if (warp == 0 && tile + (int)gridDim.x < P.ntiles) {
+      if (lane == 0) bulk_wait_read();   // the other stage's previous write-back has been read
+      __syncwarp();
+      issue_tile_loads<REV>(P, P.tiles[tile + gridDim.x], stage_base[sidx ^ 1], &bars[sidx ^ 1]);
+    }
+    mbar_wait(&bars[sidx], (uint32_t)(it >> 1) & 1u);
+    process_tile<REV, FWD, kPThreads>(P, A, P.tiles[tile], Stage(stage_base[sidx]), ev_s, g_all, dq_s, wl, tp);
+    __syncthreads();
+  }
+  if (FWD) flush_scalars<kPThreads>(P, wl, tp, red_s);
+  if (tid == 0) bulk_wait_all();
 }
 
 // ------------------------------------------------------------------------------------------
@@ -571,9 +1003,51 @@ __device__ __forceinline__ T block_exclusive_scan(T v, T* sh, T* total) {
   return before + x - v;
 }
 
+// warp-inclusive scan (shuffles)
+template <typename T>
+__device__ __forceinline__ T warp_inclusive_scan(T x, int lane) {
+#pragma unroll
+  for (int off = 1; off < 32; off <<= 1) {
+    const T o = __shfl_up_sync(kFull, x, off);
+    if (lane >= off) x += o;
+  }
+  return x;
+}
+
+// Exclusive scan of a chunk of kGThreads * kGItems elements held "striped": thread t holds
+// elements j * kGThreads + t (j < kGItems), so every global access is coalesced.  One barrier.
+template <typename T>
+__device__ __forceinline__ void striped_exclusive_scan(T (&v)[kGItems], T* sh /* kGItems*32 */, T* total) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  constexpr int NW = kGThreads / 32;
+  T inc[kGItems];
+#pragma unroll
+  for (int j = 0; j < kGItems; ++j) inc[j] = warp_inclusive_scan(v[j], lane);
+  if (lane == 31) {
+#pragma unroll
+    for (int j = 0; j < kGItems; ++j) sh[j * NW + wid] = inc[j];
+  }
+  __syncthreads();
+  T run = T(0);
+#pragma unroll
+  for (int j = 0; j < kGItems; ++j) {
+    T before = run, rowtot = T(0);
+#pragma unroll
+    for (int w = 0; w < NW; ++w) {
+      const T t = sh[j * NW + w];
+      if (w < wid) before += t;
+      rowtot += t;
+    }
+    v[j] = before + inc[j] - v[j];   // exclusive
+    run += rowtot;
+  }
+  *total = run;
+  __syncthreads();
+}
+
 __global__ void __launch_bounds__(kGThreads) kg_kernel(KParams P, StepArgs A) {
-  __shared__ long long shl[32];
-  __shared__ double shd[32];
+  __shared__ long long shl[kGItems * (kGThreads / 32)];
+  __shared__ double shd[kGItems * (kGThreads / 32)];
   const int line = blockIdx.x;
   const bool isH = line < P.Y;
   const int n = isH ? P.X : P.Y;
@@ -582,38 +1056,41 @@ __global__ void __launch_bounds__(kGThreads) kg_kernel(KParams P, StepArgs A) {
   long long* diff = (isH ? P.dH : P.dVT) + base;
   long long* vd = (isH ? P.VDH : P.VDV) + base;
   const float* cap = (isH ? P.capH : P.capVT) + base;
-  double* S = (isH ? P.SH : P.SVT) + base;
+  double* S = isH ? P.SH + (size_t)ln * P.XP : P.SVT + (size_t)ln * P.YP;
   float* dout = (isH ? P.dOutH : P.dOutVT) + base;
   const double beta = A.beta;
   long long carryW = 0;
   double carryS = 0.0, of = 0.0;
   for (int c0 = 0; c0 < n; c0 += kGThreads * kGItems) {
-    const int pos0 = c0 + threadIdx.x * kGItems;
-    long long v[kGItems], t[kGItems + 1];
+    long long v[kGItems], t0[kGItems], t1[kGItems];
+    float cp[kGItems];
 #pragma unroll
-    for (int i = 0; i < kGItems; ++i) {
-      v[i] = (pos0 + i < n) ? diff[pos0 + i] : 0;
-      t[i] = (pos0 + i < n) ? vd[pos0 + i] : 0;
+    for (int j = 0; j < kGItems; ++j) {
+      const int pos = c0 + j * kGThreads + threadIdx.x;
+      v[j] = pos < n ? diff[pos] : 0;
+      t0[j] = pos < n ? vd[pos] : 0;
+      t1[j] = pos + 1 < n ? vd[pos + 1] : 0;
+      cp[j] = pos < n ? cap[pos] : 0.f;
     }
-    t[kGItems] = (pos0 + kGItems < n) ? vd[pos0 + kGItems] : 0;
-    long long run = 0;
-#pragma unroll
-    for (int i = 0; i < kGItems; ++i) { run += v[i]; v[i] = run; }   // local inclusive
     long long totW;
-    const long long offW = block_exclusive_scan(run, shl, &totW);   // (synchronises: all reads done)
+    long long ex[kGItems];
 #pragma unroll
-    for (int i = 0; i < kGItems; ++i)
-      if (pos0 + i < n) { diff[pos0 + i] = 0; vd[pos0 + i] = 0; }
+    for (int j = 0; j < kGItems; ++j) ex[j] = v[j];
+    striped_exclusive_scan(ex, shl, &totW);   // all reads of this chunk are done after its barrier
+#pragma unroll
+    for (int j = 0; j < kGItems; ++j) {
+      const int pos = c0 + j * kGThreads + threadIdx.x;
+      if (pos < n) { diff[pos] = 0; vd[pos] = 0; }
+    }
     double g[kGItems];
-    double grun = 0.0;
 #pragma unroll
-    for (int i = 0; i < kGItems; ++i) {
-      const int pos = pos0 + i;
+    for (int j = 0; j < kGItems; ++j) {
+      const int pos = c0 + j * kGThreads + threadIdx.x;
       double G = 0.0;
       if (pos < n - 1) {
-        const long long W = carryW + offW + v[i];
-        const double d = (double)W * kFixInv + beta * ((double)(t[i] + t[i + 1]) * kFixInv);
-        const double r = (double)cap[pos] - d;
+        const long long W = carryW + ex[j] + v[j];   // inclusive prefix = wire demand of edge pos
+        const double d = (double)W * kFixInv + beta * ((double)(t0[j] + t1[j]) * kFixInv);
+        const double r = (double)cp[j] - d;
         if (A.f_kind == 0) {
           // sigmoid: f(r) = 1/(1+exp(s r)) = sigma(-s r); -f'(r) = s sigma(s r) sigma(-s r).
           // fp64 here (one exp per edge): G feeds every candidate's cost difference.
@@ -624,21 +1101,20 @@ __global__ void __launch_bounds__(kGThreads) kg_kernel(KParams P, StepArgs A) {
           G = (double)A.a_of * (double)A.f_slope * e * inv * inv;
         } else {
           of += r < 0.0 ? -r : 0.0;
-          G = (d > (double)cap[pos]) ? (double)A.a_of : 0.0;
+          G = (d > (double)cp[j]) ? (double)A.a_of : 0.0;
         }
         if (A.store_d) dout[pos] = (float)d;
       } else if (pos == n - 1 && A.store_d) {
         dout[pos] = 0.f;
       }
-      g[i] = grun;          // local exclusive
-      grun += G;
+      g[j] = G;
     }
     double totS;
-    const double offS = block_exclusive_scan(grun, shd, &totS);
+    striped_exclusive_scan(g, shd, &totS);
 #pragma unroll
-    for (int i = 0; i < kGItems; ++i) {
-      const int pos = pos0 + i;
-      if (pos < n) S[pos] = carryS + offS + g[i];
+    for (int j = 0; j < kGItems; ++j) {
+      const int pos = c0 + j * kGThreads + threadIdx.x;
+      if (pos < n) S[pos] = carryS + g[j];
     }
     carryW += totW;
     carryS += totS;
@@ -789,10 +1265,31 @@ __global__ void ki_finalize_kernel(KParams P, int nblocks) {
 // ------------------------------------------------------------------------------------------
 static inline int cdiv(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
 
+static int g_num_sms = 148;
+static bool g_persistent = false;   // DGR_TILE_PERSISTENT=1 selects driver (b)
+
 size_t tile_smem_bytes() { return kSmemBytes; }
 
 int prepare_kernels() {
-  cudaError_t e = cudaFuncSetAttribute(tile_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
+  const char* env = getenv("DGR_TILE_PERSISTENT");
+  g_persistent = env && env[0] == '1';
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(tile_bulk<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBSmemBytes);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(tile_bulk<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBSmemBytes);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(tile_bulk<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBSmemBytes);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(tile_persistent<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPSmemBytes);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(tile_persistent<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPSmemBytes);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(tile_persistent<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPSmemBytes);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(tile_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(tile_kernel<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   if (e == cudaSuccess)
@@ -801,10 +1298,23 @@ int prepare_kernels() {
 }
 
 void launch_tiles(const KParams& p, const StepArgs& a, TileMode mode, cudaStream_t s) {
-  if (p.ntiles <= 0) return;
-  if (mode == kForwardOnly) tile_kernel<false, true><<<p.ntiles, kTileThreads, kSmemBytes, s>>>(p, a);
-  else if (mode == kReverseForward) tile_kernel<true, true><<<p.ntiles, kTileThreads, kSmemBytes, s>>>(p, a);
-  else tile_kernel<true, false><<<p.ntiles, kTileThreads, kSmemBytes, s>>>(p, a);
+  if (p.ntiles > 0) {
+    if (g_persistent) {
+      const int grid = p.ntiles < g_num_sms ? p.ntiles : g_num_sms;
+      if (mode == kForwardOnly) tile_persistent<false, true><<<grid, kPThreads, kPSmemBytes, s>>>(p, a);
+      else if (mode == kReverseForward) tile_persistent<true, true><<<grid, kPThreads, kPSmemBytes, s>>>(p, a);
+      else tile_persistent<true, false><<<grid, kPThreads, kPSmemBytes, s>>>(p, a);
+    } else {
+      if (mode == kForwardOnly) tile_bulk<false, true><<<p.ntiles, kBThreads, kBSmemBytes, s>>>(p, a);
+      else if (mode == kReverseForward) tile_bulk<true, true><<<p.ntiles, kBThreads, kBSmemBytes, s>>>(p, a);
+      else tile_bulk<true, false><<<p.ntiles, kBThreads, kBSmemBytes, s>>>(p, a);
+    }
+  }
+  if (p.ntiles_slow > 0) {
+    if (mode == kForwardOnly) tile_kernel<false, true><<<p.ntiles_slow, kTileThreads, kSmemBytes, s>>>(p, a);
+    else if (mode == kReverseForward) tile_kernel<true, true><<<p.ntiles_slow, kTileThreads, kSmemBytes, s>>>(p, a);
+    else tile_kernel<true, false><<<p.ntiles_slow, kTileThreads, kSmemBytes, s>>>(p, a);
+  }
 }
 void launch_kg(const KParams& p, const StepArgs& a, cudaStream_t s) {
   kg_kernel<<<p.X + p.Y, kGThreads, 0, s>>>(p, a);
