@@ -287,6 +287,7 @@ def main():
     quality = None if args.no_quality else paper_schedule_quality(s, W)
 
     cells = f.X * f.Y
+    slow = 1 if info["n_tiles"] > info.get("n_pipe_tiles", info["n_tiles"]) else 0
     st = dict(paths=f.n_paths, subnets=f.n_subnets, trees=f.n_trees, nets=f.n_nets, bundles=info["n_bundles"],
               cells=cells)
     if world > 1:   # this rank's share of the per-candidate work
@@ -329,7 +330,7 @@ def main():
                      "share_of_step": stage_ms[dom] / sum(stage_ms.values())},
         "stage_ms_per_launch": per_launch_ms,
         "stage_launches": n_prof,
-        "gpu_launches": 3 * args.steps + 1,
+        "gpu_launches": (1 + slow) + args.steps * (3 + slow),
         "clocks": clocks,
         "induce_ms": induce_ms,
         "loss": {"total": float(loss[0]), "wl": float(loss[1]), "via": float(loss[2]), "overflow": float(loss[3])},

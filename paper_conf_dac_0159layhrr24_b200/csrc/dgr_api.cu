@@ -13,6 +13,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -426,7 +427,7 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.mt = take(4 * nt + 16);
   L.vt = take(4 * nt + 16);
   L.q = take(4 * nt + 16);
-  L.xcount = 4 * G + 2;   // dH | dV^T | VD (row-major) | VD (column-major) | E[WL], E[TP]
+  L.xcount = 3 * G + 2;   // dH | dV^T | VD | E[WL], E[TP]
   L.xbuf = take(8 * L.xcount);
   L.capH = take(4 * G);
   L.capVT = take(4 * G);
@@ -571,6 +572,7 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
   P.ntiles_slow = (int32_t)(pl.tiles.size() - pl.n_pipe_tiles);
   P.tiles_slow = P.tiles + pl.n_pipe_tiles;
   P.XP = desc->X + (desc->X & 1);
+  if (const char* sk = getenv("DGR_DEBUG_SKIP")) P.skip = atoi(sk);   // timing experiments only
   P.YP = desc->Y + (desc->Y & 1);
   P.n_nets_l = (int32_t)(pl.net_hi - pl.net_lo);
   P.path_base = pl.path_lo;
@@ -586,9 +588,8 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
   const size_t G = (size_t)desc->X * desc->Y;
   P.dH = (long long*)(ws + L.xbuf);
   P.dVT = P.dH + G;
-  P.VDH = P.dVT + G;
-  P.VDV = P.VDH + G;
-  P.scal = P.VDV + G;
+  P.VD = P.dVT + G;
+  P.scal = P.VD + G;
   P.capH = (const float*)(ws + L.capH);
   P.capVT = (const float*)(ws + L.capVT);
   P.SH = (double*)(ws + L.SH); P.SVT = (double*)(ws + L.SVT);
@@ -673,6 +674,8 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
   a.store_d = 0;
   adam_args(h->k);
   if ((rc = prof_mark(h, -1))) return rc;
+  const size_t vd_bytes = 8 * (size_t)h->X * h->Y;
+  CUDA_TRY(cudaMemsetAsync(P.VD, 0, vd_bytes, s));   // KG clears dH / dV^T in place; VD here
   launch_tiles(P, a, kForwardOnly, s);
   if ((rc = prof_mark(h, 0))) return rc;
   const int n = iters == 0 ? 1 : iters;
@@ -690,6 +693,7 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
     if ((rc = prof_mark(h, 2))) return rc;
     if (iters > 0) {
       // reverse of iteration k + (unless last) forward of k+1
+      if (!last) CUDA_TRY(cudaMemsetAsync(P.VD, 0, vd_bytes, s));
       launch_tiles(P, a, last ? kReverseOnly : kReverseForward, s);
       h->k += 1;
     }

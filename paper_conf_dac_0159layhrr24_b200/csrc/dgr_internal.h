@@ -17,7 +17,7 @@
 //   * per tree:    w, m, v, q (fp32)
 //   * grids: difference arrays of the wire demand along H rows ([Y][X]) and along V columns
 //     (stored transposed, [X][Y], so both scans run over contiguous lines), the turning-point
-//     ("via") demand per G-cell in both layouts, all int64 in 2^-24 fixed point; prefix sums S of
+//     ("via") demand per G-cell ([Y][X]), all int64 in 2^-24 fixed point; prefix sums S of
 //     the overflow gradient per line (fp64, the same two layouts).
 #pragma once
 #include <cstdint>
@@ -31,12 +31,12 @@ constexpr double kDqScale = 4294967296.0;          // dq_j accumulated in 2^-32 
 constexpr double kDqInv = 1.0 / 4294967296.0;
 
 constexpr int kTileThreads = 256;                  // 8 warps per tile CTA
-constexpr int kWinMax = 2048;                      // window cells per tile
+constexpr int kWinMax = 1536;                      // window cells per tile
 constexpr int kMaxBundles = 64;                    // bundles per tile (a whole net always fits)
-constexpr int kTargetBundles = 32;                 // planner target per tile
+constexpr int kTargetBundles = 28;                 // planner target per tile
 constexpr int kTreeMax = 512;                      // trees per tile
-constexpr int kPipeTrees = 256;                    // trees per pipelined tile
-constexpr int kPipeSubs = 512;                     // sub-nets per pipelined tile
+constexpr int kPipeTrees = 224;                    // trees per pipelined tile
+constexpr int kPipeSubs = 448;                     // sub-nets per pipelined tile
 constexpr int kEventMax = 127;                     // events per window cell-field (int32 safety)
 
 enum Shape : uint32_t {
@@ -64,6 +64,7 @@ struct KParams {
   int32_t ntiles;           // pipelined tiles (persistent kernel)
   int32_t ntiles_slow;      // global / oversized tiles (one CTA each)
   int32_t XP, YP;           // even pitches of S_H rows and S_V columns
+  int32_t skip;             // DGR_DEBUG_SKIP: timing knock-outs (results invalid), 0 in production
   int64_t path_base, tree_base;   // global index of the first local path / tree
   uint64_t seed;
   // forest encoding
@@ -76,11 +77,10 @@ struct KParams {
   float* pp;                // p_i of the last forward (the reverse of that iteration reads it)
   const int32_t* net_tree_off;    // local, n_nets_l + 1
   float *wt, *mt, *vt, *q;
-  // grids (the exchange buffer, in this order: dH | dVT | VDH | VDV | scal)
+  // grids (the exchange buffer, in this order: dH | dVT | VD | scal)
   long long* dH;            // [Y][X]
   long long* dVT;           // [X][Y]
-  long long* VDH;           // [Y][X]
-  long long* VDV;           // [X][Y]
+  long long* VD;            // [Y][X] turning points per G-cell (cleared before every forward)
   long long* scal;          // {E[WL], E[TP]} fixed point
   const float* capH;        // [Y][X]
   const float* capVT;       // [X][Y]

@@ -254,8 +254,9 @@ __device__ __forceinline__ float softmax_from_noise(const Lane& L, float w, floa
 constexpr int kWarps = kTileThreads / 32;
 constexpr int kWarpBundles = (kMaxBundles + kWarps - 1) / kWarps;
 constexpr int kWarpCand = kWarpBundles * 32;
-constexpr size_t kRegionA = 2 * sizeof(double) * kWinMax;
-static_assert(3 * sizeof(int) * kWinMax + sizeof(float) * kWarps * kWarpCand <= kRegionA, "region A too small");
+constexpr size_t kRegionA = (2 * sizeof(double) * kWinMax > 3 * sizeof(int) * kWinMax + sizeof(float) * kWarps * kWarpCand)
+                               ? 2 * sizeof(double) * kWinMax
+                               : 3 * sizeof(int) * kWinMax + sizeof(float) * kWarps * kWarpCand;
 constexpr size_t kSmemBytes = kRegionA + sizeof(float) * kMaxBundles * 32 + sizeof(long long) * kTreeMax +
                               sizeof(float) * kTreeMax + 2 * sizeof(long long);
 
@@ -392,9 +393,9 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
       if (GLOBAL) {
         const int X = P.X, Y = P.Y;
         red64(P.dH + (size_t)ya * X + xa, ah); red64(P.dVT + (size_t)xa * Y + ya, av);
-        red64(P.VDH + (size_t)ya * X + xa, ad); red64(P.VDV + (size_t)xa * Y + ya, ad);
+        red64(P.VD + (size_t)ya * X + xa, ad);
         red64(P.dH + (size_t)yb * X + xb, bh); red64(P.dVT + (size_t)xb * Y + yb, bv);
-        red64(P.VDH + (size_t)yb * X + xb, bd); red64(P.VDV + (size_t)xb * Y + yb, bd);
+        red64(P.VD + (size_t)yb * X + xb, bd);
       }
       const int ntp = fHV + fVH + 2 * fZ;
       wl += (long long)vq * ((x1 - x0) + abs(y1 - y0));
@@ -530,17 +531,13 @@ __global__ void __launch_bounds__(kTileThreads, 3) tile_kernel(KParams P, StepAr
         for (int xi = lane; xi < T.ww; xi += 32) {
           if (T.wx0 + xi >= X) break;
           red64(P.dH + g0 + xi, rowH[xi]);
-          red64(P.VDH + g0 + xi, rowD[xi]);
+          red64(P.VD + g0 + xi, rowD[xi]);
         }
       }
       for (int xi = warp; xi < T.ww; xi += kWarps) {
         const size_t g0 = (size_t)(T.wx0 + xi) * Y + T.wy0;
         const int* colV = ev_s + ncell + xi * T.wh;
-        const int* colD = ev_s + 2 * ncell + xi;
-        for (int yi = lane; yi < T.wh; yi += 32) {
-          red64(P.dVT + g0 + yi, colV[yi]);
-          red64(P.VDV + g0 + yi, colD[yi * T.ww]);
-        }
+        for (int yi = lane; yi < T.wh; yi += 32) red64(P.dVT + g0 + yi, colV[yi]);
       }
     }
     if (tid == 0) { red64(P.scal, red_s[0]); red64(P.scal + 1, red_s[1]); }
@@ -706,7 +703,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
       const float p = St.p[sl];
       const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
       double c = 0.0;
-      if (L.valid) {
+      if (L.valid && !(P.skip & 8)) {
         const short4 e = St.sxy[L.sub - s_lo];
         c = path_cost(St.S, W, X, Y, L.shape, e.x, e.y, e.z, e.w, (int)(L.pw >> 16), A);
       }
@@ -735,44 +732,68 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     __syncthreads();
   }
 
-  // ---------------- tree level ----------------
-  for (int n = tid; n < T.nnet; n += NT) {
-    const int net = T.net0 + n;
-    const int a = St.nto[net - n_lo], b = St.nto[net + 1 - n_lo];
-    if (REV) {
-      double sq = 0.0, sw = 0.0;
-      for (int j = a; j < b; ++j) {
-        const double qj = (double)St.q[j - t_lo];
-        sq += qj * ((double)dq_s[j - T.tree0] * kDqInv);
-        sw += qj;
-      }
-      sq /= sw;
-      for (int j = a; j < b; ++j) {
-        const double du = (b - a == 1) ? 0.0
-                                       : (double)St.q[j - t_lo] * (double)A.inv_t * ((double)dq_s[j - T.tree0] * kDqInv - sq);
-        float w = St.wt[j - t_lo], m = St.mt[j - t_lo], v = St.vt[j - t_lo];
-        adam_update(w, m, v, (float)du, A);
-        St.wt[j - t_lo] = w;
-        P.wt[j] = w; P.mt[j] = m; P.vt[j] = v;
-      }
+  // ---------------- tree level (one thread per tree; S window reused as scratch) ----------------
+  if (!(P.skip & 16)) {
+    double* qd = St.S;                                            // q_j dq_j
+    float* zt = reinterpret_cast<float*>(qd + kPipeTrees);        // (w_j + g_j)/t
+    float* gt = zt + kPipeTrees;                                   // Gumbel noise of the tile's trees
+    short* tfirst = reinterpret_cast<short*>(gt + kPipeTrees + 8); // first tree of the tree's net (tile-local)
+    short* tcnt = tfirst + kPipeTrees;                             // trees of that net
+    for (int n = tid; n < T.nnet; n += NT) {
+      const int a = St.nto[T.net0 + n - n_lo] - T.tree0, b = St.nto[T.net0 + n + 1 - n_lo] - T.tree0;
+      for (int j = a; j < b; ++j) { tfirst[j] = (short)a; tcnt[j] = (short)(b - a); }
     }
     if (FWD) {
-      if (b - a == 1) {
-        St.q[a - t_lo] = 1.f;
-        P.q[a] = 1.f;
-      } else {
-        float zmax = -INFINITY;
-        for (int j = a; j < b; ++j) {
-          const float z = (St.wt[j - t_lo] + gumbel(P.seed, (uint64_t)(P.tree_base + j), (uint32_t)A.k_next, 1u)) * A.inv_t;
-          St.q[j - t_lo] = z;
-          zmax = fmaxf(zmax, z);
+      // one Philox call per 4 consecutive tree candidates (stream 1)
+      const int64_t g0 = P.tree_base + T.tree0;
+      const int64_t c0 = g0 >> 2, c1 = (g0 + T.ntree - 1) >> 2;
+      const uint2 key = make_uint2((uint32_t)P.seed, (uint32_t)(P.seed >> 32));
+      for (int64_t c = c0 + tid; c <= c1; c += NT) {
+        const uint4 r = philox4x32_10(make_uint4((uint32_t)c, (uint32_t)(c >> 32), (uint32_t)A.k_next, 1u), key);
+        const uint32_t wd[4] = {r.x, r.y, r.z, r.w};
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const int64_t i = c * 4 + q - g0;
+          if (i >= 0 && i < T.ntree) gt[i] = gumbel_word(wd[q]);
         }
-        float sum = 0.f;
-        for (int j = a; j < b; ++j) { const float e = __expf(St.q[j - t_lo] - zmax); St.q[j - t_lo] = e; sum += e; }
-        const float inv = 1.f / sum;
-        for (int j = a; j < b; ++j) { St.q[j - t_lo] *= inv; P.q[j] = St.q[j - t_lo]; }
       }
     }
+    if (REV)
+      for (int j = tid; j < T.ntree; j += NT) qd[j] = (double)St.q[j + T.tree0 - t_lo] * ((double)dq_s[j] * kDqInv);
+    __syncthreads();
+    for (int j = tid; j < T.ntree; j += NT) {
+      const int a = tfirst[j], cnt = tcnt[j], jg = j + T.tree0;
+      float wj = St.wt[jg - t_lo];
+      if (REV) {
+        // du_j = (q_j/t)(dq_j - sum_l q_l dq_l / sum_l q_l); Adam on w_tree (iteration k)
+        double sq = 0.0, sw = 0.0;
+        for (int l = a; l < a + cnt; ++l) { sq += qd[l]; sw += (double)St.q[l + T.tree0 - t_lo]; }
+        const double du = cnt == 1 ? 0.0
+                                   : (double)St.q[jg - t_lo] * (double)A.inv_t * ((double)dq_s[j] * kDqInv - sq / sw);
+        float m = St.mt[jg - t_lo], v = St.vt[jg - t_lo];
+        adam_update(wj, m, v, (float)du, A);
+        P.wt[jg] = wj; P.mt[jg] = m; P.vt[jg] = v;
+      }
+      if (FWD) zt[j] = (wj + gt[j]) * A.inv_t;
+    }
+    if (FWD) {
+      __syncthreads();
+      // q_j = softmax over the net's trees of (w_j + g_j)/t, iteration k_next
+      for (int j = tid; j < T.ntree; j += NT) {
+        const int a = tfirst[j], cnt = tcnt[j], jg = j + T.tree0;
+        float q = 1.f;
+        if (cnt > 1) {
+          float zmax = -INFINITY;
+          for (int l = a; l < a + cnt; ++l) zmax = fmaxf(zmax, zt[l]);
+          float sum = 0.f;
+          for (int l = a; l < a + cnt; ++l) sum += __expf(zt[l] - zmax);
+          q = __expf(zt[j] - zmax) / sum;
+        }
+        St.q[jg - t_lo] = q;
+        P.q[jg] = q;
+      }
+    }
+    __syncthreads();
   }
 
   // ---------------- forward of iteration k_next ----------------
@@ -782,7 +803,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
       for (int i = tid; i < (3 * ncell + 3) / 4; i += NT) z[i] = make_int4(0, 0, 0, 0);
     }
     __syncthreads();
-    if (lb0 < lb1) {
+    if (lb0 < lb1 && !(P.skip & 2)) {
       const int4 bfirst = St.bi[lb0];
       const int4 blast = St.bi[lb1 - 1];
       warp_noise(g_s, P.seed, P.path_base + bfirst.x, blast.x + blast.w - bfirst.x, (uint32_t)A.k_next, lane);
@@ -829,7 +850,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
       const int bh = -fSH * vv - fHV * a - fVH * (bb + hs) + (fZH - fZV) * vv;
       const int bv = -fSV * vv + sgn * (fHV * a - fVH * (a + vs) + (fZV - fZH) * vv);
       const int bd = fHV * a + fZ * vv;
-      if (L.valid) {
+      if (L.valid && !(P.skip & 4)) {
         const int hv2 = 2 * ncell;
         const int ia_h = W.h(xa, ya), ib_h = W.h(xb, yb);
         red_shared_add(ev_base + 4u * ia_h, ah);
@@ -857,25 +878,27 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     if (FWD) bulk_s2g(P.pp + s0, St.p, slot_bytes);
     bulk_commit();
   }
-  if (FWD) {
+  if (FWD && !(P.skip & 1)) {
+    // flush: a warp per window row (dH, VD) / column (dV); cells in pairs, zero pairs skipped
+    const int hw = T.ww >> 1, hh = T.wh >> 1;
     for (int yi = warp; yi < T.wh; yi += NW) {
       if (T.wy0 + yi >= Y) break;
       const size_t g0 = (size_t)(T.wy0 + yi) * X + T.wx0;
-      const int* rowH = ev_s + yi * T.ww;
-      const int* rowD = ev_s + 2 * ncell + yi * T.ww;
-      for (int xi = lane; xi < T.ww; xi += 32) {
-        red64(P.dH + g0 + xi, rowH[xi]);
-        red64(P.VDH + g0 + xi, rowD[xi]);
+      const int2* rowH = reinterpret_cast<const int2*>(ev_s + yi * T.ww);
+      const int2* rowD = reinterpret_cast<const int2*>(ev_s + 2 * ncell + yi * T.ww);
+      for (int xp = lane; xp < hw; xp += 32) {
+        const int2 h = rowH[xp], d = rowD[xp];
+        if (h.x | h.y) { red64(P.dH + g0 + 2 * xp, h.x); red64(P.dH + g0 + 2 * xp + 1, h.y); }
+        if (d.x | d.y) { red64(P.VD + g0 + 2 * xp, d.x); red64(P.VD + g0 + 2 * xp + 1, d.y); }
       }
     }
     for (int xi = warp; xi < T.ww; xi += NW) {
       if (T.wx0 + xi >= X) break;
       const size_t g0 = (size_t)(T.wx0 + xi) * Y + T.wy0;
-      const int* colV = ev_s + ncell + xi * T.wh;
-      const int* colD = ev_s + 2 * ncell + xi;
-      for (int yi = lane; yi < T.wh; yi += 32) {
-        red64(P.dVT + g0 + yi, colV[yi]);
-        red64(P.VDV + g0 + yi, colD[yi * T.ww]);
+      const int2* colV = reinterpret_cast<const int2*>(ev_s + ncell + xi * T.wh);
+      for (int yp = lane; yp < hh; yp += 32) {
+        const int2 v = colV[yp];
+        if (v.x | v.y) { red64(P.dVT + g0 + 2 * yp, v.x); red64(P.dVT + g0 + 2 * yp + 1, v.y); }
       }
     }
   }
@@ -898,13 +921,13 @@ __device__ __forceinline__ void flush_scalars(const KParams& P, long long wl, lo
 }
 
 // (a) one tile per CTA: the whole tile arrives by bulk copies on one mbarrier; the event window
-// and noise alias the S window.  3 CTAs per SM overlap one CTA's copies with the others' math.
+// and noise alias the S window.  4 CTAs per SM overlap one CTA's copies with the others' math.
 constexpr int kBThreads = 256;
 constexpr size_t kBSmemBytes = StageLayout::bytes + 8 * kPipeTrees + 64;
 static_assert(kPEvBytes + 4 * kWinMax <= 2 * 8 * kWinMax, "event window + noise must fit the S window");
 
 template <bool REV, bool FWD>
-__global__ void __launch_bounds__(kBThreads, 3) tile_bulk(KParams P, StepArgs A) {
+__global__ void __launch_bounds__(kBThreads, 4) tile_bulk(KParams P, StepArgs A) {
   extern __shared__ __align__(128) unsigned char smem[];
   Stage St(smem);
   long long* dq_s = reinterpret_cast<long long*>(smem + StageLayout::bytes);
@@ -970,10 +993,10 @@ __global__ void __launch_bounds__(kPThreads, 1) tile_persistent(KParams P, StepA
 // KG: one CTA per line (Y H-rows, then X V-columns).  Scan of the difference array gives the
 // wire demand W; d = (W + beta (VD_a + VD_b)) 2^-24 (Eq. (10), reading Q3); overflow cost
 // f(cap - d) (Eq. (9)); G = dcost/dd = -a3 f'(cap - d); S = exclusive prefix of G (fp64).
-// The line's difference and turning-point entries are cleared for the next forward.
+// The line's difference entries are cleared for the next forward (VD is cleared by a memset).
 // ------------------------------------------------------------------------------------------
 constexpr int kGThreads = 256;
-constexpr int kGItems = 8;
+constexpr int kGItems = 4;
 
 template <typename T>
 __device__ __forceinline__ T block_exclusive_scan(T v, T* sh, T* total) {
@@ -1054,7 +1077,9 @@ __global__ void __launch_bounds__(kGThreads) kg_kernel(KParams P, StepArgs A) {
   const int ln = isH ? line : line - P.Y;
   const size_t base = (size_t)ln * n;
   long long* diff = (isH ? P.dH : P.dVT) + base;
-  long long* vd = (isH ? P.VDH : P.VDV) + base;
+  // turning points at the line's cells: contiguous for a row, stride X for a column
+  const long long* vd = isH ? P.VD + base : P.VD + ln;
+  const size_t vstep = isH ? 1 : (size_t)P.X;
   const float* cap = (isH ? P.capH : P.capVT) + base;
   double* S = isH ? P.SH + (size_t)ln * P.XP : P.SVT + (size_t)ln * P.YP;
   float* dout = (isH ? P.dOutH : P.dOutVT) + base;
@@ -1068,8 +1093,8 @@ __global__ void __launch_bounds__(kGThreads) kg_kernel(KParams P, StepArgs A) {
     for (int j = 0; j < kGItems; ++j) {
       const int pos = c0 + j * kGThreads + threadIdx.x;
       v[j] = pos < n ? diff[pos] : 0;
-      t0[j] = pos < n ? vd[pos] : 0;
-      t1[j] = pos + 1 < n ? vd[pos + 1] : 0;
+      t0[j] = pos < n ? vd[(size_t)pos * vstep] : 0;
+      t1[j] = pos + 1 < n ? vd[(size_t)(pos + 1) * vstep] : 0;
       cp[j] = pos < n ? cap[pos] : 0.f;
     }
     long long totW;
@@ -1080,7 +1105,7 @@ __global__ void __launch_bounds__(kGThreads) kg_kernel(KParams P, StepArgs A) {
 #pragma unroll
     for (int j = 0; j < kGItems; ++j) {
       const int pos = c0 + j * kGThreads + threadIdx.x;
-      if (pos < n) { diff[pos] = 0; vd[pos] = 0; }
+      if (pos < n) diff[pos] = 0;
     }
     double g[kGItems];
 #pragma unroll
