@@ -82,8 +82,10 @@ typedef struct {
   float a_wl, a_via, a_of;   /* a1, a2, a3 of Eq. (3); paper: 0.5, 4, 500 */
   float beta_via;            /* beta_v of Eqs. (2)/(10), one global value (Q3; default 0.25) */
   float n_layers;            /* L in sqrt(L) of Eqs. (5)/(12) (Q4; default 5) */
-  int32_t f_kind;            /* overflow function f of Eq. (9): 0 = sigmoid, 1 = ReLU */
-  float f_slope;             /* s in f(r) = 1 / (1 + exp(s r)) (Q2; default 1) */
+  int32_t f_kind;            /* overflow function f of Eq. (9) of x = d - cap (Q2): 0 = sigmoid(s x)
+                                (P:912), 1 = ReLU, 2 = LeakyReLU, 3 = exp(s x), 4 = CELU
+                                (the alternatives studied in Fig. 6) */
+  float f_slope;             /* sigmoid / exp: s (default 1); LeakyReLU: negative slope (0.01); CELU: alpha (1) */
 } dgr_weights;
 
 /* Loss of a forward pass: total = a_wl*wl + a_via*via + a_of*overflow, with

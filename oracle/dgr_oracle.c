@@ -88,8 +88,9 @@ typedef struct {
   double a_wl, a_via, a_of;   /* a1, a2, a3 of Eq. (3): 0.5, 4, 500 */
   double beta;                /* beta_v of Eqs. (2)/(10) (reading Q3: global, default 0.25) */
   double n_layers;            /* L of Eq. (5)/(12) (reading Q4: 5) */
-  int32_t f_kind;             /* 0 = sigmoid, 1 = ReLU */
-  double f_slope;             /* s of the sigmoid f(r) = 1/(1+exp(s r)) (reading Q2) */
+  int32_t f_kind;             /* 0 = sigmoid, 1 = ReLU, 2 = LeakyReLU, 3 = exp,
+                                 4 = CELU (the alternatives of §5.3 / Fig. 6) */
+  double f_slope;             /* sigmoid / exp: steepness s; LeakyReLU: negative slope; CELU: alpha (Q2) */
 } odgr_weights;
 
 typedef struct {
@@ -258,6 +259,28 @@ ODGR_API void odgr_forward_partial(odgr_state* s, double t, const odgr_weights* 
 
 static real sigm(real x) { return R(1) / (R(1) + exp(-x)); }
 
+/* f applied to the resource r = cap - d, written in the overflow x = d - cap = -r (reading Q2):
+ * sigmoid sigma(s x) = 1/(1+exp(s r)), ReLU max(0, x), LeakyReLU, exp(s x), CELU
+ * (Fig. 6; torch conventions, negative slope / alpha in f_slope).  f_grad = df/dx = df/dd. */
+static real f_of(int kind, real s, real x) {
+  switch (kind) {
+    case 0: return sigm(s * x);
+    case 1: return x > 0 ? x : R(0);
+    case 2: return x > 0 ? x : s * x;
+    case 3: return exp(s * x);
+    default: return x > 0 ? x : s * (exp(x / s) - R(1));
+  }
+}
+static real f_grad(int kind, real s, real x) {
+  switch (kind) {
+    case 0: return s * sigm(s * x) * sigm(-s * x);
+    case 1: return x > 0 ? R(1) : R(0);
+    case 2: return x > 0 ? R(1) : s;
+    case 3: return s * exp(s * x);
+    default: return x > 0 ? R(1) : exp(x / s);
+  }
+}
+
 /* ---- forward, part 2: the cost of Eq. (3) from the (global) demand in s->d_h, s->d_v ---- */
 static real forward_finish(odgr_state* s, real e_wl, real e_tp, const odgr_weights* W, double out[4]) {
   const int X = s->X, Y = s->Y;
@@ -270,8 +293,7 @@ static real forward_finish(odgr_state* s, real e_wl, real e_tp, const odgr_weigh
         if (dir == 0 && x > X - 2) continue;
         if (dir == 1 && y > Y - 2) continue;
         real r = (dir == 0 ? s->cap_h[e] - s->d_h[e] : s->cap_v[e] - s->d_v[e]);  /* resource */
-        if (W->f_kind == 0) of += R(1) / (R(1) + exp(slope * r));   /* sigmoid, decreasing in r */
-        else of += r < 0 ? -r : R(0);                                 /* ReLU(d - cap) */
+        of += f_of(W->f_kind, slope, -r);
       }
     }
   s->e_wl = e_wl; s->e_tp = e_tp; s->overflow = of;
@@ -306,14 +328,8 @@ static void backward(odgr_state* s, real t, const odgr_weights* W, real* dw_path
   for (int y = 0; y < Y; ++y)
     for (int x = 0; x < X; ++x) {
       size_t e = (size_t)y * X + x;
-      if (x <= X - 2) {
-        real r = s->cap_h[e] - s->d_h[e];
-        gh[e] = W->f_kind == 0 ? a3 * slope * sigm(slope * r) * sigm(-slope * r) : (s->d_h[e] > s->cap_h[e] ? a3 : R(0));
-      }
-      if (y <= Y - 2) {
-        real r = s->cap_v[e] - s->d_v[e];
-        gv[e] = W->f_kind == 0 ? a3 * slope * sigm(slope * r) * sigm(-slope * r) : (s->d_v[e] > s->cap_v[e] ? a3 : R(0));
-      }
+      if (x <= X - 2) gh[e] = a3 * f_grad(W->f_kind, slope, s->d_h[e] - s->cap_h[e]);
+      if (y <= Y - 2) gv[e] = a3 * f_grad(W->f_kind, slope, s->d_v[e] - s->cap_v[e]);
     }
   const real sqL = sqrt((real)W->n_layers);
   for (int64_t n = s->net_lo; n < s->net_hi; ++n) {

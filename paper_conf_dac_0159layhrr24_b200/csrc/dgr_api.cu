@@ -652,7 +652,9 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
   if (!h || !w) return fail(DGR_EINVAL, "NULL handle or weights");
   if (iters < 0) return fail(DGR_EINVAL, "iters < 0");
   if (!(temperature > 0.f) || !std::isfinite(temperature)) return fail(DGR_EINVAL, "temperature must be > 0");
-  if (w->f_kind != 0 && w->f_kind != 1) return fail(DGR_EINVAL, "f_kind must be 0 (sigmoid) or 1 (ReLU)");
+  if (w->f_kind < 0 || w->f_kind > 4) return fail(DGR_EINVAL, "f_kind must be 0..4 (sigmoid, ReLU, LeakyReLU, exp, CELU)");
+  if ((w->f_kind == 0 || w->f_kind == 3 || w->f_kind == 4) && !(w->f_slope > 0.f))
+    return fail(DGR_EINVAL, "f_slope must be > 0 for sigmoid / exp / CELU");
   KParams& P = h->P;
   StepArgs a{};
   a.inv_t = 1.f / temperature;

@@ -586,8 +586,8 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   asm volatile(
       "{\n\t.reg .pred P1;\n\tWAIT_%=:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
-      "@!P1 bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)), "r"(parity) : "memory");
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, %2;\n\t"
+      "@!P1 bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)), "r"(parity), "r"(1000000u) : "memory");   // suspend, don't spin
 }
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(dst)),
@@ -1115,19 +1115,28 @@ __global__ void __launch_bounds__(kGThreads) kg_kernel(KParams P, StepArgs A) {
       if (pos < n - 1) {
         const long long W = carryW + ex[j] + v[j];   // inclusive prefix = wire demand of edge pos
         const double d = (double)W * kFixInv + beta * ((double)(t0[j] + t1[j]) * kFixInv);
-        const double r = (double)cp[j] - d;
-        if (A.f_kind == 0) {
-          // sigmoid: f(r) = 1/(1+exp(s r)) = sigma(-s r); -f'(r) = s sigma(s r) sigma(-s r).
-          // fp64 here (one exp per edge): G feeds every candidate's cost difference.
-          const double sr = (double)A.f_slope * r;
-          const double e = exp(-fabs(sr));
-          const double inv = 1.0 / (1.0 + e);
-          of += (sr > 0.0) ? e * inv : inv;
-          G = (double)A.a_of * (double)A.f_slope * e * inv * inv;
-        } else {
-          of += r < 0.0 ? -r : 0.0;
-          G = (d > (double)cp[j]) ? (double)A.a_of : 0.0;
+        const double x = d - (double)cp[j];                 // overflow x = -(cap - d)
+        const double sl = (double)A.f_slope;
+        double fv, fg;                                      // f(x) and df/dx = df/dd
+        switch (A.f_kind) {
+          case 0: {   // sigmoid sigma(s x); stable for both signs; fp64 (one exp per edge)
+            const double e = exp(-fabs(sl * x));
+            const double inv = 1.0 / (1.0 + e);
+            fv = (sl * x > 0.0) ? inv : e * inv;
+            fg = sl * e * inv * inv;
+            break;
+          }
+          case 1: fv = x > 0.0 ? x : 0.0; fg = x > 0.0 ? 1.0 : 0.0; break;        // ReLU
+          case 2: fv = x > 0.0 ? x : sl * x; fg = x > 0.0 ? 1.0 : sl; break;      // LeakyReLU (Fig. 6)
+          case 3: fv = exp(sl * x); fg = sl * fv; break;                          // exp (Fig. 6)
+          default: {                                                              // CELU (Fig. 6)
+            const double e = exp(fmin(x, 0.0) / sl);
+            fv = x > 0.0 ? x : sl * (e - 1.0);
+            fg = x > 0.0 ? 1.0 : e;
+          }
         }
+        of += fv;
+        G = (double)A.a_of * fg;
         if (A.store_d) dout[pos] = (float)d;
       } else if (pos == n - 1 && A.store_d) {
         dout[pos] = 0.f;

@@ -43,13 +43,22 @@ class _Dist(ctypes.Structure):
     _fields_ = [("rank", ctypes.c_int32), ("world", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p)]
 
 
+F_KINDS = {"sigmoid": 0, "relu": 1, "leaky_relu": 2, "exp": 3, "celu": 4}
+_DEFAULT_SLOPE = {0: 1.0, 1: 1.0, 2: 0.01, 3: 1.0, 4: 1.0}
+
+
 class Weights(ctypes.Structure):
-    """dgr_weights: a1, a2, a3, beta_v (Q3), L (Q4), f kind (0 sigmoid, 1 ReLU), slope (Q2)."""
+    """dgr_weights: a1, a2, a3, beta_v (Q3), L (Q4), overflow function f (0 sigmoid, 1 ReLU,
+    2 LeakyReLU, 3 exp, 4 CELU; Fig. 6) and its slope / alpha (Q2)."""
     _fields_ = [("a_wl", ctypes.c_float), ("a_via", ctypes.c_float), ("a_of", ctypes.c_float),
                 ("beta_via", ctypes.c_float), ("n_layers", ctypes.c_float), ("f_kind", ctypes.c_int32),
                 ("f_slope", ctypes.c_float)]
 
-    def __init__(self, a_wl=0.5, a_via=4.0, a_of=500.0, beta_via=0.25, n_layers=5.0, f_kind=0, f_slope=1.0):
+    def __init__(self, a_wl=0.5, a_via=4.0, a_of=500.0, beta_via=0.25, n_layers=5.0, f_kind=0, f_slope=None):
+        if isinstance(f_kind, str):
+            f_kind = F_KINDS[f_kind]
+        if f_slope is None:
+            f_slope = _DEFAULT_SLOPE[int(f_kind)]
         super().__init__(a_wl, a_via, a_of, beta_via, n_layers, f_kind, f_slope)
 
 

@@ -99,11 +99,18 @@ def torch_cost(f, w_tree, w_path, g_tree, g_path, t, W):
     valid[0, :, : X - 1] = True
     valid[1, : Y - 1, :] = True
     valid = torch.as_tensor(valid.reshape(-1))
-    r = cap - d
+    x = d - cap                         # overflow = -(resource)
+    F = torch.nn.functional
     if W.f_kind == 0:
-        fo = torch.sigmoid(-W.f_slope * r)
+        fo = torch.sigmoid(W.f_slope * x)
+    elif W.f_kind == 1:
+        fo = torch.relu(x)
+    elif W.f_kind == 2:
+        fo = F.leaky_relu(x, negative_slope=W.f_slope)
+    elif W.f_kind == 3:
+        fo = torch.exp(W.f_slope * x)
     else:
-        fo = torch.relu(-r)
+        fo = F.celu(x, alpha=W.f_slope)
     of = fo[valid].sum()
     wl = torch.tensor([sum(int(s[3] - s[2]) for s in f.seg[f.path_seg_off[i]:f.path_seg_off[i + 1]])
                        for i in range(f.n_paths)], dtype=torch.float64)

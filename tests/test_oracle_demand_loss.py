@@ -115,9 +115,10 @@ def test_brute_force_expectation(tiny, which):
     assert len(path_sub) == f.n_paths
 
 
-@pytest.mark.parametrize("f_kind", [0, 1])
-def test_cost_matches_torch_restatement(tiny, f_kind):
-    W = oracle.weights(f_kind=f_kind)
+@pytest.mark.parametrize("f_kind,slope", [(0, 1.0), (1, 1.0), (2, 0.01), (3, 0.5), (4, 1.0)])
+def test_cost_matches_torch_restatement(tiny, f_kind, slope):
+    """sigmoid, ReLU and the LeakyReLU / exp / CELU alternatives of Fig. 6."""
+    W = oracle.weights(f_kind=f_kind, f_slope=slope)
     o = oracle.Oracle(tiny)
     o.iteration = 2
     t = 0.9

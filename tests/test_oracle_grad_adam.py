@@ -73,9 +73,9 @@ def test_gradient_central_differences_relu_away_from_kinks(tiny):
     assert checked >= 15
 
 
-@pytest.mark.parametrize("f_kind", [0, 1])
-def test_gradient_matches_torch_autograd(tiny, f_kind):
-    W = oracle.weights(f_kind=f_kind)
+@pytest.mark.parametrize("f_kind,slope", [(0, 1.0), (1, 1.0), (2, 0.01), (3, 0.5), (4, 1.0)])
+def test_gradient_matches_torch_autograd(tiny, f_kind, slope):
+    W = oracle.weights(f_kind=f_kind, f_slope=slope)
     t, k = 0.7, 5
     o, (dw, du) = _grad(tiny, k, t, W)
     g = torch.tensor([oracle.gumbel(tiny.seed, i, k, 0) for i in range(tiny.n_paths)], dtype=torch.float64)
