@@ -36,7 +36,7 @@ class _Config(ctypes.Structure):
         ("box_mode", ctypes.c_int32), ("box_min", ctypes.c_int32), ("box_max", ctypes.c_int32),
         ("box_mu", ctypes.c_double), ("cluster_frac", ctypes.c_double), ("n_hotspots", ctypes.c_int32),
         ("track", ctypes.c_double), ("beta_pin", ctypes.c_double), ("n_tree_cand", ctypes.c_int32),
-        ("z_cap", ctypes.c_int32), ("seed", ctypes.c_uint64),
+        ("z_cap", ctypes.c_int32), ("seed", ctypes.c_uint64), ("local_weight", ctypes.c_double),
     ]
 
 
@@ -97,6 +97,22 @@ def _sweep(n: int) -> dict:
                 n_tree_cand=2, z_cap=15, seed=1)
 
 
+# PAPER.md Table 1: (grid side, cap_e, #nets, box) of the ILP comparison rows.  Three
+# G-cells drawn in a box per net as pins, L-shape candidates only, uniform
+# capacity.  "Every 2-pin pair" is read as the MST's two sub-nets (ambiguous; the
+# printed overflows are not reproducible and stay unpinned).
+TABLE1_ROWS = [(20, 1, 20, 4), (50, 1, 50, 10), (50, 1, 100, 10), (50, 2, 100, 10), (50, 1, 1000, 10),
+               (50, 10, 1000, 10), (50, 10, 10000, 10), (100, 2, 1000, 20), (100, 2, 10000, 20),
+               (1000, 1, 100000, 200)]
+TABLE1_DGR = [30, 173, 1028, 0, 35445, 7407, 364536, 48846, 785664, 80237614]   # DGR* overflow column
+
+
+def _table1(side, cap, nets, box):
+    return dict(X=side, Y=side, n_nets=nets, pins_mode=0, pins_min=3, pins_max=3, box_mode=0, box_min=box,
+                box_max=box, cluster_frac=0.0, n_hotspots=0, track=float(cap), beta_pin=0.0, local_weight=0.0,
+                n_tree_cand=1, z_cap=-1, seed=1)
+
+
 CONFIGS: dict[str, dict] = {
     # 16x16, 40 nets of 2-4 pins in boxes U{2..8}, 2 trees, L+Z uncapped, T=1 uniform
     "tiny": dict(X=16, Y=16, n_nets=40, pins_mode=0, pins_min=2, pins_max=4, box_mode=0, box_min=2,
@@ -112,6 +128,7 @@ CONFIGS: dict[str, dict] = {
     "ispd19": dict(X=1000, Y=1000, n_nets=1_000_000, pins_mode=1, box_mode=1, box_mu=5.0,
                    cluster_frac=0.3, n_hotspots=32, track=4.0, beta_pin=0.25, n_tree_cand=2, z_cap=15,
                    seed=1),
+    **{f"table1_r{i + 1}": _table1(*row) for i, row in enumerate(TABLE1_ROWS)},
     "sweep1e4": _sweep(10_000),
     "sweep1e5": _sweep(100_000),
     "sweep1e6": _sweep(1_000_000),
@@ -185,7 +202,7 @@ def generate(config: str | dict, seed: int | None = None, gumbel_seed: int = GUM
     c = _Config()
     defaults = dict(pins_min=2, pins_max=4, box_min=2, box_max=8, box_mu=5.0, cluster_frac=0.0,
                     n_hotspots=0, track=1.0, beta_pin=0.0, n_tree_cand=2, z_cap=15, seed=1,
-                    pins_mode=0, box_mode=0)
+                    pins_mode=0, box_mode=0, local_weight=1.0)
     for k, v in {**defaults, **cfg}.items():
         setattr(c, k, v)
     lib = _load()

@@ -420,13 +420,13 @@ extern "C" int forestgen_generate(const forestgen_config* cp, forestgen_forest**
       if (x + 1 < X) {
         const size_t b = a + 1;
         double v = c.track * hval(2 * x + 2 < 2 * X ? 2 * x + 2 : 2 * X - 1, 2 * y + 1) -
-                   c.beta_pin * (pin_cnt[a] + pin_cnt[b]) / 2.0 - (local_cnt[a] + local_cnt[b]) / 2.0;
+                   c.beta_pin * (pin_cnt[a] + pin_cnt[b]) / 2.0 - c.local_weight * (local_cnt[a] + local_cnt[b]) / 2.0;
         f->cap_h[a] = q4(v);
       }
       if (y + 1 < Y) {
         const size_t b = a + X;
         double v = c.track * hval(2 * x + 1, 2 * y + 2 < 2 * Y ? 2 * y + 2 : 2 * Y - 1) -
-                   c.beta_pin * (pin_cnt[a] + pin_cnt[b]) / 2.0 - (local_cnt[a] + local_cnt[b]) / 2.0;
+                   c.beta_pin * (pin_cnt[a] + pin_cnt[b]) / 2.0 - c.local_weight * (local_cnt[a] + local_cnt[b]) / 2.0;
         f->cap_v[a] = q4(v);
       }
     }

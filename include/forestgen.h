@@ -46,6 +46,7 @@ typedef struct {
   int32_t n_tree_cand;     /* 1 or 2 routing-tree candidates per net */
   int32_t z_cap;           /* -1: L only; 0: all Z; >0: at most z_cap Z per direction */
   uint64_t seed;
+  double  local_weight;    /* weight of the local-net term of Eq. (1) (1 = as written; 0 for Table 1's uniform cap) */
 } forestgen_config;
 
 typedef struct forestgen_forest forestgen_forest;

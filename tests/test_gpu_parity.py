@@ -278,3 +278,28 @@ def test_full_size_sampled_parity():
     s.step(1, 1.0, 0.3)
     o.step(1, 1.0, 0.3, ow(dgr.Weights()))
     compare_state(s, o, "ispd19", probe=probes(f, [(0, 1.0), (1, 1.0)]), max_ill=1e-4)
+
+
+def test_table1_workload_relu_parity_and_optimum():
+    """Row f2: overflow-only ReLU, L-only, argmax.  Parity over 3 iterations on a Table-1
+    row and the brute-force optimum reached by the GPU on a small instance (best of 5 seeds)."""
+    from tests.test_table1 import W_T1, _small, brute_force_overflow
+    W = dgr.Weights(a_wl=0.0, a_via=0.0, a_of=1.0, beta_via=0.0, f_kind=1)
+    f = forestgen.generate("table1_r5")
+    s, o, gl, ol = run_both(f, [(3, 1.0)], W)
+    compare_state(s, o, "table1_r5", probe=probes(f, [(3, 1.0)], W), max_ill=0.02)
+    g = _small(2)
+    opt = brute_force_overflow(g)
+    best = None
+    rng = np.random.default_rng(0)
+    for run in range(5):
+        h = copy.deepcopy(g)
+        h.seed = 2000 + run
+        h.w_path0 = rng.random(g.n_paths).astype(np.float32)
+        sv = dgr.Solver(h)
+        for k in range(5):
+            sv.step(100, 0.9 ** k, 0.3, W, want_loss=False)
+        m = sv.induce(0.0).metrics[0]
+        best = m if best is None else min(best, m)
+    assert best == opt
+    assert W_T1["f_kind"] == 1
