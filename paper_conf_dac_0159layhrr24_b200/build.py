@@ -12,7 +12,7 @@ SOURCES = [os.path.join(CSRC, f) for f in ("dgr_api.cu", "dgr_kernels.cu")]
 HEADERS = [os.path.join(CSRC, "dgr_internal.h"), os.path.join(ROOT, "include", "dgr.h")]
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
-              "-Xcompiler", "-fPIC", "-shared"]
+              "-Xcompiler", "-fPIC,-fopenmp", "-shared", "-lgomp"]
 
 
 def nvcc() -> str:
@@ -32,7 +32,8 @@ def stale() -> bool:
 def build(verbose: bool = False, force: bool = False) -> str:
     if not force and not stale():
         return LIB
-    cmd = [nvcc(), *NVCC_FLAGS, "-I" + os.path.join(ROOT, "include"), "-o", LIB, *SOURCES, "-lnccl"]
+    extra = os.environ.get("DGR_NVCC_EXTRA", "").split()
+    cmd = [nvcc(), *NVCC_FLAGS, *extra, "-I" + os.path.join(ROOT, "include"), "-o", LIB, *SOURCES, "-lnccl"]
     if verbose:
         print(" ".join(cmd))
     subprocess.check_call(cmd)

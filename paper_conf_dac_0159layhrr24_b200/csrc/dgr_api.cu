@@ -224,33 +224,54 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   for (int64_t n = 0; n <= nn; ++n) pl.net_tree_off[n] = (int32_t)(d->net_tree_off[pl.net_lo + n] - pl.tree_lo);
   pl.sxy.resize(ns);
   pl.sub_first_path.resize(ns);
-  // 1. canonical sub-net endpoints + pattern words of every local candidate
+  // 1. canonical sub-net endpoints + pattern words of every local candidate (parallel over
+  //    sub-nets; the first failing sub-net, in index order, is reported)
   std::vector<uint32_t> pw_path((size_t)(pl.path_hi - pl.path_lo));
-  for (int64_t j = pl.tree_lo; j < pl.tree_hi; ++j) {
-    for (int64_t s = d->tree_sub_off[j]; s < d->tree_sub_off[j + 1]; ++s) {
-      const int32_t* e = d->sub_xy + 4 * s;
-      int x0 = e[0], y0 = e[1], x1 = e[2], y1 = e[3];
-      if (x0 > x1 || (x0 == x1 && y0 > y1)) { std::swap(x0, x1); std::swap(y0, y1); }
-      if (x0 < 0 || x1 >= X || std::min(y0, y1) < 0 || std::max(y0, y1) >= Y)
-        return fail(DGR_EINVAL, "sub-net %lld endpoints outside the grid", (long long)s);
-      if (x0 == x1 && y0 == y1) return fail(DGR_EINVAL, "sub-net %lld has zero length", (long long)s);
-      const int64_t ls = s - pl.sub_lo;
-      pl.sxy[ls] = make_short4((short)x0, (short)y0, (short)x1, (short)y1);
-      const int64_t p0 = d->sub_path_off[s], p1 = d->sub_path_off[s + 1];
-      pl.sub_first_path[ls] = p0 - pl.path_lo;
-      for (int64_t i = p0; i < p1; ++i) {
-        uint32_t shape;
-        int mid;
-        if (!classify(d, i, x0, y0, x1, y1, &shape, &mid))
-          return fail(DGR_EINVAL, "path %lld is not a straight/L/Z pattern of sub-net %lld (or its turning points are wrong)",
-                      (long long)i, (long long)s);
-        uint32_t pw = shape | ((uint32_t)mid << 16);
-        if (i == p0) {
-          pw |= kSubHead;
-          if (s == d->tree_sub_off[j]) pw |= kTreeHead;
-        }
-        pw_path[i - pl.path_lo] = pw;
+  std::vector<char> first_of_tree((size_t)ns, 0);
+  for (int64_t j = pl.tree_lo; j < pl.tree_hi; ++j) first_of_tree[d->tree_sub_off[j] - pl.sub_lo] = 1;
+  int64_t bad_sub = ns;   // smallest failing local sub-net
+#pragma omp parallel for schedule(dynamic, 4096) reduction(min : bad_sub)
+  for (int64_t ls = 0; ls < ns; ++ls) {
+    const int64_t s = pl.sub_lo + ls;
+    const int32_t* e = d->sub_xy + 4 * s;
+    int x0 = e[0], y0 = e[1], x1 = e[2], y1 = e[3];
+    if (x0 > x1 || (x0 == x1 && y0 > y1)) { std::swap(x0, x1); std::swap(y0, y1); }
+    if (x0 < 0 || x1 >= X || std::min(y0, y1) < 0 || std::max(y0, y1) >= Y || (x0 == x1 && y0 == y1)) {
+      bad_sub = std::min(bad_sub, ls);
+      continue;
+    }
+    pl.sxy[ls] = make_short4((short)x0, (short)y0, (short)x1, (short)y1);
+    const int64_t p0 = d->sub_path_off[s], p1 = d->sub_path_off[s + 1];
+    pl.sub_first_path[ls] = p0 - pl.path_lo;
+    for (int64_t i = p0; i < p1; ++i) {
+      uint32_t shape;
+      int mid;
+      if (!classify(d, i, x0, y0, x1, y1, &shape, &mid)) {
+        bad_sub = std::min(bad_sub, ls);
+        break;
       }
+      uint32_t pw = shape | ((uint32_t)mid << 16);
+      if (i == p0) {
+        pw |= kSubHead;
+        if (first_of_tree[ls]) pw |= kTreeHead;
+      }
+      pw_path[i - pl.path_lo] = pw;
+    }
+  }
+  if (bad_sub < ns) {
+    const int64_t s = pl.sub_lo + bad_sub;
+    const int32_t* e = d->sub_xy + 4 * s;
+    int x0 = e[0], y0 = e[1], x1 = e[2], y1 = e[3];
+    if (x0 > x1 || (x0 == x1 && y0 > y1)) { std::swap(x0, x1); std::swap(y0, y1); }
+    if (x0 < 0 || x1 >= X || std::min(y0, y1) < 0 || std::max(y0, y1) >= Y)
+      return fail(DGR_EINVAL, "sub-net %lld endpoints outside the grid", (long long)s);
+    if (x0 == x1 && y0 == y1) return fail(DGR_EINVAL, "sub-net %lld has zero length", (long long)s);
+    for (int64_t i = d->sub_path_off[s]; i < d->sub_path_off[s + 1]; ++i) {
+      uint32_t shape;
+      int mid;
+      if (!classify(d, i, x0, y0, x1, y1, &shape, &mid))
+        return fail(DGR_EINVAL, "path %lld is not a straight/L/Z pattern of sub-net %lld (or its turning points are wrong)",
+                    (long long)i, (long long)s);
     }
   }
   // 2. tiles of whole nets: greedy in net order while the window (union of the nets' sub-net boxes
@@ -324,70 +345,85 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     if (cur.nb > kMaxBundles) return fail(DGR_EINVAL, "net %lld needs %d > %d bundles", (long long)n, cur.nb, kMaxBundles);
   }
   starts.push_back(pl.net_hi);
-  // 3. bundles, tile by tile (packing restarts at each tile)
-  std::vector<uint16_t> cnt;
-  for (size_t t = 0; t + 1 < starts.size(); ++t) {
-    TileDesc T{};
-    T.net0 = (int32_t)(starts[t] - pl.net_lo);
-    T.nnet = (int32_t)(starts[t + 1] - starts[t]);
-    T.tree0 = (int32_t)(d->net_tree_off[starts[t]] - pl.tree_lo);
-    T.ntree = (int32_t)(d->net_tree_off[starts[t + 1]] - d->net_tree_off[starts[t]]);
-    T.b0 = (int32_t)pl.binfo.size();
-    T.global = globs[t];
-    int bx0 = X, by0 = Y, bx1 = -1, by1 = -1;
-    for (int64_t n = starts[t]; n < starts[t + 1]; ++n) {
-      int a0, b0_, a1, b1_;
-      net_box(n, a0, b0_, a1, b1_);
-      bx0 = std::min(bx0, a0); by0 = std::min(by0, b0_); bx1 = std::max(bx1, a1); by1 = std::max(by1, b1_);
-    }
-    T.wx0 = bx0 & ~1; T.wy0 = by0 & ~1;
-    T.ww = (bx1 + 1 - T.wx0 + 1) & ~1; T.wh = (by1 + 1 - T.wy0 + 1) & ~1;
-    if (T.global) { T.wx0 = 0; T.wy0 = 0; T.ww = 0; T.wh = 0; }
-    T.sub0 = (int32_t)(d->tree_sub_off[d->net_tree_off[starts[t]]] - pl.sub_lo);
-    T.nsub = (int32_t)(d->tree_sub_off[d->net_tree_off[starts[t + 1]]] - pl.sub_lo) - T.sub0;
-    int fill = 32;
-    const int64_t j0 = d->net_tree_off[starts[t]], j1 = d->net_tree_off[starts[t + 1]];
-    for (int64_t j = j0; j < j1; ++j) {
-      for (int64_t s = d->tree_sub_off[j]; s < d->tree_sub_off[j + 1]; ++s) {
-        const int64_t p0 = d->sub_path_off[s], p1 = d->sub_path_off[s + 1];
-        const int g = (int)(p1 - p0);
-        if (fill + g > 32) {
-          while (pl.pword.size() % 32) pl.pword.push_back(kPad | kSubHead);
-          pl.binfo.push_back(make_int4((int)(p0 - pl.path_lo), (int)(s - pl.sub_lo), (int)(j - pl.tree_lo), 0));
-          fill = 0;
-        }
-        for (int64_t i = p0; i < p1; ++i) pl.pword.push_back(pw_path[i - pl.path_lo]);
-        fill += g;
-        pl.binfo.back().w += g;
-      }
-    }
-    while (pl.pword.size() % 32) pl.pword.push_back(kPad | kSubHead);
-    T.nb = (int32_t)pl.binfo.size() - T.b0;
-    // int32 shared-memory accumulation is exact while no window cell-field gets more than
-    // kEventMax events (each |event| <= 2^24); otherwise run the tile against global memory.
-    if (!T.global) {
-      cnt.assign((size_t)3 * T.ww * T.wh, 0);
-      bool ok = true;
-      for (int64_t j = j0; j < j1 && ok; ++j)
-        for (int64_t s = d->tree_sub_off[j]; s < d->tree_sub_off[j + 1] && ok; ++s) {
-          const short4 e = pl.sxy[s - pl.sub_lo];
-          for (int64_t i = d->sub_path_off[s]; i < d->sub_path_off[s + 1] && ok; ++i) {
-            const uint32_t pw = pw_path[i - pl.path_lo];
-            int ex[2], ey[2], fm[2];
-            lane_events(pw & 7u, e.x, e.y, e.z, e.w, (int)(pw >> 16), ex, ey, fm);
-            for (int q = 0; q < 2 && ok; ++q)
-              for (int f = 0; f < 3; ++f)
-                if (fm[q] >> f & 1) {
-                  const size_t c = (size_t)f * T.ww * T.wh + (size_t)(ey[q] - T.wy0) * T.ww + (ex[q] - T.wx0);
-                  if (++cnt[c] > kEventMax) { ok = false; break; }
-                }
-          }
-        }
-      if (!ok) { T.global = 1; T.wx0 = T.wy0 = T.ww = T.wh = 0; }
-    }
-    pl.n_global_tiles += T.global;
-    pl.tiles.push_back(T);
+  // 3. bundles, tile by tile (packing restarts at each tile): count per tile, prefix, then fill the
+  //    tiles in parallel (each tile owns a contiguous bundle range)
+  const int64_t ntile = (int64_t)starts.size() - 1;
+  std::vector<int32_t> tb0(ntile + 1, 0);
+  for (int64_t t = 0; t < ntile; ++t) {
+    int nbt = 0, fill = 32;
+    for (int64_t n = starts[t]; n < starts[t + 1]; ++n) pack_net(n, nbt, fill);
+    tb0[t + 1] = tb0[t] + nbt;
   }
+  pl.binfo.assign(tb0[ntile], make_int4(0, 0, 0, 0));
+  pl.pword.assign((size_t)tb0[ntile] * 32, kPad | kSubHead);
+  pl.tiles.assign(ntile, TileDesc{});
+#pragma omp parallel
+  {
+    std::vector<uint16_t> cnt;
+#pragma omp for schedule(dynamic, 16)
+    for (int64_t t = 0; t < ntile; ++t) {
+      TileDesc T{};
+      T.net0 = (int32_t)(starts[t] - pl.net_lo);
+      T.nnet = (int32_t)(starts[t + 1] - starts[t]);
+      T.tree0 = (int32_t)(d->net_tree_off[starts[t]] - pl.tree_lo);
+      T.ntree = (int32_t)(d->net_tree_off[starts[t + 1]] - d->net_tree_off[starts[t]]);
+      T.b0 = tb0[t];
+      T.nb = tb0[t + 1] - tb0[t];
+      T.global = globs[t];
+      int bx0 = X, by0 = Y, bx1 = -1, by1 = -1;
+      for (int64_t n = starts[t]; n < starts[t + 1]; ++n) {
+        int a0, b0_, a1, b1_;
+        net_box(n, a0, b0_, a1, b1_);
+        bx0 = std::min(bx0, a0); by0 = std::min(by0, b0_); bx1 = std::max(bx1, a1); by1 = std::max(by1, b1_);
+      }
+      T.wx0 = bx0 & ~1; T.wy0 = by0 & ~1;
+      T.ww = (bx1 + 1 - T.wx0 + 1) & ~1; T.wh = (by1 + 1 - T.wy0 + 1) & ~1;
+      if (T.global) { T.wx0 = 0; T.wy0 = 0; T.ww = 0; T.wh = 0; }
+      T.sub0 = (int32_t)(d->tree_sub_off[d->net_tree_off[starts[t]]] - pl.sub_lo);
+      T.nsub = (int32_t)(d->tree_sub_off[d->net_tree_off[starts[t + 1]]] - pl.sub_lo) - T.sub0;
+      int fill = 32, b = T.b0 - 1;
+      const int64_t j0 = d->net_tree_off[starts[t]], j1 = d->net_tree_off[starts[t + 1]];
+      for (int64_t j = j0; j < j1; ++j) {
+        for (int64_t sn = d->tree_sub_off[j]; sn < d->tree_sub_off[j + 1]; ++sn) {
+          const int64_t p0 = d->sub_path_off[sn], p1 = d->sub_path_off[sn + 1];
+          const int g = (int)(p1 - p0);
+          if (fill + g > 32) {
+            ++b;
+            pl.binfo[b] = make_int4((int)(p0 - pl.path_lo), (int)(sn - pl.sub_lo), (int)(j - pl.tree_lo), 0);
+            fill = 0;
+          }
+          for (int64_t i = p0; i < p1; ++i) pl.pword[(size_t)b * 32 + fill + (i - p0)] = pw_path[i - pl.path_lo];
+          fill += g;
+          pl.binfo[b].w += g;
+        }
+      }
+      // int32 shared-memory accumulation is exact while no window cell-field gets more than
+      // kEventMax events (each |event| <= 2^24); otherwise run the tile against global memory.
+      if (!T.global) {
+        cnt.assign((size_t)3 * T.ww * T.wh, 0);
+        bool ok = true;
+        for (int64_t j = j0; j < j1 && ok; ++j)
+          for (int64_t sn = d->tree_sub_off[j]; sn < d->tree_sub_off[j + 1] && ok; ++sn) {
+            const short4 e = pl.sxy[sn - pl.sub_lo];
+            for (int64_t i = d->sub_path_off[sn]; i < d->sub_path_off[sn + 1] && ok; ++i) {
+              const uint32_t pw = pw_path[i - pl.path_lo];
+              int ex[2], ey[2], fm[2];
+              lane_events(pw & 7u, e.x, e.y, e.z, e.w, (int)(pw >> 16), ex, ey, fm);
+              for (int q = 0; q < 2 && ok; ++q)
+                for (int f = 0; f < 3; ++f)
+                  if (fm[q] >> f & 1) {
+                    const size_t c = (size_t)f * T.ww * T.wh + (size_t)(ey[q] - T.wy0) * T.ww + (ex[q] - T.wx0);
+                    if (++cnt[c] > kEventMax) { ok = false; break; }
+                  }
+            }
+          }
+        if (!ok) { T.global = 1; T.wx0 = T.wy0 = T.ww = T.wh = 0; }
+      }
+      pl.tiles[t] = T;
+    }
+  }
+  pl.n_global_tiles = 0;
+  for (const auto& T : pl.tiles) pl.n_global_tiles += T.global;
   pl.nb = (int)pl.binfo.size();
   // pipelined tiles (shared-memory window, <= kTargetBundles bundles) first, then the rest
   auto pipelined = [](const TileDesc& T) {

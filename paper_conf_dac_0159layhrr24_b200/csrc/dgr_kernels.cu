@@ -922,12 +922,16 @@ __device__ __forceinline__ void flush_scalars(const KParams& P, long long wl, lo
 
 // (a) one tile per CTA: the whole tile arrives by bulk copies on one mbarrier; the event window
 // and noise alias the S window.  4 CTAs per SM overlap one CTA's copies with the others' math.
-constexpr int kBThreads = 256;
+#ifndef DGR_BTHREADS
+#define DGR_BTHREADS 256
+#endif
+constexpr int kBThreads = DGR_BTHREADS;
+constexpr int kBPerSM = 1024 / kBThreads;
 constexpr size_t kBSmemBytes = StageLayout::bytes + 8 * kPipeTrees + 64;
 static_assert(kPEvBytes + 4 * kWinMax <= 2 * 8 * kWinMax, "event window + noise must fit the S window");
 
 template <bool REV, bool FWD>
-__global__ void __launch_bounds__(kBThreads, 4) tile_bulk(KParams P, StepArgs A) {
+__global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepArgs A) {
   extern __shared__ __align__(128) unsigned char smem[];
   Stage St(smem);
   long long* dq_s = reinterpret_cast<long long*>(smem + StageLayout::bytes);
@@ -949,18 +953,18 @@ __global__ void __launch_bounds__(kBThreads, 4) tile_bulk(KParams P, StepArgs A)
   if (threadIdx.x == 0) bulk_wait_read();   // the stage must outlive the bulk stores' reads
 }
 
-// (b) persistent, double-buffered: one CTA per SM, tile i+1 streams into the other stage while
-// tile i computes.
-constexpr int kPThreads = 512;
-constexpr size_t kPSmemBytes = 2 * StageLayout::bytes + kPEvBytes + 4 * kWinMax + 8 * kPipeTrees + 64;
+// (b) persistent, double-buffered: 2 CTAs per SM walk the tiles (blockIdx.x, +gridDim.x, ...); tile
+// i+1 streams into the other stage while tile i computes.  The event window and noise alias the
+// current stage's S window, as in (a).
+constexpr int kPThreads = 256;
+constexpr int kPPerSM = 2;
+constexpr size_t kPSmemBytes = 2 * StageLayout::bytes + 8 * kPipeTrees + 64;
 
 template <bool REV, bool FWD>
-__global__ void __launch_bounds__(kPThreads, 1) tile_persistent(KParams P, StepArgs A) {
+__global__ void __launch_bounds__(kPThreads, kPPerSM) tile_persistent(KParams P, StepArgs A) {
   extern __shared__ __align__(128) unsigned char smem[];
   unsigned char* stage_base[2] = {smem, smem + StageLayout::bytes};
-  int* ev_s = reinterpret_cast<int*>(smem + 2 * StageLayout::bytes);
-  float* g_all = reinterpret_cast<float*>(smem + 2 * StageLayout::bytes + kPEvBytes);
-  long long* dq_s = reinterpret_cast<long long*>(g_all + kWinMax);
+  long long* dq_s = reinterpret_cast<long long*>(smem + 2 * StageLayout::bytes);
   long long* red_s = dq_s + kPipeTrees;
   uint64_t* bars = reinterpret_cast<uint64_t*>(red_s + 2);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -982,7 +986,10 @@ __global__ void __launch_bounds__(kPThreads, 1) tile_persistent(KParams P, StepA
       issue_tile_loads<REV>(P, P.tiles[tile + gridDim.x], stage_base[sidx ^ 1], &bars[sidx ^ 1]);
     }
     mbar_wait(&bars[sidx], (uint32_t)(it >> 1) & 1u);
-    process_tile<REV, FWD, kPThreads>(P, A, P.tiles[tile], Stage(stage_base[sidx]), ev_s, g_all, dq_s, wl, tp);
+    Stage St(stage_base[sidx]);
+    int* ev_s = reinterpret_cast<int*>(St.S);
+    float* g_all = reinterpret_cast<float*>(ev_s + 3 * kWinMax);
+    process_tile<REV, FWD, kPThreads>(P, A, P.tiles[tile], St, ev_s, g_all, dq_s, wl, tp);
     __syncthreads();
   }
   if (FWD) flush_scalars<kPThreads>(P, wl, tp, red_s);
@@ -1334,7 +1341,7 @@ int prepare_kernels() {
 void launch_tiles(const KParams& p, const StepArgs& a, TileMode mode, cudaStream_t s) {
   if (p.ntiles > 0) {
     if (g_persistent) {
-      const int grid = p.ntiles < g_num_sms ? p.ntiles : g_num_sms;
+      const int grid = p.ntiles < kPPerSM * g_num_sms ? p.ntiles : kPPerSM * g_num_sms;
       if (mode == kForwardOnly) tile_persistent<false, true><<<grid, kPThreads, kPSmemBytes, s>>>(p, a);
       else if (mode == kReverseForward) tile_persistent<true, true><<<grid, kPThreads, kPSmemBytes, s>>>(p, a);
       else tile_persistent<true, false><<<grid, kPThreads, kPSmemBytes, s>>>(p, a);

@@ -15,7 +15,7 @@ from dataclasses import dataclass
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-_LIB = os.path.join(_PKG, "libdgr.so")
+_LIB = os.environ.get("DGR_LIB") or os.path.join(_PKG, "libdgr.so")   # DGR_LIB: A/B builds of libdgr
 _lib = None
 
 
