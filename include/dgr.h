@@ -9,8 +9,8 @@
  *   (5) Adam on the logits
  * and dgr_induce is the discrete selection of §4.5 (argmax tree, top-p paths).
  * The readings of the paper this library implements are listed in DESIGN.md §3
- * (grouping = sub-net, f = sigmoid(-s r) / ReLU(-r), beta_v global, sqrt(L) with L = n_layers,
- * Philox4x32-10 noise keyed on (seed, global candidate index, iteration, stream)).
+ * (grouping = sub-net, f of the overflow x = d - cap, beta_v global, sqrt(L) with L = n_layers,
+ * Philox4x32-10 noise keyed on (seed, noise index, iteration, stream); see dgr_forest_desc).
  *
  * Conventions for every entry point
  *   - return int: 0 = DGR_OK, < 0 = error code below; dgr_last_error() (thread-local) says why.
@@ -47,11 +47,20 @@ enum {
   DGR_ESTATE = -5    /* call not valid in the handle's state (e.g. dgr_get_demand before a forward) */
 };
 
-/* Message for the last error on this thread ("" if none). */
+/* Message of the last failed call on this thread; every entry point clears it first ("" = success). */
 const char* dgr_last_error(void);
 
 /* The routing DAG forest F = {T, S, P} of §3.2 as flat CSR arrays, in GLOBAL order.
- * Offsets have length n+1, start at 0 and are non-decreasing; every group is non-empty. */
+ * Offsets have length n+1, start at 0 and are non-decreasing; every group is non-empty.
+ * Path candidates are the straight / L / Z patterns of §3.1: every path must be one of
+ * them for its sub-net (its segments and turning points are checked).  A sub-net whose endpoints
+ * share a row or column has straight candidates only; any other sub-net lists exactly one HV
+ * (horizontal first) and one VH candidate, in that order, then its Z-HVH candidates, then its
+ * Z-VHV candidates (the order forestgen emits); anything else is DGR_EINVAL.
+ * Gumbel noise (Q7): a sub-net whose only candidate is a straight path draws none (its
+ * softmax is identically 1); every other candidate, in global path order, takes the next noise
+ * index n (0, 1, 2, ...) and draws g from Philox4x32-10(key = seed, counter = {n >> 2 (64 bit),
+ * k, 0}) word n & 3; tree j draws from counter {j >> 2, k, 1} word j & 3. */
 typedef struct {
   int32_t X, Y;                           /* grid; 2..32767 each */
   int64_t n_nets, n_trees, n_subnets, n_paths, n_segs, n_tps;

@@ -9,7 +9,9 @@
  * DGR differentiable solver computes, written from the paper (/root/reference/PAPER.md,
  * "P:NNN" = line NNN) in the paper's order and notation:
  *
- *   Gumbel noise g ~ Gumbel(0,1)                 §4.4, P:817-832 (reading Q7: Philox4x32-10)
+ *   Gumbel noise g ~ Gumbel(0,1)                 §4.4, P:817-832 (reading Q7: Philox4x32-10;
+ *                                                  a lone straight candidate draws none, the
+ *                                                  others are numbered in forest order)
  *   p_i = softmax_{subnet(i)}((w_i+g_i)/t)        §4.4, P:820-826 (reading Q1: group = sub-net)
  *   q_j = softmax_{net(j)}((w_j+g_j)/t)           §4.4
  *   d_e = sum_{i in P_e} q p + beta sum_{k in P_v} q p     Eq. (10), P:556-564 (reading Q3)
@@ -102,6 +104,7 @@ typedef struct {
   uint64_t seed;
   /* trainable logits and Adam state */
   real *w_tree, *w_path, *m_tree, *v_tree, *m_path, *v_path;
+  int64_t *nid;               /* noise index of each path, -1 = none (reading Q7) */
   int64_t k;                  /* global iteration counter (noise key; Adam step = k+1) */
   int64_t net_lo, net_hi;     /* shard (all nets by default) */
   /* last forward */
@@ -148,6 +151,15 @@ ODGR_API odgr_state* odgr_new(int32_t X, int32_t Y, int64_t n_nets, int64_t n_tr
   s->w_path = rzeros(n_paths);
   for (int64_t j = 0; j < n_trees; ++j) s->w_tree[j] = w_tree0[j];
   for (int64_t i = 0; i < n_paths; ++i) s->w_path[i] = w_path0[i];
+  /* Reading Q7: a sub-net whose only candidate is a straight path (one segment) draws no noise
+   * (its softmax is 1 whatever the noise); every other candidate takes the next noise index. */
+  s->nid = (int64_t*)malloc(sizeof(int64_t) * (n_paths + 1));
+  int64_t next = 0;
+  for (int64_t sn = 0; sn < n_subnets; ++sn) {
+    int64_t i0 = sub_path_off[sn], i1 = sub_path_off[sn + 1];
+    int lone_straight = (i1 - i0 == 1) && (path_seg_off[i0 + 1] - path_seg_off[i0] == 1);
+    for (int64_t i = i0; i < i1; ++i) s->nid[i] = lone_straight ? -1 : next++;
+  }
   s->m_tree = rzeros(n_trees); s->v_tree = rzeros(n_trees);
   s->m_path = rzeros(n_paths); s->v_path = rzeros(n_paths);
   s->p = rzeros(n_paths); s->q = rzeros(n_trees);
@@ -162,6 +174,7 @@ ODGR_API void odgr_free(odgr_state* s) {
   if (!s) return;
   free(s->net_tree_off); free(s->tree_sub_off); free(s->sub_path_off); free(s->path_seg_off);
   free(s->path_tp_off); free(s->seg); free(s->tp_xy); free(s->cap_h); free(s->cap_v);
+  free(s->nid);
   free(s->w_tree); free(s->w_path); free(s->m_tree); free(s->v_tree); free(s->m_path); free(s->v_path);
   free(s->p); free(s->q); free(s->d_h); free(s->d_v);
   free(s);
@@ -213,7 +226,7 @@ static void forward_partial(odgr_state* s, real t, const odgr_weights* W, int no
         int64_t i0 = s->sub_path_off[sn], i1 = s->sub_path_off[sn + 1];
         real pm = -INFINITY;
         for (int64_t i = i0; i < i1; ++i) {
-          real g = noise ? (real)odgr_gumbel(s->seed, (uint64_t)i, (uint64_t)s->k, 0) : R(0);
+          real g = (noise && s->nid[i] >= 0) ? (real)odgr_gumbel(s->seed, (uint64_t)s->nid[i], (uint64_t)s->k, 0) : R(0);
           real z = (s->w_path[i] + g) / t;
           s->p[i] = z;
           if (z > pm) pm = z;

@@ -181,12 +181,15 @@ bool classify(const dgr_forest_desc* d, int64_t i, int x0, int y0, int x1, int y
 // ---------------------------------------------------------------------------------------
 struct Plan {
   int64_t net_lo = 0, net_hi = 0, tree_lo = 0, tree_hi = 0, sub_lo = 0, sub_hi = 0, path_lo = 0, path_hi = 0;
+  int64_t nid_base = 0;                 // global noise index of the rank's first noisy candidate
   int nb = 0;
   std::vector<int4> binfo;
   std::vector<uint32_t> pword;
-  std::vector<short4> sxy;
+  std::vector<short4> sxy;              // kernel order
   std::vector<int32_t> net_tree_off;
-  std::vector<int64_t> sub_first_path;   // local path index of each local sub-net's first candidate
+  std::vector<int32_t> ksub_csr;        // kernel-order sub-net -> local CSR sub-net
+  std::vector<int64_t> sub_first_slot;  // local CSR sub-net -> slot of its first candidate
+  std::vector<int32_t> slot_path;       // slot -> local CSR path (-1: padding)
   std::vector<TileDesc> tiles;          // pipelined tiles first (see make_plan)
   int64_t n_global_tiles = 0;
   int64_t n_pipe_tiles = 0;
@@ -203,6 +206,26 @@ int lane_events(uint32_t shape, int x0, int y0, int x1, int y1, int m, int ex[2]
     case kZHVH: ex[0] = m; ey[0] = y0; fm[0] = 7; ex[1] = m; ey[1] = y1; fm[1] = 7; return 2;
     default: ex[0] = x0; ey[0] = m; fm[0] = 7; ex[1] = x1; ey[1] = m; fm[1] = 7; return 2;
   }
+}
+
+// A sub-net whose only candidate is one segment draws no noise and needs no softmax (Q7).
+inline bool lone_straight(const dgr_forest_desc* d, int64_t s) {
+  const int64_t p0 = d->sub_path_off[s];
+  return d->sub_path_off[s + 1] - p0 == 1 && d->path_seg_off[p0 + 1] - d->path_seg_off[p0] == 1;
+}
+
+// Candidate order the forward's event collapse relies on (dgr.h): straight only if aligned, else
+// HV, VH, Z-HVH..., Z-VHV...
+inline bool canonical_group(const uint32_t* shapes, int n, bool aligned) {
+  if (aligned) {
+    for (int i = 0; i < n; ++i) if (shapes[i] != kStraightH && shapes[i] != kStraightV) return false;
+    return true;
+  }
+  if (n < 2 || shapes[0] != kHV || shapes[1] != kVH) return false;
+  int i = 2;
+  while (i < n && shapes[i] == kZHVH) ++i;
+  while (i < n && shapes[i] == kZVHV) ++i;
+  return i == n;
 }
 
 int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
@@ -222,13 +245,18 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   const int X = d->X, Y = d->Y;
   pl.net_tree_off.resize(nn + 1);
   for (int64_t n = 0; n <= nn; ++n) pl.net_tree_off[n] = (int32_t)(d->net_tree_off[pl.net_lo + n] - pl.tree_lo);
-  pl.sxy.resize(ns);
-  pl.sub_first_path.resize(ns);
+  // noise indices: the candidates of earlier ranks' nets that draw noise
+  {
+    int64_t cnt = 0;
+#pragma omp parallel for schedule(static) reduction(+ : cnt)
+    for (int64_t s = 0; s < pl.sub_lo; ++s) cnt += lone_straight(d, s) ? 0 : d->sub_path_off[s + 1] - d->sub_path_off[s];
+    pl.nid_base = cnt;
+  }
   // 1. canonical sub-net endpoints + pattern words of every local candidate (parallel over
   //    sub-nets; the first failing sub-net, in index order, is reported)
+  std::vector<short4> sxy_csr(ns);
   std::vector<uint32_t> pw_path((size_t)(pl.path_hi - pl.path_lo));
-  std::vector<char> first_of_tree((size_t)ns, 0);
-  for (int64_t j = pl.tree_lo; j < pl.tree_hi; ++j) first_of_tree[d->tree_sub_off[j] - pl.sub_lo] = 1;
+  std::vector<char> single((size_t)ns, 0);
   int64_t bad_sub = ns;   // smallest failing local sub-net
 #pragma omp parallel for schedule(dynamic, 4096) reduction(min : bad_sub)
   for (int64_t ls = 0; ls < ns; ++ls) {
@@ -240,23 +268,22 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       bad_sub = std::min(bad_sub, ls);
       continue;
     }
-    pl.sxy[ls] = make_short4((short)x0, (short)y0, (short)x1, (short)y1);
+    sxy_csr[ls] = make_short4((short)x0, (short)y0, (short)x1, (short)y1);
     const int64_t p0 = d->sub_path_off[s], p1 = d->sub_path_off[s + 1];
-    pl.sub_first_path[ls] = p0 - pl.path_lo;
-    for (int64_t i = p0; i < p1; ++i) {
+    uint32_t shapes[32];
+    bool ok = true;
+    for (int64_t i = p0; i < p1 && ok; ++i) {
       uint32_t shape;
       int mid;
-      if (!classify(d, i, x0, y0, x1, y1, &shape, &mid)) {
-        bad_sub = std::min(bad_sub, ls);
-        break;
-      }
-      uint32_t pw = shape | ((uint32_t)mid << 16);
-      if (i == p0) {
-        pw |= kSubHead;
-        if (first_of_tree[ls]) pw |= kTreeHead;
-      }
-      pw_path[i - pl.path_lo] = pw;
+      if (!classify(d, i, x0, y0, x1, y1, &shape, &mid)) { ok = false; break; }
+      shapes[i - p0] = shape;
+      pw_path[i - pl.path_lo] = shape | ((uint32_t)mid << 16);
     }
+    if (!ok || !canonical_group(shapes, (int)(p1 - p0), x0 == x1 || y0 == y1)) {
+      bad_sub = std::min(bad_sub, ls);
+      continue;
+    }
+    single[ls] = (p1 - p0 == 1) && (shapes[0] == kStraightH || shapes[0] == kStraightV);
   }
   if (bad_sub < ns) {
     const int64_t s = pl.sub_lo + bad_sub;
@@ -273,33 +300,46 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
         return fail(DGR_EINVAL, "path %lld is not a straight/L/Z pattern of sub-net %lld (or its turning points are wrong)",
                     (long long)i, (long long)s);
     }
+    return fail(DGR_EINVAL, "sub-net %lld: candidates must be straight (aligned sub-net) or HV, VH, Z-HVH..., Z-VHV... in this order",
+                (long long)s);
+  }
+  // local noise index of every sub-net's first candidate (-1 for lone straight paths)
+  std::vector<int64_t> nid_sub((size_t)ns);
+  {
+    int64_t next = 0;
+    for (int64_t ls = 0; ls < ns; ++ls) {
+      const int64_t g = d->sub_path_off[pl.sub_lo + ls + 1] - d->sub_path_off[pl.sub_lo + ls];
+      nid_sub[ls] = single[ls] ? -1 : next;
+      next += single[ls] ? 0 : g;
+    }
   }
   // 2. tiles of whole nets: greedy in net order while the window (union of the nets' sub-net boxes
-  //    plus a 1-cell halo) stays <= kWinMax cells, the bundles <= kTargetBundles, trees <= kTreeMax.
-  //    A net that alone exceeds the window forms a "global" tile.
+  //    plus a 1-cell halo) stays <= kWinMax cells, the group bundles <= kTargetBundles and all
+  //    bundles <= kTileBundles, trees <= kPipeTrees, sub-nets <= kPipeSubs.  A net that alone
+  //    exceeds the window forms a "global" tile.
   pl.tiles.clear();
   pl.binfo.clear();
   pl.pword.clear();
-  struct Cur { bool open = false; int64_t net0 = 0; int nb = 0, fill = 32, ntree = 0, nsub = 0; int bx0 = 0, by0 = 0, bx1 = -1, by1 = -1; bool global = false; } cur;
-  std::vector<int64_t> tile_net0;
-  std::vector<char> tile_glob;
+  struct Pack { int nbg = 0, fill = 32, nsing = 0; int total() const { return nbg + (nsing + 31) / 32; } };
+  struct Cur { bool open = false; int64_t net0 = 0; Pack pk; int ntree = 0, nsub = 0; int bx0 = 0, by0 = 0, bx1 = -1, by1 = -1; bool global = false; } cur;
   auto net_box = [&](int64_t n, int& bx0, int& by0, int& bx1, int& by1) {
     bx0 = X; by0 = Y; bx1 = -1; by1 = -1;
     const int64_t s0 = d->tree_sub_off[d->net_tree_off[n]], s1 = d->tree_sub_off[d->net_tree_off[n + 1]];
     for (int64_t s = s0; s < s1; ++s) {
-      const short4 e = pl.sxy[s - pl.sub_lo];
+      const short4 e = sxy_csr[s - pl.sub_lo];
       bx0 = std::min<int>(bx0, e.x); bx1 = std::max<int>(bx1, e.z);
       by0 = std::min<int>(by0, std::min(e.y, e.w)); by1 = std::max<int>(by1, std::max(e.y, e.w));
     }
     bx0 = std::max(0, bx0 - 1); by0 = std::max(0, by0 - 1);
     bx1 = std::min(X - 1, bx1 + 1); by1 = std::min(Y - 1, by1 + 1);
   };
-  auto pack_net = [&](int64_t n, int& nb, int& fill) {   // bundle packing of one net's groups
+  auto pack_net = [&](int64_t n, Pack& pk) {   // bundle packing of one net's sub-nets
     const int64_t s0 = d->tree_sub_off[d->net_tree_off[n]], s1 = d->tree_sub_off[d->net_tree_off[n + 1]];
     for (int64_t s = s0; s < s1; ++s) {
+      if (single[s - pl.sub_lo]) { ++pk.nsing; continue; }
       const int g = (int)(d->sub_path_off[s + 1] - d->sub_path_off[s]);
-      if (fill + g > 32) { ++nb; fill = 0; }
-      fill += g;
+      if (pk.fill + g > 32) { ++pk.nbg; pk.fill = 0; }
+      pk.fill += g;
     }
   };
   // windows start on even cells and have even extents so their S rows / columns are 16-byte
@@ -318,20 +358,20 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     const int ntree = (int)(d->net_tree_off[n + 1] - d->net_tree_off[n]);
     const int nsub = (int)(d->tree_sub_off[d->net_tree_off[n + 1]] - d->tree_sub_off[d->net_tree_off[n]]);
     bool fits = cur.open && !cur.global && !big;
-    int nb2 = cur.nb, fill2 = cur.fill;
+    Pack pk2 = cur.pk;
     if (fits) {
       const int ux0 = std::min(cur.bx0, bx0), uy0 = std::min(cur.by0, by0);
       const int ux1 = std::max(cur.bx1, bx1), uy1 = std::max(cur.by1, by1);
-      pack_net(n, nb2, fill2);
-      fits = aligned_area(ux0, uy0, ux1, uy1) <= kWinMax && nb2 <= kTargetBundles &&
+      pack_net(n, pk2);
+      fits = aligned_area(ux0, uy0, ux1, uy1) <= kWinMax && pk2.nbg <= kTargetBundles && pk2.total() <= kTileBundles &&
              cur.ntree + ntree <= kPipeTrees && cur.nsub + nsub <= kPipeSubs;
       if (fits) { cur.bx0 = ux0; cur.by0 = uy0; cur.bx1 = ux1; cur.by1 = uy1; }
     } else if (cur.open && cur.global && big) {
-      pack_net(n, nb2, fill2);
-      fits = nb2 <= kMaxBundles && cur.ntree + ntree <= kTreeMax;
+      pack_net(n, pk2);
+      fits = pk2.total() <= kMaxBundles && cur.ntree + ntree <= kTreeMax;
     }
     if (fits) {
-      cur.nb = nb2; cur.fill = fill2; cur.ntree += ntree; cur.nsub += nsub;
+      cur.pk = pk2; cur.ntree += ntree; cur.nsub += nsub;
       continue;
     }
     // close the open tile, open a new one at net n
@@ -340,22 +380,30 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     cur = Cur();
     cur.open = true; cur.global = big; cur.net0 = n; cur.ntree = ntree; cur.nsub = nsub;
     cur.bx0 = bx0; cur.by0 = by0; cur.bx1 = bx1; cur.by1 = by1;
-    cur.nb = 0; cur.fill = 32;
-    pack_net(n, cur.nb, cur.fill);
-    if (cur.nb > kMaxBundles) return fail(DGR_EINVAL, "net %lld needs %d > %d bundles", (long long)n, cur.nb, kMaxBundles);
+    pack_net(n, cur.pk);
+    if (cur.pk.total() > kMaxBundles)
+      return fail(DGR_EINVAL, "net %lld needs %d > %d bundles", (long long)n, cur.pk.total(), kMaxBundles);
+    if (ntree > kTreeMax) return fail(DGR_EINVAL, "net %lld has %d > %d trees", (long long)n, ntree, kTreeMax);
   }
   starts.push_back(pl.net_hi);
-  // 3. bundles, tile by tile (packing restarts at each tile): count per tile, prefix, then fill the
-  //    tiles in parallel (each tile owns a contiguous bundle range)
+  // 3. bundles, tile by tile: the tile's group bundles (packing restarts at each tile), then its
+  //    singleton bundles; sub-nets renumbered in that order ("kernel order").  Count per tile,
+  //    prefix, then fill the tiles in parallel (each owns a contiguous bundle and sub-net range).
   const int64_t ntile = (int64_t)starts.size() - 1;
-  std::vector<int32_t> tb0(ntile + 1, 0);
+  std::vector<int32_t> tb0(ntile + 1, 0), tbg(ntile, 0);
   for (int64_t t = 0; t < ntile; ++t) {
-    int nbt = 0, fill = 32;
-    for (int64_t n = starts[t]; n < starts[t + 1]; ++n) pack_net(n, nbt, fill);
-    tb0[t + 1] = tb0[t] + nbt;
+    Pack pk;
+    for (int64_t n = starts[t]; n < starts[t + 1]; ++n) pack_net(n, pk);
+    tbg[t] = pk.nbg;
+    tb0[t + 1] = tb0[t] + pk.total();
   }
+  const size_t nslot = (size_t)tb0[ntile] * 32;
   pl.binfo.assign(tb0[ntile], make_int4(0, 0, 0, 0));
-  pl.pword.assign((size_t)tb0[ntile] * 32, kPad | kSubHead);
+  pl.pword.assign(nslot, kPad | kSubHead);
+  pl.slot_path.assign(nslot, -1);
+  pl.sxy.resize(ns);
+  pl.ksub_csr.resize(ns);
+  pl.sub_first_slot.resize(ns);
   pl.tiles.assign(ntile, TileDesc{});
 #pragma omp parallel
   {
@@ -369,6 +417,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       T.ntree = (int32_t)(d->net_tree_off[starts[t + 1]] - d->net_tree_off[starts[t]]);
       T.b0 = tb0[t];
       T.nb = tb0[t + 1] - tb0[t];
+      T.nbg = tbg[t];
       T.global = globs[t];
       int bx0 = X, by0 = Y, bx1 = -1, by1 = -1;
       for (int64_t n = starts[t]; n < starts[t + 1]; ++n) {
@@ -381,20 +430,68 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       if (T.global) { T.wx0 = 0; T.wy0 = 0; T.ww = 0; T.wh = 0; }
       T.sub0 = (int32_t)(d->tree_sub_off[d->net_tree_off[starts[t]]] - pl.sub_lo);
       T.nsub = (int32_t)(d->tree_sub_off[d->net_tree_off[starts[t + 1]]] - pl.sub_lo) - T.sub0;
-      int fill = 32, b = T.b0 - 1;
       const int64_t j0 = d->net_tree_off[starts[t]], j1 = d->net_tree_off[starts[t + 1]];
+      int ks = T.sub0;   // next kernel-order sub-net
+      // group bundles
+      int fill = 32, b = T.b0 - 1, prev_tree = -1;
       for (int64_t j = j0; j < j1; ++j) {
+        const int toff = (int)(j - pl.tree_lo) - T.tree0;
         for (int64_t sn = d->tree_sub_off[j]; sn < d->tree_sub_off[j + 1]; ++sn) {
+          const int64_t ls = sn - pl.sub_lo;
+          if (single[ls]) continue;
           const int64_t p0 = d->sub_path_off[sn], p1 = d->sub_path_off[sn + 1];
           const int g = (int)(p1 - p0);
           if (fill + g > 32) {
             ++b;
-            pl.binfo[b] = make_int4((int)(p0 - pl.path_lo), (int)(sn - pl.sub_lo), (int)(j - pl.tree_lo), 0);
+            pl.binfo[b] = make_int4((int)nid_sub[ls], ks, T.tree0, 0);
             fill = 0;
+            prev_tree = -1;
           }
-          for (int64_t i = p0; i < p1; ++i) pl.pword[(size_t)b * 32 + fill + (i - p0)] = pw_path[i - pl.path_lo];
+          pl.sxy[ks] = sxy_csr[ls];
+          pl.ksub_csr[ks] = (int32_t)ls;
+          pl.sub_first_slot[ls] = (int64_t)b * 32 + fill;
+          for (int64_t i = p0; i < p1; ++i) {
+            uint32_t pw = pw_path[i - pl.path_lo] | ((uint32_t)toff << kTreeShift);
+            if (i == p0) {
+              pw |= kSubHead;
+              if (toff != prev_tree) pw |= kTreeHead;
+            }
+            const size_t slot = (size_t)b * 32 + fill + (i - p0);
+            pl.pword[slot] = pw;
+            pl.slot_path[slot] = (int32_t)(i - pl.path_lo);
+          }
+          prev_tree = toff;
           fill += g;
           pl.binfo[b].w += g;
+          ++ks;
+        }
+      }
+      // singleton bundles
+      int lane = 32;
+      b = T.b0 + T.nbg - 1;
+      for (int64_t j = j0; j < j1; ++j) {
+        const int toff = (int)(j - pl.tree_lo) - T.tree0;
+        for (int64_t sn = d->tree_sub_off[j]; sn < d->tree_sub_off[j + 1]; ++sn) {
+          const int64_t ls = sn - pl.sub_lo;
+          if (!single[ls]) continue;
+          if (lane == 32) {
+            ++b;
+            pl.binfo[b] = make_int4(0, ks, T.tree0, kSingleBundle);
+            lane = 0;
+            prev_tree = -1;
+          }
+          pl.sxy[ks] = sxy_csr[ls];
+          pl.ksub_csr[ks] = (int32_t)ls;
+          const int64_t p0 = d->sub_path_off[sn];
+          const size_t slot = (size_t)b * 32 + lane;
+          pl.sub_first_slot[ls] = (int64_t)slot;
+          pl.pword[slot] = pw_path[p0 - pl.path_lo] | ((uint32_t)toff << kTreeShift) | kSubHead |
+                           (toff != prev_tree ? kTreeHead : 0u);
+          pl.slot_path[slot] = (int32_t)(p0 - pl.path_lo);
+          prev_tree = toff;
+          ++lane;
+          pl.binfo[b].w += 1;
+          ++ks;
         }
       }
       // int32 shared-memory accumulation is exact while no window cell-field gets more than
@@ -402,21 +499,20 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       if (!T.global) {
         cnt.assign((size_t)3 * T.ww * T.wh, 0);
         bool ok = true;
-        for (int64_t j = j0; j < j1 && ok; ++j)
-          for (int64_t sn = d->tree_sub_off[j]; sn < d->tree_sub_off[j + 1] && ok; ++sn) {
-            const short4 e = pl.sxy[sn - pl.sub_lo];
-            for (int64_t i = d->sub_path_off[sn]; i < d->sub_path_off[sn + 1] && ok; ++i) {
-              const uint32_t pw = pw_path[i - pl.path_lo];
-              int ex[2], ey[2], fm[2];
-              lane_events(pw & 7u, e.x, e.y, e.z, e.w, (int)(pw >> 16), ex, ey, fm);
-              for (int q = 0; q < 2 && ok; ++q)
-                for (int f = 0; f < 3; ++f)
-                  if (fm[q] >> f & 1) {
-                    const size_t c = (size_t)f * T.ww * T.wh + (size_t)(ey[q] - T.wy0) * T.ww + (ex[q] - T.wx0);
-                    if (++cnt[c] > kEventMax) { ok = false; break; }
-                  }
-            }
+        for (int64_t sn = d->tree_sub_off[j0]; sn < d->tree_sub_off[j1] && ok; ++sn) {
+          const short4 e = sxy_csr[sn - pl.sub_lo];
+          for (int64_t i = d->sub_path_off[sn]; i < d->sub_path_off[sn + 1] && ok; ++i) {
+            const uint32_t pw = pw_path[i - pl.path_lo];
+            int ex[2], ey[2], fm[2];
+            lane_events(pw & 7u, e.x, e.y, e.z, e.w, (int)(pw >> 16), ex, ey, fm);
+            for (int q = 0; q < 2 && ok; ++q)
+              for (int f = 0; f < 3; ++f)
+                if (fm[q] >> f & 1) {
+                  const size_t c = (size_t)f * T.ww * T.wh + (size_t)(ey[q] - T.wy0) * T.ww + (ex[q] - T.wx0);
+                  if (++cnt[c] > kEventMax) { ok = false; break; }
+                }
           }
+        }
         if (!ok) { T.global = 1; T.wx0 = T.wy0 = T.ww = T.wh = 0; }
       }
       pl.tiles[t] = T;
@@ -425,9 +521,9 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   pl.n_global_tiles = 0;
   for (const auto& T : pl.tiles) pl.n_global_tiles += T.global;
   pl.nb = (int)pl.binfo.size();
-  // pipelined tiles (shared-memory window, <= kTargetBundles bundles) first, then the rest
+  // pipelined tiles (shared-memory window and stage) first, then the rest
   auto pipelined = [](const TileDesc& T) {
-    return !T.global && T.nb <= kTargetBundles && T.ntree <= kPipeTrees && T.nsub <= kPipeSubs;
+    return !T.global && T.nbg <= kTargetBundles && T.nb <= kTileBundles && T.ntree <= kPipeTrees && T.nsub <= kPipeSubs;
   };
   std::stable_partition(pl.tiles.begin(), pl.tiles.end(), pipelined);
   pl.n_pipe_tiles = 0;
@@ -439,7 +535,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
 // workspace layout
 // ---------------------------------------------------------------------------------------
 struct Layout {
-  size_t tiles, binfo, pword, sxy, wp, mp, vp, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
+  size_t tiles, binfo, pword, sxy, slot_path, wp, mp, vp, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
       partial, loss, chosen, tree_choice, route, nsize, nucleus_tmp, DHVC, iscal, ipartial, metrics, total;
   size_t xcount;   // int64 elements in the exchange buffer
 };
@@ -454,6 +550,7 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.binfo = take(sizeof(int4) * pl.nb);
   L.pword = take(4 * slots);
   L.sxy = take(8 * ns + 16);
+  L.slot_path = take(4 * slots);
   L.wp = take(4 * slots);
   L.mp = take(4 * slots);
   L.vp = take(4 * slots);
@@ -536,6 +633,7 @@ extern "C" {
 const char* dgr_last_error(void) { return g_err.c_str(); }
 
 int dgr_nccl_unique_id(void* out128) {
+  g_err.clear();
   if (!out128) return fail(DGR_EINVAL, "out is NULL");
   static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
   ncclUniqueId id;
@@ -545,6 +643,7 @@ int dgr_nccl_unique_id(void* out128) {
 }
 
 int dgr_partition(const dgr_forest_desc* desc, int32_t world, int64_t* out) {
+  g_err.clear();
   int rc = validate_structure(desc);
   if (rc) return rc;
   if (!out) return fail(DGR_EINVAL, "out is NULL");
@@ -567,6 +666,7 @@ static int dist_args(const dgr_dist* dist, int* rank, int* world) {
 }
 
 int64_t dgr_workspace_size(const dgr_forest_desc* desc, const dgr_dist* dist) {
+  g_err.clear();
   int rank, world;
   if (dist_args(dist, &rank, &world)) return 0;
   Plan pl;
@@ -579,6 +679,7 @@ int64_t dgr_workspace_size(const dgr_forest_desc* desc, const dgr_dist* dist) {
 
 int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev_workspace, int64_t workspace_bytes,
                     void* cuda_stream, dgr_handle** out) {
+  g_err.clear();
   if (!out) return fail(DGR_EINVAL, "out is NULL");
   *out = nullptr;
   int rank, world, rc;
@@ -613,10 +714,12 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
   P.n_nets_l = (int32_t)(pl.net_hi - pl.net_lo);
   P.path_base = pl.path_lo;
   P.tree_base = pl.tree_lo;
+  P.nid_base = pl.nid_base;
   P.seed = desc->seed;
   P.binfo = (const int4*)(ws + L.binfo);
   P.pword = (const uint32_t*)(ws + L.pword);
   P.sxy = (const short4*)(ws + L.sxy);
+  P.slot_path = (const int32_t*)(ws + L.slot_path);
   P.wp = (float*)(ws + L.wp); P.mp = (float*)(ws + L.mp); P.vp = (float*)(ws + L.vp);
   P.pp = (float*)(ws + L.pp);
   P.net_tree_off = (const int32_t*)(ws + L.nto);
@@ -650,9 +753,12 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
   if (cudaMemsetAsync(ws, 0, L.total, s) != cudaSuccess) return cleanup(fail(DGR_ECUDA, "memset workspace failed"));
   // host-side staging of the encoded shard
   const size_t slots = (size_t)pl.nb * 32;
-  std::vector<float> wslots(slots, 0.f);
-  for (int b = 0; b < pl.nb; ++b)
-    for (int l = 0; l < pl.binfo[b].w; ++l) wslots[(size_t)b * 32 + l] = desc->w_path0[pl.path_lo + pl.binfo[b].x + l];
+  std::vector<float> wslots(slots, 0.f), pslots(slots, 0.f);
+  for (size_t sl = 0; sl < slots; ++sl)
+    if (pl.slot_path[sl] >= 0) {
+      wslots[sl] = desc->w_path0[pl.path_lo + pl.slot_path[sl]];
+      pslots[sl] = 1.f;   // p of a lone straight candidate (never rewritten by the pipelined kernel)
+    }
   std::vector<float> capVT(G);
   for (int y = 0; y < desc->Y; ++y)
     for (int x = 0; x < desc->X; ++x) capVT[(size_t)x * desc->Y + y] = desc->cap_v[(size_t)y * desc->X + x];
@@ -666,6 +772,8 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
   cp(L.pword, pl.pword.data(), 4 * slots);
   cp(L.sxy, pl.sxy.data(), 8 * pl.sxy.size());
   cp(L.wp, wslots.data(), 4 * slots);
+  cp(L.pp, pslots.data(), 4 * slots);
+  cp(L.slot_path, pl.slot_path.data(), 4 * slots);
   cp(L.nto, pl.net_tree_off.data(), 4 * pl.net_tree_off.size());
   cp(L.wt, desc->w_tree0 + pl.tree_lo, 4 * nt);
   cp(L.capH, desc->cap_h, 4 * G);
@@ -685,6 +793,7 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
 }
 
 int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w, dgr_loss* last) {
+  g_err.clear();
   if (!h || !w) return fail(DGR_EINVAL, "NULL handle or weights");
   if (iters < 0) return fail(DGR_EINVAL, "iters < 0");
   if (!(temperature > 0.f) || !std::isfinite(temperature)) return fail(DGR_EINVAL, "temperature must be > 0");
@@ -753,6 +862,7 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
 }
 
 int dgr_get_demand(dgr_handle* h, float* d_h, float* d_v) {
+  g_err.clear();
   if (!h || !d_h || !d_v) return fail(DGR_EINVAL, "NULL argument");
   if (!h->have_forward) return fail(DGR_ESTATE, "no forward has run yet");
   const size_t G = (size_t)h->X * h->Y;
@@ -766,14 +876,15 @@ int dgr_get_demand(dgr_handle* h, float* d_h, float* d_v) {
 }
 
 int dgr_get_logits(dgr_handle* h, float* w_tree, float* w_path) {
+  g_err.clear();
   if (!h) return fail(DGR_EINVAL, "NULL handle");
   const Plan& pl = h->plan;
   if (w_path) {
     std::vector<float> slots((size_t)pl.nb * 32);
     CUDA_TRY(cudaMemcpyAsync(slots.data(), h->P.wp, 4 * slots.size(), cudaMemcpyDeviceToHost, h->stream));
     CUDA_TRY(cudaStreamSynchronize(h->stream));
-    for (int b = 0; b < pl.nb; ++b)
-      for (int l = 0; l < pl.binfo[b].w; ++l) w_path[pl.path_lo + pl.binfo[b].x + l] = slots[(size_t)b * 32 + l];
+    for (size_t sl = 0; sl < slots.size(); ++sl)
+      if (pl.slot_path[sl] >= 0) w_path[pl.path_lo + pl.slot_path[sl]] = slots[sl];
   }
   if (w_tree) {
     CUDA_TRY(cudaMemcpyAsync(w_tree + pl.tree_lo, h->P.wt, 4 * (size_t)(pl.tree_hi - pl.tree_lo),
@@ -785,6 +896,7 @@ int dgr_get_logits(dgr_handle* h, float* w_tree, float* w_path) {
 
 int dgr_induce(dgr_handle* h, float top_p, int32_t* tree_choice, int32_t* route, int64_t* nucleus_off,
                int32_t* nucleus, int32_t* D_h, int32_t* D_v, double metrics[5]) {
+  g_err.clear();
   if (!h || !tree_choice || !route || !nucleus_off || !nucleus || !D_h || !D_v || !metrics)
     return fail(DGR_EINVAL, "NULL argument");
   if (!(top_p >= 0.f) || !std::isfinite(top_p)) return fail(DGR_EINVAL, "top_p must be finite and >= 0");
@@ -817,14 +929,19 @@ int dgr_induce(dgr_handle* h, float top_p, int32_t* tree_choice, int32_t* route,
     std::fill(route, route + h->n_subnets, -1);
   }
   std::copy(tc.begin(), tc.end(), tree_choice + pl.net_lo);
-  std::copy(rt.begin(), rt.end(), route + pl.sub_lo);
+  // route / nsize come in kernel sub-net order; nucleus_tmp holds each sub-net's nucleus in rank
+  // order from its first candidate's slot on
+  std::vector<int32_t> nsz_csr(ns);
+  for (int64_t ks = 0; ks < ns; ++ks) {
+    route[pl.sub_lo + pl.ksub_csr[ks]] = rt[ks];
+    nsz_csr[pl.ksub_csr[ks]] = nsz[ks];
+  }
   int64_t pos = 0;
   nucleus_off[0] = 0;
-  // nucleus_tmp holds each sub-net's nucleus in rank order at its first candidate's local index
   for (int64_t sg = 0; sg < h->n_subnets; ++sg) {
     if (sg >= pl.sub_lo && sg < pl.sub_hi) {
       const int64_t ls = sg - pl.sub_lo;
-      for (int r = 0; r < nsz[ls]; ++r) nucleus[pos++] = nuc[(size_t)pl.sub_first_path[ls] + r];
+      for (int r = 0; r < nsz_csr[ls]; ++r) nucleus[pos++] = nuc[(size_t)pl.sub_first_slot[ls] + r];
     }
     nucleus_off[sg + 1] = pos;
   }
@@ -832,6 +949,7 @@ int dgr_induce(dgr_handle* h, float top_p, int32_t* tree_choice, int32_t* route,
 }
 
 int dgr_get_info(dgr_handle* h, int64_t info[12]) {
+  g_err.clear();
   if (!h || !info) return fail(DGR_EINVAL, "NULL argument");
   info[0] = h->k; info[1] = h->plan.net_lo; info[2] = h->plan.net_hi; info[3] = h->plan.nb;
   info[4] = (int64_t)h->plan.nb * 32; info[5] = (int64_t)h->lay.total; info[6] = h->world; info[7] = h->rank;
@@ -840,6 +958,7 @@ int dgr_get_info(dgr_handle* h, int64_t info[12]) {
 }
 
 int dgr_plan_info(const dgr_forest_desc* desc, const dgr_dist* dist, int64_t out[8]) {
+  g_err.clear();
   if (!out) return fail(DGR_EINVAL, "out is NULL");
   int rank, world, rc;
   if ((rc = dist_args(dist, &rank, &world))) return rc;
@@ -849,7 +968,7 @@ int dgr_plan_info(const dgr_forest_desc* desc, const dgr_dist* dist, int64_t out
   for (const auto& T : pl.tiles) {
     maxw = std::max<int64_t>(maxw, (int64_t)T.ww * T.wh);
     if (T.global)
-      for (int b = T.b0; b < T.b0 + T.nb; ++b) gpaths += pl.binfo[b].w;
+      for (int b = T.b0; b < T.b0 + T.nb; ++b) gpaths += pl.binfo[b].w & 0xff;
   }
   dgr::KParams tmp{};
   tmp.X = desc->X;
@@ -861,6 +980,7 @@ int dgr_plan_info(const dgr_forest_desc* desc, const dgr_dist* dist, int64_t out
 }
 
 int dgr_profile(dgr_handle* h, int32_t enable) {
+  g_err.clear();
   if (!h) return fail(DGR_EINVAL, "NULL handle");
   h->prof = enable != 0;
   h->ev_used = 0;
@@ -868,6 +988,7 @@ int dgr_profile(dgr_handle* h, int32_t enable) {
 }
 
 int dgr_profile_read(dgr_handle* h, double ms[8], int64_t launches[8]) {
+  g_err.clear();
   if (!h || !ms || !launches) return fail(DGR_EINVAL, "NULL argument");
   CUDA_TRY(cudaStreamSynchronize(h->stream));
   for (int i = 0; i < 8; ++i) { ms[i] = 0.0; launches[i] = 0; }
@@ -883,6 +1004,7 @@ int dgr_profile_read(dgr_handle* h, double ms[8], int64_t launches[8]) {
 }
 
 int dgr_free(dgr_handle* h) {
+  g_err.clear();
   if (!h) return DGR_OK;
   if (h->stream) cudaStreamSynchronize(h->stream);
   for (auto e : h->ev) cudaEventDestroy(e);

@@ -2,17 +2,23 @@
 //
 // Layout in HBM:
 //   * candidates live in 32-slot "bundles": one warp processes one bundle, one lane one path
-//     candidate.  A bundle holds whole sub-nets (groups of 1..32 candidates, packed in order,
-//     never split), so the sub-net softmax is a segmented warp reduction.  Unused tail lanes
-//     are padding (shape PAD).
+//     candidate.  A "group" bundle holds whole sub-nets (groups of 1..32 candidates, packed in
+//     order, never split), so the sub-net softmax is a segmented warp reduction.  Sub-nets whose
+//     only candidate is a straight path ("singletons": p = 1 identically, no logit update) are
+//     packed 32 to a "singleton" bundle and skip noise, softmax and Adam.  Unused tail lanes are
+//     padding (shape PAD).
 //   * bundles are grouped into "tiles": whole nets whose candidates all lie inside one small
 //     G-cell window (<= kWinMax cells incl. a 1-cell halo).  One CTA owns one tile: it stages the
 //     tile's window of the gradient prefix sums in shared memory for the reverse pass, keeps the
 //     tile's tree state (dq, q) in shared memory, and accumulates the tile's demand events in a
 //     shared-memory window that it flushes once to the global difference arrays.  Tiles whose
 //     nets span a larger window run the same code against global memory ("global" tiles).
-//   * per slot:    pword (shape | flags | mid), w, m, v (fp32), p of the last forward (fp32)
-//   * per bundle:  {first local path, first local sub-net, first local tree, #valid lanes}
+//     A tile's bundles are its group bundles, then its singleton bundles; its sub-nets are stored
+//     in that "kernel order" too (a permutation of the tile's sub-net range).
+//   * per slot:    pword (shape | flags | tree offset | mid), w, m, v (fp32), p of the last
+//     forward (fp32)
+//   * per bundle:  {noise index of lane 0, first kernel-order sub-net, the tile's first tree,
+//     #valid lanes | kSingleBundle}
 //   * per sub-net: canonical endpoints (x0 <= x1; y0 < y1 if x0 == x1) as int16 x 4
 //   * per tree:    w, m, v, q (fp32)
 //   * grids: difference arrays of the wire demand along H rows ([Y][X]) and along V columns
@@ -33,26 +39,33 @@ constexpr double kDqInv = 1.0 / 4294967296.0;
 constexpr int kTileThreads = 256;                  // 8 warps per tile CTA
 constexpr int kWinMax = 1536;                      // window cells per tile
 constexpr int kMaxBundles = 64;                    // bundles per tile (a whole net always fits)
-constexpr int kTargetBundles = 28;                 // planner target per tile
+#ifndef DGR_TARGET_BUNDLES
+#define DGR_TARGET_BUNDLES 32
+#endif
+constexpr int kTargetBundles = DGR_TARGET_BUNDLES;  // group bundles per pipelined tile
+constexpr int kTileBundles = kTargetBundles + 8;   // all bundles (group + singleton) per pipelined tile
 constexpr int kTreeMax = 512;                      // trees per tile
 constexpr int kPipeTrees = 224;                    // trees per pipelined tile
-constexpr int kPipeSubs = 448;                     // sub-nets per pipelined tile
+constexpr int kPipeSubs = 512;                     // sub-nets per pipelined tile
 constexpr int kEventMax = 127;                     // events per window cell-field (int32 safety)
 
 enum Shape : uint32_t {
   kStraightH = 0, kStraightV = 1, kHV = 2, kVH = 3, kZHVH = 4, kZVHV = 5, kPad = 7
 };
 constexpr uint32_t kSubHead = 8u;    // lane starts a sub-net group
-constexpr uint32_t kTreeHead = 16u;  // sub-net is the first of its tree (set on the group head)
+constexpr uint32_t kTreeHead = 16u;  // group head whose tree differs from the previous group's in the bundle
+constexpr int kTreeShift = 5;        // bits 5..13: tree of the lane relative to the bundle's tree base
+constexpr uint32_t kTreeMask = 511u;
 // bits 16..31: x_m (Z-HVH) or y_m (Z-VHV)
+constexpr int kSingleBundle = 0x100; // binfo.w flag: a singleton bundle (binfo.w & 0xff = #valid)
 
 struct TileDesc {
   int32_t b0, nb;          // bundles [b0, b0 + nb)
   int32_t net0, nnet;      // local nets
   int32_t tree0, ntree;    // local trees
   int32_t wx0, wy0, ww, wh;  // window (cells; even origin and extents), unused for global tiles
-  int32_t global, pad;
-  int32_t sub0, nsub;      // local sub-nets
+  int32_t global, nbg;     // nbg: group bundles (the first nbg of the tile; the rest are singleton bundles)
+  int32_t sub0, nsub;      // local sub-nets (kernel order within the tile)
   int32_t pad2, pad3;
 };
 
@@ -66,13 +79,15 @@ struct KParams {
   int32_t XP, YP;           // even pitches of S_H rows and S_V columns
   int32_t skip;             // DGR_DEBUG_SKIP: timing knock-outs (results invalid), 0 in production
   int64_t path_base, tree_base;   // global index of the first local path / tree
+  int64_t nid_base;         // global noise index of the rank's first noisy candidate
   uint64_t seed;
   // forest encoding
   const TileDesc* tiles;
   const TileDesc* tiles_slow;
   const int4* binfo;
   const uint32_t* pword;
-  const short4* sxy;
+  const short4* sxy;        // kernel order
+  const int32_t* slot_path; // local CSR path of each slot (-1 for padding); induction only
   float *wp, *mp, *vp;
   float* pp;                // p_i of the last forward (the reverse of that iteration reads it)
   const int32_t* net_tree_off;    // local, n_nets_l + 1
@@ -93,9 +108,9 @@ struct KParams {
   // induce scratch
   uint8_t* chosen;          // [n_trees_l]
   int32_t* tree_choice;     // [n_nets_l] (global tree index)
-  int32_t* route;           // [n_subs_l] (global path index or -1)
-  int32_t* nsize;           // [n_subs_l]
-  int32_t* nucleus_tmp;     // indexed by local path
+  int32_t* route;           // [n_subs_l] (global path index or -1), kernel sub-net order
+  int32_t* nsize;           // [n_subs_l], kernel sub-net order
+  int32_t* nucleus_tmp;     // indexed by slot: a sub-net's nucleus from its head slot on
   int32_t* DH;              // [Y][X]
   int32_t* DV;              // [Y][X]
   int32_t* VC;              // [Y][X]

@@ -61,7 +61,8 @@ struct Lane {
   uint32_t pw, shape, le, gmask, hm, tm;
   bool valid;
   int sub, tree;
-  int64_t gid, lpath;
+  bool single;     // lane of a singleton bundle (lone straight sub-nets: p = 1, no noise)
+  int64_t nid;     // global noise index (group bundles; reading Q7)
 };
 
 __device__ __forceinline__ void lane_setup(const KParams& P, int b, Lane& L) {
@@ -78,9 +79,9 @@ __device__ __forceinline__ void lane_setup(const KParams& P, int b, Lane& L) {
   L.end = rest ? (__ffs(rest) - 2) : 31;
   L.gmask = (kFull >> (31 - L.end)) & ~((1u << L.head) - 1u);
   L.sub = bi.y + __popc(L.hm & L.le) - 1;
-  L.tree = bi.z + __popc(L.tm & L.le & ~1u);
-  L.lpath = (int64_t)bi.x + L.lane;
-  L.gid = P.path_base + L.lpath;
+  L.tree = bi.z + (int)((L.pw >> kTreeShift) & kTreeMask);
+  L.single = (bi.w & kSingleBundle) != 0;
+  L.nid = P.nid_base + bi.x + L.lane;
 }
 
 // reduction over the lane's group [head, end]; the result is valid at the head lane
@@ -103,7 +104,7 @@ struct Max {
 
 // p_i = softmax over the sub-net group of (w_i + g_i) / t (reading Q1)
 __device__ __forceinline__ float group_softmax(const KParams& P, float inv_t, uint32_t k, const Lane& L, float w) {
-  const float z = L.valid ? (w + gumbel(P.seed, (uint64_t)L.gid, k, 0u)) * inv_t : -INFINITY;
+  const float z = L.valid ? (w + (L.single ? 0.f : gumbel(P.seed, (uint64_t)L.nid, k, 0u))) * inv_t : -INFINITY;
   float m = seg_reduce(z, L.lane, L.end, Max());
   m = __shfl_sync(kFull, m, L.head);
   const float e = L.valid ? __expf(z - m) : 0.f;
@@ -225,9 +226,9 @@ __device__ __forceinline__ void lane_from(int4 bi, uint32_t pw, const KParams& P
   L.end = rest ? (__ffs(rest) - 2) : 31;
   L.gmask = (kFull >> (31 - L.end)) & ~((1u << L.head) - 1u);
   L.sub = bi.y + __popc(L.hm & L.le) - 1;
-  L.tree = bi.z + __popc(L.tm & L.le & ~1u);
-  L.lpath = (int64_t)bi.x + L.lane;
-  L.gid = P.path_base + L.lpath;
+  L.tree = bi.z + (int)((pw >> kTreeShift) & kTreeMask);
+  L.single = (bi.w & kSingleBundle) != 0;
+  L.nid = P.nid_base + bi.x + L.lane;
 }
 
 __device__ __forceinline__ float softmax_from_noise(const Lane& L, float w, float g, float inv_t) {
@@ -334,8 +335,6 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
                                              const Win& W, int* ev_s, long long* red_s) {
   const int lane = threadIdx.x & 31;
   const int4 bfirst = __ldg(&P.binfo[bw0]);
-  const int4 blast = __ldg(&P.binfo[bw1 - 1]);
-  warp_noise(g_s, P.seed, P.path_base + bfirst.x, blast.x + blast.w - bfirst.x, (uint32_t)A.k_next, lane);
   const uint32_t ev_base = (uint32_t)__cvta_generic_to_shared(ev_s);
   long long wl = 0, tpc = 0;
   size_t slot = (size_t)bw0 * 32 + lane;
@@ -354,7 +353,7 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
       if (b + 2 < bw1) { bi1 = __ldg(&P.binfo[b + 2]); pw1 = __ldg(&P.pword[slot + 64]); }
     }
     const float w = have_w ? wst[(b - T.b0) * 32 + lane] : P.wp[slot];
-    const float g = L.valid ? g_s[L.lpath - bfirst.x] : 0.f;
+    const float g = (L.valid && !L.single) ? gumbel(P.seed, (uint64_t)L.nid, (uint32_t)A.k_next, 0u) : 0.f;
     const float p = softmax_from_noise(L, w, g, A.inv_t);
     P.pp[slot] = p;
     const float q = L.valid ? q_s[L.tree - T.tree0] : 0.f;
@@ -560,12 +559,12 @@ constexpr int kPNetMax = kPipeTrees + 8;
 
 struct StageLayout {
   static constexpr size_t pw = 0;
-  static constexpr size_t w = pw + 4 * kPSlots;
+  static constexpr size_t w = pw + 4 * 32 * kTileBundles;
   static constexpr size_t m = w + 4 * kPSlots;
   static constexpr size_t v = m + 4 * kPSlots;
   static constexpr size_t p = v + 4 * kPSlots;
   static constexpr size_t bi = p + 4 * kPSlots;
-  static constexpr size_t sxy = bi + 16 * kTargetBundles;
+  static constexpr size_t sxy = bi + 16 * kTileBundles;
   static constexpr size_t nto = sxy + 8 * kPSubMax;
   static constexpr size_t q = (nto + 4 * kPNetMax + 15) / 16 * 16;
   static constexpr size_t wt = q + 4 * kPTreeMax;
@@ -574,7 +573,6 @@ struct StageLayout {
   static constexpr size_t S = (vt + 4 * kPTreeMax + 127) / 128 * 128;
   static constexpr size_t bytes = S + 2 * 8 * kWinMax;
 };
-constexpr size_t kPEvBytes = 3 * 4 * kWinMax;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
@@ -637,10 +635,10 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
   Stage S(st);
   int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
-  const uint32_t slot_bytes = (uint32_t)T.nb * 128u;
+  const uint32_t slot_bytes = (uint32_t)T.nb * 128u, gslot_bytes = (uint32_t)T.nbg * 128u;
   const uint32_t nrow = REV ? (uint32_t)T.wh : 0u, ncol = REV ? (uint32_t)T.ww : 0u;
-  const uint32_t bytes = slot_bytes * (REV ? 5u : 2u) + 16u * T.nb + 8u * (s_hi - s_lo) + 4u * (n_hi - n_lo) +
-                         4u * (t_hi - t_lo) * (REV ? 4u : 3u) + 8u * (nrow * T.ww + ncol * T.wh);
+  const uint32_t bytes = slot_bytes + gslot_bytes * (REV ? 4u : 1u) + 16u * T.nb + 8u * (s_hi - s_lo) +
+                         4u * (n_hi - n_lo) + 4u * (t_hi - t_lo) * (REV ? 4u : 3u) + 8u * (nrow * T.ww + ncol * T.wh);
   if (lane == 0) mbar_expect_tx(bar, bytes);
   __syncwarp();
   const size_t s0 = (size_t)T.b0 * 32;
@@ -650,10 +648,10 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
     if (it < 10) {
       switch (it) {
         case 0: bulk_g2s(S.pw, P.pword + s0, slot_bytes, bar); break;
-        case 1: bulk_g2s(S.w, P.wp + s0, slot_bytes, bar); break;
-        case 2: if (REV) bulk_g2s(S.m, P.mp + s0, slot_bytes, bar); break;
-        case 3: if (REV) bulk_g2s(S.v, P.vp + s0, slot_bytes, bar); break;
-        case 4: if (REV) bulk_g2s(S.p, P.pp + s0, slot_bytes, bar); break;
+        case 1: if (gslot_bytes) bulk_g2s(S.w, P.wp + s0, gslot_bytes, bar); break;
+        case 2: if (REV && gslot_bytes) bulk_g2s(S.m, P.mp + s0, gslot_bytes, bar); break;
+        case 3: if (REV && gslot_bytes) bulk_g2s(S.v, P.vp + s0, gslot_bytes, bar); break;
+        case 4: if (REV && gslot_bytes) bulk_g2s(S.p, P.pp + s0, gslot_bytes, bar); break;
         case 5: bulk_g2s(S.bi, P.binfo + T.b0, 16u * T.nb, bar); break;
         case 6: bulk_g2s(S.sxy, P.sxy + s_lo, 8u * (s_hi - s_lo), bar); break;
         case 7: bulk_g2s(S.nto, P.net_tree_off + n_lo, 4u * (n_hi - n_lo), bar); break;
@@ -672,61 +670,85 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
   }
 }
 
-// One tile, all operands in shared memory (stage St).  ev_s / g_all may alias St.S (they are
-// only touched after the reverse half is done with it).  Ends with the slot state written back
-// by bulk stores (issued by thread 0, committed) and the demand window flushed.
+// One tile, all operands in shared memory (stage St).  ev_s / gp may alias St.S (they are only
+// touched after the reverse half is done with it).  Ends with the slot state written back by bulk
+// stores (issued by thread 0, committed) and the demand window flushed.
+// Bundles go to warps round-robin; lb < T.nbg are group bundles, the rest singleton bundles (lone
+// straight sub-nets: p = 1, no noise, no softmax, no Adam, no slot state).
+constexpr size_t kGpOffset = 3 * 4 * kWinMax;   // tile path noise, after the event window in St.S
 template <bool REV, bool FWD, int NT>
 __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A, const TileDesc& T, Stage St,
-                                             int* ev_s, float* g_all, long long* dq_s, long long& wl_acc,
+                                             int* ev_s, float* gp, long long* dq_s, long long& wl_acc,
                                              long long& tp_acc) {
   constexpr int NW = NT / 32;
-  constexpr int WCAND = (kTargetBundles + NW - 1) / NW * 32;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int X = P.X, Y = P.Y;
-  float* g_s = g_all + warp * WCAND;
   int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
   const int ncell = T.ww * T.wh;
   const Win W{T.wx0, T.wy0, T.ww, T.wh, ncell};
-  const int per = (T.nb + NW - 1) / NW;
-  const int lb0 = min(warp * per, T.nb), lb1 = min((warp + 1) * per, T.nb);   // tile-local bundles
+  const int nbg = T.nbg;
 
   // ---------------- reverse of iteration k ----------------
   if (REV) {
     for (int i = tid; i < T.ntree; i += NT) dq_s[i] = 0;
     __syncthreads();
-    for (int lb = lb0; lb < lb1; ++lb) {
-      Lane L;
-      lane_from(St.bi[lb], St.pw[lb * 32 + lane], P, L);
-      const int sl = lb * 32 + lane;
-      float w = St.w[sl], m = St.m[sl], v = St.v[sl];
-      const float p = St.p[sl];
-      const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
-      double c = 0.0;
-      if (L.valid && !(P.skip & 8)) {
-        const short4 e = St.sxy[L.sub - s_lo];
-        c = path_cost(St.S, W, X, Y, L.shape, e.x, e.y, e.z, e.w, (int)(L.pw >> 16), A);
-      }
-      // softmax backward: differences to the group head's dp in fp64, reduced in fp32
-      const double dp = (double)q * c;
-      const double dref = __shfl_sync(kFull, dp, L.head);
-      const float dd = (float)(dp - dref);
-      float sa = seg_reduce(p * dd, L.lane, L.end, Sum());
-      float sb = seg_reduce(p, L.lane, L.end, Sum());
-      sa = __shfl_sync(kFull, sa, L.head);
-      sb = __shfl_sync(kFull, sb, L.head);
-      const float dw = L.valid ? p * A.inv_t * (dd - __fdividef(sa, sb)) : 0.f;
-      // dq_j partial sums (fp64 -> 2^-32 fixed point)
-      const uint32_t th = L.tm | __ballot_sync(kFull, !L.valid) | 1u;
-      const uint32_t trest = th & ~L.le;
-      const int tend = trest ? (__ffs(trest) - 2) : 31;
-      const double pc = seg_reduce(L.valid ? (double)p * c : 0.0, L.lane, tend, Sum());
-      if (L.valid && ((th >> L.lane) & 1u))
-        atomicAdd(reinterpret_cast<unsigned long long*>(&dq_s[L.tree - T.tree0]),
-                  static_cast<unsigned long long>(__double2ll_rn(pc * kDqScale)));
-      if (L.valid) {
-        adam_update(w, m, v, dw, A);
-        St.w[sl] = w; St.m[sl] = m; St.v[sl] = v;
+    for (int lb = warp; lb < T.nb; lb += NW) {
+      const int4 bi = St.bi[lb];
+      const uint32_t pw = St.pw[lb * 32 + lane];
+      if (lb < nbg) {
+        Lane L;
+        lane_from(bi, pw, P, L);
+        const int sl = lb * 32 + lane;
+        float w = St.w[sl], m = St.m[sl], v = St.v[sl];
+        const float p = St.p[sl];
+        const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
+        double c = 0.0;
+        if (L.valid && !(P.skip & 8)) {
+          const short4 e = St.sxy[L.sub - s_lo];
+          c = path_cost(St.S, W, X, Y, L.shape, e.x, e.y, e.z, e.w, (int)(L.pw >> 16), A);
+        }
+        // softmax backward: differences to the group head's dp in fp64, reduced in fp32
+        const double dp = (double)q * c;
+        const double dref = __shfl_sync(kFull, dp, L.head);
+        const float dd = (float)(dp - dref);
+        float sa = seg_reduce(p * dd, L.lane, L.end, Sum());
+        float sb = seg_reduce(p, L.lane, L.end, Sum());
+        sa = __shfl_sync(kFull, sa, L.head);
+        sb = __shfl_sync(kFull, sb, L.head);
+        const float dw = L.valid ? p * A.inv_t * (dd - __fdividef(sa, sb)) : 0.f;
+        // dq_j partial sums over runs of lanes of one tree (fp64 -> 2^-32 fixed point)
+        const uint32_t th = L.tm | __ballot_sync(kFull, !L.valid) | 1u;
+        const uint32_t trest = th & ~L.le;
+        const int tend = trest ? (__ffs(trest) - 2) : 31;
+        const double pc = seg_reduce(L.valid ? (double)p * c : 0.0, L.lane, tend, Sum());
+        if (L.valid && ((th >> L.lane) & 1u))
+          atomicAdd(reinterpret_cast<unsigned long long*>(&dq_s[L.tree - T.tree0]),
+                    static_cast<unsigned long long>(__double2ll_rn(pc * kDqScale)));
+        if (L.valid) {
+          adam_update(w, m, v, dw, A);
+          St.w[sl] = w; St.m[sl] = m; St.v[sl] = v;
+        }
+      } else {
+        // singleton bundle: c of a straight path (one segment, no turning point); p = 1
+        const bool valid = (pw & 7u) != kPad;
+        const bool isv = (pw & 7u) == kStraightV;
+        const int tree = bi.z + (int)((pw >> kTreeShift) & kTreeMask);
+        double c = 0.0;
+        if (valid && !(P.skip & 8)) {
+          const short4 e = St.sxy[bi.y + lane - s_lo];
+          const int ia = isv ? W.v(e.x, e.y) : W.h(e.x, e.y);
+          const int ib = isv ? W.v(e.x, e.w) : W.h(e.z, e.y);
+          c = (St.S[ib] - St.S[ia]) + (double)A.a_wl * (double)((e.z - e.x) + (e.w - e.y));
+        }
+        const uint32_t th = __ballot_sync(kFull, (pw & kTreeHead) || !valid) | 1u;
+        const uint32_t le = kFull >> (31 - lane);
+        const uint32_t trest = th & ~le;
+        const int tend = trest ? (__ffs(trest) - 2) : 31;
+        const double pc = seg_reduce(c, lane, tend, Sum());
+        if (valid && ((th >> lane) & 1u))
+          atomicAdd(reinterpret_cast<unsigned long long*>(&dq_s[tree - T.tree0]),
+                    static_cast<unsigned long long>(__double2ll_rn(pc * kDqScale)));
       }
     }
     __syncthreads();
@@ -793,8 +815,26 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         P.q[jg] = q;
       }
     }
-    __syncthreads();
   }
+  if (FWD && nbg > 0 && !(P.skip & 2)) {
+    // Gumbel noise of the tile's noisy candidates (stream 0): contiguous noise indices
+    // [bi[0].x, bi[nbg-1].x + #valid), one Philox call per 4 consecutive indices
+    const int64_t n0 = P.nid_base + St.bi[0].x;
+    const int4 bl = St.bi[nbg - 1];
+    const int nn = bl.x + (bl.w & 0xff) - St.bi[0].x;
+    const int64_t c0 = n0 >> 2, c1 = (n0 + nn - 1) >> 2;
+    const uint2 key = make_uint2((uint32_t)P.seed, (uint32_t)(P.seed >> 32));
+    for (int64_t c = c0 + tid; c <= c1; c += NT) {
+      const uint4 r = philox4x32_10(make_uint4((uint32_t)c, (uint32_t)(c >> 32), (uint32_t)A.k_next, 0u), key);
+      const uint32_t wd[4] = {r.x, r.y, r.z, r.w};
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int64_t i = c * 4 + q - n0;
+        if (i >= 0 && i < nn) gp[i] = gumbel_word(wd[q]);
+      }
+    }
+  }
+  __syncthreads();
 
   // ---------------- forward of iteration k_next ----------------
   if (FWD) {
@@ -803,102 +843,119 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
       for (int i = tid; i < (3 * ncell + 3) / 4; i += NT) z[i] = make_int4(0, 0, 0, 0);
     }
     __syncthreads();
-    if (lb0 < lb1 && !(P.skip & 2)) {
-      const int4 bfirst = St.bi[lb0];
-      const int4 blast = St.bi[lb1 - 1];
-      warp_noise(g_s, P.seed, P.path_base + bfirst.x, blast.x + blast.w - bfirst.x, (uint32_t)A.k_next, lane);
-    }
     const uint32_t ev_base = smem_u32(ev_s);
-    for (int lb = lb0; lb < lb1; ++lb) {
-      Lane L;
-      lane_from(St.bi[lb], St.pw[lb * 32 + lane], P, L);
-      const int sl = lb * 32 + lane;
-      const float w = St.w[sl];
-      const float g = L.valid ? g_s[L.lpath - St.bi[lb0].x] : 0.f;
-      const float p = softmax_from_noise(L, w, g, A.inv_t);
-      St.p[sl] = p;
-      const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
-      const int vq = L.valid ? __float2int_rn(q * p * kFixScale) : 0;
-      int sc = vq;
+    const int nid0 = nbg > 0 ? St.bi[0].x : 0;
+    for (int lb = warp; lb < T.nb; lb += NW) {
+      const int4 bi = St.bi[lb];
+      const uint32_t pw = St.pw[lb * 32 + lane];
+      if (lb < nbg) {
+        Lane L;
+        lane_from(bi, pw, P, L);
+        const int sl = lb * 32 + lane;
+        const float w = St.w[sl];
+        const float g = L.valid ? gp[bi.x + lane - nid0] : 0.f;
+        const float p = softmax_from_noise(L, w, g, A.inv_t);
+        St.p[sl] = p;
+        const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
+        const int vq = L.valid ? __float2int_rn(q * p * kFixScale) : 0;
+        int sc = vq;
 #pragma unroll
-      for (int off = 1; off < 32; off <<= 1) {
-        const int o = __shfl_up_sync(kFull, sc, off);
-        if (L.lane - off >= L.head) sc += o;
-      }
-      const int nh = __popc(__ballot_sync(kFull, L.shape == kZHVH) & L.gmask);
-      const int h1 = min(L.head + 1, 31), h2 = min(L.head + 1 + nh, 31);
-      const int a = __shfl_sync(kFull, vq, L.head);
-      const int bb = __shfl_sync(kFull, vq, h1);
-      const int S1 = __shfl_sync(kFull, sc, h1);
-      const int S2 = __shfl_sync(kFull, sc, h2);
-      const int Se = __shfl_sync(kFull, sc, L.end);
-      const short4 e = L.valid ? St.sxy[L.sub - s_lo] : make_short4(0, 0, 0, 0);
-      const int x0 = e.x, y0 = e.y, x1 = e.z, y1 = e.w;
-      const int sgn = (y1 > y0) ? 1 : -1;
-      const int hs = S2 - S1, vs = Se - S2, vv = vq;
-      const int mm = (int)(L.pw >> 16);
-      const int fSH = L.shape == kStraightH, fSV = L.shape == kStraightV, fHV = L.shape == kHV;
-      const int fVH = L.shape == kVH, fZH = L.shape == kZHVH, fZV = L.shape == kZVHV;
-      const int fZ = fZH + fZV;
-      const int xa = x0 + fZH * (mm - x0);
-      const int ya = y0 + fVH * (y1 - y0) + fZV * (mm - y0);
-      const int xb = x1 + fSV * (x0 - x1) + fZH * (mm - x1);
-      const int yb = y1 + (fSH + fHV) * (y0 - y1) + fZV * (mm - y1);
-      const int ah = fSH * vv + fHV * (a + hs) + fVH * bb + (fZV - fZH) * vv;
-      const int av = fSV * vv + sgn * (fHV * (bb + vs) - fVH * bb + (fZH - fZV) * vv);
-      const int ad = fVH * bb + fZ * vv;
-      const int bh = -fSH * vv - fHV * a - fVH * (bb + hs) + (fZH - fZV) * vv;
-      const int bv = -fSV * vv + sgn * (fHV * a - fVH * (a + vs) + (fZV - fZH) * vv);
-      const int bd = fHV * a + fZ * vv;
-      if (L.valid && !(P.skip & 4)) {
-        const int hv2 = 2 * ncell;
-        const int ia_h = W.h(xa, ya), ib_h = W.h(xb, yb);
-        red_shared_add(ev_base + 4u * ia_h, ah);
-        red_shared_add(ev_base + 4u * W.v(xa, ya), av);
-        red_shared_add(ev_base + 4u * (hv2 + ia_h), ad);
-        red_shared_add(ev_base + 4u * ib_h, bh);
-        red_shared_add(ev_base + 4u * W.v(xb, yb), bv);
-        red_shared_add(ev_base + 4u * (hv2 + ib_h), bd);
-        wl_acc += (long long)vq * ((x1 - x0) + abs(y1 - y0));
-        tp_acc += (long long)vq * (fHV + fVH + 2 * fZ);
+        for (int off = 1; off < 32; off <<= 1) {
+          const int o = __shfl_up_sync(kFull, sc, off);
+          if (L.lane - off >= L.head) sc += o;
+        }
+        const int nh = __popc(__ballot_sync(kFull, L.shape == kZHVH) & L.gmask);
+        const int h1 = min(L.head + 1, 31), h2 = min(L.head + 1 + nh, 31);
+        const int a = __shfl_sync(kFull, vq, L.head);
+        const int bb = __shfl_sync(kFull, vq, h1);
+        const int S1 = __shfl_sync(kFull, sc, h1);
+        const int S2 = __shfl_sync(kFull, sc, h2);
+        const int Se = __shfl_sync(kFull, sc, L.end);
+        const short4 e = L.valid ? St.sxy[L.sub - s_lo] : make_short4(0, 0, 0, 0);
+        const int x0 = e.x, y0 = e.y, x1 = e.z, y1 = e.w;
+        const int sgn = (y1 > y0) ? 1 : -1;
+        const int hs = S2 - S1, vs = Se - S2, vv = vq;
+        const int mm = (int)(L.pw >> 16);
+        const int fSH = L.shape == kStraightH, fSV = L.shape == kStraightV, fHV = L.shape == kHV;
+        const int fVH = L.shape == kVH, fZH = L.shape == kZHVH, fZV = L.shape == kZVHV;
+        const int fZ = fZH + fZV;
+        const int xa = x0 + fZH * (mm - x0);
+        const int ya = y0 + fVH * (y1 - y0) + fZV * (mm - y0);
+        const int xb = x1 + fSV * (x0 - x1) + fZH * (mm - x1);
+        const int yb = y1 + (fSH + fHV) * (y0 - y1) + fZV * (mm - y1);
+        const int ah = fSH * vv + fHV * (a + hs) + fVH * bb + (fZV - fZH) * vv;
+        const int av = fSV * vv + sgn * (fHV * (bb + vs) - fVH * bb + (fZH - fZV) * vv);
+        const int ad = fVH * bb + fZ * vv;
+        const int bh = -fSH * vv - fHV * a - fVH * (bb + hs) + (fZH - fZV) * vv;
+        const int bv = -fSV * vv + sgn * (fHV * a - fVH * (a + vs) + (fZV - fZH) * vv);
+        const int bd = fHV * a + fZ * vv;
+        if (L.valid && !(P.skip & 4)) {
+          const int hv2 = 2 * ncell;
+          const int ia_h = W.h(xa, ya), ib_h = W.h(xb, yb);
+          red_shared_add(ev_base + 4u * ia_h, ah);
+          red_shared_add(ev_base + 4u * W.v(xa, ya), av);
+          red_shared_add(ev_base + 4u * (hv2 + ia_h), ad);
+          red_shared_add(ev_base + 4u * ib_h, bh);
+          red_shared_add(ev_base + 4u * W.v(xb, yb), bv);
+          red_shared_add(ev_base + 4u * (hv2 + ib_h), bd);
+          wl_acc += (long long)vq * ((x1 - x0) + abs(y1 - y0));
+          tp_acc += (long long)vq * (fHV + fVH + 2 * fZ);
+        }
+      } else {
+        // singleton bundle: pi = q; +pi where the segment starts, -pi where it ends
+        const bool valid = (pw & 7u) != kPad;
+        if (valid && !(P.skip & 4)) {
+          const bool isv = (pw & 7u) == kStraightV;
+          const int tree = bi.z + (int)((pw >> kTreeShift) & kTreeMask);
+          const float q = St.q[tree - t_lo];
+          const int vq = __float2int_rn(q * kFixScale);
+          const short4 e = St.sxy[bi.y + lane - s_lo];
+          const int ia = isv ? W.v(e.x, e.y) : W.h(e.x, e.y);
+          const int ib = isv ? W.v(e.x, e.w) : W.h(e.z, e.y);
+          red_shared_add(ev_base + 4u * ia, vq);
+          red_shared_add(ev_base + 4u * ib, -vq);
+          wl_acc += (long long)vq * ((e.z - e.x) + (e.w - e.y));
+        }
       }
     }
   }
   __syncthreads();
-  // write back the tile's slot state with bulk stores (asynchronous; readers wait on the group)
-  if (tid == 0) {
+  // write back the tile's group slot state with bulk stores (asynchronous; readers wait on the group)
+  if (tid == 0 && nbg > 0) {
     fence_proxy_async();
     const size_t s0 = (size_t)T.b0 * 32;
-    const uint32_t slot_bytes = (uint32_t)T.nb * 128u;
+    const uint32_t gslot_bytes = (uint32_t)nbg * 128u;
     if (REV) {
-      bulk_s2g(P.wp + s0, St.w, slot_bytes);
-      bulk_s2g(P.mp + s0, St.m, slot_bytes);
-      bulk_s2g(P.vp + s0, St.v, slot_bytes);
+      bulk_s2g(P.wp + s0, St.w, gslot_bytes);
+      bulk_s2g(P.mp + s0, St.m, gslot_bytes);
+      bulk_s2g(P.vp + s0, St.v, gslot_bytes);
     }
-    if (FWD) bulk_s2g(P.pp + s0, St.p, slot_bytes);
+    if (FWD) bulk_s2g(P.pp + s0, St.p, gslot_bytes);
     bulk_commit();
   }
   if (FWD && !(P.skip & 1)) {
-    // flush: a warp per window row (dH, VD) / column (dV); cells in pairs, zero pairs skipped
+    // flush: the window's cell pairs as one flat range per field (rows of dH / VD, columns of dV;
+    // widths are even, so pair i is cells 2i, 2i+1 of the field); zero cells are skipped, and every
+    // cell outside the grid is zero (events only land on grid cells).  row = floor((i + 1/2) / half
+    // width) in fp32 is exact here: the fraction stays >= 1/(2 half) >> the rounding of i < 2^12.
     const int hw = T.ww >> 1, hh = T.wh >> 1;
-    for (int yi = warp; yi < T.wh; yi += NW) {
-      if (T.wy0 + yi >= Y) break;
-      const size_t g0 = (size_t)(T.wy0 + yi) * X + T.wx0;
-      const int2* rowH = reinterpret_cast<const int2*>(ev_s + yi * T.ww);
-      const int2* rowD = reinterpret_cast<const int2*>(ev_s + 2 * ncell + yi * T.ww);
-      for (int xp = lane; xp < hw; xp += 32) {
-        const int2 h = rowH[xp], d = rowD[xp];
-        if (h.x | h.y) { red64(P.dH + g0 + 2 * xp, h.x); red64(P.dH + g0 + 2 * xp + 1, h.y); }
-        if (d.x | d.y) { red64(P.VD + g0 + 2 * xp, d.x); red64(P.VD + g0 + 2 * xp + 1, d.y); }
+    const float inv_hw = 1.f / (float)hw, inv_hh = 1.f / (float)hh;
+    const int2* evH = reinterpret_cast<const int2*>(ev_s);
+    const int2* evV = reinterpret_cast<const int2*>(ev_s + ncell);
+    const int2* evD = reinterpret_cast<const int2*>(ev_s + 2 * ncell);
+    const int npair = ncell >> 1;
+    for (int i = tid; i < npair; i += NT) {
+      const int2 h = evH[i], d = evD[i], v = evV[i];
+      if (h.x | h.y | d.x | d.y) {
+        const int r = (int)(((float)i + 0.5f) * inv_hw);
+        const size_t g = (size_t)(T.wy0 + r) * X + T.wx0 + 2 * (i - r * hw);
+        red64(P.dH + g, h.x); red64(P.dH + g + 1, h.y);
+        red64(P.VD + g, d.x); red64(P.VD + g + 1, d.y);
       }
-    }
-    for (int xi = warp; xi < T.ww; xi += NW) {
-      if (T.wx0 + xi >= X) break;
-      const size_t g0 = (size_t)(T.wx0 + xi) * Y + T.wy0;
-      const int2* colV = reinterpret_cast<const int2*>(ev_s + ncell + xi * T.wh);
-      for (int yp = lane; yp < hh; yp += 32) {
-        const int2 v = colV[yp];
-        if (v.x | v.y) { red64(P.dVT + g0 + 2 * yp, v.x); red64(P.dVT + g0 + 2 * yp + 1, v.y); }
+      if (v.x | v.y) {
+        const int c = (int)(((float)i + 0.5f) * inv_hh);
+        const size_t g = (size_t)(T.wx0 + c) * Y + T.wy0 + 2 * (i - c * hh);
+        red64(P.dVT + g, v.x); red64(P.dVT + g + 1, v.y);
       }
     }
   }
@@ -928,7 +985,8 @@ __device__ __forceinline__ void flush_scalars(const KParams& P, long long wl, lo
 constexpr int kBThreads = DGR_BTHREADS;
 constexpr int kBPerSM = 1024 / kBThreads;
 constexpr size_t kBSmemBytes = StageLayout::bytes + 8 * kPipeTrees + 64;
-static_assert(kPEvBytes + 4 * kWinMax <= 2 * 8 * kWinMax, "event window + noise must fit the S window");
+static_assert(kGpOffset + 4 * 32 * kTargetBundles <= 2 * 8 * kWinMax, "event window + path noise must fit the S window");
+static_assert(8 * kPipeTrees + 12 * kPipeTrees + 32 + 4 * kPipeTrees <= kGpOffset, "tree scratch must not overlap the path noise");
 
 template <bool REV, bool FWD>
 __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepArgs A) {
@@ -938,7 +996,7 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
   long long* red_s = dq_s + kPipeTrees;
   uint64_t* bar = reinterpret_cast<uint64_t*>(red_s + 2);
   int* ev_s = reinterpret_cast<int*>(St.S);
-  float* g_all = reinterpret_cast<float*>(ev_s + 3 * kWinMax);
+  float* gp = reinterpret_cast<float*>(reinterpret_cast<unsigned char*>(St.S) + kGpOffset);
   const TileDesc T = P.tiles[blockIdx.x];
   if (threadIdx.x == 0) {
     mbar_init(bar, 1);
@@ -948,7 +1006,7 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
   if (threadIdx.x < 32) issue_tile_loads<REV>(P, T, smem, bar);
   mbar_wait(bar, 0u);
   long long wl = 0, tp = 0;
-  process_tile<REV, FWD, kBThreads>(P, A, T, St, ev_s, g_all, dq_s, wl, tp);
+  process_tile<REV, FWD, kBThreads>(P, A, T, St, ev_s, gp, dq_s, wl, tp);
   if (FWD) flush_scalars<kBThreads>(P, wl, tp, red_s);
   if (threadIdx.x == 0) bulk_wait_read();   // the stage must outlive the bulk stores' reads
 }
@@ -988,8 +1046,8 @@ __global__ void __launch_bounds__(kPThreads, kPPerSM) tile_persistent(KParams P,
     mbar_wait(&bars[sidx], (uint32_t)(it >> 1) & 1u);
     Stage St(stage_base[sidx]);
     int* ev_s = reinterpret_cast<int*>(St.S);
-    float* g_all = reinterpret_cast<float*>(ev_s + 3 * kWinMax);
-    process_tile<REV, FWD, kPThreads>(P, A, P.tiles[tile], St, ev_s, g_all, dq_s, wl, tp);
+    float* gp = reinterpret_cast<float*>(reinterpret_cast<unsigned char*>(St.S) + kGpOffset);
+    process_tile<REV, FWD, kPThreads>(P, A, P.tiles[tile], St, ev_s, gp, dq_s, wl, tp);
     __syncthreads();
   }
   if (FWD) flush_scalars<kPThreads>(P, wl, tp, red_s);
@@ -1233,9 +1291,10 @@ __global__ void __launch_bounds__(256) ki_path_kernel(KParams P, float inv_t, fl
     P.nsize[L.sub] = on ? __popc(inm & L.gmask) : 0;
     if (!on) P.route[L.sub] = -1;
   }
-  if (in) P.nucleus_tmp[(size_t)(L.lpath - (L.lane - L.head)) + rank] = (int32_t)L.gid;
+  const int32_t gid = L.valid ? (int32_t)(P.path_base + P.slot_path[slot]) : -1;
+  if (in) P.nucleus_tmp[(size_t)b * 32 + L.head + rank] = gid;
   if (on && rank == 0) {
-    P.route[L.sub] = (int32_t)L.gid;
+    P.route[L.sub] = gid;
     const short4 c4 = __ldg(&P.sxy[L.sub]);
     const int x0 = c4.x, y0 = c4.y, x1 = c4.z, y1 = c4.w;
     const int ylo = min(y0, y1), yhi = max(y0, y1);

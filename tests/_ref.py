@@ -10,6 +10,24 @@ import itertools
 import numpy as np
 import torch
 
+import oracle
+
+
+def path_noise(f, k):
+    """Gumbel noise g_i of every path candidate at iteration k (stream 0), reading Q7:
+    a sub-net whose only candidate is a straight path (one segment) draws none (g = 0; its softmax
+    is 1 whatever g is); every other candidate takes the next noise index in forest order."""
+    g = np.zeros(f.n_paths)
+    n = 0
+    for s in range(f.n_subnets):
+        a, b = int(f.sub_path_off[s]), int(f.sub_path_off[s + 1])
+        if b - a == 1 and f.path_seg_off[a + 1] - f.path_seg_off[a] == 1:
+            continue
+        for i in range(a, b):
+            g[i] = oracle.gumbel(f.seed, n, k, 0)
+            n += 1
+    return g
+
 
 def path_edges(f, i):
     """Edges of path i as (dir, y, x) triples; dir 0 = H edge (x,y)-(x+1,y), 1 = V edge (x,y)-(x,y+1)."""

@@ -110,3 +110,40 @@ def test_plan_tiles_cover_the_forest(name):
     for world in (2, 3):
         tot = sum(dgr.plan_info(f, rank=r, world=world)["n_paths"] for r in range(world))
         assert tot == f.n_paths
+
+
+def _permute_candidates(f, s, order):
+    """Copy of forest f with sub-net s's candidates listed in `order` (CSR arrays rebuilt)."""
+    import copy
+    g = copy.deepcopy(f)
+    p0 = int(f.sub_path_off[s])
+    perm = np.arange(f.n_paths)
+    perm[p0:p0 + len(order)] = p0 + np.asarray(order)
+    segs, tps, so, to = [], [], [0], [0]
+    for i in perm:
+        a, b = f.path_seg_off[i], f.path_seg_off[i + 1]
+        segs.append(f.seg[a:b]); so.append(so[-1] + b - a)
+        a, b = f.path_tp_off[i], f.path_tp_off[i + 1]
+        tps.append(f.tp_xy[a:b]); to.append(to[-1] + b - a)
+    g.seg = np.ascontiguousarray(np.concatenate(segs)).astype(f.seg.dtype)
+    g.tp_xy = np.ascontiguousarray(np.concatenate(tps)).astype(f.tp_xy.dtype)
+    g.path_seg_off = np.asarray(so, dtype=f.path_seg_off.dtype)
+    g.path_tp_off = np.asarray(to, dtype=f.path_tp_off.dtype)
+    g.w_path0 = np.ascontiguousarray(f.w_path0[perm])
+    return g
+
+
+def test_candidate_order_contract(tiny):
+    """dgr.h: a non-aligned sub-net lists HV, VH, then Z-HVH, then Z-VHV candidates (the forward's
+    event collapse relies on it); any other order is rejected, never silently mis-summed."""
+    n = np.diff(tiny.sub_path_off)
+    s = int(np.nonzero(n >= 4)[0][0])
+    ok, err = _ws(_permute_candidates(tiny, s, list(range(n[s]))))
+    assert ok > 0 and err == ""
+    for order in ([1, 0] + list(range(2, n[s])), [2, 0, 1] + list(range(3, n[s]))):
+        ws, err = _ws(_permute_candidates(tiny, s, order))
+        assert ws == 0 and "in this order" in err, err
+    # an L pair alone is fine; a lone L candidate is not
+    s2 = int(np.nonzero(n == 2)[0][0]) if (n == 2).any() else None
+    if s2 is not None:
+        assert _ws(_permute_candidates(tiny, s2, [0, 1]))[0] > 0

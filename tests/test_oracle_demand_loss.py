@@ -123,7 +123,7 @@ def test_cost_matches_torch_restatement(tiny, f_kind, slope):
     o.iteration = 2
     t = 0.9
     out = o.forward(t, W)
-    g = torch.tensor([oracle.gumbel(tiny.seed, i, 2, 0) for i in range(tiny.n_paths)], dtype=torch.float64)
+    g = torch.tensor(_ref.path_noise(tiny, 2), dtype=torch.float64)
     gt = torch.tensor([oracle.gumbel(tiny.seed, j, 2, 1) for j in range(tiny.n_trees)], dtype=torch.float64)
     cost, d, ewl, etp, of, _, _ = _ref.torch_cost(tiny, torch.tensor(tiny.w_tree0, dtype=torch.float64),
                                                   torch.tensor(tiny.w_path0, dtype=torch.float64), gt, g, t, W)

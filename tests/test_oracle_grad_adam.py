@@ -78,7 +78,7 @@ def test_gradient_matches_torch_autograd(tiny, f_kind, slope):
     W = oracle.weights(f_kind=f_kind, f_slope=slope)
     t, k = 0.7, 5
     o, (dw, du) = _grad(tiny, k, t, W)
-    g = torch.tensor([oracle.gumbel(tiny.seed, i, k, 0) for i in range(tiny.n_paths)], dtype=torch.float64)
+    g = torch.tensor(_ref.path_noise(tiny, k), dtype=torch.float64)
     gt = torch.tensor([oracle.gumbel(tiny.seed, j, k, 1) for j in range(tiny.n_trees)], dtype=torch.float64)
     wp = torch.tensor(tiny.w_path0, dtype=torch.float64, requires_grad=True)
     wt = torch.tensor(tiny.w_tree0, dtype=torch.float64, requires_grad=True)

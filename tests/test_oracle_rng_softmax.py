@@ -13,6 +13,7 @@ import pytest
 import torch
 
 import oracle
+from tests import _ref
 
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
 
@@ -117,7 +118,7 @@ def test_noisy_softmax_uses_the_candidate_noise(tiny):
     t = 0.37
     o.forward(t, oracle.weights())
     q, p = o.probs()
-    g = np.array([oracle.gumbel(tiny.seed, i, 11, 0) for i in range(tiny.n_paths)])
+    g = _ref.path_noise(tiny, 11)
     gt = np.array([oracle.gumbel(tiny.seed, j, 11, 1) for j in range(tiny.n_trees)])
     z = torch.tensor((tiny.w_path0.astype(np.float64) + g) / t)
     zt = torch.tensor((tiny.w_tree0.astype(np.float64) + gt) / t)
@@ -146,7 +147,7 @@ def test_low_temperature_is_argmax(tiny):
     o = oracle.Oracle(tiny)
     o.forward(1e-4, oracle.weights())
     q, p = o.probs()
-    g = np.array([oracle.gumbel(tiny.seed, i, 0, 0) for i in range(tiny.n_paths)])
+    g = _ref.path_noise(tiny, 0)
     z = tiny.w_path0.astype(np.float64) + g
     for s in range(tiny.n_subnets):
         a, b = tiny.sub_path_off[s], tiny.sub_path_off[s + 1]
