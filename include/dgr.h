@@ -113,7 +113,26 @@ int dgr_partition(const dgr_forest_desc* desc, int32_t world, int64_t* out);
 /* Bytes of device workspace this rank needs for desc (0 on error; see dgr_last_error). */
 int64_t dgr_workspace_size(const dgr_forest_desc* desc, const dgr_dist* dist);
 
-/* Validates desc, keeps this rank's nets (dgr_partition), encodes them for the device, copies
+/* Host-only first half of dgr_forest_load: validates desc, keeps this rank's nets (dgr_partition)
+ * and encodes them (tiles, bundles; SURVEY §8(b) "forest encoding").  The handle owns the plan but
+ * no device memory yet: only dgr_handle_workspace_size, dgr_bind_workspace, dgr_get_info and
+ * dgr_free are valid on it (others return DGR_ESTATE).  cuda_stream as in dgr_forest_load. */
+int dgr_forest_plan(const dgr_forest_desc* desc, const dgr_dist* dist, void* cuda_stream, struct dgr_handle** out);
+
+/* Bytes of device workspace a planned handle needs (0 on error). */
+int64_t dgr_handle_workspace_size(struct dgr_handle* h);
+
+/* Second half of dgr_forest_load: copies the planned shard into dev_workspace (>= the planned
+ * size, 256-byte aligned; caller-owned, must outlive the handle), zeroes Adam state and k and, with
+ * world > 1, creates the NCCL communicator (collective).  desc and dist must describe the same
+ * forest and ranks as at dgr_forest_plan (w_path0, w_tree0, cap_h, cap_v and seed are read here).
+ * On error the handle stays planned (the caller may retry or free it).  Synchronises. */
+int dgr_bind_workspace(struct dgr_handle* h, const dgr_forest_desc* desc, const dgr_dist* dist,
+                       void* dev_workspace, int64_t workspace_bytes);
+
+/* dgr_forest_plan + dgr_bind_workspace in one call (plans the forest once; dgr_workspace_size
+ * above plans it separately).
+ * Validates desc, keeps this rank's nets (dgr_partition), encodes them for the device, copies
  * them into dev_workspace (>= dgr_workspace_size bytes, 256-byte aligned) on cuda_stream
  * (a cudaStream_t; NULL = legacy default stream), zeroes Adam state and the iteration counter k.
  * With world > 1 this also creates the NCCL communicator (collective).  Synchronises. */
@@ -124,6 +143,8 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
  * forward (steps 1-3), reverse (step 4) and Adam (step 5), with k incremented after each.
  * iters == 0 runs one forward only (no update, k unchanged).  The Gumbel noise of iteration k
  * is keyed on the global k, so 10 calls of 100 iterations equal 1 call of 1000 at equal t.
+ * The last iteration also runs the forward of iteration k+1 (device-side state only), so a
+ * following call at the same temperature starts from it instead of recomputing it. 
  * If `last` is non-NULL it receives the loss of the last forward (synchronises). */
 int dgr_step(struct dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w,
              dgr_loss* last);
@@ -164,7 +185,7 @@ int dgr_plan_info(const dgr_forest_desc* desc, const dgr_dist* dist, int64_t out
  * dgr_profile_read synchronises and returns, per stage, the summed milliseconds and the number of
  * launches: 0 KF (forward-only tile kernel, once per dgr_step call), 1 demand allreduce (NCCL;
  * world > 1), 2 KG (scan / loss / gradient map; 2 kernels), 3 KBF (reverse of k fused with the
- * forward of k+1), 4 KB (reverse only: the last iteration of a call), 5..7 unused. */
+ * forward of k+1), 4 KB (reverse only; not launched since every call ends with KBF), 5..7 unused. */
 int dgr_profile(struct dgr_handle* h, int32_t enable);
 int dgr_profile_read(struct dgr_handle* h, double ms[8], int64_t launches[8]);
 

@@ -10,11 +10,13 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <memory>
 #include <string>
 #include <vector>
 
@@ -54,9 +56,13 @@ int fail(int code, const char* fmt, ...) {
 int check_offsets(const int64_t* off, int64_t n, int64_t total, const char* name, bool nonempty) {
   if (!off) return fail(DGR_EINVAL, "%s is NULL", name);
   if (off[0] != 0) return fail(DGR_EINVAL, "%s[0] != 0", name);
-  for (int64_t i = 0; i < n; ++i) {
-    if (off[i + 1] < off[i]) return fail(DGR_EINVAL, "%s not monotone at %lld", name, (long long)i);
-    if (nonempty && off[i + 1] == off[i]) return fail(DGR_EINVAL, "%s: empty group %lld", name, (long long)i);
+  int64_t bad = n;   // first offending group (parallel scan, reported in index order)
+#pragma omp parallel for schedule(static) reduction(min : bad)
+  for (int64_t i = 0; i < n; ++i)
+    if (off[i + 1] < off[i] || (nonempty && off[i + 1] == off[i])) bad = std::min(bad, i);
+  if (bad < n) {
+    if (off[bad + 1] < off[bad]) return fail(DGR_EINVAL, "%s not monotone at %lld", name, (long long)bad);
+    return fail(DGR_EINVAL, "%s: empty group %lld", name, (long long)bad);
   }
   if (off[n] != total) return fail(DGR_EINVAL, "%s[n] = %lld != %lld", name, (long long)off[n], (long long)total);
   return DGR_OK;
@@ -75,10 +81,13 @@ int validate_structure(const dgr_forest_desc* d) {
   if ((rc = check_offsets(d->sub_path_off, d->n_subnets, d->n_paths, "sub_path_off", true))) return rc;
   if ((rc = check_offsets(d->path_seg_off, d->n_paths, d->n_segs, "path_seg_off", true))) return rc;
   if ((rc = check_offsets(d->path_tp_off, d->n_paths, d->n_tps, "path_tp_off", false))) return rc;
+  int64_t big = d->n_subnets;
+#pragma omp parallel for schedule(static) reduction(min : big)
   for (int64_t s = 0; s < d->n_subnets; ++s)
-    if (d->sub_path_off[s + 1] - d->sub_path_off[s] > 32)
-      return fail(DGR_EINVAL, "sub-net %lld has %lld > 32 candidates", (long long)s,
-                  (long long)(d->sub_path_off[s + 1] - d->sub_path_off[s]));
+    if (d->sub_path_off[s + 1] - d->sub_path_off[s] > 32) big = std::min(big, s);
+  if (big < d->n_subnets)
+    return fail(DGR_EINVAL, "sub-net %lld has %lld > 32 candidates", (long long)big,
+                (long long)(d->sub_path_off[big + 1] - d->sub_path_off[big]));
   if ((d->n_segs && !d->seg) || (d->n_tps && !d->tp_xy) || (d->n_subnets && !d->sub_xy) || !d->cap_h ||
       !d->cap_v || (d->n_trees && !d->w_tree0) || (d->n_paths && !d->w_path0))
     return fail(DGR_EINVAL, "NULL array");
@@ -88,19 +97,22 @@ int validate_structure(const dgr_forest_desc* d) {
 int partition(const dgr_forest_desc* d, int world, std::vector<int64_t>& out) {
   if (world < 1) return fail(DGR_EINVAL, "world < 1");
   out.assign(world + 1, 0);
-  // work of a net = its paths + its segments (the per-candidate streams of KF / KB)
-  std::vector<int64_t> pref(d->n_nets + 1, 0);
-  for (int64_t n = 0; n < d->n_nets; ++n) {
-    const int64_t s0 = d->tree_sub_off[d->net_tree_off[n]], s1 = d->tree_sub_off[d->net_tree_off[n + 1]];
-    const int64_t p0 = d->sub_path_off[s0], p1 = d->sub_path_off[s1];
-    pref[n + 1] = pref[n] + (p1 - p0) + (d->path_seg_off[p1] - d->path_seg_off[p0]);
-  }
-  const int64_t total = pref[d->n_nets];
+  // work of a net = its paths + its segments (the per-candidate streams of KF / KB); the work of
+  // nets [0, n) telescopes to first_path(n) + first_seg(first_path(n)), so cut points are binary
+  // searches on that monotone function
+  auto pref = [&](int64_t n) {
+    const int64_t p = d->sub_path_off[d->tree_sub_off[d->net_tree_off[n]]];
+    return p + d->path_seg_off[p];
+  };
+  const int64_t total = pref(d->n_nets);
   for (int r = 1; r < world; ++r) {
-    const double target = (double)total * r / world;
-    const int64_t lo = out[r - 1];
-    int64_t n = std::lower_bound(pref.begin() + lo, pref.end(), (int64_t)std::ceil(target)) - pref.begin();
-    out[r] = std::min<int64_t>(std::max<int64_t>(n, lo), d->n_nets);
+    const int64_t target = (int64_t)std::ceil((double)total * r / world);
+    int64_t lo = out[r - 1], hi = d->n_nets;   // first n in [lo, n_nets] with pref(n) >= target
+    while (lo < hi) {
+      const int64_t mid = lo + (hi - lo) / 2;
+      if (pref(mid) < target) lo = mid + 1; else hi = mid;
+    }
+    out[r] = lo;
   }
   out[world] = d->n_nets;
   return DGR_OK;
@@ -110,68 +122,56 @@ int partition(const dgr_forest_desc* d, int world, std::vector<int64_t>& out) {
 // pattern recognition: each explicit path must be a straight / L / Z pattern of its sub-net
 // ---------------------------------------------------------------------------------------
 struct Seg4 { int a, b, c, d; };
-inline bool seg_less(const Seg4& x, const Seg4& y) {
-  if (x.a != y.a) return x.a < y.a;
-  if (x.b != y.b) return x.b < y.b;
-  if (x.c != y.c) return x.c < y.c;
-  return x.d < y.d;
-}
 inline bool seg_eq(const Seg4& x, const Seg4& y) { return x.a == y.a && x.b == y.b && x.c == y.c && x.d == y.d; }
-// order-insensitive equality of two small lists (n <= 3)
-inline bool same_sets(Seg4* a, Seg4* b, int n) {
-  std::sort(a, a + n, seg_less);
-  std::sort(b, b + n, seg_less);
-  for (int i = 0; i < n; ++i) if (!seg_eq(a[i], b[i])) return false;
-  return true;
-}
 
+// Which pattern of sub-net (x0,y0)-(x1,y1) (canonical: x0 <= x1) path i is, and its x_m / y_m.
+// The path's segments and turning points may come in any order: each expected one must be
+// present and the counts must agree (the expected ones of a pattern are distinct, so a duplicate
+// in the path leaves one uncovered).  The turning points fix the pattern; the segments confirm it.
 bool classify(const dgr_forest_desc* d, int64_t i, int x0, int y0, int x1, int y1, uint32_t* shape, int* mid) {
   const int64_t g0 = d->path_seg_off[i], g1 = d->path_seg_off[i + 1];
   const int64_t t0 = d->path_tp_off[i], t1 = d->path_tp_off[i + 1];
   const int ns = (int)(g1 - g0), nt = (int)(t1 - t0);
   if (ns < 1 || ns > 3 || nt != ns - 1) return false;
-  Seg4 segs[3], tps[2];
+  Seg4 segs[3];
   for (int g = 0; g < ns; ++g) {
-    const int32_t* s = d->seg + 4 * (g0 + g);
-    segs[g] = {s[0], s[1], s[2], s[3]};
+    const int32_t* sg = d->seg + 4 * (g0 + g);
+    segs[g] = {sg[0], sg[1], sg[2], sg[3]};
   }
-  for (int t = 0; t < nt; ++t) tps[t] = {d->tp_xy[2 * (t0 + t)], d->tp_xy[2 * (t0 + t) + 1], 0, 0};
-  const int ylo = std::min(y0, y1), yhi = std::max(y0, y1);
-  auto try_shape = [&](uint32_t sh, int m, std::initializer_list<Seg4> es, std::initializer_list<Seg4> et) {
-    if ((int)es.size() != ns || (int)et.size() != nt) return false;
-    Seg4 a[3], b[3], c[2], e[2];
-    int k = 0;
-    for (auto& s : es) a[k++] = s;
-    for (int q = 0; q < ns; ++q) b[q] = segs[q];
-    k = 0;
-    for (auto& s : et) c[k++] = s;
-    for (int q = 0; q < nt; ++q) e[q] = tps[q];
-    if (same_sets(a, b, ns) && same_sets(c, e, nt)) { *shape = sh; *mid = m; return true; }
+  auto has = [&](const Seg4& e) {
+    for (int q = 0; q < ns; ++q) if (seg_eq(segs[q], e)) return true;
     return false;
   };
-  if (y0 == y1) return try_shape(kStraightH, 0, {{0, y0, x0, x1}}, {});
-  if (x0 == x1) return try_shape(kStraightV, 0, {{1, x0, ylo, yhi}}, {});
-  if (ns == 2) {
-    if (try_shape(kHV, 0, {{0, y0, x0, x1}, {1, x1, ylo, yhi}}, {{x1, y0, 0, 0}})) return true;
-    return try_shape(kVH, 0, {{1, x0, ylo, yhi}, {0, y1, x0, x1}}, {{x0, y1, 0, 0}});
+  const int ylo = std::min(y0, y1), yhi = std::max(y0, y1);
+  const int32_t* tp = d->tp_xy + 2 * t0;
+  if (y0 == y1) {
+    if (ns != 1 || !has({0, y0, x0, x1})) return false;
+    *shape = kStraightH; *mid = 0; return true;
   }
-  if (ns == 3) {
-    int nh = 0;
-    for (int q = 0; q < 3; ++q) nh += segs[q].a == 0;
-    if (nh == 2) {
-      int xm = -1;
-      for (int q = 0; q < 3; ++q) if (segs[q].a == 1) xm = segs[q].b;
-      if (!(x0 < xm && xm < x1)) return false;
-      return try_shape(kZHVH, xm, {{0, y0, x0, xm}, {1, xm, ylo, yhi}, {0, y1, xm, x1}}, {{xm, y0, 0, 0}, {xm, y1, 0, 0}});
-    }
-    if (nh == 1) {
-      int ym = -1;
-      for (int q = 0; q < 3; ++q) if (segs[q].a == 0) ym = segs[q].b;
-      if (!(ylo < ym && ym < yhi)) return false;
-      return try_shape(kZVHV, ym,
-                       {{1, x0, std::min(y0, ym), std::max(y0, ym)}, {0, ym, x0, x1}, {1, x1, std::min(ym, y1), std::max(ym, y1)}},
-                       {{x0, ym, 0, 0}, {x1, ym, 0, 0}});
-    }
+  if (x0 == x1) {
+    if (ns != 1 || !has({1, x0, ylo, yhi})) return false;
+    *shape = kStraightV; *mid = 0; return true;
+  }
+  if (ns == 2) {
+    if (tp[0] == x1 && tp[1] == y0 && has({0, y0, x0, x1}) && has({1, x1, ylo, yhi})) { *shape = kHV; *mid = 0; return true; }
+    if (tp[0] == x0 && tp[1] == y1 && has({1, x0, ylo, yhi}) && has({0, y1, x0, x1})) { *shape = kVH; *mid = 0; return true; }
+    return false;
+  }
+  if (ns != 3) return false;
+  const int ax = tp[0], ay = tp[1], bx = tp[2], by = tp[3];
+  if (ax == bx && ((ay == y0 && by == y1) || (ay == y1 && by == y0))) {   // Z-HVH at x_m = ax
+    const int xm = ax;
+    if (!(x0 < xm && xm < x1)) return false;
+    if (!has({0, y0, x0, xm}) || !has({1, xm, ylo, yhi}) || !has({0, y1, xm, x1})) return false;
+    *shape = kZHVH; *mid = xm; return true;
+  }
+  if (ay == by && ((ax == x0 && bx == x1) || (ax == x1 && bx == x0))) {   // Z-VHV at y_m = ay
+    const int ym = ay;
+    if (!(ylo < ym && ym < yhi)) return false;
+    if (!has({1, x0, std::min(y0, ym), std::max(y0, ym)}) || !has({0, ym, x0, x1}) ||
+        !has({1, x1, std::min(ym, y1), std::max(ym, y1)}))
+      return false;
+    *shape = kZVHV; *mid = ym; return true;
   }
   return false;
 }
@@ -179,17 +179,32 @@ bool classify(const dgr_forest_desc* d, int64_t i, int x0, int y0, int x1, int y
 // ---------------------------------------------------------------------------------------
 // the rank's encoded shard
 // ---------------------------------------------------------------------------------------
+// Uninitialised array of a trivially copyable type (the planner writes every element in parallel;
+// std::vector would zero ~100 MB on one thread first).
+template <class T>
+struct PodBuf {
+  std::unique_ptr<T[]> p;
+  size_t n = 0;
+  void alloc(size_t count) { p.reset(count ? new T[count] : nullptr); n = count; }
+  void clear() { p.reset(); n = 0; }
+  T* data() { return p.get(); }
+  const T* data() const { return p.get(); }
+  size_t size() const { return n; }
+  T& operator[](size_t i) { return p[i]; }
+  const T& operator[](size_t i) const { return p[i]; }
+};
+
 struct Plan {
   int64_t net_lo = 0, net_hi = 0, tree_lo = 0, tree_hi = 0, sub_lo = 0, sub_hi = 0, path_lo = 0, path_hi = 0;
   int64_t nid_base = 0;                 // global noise index of the rank's first noisy candidate
   int nb = 0;
-  std::vector<int4> binfo;
-  std::vector<uint32_t> pword;
-  std::vector<short4> sxy;              // kernel order
+  PodBuf<int4> binfo;
+  PodBuf<uint32_t> pword;
+  PodBuf<short4> sxy;                   // kernel order
   std::vector<int32_t> net_tree_off;
-  std::vector<int32_t> ksub_csr;        // kernel-order sub-net -> local CSR sub-net
-  std::vector<int64_t> sub_first_slot;  // local CSR sub-net -> slot of its first candidate
-  std::vector<int32_t> slot_path;       // slot -> local CSR path (-1: padding)
+  PodBuf<int32_t> ksub_csr;             // kernel-order sub-net -> local CSR sub-net
+  PodBuf<int64_t> sub_first_slot;       // local CSR sub-net -> slot of its first candidate
+  PodBuf<int32_t> slot_path;            // slot -> local CSR path (-1: padding)
   std::vector<TileDesc> tiles;          // pipelined tiles first (see make_plan)
   int64_t n_global_tiles = 0;
   int64_t n_pipe_tiles = 0;
@@ -228,11 +243,25 @@ inline bool canonical_group(const uint32_t* shapes, int n, bool aligned) {
   return i == n;
 }
 
+struct PhaseTimer {   // DGR_PLAN_TIMING=1: host planning phases to stderr (development aid)
+  bool on = getenv("DGR_PLAN_TIMING") != nullptr;
+  std::chrono::steady_clock::time_point t = std::chrono::steady_clock::now();
+  void mark(const char* what) {
+    if (!on) return;
+    const auto n = std::chrono::steady_clock::now();
+    fprintf(stderr, "[dgr plan] %-28s %8.2f ms\n", what, std::chrono::duration<double, std::milli>(n - t).count());
+    t = n;
+  }
+};
+
 int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
+  PhaseTimer tm;
   int rc = validate_structure(d);
+  tm.mark("validate");
   if (rc) return rc;
   std::vector<int64_t> part;
   if ((rc = partition(d, world, part))) return rc;
+  tm.mark("partition");
   pl.net_lo = part[rank];
   pl.net_hi = part[rank + 1];
   pl.tree_lo = d->net_tree_off[pl.net_lo];
@@ -252,17 +281,22 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     for (int64_t s = 0; s < pl.sub_lo; ++s) cnt += lone_straight(d, s) ? 0 : d->sub_path_off[s + 1] - d->sub_path_off[s];
     pl.nid_base = cnt;
   }
+  tm.mark("noise base");
   // 1. canonical sub-net endpoints + pattern words of every local candidate (parallel over
   //    sub-nets; the first failing sub-net, in index order, is reported)
-  std::vector<short4> sxy_csr(ns);
-  std::vector<uint32_t> pw_path((size_t)(pl.path_hi - pl.path_lo));
-  std::vector<char> single((size_t)ns, 0);
+  PodBuf<short4> sxy_csr;
+  PodBuf<uint32_t> pw_path;
+  PodBuf<char> single;
+  sxy_csr.alloc(ns);
+  pw_path.alloc((size_t)(pl.path_hi - pl.path_lo));
+  single.alloc(ns);
   int64_t bad_sub = ns;   // smallest failing local sub-net
 #pragma omp parallel for schedule(dynamic, 4096) reduction(min : bad_sub)
   for (int64_t ls = 0; ls < ns; ++ls) {
     const int64_t s = pl.sub_lo + ls;
     const int32_t* e = d->sub_xy + 4 * s;
     int x0 = e[0], y0 = e[1], x1 = e[2], y1 = e[3];
+    single[ls] = 0;
     if (x0 > x1 || (x0 == x1 && y0 > y1)) { std::swap(x0, x1); std::swap(y0, y1); }
     if (x0 < 0 || x1 >= X || std::min(y0, y1) < 0 || std::max(y0, y1) >= Y || (x0 == x1 && y0 == y1)) {
       bad_sub = std::min(bad_sub, ls);
@@ -303,14 +337,30 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     return fail(DGR_EINVAL, "sub-net %lld: candidates must be straight (aligned sub-net) or HV, VH, Z-HVH..., Z-VHV... in this order",
                 (long long)s);
   }
+  tm.mark("classify");
   // local noise index of every sub-net's first candidate (-1 for lone straight paths)
-  std::vector<int64_t> nid_sub((size_t)ns);
+  PodBuf<int64_t> nid_sub;
+  nid_sub.alloc(ns);
   {
-    int64_t next = 0;
-    for (int64_t ls = 0; ls < ns; ++ls) {
-      const int64_t g = d->sub_path_off[pl.sub_lo + ls + 1] - d->sub_path_off[pl.sub_lo + ls];
-      nid_sub[ls] = single[ls] ? -1 : next;
-      next += single[ls] ? 0 : g;
+    // two-pass prefix over fixed chunks: noisy candidates per chunk, then the chunk offsets
+    constexpr int64_t kChunk = 1 << 16;
+    const int64_t nch = (ns + kChunk - 1) / kChunk;
+    std::vector<int64_t> base(nch + 1, 0);
+#pragma omp parallel for schedule(static)
+    for (int64_t ch = 0; ch < nch; ++ch) {
+      int64_t c = 0;
+      for (int64_t ls = ch * kChunk; ls < std::min(ns, (ch + 1) * kChunk); ++ls)
+        c += single[ls] ? 0 : d->sub_path_off[pl.sub_lo + ls + 1] - d->sub_path_off[pl.sub_lo + ls];
+      base[ch + 1] = c;
+    }
+    for (int64_t ch = 0; ch < nch; ++ch) base[ch + 1] += base[ch];
+#pragma omp parallel for schedule(static)
+    for (int64_t ch = 0; ch < nch; ++ch) {
+      int64_t next = base[ch];
+      for (int64_t ls = ch * kChunk; ls < std::min(ns, (ch + 1) * kChunk); ++ls) {
+        nid_sub[ls] = single[ls] ? -1 : next;
+        next += single[ls] ? 0 : d->sub_path_off[pl.sub_lo + ls + 1] - d->sub_path_off[pl.sub_lo + ls];
+      }
     }
   }
   // 2. tiles of whole nets: greedy in net order while the window (union of the nets' sub-net boxes
@@ -321,17 +371,26 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   pl.binfo.clear();
   pl.pword.clear();
   struct Pack { int nbg = 0, fill = 32, nsing = 0; int total() const { return nbg + (nsing + 31) / 32; } };
-  struct Cur { bool open = false; int64_t net0 = 0; Pack pk; int ntree = 0, nsub = 0; int bx0 = 0, by0 = 0, bx1 = -1, by1 = -1; bool global = false; } cur;
-  auto net_box = [&](int64_t n, int& bx0, int& by0, int& bx1, int& by1) {
-    bx0 = X; by0 = Y; bx1 = -1; by1 = -1;
+  struct Cur { bool open = false; int64_t net0 = 0; Pack pk; int ntree = 0, nsub = 0; int bx0 = 0, by0 = 0, bx1 = -1, by1 = -1; bool global = false; };
+  // bounding box of each net's sub-nets plus a 1-cell halo (parallel over nets)
+  PodBuf<int4> nbox;
+  nbox.alloc(nn);
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t ln = 0; ln < nn; ++ln) {
+    const int64_t n = pl.net_lo + ln;
+    int bx0 = X, by0 = Y, bx1 = -1, by1 = -1;
     const int64_t s0 = d->tree_sub_off[d->net_tree_off[n]], s1 = d->tree_sub_off[d->net_tree_off[n + 1]];
     for (int64_t s = s0; s < s1; ++s) {
       const short4 e = sxy_csr[s - pl.sub_lo];
       bx0 = std::min<int>(bx0, e.x); bx1 = std::max<int>(bx1, e.z);
       by0 = std::min<int>(by0, std::min(e.y, e.w)); by1 = std::max<int>(by1, std::max(e.y, e.w));
     }
-    bx0 = std::max(0, bx0 - 1); by0 = std::max(0, by0 - 1);
-    bx1 = std::min(X - 1, bx1 + 1); by1 = std::min(Y - 1, by1 + 1);
+    nbox[ln] = make_int4(std::max(0, bx0 - 1), std::max(0, by0 - 1), std::min(X - 1, bx1 + 1), std::min(Y - 1, by1 + 1));
+  }
+  tm.mark("net boxes");
+  auto net_box = [&](int64_t n, int& bx0, int& by0, int& bx1, int& by1) {
+    const int4 b = nbox[n - pl.net_lo];
+    bx0 = b.x; by0 = b.y; bx1 = b.z; by1 = b.w;
   };
   auto pack_net = [&](int64_t n, Pack& pk) {   // bundle packing of one net's sub-nets
     const int64_t s0 = d->tree_sub_off[d->net_tree_off[n]], s1 = d->tree_sub_off[d->net_tree_off[n + 1]];
@@ -349,62 +408,89 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     const int w = (bx1 + 1 - x0 + 1) & ~1, h = (by1 + 1 - y0 + 1) & ~1;
     return (int64_t)w * h;
   };
+  // The greedy restarts at fixed chunk boundaries (independent of the thread count) so the chunks
+  // run in parallel; each boundary costs at most one extra tile.
+  constexpr int64_t kChunkNets = 1 << 15;
+  const int64_t nchunk = std::max<int64_t>(1, (nn + kChunkNets - 1) / kChunkNets);
+  std::vector<std::vector<int64_t>> cstarts(nchunk);
+  std::vector<std::vector<char>> cglobs(nchunk);
+  std::vector<int64_t> cbad(nchunk, -1);
+#pragma omp parallel for schedule(dynamic, 1)
+  for (int64_t ch = 0; ch < nchunk; ++ch) {
+    const int64_t na = pl.net_lo + ch * kChunkNets, nb_ = std::min(pl.net_hi, na + kChunkNets);
+    Cur cur;
+    for (int64_t n = na; n < nb_; ++n) {
+      int bx0, by0, bx1, by1;
+      net_box(n, bx0, by0, bx1, by1);
+      const bool big = aligned_area(bx0, by0, bx1, by1) > kWinMax;
+      const int ntree = (int)(d->net_tree_off[n + 1] - d->net_tree_off[n]);
+      const int nsub = (int)(d->tree_sub_off[d->net_tree_off[n + 1]] - d->tree_sub_off[d->net_tree_off[n]]);
+      bool fits = cur.open && !cur.global && !big;
+      Pack pk2 = cur.pk;
+      if (fits) {
+        const int ux0 = std::min(cur.bx0, bx0), uy0 = std::min(cur.by0, by0);
+        const int ux1 = std::max(cur.bx1, bx1), uy1 = std::max(cur.by1, by1);
+        pack_net(n, pk2);
+        fits = aligned_area(ux0, uy0, ux1, uy1) <= kWinMax && pk2.nbg <= kTargetBundles && pk2.total() <= kTileBundles &&
+               cur.ntree + ntree <= kPipeTrees && cur.nsub + nsub <= kPipeSubs;
+        if (fits) { cur.bx0 = ux0; cur.by0 = uy0; cur.bx1 = ux1; cur.by1 = uy1; }
+      } else if (cur.open && cur.global && big) {
+        pack_net(n, pk2);
+        fits = pk2.total() <= kMaxBundles && cur.ntree + ntree <= kTreeMax;
+      }
+      if (fits) {
+        cur.pk = pk2; cur.ntree += ntree; cur.nsub += nsub;
+        continue;
+      }
+      // close the open tile, open a new one at net n
+      cstarts[ch].push_back(n);
+      cglobs[ch].push_back(big);
+      cur = Cur();
+      cur.open = true; cur.global = big; cur.net0 = n; cur.ntree = ntree; cur.nsub = nsub;
+      cur.bx0 = bx0; cur.by0 = by0; cur.bx1 = bx1; cur.by1 = by1;
+      pack_net(n, cur.pk);
+      if ((cur.pk.total() > kMaxBundles || ntree > kTreeMax) && cbad[ch] < 0) cbad[ch] = n;
+    }
+  }
   std::vector<int64_t> starts;
   std::vector<char> globs;
-  for (int64_t n = pl.net_lo; n < pl.net_hi; ++n) {
-    int bx0, by0, bx1, by1;
-    net_box(n, bx0, by0, bx1, by1);
-    const bool big = aligned_area(bx0, by0, bx1, by1) > kWinMax;
-    const int ntree = (int)(d->net_tree_off[n + 1] - d->net_tree_off[n]);
-    const int nsub = (int)(d->tree_sub_off[d->net_tree_off[n + 1]] - d->tree_sub_off[d->net_tree_off[n]]);
-    bool fits = cur.open && !cur.global && !big;
-    Pack pk2 = cur.pk;
-    if (fits) {
-      const int ux0 = std::min(cur.bx0, bx0), uy0 = std::min(cur.by0, by0);
-      const int ux1 = std::max(cur.bx1, bx1), uy1 = std::max(cur.by1, by1);
-      pack_net(n, pk2);
-      fits = aligned_area(ux0, uy0, ux1, uy1) <= kWinMax && pk2.nbg <= kTargetBundles && pk2.total() <= kTileBundles &&
-             cur.ntree + ntree <= kPipeTrees && cur.nsub + nsub <= kPipeSubs;
-      if (fits) { cur.bx0 = ux0; cur.by0 = uy0; cur.bx1 = ux1; cur.by1 = uy1; }
-    } else if (cur.open && cur.global && big) {
-      pack_net(n, pk2);
-      fits = pk2.total() <= kMaxBundles && cur.ntree + ntree <= kTreeMax;
+  for (int64_t ch = 0; ch < nchunk; ++ch) {
+    if (cbad[ch] >= 0) {
+      const int64_t n = cbad[ch];
+      const int ntree = (int)(d->net_tree_off[n + 1] - d->net_tree_off[n]);
+      if (ntree > kTreeMax) return fail(DGR_EINVAL, "net %lld has %d > %d trees", (long long)n, ntree, kTreeMax);
+      Pack pk;
+      pack_net(n, pk);
+      return fail(DGR_EINVAL, "net %lld needs %d > %d bundles", (long long)n, pk.total(), kMaxBundles);
     }
-    if (fits) {
-      cur.pk = pk2; cur.ntree += ntree; cur.nsub += nsub;
-      continue;
-    }
-    // close the open tile, open a new one at net n
-    starts.push_back(n);
-    globs.push_back(big);
-    cur = Cur();
-    cur.open = true; cur.global = big; cur.net0 = n; cur.ntree = ntree; cur.nsub = nsub;
-    cur.bx0 = bx0; cur.by0 = by0; cur.bx1 = bx1; cur.by1 = by1;
-    pack_net(n, cur.pk);
-    if (cur.pk.total() > kMaxBundles)
-      return fail(DGR_EINVAL, "net %lld needs %d > %d bundles", (long long)n, cur.pk.total(), kMaxBundles);
-    if (ntree > kTreeMax) return fail(DGR_EINVAL, "net %lld has %d > %d trees", (long long)n, ntree, kTreeMax);
+    starts.insert(starts.end(), cstarts[ch].begin(), cstarts[ch].end());
+    globs.insert(globs.end(), cglobs[ch].begin(), cglobs[ch].end());
   }
   starts.push_back(pl.net_hi);
+  tm.mark("tiles (greedy)");
   // 3. bundles, tile by tile: the tile's group bundles (packing restarts at each tile), then its
   //    singleton bundles; sub-nets renumbered in that order ("kernel order").  Count per tile,
   //    prefix, then fill the tiles in parallel (each owns a contiguous bundle and sub-net range).
   const int64_t ntile = (int64_t)starts.size() - 1;
   std::vector<int32_t> tb0(ntile + 1, 0), tbg(ntile, 0);
+#pragma omp parallel for schedule(dynamic, 64)
   for (int64_t t = 0; t < ntile; ++t) {
     Pack pk;
     for (int64_t n = starts[t]; n < starts[t + 1]; ++n) pack_net(n, pk);
     tbg[t] = pk.nbg;
-    tb0[t + 1] = tb0[t] + pk.total();
+    tb0[t + 1] = pk.total();
   }
+  for (int64_t t = 0; t < ntile; ++t) tb0[t + 1] += tb0[t];
   const size_t nslot = (size_t)tb0[ntile] * 32;
-  pl.binfo.assign(tb0[ntile], make_int4(0, 0, 0, 0));
-  pl.pword.assign(nslot, kPad | kSubHead);
-  pl.slot_path.assign(nslot, -1);
-  pl.sxy.resize(ns);
-  pl.ksub_csr.resize(ns);
-  pl.sub_first_slot.resize(ns);
+  // every element is written by the parallel fill below (padding slots included)
+  pl.binfo.alloc(tb0[ntile]);
+  pl.pword.alloc(nslot);
+  pl.slot_path.alloc(nslot);
+  pl.sxy.alloc(ns);
+  pl.ksub_csr.alloc(ns);
+  pl.sub_first_slot.alloc(ns);
   pl.tiles.assign(ntile, TileDesc{});
+  tm.mark("bundle counts + alloc");
 #pragma omp parallel
   {
     std::vector<uint16_t> cnt;
@@ -431,6 +517,13 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       T.sub0 = (int32_t)(d->tree_sub_off[d->net_tree_off[starts[t]]] - pl.sub_lo);
       T.nsub = (int32_t)(d->tree_sub_off[d->net_tree_off[starts[t + 1]]] - pl.sub_lo) - T.sub0;
       const int64_t j0 = d->net_tree_off[starts[t]], j1 = d->net_tree_off[starts[t + 1]];
+      for (int b = T.b0; b < T.b0 + T.nb; ++b) {
+        pl.binfo[b] = make_int4(0, 0, 0, 0);
+        for (int l = 0; l < 32; ++l) {
+          pl.pword[(size_t)b * 32 + l] = kPad | kSubHead;
+          pl.slot_path[(size_t)b * 32 + l] = -1;
+        }
+      }
       int ks = T.sub0;   // next kernel-order sub-net
       // group bundles
       int fill = 32, b = T.b0 - 1, prev_tree = -1;
@@ -518,6 +611,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       pl.tiles[t] = T;
     }
   }
+  tm.mark("bundles + event check");
   pl.n_global_tiles = 0;
   for (const auto& T : pl.tiles) pl.n_global_tiles += T.global;
   pl.nb = (int)pl.binfo.size();
@@ -603,6 +697,10 @@ struct dgr_handle {
   float t_last = 1.f;
   float beta_last = 0.25f;
   bool have_forward = false;
+  // the grids hold the demand events of the forward of iteration k at temperature t_fwd (the
+  // last iteration of the previous dgr_step call ran it), so the next call can start from them
+  bool fwd_valid = false;
+  float t_fwd = 0.f;
   double* pinned = nullptr;   // 16 doubles of pinned host memory
   // profiling: a CUDA event after every stage, attributed to that stage
   bool prof = false;
@@ -677,8 +775,7 @@ int64_t dgr_workspace_size(const dgr_forest_desc* desc, const dgr_dist* dist) {
   return (int64_t)make_layout(pl, desc->X, desc->Y, induce_metric_blocks(tmp)).total;
 }
 
-int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev_workspace, int64_t workspace_bytes,
-                    void* cuda_stream, dgr_handle** out) {
+int dgr_forest_plan(const dgr_forest_desc* desc, const dgr_dist* dist, void* cuda_stream, dgr_handle** out) {
   g_err.clear();
   if (!out) return fail(DGR_EINVAL, "out is NULL");
   *out = nullptr;
@@ -686,23 +783,58 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
   if ((rc = dist_args(dist, &rank, &world))) return rc;
   auto* h = new dgr_handle();
   if ((rc = make_plan(desc, rank, world, h->plan))) { delete h; return rc; }
-  const Plan& pl = h->plan;
   h->X = desc->X; h->Y = desc->Y;
   h->n_nets = desc->n_nets; h->n_trees = desc->n_trees; h->n_subnets = desc->n_subnets; h->n_paths = desc->n_paths;
   h->rank = rank; h->world = world;
   h->stream = (cudaStream_t)cuda_stream;
-  KParams& P = h->P;
-  P.X = desc->X; P.Y = desc->Y;
-  h->lay = make_layout(pl, desc->X, desc->Y, induce_metric_blocks(P));
-  const Layout& L = h->lay;
-  if (!dev_workspace || workspace_bytes < (int64_t)L.total) {
-    delete h;
-    return fail(DGR_ENOMEM, "workspace of %lld bytes < %zu needed", (long long)workspace_bytes, L.total);
+  h->P.X = desc->X; h->P.Y = desc->Y;
+  h->lay = make_layout(h->plan, desc->X, desc->Y, induce_metric_blocks(h->P));
+  *out = h;
+  return DGR_OK;
+}
+
+int64_t dgr_handle_workspace_size(dgr_handle* h) {
+  g_err.clear();
+  if (!h) { fail(DGR_EINVAL, "NULL handle"); return 0; }
+  return (int64_t)h->lay.total;
+}
+
+int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev_workspace, int64_t workspace_bytes,
+                    void* cuda_stream, dgr_handle** out) {
+  g_err.clear();
+  if (!out) return fail(DGR_EINVAL, "out is NULL");
+  *out = nullptr;
+  dgr_handle* h = nullptr;
+  int rc;
+  if ((rc = dgr_forest_plan(desc, dist, cuda_stream, &h))) return rc;
+  if ((rc = dgr_bind_workspace(h, desc, dist, dev_workspace, workspace_bytes))) {
+    const std::string msg = g_err;
+    dgr_free(h);
+    g_err = msg;
+    return rc;
   }
-  if (((uintptr_t)dev_workspace) & 255) { delete h; return fail(DGR_EINVAL, "workspace not 256-byte aligned"); }
-  h->ws = (char*)dev_workspace;
-  h->ws_bytes = workspace_bytes;
-  char* ws = h->ws;
+  *out = h;
+  return DGR_OK;
+}
+
+int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dist* dist, void* dev_workspace,
+                       int64_t workspace_bytes) {
+  g_err.clear();
+  if (!h || !desc) return fail(DGR_EINVAL, "NULL handle or desc");
+  if (h->ws) return fail(DGR_ESTATE, "the handle already has a workspace");
+  if (desc->X != h->X || desc->Y != h->Y || desc->n_nets != h->n_nets || desc->n_trees != h->n_trees ||
+      desc->n_subnets != h->n_subnets || desc->n_paths != h->n_paths)
+    return fail(DGR_EINVAL, "desc does not describe the planned forest");
+  int rank, world, rc;
+  if ((rc = dist_args(dist, &rank, &world))) return rc;
+  if (rank != h->rank || world != h->world) return fail(DGR_EINVAL, "dist differs from the one planned with");
+  const Plan& pl = h->plan;
+  KParams& P = h->P;
+  const Layout& L = h->lay;
+  if (!dev_workspace || workspace_bytes < (int64_t)L.total)
+    return fail(DGR_ENOMEM, "workspace of %lld bytes < %zu needed", (long long)workspace_bytes, L.total);
+  if (((uintptr_t)dev_workspace) & 255) return fail(DGR_EINVAL, "workspace not 256-byte aligned");
+  char* ws = (char*)dev_workspace;
   P.nb = pl.nb;
   P.ntiles = (int32_t)pl.n_pipe_tiles;
   P.tiles = (const TileDesc*)(ws + L.tiles);
@@ -747,19 +879,26 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
   P.ipartial = (double*)(ws + L.ipartial);
   P.metrics = (double*)(ws + L.metrics);
 
-  auto cleanup = [&](int code) { if (h->pinned) cudaFreeHost(h->pinned); delete h; return code; };
+  auto cleanup = [&](int code) {   // back to the planned state
+    if (h->pinned) { cudaFreeHost(h->pinned); h->pinned = nullptr; }
+    h->P = KParams{};
+    h->P.X = h->X; h->P.Y = h->Y;
+    return code;
+  };
   cudaStream_t s = h->stream;
   if (prepare_kernels() != 0) return cleanup(fail(DGR_ECUDA, "cudaFuncSetAttribute (tile kernel shared memory) failed"));
   if (cudaMemsetAsync(ws, 0, L.total, s) != cudaSuccess) return cleanup(fail(DGR_ECUDA, "memset workspace failed"));
   // host-side staging of the encoded shard
   const size_t slots = (size_t)pl.nb * 32;
   std::vector<float> wslots(slots, 0.f), pslots(slots, 0.f);
+#pragma omp parallel for schedule(static)
   for (size_t sl = 0; sl < slots; ++sl)
     if (pl.slot_path[sl] >= 0) {
       wslots[sl] = desc->w_path0[pl.path_lo + pl.slot_path[sl]];
       pslots[sl] = 1.f;   // p of a lone straight candidate (never rewritten by the pipelined kernel)
     }
   std::vector<float> capVT(G);
+#pragma omp parallel for schedule(static)
   for (int y = 0; y < desc->Y; ++y)
     for (int x = 0; x < desc->X; ++x) capVT[(size_t)x * desc->Y + y] = desc->cap_v[(size_t)y * desc->X + x];
   const size_t nt = (size_t)(pl.tree_hi - pl.tree_lo);
@@ -787,14 +926,15 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
     ncclResult_t r = ncclCommInitRank(&h->comm, world, id, rank);
     if (r != ncclSuccess) return cleanup(fail(DGR_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r)));
   }
-  *out = h;
-  g_err.clear();
+  h->ws = ws;
+  h->ws_bytes = workspace_bytes;
   return DGR_OK;
 }
 
 int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w, dgr_loss* last) {
   g_err.clear();
   if (!h || !w) return fail(DGR_EINVAL, "NULL handle or weights");
+  if (!h->ws) return fail(DGR_ESTATE, "no workspace bound (dgr_bind_workspace)");
   if (iters < 0) return fail(DGR_EINVAL, "iters < 0");
   if (!(temperature > 0.f) || !std::isfinite(temperature)) return fail(DGR_EINVAL, "temperature must be > 0");
   if (w->f_kind < 0 || w->f_kind > 4) return fail(DGR_EINVAL, "f_kind must be 0..4 (sigmoid, ReLU, LeakyReLU, exp, CELU)");
@@ -815,16 +955,26 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
     a.inv_sqrt_bc2 = (float)(1.0 / std::sqrt(1.0 - std::pow(0.999, step)));
   };
   int rc;
-  // forward of iteration k (q, p, demand events of the current logits at this temperature)
+  // forward of iteration k (q, p, demand events of the current logits at this temperature),
+  // unless the previous call left exactly that forward in the grids
   a.k = h->k;
   a.k_next = h->k;
   a.store_d = 0;
   adam_args(h->k);
   if ((rc = prof_mark(h, -1))) return rc;
-  const size_t vd_bytes = 8 * (size_t)h->X * h->Y;
-  CUDA_TRY(cudaMemsetAsync(P.VD, 0, vd_bytes, s));   // KG clears dH / dV^T in place; VD here
-  launch_tiles(P, a, kForwardOnly, s);
-  if ((rc = prof_mark(h, 0))) return rc;
+  const size_t grid_bytes = 8 * (size_t)h->X * h->Y;
+  if (!(h->fwd_valid && h->t_fwd == temperature)) {
+    // KG clears dH / dV^T in place after reading them; stale events of a forward at another
+    // temperature are cleared here.  VD is cleared before every forward.
+    if (h->fwd_valid) {
+      CUDA_TRY(cudaMemsetAsync(P.dH, 0, 2 * grid_bytes, s));   // dH | dV^T
+      CUDA_TRY(cudaMemsetAsync(P.scal, 0, 2 * sizeof(long long), s));
+    }
+    CUDA_TRY(cudaMemsetAsync(P.VD, 0, grid_bytes, s));
+    launch_tiles(P, a, kForwardOnly, s);
+    if ((rc = prof_mark(h, 0))) return rc;
+  }
+  h->fwd_valid = false;
   const int n = iters == 0 ? 1 : iters;
   for (int it = 0; it < n; ++it) {
     const bool last = (it == n - 1);
@@ -839,12 +989,17 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
     launch_kg(P, a, s);
     if ((rc = prof_mark(h, 2))) return rc;
     if (iters > 0) {
-      // reverse of iteration k + (unless last) forward of k+1
-      if (!last) CUDA_TRY(cudaMemsetAsync(P.VD, 0, vd_bytes, s));
-      launch_tiles(P, a, last ? kReverseOnly : kReverseForward, s);
+      // reverse of iteration k + forward of k+1 (also after the last iteration: the next call
+      // at the same temperature starts from it)
+      CUDA_TRY(cudaMemsetAsync(P.VD, 0, grid_bytes, s));
+      launch_tiles(P, a, kReverseForward, s);
       h->k += 1;
+      if ((rc = prof_mark(h, 3))) return rc;
     }
-    if (iters > 0 && (rc = prof_mark(h, last ? 4 : 3))) return rc;
+  }
+  if (iters > 0) {
+    h->fwd_valid = true;
+    h->t_fwd = temperature;
   }
   CUDA_TRY(cudaGetLastError());
   h->t_last = temperature;
@@ -864,6 +1019,7 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
 int dgr_get_demand(dgr_handle* h, float* d_h, float* d_v) {
   g_err.clear();
   if (!h || !d_h || !d_v) return fail(DGR_EINVAL, "NULL argument");
+  if (!h->ws) return fail(DGR_ESTATE, "no workspace bound (dgr_bind_workspace)");
   if (!h->have_forward) return fail(DGR_ESTATE, "no forward has run yet");
   const size_t G = (size_t)h->X * h->Y;
   std::vector<float> vt(G);
@@ -878,6 +1034,7 @@ int dgr_get_demand(dgr_handle* h, float* d_h, float* d_v) {
 int dgr_get_logits(dgr_handle* h, float* w_tree, float* w_path) {
   g_err.clear();
   if (!h) return fail(DGR_EINVAL, "NULL handle");
+  if (!h->ws) return fail(DGR_ESTATE, "no workspace bound (dgr_bind_workspace)");
   const Plan& pl = h->plan;
   if (w_path) {
     std::vector<float> slots((size_t)pl.nb * 32);
@@ -899,6 +1056,7 @@ int dgr_induce(dgr_handle* h, float top_p, int32_t* tree_choice, int32_t* route,
   g_err.clear();
   if (!h || !tree_choice || !route || !nucleus_off || !nucleus || !D_h || !D_v || !metrics)
     return fail(DGR_EINVAL, "NULL argument");
+  if (!h->ws) return fail(DGR_ESTATE, "no workspace bound (dgr_bind_workspace)");
   if (!(top_p >= 0.f) || !std::isfinite(top_p)) return fail(DGR_EINVAL, "top_p must be finite and >= 0");
   KParams& P = h->P;
   const Plan& pl = h->plan;

@@ -91,6 +91,10 @@ def load_library():
     L.dgr_workspace_size.argtypes = [c.POINTER(_Desc), c.POINTER(_Dist)]
     L.dgr_workspace_size.restype = c.c_int64
     L.dgr_forest_load.argtypes = [c.POINTER(_Desc), c.POINTER(_Dist), vp, c.c_int64, vp, c.POINTER(vp)]
+    L.dgr_forest_plan.argtypes = [c.POINTER(_Desc), c.POINTER(_Dist), vp, c.POINTER(vp)]
+    L.dgr_handle_workspace_size.argtypes = [vp]
+    L.dgr_handle_workspace_size.restype = c.c_int64
+    L.dgr_bind_workspace.argtypes = [vp, c.POINTER(_Desc), c.POINTER(_Dist), vp, c.c_int64]
     L.dgr_step.argtypes = [vp, c.c_int32, c.c_float, c.c_float, c.POINTER(Weights), c.POINTER(Loss)]
     L.dgr_get_demand.argtypes = [vp, _PF, _PF]
     L.dgr_get_logits.argtypes = [vp, _PF, _PF]
@@ -100,7 +104,8 @@ def load_library():
     L.dgr_free.argtypes = [vp]
     L.dgr_profile.argtypes = [vp, c.c_int32]
     L.dgr_profile_read.argtypes = [vp, c.POINTER(c.c_double), _P64]
-    for fn in ("dgr_nccl_unique_id", "dgr_partition", "dgr_forest_load", "dgr_step", "dgr_get_demand",
+    for fn in ("dgr_nccl_unique_id", "dgr_partition", "dgr_forest_load", "dgr_forest_plan", "dgr_bind_workspace",
+               "dgr_step", "dgr_get_demand",
                "dgr_get_logits", "dgr_induce", "dgr_get_info", "dgr_free", "dgr_profile", "dgr_profile_read", "dgr_plan_info"):
         getattr(L, fn).restype = c.c_int
     _lib = L
@@ -220,14 +225,17 @@ class Solver:
             dist = _Dist(rank, world, ctypes.cast(self._idbuf, ctypes.c_void_p))
         self._dist = dist
         distp = ctypes.byref(dist) if dist is not None else None
-        nbytes = L.dgr_workspace_size(ctypes.byref(self._d.desc), distp)
+        # plan once on the host, then bind a torch-allocated workspace (dgr_forest_plan + dgr_bind_workspace)
+        self._h = ctypes.c_void_p()
+        _check(L.dgr_forest_plan(ctypes.byref(self._d.desc), distp, ctypes.c_void_p(self.stream.cuda_stream),
+                                 ctypes.byref(self._h)))
+        nbytes = L.dgr_handle_workspace_size(self._h)
         if nbytes <= 0:
-            raise DgrError("dgr_workspace_size: " + L.dgr_last_error().decode())
+            raise DgrError("dgr_handle_workspace_size: " + L.dgr_last_error().decode())
         with torch.cuda.device(self.device):
             self.workspace = torch.empty(int(nbytes), dtype=torch.uint8, device=self.device)
-        self._h = ctypes.c_void_p()
-        _check(L.dgr_forest_load(ctypes.byref(self._d.desc), distp, ctypes.c_void_p(self.workspace.data_ptr()),
-                                 int(nbytes), ctypes.c_void_p(self.stream.cuda_stream), ctypes.byref(self._h)))
+        _check(L.dgr_bind_workspace(self._h, ctypes.byref(self._d.desc), distp,
+                                    ctypes.c_void_p(self.workspace.data_ptr()), int(nbytes)))
         self.workspace_bytes = int(nbytes)
 
     # ----------------------------------------------------------------------------------
