@@ -915,6 +915,8 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   cp(L.slot_path, pl.slot_path.data(), 4 * slots);
   cp(L.nto, pl.net_tree_off.data(), 4 * pl.net_tree_off.size());
   cp(L.wt, desc->w_tree0 + pl.tree_lo, 4 * nt);
+  const std::vector<float> ones(nt, 1.f);   // q of a net's lone tree stays 1 (never rewritten)
+  cp(L.q, ones.data(), 4 * nt);
   cp(L.capH, desc->cap_h, 4 * G);
   cp(L.capVT, capVT.data(), 4 * G);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);

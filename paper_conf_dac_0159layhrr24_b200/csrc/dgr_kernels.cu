@@ -678,8 +678,9 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
 constexpr size_t kGpOffset = 3 * 4 * kWinMax;   // tile path noise, after the event window in St.S
 template <bool REV, bool FWD, int NT>
 __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A, const TileDesc& T, Stage St,
-                                             int* ev_s, float* gp, long long* dq_s, long long& wl_acc,
-                                             long long& tp_acc) {
+                                             int* ev_s, float* gp, long long* dq_s, long long* red_s) {
+  // dq_s[0..ntree) and red_s[0..2) arrive zeroed (the caller clears them before its first barrier)
+  long long wl_acc = 0, tp_acc = 0;
   constexpr int NW = NT / 32;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int X = P.X, Y = P.Y;
@@ -690,9 +691,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   const int nbg = T.nbg;
 
   // ---------------- reverse of iteration k ----------------
-  if (REV) {
-    for (int i = tid; i < T.ntree; i += NT) dq_s[i] = 0;
-    __syncthreads();
+  if (REV) {   // dq_s was zeroed before the stage arrived
     for (int lb = warp; lb < T.nb; lb += NW) {
       const int4 bi = St.bi[lb];
       const uint32_t pw = St.pw[lb * 32 + lane];
@@ -754,65 +753,56 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     __syncthreads();
   }
 
-  // ---------------- tree level (one thread per tree; S window reused as scratch) ----------------
+  // ---------------- net level (one thread per net), event window cleared alongside ----------------
+  if (FWD) {
+    int4* z = reinterpret_cast<int4*>(ev_s);   // the S window is free after the reverse
+    for (int i = tid; i < (3 * ncell + 3) / 4; i += NT) z[i] = make_int4(0, 0, 0, 0);
+  }
   if (!(P.skip & 16)) {
-    double* qd = St.S;                                            // q_j dq_j
-    float* zt = reinterpret_cast<float*>(qd + kPipeTrees);        // (w_j + g_j)/t
-    float* gt = zt + kPipeTrees;                                   // Gumbel noise of the tile's trees
-    short* tfirst = reinterpret_cast<short*>(gt + kPipeTrees + 8); // first tree of the tree's net (tile-local)
-    short* tcnt = tfirst + kPipeTrees;                             // trees of that net
+    const uint2 key = make_uint2((uint32_t)P.seed, (uint32_t)(P.seed >> 32));
     for (int n = tid; n < T.nnet; n += NT) {
-      const int a = St.nto[T.net0 + n - n_lo] - T.tree0, b = St.nto[T.net0 + n + 1 - n_lo] - T.tree0;
-      for (int j = a; j < b; ++j) { tfirst[j] = (short)a; tcnt[j] = (short)(b - a); }
-    }
-    if (FWD) {
-      // one Philox call per 4 consecutive tree candidates (stream 1)
-      const int64_t g0 = P.tree_base + T.tree0;
-      const int64_t c0 = g0 >> 2, c1 = (g0 + T.ntree - 1) >> 2;
-      const uint2 key = make_uint2((uint32_t)P.seed, (uint32_t)(P.seed >> 32));
-      for (int64_t c = c0 + tid; c <= c1; c += NT) {
-        const uint4 r = philox4x32_10(make_uint4((uint32_t)c, (uint32_t)(c >> 32), (uint32_t)A.k_next, 1u), key);
-        const uint32_t wd[4] = {r.x, r.y, r.z, r.w};
-#pragma unroll
-        for (int q = 0; q < 4; ++q) {
-          const int64_t i = c * 4 + q - g0;
-          if (i >= 0 && i < T.ntree) gt[i] = gumbel_word(wd[q]);
-        }
+      const int a = St.nto[T.net0 + n - n_lo] - t_lo, b = St.nto[T.net0 + n + 1 - n_lo] - t_lo;   // stage indices
+      if (b - a == 1) {
+        // a lone tree: q = 1 and du = 0 always (its logit and Adam state never change)
+        if (FWD) St.q[a] = 1.f;
+        continue;
       }
-    }
-    if (REV)
-      for (int j = tid; j < T.ntree; j += NT) qd[j] = (double)St.q[j + T.tree0 - t_lo] * ((double)dq_s[j] * kDqInv);
-    __syncthreads();
-    for (int j = tid; j < T.ntree; j += NT) {
-      const int a = tfirst[j], cnt = tcnt[j], jg = j + T.tree0;
-      float wj = St.wt[jg - t_lo];
       if (REV) {
         // du_j = (q_j/t)(dq_j - sum_l q_l dq_l / sum_l q_l); Adam on w_tree (iteration k)
         double sq = 0.0, sw = 0.0;
-        for (int l = a; l < a + cnt; ++l) { sq += qd[l]; sw += (double)St.q[l + T.tree0 - t_lo]; }
-        const double du = cnt == 1 ? 0.0
-                                   : (double)St.q[jg - t_lo] * (double)A.inv_t * ((double)dq_s[j] * kDqInv - sq / sw);
-        float m = St.mt[jg - t_lo], v = St.vt[jg - t_lo];
-        adam_update(wj, m, v, (float)du, A);
-        P.wt[jg] = wj; P.mt[jg] = m; P.vt[jg] = v;
-      }
-      if (FWD) zt[j] = (wj + gt[j]) * A.inv_t;
-    }
-    if (FWD) {
-      __syncthreads();
-      // q_j = softmax over the net's trees of (w_j + g_j)/t, iteration k_next
-      for (int j = tid; j < T.ntree; j += NT) {
-        const int a = tfirst[j], cnt = tcnt[j], jg = j + T.tree0;
-        float q = 1.f;
-        if (cnt > 1) {
-          float zmax = -INFINITY;
-          for (int l = a; l < a + cnt; ++l) zmax = fmaxf(zmax, zt[l]);
-          float sum = 0.f;
-          for (int l = a; l < a + cnt; ++l) sum += __expf(zt[l] - zmax);
-          q = __expf(zt[j] - zmax) / sum;
+        for (int l = a; l < b; ++l) {
+          const double ql = (double)St.q[l];
+          sq += ql * ((double)dq_s[l + t_lo - T.tree0] * kDqInv);
+          sw += ql;
         }
-        St.q[jg - t_lo] = q;
-        P.q[jg] = q;
+        sq /= sw;
+        for (int j = a; j < b; ++j) {
+          const double du = (double)St.q[j] * (double)A.inv_t * ((double)dq_s[j + t_lo - T.tree0] * kDqInv - sq);
+          float w = St.wt[j], m = St.mt[j], v = St.vt[j];
+          adam_update(w, m, v, (float)du, A);
+          St.wt[j] = w;
+          const int jg = j + t_lo;
+          P.wt[jg] = w; P.mt[jg] = m; P.vt[jg] = v;
+        }
+      }
+      if (FWD) {
+        // q_j = softmax over the net's trees of (w_j + g_j)/t, iteration k_next (noise stream 1)
+        float zmax = -INFINITY;
+        for (int j = a; j < b; ++j) {
+          const int64_t gj = P.tree_base + t_lo + j;
+          const uint4 r = philox4x32_10(make_uint4((uint32_t)(gj >> 2), (uint32_t)(gj >> 34), (uint32_t)A.k_next, 1u), key);
+          const uint32_t wd = (gj & 3) == 0 ? r.x : (gj & 3) == 1 ? r.y : (gj & 3) == 2 ? r.z : r.w;
+          const float zj = (St.wt[j] + gumbel_word(wd)) * A.inv_t;
+          St.q[j] = zj;
+          zmax = fmaxf(zmax, zj);
+        }
+        float sum = 0.f;
+        for (int j = a; j < b; ++j) sum += __expf(St.q[j] - zmax);
+        for (int j = a; j < b; ++j) {
+          const float q = __expf(St.q[j] - zmax) / sum;
+          St.q[j] = q;
+          P.q[j + t_lo] = q;
+        }
       }
     }
   }
@@ -838,11 +828,6 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
 
   // ---------------- forward of iteration k_next ----------------
   if (FWD) {
-    {
-      int4* z = reinterpret_cast<int4*>(ev_s);
-      for (int i = tid; i < (3 * ncell + 3) / 4; i += NT) z[i] = make_int4(0, 0, 0, 0);
-    }
-    __syncthreads();
     const uint32_t ev_base = smem_u32(ev_s);
     const int nid0 = nbg > 0 ? St.bi[0].x : 0;
     for (int lb = warp; lb < T.nb; lb += NW) {
@@ -918,8 +903,16 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         }
       }
     }
+    // E[WL], E[TP] partial sums: warp reduction, then one shared atomic per warp
+    wl_acc = seg_reduce(wl_acc, lane, 31, Sum());
+    tp_acc = seg_reduce(tp_acc, lane, 31, Sum());
+    if (lane == 0) {
+      atomicAdd(reinterpret_cast<unsigned long long*>(&red_s[0]), static_cast<unsigned long long>(wl_acc));
+      atomicAdd(reinterpret_cast<unsigned long long*>(&red_s[1]), static_cast<unsigned long long>(tp_acc));
+    }
   }
   __syncthreads();
+  if (FWD && tid == 32) { red64(P.scal, red_s[0]); red64(P.scal + 1, red_s[1]); }
   // write back the tile's group slot state with bulk stores (asynchronous; readers wait on the group)
   if (tid == 0 && nbg > 0) {
     fence_proxy_async();
@@ -961,22 +954,6 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   }
 }
 
-// E[WL], E[TP] partial sums of the block -> the exchange buffer
-template <int NT>
-__device__ __forceinline__ void flush_scalars(const KParams& P, long long wl, long long tp, long long* red_s) {
-  const int lane = threadIdx.x & 31;
-  if (threadIdx.x < 2) red_s[threadIdx.x] = 0;
-  __syncthreads();
-  wl = seg_reduce(wl, lane, 31, Sum());
-  tp = seg_reduce(tp, lane, 31, Sum());
-  if (lane == 0) {
-    atomicAdd(reinterpret_cast<unsigned long long*>(&red_s[0]), static_cast<unsigned long long>(wl));
-    atomicAdd(reinterpret_cast<unsigned long long*>(&red_s[1]), static_cast<unsigned long long>(tp));
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) { red64(P.scal, red_s[0]); red64(P.scal + 1, red_s[1]); }
-}
-
 // (a) one tile per CTA: the whole tile arrives by bulk copies on one mbarrier; the event window
 // and noise alias the S window.  4 CTAs per SM overlap one CTA's copies with the others' math.
 #ifndef DGR_BTHREADS
@@ -1002,12 +979,12 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
     mbar_init(bar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  for (int i = threadIdx.x; i < kPipeTrees; i += kBThreads) dq_s[i] = 0;
+  if (threadIdx.x < 2) red_s[threadIdx.x] = 0;
   __syncthreads();
   if (threadIdx.x < 32) issue_tile_loads<REV>(P, T, smem, bar);
   mbar_wait(bar, 0u);
-  long long wl = 0, tp = 0;
-  process_tile<REV, FWD, kBThreads>(P, A, T, St, ev_s, gp, dq_s, wl, tp);
-  if (FWD) flush_scalars<kBThreads>(P, wl, tp, red_s);
+  process_tile<REV, FWD, kBThreads>(P, A, T, St, ev_s, gp, dq_s, red_s);
   if (threadIdx.x == 0) bulk_wait_read();   // the stage must outlive the bulk stores' reads
 }
 
@@ -1033,7 +1010,6 @@ __global__ void __launch_bounds__(kPThreads, kPPerSM) tile_persistent(KParams P,
   }
   __syncthreads();
   if (warp == 0 && (int)blockIdx.x < P.ntiles) issue_tile_loads<REV>(P, P.tiles[blockIdx.x], stage_base[0], &bars[0]);
-  long long wl = 0, tp = 0;
   for (int it = 0;; ++it) {
     const int tile = blockIdx.x + it * gridDim.x;
     if (tile >= P.ntiles) break;
@@ -1043,14 +1019,16 @@ __global__ void __launch_bounds__(kPThreads, kPPerSM) tile_persistent(KParams P,
       __syncwarp();
       issue_tile_loads<REV>(P, P.tiles[tile + gridDim.x], stage_base[sidx ^ 1], &bars[sidx ^ 1]);
     }
+    for (int i = tid; i < kPipeTrees; i += kPThreads) dq_s[i] = 0;
+    if (tid < 2) red_s[tid] = 0;
+    __syncthreads();
     mbar_wait(&bars[sidx], (uint32_t)(it >> 1) & 1u);
     Stage St(stage_base[sidx]);
     int* ev_s = reinterpret_cast<int*>(St.S);
     float* gp = reinterpret_cast<float*>(reinterpret_cast<unsigned char*>(St.S) + kGpOffset);
-    process_tile<REV, FWD, kPThreads>(P, A, P.tiles[tile], St, ev_s, gp, dq_s, wl, tp);
+    process_tile<REV, FWD, kPThreads>(P, A, P.tiles[tile], St, ev_s, gp, dq_s, red_s);
     __syncthreads();
   }
-  if (FWD) flush_scalars<kPThreads>(P, wl, tp, red_s);
   if (tid == 0) bulk_wait_all();
 }
 

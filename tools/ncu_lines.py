@@ -44,3 +44,25 @@ if __name__ == "__main__":
     print("\n# by stall samples")
     for f, ln, i, s, src in sorted(L, key=lambda x: -x[3])[:top]:
         print(f"{f + ':' + str(ln):28s} {100 * i / tot_i:6.2f} {100 * s / tot_s:6.2f}  {src[:90]}")
+
+
+def stall_lines(path, reason, top=15):
+    """Source lines with the most samples of one stall reason (e.g. 'stall_long_sb')."""
+    raw = subprocess.run(["ncu", "-i", path, "--page", "source", "--csv", "--print-source", "cuda,sass"],
+                         capture_output=True, text=True).stdout
+    rows = list(csv.reader(io.StringIO(raw)))
+    hdr = next(r for r in rows if r and r[0] == "Line No")
+    col = hdr.index(reason)
+    out, fname = [], None
+    for r in rows:
+        if r and r[0] == "File Path":
+            fname = r[1].split("/")[-1]
+        elif r and re.match(r"^\d+$", r[0] or ""):
+            try:
+                v = float(r[col].replace(",", ""))
+            except ValueError:
+                v = 0.0
+            out.append((v, f"{fname}:{r[0]}", r[1].strip()[:90]))
+    tot = sum(v for v, _, _ in out) or 1
+    for v, loc, src in sorted(out, reverse=True)[:top]:
+        print(f"{loc:28s} {100 * v / tot:6.2f}  {src}")
