@@ -886,7 +886,9 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
     return code;
   };
   cudaStream_t s = h->stream;
+  PhaseTimer tm;
   if (prepare_kernels() != 0) return cleanup(fail(DGR_ECUDA, "cudaFuncSetAttribute (tile kernel shared memory) failed"));
+  tm.mark("bind: prepare kernels");
   if (cudaMemsetAsync(ws, 0, L.total, s) != cudaSuccess) return cleanup(fail(DGR_ECUDA, "memset workspace failed"));
   // host-side staging of the encoded shard
   const size_t slots = (size_t)pl.nb * 32;
@@ -902,6 +904,7 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   for (int y = 0; y < desc->Y; ++y)
     for (int x = 0; x < desc->X; ++x) capVT[(size_t)x * desc->Y + y] = desc->cap_v[(size_t)y * desc->X + x];
   const size_t nt = (size_t)(pl.tree_hi - pl.tree_lo);
+  tm.mark("bind: host staging");
   cudaError_t e = cudaSuccess;
   auto cp = [&](size_t off, const void* src, size_t bytes) {
     if (bytes && e == cudaSuccess) e = cudaMemcpyAsync(ws + off, src, bytes, cudaMemcpyHostToDevice, s);
@@ -920,6 +923,7 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   cp(L.capH, desc->cap_h, 4 * G);
   cp(L.capVT, capVT.data(), 4 * G);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  tm.mark("bind: upload");
   if (e != cudaSuccess) return cleanup(fail(DGR_ECUDA, "upload: %s", cudaGetErrorString(e)));
   if (cudaMallocHost(&h->pinned, 16 * sizeof(double)) != cudaSuccess) return cleanup(fail(DGR_ECUDA, "cudaMallocHost failed"));
   if (world > 1) {
