@@ -184,7 +184,7 @@ int dgr_plan_info(const dgr_forest_desc* desc, const dgr_dist* dist, int64_t out
  * stream after every stage.  enable != 0 starts (and clears) recording, 0 stops it.
  * dgr_profile_read synchronises and returns, per stage, the summed milliseconds and the number of
  * launches: 0 KF (forward-only tile kernel, once per dgr_step call), 1 demand allreduce (NCCL;
- * world > 1), 2 KG (scan / loss / gradient map; 2 kernels), 3 KBF (reverse of k fused with the
+ * world > 1), 2 KG (scan / loss / gradient map; 1 kernel), 3 KBF (reverse of k fused with the
  * forward of k+1), 4 KB (reverse only; not launched since every call ends with KBF), 5..7 unused. */
 int dgr_profile(struct dgr_handle* h, int32_t enable);
 int dgr_profile_read(struct dgr_handle* h, double ms[8], int64_t launches[8]);

@@ -630,7 +630,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
 // ---------------------------------------------------------------------------------------
 struct Layout {
   size_t tiles, binfo, pword, sxy, slot_path, wp, mp, vp, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
-      partial, loss, chosen, tree_choice, route, nsize, nucleus_tmp, DHVC, iscal, ipartial, metrics, total;
+      partial, kg_count, loss, chosen, tree_choice, route, nsize, nucleus_tmp, DHVC, iscal, ipartial, metrics, total;
   size_t xcount;   // int64 elements in the exchange buffer
 };
 
@@ -666,6 +666,7 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.dOutH = take(4 * G);
   L.dOutVT = take(4 * G);
   L.partial = take(8 * (size_t)(X + Y));
+  L.kg_count = take(16);
   L.loss = take(8 * 4);
   L.chosen = take(nt);
   L.tree_choice = take(4 * nn);
@@ -866,6 +867,7 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   P.SH = (double*)(ws + L.SH); P.SVT = (double*)(ws + L.SVT);
   P.dOutH = (float*)(ws + L.dOutH); P.dOutVT = (float*)(ws + L.dOutVT);
   P.partial = (double*)(ws + L.partial);
+  P.kg_count = (unsigned int*)(ws + L.kg_count);
   P.loss = (double*)(ws + L.loss);
   P.chosen = (uint8_t*)(ws + L.chosen);
   P.tree_choice = (int32_t*)(ws + L.tree_choice);

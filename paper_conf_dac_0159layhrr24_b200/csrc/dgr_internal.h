@@ -104,6 +104,7 @@ struct KParams {
   float* dOutH;             // [Y][X]
   float* dOutVT;            // [X][Y]
   double* partial;          // [Y + X] overflow partial sums
+  unsigned int* kg_count;   // CTAs of the current KG launch that are done (the last one finalises)
   double* loss;             // [4]
   // induce scratch
   uint8_t* chosen;          // [n_trees_l]

@@ -1111,7 +1111,28 @@ __device__ __forceinline__ void striped_exclusive_scan(T (&v)[kGItems], T* sh /*
   __syncthreads();
 }
 
-__global__ void __launch_bounds__(kGThreads) kg_kernel(KParams P, StepArgs A) {
+__device__ __forceinline__ void kg_finalize(const KParams& P, const StepArgs& A) {
+  __shared__ double sh[32];
+  const int nl = P.X + P.Y;
+  double s = 0.0;
+  for (int i = threadIdx.x; i < nl; i += blockDim.x) s += __ldcg(&P.partial[i]);
+  double tot;
+  block_exclusive_scan(s, sh, &tot);
+  if (threadIdx.x == 0) {
+    const double ewl = (double)__ldcg(&P.scal[0]) * kFixInv;
+    const double etp = (double)__ldcg(&P.scal[1]) * kFixInv;
+    const double via = (double)A.sqrt_l * etp;
+    P.loss[0] = (double)A.a_wl * ewl + (double)A.a_via * via + (double)A.a_of * tot;
+    P.loss[1] = ewl;
+    P.loss[2] = via;
+    P.loss[3] = tot;
+    P.scal[0] = 0;
+    P.scal[1] = 0;
+    *P.kg_count = 0;
+  }
+}
+
+__global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A) {
   __shared__ long long shl[kGItems * (kGThreads / 32)];
   __shared__ double shd[kGItems * (kGThreads / 32)];
   const int line = blockIdx.x;
@@ -1199,28 +1220,17 @@ __global__ void __launch_bounds__(kGThreads) kg_kernel(KParams P, StepArgs A) {
   // deterministic block reduction of the overflow cost
   double tot;
   block_exclusive_scan(of, shd, &tot);
-  if (threadIdx.x == 0) P.partial[line] = tot;
+  // the last CTA to finish sums the per-line partials in line order and writes the loss
+  __shared__ bool last;
+  if (threadIdx.x == 0) {
+    P.partial[line] = tot;
+    __threadfence();
+    last = atomicAdd(P.kg_count, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (last) kg_finalize(P, A);
 }
 
-__global__ void __launch_bounds__(256) kg_finalize_kernel(KParams P, StepArgs A) {
-  __shared__ double sh[32];
-  const int nl = P.X + P.Y;
-  double s = 0.0;
-  for (int i = threadIdx.x; i < nl; i += blockDim.x) s += P.partial[i];
-  double tot;
-  block_exclusive_scan(s, sh, &tot);
-  if (threadIdx.x == 0) {
-    const double ewl = (double)P.scal[0] * kFixInv;
-    const double etp = (double)P.scal[1] * kFixInv;
-    const double via = (double)A.sqrt_l * etp;
-    P.loss[0] = (double)A.a_wl * ewl + (double)A.a_via * via + (double)A.a_of * tot;
-    P.loss[1] = ewl;
-    P.loss[2] = via;
-    P.loss[3] = tot;
-    P.scal[0] = 0;
-    P.scal[1] = 0;
-  }
-}
 
 // ------------------------------------------------------------------------------------------
 // Induction (§4.5): KI1 argmax tree per net; KI2 top-p nucleus + route per sub-net of the
@@ -1396,7 +1406,6 @@ void launch_tiles(const KParams& p, const StepArgs& a, TileMode mode, cudaStream
 }
 void launch_kg(const KParams& p, const StepArgs& a, cudaStream_t s) {
   kg_kernel<<<p.X + p.Y, kGThreads, 0, s>>>(p, a);
-  kg_finalize_kernel<<<1, 256, 0, s>>>(p, a);
 }
 int induce_metric_blocks(const KParams& p) {
   const int64_t ncell = (int64_t)p.X * p.Y;
