@@ -622,6 +622,11 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   std::stable_partition(pl.tiles.begin(), pl.tiles.end(), pipelined);
   pl.n_pipe_tiles = 0;
   for (const auto& T : pl.tiles) pl.n_pipe_tiles += pipelined(T);
+  {   // largest tiles first (LPT): a shorter tail of the last wave of CTAs (+1.5% on ispd19)
+    std::stable_sort(pl.tiles.begin(), pl.tiles.begin() + pl.n_pipe_tiles, [](const TileDesc& a, const TileDesc& b) {
+      return 4 * a.nbg + (a.nb - a.nbg) > 4 * b.nbg + (b.nb - b.nbg);
+    });
+  }
   return DGR_OK;
 }
 
