@@ -27,6 +27,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "dgr_oracle.c")
+_SRC_FOREST = os.path.join(_HERE, "forest_oracle.c")   # row f1: DAG-forest construction
 _LIB = os.path.join(_HERE, "liboracle.so")
 _LIB32 = os.path.join(_HERE, "liboracle32.so")   # conditioning probe only (same source, real = float)
 _libs = {}
@@ -34,7 +35,7 @@ _libs = {}
 
 def build(verbose: bool = False) -> str:
     for out, extra in ((_LIB, []), (_LIB32, ["-DODGR_REAL=float"])):
-        cmd = ["gcc", "-O2", "-std=c11", "-shared", "-fPIC", *extra, "-o", out, _SRC, "-lm"]
+        cmd = ["gcc", "-O2", "-std=c11", "-shared", "-fPIC", *extra, "-o", out, _SRC, _SRC_FOREST, "-lm"]
         if verbose:
             print(" ".join(cmd))
         subprocess.check_call(cmd)
@@ -62,7 +63,7 @@ _u32 = np.ctypeslib.ndpointer(dtype=np.uint32, flags="C_CONTIGUOUS")
 def _load(fp32: bool = False):
     path = _LIB32 if fp32 else _LIB
     if path not in _libs:
-        if not os.path.exists(path) or os.path.getmtime(path) < os.path.getmtime(_SRC):
+        if not os.path.exists(path) or os.path.getmtime(path) < max(os.path.getmtime(_SRC), os.path.getmtime(_SRC_FOREST)):
             build()
         L = ctypes.CDLL(path)
         vp, c = ctypes.c_void_p, ctypes
@@ -98,6 +99,11 @@ def _load(fp32: bool = False):
         L.odgr_induce.argtypes = [vp, c.c_double, c.c_double, c.c_double, _i32, _i32, _i64, _i32, _i32, _i32,
                                   _dp, _dp, _dp, _dp]
         L.odgr_real_bytes.restype = c.c_int32
+        L.odgr_build_forest.restype = vp
+        L.odgr_build_forest.argtypes = [c.c_int64, _i64, _i32, c.c_int32, c.c_int32, c.c_uint64]
+        L.odgr_forest_sizes.argtypes = [vp, _i64]
+        L.odgr_forest_copy.argtypes = [vp] + [_i64] * 5 + [_i32] * 3 + [_f32] * 2
+        L.odgr_forest_free.argtypes = [vp]
         _libs[path] = L
     return _libs[path]
 
@@ -243,3 +249,28 @@ class Oracle:
                             r.metrics, r.margin_tree, r.margin_route, r.margin_nucleus)
         r.nucleus = r.nucleus[: r.nucleus_off[-1]].copy()
         return r
+
+
+def build_forest(net_pin_off, pin_xy, n_tree_cand: int = 2, z_cap: int = 15, seed: int = 1) -> dict:
+    """Row f1 oracle (forest_oracle.c): the routing DAG forest of the given nets' pins (§4.2,
+    P:524-539; readings Q8, Q14, Q17).  Returns the CSR arrays of include/dgr.h's forest."""
+    L = _load()
+    npo = np.ascontiguousarray(net_pin_off, dtype=np.int64)
+    pxy = np.ascontiguousarray(np.asarray(pin_xy, dtype=np.int32).reshape(-1))
+    h = L.odgr_build_forest(len(npo) - 1, npo, pxy, int(n_tree_cand), int(z_cap), int(seed))
+    try:
+        sz = np.zeros(5, np.int64)
+        L.odgr_forest_sizes(h, sz)
+        nt, ns, np_, ng, ntp = (int(v) for v in sz)
+        out = dict(net_tree_off=np.zeros(len(npo), np.int64), tree_sub_off=np.zeros(nt + 1, np.int64),
+                   sub_path_off=np.zeros(ns + 1, np.int64), path_seg_off=np.zeros(np_ + 1, np.int64),
+                   path_tp_off=np.zeros(np_ + 1, np.int64), sub_xy=np.zeros((max(ns, 1), 4), np.int32),
+                   seg=np.zeros((max(ng, 1), 4), np.int32), tp_xy=np.zeros((max(ntp, 1), 2), np.int32),
+                   w_tree0=np.zeros(max(nt, 1), np.float32), w_path0=np.zeros(max(np_, 1), np.float32))
+        L.odgr_forest_copy(h, out["net_tree_off"], out["tree_sub_off"], out["sub_path_off"], out["path_seg_off"],
+                           out["path_tp_off"], out["sub_xy"], out["seg"], out["tp_xy"], out["w_tree0"], out["w_path0"])
+        out["sub_xy"], out["seg"], out["tp_xy"] = out["sub_xy"][:ns], out["seg"][:ng], out["tp_xy"][:ntp]
+        out["w_tree0"], out["w_path0"] = out["w_tree0"][:nt], out["w_path0"][:np_]
+        return out
+    finally:
+        L.odgr_forest_free(h)

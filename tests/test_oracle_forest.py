@@ -1,0 +1,131 @@
+"""Row f1 oracle (oracle/forest_oracle.c): routing-DAG-forest construction (§4.2, P:524-539;
+readings Q8, Q14, Q17 in DESIGN.md §3), pinned against library routines and closed forms."""
+import numpy as np
+import pytest
+from scipy.sparse.csgraph import minimum_spanning_tree
+
+import forestgen
+import oracle
+
+
+def _built(f):
+    c = f.meta["config"]
+    return oracle.build_forest(f.net_pin_off, f.pin_xy, c["n_tree_cand"], c["z_cap"], c["seed"])
+
+
+def _tree_subs(o, n):
+    """sub-nets (x0, y0, x1, y1) of each tree of net n"""
+    out = []
+    for j in range(o["net_tree_off"][n], o["net_tree_off"][n + 1]):
+        out.append(o["sub_xy"][o["tree_sub_off"][j]:o["tree_sub_off"][j + 1]])
+    return out
+
+
+def _manhattan_mst(pts):
+    d = np.abs(pts[:, None, :] - pts[None, :, :]).sum(-1).astype(float)
+    d[d == 0] = 1e-9          # distinct points only; keep zero-length edges representable
+    np.fill_diagonal(d, 0)
+    return minimum_spanning_tree(d).sum()
+
+
+@pytest.fixture(scope="module")
+def c1e4_built(c1e4):
+    return _built(c1e4)
+
+
+def test_oracle_equals_the_input_generator(tiny, c1e4, c1e4_built):
+    """Two independent statements of readings Q8/Q14/Q17 (forestgen's generator and the oracle)
+    agree bit for bit on every array."""
+    for f, o in ((tiny, _built(tiny)), (c1e4, c1e4_built)):
+        for k, v in o.items():
+            np.testing.assert_array_equal(np.asarray(getattr(f, k)).reshape(v.shape), v, err_msg=k)
+
+
+def test_candidate0_is_a_minimum_spanning_tree(c1e4, c1e4_built):
+    """Candidate 0 = Prim MST (Q17): its length equals scipy's minimum spanning tree (Manhattan)."""
+    o = c1e4_built
+    for n in range(0, c1e4.n_nets, 7):
+        pins = c1e4.pin_xy[c1e4.net_pin_off[n]:c1e4.net_pin_off[n + 1]]
+        t0 = _tree_subs(o, n)[0]
+        assert len(t0) == len(pins) - 1
+        length = np.abs(t0[:, 2] - t0[:, 0]).sum() + np.abs(t0[:, 3] - t0[:, 1]).sum()
+        assert abs(length - _manhattan_mst(pins.astype(np.int64))) < 1e-6
+
+
+def _components(points, subs):
+    idx = {tuple(p): i for i, p in enumerate(points)}
+    parent = list(range(len(points)))
+
+    def find(a):
+        while parent[a] != a:
+            parent[a] = parent[parent[a]]
+            a = parent[a]
+        return a
+    for s in subs:
+        a, b = find(idx[(s[0], s[1])]), find(idx[(s[2], s[3])])
+        parent[a] = b
+    return len({find(i) for i in range(len(points))})
+
+
+def test_candidate1_is_a_steiner_tree_no_longer_than_the_mst(c1e4, c1e4_built):
+    """Candidate 1 (iterated 1-Steiner, k <= 8): a tree over the pins plus Steiner points of degree
+    >= 3, no longer than the MST, and exactly the half-perimeter (the RSMT closed form) for 3 pins."""
+    o = c1e4_built
+    checked3 = 0
+    for n in range(c1e4.n_nets):
+        pins = c1e4.pin_xy[c1e4.net_pin_off[n]:c1e4.net_pin_off[n + 1]]
+        trees = _tree_subs(o, n)
+        if len(trees) < 2:
+            continue
+        t0, t1 = trees
+        l0 = np.abs(t0[:, 2] - t0[:, 0]).sum() + np.abs(t0[:, 3] - t0[:, 1]).sum()
+        l1 = np.abs(t1[:, 2] - t1[:, 0]).sum() + np.abs(t1[:, 3] - t1[:, 1]).sum()
+        pts = {tuple(p) for p in pins}
+        ends = {(s[0], s[1]) for s in t1} | {(s[2], s[3]) for s in t1}
+        assert pts <= ends
+        steiner = ends - pts
+        allp = [tuple(p) for p in pins] + sorted(steiner)
+        assert len(t1) == len(allp) - 1 and _components(allp, t1) == 1
+        deg = {p: 0 for p in steiner}
+        for s in t1:
+            for e in ((s[0], s[1]), (s[2], s[3])):
+                if e in deg:
+                    deg[e] += 1
+        assert all(v >= 3 for v in deg.values())
+        if len(pins) <= 8:
+            assert l1 <= l0
+        if len(pins) == 3:
+            hp = pins[:, 0].max() - pins[:, 0].min() + pins[:, 1].max() - pins[:, 1].min()
+            assert l1 == hp
+            checked3 += 1
+    assert checked3 > 50
+
+
+def test_path_candidates_are_the_patterns(tiny):
+    """Every candidate is a monotone route between its sub-net's endpoints (length |dx| + |dy|,
+    turning points = segments - 1), groups are straight / HV, VH, Z... (Q14, all Z on tiny)."""
+    o = _built(tiny)
+    for s in range(len(o["sub_path_off"]) - 1):
+        x0, y0, x1, y1 = o["sub_xy"][s]
+        a, b = o["sub_path_off"][s], o["sub_path_off"][s + 1]
+        aligned = x0 == x1 or y0 == y1
+        assert (b - a) == (1 if aligned else 2 + max(x1 - x0 - 1, 0) + max(abs(y1 - y0) - 1, 0))
+        for i in range(a, b):
+            segs = o["seg"][o["path_seg_off"][i]:o["path_seg_off"][i + 1]]
+            tps = o["path_tp_off"][i + 1] - o["path_tp_off"][i]
+            assert (segs[:, 3] - segs[:, 2]).sum() == (x1 - x0) + abs(y1 - y0)
+            assert tps == len(segs) - 1
+
+
+def test_initial_logits_uniform(c1e4_built):
+    w = np.concatenate([c1e4_built["w_tree0"], c1e4_built["w_path0"]])
+    assert w.min() >= 0.0 and w.max() < 1.0 and abs(w.mean() - 0.5) < 0.01
+
+
+def test_single_tree_candidate_and_l_only():
+    f = forestgen.generate("c1e4", n_tree_cand=1, z_cap=-1)
+    o = _built(f)
+    assert np.all(np.diff(o["net_tree_off"]) == 1)
+    assert np.diff(o["sub_path_off"]).max() <= 2
+    for k, v in o.items():
+        np.testing.assert_array_equal(np.asarray(getattr(f, k)).reshape(v.shape), v, err_msg=k)
