@@ -163,6 +163,34 @@ def paper_schedule_quality(s, W):
             "wl": float(r.metrics[3]), "tp": float(r.metrics[4]), "iterations": 1000, "top_p": 0.9}
 
 
+def forest_build_timing(f, dgr, torch, stream, with_cpu: bool) -> dict:
+    """Row f1: the workload's forest rebuilt from its nets' pins on the GPU (dgr_build_forest, one
+    thread per net), wall clock incl. the pins' H2D and the size readback; the CPU oracle of f1
+    (oracle/forest_oracle.c, one thread) on a bounded sample of the same nets alongside."""
+    c = f.meta["config"]
+    args = (f.X, f.Y, f.net_pin_off, f.pin_xy, c["n_tree_cand"], c["z_cap"], c["seed"])
+    dgr.build_forest(*args, stream=stream).close()          # warm-up (module load, pool)
+    times = []
+    for _ in range(3):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        b = dgr.build_forest(*args, stream=stream)
+        torch.cuda.synchronize()
+        times.append(time.perf_counter() - t0)
+        b.close()
+    out = {"nets": f.n_nets, "gpu_ms": 1e3 * min(times), "gpu_nets_per_s": f.n_nets / min(times),
+           "note": "GPU: pins -> trees (MST, 1-Steiner), sub-nets, L/Z paths, w0; equals the oracle's forest"}
+    if with_cpu:
+        import oracle
+        n = min(f.n_nets, 100000)
+        t0 = time.perf_counter()
+        oracle.build_forest(f.net_pin_off[:n + 1], f.pin_xy[:f.net_pin_off[n]], c["n_tree_cand"], c["z_cap"], c["seed"])
+        dt = time.perf_counter() - t0
+        out["cpu_oracle_nets_per_s"] = n / dt
+        out["cpu_sample"] = f"first {n} nets, 1 thread"
+    return out
+
+
 def cpu_baseline(f, seconds_target=12.0):
     """The oracle as it stands (fp64, single thread) on this host on a bounded sample: whole-forest
     iterations of the same workload until ~seconds_target of CPU work."""
@@ -310,6 +338,7 @@ def main():
     loss = s.step(0, 1.0, 0.3, W)
     t_ind0 = time.perf_counter(); s.induce(0.9); induce_ms = (time.perf_counter() - t_ind0) * 1e3
     quality = None if args.no_quality else paper_schedule_quality(s, W)
+    forest_build = forest_build_timing(f, dgr, torch, stream, with_cpu=(rank == 0 and not args.no_cpu_baseline))
 
     cells = f.X * f.Y
     slow = 1 if info["n_tiles"] > info.get("n_pipe_tiles", info["n_tiles"]) else 0
@@ -362,6 +391,7 @@ def main():
         "induce_ms": induce_ms,
         "loss": {"total": float(loss[0]), "wl": float(loss[1]), "via": float(loss[2]), "overflow": float(loss[3])},
         "quality": quality,
+        "forest_build": forest_build,
         "hbm_footprint_bytes": info["workspace_bytes"],
         "e2e": {"value": e2e_iters / e2e_s, "unit": "iters/s", "h2d_bytes_per_step": h2d / e2e_iters,
                 "d2h_bytes_per_step": d2h / e2e_iters,

@@ -192,6 +192,43 @@ int dgr_profile_read(struct dgr_handle* h, double ms[8], int64_t launches[8]);
 /* Releases the handle (and the NCCL communicator); the workspace stays the caller's. */
 int dgr_free(struct dgr_handle* h);
 
+/* ---------------------------------------------------------------------------------------------
+ * Row f1: routing-DAG-forest construction on the GPU, one thread per net (§4.2; the
+ * paper leaves it to "net-level parallelism").  Readings: tree
+ * candidates Q17 (Prim MST from pin 0; iterated 1-Steiner on the Hanan grid for <= 8 pins, else
+ * Prim from the last pin; a duplicate second candidate is dropped), sub-nets = tree edges in Prim
+ * order with canonical endpoints, paths Q14 (straight, or HV, VH, z_cap-limited Z-HVH / Z-VHV),
+ * initial logits Q8 (U[0,1), splitmix64 counter hash of (seed, 3 / 4, index)).  The result equals
+ * forestgen's forest for the same pins, bit for bit.
+ * ------------------------------------------------------------------------------------------- */
+typedef struct {
+  int32_t X, Y;                 /* grid, 2..32767 per side */
+  int64_t n_nets;
+  const int64_t* net_pin_off;   /* [n_nets+1] host */
+  const int32_t* pin_xy;        /* [n_pins][2] host; 2..32 distinct in-grid pins per net */
+  int32_t n_tree_cand;          /* 1 or 2 */
+  int32_t z_cap;                /* -1: L only; 0: every Z; > 0: at most z_cap Z per direction */
+  uint64_t seed;                /* of the initial logits */
+} dgr_pins_desc;
+
+struct dgr_built_forest;
+
+/* Builds the forest on cuda_stream into device memory owned by the returned object
+ * (cudaMallocAsync; released by dgr_built_forest_free).  Pins are read during the call only.
+ * Synchronises (the output sizes are data-dependent).  DGR_EINVAL for malformed pins. */
+int dgr_build_forest(const dgr_pins_desc* pins, void* cuda_stream, struct dgr_built_forest** out);
+
+/* sizes = {nets, trees, sub-nets, paths, segments, turning points} */
+int dgr_built_forest_sizes(const struct dgr_built_forest* f, int64_t sizes[6]);
+
+/* Copies the forest into caller-owned host arrays shaped like dgr_forest_desc's (any may be NULL
+ * to skip it).  Synchronises. */
+int dgr_built_forest_download(const struct dgr_built_forest* f, int64_t* net_tree_off, int64_t* tree_sub_off,
+                              int64_t* sub_path_off, int64_t* path_seg_off, int64_t* path_tp_off,
+                              int32_t* sub_xy, int32_t* seg, int32_t* tp_xy, float* w_tree0, float* w_path0);
+
+int dgr_built_forest_free(struct dgr_built_forest* f);
+
 #ifdef __cplusplus
 }
 #endif

@@ -5,7 +5,8 @@ The product is ``libdgr.so`` (C ABI in ``include/dgr.h``, sm_100a kernels in ``c
 solver iteration runs in the CUDA kernels.  There is no CPU fallback: without the
 extension or a GPU the binding raises.
 """
-from .dgr import (DgrError, Loss, Solver, Weights, lib_path, load_library, nccl_unique_id,  # noqa: F401
-                  partition, plan_info)
+from .dgr import (BuiltForest, DgrError, Loss, Solver, Weights, build_forest, lib_path, load_library,  # noqa: F401
+                  nccl_unique_id, partition, plan_info)
 
-__all__ = ["Solver", "Weights", "Loss", "DgrError", "partition", "nccl_unique_id", "load_library", "lib_path", "plan_info"]
+__all__ = ["Solver", "Weights", "Loss", "DgrError", "partition", "nccl_unique_id", "load_library", "lib_path", "plan_info",
+           "build_forest", "BuiltForest"]

@@ -8,7 +8,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libdgr.so")
-SOURCES = [os.path.join(CSRC, f) for f in ("dgr_api.cu", "dgr_kernels.cu")]
+SOURCES = [os.path.join(CSRC, f) for f in ("dgr_api.cu", "dgr_kernels.cu", "dgr_forest.cu")]
 HEADERS = [os.path.join(CSRC, "dgr_internal.h"), os.path.join(ROOT, "include", "dgr.h")]
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",

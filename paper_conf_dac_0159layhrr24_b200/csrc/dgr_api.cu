@@ -688,6 +688,11 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
 
 }  // namespace
 
+namespace dgr {
+int set_error(int code, const char* msg) { g_err = msg; return code; }
+void clear_error() { g_err.clear(); }
+}  // namespace dgr
+
 struct dgr_handle {
   int X = 0, Y = 0;
   int64_t n_nets = 0, n_trees = 0, n_subnets = 0, n_paths = 0;

@@ -140,5 +140,7 @@ void launch_induce_metrics(const KParams& p, float beta, cudaStream_t s);
 int induce_metric_blocks(const KParams& p);
 size_t tile_smem_bytes();
 int prepare_kernels();   // sets shared-memory attributes; returns cudaError_t
+int set_error(int code, const char* msg);   // the thread's dgr_last_error message (dgr_api.cu)
+void clear_error();
 
 }  // namespace dgr

@@ -39,6 +39,12 @@ class _Desc(ctypes.Structure):
                 ("seed", ctypes.c_uint64)]
 
 
+class _PinsDesc(ctypes.Structure):
+    _fields_ = [("X", ctypes.c_int32), ("Y", ctypes.c_int32), ("n_nets", ctypes.c_int64),
+                ("net_pin_off", ctypes.c_void_p), ("pin_xy", ctypes.c_void_p), ("n_tree_cand", ctypes.c_int32),
+                ("z_cap", ctypes.c_int32), ("seed", ctypes.c_uint64)]
+
+
 class _Dist(ctypes.Structure):
     _fields_ = [("rank", ctypes.c_int32), ("world", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p)]
 
@@ -104,6 +110,12 @@ def load_library():
     L.dgr_free.argtypes = [vp]
     L.dgr_profile.argtypes = [vp, c.c_int32]
     L.dgr_profile_read.argtypes = [vp, c.POINTER(c.c_double), _P64]
+    L.dgr_build_forest.argtypes = [c.POINTER(_PinsDesc), vp, c.POINTER(vp)]
+    L.dgr_built_forest_sizes.argtypes = [vp, _P64]
+    L.dgr_built_forest_download.argtypes = [vp] + [vp] * 10
+    L.dgr_built_forest_free.argtypes = [vp]
+    for fn in ("dgr_build_forest", "dgr_built_forest_sizes", "dgr_built_forest_download", "dgr_built_forest_free"):
+        getattr(L, fn).restype = c.c_int
     for fn in ("dgr_nccl_unique_id", "dgr_partition", "dgr_forest_load", "dgr_forest_plan", "dgr_bind_workspace",
                "dgr_step", "dgr_get_demand",
                "dgr_get_logits", "dgr_induce", "dgr_get_info", "dgr_free", "dgr_profile", "dgr_profile_read", "dgr_plan_info"):
@@ -307,3 +319,54 @@ class Solver:
             self.close()
         except Exception:
             pass
+
+
+class BuiltForest:
+    """Row f1: a routing DAG forest built on the GPU from the nets' pins (dgr_build_forest).
+    The device arrays are owned by libdgr; download() copies them into host numpy arrays."""
+
+    def __init__(self, X: int, Y: int, net_pin_off, pin_xy, n_tree_cand: int = 2, z_cap: int = 15, seed: int = 1,
+                 stream=None):
+        import torch
+        if not torch.cuda.is_available():
+            raise DgrError("libdgr needs a CUDA device (no CPU fallback)")
+        L = load_library()
+        self.X, self.Y = int(X), int(Y)
+        npo = np.ascontiguousarray(net_pin_off, np.int64)
+        pxy = np.ascontiguousarray(np.asarray(pin_xy, np.int32).reshape(-1))
+        st = stream if stream is not None else torch.cuda.current_stream()
+        d = _PinsDesc(self.X, self.Y, len(npo) - 1, npo.ctypes.data, pxy.ctypes.data, int(n_tree_cand), int(z_cap),
+                      int(seed))
+        self._h = ctypes.c_void_p()
+        _check(L.dgr_build_forest(ctypes.byref(d), ctypes.c_void_p(st.cuda_stream), ctypes.byref(self._h)))
+        sz = np.zeros(6, np.int64)
+        _check(L.dgr_built_forest_sizes(self._h, sz.ctypes.data_as(ctypes.POINTER(ctypes.c_int64))))
+        self.n_nets, self.n_trees, self.n_subnets, self.n_paths, self.n_segs, self.n_tps = (int(v) for v in sz)
+
+    def download(self) -> dict:
+        out = dict(net_tree_off=np.zeros(self.n_nets + 1, np.int64), tree_sub_off=np.zeros(self.n_trees + 1, np.int64),
+                   sub_path_off=np.zeros(self.n_subnets + 1, np.int64),
+                   path_seg_off=np.zeros(self.n_paths + 1, np.int64), path_tp_off=np.zeros(self.n_paths + 1, np.int64),
+                   sub_xy=np.zeros((self.n_subnets, 4), np.int32), seg=np.zeros((self.n_segs, 4), np.int32),
+                   tp_xy=np.zeros((self.n_tps, 2), np.int32), w_tree0=np.zeros(self.n_trees, np.float32),
+                   w_path0=np.zeros(self.n_paths, np.float32))
+        order = ("net_tree_off", "tree_sub_off", "sub_path_off", "path_seg_off", "path_tp_off", "sub_xy", "seg",
+                 "tp_xy", "w_tree0", "w_path0")
+        _check(load_library().dgr_built_forest_download(self._h, *[ctypes.c_void_p(out[k].ctypes.data) for k in order]))
+        return out
+
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            load_library().dgr_built_forest_free(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def build_forest(X, Y, net_pin_off, pin_xy, n_tree_cand=2, z_cap=15, seed=1, stream=None) -> BuiltForest:
+    """dgr_build_forest (row f1): the routing DAG forest of the nets' pins, built on the GPU."""
+    return BuiltForest(X, Y, net_pin_off, pin_xy, n_tree_cand, z_cap, seed, stream)
