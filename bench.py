@@ -169,12 +169,13 @@ def forest_build_timing(f, dgr, torch, stream, with_cpu: bool) -> dict:
     (oracle/forest_oracle.c, one thread) on a bounded sample of the same nets alongside."""
     c = f.meta["config"]
     args = (f.X, f.Y, f.net_pin_off, f.pin_xy, c["n_tree_cand"], c["z_cap"], c["seed"])
-    dgr.build_forest(*args, stream=stream).close()          # warm-up (module load, pool)
+    kw = dict(stream=stream, c_cap=c.get("c_cap", 0))
+    dgr.build_forest(*args, **kw).close()          # warm-up (module load, pool)
     times = []
     for _ in range(3):
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        b = dgr.build_forest(*args, stream=stream)
+        b = dgr.build_forest(*args, **kw)
         torch.cuda.synchronize()
         times.append(time.perf_counter() - t0)
         b.close()
@@ -184,7 +185,8 @@ def forest_build_timing(f, dgr, torch, stream, with_cpu: bool) -> dict:
         import oracle
         n = min(f.n_nets, 100000)
         t0 = time.perf_counter()
-        oracle.build_forest(f.net_pin_off[:n + 1], f.pin_xy[:f.net_pin_off[n]], c["n_tree_cand"], c["z_cap"], c["seed"])
+        oracle.build_forest(f.X, f.Y, f.net_pin_off[:n + 1], f.pin_xy[:f.net_pin_off[n]], c["n_tree_cand"], c["z_cap"],
+                            c["seed"], c.get("c_cap", 0))
         dt = time.perf_counter() - t0
         out["cpu_oracle_nets_per_s"] = n / dt
         out["cpu_sample"] = f"first {n} nets, 1 thread"

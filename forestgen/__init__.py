@@ -37,6 +37,7 @@ class _Config(ctypes.Structure):
         ("box_mu", ctypes.c_double), ("cluster_frac", ctypes.c_double), ("n_hotspots", ctypes.c_int32),
         ("track", ctypes.c_double), ("beta_pin", ctypes.c_double), ("n_tree_cand", ctypes.c_int32),
         ("z_cap", ctypes.c_int32), ("seed", ctypes.c_uint64), ("local_weight", ctypes.c_double),
+        ("c_cap", ctypes.c_int32),
     ]
 
 
@@ -128,6 +129,15 @@ CONFIGS: dict[str, dict] = {
     "ispd19": dict(X=1000, Y=1000, n_nets=1_000_000, pins_mode=1, box_mode=1, box_mu=5.0,
                    cluster_frac=0.3, n_hotspots=32, track=4.0, beta_pin=0.25, n_tree_cand=2, z_cap=15,
                    seed=1),
+    # row f4 (C-shape detours, Q14b): groups stay <= 32 (2 L + 2x11 Z + up to 2x2x2 C)
+    "tiny_c": dict(X=16, Y=16, n_nets=40, pins_mode=0, pins_min=2, pins_max=4, box_mode=0, box_min=2,
+                   box_max=8, cluster_frac=0.0, n_hotspots=0, track=1.0, beta_pin=0.0, n_tree_cand=2,
+                   z_cap=0, c_cap=2, seed=3),
+    "c1e4_c": dict(X=256, Y=256, n_nets=10_000, pins_mode=1, box_mode=1, box_mu=8.0, cluster_frac=0.0,
+                   n_hotspots=0, track=1.0, beta_pin=0.25, n_tree_cand=2, z_cap=11, c_cap=2, seed=1),
+    "ispd19_c": dict(X=1000, Y=1000, n_nets=1_000_000, pins_mode=1, box_mode=1, box_mu=5.0,
+                     cluster_frac=0.3, n_hotspots=32, track=4.0, beta_pin=0.25, n_tree_cand=2, z_cap=11,
+                     c_cap=2, seed=1),
     **{f"table1_r{i + 1}": _table1(*row) for i, row in enumerate(TABLE1_ROWS)},
     "sweep1e4": _sweep(10_000),
     "sweep1e5": _sweep(100_000),
@@ -202,7 +212,7 @@ def generate(config: str | dict, seed: int | None = None, gumbel_seed: int = GUM
     c = _Config()
     defaults = dict(pins_min=2, pins_max=4, box_min=2, box_max=8, box_mu=5.0, cluster_frac=0.0,
                     n_hotspots=0, track=1.0, beta_pin=0.0, n_tree_cand=2, z_cap=15, seed=1,
-                    pins_mode=0, box_mode=0, local_weight=1.0)
+                    pins_mode=0, box_mode=0, local_weight=1.0, c_cap=0)
     for k, v in {**defaults, **cfg}.items():
         setattr(c, k, v)
     lib = _load()

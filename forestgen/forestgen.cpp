@@ -7,7 +7,8 @@
 //       candidate 0 = Prim rectilinear MST, candidate 1 = iterated 1-Steiner on the
 //       Hanan grid (k <= 8 pins) else a re-rooted MST; duplicates dropped
 //   * tree -> 2-pin sub-nets                    — P:534-536
-//   * L-shape path enumeration plus Z-shapes (§3.1)
+//   * L-shape path enumeration plus Z-shapes (§3.1) and
+//     optional C-shape detours (Q14b, row f4)
 //   * capacities per Eq. (1) with a hotspot map
 //   * random initial logits w0 ~ U[0,1)
 // None of the solver's arithmetic lives here.
@@ -159,7 +160,14 @@ inline void add_seg(NetOut& o, int dir, int line, int a, int b) {
 }
 inline void add_tp(NetOut& o, int x, int y) { o.tp.push_back(x); o.tp.push_back(y); }
 
-void enumerate_paths(const Sub& s, int z_cap, NetOut& o) {
+// C-shape detour positions outside [lo, hi] (reading Q14b): lo-c .. lo-1, then hi+1 .. hi+c, inside [0, n)
+void c_positions(int lo, int hi, int c_cap, int n, std::vector<int>* pos) {
+  pos->clear();
+  for (int d = c_cap; d >= 1; --d) if (lo - d >= 0) pos->push_back(lo - d);
+  for (int d = 1; d <= c_cap; ++d) if (hi + d < n) pos->push_back(hi + d);
+}
+
+void enumerate_paths(const Sub& s, int z_cap, int c_cap, int X, int Y, NetOut& o) {
   const int x0 = s.x0, y0 = s.y0, x1 = s.x1, y1 = s.y1;
   int np = 0;
   if (y0 == y1) {                       // straight H
@@ -186,6 +194,18 @@ void enumerate_paths(const Sub& s, int z_cap, NetOut& o) {
     z_offsets(std::abs(y1 - y0), z_cap, &off);
     for (int d : off) {                 // Z-VHV, y_m ascending
       const int ym = ylo + d;
+      add_seg(o, 1, x0, y0, ym); add_seg(o, 0, ym, x0, x1); add_seg(o, 1, x1, ym, y1);
+      add_tp(o, x0, ym); add_tp(o, x1, ym);
+      o.path_nseg.push_back(3); o.path_ntp.push_back(2); ++np;
+    }
+    c_positions(x0, x1, c_cap, X, &off);
+    for (int xm : off) {                // C-HVH, x_m ascending (outside [x0, x1])
+      add_seg(o, 0, y0, x0, xm); add_seg(o, 1, xm, y0, y1); add_seg(o, 0, y1, xm, x1);
+      add_tp(o, xm, y0); add_tp(o, xm, y1);
+      o.path_nseg.push_back(3); o.path_ntp.push_back(2); ++np;
+    }
+    c_positions(ylo, std::max(y0, y1), c_cap, Y, &off);
+    for (int ym : off) {                // C-VHV, y_m ascending (outside [ylo, yhi])
       add_seg(o, 1, x0, y0, ym); add_seg(o, 0, ym, x0, x1); add_seg(o, 1, x1, ym, y1);
       add_tp(o, x0, ym); add_tp(o, x1, ym);
       o.path_nseg.push_back(3); o.path_ntp.push_back(2); ++np;
@@ -249,7 +269,7 @@ void build_trees(const forestgen_config& c, NetOut& o) {
     o.tree_nsub.push_back((int)t.size());
     for (auto& s : t) {
       o.subs.push_back(s);
-      enumerate_paths(s, c.z_cap, o);
+      enumerate_paths(s, c.z_cap, c.c_cap, c.X, c.Y, o);
     }
   }
 }
@@ -282,6 +302,7 @@ extern "C" int forestgen_generate(const forestgen_config* cp, forestgen_forest**
   if (c.pins_mode == 0 && (c.pins_min < 2 || c.pins_max < c.pins_min)) { g_err = "bad pins range"; return -1; }
   if (c.box_mode == 0 && (c.box_min < 1 || c.box_max < c.box_min)) { g_err = "bad box range"; return -1; }
   if (c.n_tree_cand < 1 || c.n_tree_cand > 2) { g_err = "n_tree_cand must be 1 or 2"; return -1; }
+  if (c.c_cap < 0) { g_err = "c_cap < 0"; return -1; }
   const int X = c.X, Y = c.Y;
 
   // hotspots (global stream)

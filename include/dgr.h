@@ -197,7 +197,8 @@ int dgr_free(struct dgr_handle* h);
  * paper leaves it to "net-level parallelism").  Readings: tree
  * candidates Q17 (Prim MST from pin 0; iterated 1-Steiner on the Hanan grid for <= 8 pins, else
  * Prim from the last pin; a duplicate second candidate is dropped), sub-nets = tree edges in Prim
- * order with canonical endpoints, paths Q14 (straight, or HV, VH, z_cap-limited Z-HVH / Z-VHV),
+ * order with canonical endpoints, paths Q14 (straight, or HV, VH, z_cap-limited Z-HVH / Z-VHV, then
+ * c_cap C-HVH / C-VHV detours per side, Q14b),
  * initial logits Q8 (U[0,1), splitmix64 counter hash of (seed, 3 / 4, index)).  The result equals
  * forestgen's forest for the same pins, bit for bit.
  * ------------------------------------------------------------------------------------------- */
@@ -209,6 +210,7 @@ typedef struct {
   int32_t n_tree_cand;          /* 1 or 2 */
   int32_t z_cap;                /* -1: L only; 0: every Z; > 0: at most z_cap Z per direction */
   uint64_t seed;                /* of the initial logits */
+  int32_t c_cap;                /* C-shape detours per side of a non-aligned sub-net (0 = none; Q14b, row f4) */
 } dgr_pins_desc;
 
 struct dgr_built_forest;

@@ -100,7 +100,8 @@ def _load(fp32: bool = False):
                                   _dp, _dp, _dp, _dp]
         L.odgr_real_bytes.restype = c.c_int32
         L.odgr_build_forest.restype = vp
-        L.odgr_build_forest.argtypes = [c.c_int64, _i64, _i32, c.c_int32, c.c_int32, c.c_uint64]
+        L.odgr_build_forest.argtypes = [c.c_int32, c.c_int32, c.c_int64, _i64, _i32, c.c_int32, c.c_int32, c.c_int32,
+                                        c.c_uint64]
         L.odgr_forest_sizes.argtypes = [vp, _i64]
         L.odgr_forest_copy.argtypes = [vp] + [_i64] * 5 + [_i32] * 3 + [_f32] * 2
         L.odgr_forest_free.argtypes = [vp]
@@ -251,13 +252,14 @@ class Oracle:
         return r
 
 
-def build_forest(net_pin_off, pin_xy, n_tree_cand: int = 2, z_cap: int = 15, seed: int = 1) -> dict:
+def build_forest(X: int, Y: int, net_pin_off, pin_xy, n_tree_cand: int = 2, z_cap: int = 15, seed: int = 1,
+                 c_cap: int = 0) -> dict:
     """Row f1 oracle (forest_oracle.c): the routing DAG forest of the given nets' pins (§4.2,
-    P:524-539; readings Q8, Q14, Q17).  Returns the CSR arrays of include/dgr.h's forest."""
+    P:524-539; readings Q8, Q14, Q14b, Q17).  Returns the CSR arrays of include/dgr.h's forest."""
     L = _load()
     npo = np.ascontiguousarray(net_pin_off, dtype=np.int64)
     pxy = np.ascontiguousarray(np.asarray(pin_xy, dtype=np.int32).reshape(-1))
-    h = L.odgr_build_forest(len(npo) - 1, npo, pxy, int(n_tree_cand), int(z_cap), int(seed))
+    h = L.odgr_build_forest(int(X), int(Y), len(npo) - 1, npo, pxy, int(n_tree_cand), int(z_cap), int(c_cap), int(seed))
     try:
         sz = np.zeros(5, np.int64)
         L.odgr_forest_sizes(h, sz)

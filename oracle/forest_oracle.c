@@ -13,7 +13,9 @@
  *     (x0 <= x1; y0 < y1 if x0 == x1);
  *   path candidates per sub-net (§3.1, reading Q14): the straight path if
  *     aligned, else HV, VH, Z-HVH (x_m ascending), Z-VHV (y_m ascending); at most z_cap Z per
- *     direction at offsets floor(j a/(z_cap+1) + 1/2) (z_cap 0 = all, -1 = none);
+ *     direction at offsets floor(j a/(z_cap+1) + 1/2) (z_cap 0 = all, -1 = none); then the
+ *     C-shape detours of reading Q14b (row f4): C-HVH at x_m = x0-c_cap .. x0-1, x1+1 .. x1+c_cap,
+ *     C-VHV at y_m = ylo-c_cap .. ylo-1, yhi+1 .. yhi+c_cap, those inside the grid;
  *   initial logits w0 ~ U[0,1) (reading Q8): a splitmix64-finalised counter hash of
  *     (seed, stream 3 trees / 4 paths, global index), 53 random bits.
  * No blocking, no parallelism, no incremental MST: every candidate evaluation re-runs Prim.
@@ -161,7 +163,7 @@ static void end_path(odgr_forest* f) {
 }
 
 /* the path candidates of one canonical sub-net (x0,y0)-(x1,y1) */
-static void enumerate(odgr_forest* f, const int s[4], int z_cap) {
+static void enumerate(odgr_forest* f, const int s[4], int z_cap, int c_cap, int X, int Y) {
   const int x0 = s[0], y0 = s[1], x1 = s[2], y1 = s[3];
   const int ylo = y0 < y1 ? y0 : y1, yhi = y0 < y1 ? y1 : y0;
   if (y0 == y1) { add_seg(f, 0, y0, x0, x1); end_path(f); }
@@ -182,6 +184,20 @@ static void enumerate(odgr_forest* f, const int s[4], int z_cap) {
       add_seg(f, 1, x0, y0, ym); add_seg(f, 0, ym, x0, x1); add_seg(f, 1, x1, ym, y1);
       add_tp(f, x0, ym); add_tp(f, x1, ym); end_path(f);
     }
+    for (int side = 0; side < 2; ++side)                                                       /* C-HVH */
+      for (int q = 0; q < c_cap; ++q) {
+        const int xm = side == 0 ? x0 - (c_cap - q) : x1 + 1 + q;
+        if (xm < 0 || xm >= X) continue;
+        add_seg(f, 0, y0, x0, xm); add_seg(f, 1, xm, y0, y1); add_seg(f, 0, y1, xm, x1);
+        add_tp(f, xm, y0); add_tp(f, xm, y1); end_path(f);
+      }
+    for (int side = 0; side < 2; ++side)                                                       /* C-VHV */
+      for (int q = 0; q < c_cap; ++q) {
+        const int ym = side == 0 ? ylo - (c_cap - q) : yhi + 1 + q;
+        if (ym < 0 || ym >= Y) continue;
+        add_seg(f, 1, x0, y0, ym); add_seg(f, 0, ym, x0, x1); add_seg(f, 1, x1, ym, y1);
+        add_tp(f, x0, ym); add_tp(f, x1, ym); end_path(f);
+      }
   }
   ov_i64(&f->sub_path_off, (int64_t)(f->path_seg_off.n - 1));
 }
@@ -198,8 +214,9 @@ static double u01(uint64_t seed, uint64_t stream, uint64_t idx) {
   return (double)(mix64(s) >> 11) * (1.0 / 9007199254740992.0);
 }
 
-ODGR_API odgr_forest* odgr_build_forest(int64_t n_nets, const int64_t* net_pin_off, const int32_t* pin_xy,
-                                        int32_t n_tree_cand, int32_t z_cap, uint64_t seed) {
+ODGR_API odgr_forest* odgr_build_forest(int32_t X, int32_t Y, int64_t n_nets, const int64_t* net_pin_off,
+                                        const int32_t* pin_xy, int32_t n_tree_cand, int32_t z_cap, int32_t c_cap,
+                                        uint64_t seed) {
   odgr_forest* f = (odgr_forest*)calloc(1, sizeof(odgr_forest));
   ov_init(&f->net_tree_off, 8); ov_init(&f->tree_sub_off, 8); ov_init(&f->sub_path_off, 8);
   ov_init(&f->path_seg_off, 8); ov_init(&f->path_tp_off, 8);
@@ -243,7 +260,7 @@ ODGR_API odgr_forest* odgr_build_forest(int64_t n_nets, const int64_t* net_pin_o
       int ne = t == 0 ? ne0 : nt1;
       for (int q = 0; q < ne; ++q) {
         for (int c = 0; c < 4; ++c) ov_i32(&f->sub_xy, tr[q][c]);
-        enumerate(f, tr[q], z_cap);
+        enumerate(f, tr[q], z_cap, c_cap, X, Y);
       }
       ov_i64(&f->tree_sub_off, (int64_t)(f->sub_xy.n / 4));
     }

@@ -153,7 +153,17 @@ __device__ __forceinline__ int z_offset(int a, int z_cap, int j) {   // j = 0 ..
   return (2 * (j + 1) * a + den) / (2 * den);
 }
 
+// C-shape detours (reading Q14b): positions lo-c .. lo-1 then hi+1 .. hi+c, inside [0, n)
+__device__ __forceinline__ int c_count(int lo, int hi, int c_cap, int n) {
+  return min(c_cap, lo) + min(c_cap, n - 1 - hi);
+}
+__device__ __forceinline__ int c_position(int lo, int hi, int c_cap, int j) {   // j = 0 .. c_count-1
+  const int left = min(c_cap, lo);
+  return j < left ? lo - left + j : hi + 1 + (j - left);
+}
+
 struct BuildArgs {
+  int32_t X, Y, c_cap;
   int64_t n_nets;
   const int64_t* net_pin_off;
   const int2* pin_xy;
@@ -214,7 +224,8 @@ __global__ void __launch_bounds__(128) kb_trees(BuildArgs B) {
   for (int q = 0; q < nsub; ++q) {
     const short4 s = out[q];
     if (s.x == s.z || s.y == s.w) { np += 1; ns += 1; continue; }
-    const int nz = z_count(s.z - s.x, B.z_cap) + z_count(abs(s.w - s.y), B.z_cap);
+    const int nz = z_count(s.z - s.x, B.z_cap) + z_count(abs(s.w - s.y), B.z_cap) +
+                   c_count(s.x, s.z, B.c_cap, B.X) + c_count(min(s.y, s.w), max(s.y, s.w), B.c_cap, B.Y);
     np += 2 + nz; ns += 4 + 3 * nz; nt += 2 + 2 * nz;
   }
   B.cnt[n] = ntree;
@@ -306,6 +317,16 @@ __global__ void __launch_bounds__(128) kb_fill(BuildArgs B, const int64_t* off) 
       const int ym = ylo + z_offset(ay, B.z_cap, j);
       seg(1, x0, y0, ym); seg(0, ym, x0, x1); seg(1, x1, ym, y1); turn(x0, ym); turn(x1, ym); done();
     }
+    const int ncx = c_count(x0, x1, B.c_cap, B.X);
+    for (int j = 0; j < ncx; ++j) {                                  // C-HVH, x_m ascending
+      const int xm = c_position(x0, x1, B.c_cap, j);
+      seg(0, y0, x0, xm); seg(1, xm, y0, y1); seg(0, y1, xm, x1); turn(xm, y0); turn(xm, y1); done();
+    }
+    const int yhi = max(y0, y1), ncy = c_count(ylo, yhi, B.c_cap, B.Y);
+    for (int j = 0; j < ncy; ++j) {                                  // C-VHV, y_m ascending
+      const int ym = c_position(ylo, yhi, B.c_cap, j);
+      seg(1, x0, y0, ym); seg(0, ym, x0, x1); seg(1, x1, ym, y1); turn(x0, ym); turn(x1, ym); done();
+    }
   }
 }
 
@@ -355,6 +376,7 @@ int dgr_build_forest(const dgr_pins_desc* d, void* cuda_stream, dgr_built_forest
   if (d->X < 2 || d->Y < 2 || d->X > 32767 || d->Y > 32767) return ffail(DGR_EINVAL, "grid must be 2..32767 per side");
   if (d->n_nets < 0 || !d->net_pin_off || (d->n_nets > 0 && !d->pin_xy)) return ffail(DGR_EINVAL, "bad pins arrays");
   if (d->n_tree_cand < 1 || d->n_tree_cand > 2) return ffail(DGR_EINVAL, "n_tree_cand must be 1 or 2");
+  if (d->c_cap < 0) return ffail(DGR_EINVAL, "c_cap must be >= 0");
   const int64_t N = d->n_nets;
   if (d->net_pin_off[0] != 0) return ffail(DGR_EINVAL, "net_pin_off[0] != 0");
   int64_t bad = -1;
@@ -411,6 +433,7 @@ int dgr_build_forest(const dgr_pins_desc* d, void* cuda_stream, dgr_built_forest
   FCUDA(cudaMemcpyAsync(pins_d, d->pin_xy, 8 * P, cudaMemcpyHostToDevice, s));
   B.n_nets = N; B.net_pin_off = pin_off_d; B.pin_xy = pins_d;
   B.n_tree_cand = d->n_tree_cand; B.z_cap = d->z_cap; B.seed = d->seed;
+  B.X = d->X; B.Y = d->Y; B.c_cap = d->c_cap;
   B.subs = subs_d; B.cnt = cnt_d; B.nsub0 = nsub0_d;
   kb_trees<<<(unsigned)((N + 127) / 128), 128, 0, s>>>(B);
   for (int a = 0; a < 5; ++a) {

@@ -42,7 +42,7 @@ class _Desc(ctypes.Structure):
 class _PinsDesc(ctypes.Structure):
     _fields_ = [("X", ctypes.c_int32), ("Y", ctypes.c_int32), ("n_nets", ctypes.c_int64),
                 ("net_pin_off", ctypes.c_void_p), ("pin_xy", ctypes.c_void_p), ("n_tree_cand", ctypes.c_int32),
-                ("z_cap", ctypes.c_int32), ("seed", ctypes.c_uint64)]
+                ("z_cap", ctypes.c_int32), ("seed", ctypes.c_uint64), ("c_cap", ctypes.c_int32)]
 
 
 class _Dist(ctypes.Structure):
@@ -326,7 +326,7 @@ class BuiltForest:
     The device arrays are owned by libdgr; download() copies them into host numpy arrays."""
 
     def __init__(self, X: int, Y: int, net_pin_off, pin_xy, n_tree_cand: int = 2, z_cap: int = 15, seed: int = 1,
-                 stream=None):
+                 stream=None, c_cap: int = 0):
         import torch
         if not torch.cuda.is_available():
             raise DgrError("libdgr needs a CUDA device (no CPU fallback)")
@@ -336,7 +336,7 @@ class BuiltForest:
         pxy = np.ascontiguousarray(np.asarray(pin_xy, np.int32).reshape(-1))
         st = stream if stream is not None else torch.cuda.current_stream()
         d = _PinsDesc(self.X, self.Y, len(npo) - 1, npo.ctypes.data, pxy.ctypes.data, int(n_tree_cand), int(z_cap),
-                      int(seed))
+                      int(seed), int(c_cap))
         self._h = ctypes.c_void_p()
         _check(L.dgr_build_forest(ctypes.byref(d), ctypes.c_void_p(st.cuda_stream), ctypes.byref(self._h)))
         sz = np.zeros(6, np.int64)
@@ -367,6 +367,6 @@ class BuiltForest:
             pass
 
 
-def build_forest(X, Y, net_pin_off, pin_xy, n_tree_cand=2, z_cap=15, seed=1, stream=None) -> BuiltForest:
+def build_forest(X, Y, net_pin_off, pin_xy, n_tree_cand=2, z_cap=15, seed=1, stream=None, c_cap=0) -> BuiltForest:
     """dgr_build_forest (row f1): the routing DAG forest of the nets' pins, built on the GPU."""
-    return BuiltForest(X, Y, net_pin_off, pin_xy, n_tree_cand, z_cap, seed, stream)
+    return BuiltForest(X, Y, net_pin_off, pin_xy, n_tree_cand, z_cap, seed, stream, c_cap)

@@ -23,3 +23,10 @@ def tiny():
 def c1e4():
     import forestgen
     return forestgen.generate("c1e4")
+
+
+@pytest.fixture(scope="session", params=["tiny", "tiny_c"])
+def tinyx(request):
+    """tiny, and tiny with C-shape detours (row f4, reading Q14b)"""
+    import forestgen
+    return forestgen.generate(request.param)

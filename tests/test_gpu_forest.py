@@ -11,8 +11,8 @@ import paper_conf_dac_0159layhrr24_b200 as dgr
 from paper_conf_dac_0159layhrr24_b200 import dgr as binding
 
 
-def _oracle(net_pin_off, pin_xy, n_tree_cand, z_cap, seed):
-    return oracle.build_forest(net_pin_off, pin_xy, n_tree_cand, z_cap, seed)
+def _oracle(X, Y, net_pin_off, pin_xy, n_tree_cand, z_cap, seed, c_cap=0):
+    return oracle.build_forest(X, Y, net_pin_off, pin_xy, n_tree_cand, z_cap, seed, c_cap)
 
 
 def _assert_same(gpu: dict, ref: dict):
@@ -22,12 +22,15 @@ def _assert_same(gpu: dict, ref: dict):
 
 @pytest.mark.gpu
 @pytest.mark.parametrize("name,kw", [("tiny", {}), ("c1e4", {}), ("ispd18", {}), ("c1e4", {"n_tree_cand": 1}),
-                                     ("c1e4", {"z_cap": -1}), ("c1e4", {"z_cap": 0})])
+                                     ("c1e4", {"z_cap": -1}), ("c1e4", {"z_cap": 0}), ("tiny_c", {}),
+                                     ("c1e4_c", {})])
 def test_gpu_forest_equals_oracle(name, kw):
     f = forestgen.generate(name, **kw)
     c = f.meta["config"]
-    b = dgr.build_forest(f.X, f.Y, f.net_pin_off, f.pin_xy, c["n_tree_cand"], c["z_cap"], c["seed"])
-    _assert_same(b.download(), _oracle(f.net_pin_off, f.pin_xy, c["n_tree_cand"], c["z_cap"], c["seed"]))
+    b = dgr.build_forest(f.X, f.Y, f.net_pin_off, f.pin_xy, c["n_tree_cand"], c["z_cap"], c["seed"],
+                         c_cap=c.get("c_cap", 0))
+    _assert_same(b.download(), _oracle(f.X, f.Y, f.net_pin_off, f.pin_xy, c["n_tree_cand"], c["z_cap"], c["seed"],
+                                       c.get("c_cap", 0)))
 
 
 @pytest.mark.gpu
@@ -36,7 +39,7 @@ def test_gpu_forest_full_size_ispd19():
     f = forestgen.generate("ispd19")
     c = f.meta["config"]
     b = dgr.build_forest(f.X, f.Y, f.net_pin_off, f.pin_xy, c["n_tree_cand"], c["z_cap"], c["seed"])
-    _assert_same(b.download(), _oracle(f.net_pin_off, f.pin_xy, c["n_tree_cand"], c["z_cap"], c["seed"]))
+    _assert_same(b.download(), _oracle(f.X, f.Y, f.net_pin_off, f.pin_xy, c["n_tree_cand"], c["z_cap"], c["seed"]))
 
 
 def _synthetic_pins(rng, n_nets, kmin, kmax, X, Y, box):
@@ -61,9 +64,9 @@ def test_gpu_forest_edge_cases(kmin, kmax, box):
     crowded boxes (many aligned / colinear pins), mixed sizes."""
     rng = np.random.default_rng(kmin * 100 + kmax)
     off, pts = _synthetic_pins(rng, 700, kmin, kmax, 64, 64, box)
-    for ntc, zc in ((2, 15), (2, 0), (1, -1)):
-        b = dgr.build_forest(64, 64, off, pts, ntc, zc, 7)
-        _assert_same(b.download(), _oracle(off, pts, ntc, zc, 7))
+    for ntc, zc, cc in ((2, 15, 0), (2, 0, 0), (1, -1, 0), (2, 11, 2), (2, 3, 5)):
+        b = dgr.build_forest(64, 64, off, pts, ntc, zc, 7, c_cap=cc)
+        _assert_same(b.download(), _oracle(64, 64, off, pts, ntc, zc, 7, cc))
 
 
 @pytest.mark.gpu

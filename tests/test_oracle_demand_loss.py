@@ -28,38 +28,38 @@ def _one_hot_logits(f, rng):
 
 
 @pytest.mark.parametrize("beta", [0.0, 0.25])
-def test_one_hot_demand_equals_integer_rasterisation(tiny, beta):
+def test_one_hot_demand_equals_integer_rasterisation(tinyx, beta):
     rng = np.random.default_rng(5)
-    o = oracle.Oracle(tiny)
-    wt, wp, tree_pick, path_pick = _one_hot_logits(tiny, rng)
+    o = oracle.Oracle(tinyx)
+    wt, wp, tree_pick, path_pick = _one_hot_logits(tinyx, rng)
     o.set_logits(wt, wp)
     o.forward(1.0, oracle.weights(beta=beta))
     q, p = o.probs()
     assert set(np.unique(q)) <= {0.0, 1.0} and set(np.unique(p)) <= {0.0, 1.0}
     sel = []
     for j in tree_pick:
-        for s in range(tiny.tree_sub_off[j], tiny.tree_sub_off[j + 1]):
+        for s in range(tinyx.tree_sub_off[j], tinyx.tree_sub_off[j + 1]):
             sel.append(path_pick[s])
-    dh_ref, dv_ref = _ref.rasterise(tiny, sel, beta=beta)
+    dh_ref, dv_ref = _ref.rasterise(tinyx, sel, beta=beta)
     dh, dv = o.demand()
     assert np.array_equal(dh, dh_ref) and np.array_equal(dv, dv_ref)
 
 
-def test_conservation(tiny):
+def test_conservation(tinyx):
     beta = 0.25
-    o = oracle.Oracle(tiny)
+    o = oracle.Oracle(tinyx)
     out = o.forward(0.8, oracle.weights(beta=beta))
     q, p = o.probs()
-    path_tree = np.repeat(np.repeat(np.arange(tiny.n_trees), np.diff(tiny.tree_sub_off)), np.diff(tiny.sub_path_off))
+    path_tree = np.repeat(np.repeat(np.arange(tinyx.n_trees), np.diff(tinyx.tree_sub_off)), np.diff(tinyx.sub_path_off))
     pi = q[path_tree] * p
     dh, dv = o.demand()
     ewl = out[1]
     via_total = 0.0
-    for i in range(tiny.n_paths):
-        for (x, y) in _ref.path_tps(tiny, i):
-            via_total += pi[i] * len(_ref.incident_edges(tiny.X, tiny.Y, x, y))
+    for i in range(tinyx.n_paths):
+        for (x, y) in _ref.path_tps(tinyx, i):
+            via_total += pi[i] * len(_ref.incident_edges(tinyx.X, tinyx.Y, x, y))
     assert abs(dh.sum() + dv.sum() - (ewl + beta * via_total)) < 1e-9
-    o0 = oracle.Oracle(tiny)
+    o0 = oracle.Oracle(tinyx)
     out0 = o0.forward(0.8, oracle.weights(beta=0.0))
     dh0, dv0 = o0.demand()
     assert abs(dh0.sum() + dv0.sum() - out0[1]) < 1e-9          # beta = 0: sum_e W_e = E[WL]
@@ -85,12 +85,12 @@ def _small_subforest(f, max_space=20000):
 
 
 @pytest.mark.parametrize("which", [0, 1, 2])
-def test_brute_force_expectation(tiny, which):
+def test_brute_force_expectation(tinyx, which):
     """E[D_e], E[WL], E[TP] of Eq. (10)-(12) equal the enumeration of every discrete selection."""
-    los = _small_subforest(tiny)
+    los = _small_subforest(tinyx)
     assert len(los) > which
     lo = los[which * (len(los) // 3)]
-    f = forestgen.subset(tiny, lo, lo + 3)
+    f = forestgen.subset(tinyx, lo, lo + 3)
     beta = 0.25
     o = oracle.Oracle(f)
     o.iteration = 4
@@ -116,17 +116,17 @@ def test_brute_force_expectation(tiny, which):
 
 
 @pytest.mark.parametrize("f_kind,slope", [(0, 1.0), (1, 1.0), (2, 0.01), (3, 0.5), (4, 1.0)])
-def test_cost_matches_torch_restatement(tiny, f_kind, slope):
+def test_cost_matches_torch_restatement(tinyx, f_kind, slope):
     """sigmoid, ReLU and the LeakyReLU / exp / CELU alternatives of Fig. 6."""
     W = oracle.weights(f_kind=f_kind, f_slope=slope)
-    o = oracle.Oracle(tiny)
+    o = oracle.Oracle(tinyx)
     o.iteration = 2
     t = 0.9
     out = o.forward(t, W)
-    g = torch.tensor(_ref.path_noise(tiny, 2), dtype=torch.float64)
-    gt = torch.tensor([oracle.gumbel(tiny.seed, j, 2, 1) for j in range(tiny.n_trees)], dtype=torch.float64)
-    cost, d, ewl, etp, of, _, _ = _ref.torch_cost(tiny, torch.tensor(tiny.w_tree0, dtype=torch.float64),
-                                                  torch.tensor(tiny.w_path0, dtype=torch.float64), gt, g, t, W)
+    g = torch.tensor(_ref.path_noise(tinyx, 2), dtype=torch.float64)
+    gt = torch.tensor([oracle.gumbel(tinyx.seed, j, 2, 1) for j in range(tinyx.n_trees)], dtype=torch.float64)
+    cost, d, ewl, etp, of, _, _ = _ref.torch_cost(tinyx, torch.tensor(tinyx.w_tree0, dtype=torch.float64),
+                                                  torch.tensor(tinyx.w_path0, dtype=torch.float64), gt, g, t, W)
     assert abs(out[0] - cost.item()) <= 1e-11 * abs(cost.item())
     assert abs(out[1] - ewl.item()) < 1e-10
     assert abs(out[3] - of.item()) < 1e-9

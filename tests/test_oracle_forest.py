@@ -10,7 +10,8 @@ import oracle
 
 def _built(f):
     c = f.meta["config"]
-    return oracle.build_forest(f.net_pin_off, f.pin_xy, c["n_tree_cand"], c["z_cap"], c["seed"])
+    return oracle.build_forest(f.X, f.Y, f.net_pin_off, f.pin_xy, c["n_tree_cand"], c["z_cap"], c["seed"],
+                               c.get("c_cap", 0))
 
 
 def _tree_subs(o, n):
@@ -129,3 +130,39 @@ def test_single_tree_candidate_and_l_only():
     assert np.diff(o["sub_path_off"]).max() <= 2
     for k, v in o.items():
         np.testing.assert_array_equal(np.asarray(getattr(f, k)).reshape(v.shape), v, err_msg=k)
+
+
+def test_c_shape_detours():
+    """Reading Q14b (row f4): C-HVH / C-VHV candidates after the Z's, x_m (y_m) outside the sub-net's
+    span by 1..c_cap on each side inside the grid; length = |dx| + |dy| + 2 x detour, 2 turning points."""
+    f = forestgen.generate("tiny_c")
+    o = _built(f)
+    c = f.meta["config"]["c_cap"]
+    nc = 0
+    for s in range(len(o["sub_path_off"]) - 1):
+        x0, y0, x1, y1 = o["sub_xy"][s]
+        a, b = o["sub_path_off"][s], o["sub_path_off"][s + 1]
+        if x0 == x1 or y0 == y1:
+            assert b - a == 1
+            continue
+        ylo, yhi = min(y0, y1), max(y0, y1)
+        ncx = min(c, x0) + min(c, f.X - 1 - x1)
+        ncy = min(c, ylo) + min(c, f.Y - 1 - yhi)
+        nz = (x1 - x0 - 1) + (yhi - ylo - 1)          # tiny_c: every Z
+        assert b - a == 2 + nz + ncx + ncy
+        for r, i in enumerate(range(b - ncx - ncy, b)):
+            segs = o["seg"][o["path_seg_off"][i]:o["path_seg_off"][i + 1]]
+            tp = o["tp_xy"][o["path_tp_off"][i]:o["path_tp_off"][i + 1]]
+            assert len(segs) == 3 and len(tp) == 2
+            if r < ncx:    # C-HVH: turning points on column x_m outside [x0, x1]
+                m = tp[0, 0]
+                assert tp[1, 0] == m and (m < x0 or m > x1)
+                det = x0 - m if m < x0 else m - x1
+            else:          # C-VHV: turning points on row y_m outside [ylo, yhi]
+                m = tp[0, 1]
+                assert tp[1, 1] == m and (m < ylo or m > yhi)
+                det = ylo - m if m < ylo else m - yhi
+            assert 1 <= det <= c
+            assert (segs[:, 3] - segs[:, 2]).sum() == (x1 - x0) + (yhi - ylo) + 2 * det
+            nc += 1
+    assert nc > 100

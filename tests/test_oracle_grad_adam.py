@@ -74,27 +74,27 @@ def test_gradient_central_differences_relu_away_from_kinks(tiny):
 
 
 @pytest.mark.parametrize("f_kind,slope", [(0, 1.0), (1, 1.0), (2, 0.01), (3, 0.5), (4, 1.0)])
-def test_gradient_matches_torch_autograd(tiny, f_kind, slope):
+def test_gradient_matches_torch_autograd(tinyx, f_kind, slope):
     W = oracle.weights(f_kind=f_kind, f_slope=slope)
     t, k = 0.7, 5
-    o, (dw, du) = _grad(tiny, k, t, W)
-    g = torch.tensor(_ref.path_noise(tiny, k), dtype=torch.float64)
-    gt = torch.tensor([oracle.gumbel(tiny.seed, j, k, 1) for j in range(tiny.n_trees)], dtype=torch.float64)
-    wp = torch.tensor(tiny.w_path0, dtype=torch.float64, requires_grad=True)
-    wt = torch.tensor(tiny.w_tree0, dtype=torch.float64, requires_grad=True)
-    cost, *_ = _ref.torch_cost(tiny, wt, wp, gt, g, t, W)
+    o, (dw, du) = _grad(tinyx, k, t, W)
+    g = torch.tensor(_ref.path_noise(tinyx, k), dtype=torch.float64)
+    gt = torch.tensor([oracle.gumbel(tinyx.seed, j, k, 1) for j in range(tinyx.n_trees)], dtype=torch.float64)
+    wp = torch.tensor(tinyx.w_path0, dtype=torch.float64, requires_grad=True)
+    wt = torch.tensor(tinyx.w_tree0, dtype=torch.float64, requires_grad=True)
+    cost, *_ = _ref.torch_cost(tinyx, wt, wp, gt, g, t, W)
     cost.backward()
     np.testing.assert_allclose(dw, wp.grad.numpy(), rtol=1e-9, atol=1e-9)
     np.testing.assert_allclose(du, wt.grad.numpy(), rtol=1e-9, atol=1e-9)
 
 
-def test_group_gradient_sums_to_zero(tiny):
-    o, (dw, du) = _grad(tiny, 0, 1.0, oracle.weights())
-    for s in range(tiny.n_subnets):
-        a, b = tiny.sub_path_off[s], tiny.sub_path_off[s + 1]
+def test_group_gradient_sums_to_zero(tinyx):
+    o, (dw, du) = _grad(tinyx, 0, 1.0, oracle.weights())
+    for s in range(tinyx.n_subnets):
+        a, b = tinyx.sub_path_off[s], tinyx.sub_path_off[s + 1]
         assert abs(dw[a:b].sum()) <= 1e-9 * max(1.0, np.abs(dw[a:b]).max())
-    for n in range(tiny.n_nets):
-        a, b = tiny.net_tree_off[n], tiny.net_tree_off[n + 1]
+    for n in range(tinyx.n_nets):
+        a, b = tinyx.net_tree_off[n], tinyx.net_tree_off[n + 1]
         assert abs(du[a:b].sum()) <= 1e-9 * max(1.0, np.abs(du[a:b]).max())
 
 
