@@ -124,11 +124,14 @@ int partition(const dgr_forest_desc* d, int world, std::vector<int64_t>& out) {
 struct Seg4 { int a, b, c, d; };
 inline bool seg_eq(const Seg4& x, const Seg4& y) { return x.a == y.a && x.b == y.b && x.c == y.c && x.d == y.d; }
 
-// Which pattern of sub-net (x0,y0)-(x1,y1) (canonical: x0 <= x1) path i is, and its x_m / y_m.
+// Which pattern of sub-net (x0,y0)-(x1,y1) (canonical: x0 <= x1) path i is, and its x_m / y_m;
+// *outside: a Z pattern whose x_m / y_m lies outside the sub-net's span (a C-shape detour, Q14b).
 // The path's segments and turning points may come in any order: each expected one must be
 // present and the counts must agree (the expected ones of a pattern are distinct, so a duplicate
 // in the path leaves one uncovered).  The turning points fix the pattern; the segments confirm it.
-bool classify(const dgr_forest_desc* d, int64_t i, int x0, int y0, int x1, int y1, uint32_t* shape, int* mid) {
+bool classify(const dgr_forest_desc* d, int64_t i, int x0, int y0, int x1, int y1, uint32_t* shape, int* mid,
+              bool* outside) {
+  *outside = false;
   const int64_t g0 = d->path_seg_off[i], g1 = d->path_seg_off[i + 1];
   const int64_t t0 = d->path_tp_off[i], t1 = d->path_tp_off[i + 1];
   const int ns = (int)(g1 - g0), nt = (int)(t1 - t0);
@@ -159,15 +162,18 @@ bool classify(const dgr_forest_desc* d, int64_t i, int x0, int y0, int x1, int y
   }
   if (ns != 3) return false;
   const int ax = tp[0], ay = tp[1], bx = tp[2], by = tp[3];
-  if (ax == bx && ((ay == y0 && by == y1) || (ay == y1 && by == y0))) {   // Z-HVH at x_m = ax
+  if (ax == bx && ((ay == y0 && by == y1) || (ay == y1 && by == y0))) {   // Z-HVH (or C-HVH) at x_m = ax
     const int xm = ax;
-    if (!(x0 < xm && xm < x1)) return false;
-    if (!has({0, y0, x0, xm}) || !has({1, xm, ylo, yhi}) || !has({0, y1, xm, x1})) return false;
-    *shape = kZHVH; *mid = xm; return true;
+    if (xm == x0 || xm == x1) return false;
+    if (!has({0, y0, std::min(x0, xm), std::max(x0, xm)}) || !has({1, xm, ylo, yhi}) ||
+        !has({0, y1, std::min(xm, x1), std::max(xm, x1)}))
+      return false;
+    *shape = kZHVH; *mid = xm; *outside = xm < x0 || xm > x1; return true;
   }
-  if (ay == by && ((ax == x0 && bx == x1) || (ax == x1 && bx == x0))) {   // Z-VHV at y_m = ay
+  if (ay == by && ((ax == x0 && bx == x1) || (ax == x1 && bx == x0))) {   // Z-VHV (or C-VHV) at y_m = ay
     const int ym = ay;
-    if (!(ylo < ym && ym < yhi)) return false;
+    if (ym == y0 || ym == y1) return false;
+    *outside = ym < ylo || ym > yhi;
     if (!has({1, x0, std::min(y0, ym), std::max(y0, ym)}) || !has({0, ym, x0, x1}) ||
         !has({1, x1, std::min(ym, y1), std::max(ym, y1)}))
       return false;
@@ -210,17 +216,41 @@ struct Plan {
   int64_t n_pipe_tiles = 0;
 };
 
-// Cells (x, y) touched by one candidate's demand events (see forward_bundle in dgr_kernels.cu)
-// and the fields they touch (bit 0 dH, 1 dV, 2 VD).
-int lane_events(uint32_t shape, int x0, int y0, int x1, int y1, int m, int ex[2], int ey[2], int fm[2]) {
-  switch (shape) {
-    case kStraightH: ex[0] = x0; ey[0] = y0; fm[0] = 1; ex[1] = x1; ey[1] = y0; fm[1] = 1; return 2;
-    case kStraightV: ex[0] = x0; ey[0] = y0; fm[0] = 2; ex[1] = x0; ey[1] = y1; fm[1] = 2; return 2;
-    case kHV: ex[0] = x0; ey[0] = y0; fm[0] = 3; ex[1] = x1; ey[1] = y0; fm[1] = 7; return 2;
-    case kVH: ex[0] = x0; ey[0] = y1; fm[0] = 7; ex[1] = x1; ey[1] = y1; fm[1] = 3; return 2;
-    case kZHVH: ex[0] = m; ey[0] = y0; fm[0] = 7; ex[1] = m; ey[1] = y1; fm[1] = 7; return 2;
-    default: ex[0] = x0; ey[0] = m; fm[0] = 7; ex[1] = x1; ey[1] = m; fm[1] = 7; return 2;
+// (cell, field) pairs of one candidate's demand events in the tile kernel (field 0 dH, 1 dV, 2 VD;
+// see process_tile in dgr_kernels.cu): the collapsed corner events of straight / L / Z lanes, and
+// the eight own events of a C-shape lane.  Returns their number (<= 8).
+int lane_events(uint32_t pw, int x0, int y0, int x1, int y1, int ex[8], int ey[8], int ef[8]) {
+  const uint32_t shape = pw & 7u;
+  const int m = (int)(pw >> 16);
+  int n = 0;
+  auto ev = [&](int x, int y, int mask) {
+    for (int f = 0; f < 3; ++f) if (mask >> f & 1) { ex[n] = x; ey[n] = y; ef[n] = f; ++n; }
+  };
+  if (pw & kOutside) {
+    const int ylo = std::min(y0, y1), yhi = std::max(y0, y1);
+    if (shape == kZHVH) {   // C-HVH
+      ev(std::min(x0, m), y0, 1); ev(std::max(x0, m), y0, 1); ev(std::min(m, x1), y1, 1); ev(std::max(m, x1), y1, 1);
+      ev(m, ylo, 2); ev(m, yhi, 2);
+      ex[n] = m; ey[n] = y0; ef[n++] = 2;
+      ex[n] = m; ey[n] = y1; ef[n++] = 2;
+      return n;
+    }
+    // C-VHV
+    ev(x0, std::min(y0, m), 2); ev(x0, std::max(y0, m), 2); ev(x1, std::min(m, y1), 2); ev(x1, std::max(m, y1), 2);
+    ev(x0, m, 1); ev(x1, m, 1);
+    ex[n] = x0; ey[n] = m; ef[n++] = 2;
+    ex[n] = x1; ey[n] = m; ef[n++] = 2;
+    return n;
   }
+  switch (shape) {
+    case kStraightH: ev(x0, y0, 1); ev(x1, y0, 1); break;
+    case kStraightV: ev(x0, y0, 2); ev(x0, y1, 2); break;
+    case kHV: ev(x0, y0, 3); ev(x1, y0, 7); break;
+    case kVH: ev(x0, y1, 7); ev(x1, y1, 3); break;
+    case kZHVH: ev(m, y0, 7); ev(m, y1, 7); break;
+    default: ev(x0, m, 7); ev(x1, m, 7); break;
+  }
+  return n;
 }
 
 // A sub-net whose only candidate is one segment draws no noise and needs no softmax (Q7).
@@ -230,7 +260,7 @@ inline bool lone_straight(const dgr_forest_desc* d, int64_t s) {
 }
 
 // Candidate order the forward's event collapse relies on (dgr.h): straight only if aligned, else
-// HV, VH, Z-HVH..., Z-VHV...
+// HV, VH, Z-HVH..., Z-VHV..., then C-shapes (shapes[] carry kOutside)
 inline bool canonical_group(const uint32_t* shapes, int n, bool aligned) {
   if (aligned) {
     for (int i = 0; i < n; ++i) if (shapes[i] != kStraightH && shapes[i] != kStraightV) return false;
@@ -240,6 +270,7 @@ inline bool canonical_group(const uint32_t* shapes, int n, bool aligned) {
   int i = 2;
   while (i < n && shapes[i] == kZHVH) ++i;
   while (i < n && shapes[i] == kZVHV) ++i;
+  while (i < n && (shapes[i] == (kZHVH | kOutside) || shapes[i] == (kZVHV | kOutside))) ++i;
   return i == n;
 }
 
@@ -284,10 +315,11 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   tm.mark("noise base");
   // 1. canonical sub-net endpoints + pattern words of every local candidate (parallel over
   //    sub-nets; the first failing sub-net, in index order, is reported)
-  PodBuf<short4> sxy_csr;
+  PodBuf<short4> sxy_csr, sub_ext;
   PodBuf<uint32_t> pw_path;
   PodBuf<char> single;
   sxy_csr.alloc(ns);
+  sub_ext.alloc(ns);
   pw_path.alloc((size_t)(pl.path_hi - pl.path_lo));
   single.alloc(ns);
   int64_t bad_sub = ns;   // smallest failing local sub-net
@@ -306,13 +338,18 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     const int64_t p0 = d->sub_path_off[s], p1 = d->sub_path_off[s + 1];
     uint32_t shapes[32];
     bool ok = true;
+    int ex0 = x0, ex1 = x1, ey0 = std::min(y0, y1), ey1 = std::max(y0, y1);   // extent incl. detours
     for (int64_t i = p0; i < p1 && ok; ++i) {
       uint32_t shape;
       int mid;
-      if (!classify(d, i, x0, y0, x1, y1, &shape, &mid)) { ok = false; break; }
-      shapes[i - p0] = shape;
-      pw_path[i - pl.path_lo] = shape | ((uint32_t)mid << 16);
+      bool outside;
+      if (!classify(d, i, x0, y0, x1, y1, &shape, &mid, &outside)) { ok = false; break; }
+      shapes[i - p0] = shape | (outside ? kOutside : 0u);
+      pw_path[i - pl.path_lo] = shape | (outside ? kOutside : 0u) | ((uint32_t)mid << 16);
+      if (outside && shape == kZHVH) { ex0 = std::min(ex0, mid); ex1 = std::max(ex1, mid); }
+      if (outside && shape == kZVHV) { ey0 = std::min(ey0, mid); ey1 = std::max(ey1, mid); }
     }
+    sub_ext[ls] = make_short4((short)ex0, (short)ey0, (short)ex1, (short)ey1);
     if (!ok || !canonical_group(shapes, (int)(p1 - p0), x0 == x1 || y0 == y1)) {
       bad_sub = std::min(bad_sub, ls);
       continue;
@@ -330,11 +367,12 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     for (int64_t i = d->sub_path_off[s]; i < d->sub_path_off[s + 1]; ++i) {
       uint32_t shape;
       int mid;
-      if (!classify(d, i, x0, y0, x1, y1, &shape, &mid))
+      bool outside;
+      if (!classify(d, i, x0, y0, x1, y1, &shape, &mid, &outside))
         return fail(DGR_EINVAL, "path %lld is not a straight/L/Z pattern of sub-net %lld (or its turning points are wrong)",
                     (long long)i, (long long)s);
     }
-    return fail(DGR_EINVAL, "sub-net %lld: candidates must be straight (aligned sub-net) or HV, VH, Z-HVH..., Z-VHV... in this order",
+    return fail(DGR_EINVAL, "sub-net %lld: candidates must be straight (aligned sub-net) or HV, VH, Z-HVH..., Z-VHV..., C... in this order",
                 (long long)s);
   }
   tm.mark("classify");
@@ -380,10 +418,10 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     const int64_t n = pl.net_lo + ln;
     int bx0 = X, by0 = Y, bx1 = -1, by1 = -1;
     const int64_t s0 = d->tree_sub_off[d->net_tree_off[n]], s1 = d->tree_sub_off[d->net_tree_off[n + 1]];
-    for (int64_t s = s0; s < s1; ++s) {
-      const short4 e = sxy_csr[s - pl.sub_lo];
+    for (int64_t s = s0; s < s1; ++s) {   // sub-net extents incl. C-shape detours
+      const short4 e = sub_ext[s - pl.sub_lo];
       bx0 = std::min<int>(bx0, e.x); bx1 = std::max<int>(bx1, e.z);
-      by0 = std::min<int>(by0, std::min(e.y, e.w)); by1 = std::max<int>(by1, std::max(e.y, e.w));
+      by0 = std::min<int>(by0, e.y); by1 = std::max<int>(by1, e.w);
     }
     nbox[ln] = make_int4(std::max(0, bx0 - 1), std::max(0, by0 - 1), std::min(X - 1, bx1 + 1), std::min(Y - 1, by1 + 1));
   }
@@ -596,14 +634,14 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
           const short4 e = sxy_csr[sn - pl.sub_lo];
           for (int64_t i = d->sub_path_off[sn]; i < d->sub_path_off[sn + 1] && ok; ++i) {
             const uint32_t pw = pw_path[i - pl.path_lo];
-            int ex[2], ey[2], fm[2];
-            lane_events(pw & 7u, e.x, e.y, e.z, e.w, (int)(pw >> 16), ex, ey, fm);
-            for (int q = 0; q < 2 && ok; ++q)
-              for (int f = 0; f < 3; ++f)
-                if (fm[q] >> f & 1) {
-                  const size_t c = (size_t)f * T.ww * T.wh + (size_t)(ey[q] - T.wy0) * T.ww + (ex[q] - T.wx0);
-                  if (++cnt[c] > kEventMax) { ok = false; break; }
-                }
+            int ex[8], ey[8], ef[8];
+            const int ne = lane_events(pw, e.x, e.y, e.z, e.w, ex, ey, ef);
+            for (int q = 0; q < ne && ok; ++q) {
+              // the event windows of the H / VD fields are row-major, the V field's column-major;
+              // any fixed cell index works for counting
+              const size_t c = (size_t)ef[q] * T.ww * T.wh + (size_t)(ey[q] - T.wy0) * T.ww + (ex[q] - T.wx0);
+              if (++cnt[c] > kEventMax) ok = false;
+            }
           }
         }
         if (!ok) { T.global = 1; T.wx0 = T.wy0 = T.ww = T.wh = 0; }

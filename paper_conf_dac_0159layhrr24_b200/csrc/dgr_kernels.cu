@@ -145,15 +145,25 @@ struct Shape6 {
 // the G of the incident edges; a segment's sum is S[hi] - S[lo].  Branch-free: the pattern selects
 // up to three segments and two turning points (straight, HV, VH, Z-HVH(x_m), Z-VHV(y_m)); unused
 // slots read valid cells and are weighted by 0.
-__device__ __forceinline__ double path_cost(const double* S, const Win& W, int X, int Y, uint32_t shape, int x0,
-                                            int y0, int x1, int y1, int m, const StepArgs& A) {
+__device__ __forceinline__ int detour(uint32_t pw, int x0, int y0, int x1, int y1) {   // C-shape (Q14b)
+  if (!(pw & kOutside)) return 0;
+  const int m = (int)(pw >> 16);
+  if ((pw & 7u) == kZHVH) return m < x0 ? x0 - m : m - x1;
+  const int ylo = min(y0, y1), yhi = max(y0, y1);
+  return m < ylo ? ylo - m : m - yhi;
+}
+
+__device__ __forceinline__ double path_cost(const double* S, const Win& W, int X, int Y, uint32_t pw, int x0,
+                                            int y0, int x1, int y1, const StepArgs& A) {
+  const uint32_t shape = pw & 7u;
+  const int m = (int)(pw >> 16);
   const Shape6 k(shape);
   const int ylo = min(y0, y1), yhi = max(y0, y1);
-  // segment 1 (always)
+  // segment 1 (always); Z / C segments between x0 (y0) and m in either order
   const bool v1 = k.sv | k.vh | k.zv;
   const int l1 = v1 ? x0 : y0;
-  const int a1 = v1 ? (k.zv ? min(y0, m) : ylo) : x0;
-  const int b1 = v1 ? (k.zv ? max(y0, m) : yhi) : (k.zh ? m : x1);
+  const int a1 = v1 ? (k.zv ? min(y0, m) : ylo) : (k.zh ? min(x0, m) : x0);
+  const int b1 = v1 ? (k.zv ? max(y0, m) : yhi) : (k.zh ? max(x0, m) : x1);
   // segment 2 (L and Z)
   const bool v2 = k.hv | k.zh;
   const int l2 = k.hv ? x1 : (k.vh ? y1 : m);
@@ -161,8 +171,8 @@ __device__ __forceinline__ double path_cost(const double* S, const Win& W, int X
   const int b2 = v2 ? yhi : x1;
   // segment 3 (Z)
   const int l3 = k.zh ? y1 : x1;
-  const int a3 = k.zh ? m : min(m, y1);
-  const int b3 = k.zh ? x1 : max(m, y1);
+  const int a3 = k.zh ? min(m, x1) : min(m, y1);
+  const int b3 = k.zh ? max(m, x1) : max(m, y1);
   const bool s2 = !(k.sh | k.sv), s3 = k.zh | k.zv;
   // turning points (default cell (x0, y0) when unused)
   const int tx0 = k.hv ? x1 : (k.zh ? m : x0);
@@ -181,13 +191,32 @@ __device__ __forceinline__ double path_cost(const double* S, const Win& W, int X
   };
   const double t0 = tp(tx0, ty0), t1 = tp(tx1, ty1);
   const double tps = (ntp >= 1 ? t0 : 0.0) + (ntp >= 2 ? t1 : 0.0);
-  return seg + (double)A.beta * tps + (double)A.a_wl * (double)((x1 - x0) + (yhi - ylo)) +
+  return seg + (double)A.beta * tps + (double)A.a_wl * (double)((x1 - x0) + (yhi - ylo) + 2 * detour(pw, x0, y0, x1, y1)) +
          (double)A.a_via * (double)A.sqrt_l * ntp;
 }
 
 __device__ __forceinline__ void red_shared_add(uint32_t saddr, int v) {
   asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.s32 p, %1, 0;\n\t@p red.shared.add.s32 [%0], %1;\n\t}" ::"r"(saddr), "r"(v)
                : "memory");
+}
+
+// A C-shape lane's own demand events (its corners are not shared with the L / Z collapse):
+// emit(field, x, y, value) with field 0 = dH (rows), 1 = dV (columns), 2 = turning points.
+template <typename Emit>
+__device__ __forceinline__ void c_events(uint32_t pw, int x0, int y0, int x1, int y1, int v, Emit emit) {
+  const int m = (int)(pw >> 16);
+  const int ylo = min(y0, y1), yhi = max(y0, y1);
+  if ((pw & 7u) == kZHVH) {
+    emit(0, min(x0, m), y0, v); emit(0, max(x0, m), y0, -v);
+    emit(0, min(m, x1), y1, v); emit(0, max(m, x1), y1, -v);
+    emit(1, m, ylo, v); emit(1, m, yhi, -v);
+    emit(2, m, y0, v); emit(2, m, y1, v);
+  } else {
+    emit(1, x0, min(y0, m), v); emit(1, x0, max(y0, m), -v);
+    emit(1, x1, min(m, y1), v); emit(1, x1, max(m, y1), -v);
+    emit(0, x0, m, v); emit(0, x1, m, -v);
+    emit(2, x0, m, v); emit(2, x1, m, v);
+  }
 }
 
 // g = -ln(-ln u) from one Philox word
@@ -287,7 +316,7 @@ __device__ __forceinline__ void reverse_warp(const KParams& P, const StepArgs& A
       if (b + 2 < bw1) { bi1 = __ldg(&P.binfo[b + 2]); pw1 = __ldg(&P.pword[slot + 64]); }
     }
     const float q = L.valid ? q_s[L.tree - T.tree0] : 0.f;
-    const double c = L.valid ? path_cost(S, W, P.X, P.Y, L.shape, e.x, e.y, e.z, e.w, (int)(L.pw >> 16), A) : 0.0;
+    const double c = L.valid ? path_cost(S, W, P.X, P.Y, L.pw, e.x, e.y, e.z, e.w, A) : 0.0;
     // softmax backward dw_i = (p_i/t)(dp_i - sum_k p_k dp_k / sum_k p_k): differences to the group
     // head's dp are formed in fp64 and reduced in fp32, so neither the magnitude of c nor
     // sum_k p_k != 1 (rounding) leaks into dw.
@@ -364,19 +393,21 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
       const int o = __shfl_up_sync(kFull, sc, off);
       if (L.lane - off >= L.head) sc += o;
     }
-    const int nh = __popc(__ballot_sync(kFull, L.shape == kZHVH) & L.gmask);
-    const int h1 = min(L.head + 1, 31), h2 = min(L.head + 1 + nh, 31);
+    const bool outside = (L.pw & kOutside) != 0;   // C-shape lanes: own events, outside the collapse
+    const int nh = __popc(__ballot_sync(kFull, L.shape == kZHVH && !outside) & L.gmask);
+    const int nv = __popc(__ballot_sync(kFull, L.shape == kZVHV && !outside) & L.gmask);
+    const int h1 = min(L.head + 1, 31), h2 = min(L.head + 1 + nh, 31), h3 = min(L.head + 1 + nh + nv, 31);
     const int a = __shfl_sync(kFull, vq, L.head);
     const int bb = __shfl_sync(kFull, vq, h1);
     const int S1 = __shfl_sync(kFull, sc, h1);
     const int S2 = __shfl_sync(kFull, sc, h2);
-    const int Se = __shfl_sync(kFull, sc, L.end);
+    const int S3 = __shfl_sync(kFull, sc, h3);
     const int x0 = e.x, y0 = e.y, x1 = e.z, y1 = e.w;
     const int s = (y1 > y0) ? 1 : -1;
-    const int hs = S2 - S1, vs = Se - S2, v = vq;
+    const int hs = S2 - S1, vs = S3 - S2, v = vq;
     const int mm = (int)(L.pw >> 16);
     const int fSH = L.shape == kStraightH, fSV = L.shape == kStraightV, fHV = L.shape == kHV;
-    const int fVH = L.shape == kVH, fZH = L.shape == kZHVH, fZV = L.shape == kZVHV;
+    const int fVH = L.shape == kVH, fZH = L.shape == kZHVH && !outside, fZV = L.shape == kZVHV && !outside;
     const int fZ = fZH + fZV;
     const int xa = x0 + fZH * (mm - x0);
     const int ya = y0 + fVH * (y1 - y0) + fZV * (mm - y0);
@@ -396,9 +427,21 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
         red64(P.dH + (size_t)yb * X + xb, bh); red64(P.dVT + (size_t)xb * Y + yb, bv);
         red64(P.VD + (size_t)yb * X + xb, bd);
       }
-      const int ntp = fHV + fVH + 2 * fZ;
-      wl += (long long)vq * ((x1 - x0) + abs(y1 - y0));
+      const int ntp = fHV + fVH + 2 * fZ + 2 * outside;
+      wl += (long long)vq * ((x1 - x0) + abs(y1 - y0) + 2 * detour(L.pw, x0, y0, x1, y1));
       tpc += (long long)vq * ntp;
+      if (outside) {
+        if (GLOBAL) {
+          const int X = P.X, Y = P.Y;
+          c_events(L.pw, x0, y0, x1, y1, vq, [&](int fld, int x, int y, int val) {
+            red64(fld == 0 ? P.dH + (size_t)y * X + x : fld == 1 ? P.dVT + (size_t)x * Y + y : P.VD + (size_t)y * X + x, val);
+          });
+        } else {
+          c_events(L.pw, x0, y0, x1, y1, vq, [&](int fld, int x, int y, int val) {
+            red_shared_add(ev_base + 4u * (fld == 0 ? W.h(x, y) : fld == 1 ? W.v(x, y) : 2 * W.hv + W.h(x, y)), val);
+          });
+        }
+      }
     }
     if (!GLOBAL) {
       const int hv2 = 2 * W.hv;   // VD part of the event window
@@ -705,7 +748,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         double c = 0.0;
         if (L.valid && !(P.skip & 8)) {
           const short4 e = St.sxy[L.sub - s_lo];
-          c = path_cost(St.S, W, X, Y, L.shape, e.x, e.y, e.z, e.w, (int)(L.pw >> 16), A);
+          c = path_cost(St.S, W, X, Y, L.pw, e.x, e.y, e.z, e.w, A);
         }
         // softmax backward: differences to the group head's dp in fp64, reduced in fp32
         const double dp = (double)q * c;
@@ -849,20 +892,22 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
           const int o = __shfl_up_sync(kFull, sc, off);
           if (L.lane - off >= L.head) sc += o;
         }
-        const int nh = __popc(__ballot_sync(kFull, L.shape == kZHVH) & L.gmask);
-        const int h1 = min(L.head + 1, 31), h2 = min(L.head + 1 + nh, 31);
+        const bool outside = (L.pw & kOutside) != 0;   // C-shape lanes: own events, outside the collapse
+        const int nh = __popc(__ballot_sync(kFull, L.shape == kZHVH && !outside) & L.gmask);
+        const int nv = __popc(__ballot_sync(kFull, L.shape == kZVHV && !outside) & L.gmask);
+        const int h1 = min(L.head + 1, 31), h2 = min(L.head + 1 + nh, 31), h3 = min(L.head + 1 + nh + nv, 31);
         const int a = __shfl_sync(kFull, vq, L.head);
         const int bb = __shfl_sync(kFull, vq, h1);
         const int S1 = __shfl_sync(kFull, sc, h1);
         const int S2 = __shfl_sync(kFull, sc, h2);
-        const int Se = __shfl_sync(kFull, sc, L.end);
+        const int S3 = __shfl_sync(kFull, sc, h3);
         const short4 e = L.valid ? St.sxy[L.sub - s_lo] : make_short4(0, 0, 0, 0);
         const int x0 = e.x, y0 = e.y, x1 = e.z, y1 = e.w;
         const int sgn = (y1 > y0) ? 1 : -1;
-        const int hs = S2 - S1, vs = Se - S2, vv = vq;
+        const int hs = S2 - S1, vs = S3 - S2, vv = vq;
         const int mm = (int)(L.pw >> 16);
         const int fSH = L.shape == kStraightH, fSV = L.shape == kStraightV, fHV = L.shape == kHV;
-        const int fVH = L.shape == kVH, fZH = L.shape == kZHVH, fZV = L.shape == kZVHV;
+        const int fVH = L.shape == kVH, fZH = L.shape == kZHVH && !outside, fZV = L.shape == kZVHV && !outside;
         const int fZ = fZH + fZV;
         const int xa = x0 + fZH * (mm - x0);
         const int ya = y0 + fVH * (y1 - y0) + fZV * (mm - y0);
@@ -885,6 +930,13 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
           red_shared_add(ev_base + 4u * (hv2 + ib_h), bd);
           wl_acc += (long long)vq * ((x1 - x0) + abs(y1 - y0));
           tp_acc += (long long)vq * (fHV + fVH + 2 * fZ);
+          if (outside) {
+            c_events(L.pw, x0, y0, x1, y1, vq, [&](int fld, int x, int y, int val) {
+              red_shared_add(ev_base + 4u * (fld == 0 ? W.h(x, y) : fld == 1 ? W.v(x, y) : hv2 + W.h(x, y)), val);
+            });
+            wl_acc += (long long)vq * (2 * detour(L.pw, x0, y0, x1, y1));
+            tp_acc += 2 * (long long)vq;
+          }
         }
       } else {
         // singleton bundle: pi = q; +pi where the segment starts, -pi where it ends
@@ -1300,7 +1352,8 @@ __global__ void __launch_bounds__(256) ki_path_kernel(KParams P, float inv_t, fl
       case kZHVH: hseg(y0, x0, mid); vseg(mid, ylo, yhi); hseg(y1, mid, x1); tp(mid, y0); tp(mid, y1); ntp = 2; break;
       default: vseg(x0, y0, mid); hseg(mid, x0, x1); vseg(x1, mid, y1); tp(x0, mid); tp(x1, mid); ntp = 2; break;
     }
-    atomicAdd(reinterpret_cast<unsigned long long*>(P.iscal), (unsigned long long)((x1 - x0) + abs(y1 - y0)));
+    atomicAdd(reinterpret_cast<unsigned long long*>(P.iscal),
+              (unsigned long long)((x1 - x0) + abs(y1 - y0) + 2 * detour(L.pw, x0, y0, x1, y1)));
     atomicAdd(reinterpret_cast<unsigned long long*>(P.iscal + 1), (unsigned long long)ntp);
   }
 }

@@ -37,7 +37,7 @@ def ow(w: dgr.Weights):
 
 @pytest.fixture(scope="module")
 def forests():
-    return {n: forestgen.generate(n) for n in ("tiny", "c1e4", "ispd18")}
+    return {n: forestgen.generate(n) for n in ("tiny", "c1e4", "ispd18", "tiny_c", "c1e4_c")}
 
 
 def run_both(f, schedule, W=None, lr=0.3):
@@ -99,8 +99,9 @@ def compare_state(s, o, what, probe=None, max_ill=0.01):
 
 
 @pytest.mark.parametrize("beta", [0.0, 0.25])
-def test_one_hot_demand_is_bit_exact(forests, beta):
-    f = copy.deepcopy(forests["c1e4"])
+@pytest.mark.parametrize("name", ["c1e4", "c1e4_c"])
+def test_one_hot_demand_is_bit_exact(forests, beta, name):
+    f = copy.deepcopy(forests[name])
     rng = np.random.default_rng(0)
     wt = np.zeros(f.n_trees, np.float32); wp = np.zeros(f.n_paths, np.float32)
     pick = [int(rng.integers(f.sub_path_off[sn], f.sub_path_off[sn + 1])) for sn in range(f.n_subnets)]
@@ -122,7 +123,7 @@ def test_one_hot_demand_is_bit_exact(forests, beta):
     assert np.array_equal(gdh.astype(np.float64), odh) and np.array_equal(gdv.astype(np.float64), odv)
 
 
-@pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18"])
+@pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18", "tiny_c", "c1e4_c"])
 @pytest.mark.parametrize("f_kind", [0, 1, 2, 3, 4])
 def test_forward_parity(forests, name, f_kind):
     """sigmoid, ReLU and the LeakyReLU / exp / CELU of Fig. 6."""
@@ -137,7 +138,7 @@ def test_forward_parity(forests, name, f_kind):
     assert s.iteration == 0
 
 
-@pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18"])
+@pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18", "tiny_c", "c1e4_c"])
 def test_one_iteration_parity(forests, name):
     """After one Adam step the update of a coordinate whose gradient is ~eps depends on that
     gradient's last bits (Q21b), so the fp32 probe applies from the first step on."""
@@ -149,6 +150,8 @@ def test_one_iteration_parity(forests, name):
 @pytest.mark.parametrize("name,schedule", [
     ("tiny", [(100, 1.0), (100, 0.9)]),                  # BASELINE.json: tiny, 200 iterations
     ("c1e4", [(100, 1.0)]),
+    ("tiny_c", [(100, 1.0), (100, 0.9)]),                # row f4: C-shape detours
+    ("c1e4_c", [(100, 1.0)]),
 ])
 def test_trajectory_parity(forests, name, schedule):
     f = forests[name]
@@ -206,7 +209,7 @@ def test_split_calls_and_determinism(forests):
     assert all(np.array_equal(x, y) for x, y in zip(a.demand(), b.demand()))
 
 
-@pytest.mark.parametrize("name", ["tiny", "c1e4"])
+@pytest.mark.parametrize("name", ["tiny", "c1e4", "c1e4_c"])
 def test_induce_parity(forests, name):
     f = forests[name]
     s, o, _, _ = run_both(f, [(60, 1.0), (40, 0.9)])
