@@ -37,7 +37,10 @@ constexpr double kDqScale = 4294967296.0;          // dq_j accumulated in 2^-32 
 constexpr double kDqInv = 1.0 / 4294967296.0;
 
 constexpr int kTileThreads = 256;                  // 8 warps per tile CTA
-constexpr int kWinMax = 1536;                      // window cells per tile
+#ifndef DGR_WINMAX
+#define DGR_WINMAX 1536
+#endif
+constexpr int kWinMax = DGR_WINMAX;                // window cells per tile
 constexpr int kMaxBundles = 64;                    // bundles per tile (a whole net always fits)
 #ifndef DGR_TARGET_BUNDLES
 #define DGR_TARGET_BUNDLES 32

@@ -600,20 +600,27 @@ constexpr int kPSubMax = kPipeSubs + 2;                     // + alignment slack
 constexpr int kPTreeMax = kPipeTrees + 4;
 constexpr int kPNetMax = kPipeTrees + 8;
 
+// Slim stage (default): the Adam moments m, v and the stored p of the paths, and m, v of the trees,
+// stay in global memory (each warp reads / writes its bundle's 128-byte rows directly); the stage
+// keeps what several phases share.  The smaller stage fits 5 CTAs per SM instead of 4.
+#ifndef DGR_SLIM_STAGE
+#define DGR_SLIM_STAGE 1
+#endif
+constexpr bool kSlim = DGR_SLIM_STAGE != 0;
 struct StageLayout {
   static constexpr size_t pw = 0;
   static constexpr size_t w = pw + 4 * 32 * kTileBundles;
   static constexpr size_t m = w + 4 * kPSlots;
-  static constexpr size_t v = m + 4 * kPSlots;
-  static constexpr size_t p = v + 4 * kPSlots;
-  static constexpr size_t bi = p + 4 * kPSlots;
+  static constexpr size_t v = m + (kSlim ? 0 : 4 * kPSlots);
+  static constexpr size_t p = v + (kSlim ? 0 : 4 * kPSlots);
+  static constexpr size_t bi = p + (kSlim ? 0 : 4 * kPSlots);
   static constexpr size_t sxy = bi + 16 * kTileBundles;
   static constexpr size_t nto = sxy + 8 * kPSubMax;
   static constexpr size_t q = (nto + 4 * kPNetMax + 15) / 16 * 16;
   static constexpr size_t wt = q + 4 * kPTreeMax;
   static constexpr size_t mt = wt + 4 * kPTreeMax;
-  static constexpr size_t vt = mt + 4 * kPTreeMax;
-  static constexpr size_t S = (vt + 4 * kPTreeMax + 127) / 128 * 128;
+  static constexpr size_t vt = mt + (kSlim ? 0 : 4 * kPTreeMax);
+  static constexpr size_t S = (vt + (kSlim ? 0 : 4 * kPTreeMax) + 127) / 128 * 128;
   static constexpr size_t bytes = S + 2 * 8 * kWinMax;
 };
 
@@ -680,8 +687,9 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
   const uint32_t slot_bytes = (uint32_t)T.nb * 128u, gslot_bytes = (uint32_t)T.nbg * 128u;
   const uint32_t nrow = REV ? (uint32_t)T.wh : 0u, ncol = REV ? (uint32_t)T.ww : 0u;
-  const uint32_t bytes = slot_bytes + gslot_bytes * (REV ? 4u : 1u) + 16u * T.nb + 8u * (s_hi - s_lo) +
-                         4u * (n_hi - n_lo) + 4u * (t_hi - t_lo) * (REV ? 4u : 3u) + 8u * (nrow * T.ww + ncol * T.wh);
+  const uint32_t bytes = slot_bytes + gslot_bytes * (REV && !kSlim ? 4u : 1u) + 16u * T.nb + 8u * (s_hi - s_lo) +
+                         4u * (n_hi - n_lo) + 4u * (t_hi - t_lo) * (kSlim ? (REV ? 2u : 1u) : (REV ? 4u : 3u)) +
+                         8u * (nrow * T.ww + ncol * T.wh);
   if (lane == 0) mbar_expect_tx(bar, bytes);
   __syncwarp();
   const size_t s0 = (size_t)T.b0 * 32;
@@ -692,15 +700,15 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
       switch (it) {
         case 0: bulk_g2s(S.pw, P.pword + s0, slot_bytes, bar); break;
         case 1: if (gslot_bytes) bulk_g2s(S.w, P.wp + s0, gslot_bytes, bar); break;
-        case 2: if (REV && gslot_bytes) bulk_g2s(S.m, P.mp + s0, gslot_bytes, bar); break;
-        case 3: if (REV && gslot_bytes) bulk_g2s(S.v, P.vp + s0, gslot_bytes, bar); break;
-        case 4: if (REV && gslot_bytes) bulk_g2s(S.p, P.pp + s0, gslot_bytes, bar); break;
+        case 2: if (!kSlim && REV && gslot_bytes) bulk_g2s(S.m, P.mp + s0, gslot_bytes, bar); break;
+        case 3: if (!kSlim && REV && gslot_bytes) bulk_g2s(S.v, P.vp + s0, gslot_bytes, bar); break;
+        case 4: if (!kSlim && REV && gslot_bytes) bulk_g2s(S.p, P.pp + s0, gslot_bytes, bar); break;
         case 5: bulk_g2s(S.bi, P.binfo + T.b0, 16u * T.nb, bar); break;
         case 6: bulk_g2s(S.sxy, P.sxy + s_lo, 8u * (s_hi - s_lo), bar); break;
         case 7: bulk_g2s(S.nto, P.net_tree_off + n_lo, 4u * (n_hi - n_lo), bar); break;
         case 8: bulk_g2s(S.wt, P.wt + t_lo, 4u * (t_hi - t_lo), bar);
-                bulk_g2s(S.mt, P.mt + t_lo, 4u * (t_hi - t_lo), bar); break;
-        default: bulk_g2s(S.vt, P.vt + t_lo, 4u * (t_hi - t_lo), bar);
+                if (!kSlim) bulk_g2s(S.mt, P.mt + t_lo, 4u * (t_hi - t_lo), bar); break;
+        default: if (!kSlim) bulk_g2s(S.vt, P.vt + t_lo, 4u * (t_hi - t_lo), bar);
                  if (REV) bulk_g2s(S.q, P.q + t_lo, 4u * (t_hi - t_lo), bar); break;
       }
     } else if (it < 10 + (int)nrow) {
@@ -742,8 +750,10 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         Lane L;
         lane_from(bi, pw, P, L);
         const int sl = lb * 32 + lane;
-        float w = St.w[sl], m = St.m[sl], v = St.v[sl];
-        const float p = St.p[sl];
+        const size_t gsl = (size_t)T.b0 * 32 + sl;
+        float w = St.w[sl];
+        float m = kSlim ? P.mp[gsl] : St.m[sl], v = kSlim ? P.vp[gsl] : St.v[sl];
+        const float p = kSlim ? P.pp[gsl] : St.p[sl];
         const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
         double c = 0.0;
         if (L.valid && !(P.skip & 8)) {
@@ -769,7 +779,8 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
                     static_cast<unsigned long long>(__double2ll_rn(pc * kDqScale)));
         if (L.valid) {
           adam_update(w, m, v, dw, A);
-          St.w[sl] = w; St.m[sl] = m; St.v[sl] = v;
+          St.w[sl] = w;
+          if (kSlim) { P.mp[gsl] = m; P.vp[gsl] = v; } else { St.m[sl] = m; St.v[sl] = v; }
         }
       } else {
         // singleton bundle: c of a straight path (one segment, no turning point); p = 1
@@ -821,7 +832,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         sq /= sw;
         for (int j = a; j < b; ++j) {
           const double du = (double)St.q[j] * (double)A.inv_t * ((double)dq_s[j + t_lo - T.tree0] * kDqInv - sq);
-          float w = St.wt[j], m = St.mt[j], v = St.vt[j];
+          float w = St.wt[j], m = kSlim ? P.mt[j + t_lo] : St.mt[j], v = kSlim ? P.vt[j + t_lo] : St.vt[j];
           adam_update(w, m, v, (float)du, A);
           St.wt[j] = w;
           const int jg = j + t_lo;
@@ -883,7 +894,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         const float w = St.w[sl];
         const float g = L.valid ? gp[bi.x + lane - nid0] : 0.f;
         const float p = softmax_from_noise(L, w, g, A.inv_t);
-        St.p[sl] = p;
+        if (kSlim) P.pp[(size_t)T.b0 * 32 + sl] = p; else St.p[sl] = p;
         const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
         const int vq = L.valid ? __float2int_rn(q * p * kFixScale) : 0;
         int sc = vq;
@@ -972,10 +983,12 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     const uint32_t gslot_bytes = (uint32_t)nbg * 128u;
     if (REV) {
       bulk_s2g(P.wp + s0, St.w, gslot_bytes);
-      bulk_s2g(P.mp + s0, St.m, gslot_bytes);
-      bulk_s2g(P.vp + s0, St.v, gslot_bytes);
+      if (!kSlim) {
+        bulk_s2g(P.mp + s0, St.m, gslot_bytes);
+        bulk_s2g(P.vp + s0, St.v, gslot_bytes);
+      }
     }
-    if (FWD) bulk_s2g(P.pp + s0, St.p, gslot_bytes);
+    if (FWD && !kSlim) bulk_s2g(P.pp + s0, St.p, gslot_bytes);
     bulk_commit();
   }
   if (FWD && !(P.skip & 1)) {
@@ -1012,7 +1025,10 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
 #define DGR_BTHREADS 256
 #endif
 constexpr int kBThreads = DGR_BTHREADS;
-constexpr int kBPerSM = 1024 / kBThreads;
+#ifndef DGR_BPERSM
+#define DGR_BPERSM (DGR_SLIM_STAGE ? 5 : 4)
+#endif
+constexpr int kBPerSM = DGR_BPERSM;
 constexpr size_t kBSmemBytes = StageLayout::bytes + 8 * kPipeTrees + 64;
 static_assert(kGpOffset + 4 * 32 * kTargetBundles <= 2 * 8 * kWinMax, "event window + path noise must fit the S window");
 static_assert(8 * kPipeTrees + 12 * kPipeTrees + 32 + 4 * kPipeTrees <= kGpOffset, "tree scratch must not overlap the path noise");
