@@ -607,10 +607,15 @@ constexpr int kPNetMax = kPipeTrees + 8;
 #define DGR_SLIM_STAGE 1
 #endif
 constexpr bool kSlim = DGR_SLIM_STAGE != 0;
+// Lean stage: the pattern words and logits of the paths are read (and w written) directly too.
+#ifndef DGR_LEAN_STAGE
+#define DGR_LEAN_STAGE 0
+#endif
+constexpr bool kLean = kSlim && DGR_LEAN_STAGE != 0;
 struct StageLayout {
   static constexpr size_t pw = 0;
-  static constexpr size_t w = pw + 4 * 32 * kTileBundles;
-  static constexpr size_t m = w + 4 * kPSlots;
+  static constexpr size_t w = pw + (kLean ? 0 : 4 * 32 * kTileBundles);
+  static constexpr size_t m = w + (kLean ? 0 : 4 * kPSlots);
   static constexpr size_t v = m + (kSlim ? 0 : 4 * kPSlots);
   static constexpr size_t p = v + (kSlim ? 0 : 4 * kPSlots);
   static constexpr size_t bi = p + (kSlim ? 0 : 4 * kPSlots);
@@ -687,7 +692,7 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
   const uint32_t slot_bytes = (uint32_t)T.nb * 128u, gslot_bytes = (uint32_t)T.nbg * 128u;
   const uint32_t nrow = REV ? (uint32_t)T.wh : 0u, ncol = REV ? (uint32_t)T.ww : 0u;
-  const uint32_t bytes = slot_bytes + gslot_bytes * (REV && !kSlim ? 4u : 1u) + 16u * T.nb + 8u * (s_hi - s_lo) +
+  const uint32_t bytes = (kLean ? 0u : slot_bytes + gslot_bytes * (REV && !kSlim ? 4u : 1u)) + 16u * T.nb + 8u * (s_hi - s_lo) +
                          4u * (n_hi - n_lo) + 4u * (t_hi - t_lo) * (kSlim ? (REV ? 2u : 1u) : (REV ? 4u : 3u)) +
                          8u * (nrow * T.ww + ncol * T.wh);
   if (lane == 0) mbar_expect_tx(bar, bytes);
@@ -698,8 +703,8 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
   for (int it = lane; it < nitems; it += 32) {
     if (it < 10) {
       switch (it) {
-        case 0: bulk_g2s(S.pw, P.pword + s0, slot_bytes, bar); break;
-        case 1: if (gslot_bytes) bulk_g2s(S.w, P.wp + s0, gslot_bytes, bar); break;
+        case 0: if (!kLean) bulk_g2s(S.pw, P.pword + s0, slot_bytes, bar); break;
+        case 1: if (!kLean && gslot_bytes) bulk_g2s(S.w, P.wp + s0, gslot_bytes, bar); break;
         case 2: if (!kSlim && REV && gslot_bytes) bulk_g2s(S.m, P.mp + s0, gslot_bytes, bar); break;
         case 3: if (!kSlim && REV && gslot_bytes) bulk_g2s(S.v, P.vp + s0, gslot_bytes, bar); break;
         case 4: if (!kSlim && REV && gslot_bytes) bulk_g2s(S.p, P.pp + s0, gslot_bytes, bar); break;
@@ -745,13 +750,13 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   if (REV) {   // dq_s was zeroed before the stage arrived
     for (int lb = warp; lb < T.nb; lb += NW) {
       const int4 bi = St.bi[lb];
-      const uint32_t pw = St.pw[lb * 32 + lane];
+      const uint32_t pw = kLean ? P.pword[(size_t)(T.b0 + lb) * 32 + lane] : St.pw[lb * 32 + lane];
       if (lb < nbg) {
         Lane L;
         lane_from(bi, pw, P, L);
         const int sl = lb * 32 + lane;
         const size_t gsl = (size_t)T.b0 * 32 + sl;
-        float w = St.w[sl];
+        float w = kLean ? P.wp[gsl] : St.w[sl];
         float m = kSlim ? P.mp[gsl] : St.m[sl], v = kSlim ? P.vp[gsl] : St.v[sl];
         const float p = kSlim ? P.pp[gsl] : St.p[sl];
         const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
@@ -779,7 +784,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
                     static_cast<unsigned long long>(__double2ll_rn(pc * kDqScale)));
         if (L.valid) {
           adam_update(w, m, v, dw, A);
-          St.w[sl] = w;
+          if (kLean) P.wp[gsl] = w; else St.w[sl] = w;
           if (kSlim) { P.mp[gsl] = m; P.vp[gsl] = v; } else { St.m[sl] = m; St.v[sl] = v; }
         }
       } else {
@@ -886,12 +891,12 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     const int nid0 = nbg > 0 ? St.bi[0].x : 0;
     for (int lb = warp; lb < T.nb; lb += NW) {
       const int4 bi = St.bi[lb];
-      const uint32_t pw = St.pw[lb * 32 + lane];
+      const uint32_t pw = kLean ? P.pword[(size_t)(T.b0 + lb) * 32 + lane] : St.pw[lb * 32 + lane];
       if (lb < nbg) {
         Lane L;
         lane_from(bi, pw, P, L);
         const int sl = lb * 32 + lane;
-        const float w = St.w[sl];
+        const float w = kLean ? P.wp[(size_t)T.b0 * 32 + sl] : St.w[sl];
         const float g = L.valid ? gp[bi.x + lane - nid0] : 0.f;
         const float p = softmax_from_noise(L, w, g, A.inv_t);
         if (kSlim) P.pp[(size_t)T.b0 * 32 + sl] = p; else St.p[sl] = p;
@@ -981,7 +986,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     fence_proxy_async();
     const size_t s0 = (size_t)T.b0 * 32;
     const uint32_t gslot_bytes = (uint32_t)nbg * 128u;
-    if (REV) {
+    if (REV && !kLean) {
       bulk_s2g(P.wp + s0, St.w, gslot_bytes);
       if (!kSlim) {
         bulk_s2g(P.mp + s0, St.m, gslot_bytes);
@@ -1026,7 +1031,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
 #endif
 constexpr int kBThreads = DGR_BTHREADS;
 #ifndef DGR_BPERSM
-#define DGR_BPERSM (DGR_SLIM_STAGE ? 5 : 4)
+#define DGR_BPERSM (DGR_SLIM_STAGE ? (DGR_LEAN_STAGE ? 6 : 5) : 4)
 #endif
 constexpr int kBPerSM = DGR_BPERSM;
 constexpr size_t kBSmemBytes = StageLayout::bytes + 8 * kPipeTrees + 64;
