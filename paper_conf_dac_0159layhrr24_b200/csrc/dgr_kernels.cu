@@ -464,9 +464,12 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
   }
 }
 
+// The tile body for "global" tiles (nets spanning more than a window, or too many events on a
+// window cell): operands straight from global memory, no TMA stage.  Run by the first CTAs of the
+// tile_bulk launch (so these long tiles start first and overlap the pipelined ones) or by
+// tile_kernel (persistent driver).
 template <bool REV, bool FWD>
-__global__ void __launch_bounds__(kTileThreads, 3) tile_kernel(KParams P, StepArgs A) {
-  extern __shared__ __align__(128) unsigned char smem[];
+__device__ __forceinline__ void slow_tile(const KParams& P, const StepArgs& A, const TileDesc T, unsigned char* smem) {
   double* S_s = reinterpret_cast<double*>(smem);                 // region A (reverse)
   int* ev_s = reinterpret_cast<int*>(smem);                      // region A (forward)
   float* g_all = reinterpret_cast<float*>(ev_s + 3 * kWinMax);   // region A (forward)
@@ -475,7 +478,6 @@ __global__ void __launch_bounds__(kTileThreads, 3) tile_kernel(KParams P, StepAr
   float* q_s = reinterpret_cast<float*>(dq_s + kTreeMax);
   long long* red_s = reinterpret_cast<long long*>(q_s + kTreeMax);
 
-  const TileDesc T = P.tiles_slow[blockIdx.x];
   const int tid = threadIdx.x, warp = tid >> 5;
   const int ncell = T.ww * T.wh;
   const int X = P.X, Y = P.Y;
@@ -584,6 +586,12 @@ __global__ void __launch_bounds__(kTileThreads, 3) tile_kernel(KParams P, StepAr
     }
     if (tid == 0) { red64(P.scal, red_s[0]); red64(P.scal + 1, red_s[1]); }
   }
+}
+
+template <bool REV, bool FWD>
+__global__ void __launch_bounds__(kTileThreads, 3) tile_kernel(KParams P, StepArgs A) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  slow_tile<REV, FWD>(P, A, P.tiles_slow[blockIdx.x], smem);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1034,7 +1042,8 @@ constexpr int kBThreads = DGR_BTHREADS;
 #define DGR_BPERSM (DGR_SLIM_STAGE ? (DGR_LEAN_STAGE ? 6 : 5) : 4)
 #endif
 constexpr int kBPerSM = DGR_BPERSM;
-constexpr size_t kBSmemBytes = StageLayout::bytes + 8 * kPipeTrees + 64;
+constexpr size_t kBSmemBytes = (StageLayout::bytes + 8 * kPipeTrees + 64) > kSmemBytes ? (StageLayout::bytes + 8 * kPipeTrees + 64)
+                                                                                      : kSmemBytes;
 static_assert(kGpOffset + 4 * 32 * kTargetBundles <= 2 * 8 * kWinMax, "event window + path noise must fit the S window");
 static_assert(8 * kPipeTrees + 12 * kPipeTrees + 32 + 4 * kPipeTrees <= kGpOffset, "tree scratch must not overlap the path noise");
 
@@ -1045,9 +1054,13 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
   long long* dq_s = reinterpret_cast<long long*>(smem + StageLayout::bytes);
   long long* red_s = dq_s + kPipeTrees;
   uint64_t* bar = reinterpret_cast<uint64_t*>(red_s + 2);
+  if ((int)blockIdx.x < P.ntiles_slow) {   // global tiles first: the longest CTAs start earliest
+    slow_tile<REV, FWD>(P, A, P.tiles_slow[blockIdx.x], smem);
+    return;
+  }
   int* ev_s = reinterpret_cast<int*>(St.S);
   float* gp = reinterpret_cast<float*>(reinterpret_cast<unsigned char*>(St.S) + kGpOffset);
-  const TileDesc T = P.tiles[blockIdx.x];
+  const TileDesc T = P.tiles[blockIdx.x - P.ntiles_slow];
   if (threadIdx.x == 0) {
     mbar_init(bar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -1466,10 +1479,12 @@ void launch_tiles(const KParams& p, const StepArgs& a, TileMode mode, cudaStream
       if (mode == kForwardOnly) tile_persistent<false, true><<<grid, kPThreads, kPSmemBytes, s>>>(p, a);
       else if (mode == kReverseForward) tile_persistent<true, true><<<grid, kPThreads, kPSmemBytes, s>>>(p, a);
       else tile_persistent<true, false><<<grid, kPThreads, kPSmemBytes, s>>>(p, a);
-    } else {
-      if (mode == kForwardOnly) tile_bulk<false, true><<<p.ntiles, kBThreads, kBSmemBytes, s>>>(p, a);
-      else if (mode == kReverseForward) tile_bulk<true, true><<<p.ntiles, kBThreads, kBSmemBytes, s>>>(p, a);
-      else tile_bulk<true, false><<<p.ntiles, kBThreads, kBSmemBytes, s>>>(p, a);
+    } else {   // one launch: global tiles in the first CTAs, then the pipelined tiles
+      const int grid = p.ntiles + p.ntiles_slow;
+      if (mode == kForwardOnly) tile_bulk<false, true><<<grid, kBThreads, kBSmemBytes, s>>>(p, a);
+      else if (mode == kReverseForward) tile_bulk<true, true><<<grid, kBThreads, kBSmemBytes, s>>>(p, a);
+      else tile_bulk<true, false><<<grid, kBThreads, kBSmemBytes, s>>>(p, a);
+      return;
     }
   }
   if (p.ntiles_slow > 0) {
