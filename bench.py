@@ -343,7 +343,6 @@ def main():
     forest_build = forest_build_timing(f, dgr, torch, stream, with_cpu=(rank == 0 and not args.no_cpu_baseline))
 
     cells = f.X * f.Y
-    slow = 1 if info["n_tiles"] > info.get("n_pipe_tiles", info["n_tiles"]) else 0
     st = dict(paths=f.n_paths, single_paths=single_paths(f), subnets=f.n_subnets, trees=f.n_trees, nets=f.n_nets,
               bundles=info["n_bundles"], cells=cells)
     if world > 1:   # this rank's share of the per-candidate work
