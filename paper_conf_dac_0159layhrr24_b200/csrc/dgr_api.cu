@@ -216,40 +216,21 @@ struct Plan {
   int64_t n_pipe_tiles = 0;
 };
 
-// (cell, field) pairs of one candidate's demand events in the tile kernel (field 0 dH, 1 dV, 2 VD;
-// see process_tile in dgr_kernels.cu): the collapsed corner events of straight / L / Z lanes, and
-// the eight own events of a C-shape lane.  Returns their number (<= 8).
+// (cell, field) pairs of one candidate's demand events in the pipelined tile kernel (field 0 dH,
+// 1 dV, 2 VD; see process_tile in dgr_kernels.cu): the Z(o, m) form's segment ends and turning
+// points.  Returns their number (<= 8); zero-length segments emit nothing.
 int lane_events(uint32_t pw, int x0, int y0, int x1, int y1, int ex[8], int ey[8], int ef[8]) {
-  const uint32_t shape = pw & 7u;
-  const int m = (int)(pw >> 16);
+  const int o = pw & 1, ntp = (pw >> 1) & 3, m = (int)(pw >> 16);
+  const int p0 = o ? y0 : x0, p1 = o ? y1 : x1, q0 = o ? x0 : y0, q1 = o ? x1 : y1;
   int n = 0;
-  auto ev = [&](int x, int y, int mask) {
-    for (int f = 0; f < 3; ++f) if (mask >> f & 1) { ex[n] = x; ey[n] = y; ef[n] = f; ++n; }
+  auto ev = [&](int f, int p, int q) {   // (p, q) of orientation o -> (x, y)
+    ex[n] = o ? q : p; ey[n] = o ? p : q; ef[n] = f; ++n;
   };
-  if (pw & kOutside) {
-    const int ylo = std::min(y0, y1), yhi = std::max(y0, y1);
-    if (shape == kZHVH) {   // C-HVH
-      ev(std::min(x0, m), y0, 1); ev(std::max(x0, m), y0, 1); ev(std::min(m, x1), y1, 1); ev(std::max(m, x1), y1, 1);
-      ev(m, ylo, 2); ev(m, yhi, 2);
-      ex[n] = m; ey[n] = y0; ef[n++] = 2;
-      ex[n] = m; ey[n] = y1; ef[n++] = 2;
-      return n;
-    }
-    // C-VHV
-    ev(x0, std::min(y0, m), 2); ev(x0, std::max(y0, m), 2); ev(x1, std::min(m, y1), 2); ev(x1, std::max(m, y1), 2);
-    ev(x0, m, 1); ev(x1, m, 1);
-    ex[n] = x0; ey[n] = m; ef[n++] = 2;
-    ex[n] = x1; ey[n] = m; ef[n++] = 2;
-    return n;
-  }
-  switch (shape) {
-    case kStraightH: ev(x0, y0, 1); ev(x1, y0, 1); break;
-    case kStraightV: ev(x0, y0, 2); ev(x0, y1, 2); break;
-    case kHV: ev(x0, y0, 3); ev(x1, y0, 7); break;
-    case kVH: ev(x0, y1, 7); ev(x1, y1, 3); break;
-    case kZHVH: ev(m, y0, 7); ev(m, y1, 7); break;
-    default: ev(x0, m, 7); ev(x1, m, 7); break;
-  }
+  if (m != p0) { ev(o, p0, q0); ev(o, m, q0); }
+  if (p1 != m) { ev(o, m, q1); ev(o, p1, q1); }
+  if (q1 != q0) { ev(1 - o, m, q0); ev(1 - o, m, q1); }
+  if (ntp >= 1) ev(2, m, q0);
+  if (ntp == 2) ev(2, m, q1);
   return n;
 }
 
@@ -345,6 +326,8 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       bool outside;
       if (!classify(d, i, x0, y0, x1, y1, &shape, &mid, &outside)) { ok = false; break; }
       shapes[i - p0] = shape | (outside ? kOutside : 0u);
+      if (shape == kStraightH || shape == kHV) mid = x1;   // m = p1: the Z(o, m) form of path_cost
+      if (shape == kStraightV || shape == kVH) mid = y1;
       pw_path[i - pl.path_lo] = shape | (outside ? kOutside : 0u) | ((uint32_t)mid << 16);
       if (outside && shape == kZHVH) { ex0 = std::min(ex0, mid); ex1 = std::max(ex1, mid); }
       if (outside && shape == kZVHV) { ey0 = std::min(ey0, mid); ey1 = std::max(ey1, mid); }
@@ -532,6 +515,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
 #pragma omp parallel
   {
     std::vector<uint16_t> cnt;
+    std::vector<size_t> cell_buf;
 #pragma omp for schedule(dynamic, 16)
     for (int64_t t = 0; t < ntile; ++t) {
       TileDesc T{};
@@ -625,24 +609,28 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
           ++ks;
         }
       }
-      // int32 shared-memory accumulation is exact while no window cell-field gets more than
-      // kEventMax events (each |event| <= 2^24); otherwise run the tile against global memory.
+      // int32 shared-memory accumulation is exact while no window cell-field is touched by more
+      // than kEventMax sub-nets: the events one sub-net puts on one cell-field sum to at most
+      // sum_j |pi_j| <= 2^24 + 32 in magnitude.  Otherwise run the tile against global memory.
       if (!T.global) {
         cnt.assign((size_t)3 * T.ww * T.wh, 0);
         bool ok = true;
+        std::vector<size_t>& cells = cell_buf;
         for (int64_t sn = d->tree_sub_off[j0]; sn < d->tree_sub_off[j1] && ok; ++sn) {
           const short4 e = sxy_csr[sn - pl.sub_lo];
-          for (int64_t i = d->sub_path_off[sn]; i < d->sub_path_off[sn + 1] && ok; ++i) {
+          cells.clear();
+          for (int64_t i = d->sub_path_off[sn]; i < d->sub_path_off[sn + 1]; ++i) {
             const uint32_t pw = pw_path[i - pl.path_lo];
             int ex[8], ey[8], ef[8];
             const int ne = lane_events(pw, e.x, e.y, e.z, e.w, ex, ey, ef);
-            for (int q = 0; q < ne && ok; ++q) {
+            for (int q = 0; q < ne; ++q)
               // the event windows of the H / VD fields are row-major, the V field's column-major;
               // any fixed cell index works for counting
-              const size_t c = (size_t)ef[q] * T.ww * T.wh + (size_t)(ey[q] - T.wy0) * T.ww + (ex[q] - T.wx0);
-              if (++cnt[c] > kEventMax) ok = false;
-            }
+              cells.push_back((size_t)ef[q] * T.ww * T.wh + (size_t)(ey[q] - T.wy0) * T.ww + (ex[q] - T.wx0));
           }
+          std::sort(cells.begin(), cells.end());
+          for (size_t q = 0; q < cells.size() && ok; ++q)
+            if ((q == 0 || cells[q] != cells[q - 1]) && ++cnt[cells[q]] > kEventMax) ok = false;
         }
         if (!ok) { T.global = 1; T.wx0 = T.wy0 = T.ww = T.wh = 0; }
       }

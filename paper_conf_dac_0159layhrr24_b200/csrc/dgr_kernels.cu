@@ -120,8 +120,10 @@ __device__ __forceinline__ void red64(long long* p, long long v) {
 __device__ __forceinline__ void adam_update(float& w, float& m, float& v, float g, const StepArgs& A) {
   m = fmaf(0.1f, g - m, m);                         // m.lerp_(g, 1 - beta1)
   v = fmaf(0.999f, v, 0.001f * g * g);              // v * beta2 + (1 - beta2) g^2
-  const float denom = sqrtf(v) * A.inv_sqrt_bc2 + 1e-8f;
-  w -= A.lr_over_bc1 * (m / denom);
+  // sqrt(v) = v rsqrt(v) (MUFU, v >= 0) and a MUFU division: ~1e-7 relative, well inside the 1e-4 bar
+  const float sq = v > 0.f ? v * rsqrtf(v) : 0.f;
+  const float denom = sq * A.inv_sqrt_bc2 + 1e-8f;
+  w -= A.lr_over_bc1 * __fdividef(m, denom);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -135,17 +137,21 @@ struct Win {
   __device__ __forceinline__ int v(int x, int y) const { return hv + (x - ox) * vs + (y - oy); }
 };
 
-struct Shape6 {
-  bool sh, sv, hv, vh, zh, zv;
-  __device__ __forceinline__ explicit Shape6(uint32_t s)
-      : sh(s == kStraightH), sv(s == kStraightV), hv(s == kHV), vh(s == kVH), zh(s == kZHVH), zv(s == kZVHV) {}
-};
+// Orientation-neutral pattern form.  Every pattern is "Z(o, m)": o = 0 lays the first and third
+// segments along H rows (straight H, HV, Z-HVH), o = 1 along V columns (straight V, VH, Z-VHV).
+// With (p, q) = (x, y) for o = 0 and (y, x) for o = 1, the sub-net runs from (p0, q0) to (p1, q1)
+// and the pattern word carries m:
+//   seg 1: primary line q0 from p0 to m;     seg 2: secondary line m from q0 to q1;
+//   seg 3: primary line q1 from m to p1;     turning points (m, q0) [ntp >= 1], (m, q1) [ntp = 2].
+// L shapes have m = p1 (seg 3 empty, one turning point), straight paths m = p1 and q0 = q1, Z
+// shapes m strictly between p0 and p1, C-shapes (row f4, Q14b) m outside [p0, p1].  For the Shape
+// enum o = shape & 1 and ntp = shape >> 1.  A segment "from a to b" covers the edges
+// [min(a,b), max(a,b)) of its line, so its G sum is sgn(b - a) (S[b] - S[a]), S the line's
+// exclusive prefix.
+__device__ __forceinline__ int isgn(int d) { return (d > 0) - (d < 0); }
 
-// c_i = a1 WL + a2 sqrt(L) TP + sum over the path's edges of G + beta sum over its turning points of
-// the G of the incident edges; a segment's sum is S[hi] - S[lo].  Branch-free: the pattern selects
-// up to three segments and two turning points (straight, HV, VH, Z-HVH(x_m), Z-VHV(y_m)); unused
-// slots read valid cells and are weighted by 0.
-__device__ __forceinline__ int detour(uint32_t pw, int x0, int y0, int x1, int y1) {   // C-shape (Q14b)
+// detour length of a C-shape (row f4, reading Q14b): how far x_m / y_m lies outside the span
+__device__ __forceinline__ int detour(uint32_t pw, int x0, int y0, int x1, int y1) {
   if (!(pw & kOutside)) return 0;
   const int m = (int)(pw >> 16);
   if ((pw & 7u) == kZHVH) return m < x0 ? x0 - m : m - x1;
@@ -153,46 +159,28 @@ __device__ __forceinline__ int detour(uint32_t pw, int x0, int y0, int x1, int y
   return m < ylo ? ylo - m : m - yhi;
 }
 
+// c_i = a1 WL + a2 sqrt(L) TP + sum over the path's edges of G + beta sum over its turning points
+// of the G of the incident edges (Eqs. (9)-(12) chain rule, reading Q3).  Element (a, b) of
+// orientation o (H: a = y, b = x; V: a = x, b = y) of the window / grid W is at a * L[o] + b + B[o].
 __device__ __forceinline__ double path_cost(const double* S, const Win& W, int X, int Y, uint32_t pw, int x0,
                                             int y0, int x1, int y1, const StepArgs& A) {
-  const uint32_t shape = pw & 7u;
-  const int m = (int)(pw >> 16);
-  const Shape6 k(shape);
-  const int ylo = min(y0, y1), yhi = max(y0, y1);
-  // segment 1 (always); Z / C segments between x0 (y0) and m in either order
-  const bool v1 = k.sv | k.vh | k.zv;
-  const int l1 = v1 ? x0 : y0;
-  const int a1 = v1 ? (k.zv ? min(y0, m) : ylo) : (k.zh ? min(x0, m) : x0);
-  const int b1 = v1 ? (k.zv ? max(y0, m) : yhi) : (k.zh ? max(x0, m) : x1);
-  // segment 2 (L and Z)
-  const bool v2 = k.hv | k.zh;
-  const int l2 = k.hv ? x1 : (k.vh ? y1 : m);
-  const int a2 = v2 ? ylo : x0;
-  const int b2 = v2 ? yhi : x1;
-  // segment 3 (Z)
-  const int l3 = k.zh ? y1 : x1;
-  const int a3 = k.zh ? min(m, x1) : min(m, y1);
-  const int b3 = k.zh ? max(m, x1) : max(m, y1);
-  const bool s2 = !(k.sh | k.sv), s3 = k.zh | k.zv;
-  // turning points (default cell (x0, y0) when unused)
-  const int tx0 = k.hv ? x1 : (k.zh ? m : x0);
-  const int ty0 = k.hv ? y0 : (k.vh ? y1 : (k.zv ? m : y0));
-  const int tx1 = k.zh ? m : (k.zv ? x1 : x0);
-  const int ty1 = k.zh ? y1 : (k.zv ? m : y0);
-  const int ntp = (k.hv | k.vh) ? 1 : (s3 ? 2 : 0);
-  auto sidx = [&](bool isv, int line, int pos) { return isv ? W.v(line, pos) : W.h(pos, line); };
-  const int i1b = sidx(v1, l1, b1), i1a = sidx(v1, l1, a1);
-  const int i2b = s2 ? sidx(v2, l2, b2) : i1b, i2a = s2 ? sidx(v2, l2, a2) : i1b;
-  const int i3b = s3 ? sidx(k.zv, l3, b3) : i1b, i3a = s3 ? sidx(k.zv, l3, a3) : i1b;
-  const double seg = (S[i1b] - S[i1a]) + (S[i2b] - S[i2a]) + (S[i3b] - S[i3a]);
-  auto tp = [&](int x, int y) -> double {
-    return S[W.h(min(x + 1, X - 1), y)] - S[W.h(max(x - 1, 0), y)] + S[W.v(x, min(y + 1, Y - 1))] -
-           S[W.v(x, max(y - 1, 0))];
-  };
-  const double t0 = tp(tx0, ty0), t1 = tp(tx1, ty1);
-  const double tps = (ntp >= 1 ? t0 : 0.0) + (ntp >= 2 ? t1 : 0.0);
-  return seg + (double)A.beta * tps + (double)A.a_wl * (double)((x1 - x0) + (yhi - ylo) + 2 * detour(pw, x0, y0, x1, y1)) +
-         (double)A.a_via * (double)A.sqrt_l * ntp;
+  const int o = pw & 1, ntp = (pw >> 1) & 3, m = (int)(pw >> 16);
+  const int p0 = o ? y0 : x0, p1 = o ? y1 : x1, q0 = o ? x0 : y0, q1 = o ? x1 : y1;
+  const int Lp = o ? W.vs : W.hs, Ls = o ? W.hs : W.vs;
+  const int B0 = -(W.oy * W.hs + W.ox), B1 = W.hv - W.ox * W.vs - W.oy;
+  const int Bp = o ? B1 : B0, Bs = o ? B0 : B1;
+  const int r0 = q0 * Lp + Bp, r1 = q1 * Lp + Bp, sb = m * Ls + Bs;
+  const int a0 = r0 + m, a1 = r1 + m, s0 = sb + q0, s1 = sb + q1;
+  const int g1 = isgn(m - p0), g2 = isgn(q1 - q0), g3 = isgn(p1 - m);
+  double c = (double)g1 * (S[a0] - S[r0 + p0]) + (double)g2 * (S[s1] - S[s0]) + (double)g3 * (S[r1 + p1] - S[a1]);
+  // turning-point windows: the (clipped) edges left / right and below / above the cell
+  const int pmax = (o ? Y : X) - 1, qmax = (o ? X : Y) - 1;
+  const int mp = m < pmax, mn = m > 0;
+  double tp = 0.0;
+  if (ntp >= 1) tp = (S[a0 + mp] - S[a0 - mn]) + (S[s0 + (q0 < qmax)] - S[s0 - (q0 > 0)]);
+  if (ntp == 2) tp += (S[a1 + mp] - S[a1 - mn]) + (S[s1 + (q1 < qmax)] - S[s1 - (q1 > 0)]);
+  const int wl = abs(m - p0) + abs(p1 - m) + abs(q1 - q0);
+  return c + (double)A.beta * tp + (double)A.a_wl * (double)wl + (double)A.a_via * (double)A.sqrt_l * (double)ntp;
 }
 
 __device__ __forceinline__ void red_shared_add(uint32_t saddr, int v) {
@@ -752,6 +740,8 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
   const int ncell = T.ww * T.wh;
   const Win W{T.wx0, T.wy0, T.ww, T.wh, ncell};
+  const int wB0 = -(T.wy0 * T.ww + T.wx0), wB1 = ncell - T.wx0 * T.wh - T.wy0;   // orientation bases
+  const int hv2 = 2 * ncell;                                                    // VD part of the window
   const int nbg = T.nbg;
 
   // ---------------- reverse of iteration k ----------------
@@ -777,11 +767,9 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         const double dp = (double)q * c;
         const double dref = __shfl_sync(kFull, dp, L.head);
         const float dd = (float)(dp - dref);
-        float sa = seg_reduce(p * dd, L.lane, L.end, Sum());
-        float sb = seg_reduce(p, L.lane, L.end, Sum());
+        float sa = seg_reduce(p * dd, L.lane, L.end, Sum());   // sum_k p_k = 1 up to rounding (~1e-7)
         sa = __shfl_sync(kFull, sa, L.head);
-        sb = __shfl_sync(kFull, sb, L.head);
-        const float dw = L.valid ? p * A.inv_t * (dd - __fdividef(sa, sb)) : 0.f;
+        const float dw = L.valid ? p * A.inv_t * (dd - sa) : 0.f;
         // dq_j partial sums over runs of lanes of one tree (fp64 -> 2^-32 fixed point)
         const uint32_t th = L.tm | __ballot_sync(kFull, !L.valid) | 1u;
         const uint32_t trest = th & ~L.le;
@@ -910,57 +898,31 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         if (kSlim) P.pp[(size_t)T.b0 * 32 + sl] = p; else St.p[sl] = p;
         const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
         const int vq = L.valid ? __float2int_rn(q * p * kFixScale) : 0;
-        int sc = vq;
-#pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {
-          const int o = __shfl_up_sync(kFull, sc, off);
-          if (L.lane - off >= L.head) sc += o;
-        }
-        const bool outside = (L.pw & kOutside) != 0;   // C-shape lanes: own events, outside the collapse
-        const int nh = __popc(__ballot_sync(kFull, L.shape == kZHVH && !outside) & L.gmask);
-        const int nv = __popc(__ballot_sync(kFull, L.shape == kZVHV && !outside) & L.gmask);
-        const int h1 = min(L.head + 1, 31), h2 = min(L.head + 1 + nh, 31), h3 = min(L.head + 1 + nh + nv, 31);
-        const int a = __shfl_sync(kFull, vq, L.head);
-        const int bb = __shfl_sync(kFull, vq, h1);
-        const int S1 = __shfl_sync(kFull, sc, h1);
-        const int S2 = __shfl_sync(kFull, sc, h2);
-        const int S3 = __shfl_sync(kFull, sc, h3);
-        const short4 e = L.valid ? St.sxy[L.sub - s_lo] : make_short4(0, 0, 0, 0);
-        const int x0 = e.x, y0 = e.y, x1 = e.z, y1 = e.w;
-        const int sgn = (y1 > y0) ? 1 : -1;
-        const int hs = S2 - S1, vs = S3 - S2, vv = vq;
-        const int mm = (int)(L.pw >> 16);
-        const int fSH = L.shape == kStraightH, fSV = L.shape == kStraightV, fHV = L.shape == kHV;
-        const int fVH = L.shape == kVH, fZH = L.shape == kZHVH && !outside, fZV = L.shape == kZVHV && !outside;
-        const int fZ = fZH + fZV;
-        const int xa = x0 + fZH * (mm - x0);
-        const int ya = y0 + fVH * (y1 - y0) + fZV * (mm - y0);
-        const int xb = x1 + fSV * (x0 - x1) + fZH * (mm - x1);
-        const int yb = y1 + (fSH + fHV) * (y0 - y1) + fZV * (mm - y1);
-        const int ah = fSH * vv + fHV * (a + hs) + fVH * bb + (fZV - fZH) * vv;
-        const int av = fSV * vv + sgn * (fHV * (bb + vs) - fVH * bb + (fZH - fZV) * vv);
-        const int ad = fVH * bb + fZ * vv;
-        const int bh = -fSH * vv - fHV * a - fVH * (bb + hs) + (fZH - fZV) * vv;
-        const int bv = -fSV * vv + sgn * (fHV * a - fVH * (a + vs) + (fZV - fZH) * vv);
-        const int bd = fHV * a + fZ * vv;
         if (L.valid && !(P.skip & 4)) {
-          const int hv2 = 2 * ncell;
-          const int ia_h = W.h(xa, ya), ib_h = W.h(xb, yb);
-          red_shared_add(ev_base + 4u * ia_h, ah);
-          red_shared_add(ev_base + 4u * W.v(xa, ya), av);
-          red_shared_add(ev_base + 4u * (hv2 + ia_h), ad);
-          red_shared_add(ev_base + 4u * ib_h, bh);
-          red_shared_add(ev_base + 4u * W.v(xb, yb), bv);
-          red_shared_add(ev_base + 4u * (hv2 + ib_h), bd);
-          wl_acc += (long long)vq * ((x1 - x0) + abs(y1 - y0));
-          tp_acc += (long long)vq * (fHV + fVH + 2 * fZ);
-          if (outside) {
-            c_events(L.pw, x0, y0, x1, y1, vq, [&](int fld, int x, int y, int val) {
-              red_shared_add(ev_base + 4u * (fld == 0 ? W.h(x, y) : fld == 1 ? W.v(x, y) : hv2 + W.h(x, y)), val);
-            });
-            wl_acc += (long long)vq * (2 * detour(L.pw, x0, y0, x1, y1));
-            tp_acc += 2 * (long long)vq;
-          }
+          // the candidate's own demand events in the Z(o, m) form (see path_cost): seg 1 from p0
+          // to m on line q0, seg 2 from q0 to q1 on line m, seg 3 from m to p1 on line q1, each
+          // +-sgn v at its two ends, plus its turning points.  No cross-lane collapse: lanes of one
+          // sub-net that share a corner cell meet in the shared-memory reduction.
+          const short4 e = St.sxy[L.sub - s_lo];
+          const int x0 = e.x, y0 = e.y, x1 = e.z, y1 = e.w;
+          const int o = L.pw & 1, ntp = (L.pw >> 1) & 3, m = (int)(L.pw >> 16);
+          const int p0 = o ? y0 : x0, p1 = o ? y1 : x1, q0 = o ? x0 : y0, q1 = o ? x1 : y1;
+          const int g1 = isgn(m - p0) * vq, g2 = isgn(q1 - q0) * vq, g3 = isgn(p1 - m) * vq;
+          const int Lp = o ? W.vs : W.hs, Ls = o ? W.hs : W.vs;
+          const int Bp = o ? wB1 : wB0, Bs = o ? wB0 : wB1;
+          const int r0 = q0 * Lp + Bp, r1 = q1 * Lp + Bp, sb = m * Ls + Bs;
+          const int a0 = r0 + m, a1 = r1 + m, s0 = sb + q0, s1 = sb + q1;
+          red_shared_add(ev_base + 4u * (r0 + p0), g1);
+          red_shared_add(ev_base + 4u * a0, -g1);
+          red_shared_add(ev_base + 4u * a1, g3);
+          red_shared_add(ev_base + 4u * (r1 + p1), -g3);
+          red_shared_add(ev_base + 4u * s0, g2);
+          red_shared_add(ev_base + 4u * s1, -g2);
+          // turning points: VD takes the H-orientation index of the cell (a for o = 0, s for o = 1)
+          red_shared_add(ev_base + 4u * (hv2 + (o ? s0 : a0)), ntp >= 1 ? vq : 0);
+          red_shared_add(ev_base + 4u * (hv2 + (o ? s1 : a1)), ntp == 2 ? vq : 0);
+          wl_acc += (long long)vq * (abs(m - p0) + abs(p1 - m) + abs(q1 - q0));
+          tp_acc += (long long)vq * ntp;
         }
       } else {
         // singleton bundle: pi = q; +pi where the segment starts, -pi where it ends
