@@ -763,21 +763,18 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
           const short4 e = St.sxy[L.sub - s_lo];
           c = path_cost(St.S, W, X, Y, L.pw, e.x, e.y, e.z, e.w, A);
         }
-        // softmax backward: differences to the group head's dp in fp64, reduced in fp32
-        const double dp = (double)q * c;
-        const double dref = __shfl_sync(kFull, dp, L.head);
-        const float dd = (float)(dp - dref);
-        float sa = seg_reduce(p * dd, L.lane, L.end, Sum());   // sum_k p_k = 1 up to rounding (~1e-7)
+        // softmax backward over the sub-net: with c_h the head's c and dd = c - c_h (fp64
+        // difference, then fp32), sum_k p_k c_k = c_h + sa where sa = sum_k p_k dd_k (sum_k p_k = 1
+        // up to ~1e-7), so dw_i = (p_i / t) q (dd_i - sa) and the head adds c_h + sa to dq_tree
+        // (2^-32 fixed point): no cross-lane reduction over the tree's lanes.
+        const double ch = __shfl_sync(kFull, c, L.head);
+        const float dd = (float)(c - ch);
+        float sa = seg_reduce(p * dd, L.lane, L.end, Sum());
         sa = __shfl_sync(kFull, sa, L.head);
-        const float dw = L.valid ? p * A.inv_t * (dd - sa) : 0.f;
-        // dq_j partial sums over runs of lanes of one tree (fp64 -> 2^-32 fixed point)
-        const uint32_t th = L.tm | __ballot_sync(kFull, !L.valid) | 1u;
-        const uint32_t trest = th & ~L.le;
-        const int tend = trest ? (__ffs(trest) - 2) : 31;
-        const double pc = seg_reduce(L.valid ? (double)p * c : 0.0, L.lane, tend, Sum());
-        if (L.valid && ((th >> L.lane) & 1u))
+        const float dw = L.valid ? p * A.inv_t * q * (dd - sa) : 0.f;
+        if (L.valid && L.lane == L.head)
           atomicAdd(reinterpret_cast<unsigned long long*>(&dq_s[L.tree - T.tree0]),
-                    static_cast<unsigned long long>(__double2ll_rn(pc * kDqScale)));
+                    static_cast<unsigned long long>(__double2ll_rn((c + (double)sa) * kDqScale)));
         if (L.valid) {
           adam_update(w, m, v, dw, A);
           if (kLean) P.wp[gsl] = w; else St.w[sl] = w;
@@ -1129,11 +1126,13 @@ __device__ __forceinline__ T warp_inclusive_scan(T x, int lane) {
 }
 
 // Exclusive scan of a chunk of kGThreads * kGItems elements held "striped": thread t holds
-// elements j * kGThreads + t (j < kGItems), so every global access is coalesced.  One barrier.
+// elements j * kGThreads + t (j < kGItems), so every global access is coalesced.  Warp scans of
+// each item, then one warp scans the kGItems * NW warp totals (in position order), two barriers.
 template <typename T>
 __device__ __forceinline__ void striped_exclusive_scan(T (&v)[kGItems], T* sh /* kGItems*32 */, T* total) {
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   constexpr int NW = kGThreads / 32;
+  static_assert(kGItems * NW <= 32, "one warp scans the segment totals");
   T inc[kGItems];
 #pragma unroll
   for (int j = 0; j < kGItems; ++j) inc[j] = warp_inclusive_scan(v[j], lane);
@@ -1142,20 +1141,16 @@ __device__ __forceinline__ void striped_exclusive_scan(T (&v)[kGItems], T* sh /*
     for (int j = 0; j < kGItems; ++j) sh[j * NW + wid] = inc[j];
   }
   __syncthreads();
-  T run = T(0);
-#pragma unroll
-  for (int j = 0; j < kGItems; ++j) {
-    T before = run, rowtot = T(0);
-#pragma unroll
-    for (int w = 0; w < NW; ++w) {
-      const T t = sh[j * NW + w];
-      if (w < wid) before += t;
-      rowtot += t;
-    }
-    v[j] = before + inc[j] - v[j];   // exclusive
-    run += rowtot;
+  if (wid == 0) {
+    const T t = lane < kGItems * NW ? sh[lane] : T(0);
+    const T x = warp_inclusive_scan(t, lane);
+    if (lane < kGItems * NW) sh[lane] = x - t;        // exclusive prefix of the segment totals
+    if (lane == kGItems * NW - 1) sh[32] = x;         // chunk total
   }
-  *total = run;
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < kGItems; ++j) v[j] = sh[j * NW + wid] + inc[j] - v[j];   // exclusive
+  *total = sh[32];
   __syncthreads();
 }
 
@@ -1181,8 +1176,8 @@ __device__ __forceinline__ void kg_finalize(const KParams& P, const StepArgs& A)
 }
 
 __global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A) {
-  __shared__ long long shl[kGItems * (kGThreads / 32)];
-  __shared__ double shd[kGItems * (kGThreads / 32)];
+  __shared__ long long shl[33];
+  __shared__ double shd[33];
   const int line = blockIdx.x;
   const bool isH = line < P.Y;
   const int n = isH ? P.X : P.Y;
@@ -1228,23 +1223,25 @@ __global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A)
         const long long W = carryW + ex[j] + v[j];   // inclusive prefix = wire demand of edge pos
         const double d = (double)W * kFixInv + beta * ((double)(t0[j] + t1[j]) * kFixInv);
         const double x = d - (double)cp[j];                 // overflow x = -(cap - d)
-        const double sl = (double)A.f_slope;
-        double fv, fg;                                      // f(x) and df/dx = df/dd
+        // f(x) and df/dx = df/dd in fp32 (x itself in fp64: d comes from exact fixed point);
+        // relative error ~1e-6, well inside the 1e-4 bar, at a fraction of fp64 exp's cost
+        const float xf = (float)x, sf = A.f_slope;
+        double fv, fg;
         switch (A.f_kind) {
-          case 0: {   // sigmoid sigma(s x); stable for both signs; fp64 (one exp per edge)
-            const double e = exp(-fabs(sl * x));
-            const double inv = 1.0 / (1.0 + e);
-            fv = (sl * x > 0.0) ? inv : e * inv;
-            fg = sl * e * inv * inv;
+          case 0: {   // sigmoid sigma(s x); stable for both signs
+            const float e = __expf(-fabsf(sf * xf));
+            const float inv = __fdividef(1.f, 1.f + e);
+            fv = (sf * xf > 0.f) ? inv : e * inv;
+            fg = sf * e * inv * inv;
             break;
           }
           case 1: fv = x > 0.0 ? x : 0.0; fg = x > 0.0 ? 1.0 : 0.0; break;        // ReLU
-          case 2: fv = x > 0.0 ? x : sl * x; fg = x > 0.0 ? 1.0 : sl; break;      // LeakyReLU (Fig. 6)
-          case 3: fv = exp(sl * x); fg = sl * fv; break;                          // exp (Fig. 6)
+          case 2: fv = x > 0.0 ? x : (double)sf * x; fg = x > 0.0 ? 1.0 : (double)sf; break;   // LeakyReLU (Fig. 6)
+          case 3: fv = exp((double)sf * x); fg = (double)sf * fv; break;          // exp (Fig. 6): fp64 range
           default: {                                                              // CELU (Fig. 6)
-            const double e = exp(fmin(x, 0.0) / sl);
-            fv = x > 0.0 ? x : sl * (e - 1.0);
-            fg = x > 0.0 ? 1.0 : e;
+            const float e = expf(fminf(xf, 0.f) / sf);
+            fv = x > 0.0 ? x : (double)(sf * (e - 1.f));
+            fg = x > 0.0 ? 1.0 : (double)e;
           }
         }
         of += fv;
