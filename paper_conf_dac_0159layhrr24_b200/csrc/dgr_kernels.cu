@@ -171,8 +171,9 @@ __device__ __forceinline__ double path_cost(const double* S, const Win& W, int X
   const int Bp = o ? B1 : B0, Bs = o ? B0 : B1;
   const int r0 = q0 * Lp + Bp, r1 = q1 * Lp + Bp, sb = m * Ls + Bs;
   const int a0 = r0 + m, a1 = r1 + m, s0 = sb + q0, s1 = sb + q1;
-  const int g1 = isgn(m - p0), g2 = isgn(q1 - q0), g3 = isgn(p1 - m);
-  double c = (double)g1 * (S[a0] - S[r0 + p0]) + (double)g2 * (S[s1] - S[s0]) + (double)g3 * (S[r1 + p1] - S[a1]);
+  // each segment's G sum as S[max] - S[min] (a zero-length segment gives 0)
+  double c = (S[r0 + max(p0, m)] - S[r0 + min(p0, m)]) + (S[sb + max(q0, q1)] - S[sb + min(q0, q1)]) +
+             (S[r1 + max(m, p1)] - S[r1 + min(m, p1)]);
   // turning-point windows: the (clipped) edges left / right and below / above the cell
   const int pmax = (o ? Y : X) - 1, qmax = (o ? X : Y) - 1;
   const int mp = m < pmax, mn = m > 0;
@@ -353,7 +354,6 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
   const int lane = threadIdx.x & 31;
   const int4 bfirst = __ldg(&P.binfo[bw0]);
   const uint32_t ev_base = (uint32_t)__cvta_generic_to_shared(ev_s);
-  long long wl = 0, tpc = 0;
   size_t slot = (size_t)bw0 * 32 + lane;
   Lane L;
   lane_from(bfirst, __ldg(&P.pword[slot]), P, L);
@@ -415,9 +415,6 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
         red64(P.dH + (size_t)yb * X + xb, bh); red64(P.dVT + (size_t)xb * Y + yb, bv);
         red64(P.VD + (size_t)yb * X + xb, bd);
       }
-      const int ntp = fHV + fVH + 2 * fZ + 2 * outside;
-      wl += (long long)vq * ((x1 - x0) + abs(y1 - y0) + 2 * detour(L.pw, x0, y0, x1, y1));
-      tpc += (long long)vq * ntp;
       if (outside) {
         if (GLOBAL) {
           const int X = P.X, Y = P.Y;
@@ -444,12 +441,7 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
     L = Ln; e = en;
     slot += 32;
   }
-  wl = seg_reduce(wl, lane, 31, Sum());
-  tpc = seg_reduce(tpc, lane, 31, Sum());
-  if (lane == 0) {
-    atomicAdd(reinterpret_cast<unsigned long long*>(&red_s[0]), static_cast<unsigned long long>(wl));
-    atomicAdd(reinterpret_cast<unsigned long long*>(&red_s[1]), static_cast<unsigned long long>(tpc));
-  }
+
 }
 
 // The tile body for "global" tiles (nets spanning more than a window, or too many events on a
@@ -572,7 +564,6 @@ __device__ __forceinline__ void slow_tile(const KParams& P, const StepArgs& A, c
         for (int yi = lane; yi < T.wh; yi += 32) red64(P.dVT + g0 + yi, colV[yi]);
       }
     }
-    if (tid == 0) { red64(P.scal, red_s[0]); red64(P.scal + 1, red_s[1]); }
   }
 }
 
@@ -732,7 +723,6 @@ template <bool REV, bool FWD, int NT>
 __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A, const TileDesc& T, Stage St,
                                              int* ev_s, float* gp, long long* dq_s, long long* red_s) {
   // dq_s[0..ntree) and red_s[0..2) arrive zeroed (the caller clears them before its first barrier)
-  long long wl_acc = 0, tp_acc = 0;
   constexpr int NW = NT / 32;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int X = P.X, Y = P.Y;
@@ -840,9 +830,14 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
       if (FWD) {
         // q_j = softmax over the net's trees of (w_j + g_j)/t, iteration k_next (noise stream 1)
         float zmax = -INFINITY;
+        int64_t cq = -1;   // one Philox call per aligned quad of tree indices
+        uint4 r = make_uint4(0u, 0u, 0u, 0u);
         for (int j = a; j < b; ++j) {
           const int64_t gj = P.tree_base + t_lo + j;
-          const uint4 r = philox4x32_10(make_uint4((uint32_t)(gj >> 2), (uint32_t)(gj >> 34), (uint32_t)A.k_next, 1u), key);
+          if ((gj >> 2) != cq) {
+            cq = gj >> 2;
+            r = philox4x32_10(make_uint4((uint32_t)cq, (uint32_t)(cq >> 32), (uint32_t)A.k_next, 1u), key);
+          }
           const uint32_t wd = (gj & 3) == 0 ? r.x : (gj & 3) == 1 ? r.y : (gj & 3) == 2 ? r.z : r.w;
           const float zj = (St.wt[j] + gumbel_word(wd)) * A.inv_t;
           St.q[j] = zj;
@@ -898,28 +893,27 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         if (L.valid && !(P.skip & 4)) {
           // the candidate's own demand events in the Z(o, m) form (see path_cost): seg 1 from p0
           // to m on line q0, seg 2 from q0 to q1 on line m, seg 3 from m to p1 on line q1, each
-          // +-sgn v at its two ends, plus its turning points.  No cross-lane collapse: lanes of one
+          // +v at its lower and -v at its upper end, plus its turning points.  No cross-lane collapse: lanes of one
           // sub-net that share a corner cell meet in the shared-memory reduction.
           const short4 e = St.sxy[L.sub - s_lo];
           const int x0 = e.x, y0 = e.y, x1 = e.z, y1 = e.w;
           const int o = L.pw & 1, ntp = (L.pw >> 1) & 3, m = (int)(L.pw >> 16);
           const int p0 = o ? y0 : x0, p1 = o ? y1 : x1, q0 = o ? x0 : y0, q1 = o ? x1 : y1;
-          const int g1 = isgn(m - p0) * vq, g2 = isgn(q1 - q0) * vq, g3 = isgn(p1 - m) * vq;
           const int Lp = o ? W.vs : W.hs, Ls = o ? W.hs : W.vs;
           const int Bp = o ? wB1 : wB0, Bs = o ? wB0 : wB1;
           const int r0 = q0 * Lp + Bp, r1 = q1 * Lp + Bp, sb = m * Ls + Bs;
           const int a0 = r0 + m, a1 = r1 + m, s0 = sb + q0, s1 = sb + q1;
-          red_shared_add(ev_base + 4u * (r0 + p0), g1);
-          red_shared_add(ev_base + 4u * a0, -g1);
-          red_shared_add(ev_base + 4u * a1, g3);
-          red_shared_add(ev_base + 4u * (r1 + p1), -g3);
-          red_shared_add(ev_base + 4u * s0, g2);
-          red_shared_add(ev_base + 4u * s1, -g2);
+          // each segment: +v at its lower end, -v at its upper end (nothing if zero-length)
+          const int v1 = m != p0 ? vq : 0, v2 = q1 != q0 ? vq : 0, v3 = p1 != m ? vq : 0;
+          red_shared_add(ev_base + 4u * (r0 + min(p0, m)), v1);
+          red_shared_add(ev_base + 4u * (r0 + max(p0, m)), -v1);
+          red_shared_add(ev_base + 4u * (sb + min(q0, q1)), v2);
+          red_shared_add(ev_base + 4u * (sb + max(q0, q1)), -v2);
+          red_shared_add(ev_base + 4u * (r1 + min(m, p1)), v3);
+          red_shared_add(ev_base + 4u * (r1 + max(m, p1)), -v3);
           // turning points: VD takes the H-orientation index of the cell (a for o = 0, s for o = 1)
           red_shared_add(ev_base + 4u * (hv2 + (o ? s0 : a0)), ntp >= 1 ? vq : 0);
           red_shared_add(ev_base + 4u * (hv2 + (o ? s1 : a1)), ntp == 2 ? vq : 0);
-          wl_acc += (long long)vq * (abs(m - p0) + abs(p1 - m) + abs(q1 - q0));
-          tp_acc += (long long)vq * ntp;
         }
       } else {
         // singleton bundle: pi = q; +pi where the segment starts, -pi where it ends
@@ -934,20 +928,11 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
           const int ib = isv ? W.v(e.x, e.w) : W.h(e.z, e.y);
           red_shared_add(ev_base + 4u * ia, vq);
           red_shared_add(ev_base + 4u * ib, -vq);
-          wl_acc += (long long)vq * ((e.z - e.x) + (e.w - e.y));
         }
       }
     }
-    // E[WL], E[TP] partial sums: warp reduction, then one shared atomic per warp
-    wl_acc = seg_reduce(wl_acc, lane, 31, Sum());
-    tp_acc = seg_reduce(tp_acc, lane, 31, Sum());
-    if (lane == 0) {
-      atomicAdd(reinterpret_cast<unsigned long long*>(&red_s[0]), static_cast<unsigned long long>(wl_acc));
-      atomicAdd(reinterpret_cast<unsigned long long*>(&red_s[1]), static_cast<unsigned long long>(tp_acc));
-    }
   }
   __syncthreads();
-  if (FWD && tid == 32) { red64(P.scal, red_s[0]); red64(P.scal + 1, red_s[1]); }
   // write back the tile's group slot state with bulk stores (asynchronous; readers wait on the group)
   if (tid == 0 && nbg > 0) {
     fence_proxy_async();
@@ -1192,7 +1177,9 @@ __global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A)
   float* dout = (isH ? P.dOutH : P.dOutVT) + base;
   const double beta = A.beta;
   long long carryW = 0;
+  long long wsum = 0, tsum = 0;   // E[WL] = sum_e W_e, E[TP] = sum_cells VD (rows pass), 2^-24 fixed point
   double carryS = 0.0, of = 0.0;
+  const int lane = threadIdx.x & 31;
   for (int c0 = 0; c0 < n; c0 += kGThreads * kGItems) {
     long long v[kGItems], t0[kGItems], t1[kGItems];
     float cp[kGItems];
@@ -1201,8 +1188,14 @@ __global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A)
       const int pos = c0 + j * kGThreads + threadIdx.x;
       v[j] = pos < n ? diff[pos] : 0;
       t0[j] = pos < n ? vd[(size_t)pos * vstep] : 0;
-      t1[j] = pos + 1 < n ? vd[(size_t)(pos + 1) * vstep] : 0;
       cp[j] = pos < n ? cap[pos] : 0.f;
+    }
+#pragma unroll
+    for (int j = 0; j < kGItems; ++j) {   // the next cell's turning points: the next lane's t0
+      const int pos = c0 + j * kGThreads + threadIdx.x;
+      t1[j] = __shfl_down_sync(kFull, t0[j], 1);
+      if (lane == 31) t1[j] = pos + 1 < n ? vd[(size_t)(pos + 1) * vstep] : 0;
+      if (isH) tsum += t0[j];
     }
     long long totW;
     long long ex[kGItems];
@@ -1221,6 +1214,7 @@ __global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A)
       double G = 0.0;
       if (pos < n - 1) {
         const long long W = carryW + ex[j] + v[j];   // inclusive prefix = wire demand of edge pos
+        wsum += W;
         const double d = (double)W * kFixInv + beta * ((double)(t0[j] + t1[j]) * kFixInv);
         const double x = d - (double)cp[j];                 // overflow x = -(cap - d)
         // f(x) and df/dx = df/dd in fp32 (x itself in fp64: d comes from exact fixed point);
@@ -1262,6 +1256,13 @@ __global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A)
     carryW += totW;
     carryS += totS;
   }
+  // E[WL], E[TP] partial sums (exact integers): warp reduction, one global reduction per warp
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {
+    wsum += __shfl_down_sync(kFull, wsum, off);
+    tsum += __shfl_down_sync(kFull, tsum, off);
+  }
+  if (lane == 0) { red64(P.scal, wsum); red64(P.scal + 1, tsum); }
   // deterministic block reduction of the overflow cost
   double tot;
   block_exclusive_scan(of, shd, &tot);
