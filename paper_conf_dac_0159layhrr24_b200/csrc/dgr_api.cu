@@ -208,6 +208,7 @@ struct Plan {
   PodBuf<uint32_t> pword;
   PodBuf<short4> sxy;                   // kernel order
   std::vector<int32_t> net_tree_off;
+  std::vector<int32_t> mnets;           // per tile: offsets of its nets with >= 2 trees (TileDesc mn0 / nmn)
   PodBuf<int32_t> ksub_csr;             // kernel-order sub-net -> local CSR sub-net
   PodBuf<int64_t> sub_first_slot;       // local CSR sub-net -> slot of its first candidate
   PodBuf<int32_t> slot_path;            // slot -> local CSR path (-1: padding)
@@ -493,15 +494,19 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   //    singleton bundles; sub-nets renumbered in that order ("kernel order").  Count per tile,
   //    prefix, then fill the tiles in parallel (each owns a contiguous bundle and sub-net range).
   const int64_t ntile = (int64_t)starts.size() - 1;
-  std::vector<int32_t> tb0(ntile + 1, 0), tbg(ntile, 0);
+  std::vector<int32_t> tb0(ntile + 1, 0), tbg(ntile, 0), tmn(ntile + 1, 0);
 #pragma omp parallel for schedule(dynamic, 64)
   for (int64_t t = 0; t < ntile; ++t) {
     Pack pk;
-    for (int64_t n = starts[t]; n < starts[t + 1]; ++n) pack_net(n, pk);
+    for (int64_t n = starts[t]; n < starts[t + 1]; ++n) {
+      pack_net(n, pk);
+      tmn[t + 1] += d->net_tree_off[n + 1] - d->net_tree_off[n] > 1;
+    }
     tbg[t] = pk.nbg;
     tb0[t + 1] = pk.total();
   }
-  for (int64_t t = 0; t < ntile; ++t) tb0[t + 1] += tb0[t];
+  for (int64_t t = 0; t < ntile; ++t) { tb0[t + 1] += tb0[t]; tmn[t + 1] += tmn[t]; }
+  pl.mnets.assign(tmn[ntile], 0);
   const size_t nslot = (size_t)tb0[ntile] * 32;
   // every element is written by the parallel fill below (padding slots included)
   pl.binfo.alloc(tb0[ntile]);
@@ -525,6 +530,10 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       T.ntree = (int32_t)(d->net_tree_off[starts[t + 1]] - d->net_tree_off[starts[t]]);
       T.b0 = tb0[t];
       T.nb = tb0[t + 1] - tb0[t];
+      T.mn0 = tmn[t];
+      T.nmn = tmn[t + 1] - tmn[t];
+      for (int64_t n = starts[t], k = T.mn0; n < starts[t + 1]; ++n)
+        if (d->net_tree_off[n + 1] - d->net_tree_off[n] > 1) pl.mnets[k++] = (int32_t)(n - starts[t]);
       T.nbg = tbg[t];
       T.global = globs[t];
       int bx0 = X, by0 = Y, bx1 = -1, by1 = -1;
@@ -660,8 +669,8 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
 // workspace layout
 // ---------------------------------------------------------------------------------------
 struct Layout {
-  size_t tiles, binfo, pword, sxy, slot_path, wp, mp, vp, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
-      partial, kg_count, loss, chosen, tree_choice, route, nsize, nucleus_tmp, DHVC, iscal, ipartial, metrics, total;
+  size_t tiles, mnets, binfo, pword, sxy, slot_path, wp, mp, vp, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
+      partial, lpart, loss, chosen, tree_choice, route, nsize, nucleus_tmp, DHVC, iscal, ipartial, metrics, total;
   size_t xcount;   // int64 elements in the exchange buffer
 };
 
@@ -672,6 +681,7 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   const size_t slots = (size_t)pl.nb * 32, ns = pl.sxy.size(), nt = (size_t)(pl.tree_hi - pl.tree_lo),
                nn = (size_t)(pl.net_hi - pl.net_lo), G = (size_t)X * Y;
   L.tiles = take(sizeof(TileDesc) * pl.tiles.size());
+  L.mnets = take(4 * pl.mnets.size() + 16);   // +16 B: 16-byte aligned bulk reads may run past the end
   L.binfo = take(sizeof(int4) * pl.nb);
   L.pword = take(4 * slots);
   L.sxy = take(8 * ns + 16);
@@ -697,7 +707,7 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.dOutH = take(4 * G);
   L.dOutVT = take(4 * G);
   L.partial = take(8 * (size_t)(X + Y));
-  L.kg_count = take(16);
+  L.lpart = take(16 * (size_t)(X + Y));
   L.loss = take(8 * 4);
   L.chosen = take(nt);
   L.tree_choice = take(4 * nn);
@@ -885,6 +895,11 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   P.tree_base = pl.tree_lo;
   P.nid_base = pl.nid_base;
   P.seed = desc->seed;
+  P.mnets = (const int32_t*)(ws + L.mnets);
+  for (int r = 0; r < 10; ++r) {   // Philox4x32-10 round keys of the seed
+    P.rk[2 * r] = (uint32_t)desc->seed + (uint32_t)r * 0x9E3779B9u;
+    P.rk[2 * r + 1] = (uint32_t)(desc->seed >> 32) + (uint32_t)r * 0xBB67AE85u;
+  }
   P.binfo = (const int4*)(ws + L.binfo);
   P.pword = (const uint32_t*)(ws + L.pword);
   P.sxy = (const short4*)(ws + L.sxy);
@@ -903,7 +918,7 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   P.SH = (double*)(ws + L.SH); P.SVT = (double*)(ws + L.SVT);
   P.dOutH = (float*)(ws + L.dOutH); P.dOutVT = (float*)(ws + L.dOutVT);
   P.partial = (double*)(ws + L.partial);
-  P.kg_count = (unsigned int*)(ws + L.kg_count);
+  P.lpart = (long long*)(ws + L.lpart);
   P.loss = (double*)(ws + L.loss);
   P.chosen = (uint8_t*)(ws + L.chosen);
   P.tree_choice = (int32_t*)(ws + L.tree_choice);
@@ -948,6 +963,7 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
     if (bytes && e == cudaSuccess) e = cudaMemcpyAsync(ws + off, src, bytes, cudaMemcpyHostToDevice, s);
   };
   cp(L.tiles, pl.tiles.data(), sizeof(TileDesc) * pl.tiles.size());
+  cp(L.mnets, pl.mnets.data(), 4 * pl.mnets.size());
   cp(L.binfo, pl.binfo.data(), sizeof(int4) * pl.nb);
   cp(L.pword, pl.pword.data(), 4 * slots);
   cp(L.sxy, pl.sxy.data(), 8 * pl.sxy.size());
@@ -1031,6 +1047,7 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
       if ((rc = prof_mark(h, 1))) return rc;
     }
     launch_kg(P, a, s);
+    if (last) launch_kg_loss(P, a, s);
     if ((rc = prof_mark(h, 2))) return rc;
     if (iters > 0) {
       // reverse of iteration k + forward of k+1 (also after the last iteration: the next call

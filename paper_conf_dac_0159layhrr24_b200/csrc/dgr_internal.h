@@ -50,6 +50,7 @@ constexpr int kTileBundles = kTargetBundles + 8;   // all bundles (group + singl
 constexpr int kTreeMax = 512;                      // trees per tile
 constexpr int kPipeTrees = 224;                    // trees per pipelined tile
 constexpr int kPipeSubs = 512;                     // sub-nets per pipelined tile
+constexpr int kKgWarps = 8;                        // warps per KG CTA (one line per CTA)
 constexpr int kEventMax = 127;                     // events per window cell-field (int32 safety)
 
 enum Shape : uint32_t {
@@ -71,7 +72,7 @@ struct TileDesc {
   int32_t wx0, wy0, ww, wh;  // window (cells; even origin and extents), unused for global tiles
   int32_t global, nbg;     // nbg: group bundles (the first nbg of the tile; the rest are singleton bundles)
   int32_t sub0, nsub;      // local sub-nets (kernel order within the tile)
-  int32_t pad2, pad3;
+  int32_t mn0, nmn;        // the tile's nets with >= 2 trees: mnets[mn0 .. mn0 + nmn) (net offsets in the tile)
 };
 
 struct KParams {
@@ -86,6 +87,7 @@ struct KParams {
   int64_t path_base, tree_base;   // global index of the first local path / tree
   int64_t nid_base;         // global noise index of the rank's first noisy candidate
   uint64_t seed;
+  uint32_t rk[20];          // Philox4x32-10 round keys of the seed (key + r (0x9E3779B9, 0xBB67AE85))
   // forest encoding
   const TileDesc* tiles;
   const TileDesc* tiles_slow;
@@ -96,6 +98,7 @@ struct KParams {
   float *wp, *mp, *vp;
   float* pp;                // p_i of the last forward (the reverse of that iteration reads it)
   const int32_t* net_tree_off;    // local, n_nets_l + 1
+  const int32_t* mnets;     // per tile: offsets (in the tile) of its nets with >= 2 trees
   float *wt, *mt, *vt, *q;
   // grids (the exchange buffer, in this order: dH | dVT | VD | scal)
   long long* dH;            // [Y][X]
@@ -108,8 +111,8 @@ struct KParams {
   double* SVT;              // [X][YP] (contiguous after SH)
   float* dOutH;             // [Y][X]
   float* dOutVT;            // [X][Y]
-  double* partial;          // [Y + X] overflow partial sums
-  unsigned int* kg_count;   // CTAs of the current KG launch that are done (the last one finalises)
+  double* partial;          // [Y + X] overflow partial sums per line
+  long long* lpart;         // [2 (Y + X)] per-line E[WL], E[TP] partial sums (2^-24 fixed point)
   double* loss;             // [4]
   // induce scratch
   uint8_t* chosen;          // [n_trees_l]
@@ -140,6 +143,7 @@ struct StepArgs {
 enum TileMode { kForwardOnly = 0, kReverseForward = 1, kReverseOnly = 2 };
 void launch_tiles(const KParams& p, const StepArgs& a, TileMode mode, cudaStream_t s);
 void launch_kg(const KParams& p, const StepArgs& a, cudaStream_t s);
+void launch_kg_loss(const KParams& p, const StepArgs& a, cudaStream_t s);   // the loss of the last KG
 void launch_induce(const KParams& p, float t_final, float top_p, float beta, cudaStream_t s);
 void launch_induce_metrics(const KParams& p, float beta, cudaStream_t s);
 int induce_metric_blocks(const KParams& p);

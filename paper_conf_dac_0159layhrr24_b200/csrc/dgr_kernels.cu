@@ -44,6 +44,17 @@ __device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint2 key) {
   return c;
 }
 
+// the same generator with the round keys precomputed on the host (KParams::rk, constant bank)
+__device__ __forceinline__ uint4 philox_rk(uint4 c, const uint32_t* rk) {
+#pragma unroll
+  for (int r = 0; r < 10; ++r) {
+    const uint32_t hi0 = __umulhi(0xD2511F53u, c.x), lo0 = 0xD2511F53u * c.x;
+    const uint32_t hi1 = __umulhi(0xCD9E8D57u, c.z), lo1 = 0xCD9E8D57u * c.z;
+    c = make_uint4(hi1 ^ c.y ^ rk[2 * r], lo1, hi0 ^ c.w ^ rk[2 * r + 1], lo0);
+  }
+  return c;
+}
+
 __device__ __forceinline__ float gumbel(uint64_t seed, uint64_t idx, uint32_t k, uint32_t stream) {
   const uint4 r = philox4x32_10(make_uint4((uint32_t)(idx >> 2), (uint32_t)(idx >> 34), k, stream),
                                 make_uint2((uint32_t)seed, (uint32_t)(seed >> 32)));
@@ -111,6 +122,21 @@ __device__ __forceinline__ float group_softmax(const KParams& P, float inv_t, ui
   float s = seg_reduce(e, L.lane, L.end, Sum());
   s = __shfl_sync(kFull, s, L.head);
   return L.valid ? e / s : 0.f;
+}
+
+// dq_j in 2^-32 fixed point, accumulated in shared memory as three 32-bit limbs (a 64-bit shared
+// atomic is a CAS loop on sm_100): v = hi 2^42 + mid 2^21 + lo with lo, mid in [0, 2^21) (up to 1024
+// contributions per tree cannot overflow a limb) and hi = v >> 42 signed; exact for any int64 v.
+__device__ __forceinline__ void dq_add(int* dq3, int tree, long long v) {
+  int* d = dq3 + 3 * tree;
+  atomicAdd(d, (int)(v & 0x1FFFFF));
+  atomicAdd(d + 1, (int)((v >> 21) & 0x1FFFFF));
+  atomicAdd(d + 2, (int)(v >> 42));
+}
+__device__ __forceinline__ double dq_get(const int* dq3, int tree) {
+  const int* d = dq3 + 3 * tree;
+  const long long v = ((long long)d[2] << 42) + ((long long)(unsigned)d[1] << 21) + (long long)(unsigned)d[0];
+  return (double)v * kDqInv;
 }
 
 __device__ __forceinline__ void red64(long long* p, long long v) {
@@ -567,11 +593,6 @@ __device__ __forceinline__ void slow_tile(const KParams& P, const StepArgs& A, c
   }
 }
 
-template <bool REV, bool FWD>
-__global__ void __launch_bounds__(kTileThreads, 3) tile_kernel(KParams P, StepArgs A) {
-  extern __shared__ __align__(128) unsigned char smem[];
-  slow_tile<REV, FWD>(P, A, P.tiles_slow[blockIdx.x], smem);
-}
 
 // ------------------------------------------------------------------------------------------
 // Persistent, TMA-pipelined tile kernel (the hot loop).  One CTA per SM walks its tiles
@@ -587,32 +608,21 @@ constexpr int kPSubMax = kPipeSubs + 2;                     // + alignment slack
 constexpr int kPTreeMax = kPipeTrees + 4;
 constexpr int kPNetMax = kPipeTrees + 8;
 
-// Slim stage (default): the Adam moments m, v and the stored p of the paths, and m, v of the trees,
-// stay in global memory (each warp reads / writes its bundle's 128-byte rows directly); the stage
-// keeps what several phases share.  The smaller stage fits 5 CTAs per SM instead of 4.
-#ifndef DGR_SLIM_STAGE
-#define DGR_SLIM_STAGE 1
-#endif
-constexpr bool kSlim = DGR_SLIM_STAGE != 0;
-// Lean stage: the pattern words and logits of the paths are read (and w written) directly too.
-#ifndef DGR_LEAN_STAGE
-#define DGR_LEAN_STAGE 0
-#endif
-constexpr bool kLean = kSlim && DGR_LEAN_STAGE != 0;
+// The stage keeps what several phases share: pattern words and logits of the tile's slots, bundle
+// info, sub-net endpoints, net->tree offsets, the multi-tree net list, tree logits and q, and the S
+// window.  Adam moments and the stored p of the paths, and m, v of the trees, are read / written
+// directly (each warp its bundle's 128-byte rows), so the stage fits 5 CTAs per SM.
+constexpr int kPMnMax = kPipeTrees / 2 + 4;                 // nets with >= 2 trees per tile (+ slack)
 struct StageLayout {
   static constexpr size_t pw = 0;
-  static constexpr size_t w = pw + (kLean ? 0 : 4 * 32 * kTileBundles);
-  static constexpr size_t m = w + (kLean ? 0 : 4 * kPSlots);
-  static constexpr size_t v = m + (kSlim ? 0 : 4 * kPSlots);
-  static constexpr size_t p = v + (kSlim ? 0 : 4 * kPSlots);
-  static constexpr size_t bi = p + (kSlim ? 0 : 4 * kPSlots);
+  static constexpr size_t w = pw + 4 * 32 * kTileBundles;
+  static constexpr size_t bi = w + 4 * kPSlots;
   static constexpr size_t sxy = bi + 16 * kTileBundles;
   static constexpr size_t nto = sxy + 8 * kPSubMax;
-  static constexpr size_t q = (nto + 4 * kPNetMax + 15) / 16 * 16;
+  static constexpr size_t mn = (nto + 4 * kPNetMax + 15) / 16 * 16;
+  static constexpr size_t q = (mn + 4 * kPMnMax + 15) / 16 * 16;
   static constexpr size_t wt = q + 4 * kPTreeMax;
-  static constexpr size_t mt = wt + 4 * kPTreeMax;
-  static constexpr size_t vt = mt + (kSlim ? 0 : 4 * kPTreeMax);
-  static constexpr size_t S = (vt + (kSlim ? 0 : 4 * kPTreeMax) + 127) / 128 * 128;
+  static constexpr size_t S = (wt + 4 * kPTreeMax + 127) / 128 * 128;
   static constexpr size_t bytes = S + 2 * 8 * kWinMax;
 };
 
@@ -640,30 +650,26 @@ __device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t by
 }
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
-__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
 struct Stage {
-  uint32_t* pw; float *w, *m, *v, *p;
-  int4* bi; short4* sxy; int* nto; float *q, *wt, *mt, *vt; double* S;
+  uint32_t* pw; float* w;
+  int4* bi; short4* sxy; int *nto, *mn; float *q, *wt; double* S;
   __device__ __forceinline__ explicit Stage(unsigned char* base) {
     pw = reinterpret_cast<uint32_t*>(base + StageLayout::pw);
     w = reinterpret_cast<float*>(base + StageLayout::w);
-    m = reinterpret_cast<float*>(base + StageLayout::m);
-    v = reinterpret_cast<float*>(base + StageLayout::v);
-    p = reinterpret_cast<float*>(base + StageLayout::p);
     bi = reinterpret_cast<int4*>(base + StageLayout::bi);
     sxy = reinterpret_cast<short4*>(base + StageLayout::sxy);
     nto = reinterpret_cast<int*>(base + StageLayout::nto);
+    mn = reinterpret_cast<int*>(base + StageLayout::mn);
     q = reinterpret_cast<float*>(base + StageLayout::q);
     wt = reinterpret_cast<float*>(base + StageLayout::wt);
-    mt = reinterpret_cast<float*>(base + StageLayout::mt);
-    vt = reinterpret_cast<float*>(base + StageLayout::vt);
     S = reinterpret_cast<double*>(base + StageLayout::S);
   }
 };
 
-// aligned element ranges of a tile's sub-nets / nets / trees (16-byte bulk granularity)
+// aligned element ranges of a tile's sub-nets / nets / multi-tree nets / trees (16-byte bulk
+// granularity)
 __device__ __forceinline__ void tile_ranges(const TileDesc& T, int& s_lo, int& s_hi, int& n_lo, int& n_hi, int& t_lo, int& t_hi) {
   s_lo = T.sub0 & ~1; s_hi = (T.sub0 + T.nsub + 1) & ~1;
   n_lo = T.net0 & ~3; n_hi = (T.net0 + T.nnet + 1 + 3) & ~3;
@@ -677,37 +683,33 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
   Stage S(st);
   int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
+  const int mn_lo = T.mn0 & ~3, mn_hi = (T.mn0 + T.nmn + 3) & ~3;
   const uint32_t slot_bytes = (uint32_t)T.nb * 128u, gslot_bytes = (uint32_t)T.nbg * 128u;
   const uint32_t nrow = REV ? (uint32_t)T.wh : 0u, ncol = REV ? (uint32_t)T.ww : 0u;
-  const uint32_t bytes = (kLean ? 0u : slot_bytes + gslot_bytes * (REV && !kSlim ? 4u : 1u)) + 16u * T.nb + 8u * (s_hi - s_lo) +
-                         4u * (n_hi - n_lo) + 4u * (t_hi - t_lo) * (kSlim ? (REV ? 2u : 1u) : (REV ? 4u : 3u)) +
-                         8u * (nrow * T.ww + ncol * T.wh);
+  const uint32_t bytes = slot_bytes + gslot_bytes + 16u * T.nb + 8u * (s_hi - s_lo) + 4u * (n_hi - n_lo) +
+                         4u * (mn_hi - mn_lo) + 8u * (t_hi - t_lo) + 8u * (nrow * T.ww + ncol * T.wh);
   if (lane == 0) mbar_expect_tx(bar, bytes);
   __syncwarp();
   const size_t s0 = (size_t)T.b0 * 32;
-  // work items: 0..9 the 1-D arrays, then window rows, then window columns
-  const int nitems = 10 + (int)nrow + (int)ncol;
+  // work items: 0..7 the 1-D arrays, then window rows, then window columns
+  const int nitems = 8 + (int)nrow + (int)ncol;
   for (int it = lane; it < nitems; it += 32) {
-    if (it < 10) {
+    if (it < 8) {
       switch (it) {
-        case 0: if (!kLean) bulk_g2s(S.pw, P.pword + s0, slot_bytes, bar); break;
-        case 1: if (!kLean && gslot_bytes) bulk_g2s(S.w, P.wp + s0, gslot_bytes, bar); break;
-        case 2: if (!kSlim && REV && gslot_bytes) bulk_g2s(S.m, P.mp + s0, gslot_bytes, bar); break;
-        case 3: if (!kSlim && REV && gslot_bytes) bulk_g2s(S.v, P.vp + s0, gslot_bytes, bar); break;
-        case 4: if (!kSlim && REV && gslot_bytes) bulk_g2s(S.p, P.pp + s0, gslot_bytes, bar); break;
-        case 5: bulk_g2s(S.bi, P.binfo + T.b0, 16u * T.nb, bar); break;
-        case 6: bulk_g2s(S.sxy, P.sxy + s_lo, 8u * (s_hi - s_lo), bar); break;
-        case 7: bulk_g2s(S.nto, P.net_tree_off + n_lo, 4u * (n_hi - n_lo), bar); break;
-        case 8: bulk_g2s(S.wt, P.wt + t_lo, 4u * (t_hi - t_lo), bar);
-                if (!kSlim) bulk_g2s(S.mt, P.mt + t_lo, 4u * (t_hi - t_lo), bar); break;
-        default: if (!kSlim) bulk_g2s(S.vt, P.vt + t_lo, 4u * (t_hi - t_lo), bar);
-                 if (REV) bulk_g2s(S.q, P.q + t_lo, 4u * (t_hi - t_lo), bar); break;
+        case 0: bulk_g2s(S.pw, P.pword + s0, slot_bytes, bar); break;
+        case 1: if (gslot_bytes) bulk_g2s(S.w, P.wp + s0, gslot_bytes, bar); break;
+        case 2: bulk_g2s(S.bi, P.binfo + T.b0, 16u * T.nb, bar); break;
+        case 3: bulk_g2s(S.sxy, P.sxy + s_lo, 8u * (s_hi - s_lo), bar); break;
+        case 4: bulk_g2s(S.nto, P.net_tree_off + n_lo, 4u * (n_hi - n_lo), bar); break;
+        case 5: if (mn_hi > mn_lo) bulk_g2s(S.mn, P.mnets + mn_lo, 4u * (mn_hi - mn_lo), bar); break;
+        case 6: bulk_g2s(S.wt, P.wt + t_lo, 4u * (t_hi - t_lo), bar); break;
+        default: bulk_g2s(S.q, P.q + t_lo, 4u * (t_hi - t_lo), bar); break;   // also a lone tree's q = 1
       }
-    } else if (it < 10 + (int)nrow) {
-      const int yi = it - 10;
+    } else if (it < 8 + (int)nrow) {
+      const int yi = it - 8;
       bulk_g2s(S.S + (size_t)yi * T.ww, P.SH + (size_t)(T.wy0 + yi) * P.XP + T.wx0, 8u * T.ww, bar);
     } else {
-      const int xi = it - 10 - (int)nrow;
+      const int xi = it - 8 - (int)nrow;
       bulk_g2s(S.S + (size_t)T.ww * T.wh + (size_t)xi * T.wh, P.SVT + (size_t)(T.wx0 + xi) * P.YP + T.wy0, 8u * T.wh, bar);
     }
   }
@@ -721,13 +723,14 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
 constexpr size_t kGpOffset = 3 * 4 * kWinMax;   // tile path noise, after the event window in St.S
 template <bool REV, bool FWD, int NT>
 __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A, const TileDesc& T, Stage St,
-                                             int* ev_s, float* gp, long long* dq_s, long long* red_s) {
-  // dq_s[0..ntree) and red_s[0..2) arrive zeroed (the caller clears them before its first barrier)
+                                             int* ev_s, float* gp, int* dq3) {
+  // dq3[0..3 ntree) arrives zeroed (the caller clears it before its first barrier)
   constexpr int NW = NT / 32;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int X = P.X, Y = P.Y;
   int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
+  const int mn_lo = T.mn0 & ~3;
   const int ncell = T.ww * T.wh;
   const Win W{T.wx0, T.wy0, T.ww, T.wh, ncell};
   const int wB0 = -(T.wy0 * T.ww + T.wx0), wB1 = ncell - T.wx0 * T.wh - T.wy0;   // orientation bases
@@ -735,18 +738,18 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   const int nbg = T.nbg;
 
   // ---------------- reverse of iteration k ----------------
-  if (REV) {   // dq_s was zeroed before the stage arrived
+  if (REV) {   // dq3 was zeroed before the stage arrived
     for (int lb = warp; lb < T.nb; lb += NW) {
       const int4 bi = St.bi[lb];
-      const uint32_t pw = kLean ? P.pword[(size_t)(T.b0 + lb) * 32 + lane] : St.pw[lb * 32 + lane];
+      const uint32_t pw = St.pw[lb * 32 + lane];
       if (lb < nbg) {
         Lane L;
         lane_from(bi, pw, P, L);
         const int sl = lb * 32 + lane;
         const size_t gsl = (size_t)T.b0 * 32 + sl;
-        float w = kLean ? P.wp[gsl] : St.w[sl];
-        float m = kSlim ? P.mp[gsl] : St.m[sl], v = kSlim ? P.vp[gsl] : St.v[sl];
-        const float p = kSlim ? P.pp[gsl] : St.p[sl];
+        float w = St.w[sl];
+        float m = P.mp[gsl], v = P.vp[gsl];
+        const float p = P.pp[gsl];
         const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
         double c = 0.0;
         if (L.valid && !(P.skip & 8)) {
@@ -763,12 +766,11 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         sa = __shfl_sync(kFull, sa, L.head);
         const float dw = L.valid ? p * A.inv_t * q * (dd - sa) : 0.f;
         if (L.valid && L.lane == L.head)
-          atomicAdd(reinterpret_cast<unsigned long long*>(&dq_s[L.tree - T.tree0]),
-                    static_cast<unsigned long long>(__double2ll_rn((c + (double)sa) * kDqScale)));
+          dq_add(dq3, L.tree - T.tree0, __double2ll_rn((c + (double)sa) * kDqScale));
         if (L.valid) {
           adam_update(w, m, v, dw, A);
-          if (kLean) P.wp[gsl] = w; else St.w[sl] = w;
-          if (kSlim) { P.mp[gsl] = m; P.vp[gsl] = v; } else { St.m[sl] = m; St.v[sl] = v; }
+          St.w[sl] = w;
+          P.mp[gsl] = m; P.vp[gsl] = v;
         }
       } else {
         // singleton bundle: c of a straight path (one segment, no turning point); p = 1
@@ -788,8 +790,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         const int tend = trest ? (__ffs(trest) - 2) : 31;
         const double pc = seg_reduce(c, lane, tend, Sum());
         if (valid && ((th >> lane) & 1u))
-          atomicAdd(reinterpret_cast<unsigned long long*>(&dq_s[tree - T.tree0]),
-                    static_cast<unsigned long long>(__double2ll_rn(pc * kDqScale)));
+          dq_add(dq3, tree - T.tree0, __double2ll_rn(pc * kDqScale));
       }
     }
     __syncthreads();
@@ -800,56 +801,51 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     int4* z = reinterpret_cast<int4*>(ev_s);   // the S window is free after the reverse
     for (int i = tid; i < (3 * ncell + 3) / 4; i += NT) z[i] = make_int4(0, 0, 0, 0);
   }
-  if (!(P.skip & 16)) {
-    const uint2 key = make_uint2((uint32_t)P.seed, (uint32_t)(P.seed >> 32));
-    for (int n = tid; n < T.nnet; n += NT) {
-      const int a = St.nto[T.net0 + n - n_lo] - t_lo, b = St.nto[T.net0 + n + 1 - n_lo] - t_lo;   // stage indices
-      if (b - a == 1) {
-        // a lone tree: q = 1 and du = 0 always (its logit and Adam state never change)
-        if (FWD) St.q[a] = 1.f;
-        continue;
+  // the tile's nets with >= 2 trees (a lone tree has q = 1 and du = 0 always: its logit and Adam
+  // state never change, and its q = 1 arrives with the stage)
+  for (int i = tid; i < T.nmn; i += NT) {
+    const int n = St.mn[T.mn0 + i - mn_lo];
+    const int a = St.nto[T.net0 + n - n_lo] - t_lo, b = St.nto[T.net0 + n + 1 - n_lo] - t_lo;   // stage indices
+    if (REV) {
+      // du_j = (q_j/t)(dq_j - sum_l q_l dq_l / sum_l q_l); Adam on w_tree (iteration k)
+      double sq = 0.0, sw = 0.0;
+      for (int l = a; l < b; ++l) {
+        const double ql = (double)St.q[l];
+        sq += ql * dq_get(dq3, l + t_lo - T.tree0);
+        sw += ql;
       }
-      if (REV) {
-        // du_j = (q_j/t)(dq_j - sum_l q_l dq_l / sum_l q_l); Adam on w_tree (iteration k)
-        double sq = 0.0, sw = 0.0;
-        for (int l = a; l < b; ++l) {
-          const double ql = (double)St.q[l];
-          sq += ql * ((double)dq_s[l + t_lo - T.tree0] * kDqInv);
-          sw += ql;
-        }
-        sq /= sw;
-        for (int j = a; j < b; ++j) {
-          const double du = (double)St.q[j] * (double)A.inv_t * ((double)dq_s[j + t_lo - T.tree0] * kDqInv - sq);
-          float w = St.wt[j], m = kSlim ? P.mt[j + t_lo] : St.mt[j], v = kSlim ? P.vt[j + t_lo] : St.vt[j];
-          adam_update(w, m, v, (float)du, A);
-          St.wt[j] = w;
-          const int jg = j + t_lo;
-          P.wt[jg] = w; P.mt[jg] = m; P.vt[jg] = v;
-        }
+      sq /= sw;
+      for (int j = a; j < b; ++j) {
+        const double du = (double)St.q[j] * (double)A.inv_t * (dq_get(dq3, j + t_lo - T.tree0) - sq);
+        const int jg = j + t_lo;
+        float w = St.wt[j], m = P.mt[jg], v = P.vt[jg];
+        adam_update(w, m, v, (float)du, A);
+        St.wt[j] = w;
+        P.wt[jg] = w; P.mt[jg] = m; P.vt[jg] = v;
       }
-      if (FWD) {
-        // q_j = softmax over the net's trees of (w_j + g_j)/t, iteration k_next (noise stream 1)
-        float zmax = -INFINITY;
-        int64_t cq = -1;   // one Philox call per aligned quad of tree indices
-        uint4 r = make_uint4(0u, 0u, 0u, 0u);
-        for (int j = a; j < b; ++j) {
-          const int64_t gj = P.tree_base + t_lo + j;
-          if ((gj >> 2) != cq) {
-            cq = gj >> 2;
-            r = philox4x32_10(make_uint4((uint32_t)cq, (uint32_t)(cq >> 32), (uint32_t)A.k_next, 1u), key);
-          }
-          const uint32_t wd = (gj & 3) == 0 ? r.x : (gj & 3) == 1 ? r.y : (gj & 3) == 2 ? r.z : r.w;
-          const float zj = (St.wt[j] + gumbel_word(wd)) * A.inv_t;
-          St.q[j] = zj;
-          zmax = fmaxf(zmax, zj);
+    }
+    if (FWD) {
+      // q_j = softmax over the net's trees of (w_j + g_j)/t, iteration k_next (noise stream 1)
+      float zmax = -INFINITY;
+      int64_t cq = -1;   // one Philox call per aligned quad of tree indices
+      uint4 r = make_uint4(0u, 0u, 0u, 0u);
+      for (int j = a; j < b; ++j) {
+        const int64_t gj = P.tree_base + t_lo + j;
+        if ((gj >> 2) != cq) {
+          cq = gj >> 2;
+          r = philox_rk(make_uint4((uint32_t)cq, (uint32_t)(cq >> 32), (uint32_t)A.k_next, 1u), P.rk);
         }
-        float sum = 0.f;
-        for (int j = a; j < b; ++j) sum += __expf(St.q[j] - zmax);
-        for (int j = a; j < b; ++j) {
-          const float q = __expf(St.q[j] - zmax) / sum;
-          St.q[j] = q;
-          P.q[j + t_lo] = q;
-        }
+        const uint32_t wd = (gj & 3) == 0 ? r.x : (gj & 3) == 1 ? r.y : (gj & 3) == 2 ? r.z : r.w;
+        const float zj = (St.wt[j] + gumbel_word(wd)) * A.inv_t;
+        St.q[j] = zj;
+        zmax = fmaxf(zmax, zj);
+      }
+      float sum = 0.f;
+      for (int j = a; j < b; ++j) sum += __expf(St.q[j] - zmax);
+      for (int j = a; j < b; ++j) {
+        const float q = __expf(St.q[j] - zmax) / sum;
+        St.q[j] = q;
+        P.q[j + t_lo] = q;
       }
     }
   }
@@ -860,9 +856,8 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     const int4 bl = St.bi[nbg - 1];
     const int nn = bl.x + (bl.w & 0xff) - St.bi[0].x;
     const int64_t c0 = n0 >> 2, c1 = (n0 + nn - 1) >> 2;
-    const uint2 key = make_uint2((uint32_t)P.seed, (uint32_t)(P.seed >> 32));
     for (int64_t c = c0 + tid; c <= c1; c += NT) {
-      const uint4 r = philox4x32_10(make_uint4((uint32_t)c, (uint32_t)(c >> 32), (uint32_t)A.k_next, 0u), key);
+      const uint4 r = philox_rk(make_uint4((uint32_t)c, (uint32_t)(c >> 32), (uint32_t)A.k_next, 0u), P.rk);
       const uint32_t wd[4] = {r.x, r.y, r.z, r.w};
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
@@ -879,15 +874,15 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     const int nid0 = nbg > 0 ? St.bi[0].x : 0;
     for (int lb = warp; lb < T.nb; lb += NW) {
       const int4 bi = St.bi[lb];
-      const uint32_t pw = kLean ? P.pword[(size_t)(T.b0 + lb) * 32 + lane] : St.pw[lb * 32 + lane];
+      const uint32_t pw = St.pw[lb * 32 + lane];
       if (lb < nbg) {
         Lane L;
         lane_from(bi, pw, P, L);
         const int sl = lb * 32 + lane;
-        const float w = kLean ? P.wp[(size_t)T.b0 * 32 + sl] : St.w[sl];
+        const float w = St.w[sl];
         const float g = L.valid ? gp[bi.x + lane - nid0] : 0.f;
         const float p = softmax_from_noise(L, w, g, A.inv_t);
-        if (kSlim) P.pp[(size_t)T.b0 * 32 + sl] = p; else St.p[sl] = p;
+        P.pp[(size_t)T.b0 * 32 + sl] = p;
         const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
         const int vq = L.valid ? __float2int_rn(q * p * kFixScale) : 0;
         if (L.valid && !(P.skip & 4)) {
@@ -938,14 +933,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     fence_proxy_async();
     const size_t s0 = (size_t)T.b0 * 32;
     const uint32_t gslot_bytes = (uint32_t)nbg * 128u;
-    if (REV && !kLean) {
-      bulk_s2g(P.wp + s0, St.w, gslot_bytes);
-      if (!kSlim) {
-        bulk_s2g(P.mp + s0, St.m, gslot_bytes);
-        bulk_s2g(P.vp + s0, St.v, gslot_bytes);
-      }
-    }
-    if (FWD && !kSlim) bulk_s2g(P.pp + s0, St.p, gslot_bytes);
+    if (REV) bulk_s2g(P.wp + s0, St.w, gslot_bytes);
     bulk_commit();
   }
   if (FWD && !(P.skip & 1)) {
@@ -983,21 +971,19 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
 #endif
 constexpr int kBThreads = DGR_BTHREADS;
 #ifndef DGR_BPERSM
-#define DGR_BPERSM (DGR_SLIM_STAGE ? (DGR_LEAN_STAGE ? 6 : 5) : 4)
+#define DGR_BPERSM 5
 #endif
 constexpr int kBPerSM = DGR_BPERSM;
-constexpr size_t kBSmemBytes = (StageLayout::bytes + 8 * kPipeTrees + 64) > kSmemBytes ? (StageLayout::bytes + 8 * kPipeTrees + 64)
-                                                                                      : kSmemBytes;
+constexpr size_t kTailBytes = 12 * kPipeTrees + 16;   // dq limbs, mbarrier
+constexpr size_t kBSmemBytes = (StageLayout::bytes + kTailBytes) > kSmemBytes ? (StageLayout::bytes + kTailBytes) : kSmemBytes;
 static_assert(kGpOffset + 4 * 32 * kTargetBundles <= 2 * 8 * kWinMax, "event window + path noise must fit the S window");
-static_assert(8 * kPipeTrees + 12 * kPipeTrees + 32 + 4 * kPipeTrees <= kGpOffset, "tree scratch must not overlap the path noise");
 
 template <bool REV, bool FWD>
 __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepArgs A) {
   extern __shared__ __align__(128) unsigned char smem[];
   Stage St(smem);
-  long long* dq_s = reinterpret_cast<long long*>(smem + StageLayout::bytes);
-  long long* red_s = dq_s + kPipeTrees;
-  uint64_t* bar = reinterpret_cast<uint64_t*>(red_s + 2);
+  int* dq3 = reinterpret_cast<int*>(smem + StageLayout::bytes);
+  uint64_t* bar = reinterpret_cast<uint64_t*>(dq3 + 3 * kPipeTrees);
   if ((int)blockIdx.x < P.ntiles_slow) {   // global tiles first: the longest CTAs start earliest
     slow_tile<REV, FWD>(P, A, P.tiles_slow[blockIdx.x], smem);
     return;
@@ -1009,57 +995,12 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
     mbar_init(bar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  for (int i = threadIdx.x; i < kPipeTrees; i += kBThreads) dq_s[i] = 0;
-  if (threadIdx.x < 2) red_s[threadIdx.x] = 0;
+  for (int i = threadIdx.x; i < 3 * kPipeTrees; i += kBThreads) dq3[i] = 0;
   __syncthreads();
   if (threadIdx.x < 32) issue_tile_loads<REV>(P, T, smem, bar);
   mbar_wait(bar, 0u);
-  process_tile<REV, FWD, kBThreads>(P, A, T, St, ev_s, gp, dq_s, red_s);
+  process_tile<REV, FWD, kBThreads>(P, A, T, St, ev_s, gp, dq3);
   if (threadIdx.x == 0) bulk_wait_read();   // the stage must outlive the bulk stores' reads
-}
-
-// (b) persistent, double-buffered: 2 CTAs per SM walk the tiles (blockIdx.x, +gridDim.x, ...); tile
-// i+1 streams into the other stage while tile i computes.  The event window and noise alias the
-// current stage's S window, as in (a).
-constexpr int kPThreads = 256;
-constexpr int kPPerSM = 2;
-constexpr size_t kPSmemBytes = 2 * StageLayout::bytes + 8 * kPipeTrees + 64;
-
-template <bool REV, bool FWD>
-__global__ void __launch_bounds__(kPThreads, kPPerSM) tile_persistent(KParams P, StepArgs A) {
-  extern __shared__ __align__(128) unsigned char smem[];
-  unsigned char* stage_base[2] = {smem, smem + StageLayout::bytes};
-  long long* dq_s = reinterpret_cast<long long*>(smem + 2 * StageLayout::bytes);
-  long long* red_s = dq_s + kPipeTrees;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(red_s + 2);
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  if (tid == 0) {
-    mbar_init(&bars[0], 1);
-    mbar_init(&bars[1], 1);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  if (warp == 0 && (int)blockIdx.x < P.ntiles) issue_tile_loads<REV>(P, P.tiles[blockIdx.x], stage_base[0], &bars[0]);
-  for (int it = 0;; ++it) {
-    const int tile = blockIdx.x + it * gridDim.x;
-    if (tile >= P.ntiles) break;
-    const int sidx = it & 1;
-    if (warp == 0 && tile + (int)gridDim.x < P.ntiles) {
-      if (lane == 0) bulk_wait_read();   // the other stage's previous write-back has been read
-      __syncwarp();
-      issue_tile_loads<REV>(P, P.tiles[tile + gridDim.x], stage_base[sidx ^ 1], &bars[sidx ^ 1]);
-    }
-    for (int i = tid; i < kPipeTrees; i += kPThreads) dq_s[i] = 0;
-    if (tid < 2) red_s[tid] = 0;
-    __syncthreads();
-    mbar_wait(&bars[sidx], (uint32_t)(it >> 1) & 1u);
-    Stage St(stage_base[sidx]);
-    int* ev_s = reinterpret_cast<int*>(St.S);
-    float* gp = reinterpret_cast<float*>(reinterpret_cast<unsigned char*>(St.S) + kGpOffset);
-    process_tile<REV, FWD, kPThreads>(P, A, P.tiles[tile], St, ev_s, gp, dq_s, red_s);
-    __syncthreads();
-  }
-  if (tid == 0) bulk_wait_all();
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1068,7 +1009,7 @@ __global__ void __launch_bounds__(kPThreads, kPPerSM) tile_persistent(KParams P,
 // f(cap - d) (Eq. (9)); G = dcost/dd = -a3 f'(cap - d); S = exclusive prefix of G (fp64).
 // The line's difference entries are cleared for the next forward (VD is cleared by a memset).
 // ------------------------------------------------------------------------------------------
-constexpr int kGThreads = 256;
+constexpr int kGThreads = 32 * kKgWarps;
 constexpr int kGItems = 4;
 
 template <typename T>
@@ -1113,6 +1054,7 @@ __device__ __forceinline__ T warp_inclusive_scan(T x, int lane) {
 // Exclusive scan of a chunk of kGThreads * kGItems elements held "striped": thread t holds
 // elements j * kGThreads + t (j < kGItems), so every global access is coalesced.  Warp scans of
 // each item, then one warp scans the kGItems * NW warp totals (in position order), two barriers.
+// The caller puts a barrier between two uses of the same sh.
 template <typename T>
 __device__ __forceinline__ void striped_exclusive_scan(T (&v)[kGItems], T* sh /* kGItems*32 */, T* total) {
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -1136,33 +1078,43 @@ __device__ __forceinline__ void striped_exclusive_scan(T (&v)[kGItems], T* sh /*
 #pragma unroll
   for (int j = 0; j < kGItems; ++j) v[j] = sh[j * NW + wid] + inc[j] - v[j];   // exclusive
   *total = sh[32];
-  __syncthreads();
+  // no trailing barrier: the caller separates reuses of sh (the next chunk of a line) by one
 }
 
-__device__ __forceinline__ void kg_finalize(const KParams& P, const StepArgs& A) {
-  __shared__ double sh[32];
+// The loss of the last KG launch (Eqs. (9), (11), (12)): sums of the per-line partials in line
+// order (deterministic).  One CTA, launched once per dgr_step call after its last KG.
+__global__ void __launch_bounds__(256) kg_loss_kernel(KParams P, StepArgs A) {
+  __shared__ double sh[33];
+  __shared__ long long shl[33];
   const int nl = P.X + P.Y;
   double s = 0.0;
-  for (int i = threadIdx.x; i < nl; i += blockDim.x) s += __ldcg(&P.partial[i]);
+  long long w = 0, t = 0;
+  for (int i = threadIdx.x; i < nl; i += blockDim.x) {
+    s += P.partial[i];
+    w += P.lpart[2 * i];
+    t += P.lpart[2 * i + 1];
+  }
   double tot;
+  long long wt, tt;
   block_exclusive_scan(s, sh, &tot);
+  block_exclusive_scan(w, shl, &wt);
+  block_exclusive_scan(t, shl, &tt);
   if (threadIdx.x == 0) {
-    const double ewl = (double)__ldcg(&P.scal[0]) * kFixInv;
-    const double etp = (double)__ldcg(&P.scal[1]) * kFixInv;
+    const double ewl = (double)wt * kFixInv;
+    const double etp = (double)tt * kFixInv;
     const double via = (double)A.sqrt_l * etp;
     P.loss[0] = (double)A.a_wl * ewl + (double)A.a_via * via + (double)A.a_of * tot;
     P.loss[1] = ewl;
     P.loss[2] = via;
     P.loss[3] = tot;
-    P.scal[0] = 0;
-    P.scal[1] = 0;
-    *P.kg_count = 0;
   }
 }
 
 __global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A) {
   __shared__ long long shl[33];
   __shared__ double shd[33];
+  __shared__ double shw[kKgWarps];
+  __shared__ long long shwl[2 * kKgWarps];
   const int line = blockIdx.x;
   const bool isH = line < P.Y;
   const int n = isH ? P.X : P.Y;
@@ -1255,26 +1207,32 @@ __global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A)
     }
     carryW += totW;
     carryS += totS;
+    if (c0 + kGThreads * kGItems < n) __syncthreads();   // the next chunk reuses shl / shd
   }
-  // E[WL], E[TP] partial sums (exact integers): warp reduction, one global reduction per warp
+  // per-line partials of the overflow cost and of E[WL], E[TP] (exact integers): warp sums, then
+  // thread 0 sums the warps in order (deterministic); kg_loss_kernel sums the lines
 #pragma unroll
   for (int off = 16; off > 0; off >>= 1) {
+    of += __shfl_down_sync(kFull, of, off);
     wsum += __shfl_down_sync(kFull, wsum, off);
     tsum += __shfl_down_sync(kFull, tsum, off);
   }
-  if (lane == 0) { red64(P.scal, wsum); red64(P.scal + 1, tsum); }
-  // deterministic block reduction of the overflow cost
-  double tot;
-  block_exclusive_scan(of, shd, &tot);
-  // the last CTA to finish sums the per-line partials in line order and writes the loss
-  __shared__ bool last;
-  if (threadIdx.x == 0) {
-    P.partial[line] = tot;
-    __threadfence();
-    last = atomicAdd(P.kg_count, 1u) == gridDim.x - 1;
+  if (lane == 0) {
+    const int w = threadIdx.x >> 5;
+    shw[w] = of;
+    shwl[2 * w] = wsum;
+    shwl[2 * w + 1] = tsum;
   }
   __syncthreads();
-  if (last) kg_finalize(P, A);
+  if (threadIdx.x == 0) {
+    double tot = 0.0;
+    long long ws = 0, ts = 0;
+#pragma unroll
+    for (int w = 0; w < kKgWarps; ++w) { tot += shw[w]; ws += shwl[2 * w]; ts += shwl[2 * w + 1]; }
+    P.partial[line] = tot;
+    P.lpart[2 * line] = ws;
+    P.lpart[2 * line + 1] = ts;
+  }
 }
 
 
@@ -1401,58 +1359,31 @@ __global__ void ki_finalize_kernel(KParams P, int nblocks) {
 static inline int cdiv(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
 
 static int g_num_sms = 148;
-static bool g_persistent = false;   // DGR_TILE_PERSISTENT=1 selects driver (b)
 
-size_t tile_smem_bytes() { return kSmemBytes; }
+size_t tile_smem_bytes() { return kBSmemBytes; }
 
 int prepare_kernels() {
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
-  const char* env = getenv("DGR_TILE_PERSISTENT");
-  g_persistent = env && env[0] == '1';
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(tile_bulk<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBSmemBytes);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(tile_bulk<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBSmemBytes);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(tile_bulk<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBSmemBytes);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(tile_persistent<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPSmemBytes);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(tile_persistent<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPSmemBytes);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(tile_persistent<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPSmemBytes);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(tile_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(tile_kernel<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(tile_kernel<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   return (int)e;
 }
 
 void launch_tiles(const KParams& p, const StepArgs& a, TileMode mode, cudaStream_t s) {
-  if (p.ntiles > 0) {
-    if (g_persistent) {
-      const int grid = p.ntiles < kPPerSM * g_num_sms ? p.ntiles : kPPerSM * g_num_sms;
-      if (mode == kForwardOnly) tile_persistent<false, true><<<grid, kPThreads, kPSmemBytes, s>>>(p, a);
-      else if (mode == kReverseForward) tile_persistent<true, true><<<grid, kPThreads, kPSmemBytes, s>>>(p, a);
-      else tile_persistent<true, false><<<grid, kPThreads, kPSmemBytes, s>>>(p, a);
-    } else {   // one launch: global tiles in the first CTAs, then the pipelined tiles
-      const int grid = p.ntiles + p.ntiles_slow;
-      if (mode == kForwardOnly) tile_bulk<false, true><<<grid, kBThreads, kBSmemBytes, s>>>(p, a);
-      else if (mode == kReverseForward) tile_bulk<true, true><<<grid, kBThreads, kBSmemBytes, s>>>(p, a);
-      else tile_bulk<true, false><<<grid, kBThreads, kBSmemBytes, s>>>(p, a);
-      return;
-    }
-  }
-  if (p.ntiles_slow > 0) {
-    if (mode == kForwardOnly) tile_kernel<false, true><<<p.ntiles_slow, kTileThreads, kSmemBytes, s>>>(p, a);
-    else if (mode == kReverseForward) tile_kernel<true, true><<<p.ntiles_slow, kTileThreads, kSmemBytes, s>>>(p, a);
-    else tile_kernel<true, false><<<p.ntiles_slow, kTileThreads, kSmemBytes, s>>>(p, a);
-  }
+  // one launch: global tiles in the first CTAs (the longest start earliest), then the pipelined tiles
+  const int grid = p.ntiles + p.ntiles_slow;
+  if (grid == 0) return;
+  if (mode == kForwardOnly) tile_bulk<false, true><<<grid, kBThreads, kBSmemBytes, s>>>(p, a);
+  else if (mode == kReverseForward) tile_bulk<true, true><<<grid, kBThreads, kBSmemBytes, s>>>(p, a);
+  else tile_bulk<true, false><<<grid, kBThreads, kBSmemBytes, s>>>(p, a);
 }
+void launch_kg_loss(const KParams& p, const StepArgs& a, cudaStream_t s) { kg_loss_kernel<<<1, 256, 0, s>>>(p, a); }
 void launch_kg(const KParams& p, const StepArgs& a, cudaStream_t s) {
   kg_kernel<<<p.X + p.Y, kGThreads, 0, s>>>(p, a);
 }
