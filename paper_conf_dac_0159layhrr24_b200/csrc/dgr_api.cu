@@ -3,7 +3,7 @@
 //
 // The data-parallel unit is the net (§3.2: nets couple only through the demand d of
 // Eq. (10)).  Rank r keeps a contiguous, work-balanced range of nets; per iteration
-// the ranks exchange one int64 buffer [dH | dV^T | VD | E[WL] | E[TP]] with ncclAllReduce —
+// the ranks exchange one int64 buffer [dH | dV^T | VD | VD^T] with ncclAllReduce —
 // fixed point makes the sum exact, so every rank then runs the (replicated) grid pass on
 // identical data and the result does not depend on the number of ranks.
 #include <cuda_runtime.h>
@@ -695,7 +695,7 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.mt = take(4 * nt + 16);
   L.vt = take(4 * nt + 16);
   L.q = take(4 * nt + 16);
-  L.xcount = 3 * G + 2;   // dH | dV^T | VD | E[WL], E[TP]
+  L.xcount = 4 * G;   // dH | dV^T | VD | VD^T
   L.xbuf = take(8 * L.xcount);
   L.capH = take(4 * G);
   L.capVT = take(4 * G);
@@ -912,7 +912,7 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   P.dH = (long long*)(ws + L.xbuf);
   P.dVT = P.dH + G;
   P.VD = P.dVT + G;
-  P.scal = P.VD + G;
+  P.VDT = P.VD + G;
   P.capH = (const float*)(ws + L.capH);
   P.capVT = (const float*)(ws + L.capVT);
   P.SH = (double*)(ws + L.SH); P.SVT = (double*)(ws + L.SVT);
@@ -1024,13 +1024,9 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
   if ((rc = prof_mark(h, -1))) return rc;
   const size_t grid_bytes = 8 * (size_t)h->X * h->Y;
   if (!(h->fwd_valid && h->t_fwd == temperature)) {
-    // KG clears dH / dV^T in place after reading them; stale events of a forward at another
-    // temperature are cleared here.  VD is cleared before every forward.
-    if (h->fwd_valid) {
-      CUDA_TRY(cudaMemsetAsync(P.dH, 0, 2 * grid_bytes, s));   // dH | dV^T
-      CUDA_TRY(cudaMemsetAsync(P.scal, 0, 2 * sizeof(long long), s));
-    }
-    CUDA_TRY(cudaMemsetAsync(P.VD, 0, grid_bytes, s));
+    // KG clears the event grids in place after reading them; stale events of a forward at another
+    // temperature are cleared here
+    if (h->fwd_valid) CUDA_TRY(cudaMemsetAsync(P.dH, 0, 4 * grid_bytes, s));   // dH | dV^T | VD | VD^T
     launch_tiles(P, a, kForwardOnly, s);
     if ((rc = prof_mark(h, 0))) return rc;
   }
@@ -1052,7 +1048,6 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
     if (iters > 0) {
       // reverse of iteration k + forward of k+1 (also after the last iteration: the next call
       // at the same temperature starts from it)
-      CUDA_TRY(cudaMemsetAsync(P.VD, 0, grid_bytes, s));
       launch_tiles(P, a, kReverseForward, s);
       h->k += 1;
       if ((rc = prof_mark(h, 3))) return rc;

@@ -100,11 +100,11 @@ struct KParams {
   const int32_t* net_tree_off;    // local, n_nets_l + 1
   const int32_t* mnets;     // per tile: offsets (in the tile) of its nets with >= 2 trees
   float *wt, *mt, *vt, *q;
-  // grids (the exchange buffer, in this order: dH | dVT | VD | scal)
+  // grids (the exchange buffer, in this order: dH | dVT | VD | VDT)
   long long* dH;            // [Y][X]
   long long* dVT;           // [X][Y]
-  long long* VD;            // [Y][X] turning points per G-cell (cleared before every forward)
-  long long* scal;          // {E[WL], E[TP]} fixed point
+  long long* VD;            // [Y][X] turning points per G-cell
+  long long* VDT;           // [X][Y] the same, column-major (KG's column pass)
   const float* capH;        // [Y][X]
   const float* capVT;       // [X][Y]
   double* SH;               // [Y][XP]

@@ -437,15 +437,16 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
       if (GLOBAL) {
         const int X = P.X, Y = P.Y;
         red64(P.dH + (size_t)ya * X + xa, ah); red64(P.dVT + (size_t)xa * Y + ya, av);
-        red64(P.VD + (size_t)ya * X + xa, ad);
+        red64(P.VD + (size_t)ya * X + xa, ad); red64(P.VDT + (size_t)xa * Y + ya, ad);
         red64(P.dH + (size_t)yb * X + xb, bh); red64(P.dVT + (size_t)xb * Y + yb, bv);
-        red64(P.VD + (size_t)yb * X + xb, bd);
+        red64(P.VD + (size_t)yb * X + xb, bd); red64(P.VDT + (size_t)xb * Y + yb, bd);
       }
       if (outside) {
         if (GLOBAL) {
           const int X = P.X, Y = P.Y;
           c_events(L.pw, x0, y0, x1, y1, vq, [&](int fld, int x, int y, int val) {
             red64(fld == 0 ? P.dH + (size_t)y * X + x : fld == 1 ? P.dVT + (size_t)x * Y + y : P.VD + (size_t)y * X + x, val);
+            if (fld == 2) red64(P.VDT + (size_t)x * Y + y, val);
           });
         } else {
           c_events(L.pw, x0, y0, x1, y1, vq, [&](int fld, int x, int y, int val) {
@@ -582,6 +583,7 @@ __device__ __forceinline__ void slow_tile(const KParams& P, const StepArgs& A, c
           if (T.wx0 + xi >= X) break;
           red64(P.dH + g0 + xi, rowH[xi]);
           red64(P.VD + g0 + xi, rowD[xi]);
+          red64(P.VDT + (size_t)(T.wx0 + xi) * Y + T.wy0 + yi, rowD[xi]);
         }
       }
       for (int xi = warp; xi < T.ww; xi += kWarps) {
@@ -954,6 +956,10 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         const size_t g = (size_t)(T.wy0 + r) * X + T.wx0 + 2 * (i - r * hw);
         red64(P.dH + g, h.x); red64(P.dH + g + 1, h.y);
         red64(P.VD + g, d.x); red64(P.VD + g + 1, d.y);
+        if (d.x | d.y) {   // the turning points also column-major, for KG's column pass
+          const size_t gt = (size_t)(T.wx0 + 2 * (i - r * hw)) * Y + T.wy0 + r;
+          red64(P.VDT + gt, d.x); red64(P.VDT + gt + Y, d.y);
+        }
       }
       if (v.x | v.y) {
         const int c = (int)(((float)i + 0.5f) * inv_hh);
@@ -1007,7 +1013,7 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
 // KG: one CTA per line (Y H-rows, then X V-columns).  Scan of the difference array gives the
 // wire demand W; d = (W + beta (VD_a + VD_b)) 2^-24 (Eq. (10), reading Q3); overflow cost
 // f(cap - d) (Eq. (9)); G = dcost/dd = -a3 f'(cap - d); S = exclusive prefix of G (fp64).
-// The line's difference entries are cleared for the next forward (VD is cleared by a memset).
+// The line's difference and turning-point entries are cleared for the next forward.
 // ------------------------------------------------------------------------------------------
 constexpr int kGThreads = 32 * kKgWarps;
 constexpr int kGItems = 4;
@@ -1121,9 +1127,8 @@ __global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A)
   const int ln = isH ? line : line - P.Y;
   const size_t base = (size_t)ln * n;
   long long* diff = (isH ? P.dH : P.dVT) + base;
-  // turning points at the line's cells: contiguous for a row, stride X for a column
-  const long long* vd = isH ? P.VD + base : P.VD + ln;
-  const size_t vstep = isH ? 1 : (size_t)P.X;
+  // turning points at the line's cells (VD for rows, its column-major copy VD^T for columns)
+  long long* vd = (isH ? P.VD : P.VDT) + base;
   const float* cap = (isH ? P.capH : P.capVT) + base;
   double* S = isH ? P.SH + (size_t)ln * P.XP : P.SVT + (size_t)ln * P.YP;
   float* dout = (isH ? P.dOutH : P.dOutVT) + base;
@@ -1139,14 +1144,14 @@ __global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A)
     for (int j = 0; j < kGItems; ++j) {
       const int pos = c0 + j * kGThreads + threadIdx.x;
       v[j] = pos < n ? diff[pos] : 0;
-      t0[j] = pos < n ? vd[(size_t)pos * vstep] : 0;
+      t0[j] = pos < n ? vd[pos] : 0;
       cp[j] = pos < n ? cap[pos] : 0.f;
     }
 #pragma unroll
     for (int j = 0; j < kGItems; ++j) {   // the next cell's turning points: the next lane's t0
       const int pos = c0 + j * kGThreads + threadIdx.x;
       t1[j] = __shfl_down_sync(kFull, t0[j], 1);
-      if (lane == 31) t1[j] = pos + 1 < n ? vd[(size_t)(pos + 1) * vstep] : 0;
+      if (lane == 31) t1[j] = pos + 1 < n ? vd[pos + 1] : 0;
       if (isH) tsum += t0[j];
     }
     long long totW;
@@ -1157,7 +1162,7 @@ __global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A)
 #pragma unroll
     for (int j = 0; j < kGItems; ++j) {
       const int pos = c0 + j * kGThreads + threadIdx.x;
-      if (pos < n) diff[pos] = 0;
+      if (pos < n) { diff[pos] = 0; vd[pos] = 0; }   // cleared for the next forward
     }
     double g[kGItems];
 #pragma unroll
