@@ -520,7 +520,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
 #pragma omp parallel
   {
     std::vector<uint16_t> cnt;
-    std::vector<size_t> cell_buf;
+    std::vector<int> stamp;
 #pragma omp for schedule(dynamic, 16)
     for (int64_t t = 0; t < ntile; ++t) {
       TileDesc T{};
@@ -623,23 +623,25 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       // sum_j |pi_j| <= 2^24 + 32 in magnitude.  Otherwise run the tile against global memory.
       if (!T.global) {
         cnt.assign((size_t)3 * T.ww * T.wh, 0);
+        stamp.assign((size_t)3 * T.ww * T.wh, -1);   // last sub-net counted at a cell-field
         bool ok = true;
-        std::vector<size_t>& cells = cell_buf;
         for (int64_t sn = d->tree_sub_off[j0]; sn < d->tree_sub_off[j1] && ok; ++sn) {
           const short4 e = sxy_csr[sn - pl.sub_lo];
-          cells.clear();
-          for (int64_t i = d->sub_path_off[sn]; i < d->sub_path_off[sn + 1]; ++i) {
+          const int id = (int)(sn - d->tree_sub_off[j0]);
+          for (int64_t i = d->sub_path_off[sn]; i < d->sub_path_off[sn + 1] && ok; ++i) {
             const uint32_t pw = pw_path[i - pl.path_lo];
             int ex[8], ey[8], ef[8];
             const int ne = lane_events(pw, e.x, e.y, e.z, e.w, ex, ey, ef);
-            for (int q = 0; q < ne; ++q)
+            for (int q = 0; q < ne; ++q) {
               // the event windows of the H / VD fields are row-major, the V field's column-major;
               // any fixed cell index works for counting
-              cells.push_back((size_t)ef[q] * T.ww * T.wh + (size_t)(ey[q] - T.wy0) * T.ww + (ex[q] - T.wx0));
+              const size_t c = (size_t)ef[q] * T.ww * T.wh + (size_t)(ey[q] - T.wy0) * T.ww + (ex[q] - T.wx0);
+              if (stamp[c] != id) {
+                stamp[c] = id;
+                if (++cnt[c] > kEventMax) ok = false;
+              }
+            }
           }
-          std::sort(cells.begin(), cells.end());
-          for (size_t q = 0; q < cells.size() && ok; ++q)
-            if ((q == 0 || cells[q] != cells[q - 1]) && ++cnt[cells[q]] > kEventMax) ok = false;
         }
         if (!ok) { T.global = 1; T.wx0 = T.wy0 = T.ww = T.wh = 0; }
       }
