@@ -387,7 +387,7 @@ def main():
         "stage_launches": n_prof,
         # our kernels in the timed region (the profiled repeat of it launches the same ones):
         # KF / KBF / KB = one tile kernel (global tiles in its first CTAs), KG = 1 kernel
-        "gpu_launches": n_prof["KF"] + n_prof["KBF"] + n_prof["KB"] + n_prof["KG"],
+        "gpu_launches": n_prof["KF"] + n_prof["KBF"] + n_prof["KB"] + n_prof["KG"] + n_prof["KL"],
         "clocks": clocks,
         "induce_ms": induce_ms,
         "loss": {"total": float(loss[0]), "wl": float(loss[1]), "via": float(loss[2]), "overflow": float(loss[3])},

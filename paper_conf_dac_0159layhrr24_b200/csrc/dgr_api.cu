@@ -17,6 +17,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <memory>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -199,6 +200,37 @@ struct PodBuf {
   T& operator[](size_t i) { return p[i]; }
   const T& operator[](size_t i) const { return p[i]; }
 };
+
+// Process-wide pinned staging buffer for the workspace upload (grow-only, reused by every handle;
+// the driver's pageable copies would stage through a small bounce buffer instead).  Callers hold
+// the lock from staging until their copies have completed.
+struct PinnedPool {
+  std::mutex m;
+  char* p = nullptr;
+  size_t n = 0;
+  char* get(size_t bytes) {   // with m held
+    if (bytes <= n) return p;
+    if (p) cudaFreeHost(p);
+    p = nullptr;
+    n = 0;
+    if (cudaHostAlloc(reinterpret_cast<void**>(&p), bytes, cudaHostAllocDefault) != cudaSuccess) { p = nullptr; return nullptr; }
+    n = bytes;
+    return p;
+  }
+};
+PinnedPool g_pin;
+
+// parallel copy into pinned staging memory
+void par_copy(char* dst, const void* src, size_t bytes) {
+  const char* s = static_cast<const char*>(src);
+  constexpr size_t kChunk = 1 << 20;
+  const int64_t nch = (int64_t)((bytes + kChunk - 1) / kChunk);
+#pragma omp parallel for schedule(static)
+  for (int64_t c = 0; c < nch; ++c) {
+    const size_t o = (size_t)c * kChunk;
+    memcpy(dst + o, s + o, std::min(kChunk, bytes - o));
+  }
+}
 
 struct Plan {
   int64_t net_lo = 0, net_hi = 0, tree_lo = 0, tree_hi = 0, sub_lo = 0, sub_hi = 0, path_lo = 0, path_hi = 0;
@@ -659,7 +691,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   std::stable_partition(pl.tiles.begin(), pl.tiles.end(), pipelined);
   pl.n_pipe_tiles = 0;
   for (const auto& T : pl.tiles) pl.n_pipe_tiles += pipelined(T);
-  {   // largest tiles first (LPT): a shorter tail of the last wave of CTAs (+1.5% on ispd19)
+  if (!getenv("DGR_TILE_SPATIAL")) {   // largest tiles first (LPT): a shorter tail of the last wave of CTAs (+1.5% on ispd19)
     std::stable_sort(pl.tiles.begin(), pl.tiles.begin() + pl.n_pipe_tiles, [](const TileDesc& a, const TileDesc& b) {
       return 4 * a.nbg + (a.nb - a.nbg) > 4 * b.nbg + (b.nb - b.nbg);
     });
@@ -671,7 +703,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
 // workspace layout
 // ---------------------------------------------------------------------------------------
 struct Layout {
-  size_t tiles, mnets, binfo, pword, sxy, slot_path, wp, mp, vp, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
+  size_t tiles, mnets, binfo, pword, sxy, slot_path, wp, mv, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
       partial, lpart, loss, chosen, tree_choice, route, nsize, nucleus_tmp, DHVC, iscal, ipartial, metrics, total;
   size_t xcount;   // int64 elements in the exchange buffer
 };
@@ -689,8 +721,7 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.sxy = take(8 * ns + 16);
   L.slot_path = take(4 * slots);
   L.wp = take(4 * slots);
-  L.mp = take(4 * slots);
-  L.vp = take(4 * slots);
+  L.mv = take(8 * slots);
   L.pp = take(4 * slots);   // p of the last forward (read by the next reverse)
   L.nto = take(4 * (nn + 1) + 16);   // +16 B: 16-byte aligned bulk reads may run past the end
   L.wt = take(4 * nt + 16);
@@ -906,7 +937,7 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   P.pword = (const uint32_t*)(ws + L.pword);
   P.sxy = (const short4*)(ws + L.sxy);
   P.slot_path = (const int32_t*)(ws + L.slot_path);
-  P.wp = (float*)(ws + L.wp); P.mp = (float*)(ws + L.mp); P.vp = (float*)(ws + L.vp);
+  P.wp = (float*)(ws + L.wp); P.mv = (float2*)(ws + L.mv);
   P.pp = (float*)(ws + L.pp);
   P.net_tree_off = (const int32_t*)(ws + L.nto);
   P.wt = (float*)(ws + L.wt); P.mt = (float*)(ws + L.mt); P.vt = (float*)(ws + L.vt); P.q = (float*)(ws + L.q);
@@ -945,39 +976,49 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   if (prepare_kernels() != 0) return cleanup(fail(DGR_ECUDA, "cudaFuncSetAttribute (tile kernel shared memory) failed"));
   tm.mark("bind: prepare kernels");
   if (cudaMemsetAsync(ws, 0, L.total, s) != cudaSuccess) return cleanup(fail(DGR_ECUDA, "memset workspace failed"));
-  // host-side staging of the encoded shard
+  // host-side staging of the encoded shard, packed into pinned memory, then one copy per region
   const size_t slots = (size_t)pl.nb * 32;
-  std::vector<float> wslots(slots, 0.f), pslots(slots, 0.f);
+  const size_t nt = (size_t)(pl.tree_hi - pl.tree_lo);
+  struct Region { size_t off, bytes; const void* src; };   // src == nullptr: filled in place below
+  std::vector<Region> regs = {
+      {L.tiles, sizeof(TileDesc) * pl.tiles.size(), pl.tiles.data()},
+      {L.mnets, 4 * pl.mnets.size(), pl.mnets.data()},
+      {L.binfo, sizeof(int4) * pl.nb, pl.binfo.data()},
+      {L.pword, 4 * slots, pl.pword.data()},
+      {L.sxy, 8 * pl.sxy.size(), pl.sxy.data()},
+      {L.wp, 4 * slots, nullptr},
+      {L.pp, 4 * slots, nullptr},
+      {L.slot_path, 4 * slots, pl.slot_path.data()},
+      {L.nto, 4 * pl.net_tree_off.size(), pl.net_tree_off.data()},
+      {L.wt, 4 * nt, desc->w_tree0 + pl.tree_lo},
+      {L.q, 4 * nt, nullptr},
+      {L.capH, 4 * G, desc->cap_h},
+      {L.capVT, 4 * G, nullptr}};
+  std::vector<size_t> at(regs.size() + 1, 0);
+  for (size_t i = 0; i < regs.size(); ++i) at[i + 1] = at[i] + ((regs[i].bytes + 255) & ~(size_t)255);
+  std::lock_guard<std::mutex> lock(g_pin.m);
+  char* pin = g_pin.get(at.back());
+  if (!pin) return cleanup(fail(DGR_ENOMEM, "cudaHostAlloc of %zu staging bytes failed", at.back()));
+  float* wslots = reinterpret_cast<float*>(pin + at[5]);
+  float* pslots = reinterpret_cast<float*>(pin + at[6]);
+  float* qs = reinterpret_cast<float*>(pin + at[10]);
+  float* capVT = reinterpret_cast<float*>(pin + at[12]);
 #pragma omp parallel for schedule(static)
-  for (size_t sl = 0; sl < slots; ++sl)
-    if (pl.slot_path[sl] >= 0) {
-      wslots[sl] = desc->w_path0[pl.path_lo + pl.slot_path[sl]];
-      pslots[sl] = 1.f;   // p of a lone straight candidate (never rewritten by the pipelined kernel)
-    }
-  std::vector<float> capVT(G);
+  for (size_t sl = 0; sl < slots; ++sl) {
+    const bool v = pl.slot_path[sl] >= 0;
+    wslots[sl] = v ? desc->w_path0[pl.path_lo + pl.slot_path[sl]] : 0.f;
+    pslots[sl] = v ? 1.f : 0.f;   // p of a lone straight candidate (never rewritten by the pipelined kernel)
+  }
+  for (size_t j = 0; j < nt; ++j) qs[j] = 1.f;   // q of a net's lone tree stays 1 (never rewritten)
 #pragma omp parallel for schedule(static)
   for (int y = 0; y < desc->Y; ++y)
     for (int x = 0; x < desc->X; ++x) capVT[(size_t)x * desc->Y + y] = desc->cap_v[(size_t)y * desc->X + x];
-  const size_t nt = (size_t)(pl.tree_hi - pl.tree_lo);
+  for (size_t i = 0; i < regs.size(); ++i)
+    if (regs[i].src && regs[i].bytes) par_copy(pin + at[i], regs[i].src, regs[i].bytes);
   tm.mark("bind: host staging");
   cudaError_t e = cudaSuccess;
-  auto cp = [&](size_t off, const void* src, size_t bytes) {
-    if (bytes && e == cudaSuccess) e = cudaMemcpyAsync(ws + off, src, bytes, cudaMemcpyHostToDevice, s);
-  };
-  cp(L.tiles, pl.tiles.data(), sizeof(TileDesc) * pl.tiles.size());
-  cp(L.mnets, pl.mnets.data(), 4 * pl.mnets.size());
-  cp(L.binfo, pl.binfo.data(), sizeof(int4) * pl.nb);
-  cp(L.pword, pl.pword.data(), 4 * slots);
-  cp(L.sxy, pl.sxy.data(), 8 * pl.sxy.size());
-  cp(L.wp, wslots.data(), 4 * slots);
-  cp(L.pp, pslots.data(), 4 * slots);
-  cp(L.slot_path, pl.slot_path.data(), 4 * slots);
-  cp(L.nto, pl.net_tree_off.data(), 4 * pl.net_tree_off.size());
-  cp(L.wt, desc->w_tree0 + pl.tree_lo, 4 * nt);
-  const std::vector<float> ones(nt, 1.f);   // q of a net's lone tree stays 1 (never rewritten)
-  cp(L.q, ones.data(), 4 * nt);
-  cp(L.capH, desc->cap_h, 4 * G);
-  cp(L.capVT, capVT.data(), 4 * G);
+  for (size_t i = 0; i < regs.size() && e == cudaSuccess; ++i)
+    if (regs[i].bytes) e = cudaMemcpyAsync(ws + regs[i].off, pin + at[i], regs[i].bytes, cudaMemcpyHostToDevice, s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
   tm.mark("bind: upload");
   if (e != cudaSuccess) return cleanup(fail(DGR_ECUDA, "upload: %s", cudaGetErrorString(e)));
@@ -1045,8 +1086,11 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
       if ((rc = prof_mark(h, 1))) return rc;
     }
     launch_kg(P, a, s);
-    if (last) launch_kg_loss(P, a, s);
     if ((rc = prof_mark(h, 2))) return rc;
+    if (last) {   // the reported loss of this call's last forward
+      launch_kg_loss(P, a, s);
+      if ((rc = prof_mark(h, 5))) return rc;
+    }
     if (iters > 0) {
       // reverse of iteration k + forward of k+1 (also after the last iteration: the next call
       // at the same temperature starts from it)

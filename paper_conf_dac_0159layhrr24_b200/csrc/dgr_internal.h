@@ -95,7 +95,8 @@ struct KParams {
   const uint32_t* pword;
   const short4* sxy;        // kernel order
   const int32_t* slot_path; // local CSR path of each slot (-1 for padding); induction only
-  float *wp, *mp, *vp;
+  float* wp;
+  float2* mv;               // Adam moments (m, v) of each slot, interleaved (one 8-byte access)
   float* pp;                // p_i of the last forward (the reverse of that iteration reads it)
   const int32_t* net_tree_off;    // local, n_nets_l + 1
   const int32_t* mnets;     // per tile: offsets (in the tile) of its nets with >= 2 trees

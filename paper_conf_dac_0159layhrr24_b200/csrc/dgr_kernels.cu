@@ -146,8 +146,9 @@ __device__ __forceinline__ void red64(long long* p, long long v) {
 __device__ __forceinline__ void adam_update(float& w, float& m, float& v, float g, const StepArgs& A) {
   m = fmaf(0.1f, g - m, m);                         // m.lerp_(g, 1 - beta1)
   v = fmaf(0.999f, v, 0.001f * g * g);              // v * beta2 + (1 - beta2) g^2
-  // sqrt(v) = v rsqrt(v) (MUFU, v >= 0) and a MUFU division: ~1e-7 relative, well inside the 1e-4 bar
-  const float sq = v > 0.f ? v * rsqrtf(v) : 0.f;
+  // MUFU square root and division: ~1e-7 relative, well inside the 1e-4 bar
+  float sq;
+  asm("sqrt.approx.f32 %0, %1;" : "=f"(sq) : "f"(v));
   const float denom = sq * A.inv_sqrt_bc2 + 1e-8f;
   w -= A.lr_over_bc1 * __fdividef(m, denom);
 }
@@ -316,7 +317,7 @@ __device__ __forceinline__ void reverse_warp(const KParams& P, const StepArgs& A
   Lane L;
   lane_from(__ldg(&P.binfo[bw0]), __ldg(&P.pword[slot]), P, L);
   short4 e = L.valid ? __ldg(&P.sxy[L.sub]) : make_short4(0, 0, 0, 0);
-  float w = P.wp[slot], m = P.mp[slot], v = P.vp[slot], p = P.pp[slot];
+  float w = P.wp[slot], m = P.mv[slot].x, v = P.mv[slot].y, p = P.pp[slot];
   int4 bi1 = make_int4(0, 0, 0, 0);
   uint32_t pw1 = kPad | kSubHead;
   if (bw0 + 1 < bw1) { bi1 = __ldg(&P.binfo[bw0 + 1]); pw1 = __ldg(&P.pword[slot + 32]); }
@@ -327,7 +328,7 @@ __device__ __forceinline__ void reverse_warp(const KParams& P, const StepArgs& A
     if (b + 1 < bw1) {
       lane_from(bi1, pw1, P, Ln);
       if (Ln.valid) en = __ldg(&P.sxy[Ln.sub]);
-      wn = P.wp[slot + 32]; mn = P.mp[slot + 32]; vn = P.vp[slot + 32]; pn = P.pp[slot + 32];
+      wn = P.wp[slot + 32]; mn = P.mv[slot + 32].x; vn = P.mv[slot + 32].y; pn = P.pp[slot + 32];
       if (b + 2 < bw1) { bi1 = __ldg(&P.binfo[b + 2]); pw1 = __ldg(&P.pword[slot + 64]); }
     }
     const float q = L.valid ? q_s[L.tree - T.tree0] : 0.f;
@@ -355,8 +356,7 @@ __device__ __forceinline__ void reverse_warp(const KParams& P, const StepArgs& A
     if (L.valid) {
       adam_update(w, m, v, dw, A);
       P.wp[slot] = w;
-      P.mp[slot] = m;
-      P.vp[slot] = v;
+      P.mv[slot] = make_float2(m, v);
     }
     wst[(b - T.b0) * 32 + lane] = w;
     L = Ln; e = en; w = wn; m = mn; v = vn; p = pn;
@@ -650,6 +650,49 @@ __device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t by
   asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src)), "r"(bytes)
                : "memory");
 }
+// L2 eviction policy for data streamed once per iteration (slot state, pattern words, per-bundle
+// and per-sub-net records): evict first, so the S prefix sums (re-read by neighbouring tiles) and the
+// demand grids (int64 reductions from every tile) stay resident in L2.
+#ifndef DGR_L2_HINTS
+#define DGR_L2_HINTS 1
+#endif
+__device__ __forceinline__ uint64_t policy_stream() {
+  uint64_t p;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ void bulk_g2s_stream(void* dst, const void* src, uint32_t bytes, uint64_t* bar, uint64_t pol) {
+  if (!DGR_L2_HINTS) { bulk_g2s(dst, src, bytes, bar); return; }
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+               ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_s2g_stream(void* dst, const void* src, uint32_t bytes, uint64_t pol) {
+  if (!DGR_L2_HINTS) { bulk_s2g(dst, src, bytes); return; }
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;" ::"l"(dst), "r"(smem_u32(src)),
+               "r"(bytes), "l"(pol)
+               : "memory");
+}
+__device__ __forceinline__ float ld_stream(const float* p, uint64_t pol) {
+  if (!DGR_L2_HINTS) return *p;
+  float v;
+  asm volatile("ld.global.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ float2 ld_stream2(const float2* p, uint64_t pol) {
+  if (!DGR_L2_HINTS) return *p;
+  float2 v;
+  asm volatile("ld.global.L2::cache_hint.v2.f32 {%0, %1}, [%2], %3;" : "=f"(v.x), "=f"(v.y) : "l"(p), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ void st_stream(float* p, float v, uint64_t pol) {
+  if (!DGR_L2_HINTS) { *p = v; return; }
+  asm volatile("st.global.L2::cache_hint.f32 [%0], %1, %2;" ::"l"(p), "f"(v), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void st_stream2(float2* p, float2 v, uint64_t pol) {
+  if (!DGR_L2_HINTS) { *p = v; return; }
+  asm volatile("st.global.L2::cache_hint.v2.f32 [%0], {%1, %2}, %3;" ::"l"(p), "f"(v.x), "f"(v.y), "l"(pol) : "memory");
+}
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
@@ -693,16 +736,17 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
   if (lane == 0) mbar_expect_tx(bar, bytes);
   __syncwarp();
   const size_t s0 = (size_t)T.b0 * 32;
+  const uint64_t pol = policy_stream();
   // work items: 0..7 the 1-D arrays, then window rows, then window columns
   const int nitems = 8 + (int)nrow + (int)ncol;
   for (int it = lane; it < nitems; it += 32) {
     if (it < 8) {
       switch (it) {
-        case 0: bulk_g2s(S.pw, P.pword + s0, slot_bytes, bar); break;
-        case 1: if (gslot_bytes) bulk_g2s(S.w, P.wp + s0, gslot_bytes, bar); break;
-        case 2: bulk_g2s(S.bi, P.binfo + T.b0, 16u * T.nb, bar); break;
-        case 3: bulk_g2s(S.sxy, P.sxy + s_lo, 8u * (s_hi - s_lo), bar); break;
-        case 4: bulk_g2s(S.nto, P.net_tree_off + n_lo, 4u * (n_hi - n_lo), bar); break;
+        case 0: bulk_g2s_stream(S.pw, P.pword + s0, slot_bytes, bar, pol); break;
+        case 1: if (gslot_bytes) bulk_g2s_stream(S.w, P.wp + s0, gslot_bytes, bar, pol); break;
+        case 2: bulk_g2s_stream(S.bi, P.binfo + T.b0, 16u * T.nb, bar, pol); break;
+        case 3: bulk_g2s_stream(S.sxy, P.sxy + s_lo, 8u * (s_hi - s_lo), bar, pol); break;
+        case 4: bulk_g2s_stream(S.nto, P.net_tree_off + n_lo, 4u * (n_hi - n_lo), bar, pol); break;
         case 5: if (mn_hi > mn_lo) bulk_g2s(S.mn, P.mnets + mn_lo, 4u * (mn_hi - mn_lo), bar); break;
         case 6: bulk_g2s(S.wt, P.wt + t_lo, 4u * (t_hi - t_lo), bar); break;
         default: bulk_g2s(S.q, P.q + t_lo, 4u * (t_hi - t_lo), bar); break;   // also a lone tree's q = 1
@@ -733,6 +777,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
   const int mn_lo = T.mn0 & ~3;
+  const uint64_t pol = policy_stream();   // L2 evict-first for the streamed slot state
   const int ncell = T.ww * T.wh;
   const Win W{T.wx0, T.wy0, T.ww, T.wh, ncell};
   const int wB0 = -(T.wy0 * T.ww + T.wx0), wB1 = ncell - T.wx0 * T.wh - T.wy0;   // orientation bases
@@ -750,8 +795,9 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         const int sl = lb * 32 + lane;
         const size_t gsl = (size_t)T.b0 * 32 + sl;
         float w = St.w[sl];
-        float m = P.mp[gsl], v = P.vp[gsl];
-        const float p = P.pp[gsl];
+        const float2 mv = ld_stream2(&P.mv[gsl], pol);
+        float m = mv.x, v = mv.y;
+        const float p = ld_stream(&P.pp[gsl], pol);
         const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
         double c = 0.0;
         if (L.valid && !(P.skip & 8)) {
@@ -772,7 +818,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         if (L.valid) {
           adam_update(w, m, v, dw, A);
           St.w[sl] = w;
-          P.mp[gsl] = m; P.vp[gsl] = v;
+          st_stream2(&P.mv[gsl], make_float2(m, v), pol);
         }
       } else {
         // singleton bundle: c of a straight path (one segment, no turning point); p = 1
@@ -884,7 +930,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         const float w = St.w[sl];
         const float g = L.valid ? gp[bi.x + lane - nid0] : 0.f;
         const float p = softmax_from_noise(L, w, g, A.inv_t);
-        P.pp[(size_t)T.b0 * 32 + sl] = p;
+        st_stream(&P.pp[(size_t)T.b0 * 32 + sl], p, pol);
         const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
         const int vq = L.valid ? __float2int_rn(q * p * kFixScale) : 0;
         if (L.valid && !(P.skip & 4)) {
@@ -935,7 +981,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     fence_proxy_async();
     const size_t s0 = (size_t)T.b0 * 32;
     const uint32_t gslot_bytes = (uint32_t)nbg * 128u;
-    if (REV) bulk_s2g(P.wp + s0, St.w, gslot_bytes);
+    if (REV) bulk_s2g_stream(P.wp + s0, St.w, gslot_bytes, policy_stream());
     bulk_commit();
   }
   if (FWD && !(P.skip & 1)) {

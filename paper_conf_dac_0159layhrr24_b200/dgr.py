@@ -289,7 +289,7 @@ class Solver:
                     workspace_bytes=int(a[5]), world=int(a[6]), rank=int(a[7]), n_tiles=int(a[8]),
                     n_global_tiles=int(a[9]), n_pipe_tiles=int(a[10]))
 
-    STAGES = ("KF", "allreduce", "KG", "KBF", "KB")
+    STAGES = ("KF", "allreduce", "KG", "KBF", "KB", "KL")   # KL: the loss kernel, once per call
 
     def profile(self, enable: bool = True):
         """Start (and clear) / stop per-stage CUDA-event timing of dgr_step."""
