@@ -552,7 +552,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
 #pragma omp parallel
   {
     std::vector<uint16_t> cnt;
-    std::vector<int> stamp;
+    std::vector<int> stamp, cov;
 #pragma omp for schedule(dynamic, 16)
     for (int64_t t = 0; t < ntile; ++t) {
       TileDesc T{};
@@ -653,7 +653,30 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       // int32 shared-memory accumulation is exact while no window cell-field is touched by more
       // than kEventMax sub-nets: the events one sub-net puts on one cell-field sum to at most
       // sum_j |pi_j| <= 2^24 + 32 in magnitude.  Otherwise run the tile against global memory.
+      // Fast sufficient test first: a sub-net's events all lie inside its box (detours included),
+      // so if no window cell is covered by more than kEventMax sub-net boxes (2-D difference array
+      // over the window), no cell-field can be touched by more than kEventMax sub-nets.
+      bool safe = false;
       if (!T.global) {
+        const int W1 = T.ww + 1;
+        cov.assign((size_t)W1 * (T.wh + 1), 0);
+        for (int64_t sn = d->tree_sub_off[j0]; sn < d->tree_sub_off[j1]; ++sn) {
+          const short4 b = sub_ext[sn - pl.sub_lo];
+          const int bx0 = b.x - T.wx0, by0 = b.y - T.wy0, bx1 = b.z - T.wx0 + 1, by1 = b.w - T.wy0 + 1;
+          cov[(size_t)by0 * W1 + bx0] += 1; cov[(size_t)by0 * W1 + bx1] -= 1;
+          cov[(size_t)by1 * W1 + bx0] -= 1; cov[(size_t)by1 * W1 + bx1] += 1;
+        }
+        int mx = 0;
+        for (int y = 0; y < T.wh; ++y)
+          for (int x = 0; x < T.ww; ++x) {
+            int& c = cov[(size_t)y * W1 + x];
+            c += (x > 0 ? cov[(size_t)y * W1 + x - 1] : 0) + (y > 0 ? cov[(size_t)(y - 1) * W1 + x] : 0) -
+                 (x > 0 && y > 0 ? cov[(size_t)(y - 1) * W1 + x - 1] : 0);
+            mx = std::max(mx, c);
+          }
+        safe = mx <= kEventMax;
+      }
+      if (!T.global && !safe) {
         cnt.assign((size_t)3 * T.ww * T.wh, 0);
         stamp.assign((size_t)3 * T.ww * T.wh, -1);   // last sub-net counted at a cell-field
         bool ok = true;

@@ -654,7 +654,7 @@ __device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t by
 // and per-sub-net records): evict first, so the S prefix sums (re-read by neighbouring tiles) and the
 // demand grids (int64 reductions from every tile) stay resident in L2.
 #ifndef DGR_L2_HINTS
-#define DGR_L2_HINTS 1
+#define DGR_L2_HINTS 0
 #endif
 __device__ __forceinline__ uint64_t policy_stream() {
   uint64_t p;
