@@ -945,6 +945,8 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   P.tiles_slow = P.tiles + pl.n_pipe_tiles;
   P.XP = desc->X + (desc->X & 1);
   if (const char* sk = getenv("DGR_DEBUG_SKIP")) P.skip = atoi(sk);   // timing experiments only
+  P.pf = 0;   // L2 prefetch off: with the cp.async stage it costs 0.5% (A/B)
+  if (const char* e = getenv("DGR_PF")) P.pf = atoi(e);
   P.YP = desc->Y + (desc->Y & 1);
   P.n_nets_l = (int32_t)(pl.net_hi - pl.net_lo);
   P.path_base = pl.path_lo;
@@ -1127,6 +1129,15 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
     h->t_fwd = temperature;
   }
   CUDA_TRY(cudaGetLastError());
+  if ((P.skip & 256) && getenv("DGR_PROF_OUT")) {   // diagnostics: per-tile phase clocks of the last KBF
+    CUDA_TRY(cudaStreamSynchronize(s));
+    std::vector<long long> buf(8 * (size_t)P.ntiles);
+    CUDA_TRY((cudaError_t)read_tile_prof(buf.data(), P.ntiles));
+    if (FILE* f = fopen(getenv("DGR_PROF_OUT"), "wb")) {
+      fwrite(buf.data(), 8, buf.size(), f);
+      fclose(f);
+    }
+  }
   h->t_last = temperature;
   h->beta_last = w->beta_via;
   h->have_forward = true;

@@ -84,6 +84,7 @@ struct KParams {
   int32_t ntiles_slow;      // global / oversized tiles (one CTA each)
   int32_t XP, YP;           // even pitches of S_H rows and S_V columns
   int32_t skip;             // DGR_DEBUG_SKIP: timing knock-outs (results invalid), 0 in production
+  int32_t pf;               // bit 0: L2 prefetch of the state a tile reads directly (DGR_PF, default 0)
   int64_t path_base, tree_base;   // global index of the first local path / tree
   int64_t nid_base;         // global noise index of the rank's first noisy candidate
   uint64_t seed;
@@ -149,6 +150,7 @@ void launch_induce(const KParams& p, float t_final, float top_p, float beta, cud
 void launch_induce_metrics(const KParams& p, float beta, cudaStream_t s);
 int induce_metric_blocks(const KParams& p);
 size_t tile_smem_bytes();
+int read_tile_prof(long long* out, int n);   // diagnostics: per-tile phase clocks
 int prepare_kernels();   // sets shared-memory attributes; returns cudaError_t
 int set_error(int code, const char* msg);   // the thread's dgr_last_error message (dgr_api.cu)
 void clear_error();

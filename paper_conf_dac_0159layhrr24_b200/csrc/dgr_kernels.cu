@@ -28,6 +28,13 @@ namespace dgr {
 
 constexpr unsigned kFull = 0xffffffffu;
 
+// Timing knock-outs and per-tile phase clocks (DGR_DEBUG_SKIP bits; results invalid) exist only in
+// diagnostic builds (DGR_NVCC_EXTRA=-DDGR_DIAG=1): production code carries no checks for them.
+#ifndef DGR_DIAG
+#define DGR_DIAG 0
+#endif
+#define KO(bit) (DGR_DIAG && (P.skip & (bit)))
+
 // ------------------------------------------------------------------------------------------
 // Counter-based noise: Philox4x32-10 keyed on (seed; idx>>2, k, stream), word idx & 3.
 // u = ((r >> 9) + 1/2) 2^-23 is exact in fp32; g = -ln(-ln u) (reading Q7).
@@ -496,7 +503,7 @@ __device__ __forceinline__ void slow_tile(const KParams& P, const StepArgs& A, c
   const int bw0 = T.b0 + min(warp * per, T.nb), bw1 = T.b0 + min((warp + 1) * per, T.nb);
 
   // ---------------- reverse of iteration k ----------------
-  if (REV) {
+  if (REV && !(KO(64))) {
     if (!T.global) {
       const int lane = tid & 31;
       for (int yi = warp; yi < T.wh; yi += kWarps) {
@@ -693,6 +700,9 @@ __device__ __forceinline__ void st_stream2(float2* p, float2 v, uint64_t pol) {
   if (!DGR_L2_HINTS) { *p = v; return; }
   asm volatile("st.global.L2::cache_hint.v2.f32 [%0], {%1, %2}, %3;" ::"l"(p), "f"(v.x), "f"(v.y), "l"(pol) : "memory");
 }
+__device__ __forceinline__ void prefetch_l2(const void* src, uint32_t bytes) {
+  if (bytes) asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+}
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
@@ -730,7 +740,8 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
   const int mn_lo = T.mn0 & ~3, mn_hi = (T.mn0 + T.nmn + 3) & ~3;
   const uint32_t slot_bytes = (uint32_t)T.nb * 128u, gslot_bytes = (uint32_t)T.nbg * 128u;
-  const uint32_t nrow = REV ? (uint32_t)T.wh : 0u, ncol = REV ? (uint32_t)T.ww : 0u;
+  const bool sw = REV && !(KO(32));   // knock-out 32: no S window (timing only)
+  const uint32_t nrow = sw ? (uint32_t)T.wh : 0u, ncol = sw ? (uint32_t)T.ww : 0u;
   const uint32_t bytes = slot_bytes + gslot_bytes + 16u * T.nb + 8u * (s_hi - s_lo) + 4u * (n_hi - n_lo) +
                          4u * (mn_hi - mn_lo) + 8u * (t_hi - t_lo) + 8u * (nrow * T.ww + ncol * T.wh);
   if (lane == 0) mbar_expect_tx(bar, bytes);
@@ -761,11 +772,83 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
   }
 }
 
+// The same stage filled by all threads with 16-byte cp.async copies (LSU path, no registers):
+// each warp copies one of the eight 1-D arrays, then all threads the S window rows / columns.
+// Measured per tile (scratch/tprof.py): the ~90 bulk copies of a tile queue behind those of the
+// other resident tiles in the SM's bulk-copy engine (12,000 cycles from issue to arrival).
+__device__ __forceinline__ void cp16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_copy(void* dst, const void* src, uint32_t bytes, int lane) {
+  char* d = reinterpret_cast<char*>(dst);
+  const char* g = reinterpret_cast<const char*>(src);
+  for (uint32_t o = 16u * lane; o < bytes; o += 512u) cp16(d + o, g + o);
+}
+template <bool REV, int NT>
+__device__ __forceinline__ void lsu_tile_loads(const KParams& P, const TileDesc& T, unsigned char* st) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  Stage S(st);
+  int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
+  tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
+  const int mn_lo = T.mn0 & ~3, mn_hi = (T.mn0 + T.nmn + 3) & ~3;
+  const size_t s0 = (size_t)T.b0 * 32;
+  switch (warp & 7) {
+    case 0: cp_copy(S.pw, P.pword + s0, (uint32_t)T.nb * 128u, lane); break;
+    case 1: cp_copy(S.w, P.wp + s0, (uint32_t)T.nbg * 128u, lane); break;
+    case 2: cp_copy(S.bi, P.binfo + T.b0, 16u * T.nb, lane); break;
+    case 3: cp_copy(S.sxy, P.sxy + s_lo, 8u * (s_hi - s_lo), lane); break;
+    case 4: cp_copy(S.nto, P.net_tree_off + n_lo, 4u * (n_hi - n_lo), lane); break;
+    case 5: cp_copy(S.mn, P.mnets + mn_lo, 4u * (mn_hi - mn_lo), lane); break;
+    case 6: cp_copy(S.wt, P.wt + t_lo, 4u * (t_hi - t_lo), lane); break;
+    default: cp_copy(S.q, P.q + t_lo, 4u * (t_hi - t_lo), lane); break;
+  }
+  if (REV && !(KO(32))) {
+    // S_H window rows (ww doubles = ww/2 chunks each), then S_V window columns (wh/2 chunks each);
+    // row = floor((i + 1/2) / half) in fp32 is exact for i < 2^12 (see the flush)
+    const int hw = T.ww >> 1, hh = T.wh >> 1, n = hw * T.wh;
+    const float inv_hw = 1.f / (float)hw, inv_hh = 1.f / (float)hh;
+    for (int i = tid; i < n; i += NT) {
+      const int r = (int)(((float)i + 0.5f) * inv_hw), c = i - r * hw;
+      cp16(S.S + (size_t)r * T.ww + 2 * c, P.SH + (size_t)(T.wy0 + r) * P.XP + T.wx0 + 2 * c);
+    }
+    double* SV = S.S + (size_t)T.ww * T.wh;
+    for (int i = tid; i < n; i += NT) {
+      const int r = (int)(((float)i + 0.5f) * inv_hh), c = i - r * hh;
+      cp16(SV + (size_t)r * T.wh + 2 * c, P.SVT + (size_t)(T.wx0 + r) * P.YP + T.wy0 + 2 * c);
+    }
+  }
+  asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
+// L2 prefetch of what a tile reads directly (not through the stage): the group slots' Adam moments
+// and stored p, the trees' Adam moments; issued next to the stage's bulk copies, so the direct loads
+// of the reverse and net-level phases hit L2.
+__device__ __forceinline__ void prefetch_tile(const KParams& P, const TileDesc& T) {
+  const int lane = threadIdx.x & 31;
+  const size_t s0 = (size_t)T.b0 * 32;
+  const int t_lo = T.tree0 & ~3, t_hi = (T.tree0 + T.ntree + 3) & ~3;
+  const uint32_t gs = (uint32_t)T.nbg * 32u;
+  switch (lane) {
+    case 0: if (gs) prefetch_l2(P.mv + s0, 8u * gs); break;
+    case 1: if (gs) prefetch_l2(P.pp + s0, 4u * gs); break;
+    case 2: prefetch_l2(P.mt + t_lo, 4u * (t_hi - t_lo)); break;
+    case 3: prefetch_l2(P.vt + t_lo, 4u * (t_hi - t_lo)); break;
+    default: break;
+  }
+}
+
 // One tile, all operands in shared memory (stage St).  ev_s / gp may alias St.S (they are only
 // touched after the reverse half is done with it).  Ends with the slot state written back by bulk
 // stores (issued by thread 0, committed) and the demand window flushed.
 // Bundles go to warps round-robin; lb < T.nbg are group bundles, the rest singleton bundles (lone
 // straight sub-nets: p = 1, no noise, no softmax, no Adam, no slot state).
+// Phase timing (DGR_DEBUG_SKIP bit 256, diagnostics only): per pipelined tile, SM clock at
+// [start, stage arrived, reverse done, net level done, forward done, end], SM id, global timer.
+constexpr int kProfTiles = 16384;
+__device__ long long g_tile_prof[kProfTiles * 8];
+__device__ __forceinline__ void stamp(const KParams& P, int tile, int k) {
+  if ((KO(256)) && threadIdx.x == 0 && tile < kProfTiles) g_tile_prof[tile * 8 + k] = clock64();
+}
 constexpr size_t kGpOffset = 3 * 4 * kWinMax;   // tile path noise, after the event window in St.S
 template <bool REV, bool FWD, int NT>
 __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A, const TileDesc& T, Stage St,
@@ -785,7 +868,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   const int nbg = T.nbg;
 
   // ---------------- reverse of iteration k ----------------
-  if (REV) {   // dq3 was zeroed before the stage arrived
+  if (REV && !(KO(64))) {   // dq3 was zeroed before the stage arrived
     for (int lb = warp; lb < T.nb; lb += NW) {
       const int4 bi = St.bi[lb];
       const uint32_t pw = St.pw[lb * 32 + lane];
@@ -800,7 +883,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         const float p = ld_stream(&P.pp[gsl], pol);
         const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
         double c = 0.0;
-        if (L.valid && !(P.skip & 8)) {
+        if (L.valid && !(KO(8))) {
           const short4 e = St.sxy[L.sub - s_lo];
           c = path_cost(St.S, W, X, Y, L.pw, e.x, e.y, e.z, e.w, A);
         }
@@ -826,7 +909,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         const bool isv = (pw & 7u) == kStraightV;
         const int tree = bi.z + (int)((pw >> kTreeShift) & kTreeMask);
         double c = 0.0;
-        if (valid && !(P.skip & 8)) {
+        if (valid && !(KO(8))) {
           const short4 e = St.sxy[bi.y + lane - s_lo];
           const int ia = isv ? W.v(e.x, e.y) : W.h(e.x, e.y);
           const int ib = isv ? W.v(e.x, e.w) : W.h(e.z, e.y);
@@ -843,6 +926,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     }
     __syncthreads();
   }
+  stamp(P, (int)blockIdx.x - P.ntiles_slow, 2);
 
   // ---------------- net level (one thread per net), event window cleared alongside ----------------
   if (FWD) {
@@ -851,7 +935,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   }
   // the tile's nets with >= 2 trees (a lone tree has q = 1 and du = 0 always: its logit and Adam
   // state never change, and its q = 1 arrives with the stage)
-  for (int i = tid; i < T.nmn; i += NT) {
+  for (int i = tid; i < ((KO(128)) ? 0 : T.nmn); i += NT) {
     const int n = St.mn[T.mn0 + i - mn_lo];
     const int a = St.nto[T.net0 + n - n_lo] - t_lo, b = St.nto[T.net0 + n + 1 - n_lo] - t_lo;   // stage indices
     if (REV) {
@@ -897,7 +981,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
       }
     }
   }
-  if (FWD && nbg > 0 && !(P.skip & 2)) {
+  if (FWD && nbg > 0 && !(KO(2))) {
     // Gumbel noise of the tile's noisy candidates (stream 0): contiguous noise indices
     // [bi[0].x, bi[nbg-1].x + #valid), one Philox call per 4 consecutive indices
     const int64_t n0 = P.nid_base + St.bi[0].x;
@@ -915,6 +999,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     }
   }
   __syncthreads();
+  stamp(P, (int)blockIdx.x - P.ntiles_slow, 3);
 
   // ---------------- forward of iteration k_next ----------------
   if (FWD) {
@@ -933,7 +1018,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         st_stream(&P.pp[(size_t)T.b0 * 32 + sl], p, pol);
         const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
         const int vq = L.valid ? __float2int_rn(q * p * kFixScale) : 0;
-        if (L.valid && !(P.skip & 4)) {
+        if (L.valid && !(KO(4))) {
           // the candidate's own demand events in the Z(o, m) form (see path_cost): seg 1 from p0
           // to m on line q0, seg 2 from q0 to q1 on line m, seg 3 from m to p1 on line q1, each
           // +v at its lower and -v at its upper end, plus its turning points.  No cross-lane collapse: lanes of one
@@ -961,7 +1046,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
       } else {
         // singleton bundle: pi = q; +pi where the segment starts, -pi where it ends
         const bool valid = (pw & 7u) != kPad;
-        if (valid && !(P.skip & 4)) {
+        if (valid && !(KO(4))) {
           const bool isv = (pw & 7u) == kStraightV;
           const int tree = bi.z + (int)((pw >> kTreeShift) & kTreeMask);
           const float q = St.q[tree - t_lo];
@@ -976,6 +1061,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     }
   }
   __syncthreads();
+  stamp(P, (int)blockIdx.x - P.ntiles_slow, 4);
   // write back the tile's group slot state with bulk stores (asynchronous; readers wait on the group)
   if (tid == 0 && nbg > 0) {
     fence_proxy_async();
@@ -984,7 +1070,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     if (REV) bulk_s2g_stream(P.wp + s0, St.w, gslot_bytes, policy_stream());
     bulk_commit();
   }
-  if (FWD && !(P.skip & 1)) {
+  if (FWD && !(KO(1))) {
     // flush: the window's cell pairs as one flat range per field (rows of dH / VD, columns of dV;
     // widths are even, so pair i is cells 2i, 2i+1 of the field); zero cells are skipped, and every
     // cell outside the grid is zero (events only land on grid cells).  row = floor((i + 1/2) / half
@@ -1022,6 +1108,9 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
 #define DGR_BTHREADS 256
 #endif
 constexpr int kBThreads = DGR_BTHREADS;
+#ifndef DGR_LSU_STAGE
+#define DGR_LSU_STAGE 1   // stage filled by cp.async (1) or by cp.async.bulk on an mbarrier (0)
+#endif
 #ifndef DGR_BPERSM
 #define DGR_BPERSM 5
 #endif
@@ -1043,15 +1132,39 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
   int* ev_s = reinterpret_cast<int*>(St.S);
   float* gp = reinterpret_cast<float*>(reinterpret_cast<unsigned char*>(St.S) + kGpOffset);
   const TileDesc T = P.tiles[blockIdx.x - P.ntiles_slow];
+  const int tix = (int)blockIdx.x - P.ntiles_slow;
+  stamp(P, tix, 0);
+  if ((KO(256)) && threadIdx.x == 0 && tix < kProfTiles) {
+    unsigned sm, gt_lo;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+    long long gt;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt));
+    g_tile_prof[tix * 8 + 6] = sm;
+    g_tile_prof[tix * 8 + 7] = gt;
+    (void)gt_lo;
+  }
   if (threadIdx.x == 0) {
     mbar_init(bar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   for (int i = threadIdx.x; i < 3 * kPipeTrees; i += kBThreads) dq3[i] = 0;
   __syncthreads();
-  if (threadIdx.x < 32) issue_tile_loads<REV>(P, T, smem, bar);
+#if DGR_LSU_STAGE
+  if (threadIdx.x < 32 && (P.pf & 1)) prefetch_tile(P, T);
+  lsu_tile_loads<REV, kBThreads>(P, T, smem);
+  asm volatile("cp.async.wait_group 0;" ::: "memory");
+  __syncthreads();
+#else
+  if (threadIdx.x < 32) {
+    issue_tile_loads<REV>(P, T, smem, bar);
+    if (P.pf & 1) prefetch_tile(P, T);
+  }
   mbar_wait(bar, 0u);
-  process_tile<REV, FWD, kBThreads>(P, A, T, St, ev_s, gp, dq3);
+#endif
+  stamp(P, tix, 1);
+  if (!(KO(16))) process_tile<REV, FWD, kBThreads>(P, A, T, St, ev_s, gp, dq3);
+  if (KO(256)) __syncthreads();   // (diagnostics: the flush of every warp is done)
+  stamp(P, tix, 5);
   if (threadIdx.x == 0) bulk_wait_read();   // the stage must outlive the bulk stores' reads
 }
 
@@ -1412,6 +1525,9 @@ static inline int cdiv(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
 static int g_num_sms = 148;
 
 size_t tile_smem_bytes() { return kBSmemBytes; }
+int read_tile_prof(long long* out, int n) {   // diagnostics (DGR_DEBUG_SKIP bit 256)
+  return (int)cudaMemcpyFromSymbol(out, g_tile_prof, sizeof(long long) * 8 * (size_t)(n < kProfTiles ? n : kProfTiles));
+}
 
 int prepare_kernels() {
   int dev = 0;
