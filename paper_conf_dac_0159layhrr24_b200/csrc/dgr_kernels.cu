@@ -700,6 +700,13 @@ __device__ __forceinline__ void st_stream2(float2* p, float2 v, uint64_t pol) {
   if (!DGR_L2_HINTS) { *p = v; return; }
   asm volatile("st.global.L2::cache_hint.v2.f32 [%0], {%1, %2}, %3;" ::"l"(p), "f"(v.x), "f"(v.y), "l"(pol) : "memory");
 }
+// Programmatic dependent launch: KBF and KG are launched with programmatic stream serialization,
+// so the next kernel's CTAs are scheduled into the slots the previous kernel's last wave leaves
+// free; each waits here (griddepcontrol.wait: the previous grid has completed and its writes are
+// visible) before it touches anything that grid writes.
+__device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void griddep_launch() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 __device__ __forceinline__ void prefetch_l2(const void* src, uint32_t bytes) {
   if (bytes) asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
 }
@@ -1125,7 +1132,9 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
   Stage St(smem);
   int* dq3 = reinterpret_cast<int*>(smem + StageLayout::bytes);
   uint64_t* bar = reinterpret_cast<uint64_t*>(dq3 + 3 * kPipeTrees);
+  griddep_launch();
   if ((int)blockIdx.x < P.ntiles_slow) {   // global tiles first: the longest CTAs start earliest
+    griddep_wait();
     slow_tile<REV, FWD>(P, A, P.tiles_slow[blockIdx.x], smem);
     return;
   }
@@ -1149,6 +1158,7 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
   }
   for (int i = threadIdx.x; i < 3 * kPipeTrees; i += kBThreads) dq3[i] = 0;
   __syncthreads();
+  griddep_wait();   // S, logits, q and the event grids come from the previous kernels
 #if DGR_LSU_STAGE
   if (threadIdx.x < 32 && (P.pf & 1)) prefetch_tile(P, T);
   lsu_tile_loads<REV, kBThreads>(P, T, smem);
@@ -1280,6 +1290,8 @@ __global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A)
   __shared__ double shd[33];
   __shared__ double shw[kKgWarps];
   __shared__ long long shwl[2 * kKgWarps];
+  griddep_launch();
+  griddep_wait();   // the difference arrays are complete (the previous KBF / allreduce)
   const int line = blockIdx.x;
   const bool isH = line < P.Y;
   const int n = isH ? P.X : P.Y;
@@ -1542,17 +1554,36 @@ int prepare_kernels() {
   return (int)e;
 }
 
+#ifndef DGR_PDL
+#define DGR_PDL 1
+#endif
+static cudaLaunchConfig_t pdl_config(int grid, int block, size_t smem, cudaStream_t s, cudaLaunchAttribute* attr) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(block);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  attr->id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr->val.programmaticStreamSerializationAllowed = DGR_PDL;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cfg;
+}
 void launch_tiles(const KParams& p, const StepArgs& a, TileMode mode, cudaStream_t s) {
   // one launch: global tiles in the first CTAs (the longest start earliest), then the pipelined tiles
   const int grid = p.ntiles + p.ntiles_slow;
   if (grid == 0) return;
-  if (mode == kForwardOnly) tile_bulk<false, true><<<grid, kBThreads, kBSmemBytes, s>>>(p, a);
-  else if (mode == kReverseForward) tile_bulk<true, true><<<grid, kBThreads, kBSmemBytes, s>>>(p, a);
-  else tile_bulk<true, false><<<grid, kBThreads, kBSmemBytes, s>>>(p, a);
+  cudaLaunchAttribute attr;
+  cudaLaunchConfig_t cfg = pdl_config(grid, kBThreads, kBSmemBytes, s, &attr);
+  if (mode == kForwardOnly) cudaLaunchKernelEx(&cfg, tile_bulk<false, true>, p, a);
+  else if (mode == kReverseForward) cudaLaunchKernelEx(&cfg, tile_bulk<true, true>, p, a);
+  else cudaLaunchKernelEx(&cfg, tile_bulk<true, false>, p, a);
 }
 void launch_kg_loss(const KParams& p, const StepArgs& a, cudaStream_t s) { kg_loss_kernel<<<1, 256, 0, s>>>(p, a); }
 void launch_kg(const KParams& p, const StepArgs& a, cudaStream_t s) {
-  kg_kernel<<<p.X + p.Y, kGThreads, 0, s>>>(p, a);
+  cudaLaunchAttribute attr;
+  cudaLaunchConfig_t cfg = pdl_config(p.X + p.Y, kGThreads, 0, s, &attr);
+  cudaLaunchKernelEx(&cfg, kg_kernel, p, a);
 }
 int induce_metric_blocks(const KParams& p) {
   const int64_t ncell = (int64_t)p.X * p.Y;
