@@ -48,9 +48,18 @@ constexpr int kMaxBundles = 64;                    // bundles per tile (a whole 
 constexpr int kTargetBundles = DGR_TARGET_BUNDLES;  // group bundles per pipelined tile
 constexpr int kTileBundles = kTargetBundles + 8;   // all bundles (group + singleton) per pipelined tile
 constexpr int kTreeMax = 512;                      // trees per tile
-constexpr int kPipeTrees = 224;                    // trees per pipelined tile
-constexpr int kPipeSubs = 512;                     // sub-nets per pipelined tile
-constexpr int kKgWarps = 8;                        // warps per KG CTA (one line per CTA)
+#ifndef DGR_PIPE_TREES
+#define DGR_PIPE_TREES 224
+#endif
+constexpr int kPipeTrees = DGR_PIPE_TREES;         // trees per pipelined tile
+#ifndef DGR_PIPE_SUBS
+#define DGR_PIPE_SUBS 512
+#endif
+constexpr int kPipeSubs = DGR_PIPE_SUBS;           // sub-nets per pipelined tile
+#ifndef DGR_KG_WARPS
+#define DGR_KG_WARPS 8
+#endif
+constexpr int kKgWarps = DGR_KG_WARPS;             // warps per KG CTA (one line per CTA)
 constexpr int kEventMax = 127;                     // events per window cell-field (int32 safety)
 
 enum Shape : uint32_t {

@@ -1185,7 +1185,10 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
 // The line's difference and turning-point entries are cleared for the next forward.
 // ------------------------------------------------------------------------------------------
 constexpr int kGThreads = 32 * kKgWarps;
-constexpr int kGItems = 4;
+#ifndef DGR_KG_ITEMS
+#define DGR_KG_ITEMS 4
+#endif
+constexpr int kGItems = DGR_KG_ITEMS;
 
 template <typename T>
 __device__ __forceinline__ T block_exclusive_scan(T v, T* sh, T* total) {
@@ -1285,7 +1288,10 @@ __global__ void __launch_bounds__(256) kg_loss_kernel(KParams P, StepArgs A) {
   }
 }
 
-__global__ void __launch_bounds__(kGThreads, 4) kg_kernel(KParams P, StepArgs A) {
+#ifndef DGR_KG_MINB
+#define DGR_KG_MINB 4
+#endif
+__global__ void __launch_bounds__(kGThreads, DGR_KG_MINB) kg_kernel(KParams P, StepArgs A) {
   __shared__ long long shl[33];
   __shared__ double shd[33];
   __shared__ double shw[kKgWarps];
