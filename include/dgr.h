@@ -149,6 +149,16 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
 int dgr_step(struct dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w,
              dgr_loss* last);
 
+/* dgr_step without host synchronisation: the same iterations, then a stream-ordered copy of the
+ * loss of the last forward (4 doubles: total, wl, via, overflow, as dgr_loss) into loss_out
+ * (host memory, caller-owned; pinned memory keeps the call asynchronous).  loss_out is valid
+ * after dgr_sync or any synchronising call on the handle.  NULL loss_out: DGR_EINVAL. */
+int dgr_step_async(struct dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w,
+                   double* loss_out);
+
+/* Waits for all work the handle has enqueued on its stream. */
+int dgr_sync(struct dgr_handle* h);
+
 /* Demand d_e (Eq. 10) of the last forward, full grids [Y][X] (H padding column / V padding
  * row are 0).  With world > 1 this is the global (all-rank) demand.  Synchronises. */
 int dgr_get_demand(struct dgr_handle* h, float* d_h, float* d_v);

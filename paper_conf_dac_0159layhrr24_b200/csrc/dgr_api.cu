@@ -1059,7 +1059,29 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   return DGR_OK;
 }
 
+static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w, dgr_loss* last,
+                     double* loss_async);
+
 int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w, dgr_loss* last) {
+  return step_impl(h, iters, temperature, lr, w, last, nullptr);
+}
+
+int dgr_step_async(dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w,
+                   double* loss_out) {
+  g_err.clear();
+  if (!loss_out) return fail(DGR_EINVAL, "NULL loss_out");
+  return step_impl(h, iters, temperature, lr, w, nullptr, loss_out);
+}
+
+int dgr_sync(dgr_handle* h) {
+  g_err.clear();
+  if (!h) return fail(DGR_EINVAL, "NULL handle");
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return DGR_OK;
+}
+
+static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w, dgr_loss* last,
+                     double* loss_async) {
   g_err.clear();
   if (!h || !w) return fail(DGR_EINVAL, "NULL handle or weights");
   if (!h->ws) return fail(DGR_ESTATE, "no workspace bound (dgr_bind_workspace)");
@@ -1141,6 +1163,8 @@ int dgr_step(dgr_handle* h, int32_t iters, float temperature, float lr, const dg
   h->t_last = temperature;
   h->beta_last = w->beta_via;
   h->have_forward = true;
+  if (loss_async)   // stream-ordered read of this call's loss; no host synchronisation
+    CUDA_TRY(cudaMemcpyAsync(loss_async, P.loss, 4 * sizeof(double), cudaMemcpyDeviceToHost, s));
   if (last) {
     CUDA_TRY(cudaMemcpyAsync(h->pinned, P.loss, 4 * sizeof(double), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));

@@ -1261,30 +1261,48 @@ __device__ __forceinline__ void striped_exclusive_scan(T (&v)[kGItems], T* sh /*
 
 // The loss of the last KG launch (Eqs. (9), (11), (12)): sums of the per-line partials in line
 // order (deterministic).  One CTA, launched once per dgr_step call after its last KG.
-__global__ void __launch_bounds__(256) kg_loss_kernel(KParams P, StepArgs A) {
-  __shared__ double sh[33];
-  __shared__ long long shl[33];
-  const int nl = P.X + P.Y;
+__global__ void __launch_bounds__(1024) kg_loss_kernel(KParams P, StepArgs A) {
+  // fixed-shape tree reduction (strided thread sums, warp shuffles, warp totals in warp order):
+  // deterministic, one pass, no block scans
+  __shared__ double shs[32];
+  __shared__ long long shw[32], sht[32];
+  const int nl = P.X + P.Y, lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   double s = 0.0;
   long long w = 0, t = 0;
   for (int i = threadIdx.x; i < nl; i += blockDim.x) {
     s += P.partial[i];
-    w += P.lpart[2 * i];
-    t += P.lpart[2 * i + 1];
+    const longlong2 l = reinterpret_cast<const longlong2*>(P.lpart)[i];
+    w += l.x;
+    t += l.y;
   }
-  double tot;
-  long long wt, tt;
-  block_exclusive_scan(s, sh, &tot);
-  block_exclusive_scan(w, shl, &wt);
-  block_exclusive_scan(t, shl, &tt);
-  if (threadIdx.x == 0) {
-    const double ewl = (double)wt * kFixInv;
-    const double etp = (double)tt * kFixInv;
-    const double via = (double)A.sqrt_l * etp;
-    P.loss[0] = (double)A.a_wl * ewl + (double)A.a_via * via + (double)A.a_of * tot;
-    P.loss[1] = ewl;
-    P.loss[2] = via;
-    P.loss[3] = tot;
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {
+    s += __shfl_down_sync(kFull, s, off);
+    w += __shfl_down_sync(kFull, w, off);
+    t += __shfl_down_sync(kFull, t, off);
+  }
+  if (lane == 0) { shs[wid] = s; shw[wid] = w; sht[wid] = t; }
+  __syncthreads();
+  if (wid == 0) {
+    const int nw = blockDim.x >> 5;
+    s = lane < nw ? shs[lane] : 0.0;
+    w = lane < nw ? shw[lane] : 0;
+    t = lane < nw ? sht[lane] : 0;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+      s += __shfl_down_sync(kFull, s, off);
+      w += __shfl_down_sync(kFull, w, off);
+      t += __shfl_down_sync(kFull, t, off);
+    }
+    if (lane == 0) {
+      const double ewl = (double)w * kFixInv;
+      const double etp = (double)t * kFixInv;
+      const double via = (double)A.sqrt_l * etp;
+      P.loss[0] = (double)A.a_wl * ewl + (double)A.a_via * via + (double)A.a_of * s;
+      P.loss[1] = ewl;
+      P.loss[2] = via;
+      P.loss[3] = s;
+    }
   }
 }
 
@@ -1585,7 +1603,7 @@ void launch_tiles(const KParams& p, const StepArgs& a, TileMode mode, cudaStream
   else if (mode == kReverseForward) cudaLaunchKernelEx(&cfg, tile_bulk<true, true>, p, a);
   else cudaLaunchKernelEx(&cfg, tile_bulk<true, false>, p, a);
 }
-void launch_kg_loss(const KParams& p, const StepArgs& a, cudaStream_t s) { kg_loss_kernel<<<1, 256, 0, s>>>(p, a); }
+void launch_kg_loss(const KParams& p, const StepArgs& a, cudaStream_t s) { kg_loss_kernel<<<1, 1024, 0, s>>>(p, a); }
 void launch_kg(const KParams& p, const StepArgs& a, cudaStream_t s) {
   cudaLaunchAttribute attr;
   cudaLaunchConfig_t cfg = pdl_config(p.X + p.Y, kGThreads, 0, s, &attr);

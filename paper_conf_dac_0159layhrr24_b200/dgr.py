@@ -102,6 +102,8 @@ def load_library():
     L.dgr_handle_workspace_size.restype = c.c_int64
     L.dgr_bind_workspace.argtypes = [vp, c.POINTER(_Desc), c.POINTER(_Dist), vp, c.c_int64]
     L.dgr_step.argtypes = [vp, c.c_int32, c.c_float, c.c_float, c.POINTER(Weights), c.POINTER(Loss)]
+    L.dgr_step_async.argtypes = [vp, c.c_int32, c.c_float, c.c_float, c.POINTER(Weights), c.POINTER(c.c_double)]
+    L.dgr_sync.argtypes = [vp]
     L.dgr_get_demand.argtypes = [vp, _PF, _PF]
     L.dgr_get_logits.argtypes = [vp, _PF, _PF]
     L.dgr_induce.argtypes = [vp, c.c_float, _P32, _P32, _P64, _P32, _P32, _P32, c.POINTER(c.c_double)]
@@ -117,7 +119,7 @@ def load_library():
     for fn in ("dgr_build_forest", "dgr_built_forest_sizes", "dgr_built_forest_download", "dgr_built_forest_free"):
         getattr(L, fn).restype = c.c_int
     for fn in ("dgr_nccl_unique_id", "dgr_partition", "dgr_forest_load", "dgr_forest_plan", "dgr_bind_workspace",
-               "dgr_step", "dgr_get_demand",
+               "dgr_step", "dgr_step_async", "dgr_sync", "dgr_get_demand",
                "dgr_get_logits", "dgr_induce", "dgr_get_info", "dgr_free", "dgr_profile", "dgr_profile_read", "dgr_plan_info"):
         getattr(L, fn).restype = c.c_int
     _lib = L
@@ -258,6 +260,18 @@ class Solver:
         _check(load_library().dgr_step(self._h, int(iters), float(temperature), float(lr), ctypes.byref(w),
                                        ctypes.byref(loss) if want_loss else None))
         return loss.as_array() if want_loss else None
+
+    def step_async(self, iters: int, temperature: float, lr: float, weights: Weights | None,
+                   loss_out: np.ndarray):
+        """dgr_step_async: enqueue the iterations and a copy of their last loss into loss_out (4 float64,
+        host memory, ideally pinned); valid after sync()."""
+        assert loss_out.dtype == np.float64 and loss_out.size >= 4 and loss_out.flags.c_contiguous
+        w = weights if weights is not None else Weights()
+        _check(load_library().dgr_step_async(self._h, int(iters), float(temperature), float(lr), ctypes.byref(w),
+                                             loss_out.ctypes.data_as(ctypes.POINTER(ctypes.c_double))))
+
+    def sync(self):
+        _check(load_library().dgr_sync(self._h))
 
     def demand(self):
         dh = np.zeros((self.Y, self.X), np.float32); dv = np.zeros((self.Y, self.X), np.float32)

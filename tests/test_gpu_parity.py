@@ -209,6 +209,19 @@ def test_split_calls_and_determinism(forests):
     assert all(np.array_equal(x, y) for x, y in zip(a.demand(), b.demand()))
 
 
+def test_step_async_equals_step(forests):
+    """dgr_step_async (no host sync, loss copied stream-ordered) is dgr_step: same losses, same state."""
+    f = forests["c1e4"]
+    a = dgr.Solver(f); b = dgr.Solver(f)
+    la = np.array([a.step(1, 0.9, 0.3) for _ in range(5)])
+    lb = np.zeros((5, 4))
+    for i in range(5):
+        b.step_async(1, 0.9, 0.3, None, lb[i])
+    b.sync()
+    assert np.array_equal(la, lb)
+    assert np.array_equal(a.logits()[1], b.logits()[1]) and np.array_equal(a.logits()[0], b.logits()[0])
+
+
 @pytest.mark.parametrize("name", ["tiny", "c1e4", "c1e4_c"])
 def test_induce_parity(forests, name):
     f = forests[name]
