@@ -740,14 +740,15 @@ __device__ __forceinline__ void tile_ranges(const TileDesc& T, int& s_lo, int& s
 
 // warp 0 issues the bulk copies of tile T into stage `st`, completing on `bar`
 template <bool REV>
-__device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDesc& T, unsigned char* st, uint64_t* bar) {
+__device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDesc& T, unsigned char* st, uint64_t* bar,
+                                                 bool window = true) {
   const int lane = threadIdx.x & 31;
   Stage S(st);
   int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
   const int mn_lo = T.mn0 & ~3, mn_hi = (T.mn0 + T.nmn + 3) & ~3;
   const uint32_t slot_bytes = (uint32_t)T.nb * 128u, gslot_bytes = (uint32_t)T.nbg * 128u;
-  const bool sw = REV && !(KO(32));   // knock-out 32: no S window (timing only)
+  const bool sw = REV && window && !(KO(32));   // knock-out 32: no S window (timing only)
   const uint32_t nrow = sw ? (uint32_t)T.wh : 0u, ncol = sw ? (uint32_t)T.ww : 0u;
   const uint32_t bytes = slot_bytes + gslot_bytes + 16u * T.nb + 8u * (s_hi - s_lo) + 4u * (n_hi - n_lo) +
                          4u * (mn_hi - mn_lo) + 8u * (t_hi - t_lo) + 8u * (nrow * T.ww + ncol * T.wh);
@@ -792,14 +793,15 @@ __device__ __forceinline__ void cp_copy(void* dst, const void* src, uint32_t byt
   for (uint32_t o = 16u * lane; o < bytes; o += 512u) cp16(d + o, g + o);
 }
 template <bool REV, int NT>
-__device__ __forceinline__ void lsu_tile_loads(const KParams& P, const TileDesc& T, unsigned char* st) {
+__device__ __forceinline__ void lsu_tile_loads(const KParams& P, const TileDesc& T, unsigned char* st,
+                                               bool arrays = true) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   Stage S(st);
   int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
   const int mn_lo = T.mn0 & ~3, mn_hi = (T.mn0 + T.nmn + 3) & ~3;
   const size_t s0 = (size_t)T.b0 * 32;
-  switch (warp & 7) {
+  if (arrays) switch (warp & 7) {
     case 0: cp_copy(S.pw, P.pword + s0, (uint32_t)T.nb * 128u, lane); break;
     case 1: cp_copy(S.w, P.wp + s0, (uint32_t)T.nbg * 128u, lane); break;
     case 2: cp_copy(S.bi, P.binfo + T.b0, 16u * T.nb, lane); break;
@@ -1116,7 +1118,8 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
 #endif
 constexpr int kBThreads = DGR_BTHREADS;
 #ifndef DGR_LSU_STAGE
-#define DGR_LSU_STAGE 1   // stage filled by cp.async (1) or by cp.async.bulk on an mbarrier (0)
+#define DGR_LSU_STAGE 2   // stage: 1-D arrays by bulk copies + S window by cp.async (2), all by
+                          // cp.async (1), all by cp.async.bulk on an mbarrier (0)
 #endif
 #ifndef DGR_BPERSM
 #define DGR_BPERSM 5
@@ -1159,7 +1162,14 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
   for (int i = threadIdx.x; i < 3 * kPipeTrees; i += kBThreads) dq3[i] = 0;
   __syncthreads();
   griddep_wait();   // S, logits, q and the event grids come from the previous kernels
-#if DGR_LSU_STAGE
+#if DGR_LSU_STAGE == 2
+  // the eight 1-D arrays by bulk copies (8 per tile: few and large), the S window by cp.async
+  if (threadIdx.x < 32) issue_tile_loads<REV>(P, T, smem, bar, false);
+  lsu_tile_loads<REV, kBThreads>(P, T, smem, false);
+  asm volatile("cp.async.wait_group 0;" ::: "memory");
+  mbar_wait(bar, 0u);
+  __syncthreads();
+#elif DGR_LSU_STAGE
   if (threadIdx.x < 32 && (P.pf & 1)) prefetch_tile(P, T);
   lsu_tile_loads<REV, kBThreads>(P, T, smem);
   asm volatile("cp.async.wait_group 0;" ::: "memory");
