@@ -79,11 +79,21 @@ typedef struct {
   uint64_t seed;                          /* Philox key of the Gumbel noise */
 } dgr_forest_desc;
 
+/* Caller-supplied exchange (optional, replaces NCCL): an in-place sum over the ranks of `count`
+ * elements at device pointer `buf` (dtype 0 = int64, 1 = int32), ordered after the work already
+ * enqueued on `cuda_stream` and visible to the work enqueued after the call returns.  Returns 0 on
+ * success; any other value makes the calling dgr_* function fail with DGR_ENCCL.  Used to run
+ * several ranks in one process (e.g. on one GPU, for testing the sharded path without NCCL). */
+typedef int (*dgr_allreduce_fn)(void* user, void* buf, int64_t count, int32_t dtype, void* cuda_stream);
+
 /* Multi-GPU: one process per GPU.  rank 0 calls dgr_nccl_unique_id and broadcasts the 128
- * bytes (e.g. over torch.distributed); every rank passes them here. NULL or world == 1: single GPU. */
+ * bytes (e.g. over torch.distributed); every rank passes them here. NULL or world == 1: single GPU.
+ * With `allreduce` non-NULL the ranks exchange through it instead (nccl_unique_id unused). */
 typedef struct {
   int32_t rank, world;
   const void* nccl_unique_id;             /* 128 bytes */
+  dgr_allreduce_fn allreduce;             /* NULL: NCCL */
+  void* allreduce_user;
 } dgr_dist;
 
 /* Cost weights and model constants. */

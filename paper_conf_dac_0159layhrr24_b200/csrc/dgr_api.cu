@@ -708,8 +708,10 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   for (const auto& T : pl.tiles) pl.n_global_tiles += T.global;
   pl.nb = (int)pl.binfo.size();
   // pipelined tiles (shared-memory window and stage) first, then the rest
-  auto pipelined = [](const TileDesc& T) {
-    return !T.global && T.nbg <= kTargetBundles && T.nb <= kTileBundles && T.ntree <= kPipeTrees && T.nsub <= kPipeSubs;
+  const bool all_slow = getenv("DGR_ALL_SLOW") != nullptr;   // diagnostics: every tile on the slow path
+  auto pipelined = [all_slow](const TileDesc& T) {
+    return !all_slow && !T.global && T.nbg <= kTargetBundles && T.nb <= kTileBundles && T.ntree <= kPipeTrees &&
+           T.nsub <= kPipeSubs;
   };
   std::stable_partition(pl.tiles.begin(), pl.tiles.end(), pipelined);
   pl.n_pipe_tiles = 0;
@@ -794,6 +796,8 @@ struct dgr_handle {
   cudaStream_t stream = nullptr;
   int rank = 0, world = 1;
   ncclComm_t comm = nullptr;
+  dgr_allreduce_fn ar_fn = nullptr;   // caller-supplied exchange instead of NCCL (dgr_dist.allreduce)
+  void* ar_user = nullptr;
   char* ws = nullptr;
   int64_t ws_bytes = 0;
   int64_t k = 0;
@@ -854,6 +858,16 @@ int dgr_partition(const dgr_forest_desc* desc, int32_t world, int64_t* out) {
   return DGR_OK;
 }
 
+// in-place sum over the ranks on the handle's stream: NCCL, or the caller's exchange
+static int allreduce(dgr_handle* h, void* buf, int64_t count, int dtype) {
+  if (h->ar_fn) {
+    const int r = h->ar_fn(h->ar_user, buf, count, dtype, (void*)h->stream);
+    return r ? fail(DGR_ENCCL, "allreduce callback returned %d", r) : DGR_OK;
+  }
+  NCCL_TRY(ncclAllReduce(buf, buf, (size_t)count, dtype ? ncclInt32 : ncclInt64, ncclSum, h->comm, h->stream));
+  return DGR_OK;
+}
+
 static int dist_args(const dgr_dist* dist, int* rank, int* world) {
   *rank = 0;
   *world = 1;
@@ -862,7 +876,8 @@ static int dist_args(const dgr_dist* dist, int* rank, int* world) {
     *world = dist->world;
   }
   if (*world < 1 || *rank < 0 || *rank >= *world) return fail(DGR_EINVAL, "bad rank/world %d/%d", *rank, *world);
-  if (*world > 1 && (!dist || !dist->nccl_unique_id)) return fail(DGR_EINVAL, "world > 1 needs an NCCL unique id");
+  if (*world > 1 && (!dist || (!dist->nccl_unique_id && !dist->allreduce)))
+    return fail(DGR_EINVAL, "world > 1 needs an NCCL unique id or an allreduce callback");
   return DGR_OK;
 }
 
@@ -1048,7 +1063,10 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   tm.mark("bind: upload");
   if (e != cudaSuccess) return cleanup(fail(DGR_ECUDA, "upload: %s", cudaGetErrorString(e)));
   if (cudaMallocHost(&h->pinned, 16 * sizeof(double)) != cudaSuccess) return cleanup(fail(DGR_ECUDA, "cudaMallocHost failed"));
-  if (world > 1) {
+  if (world > 1 && dist->allreduce) {
+    h->ar_fn = dist->allreduce;
+    h->ar_user = dist->allreduce_user;
+  } else if (world > 1) {
     ncclUniqueId id;
     memcpy(&id, dist->nccl_unique_id, sizeof(id));
     ncclResult_t r = ncclCommInitRank(&h->comm, world, id, rank);
@@ -1129,7 +1147,7 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
     a.store_d = last;
     adam_args(h->k);
     if (h->world > 1) {
-      NCCL_TRY(ncclAllReduce(P.dH, P.dH, h->lay.xcount, ncclInt64, ncclSum, h->comm, s));
+      if ((rc = allreduce(h, P.dH, (int64_t)h->lay.xcount, 0))) return rc;
       if ((rc = prof_mark(h, 1))) return rc;
     }
     launch_kg(P, a, s);
@@ -1226,8 +1244,9 @@ int dgr_induce(dgr_handle* h, float top_p, int32_t* tree_choice, int32_t* route,
   CUDA_TRY(cudaMemsetAsync(P.iscal, 0, 16, s));
   launch_induce(P, h->t_last, top_p, h->beta_last, s);
   if (h->world > 1) {
-    NCCL_TRY(ncclAllReduce(P.DH, P.DH, 3 * G, ncclInt32, ncclSum, h->comm, s));
-    NCCL_TRY(ncclAllReduce(P.iscal, P.iscal, 2, ncclInt64, ncclSum, h->comm, s));
+    int rc;
+    if ((rc = allreduce(h, P.DH, (int64_t)(3 * G), 1))) return rc;
+    if ((rc = allreduce(h, P.iscal, 2, 0))) return rc;
   }
   launch_induce_metrics(P, h->beta_last, s);
   CUDA_TRY(cudaGetLastError());

@@ -62,13 +62,17 @@ __device__ __forceinline__ uint4 philox_rk(uint4 c, const uint32_t* rk) {
   return c;
 }
 
+// g = -ln(-ln u) from one Philox word (the outer log by MUFU: |error| < 1e-6 on g)
+__device__ __forceinline__ float gumbel_word(uint32_t w) {
+  const float u = ((float)(w >> 9) + 0.5f) * (1.0f / 8388608.0f);
+  return -__logf(-logf(u));
+}
+
 __device__ __forceinline__ float gumbel(uint64_t seed, uint64_t idx, uint32_t k, uint32_t stream) {
   const uint4 r = philox4x32_10(make_uint4((uint32_t)(idx >> 2), (uint32_t)(idx >> 34), k, stream),
                                 make_uint2((uint32_t)seed, (uint32_t)(seed >> 32)));
   const uint32_t s = (uint32_t)idx & 3u;
-  const uint32_t w = s == 0 ? r.x : (s == 1 ? r.y : (s == 2 ? r.z : r.w));
-  const float u = ((float)(w >> 9) + 0.5f) * (1.0f / 8388608.0f);
-  return -logf(-logf(u));
+  return gumbel_word(s == 0 ? r.x : (s == 1 ? r.y : (s == 2 ? r.z : r.w)));
 }
 
 // ------------------------------------------------------------------------------------------
@@ -242,11 +246,6 @@ __device__ __forceinline__ void c_events(uint32_t pw, int x0, int y0, int x1, in
   }
 }
 
-// g = -ln(-ln u) from one Philox word
-__device__ __forceinline__ float gumbel_word(uint32_t w) {
-  const float u = ((float)(w >> 9) + 0.5f) * (1.0f / 8388608.0f);
-  return -__logf(-logf(u));   // outer log: MUFU approximation, |error| < 1e-6 on g
-}
 
 // Gumbel noise of a warp's contiguous candidates gid0 .. gid0+n-1 into g[0..n): one Philox4x32-10
 // call per 4 consecutive candidates (counter gid >> 2), spread over the lanes.
@@ -343,27 +342,33 @@ __device__ __forceinline__ void reverse_warp(const KParams& P, const StepArgs& A
     // softmax backward dw_i = (p_i/t)(dp_i - sum_k p_k dp_k / sum_k p_k): differences to the group
     // head's dp are formed in fp64 and reduced in fp32, so neither the magnitude of c nor
     // sum_k p_k != 1 (rounding) leaks into dw.
-    const double dp = (double)q * c;
-    const double dref = __shfl_sync(kFull, dp, L.head);
-    const float dd = (float)(dp - dref);
-    float sa = seg_reduce(p * dd, L.lane, L.end, Sum());
-    float sb = seg_reduce(p, L.lane, L.end, Sum());
-    sa = __shfl_sync(kFull, sa, L.head);
-    sb = __shfl_sync(kFull, sb, L.head);
-    const float dw = L.valid ? p * A.inv_t * (dd - __fdividef(sa, sb)) : 0.f;
-    // dq_j = sum_{i in tree j} p_i c_i: reduce over this warp's lanes of each tree (fp64: the tree
-    // gradient is a difference of such sums)
-    const uint32_t th = L.tm | __ballot_sync(kFull, !L.valid) | 1u;
-    const uint32_t trest = th & ~L.le;
-    const int tend = trest ? (__ffs(trest) - 2) : 31;
-    const double pc = seg_reduce(L.valid ? (double)p * c : 0.0, L.lane, tend, Sum());
-    if (L.valid && ((th >> L.lane) & 1u))
-      atomicAdd(reinterpret_cast<unsigned long long*>(&dq_s[L.tree - T.tree0]),
-                static_cast<unsigned long long>(__double2ll_rn(pc * kDqScale)));
-    if (L.valid) {
-      adam_update(w, m, v, dw, A);
-      P.wp[slot] = w;
-      P.mv[slot] = make_float2(m, v);
+    // exactly the arithmetic of process_tile (pipelined tiles), so that a net gives bit-identical
+    // results whichever kind of tile it lands in (tile composition depends on the rank count):
+    if (L.single) {
+      // singleton bundle (lone straight sub-nets, p = 1): tree-run sums of c into dq; no Adam (the
+      // logit of a lone straight candidate never changes)
+      const uint32_t th = __ballot_sync(kFull, (L.pw & kTreeHead) || !L.valid) | 1u;
+      const uint32_t trest = th & ~L.le;
+      const int tend = trest ? (__ffs(trest) - 2) : 31;
+      const long long pc = seg_reduce(L.valid ? __double2ll_rn(c * kDqScale) : 0ll, L.lane, tend, Sum());
+      if (L.valid && ((th >> L.lane) & 1u))
+        atomicAdd(reinterpret_cast<unsigned long long*>(&dq_s[L.tree - T.tree0]), static_cast<unsigned long long>(pc));
+    } else {
+      // softmax backward over the sub-net with dd = c - c_head (fp64 difference, then fp32):
+      // dw_i = (p_i / t) q (dd_i - sum_k p_k dd_k); the head adds c_head + sum_k p_k dd_k to dq
+      const double ch = __shfl_sync(kFull, c, L.head);
+      const float dd = (float)(c - ch);
+      float sa = seg_reduce(p * dd, L.lane, L.end, Sum());
+      sa = __shfl_sync(kFull, sa, L.head);
+      const float dw = L.valid ? p * A.inv_t * q * (dd - sa) : 0.f;
+      if (L.valid && L.lane == L.head)
+        atomicAdd(reinterpret_cast<unsigned long long*>(&dq_s[L.tree - T.tree0]),
+                  static_cast<unsigned long long>(__double2ll_rn((c + (double)sa) * kDqScale)));
+      if (L.valid) {
+        adam_update(w, m, v, dw, A);
+        P.wp[slot] = w;
+        P.mv[slot] = make_float2(m, v);
+      }
     }
     wst[(b - T.b0) * 32 + lane] = w;
     L = Ln; e = en; w = wn; m = mn; v = vn; p = pn;
@@ -557,10 +562,13 @@ __device__ __forceinline__ void slow_tile(const KParams& P, const StepArgs& A, c
           q_s[j - T.tree0] = z;
           zmax = fmaxf(zmax, z);
         }
-        float s = 0.f;
-        for (int j = a; j < b; ++j) { const float e = __expf(q_s[j - T.tree0] - zmax); q_s[j - T.tree0] = e; s += e; }
-        const float inv = 1.f / s;
-        for (int j = a; j < b; ++j) { q_s[j - T.tree0] *= inv; P.q[j] = q_s[j - T.tree0]; }
+        float sum = 0.f;   // the normalisation of process_tile, operation for operation
+        for (int j = a; j < b; ++j) sum += __expf(q_s[j - T.tree0] - zmax);
+        for (int j = a; j < b; ++j) {
+          const float q = __expf(q_s[j - T.tree0] - zmax) / sum;
+          q_s[j - T.tree0] = q;
+          P.q[j] = q;
+        }
       }
     }
   }
@@ -928,9 +936,10 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         const uint32_t le = kFull >> (31 - lane);
         const uint32_t trest = th & ~le;
         const int tend = trest ? (__ffs(trest) - 2) : 31;
-        const double pc = seg_reduce(c, lane, tend, Sum());
-        if (valid && ((th >> lane) & 1u))
-          dq_add(dq3, tree - T.tree0, __double2ll_rn(pc * kDqScale));
+        // each c rounded to the 2^-32 fixed point of dq BEFORE the tree-run sum: the run's split over
+        // singleton bundles depends on the tile (and so on the rank count), integer sums do not
+        const long long pc = seg_reduce(valid ? __double2ll_rn(c * kDqScale) : 0ll, lane, tend, Sum());
+        if (valid && ((th >> lane) & 1u)) dq_add(dq3, tree - T.tree0, pc);
       }
     }
     __syncthreads();

@@ -45,8 +45,13 @@ class _PinsDesc(ctypes.Structure):
                 ("z_cap", ctypes.c_int32), ("seed", ctypes.c_uint64), ("c_cap", ctypes.c_int32)]
 
 
+ALLREDUCE_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32,
+                                ctypes.c_void_p)
+
+
 class _Dist(ctypes.Structure):
-    _fields_ = [("rank", ctypes.c_int32), ("world", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p)]
+    _fields_ = [("rank", ctypes.c_int32), ("world", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p),
+                ("allreduce", ALLREDUCE_FN), ("allreduce_user", ctypes.c_void_p)]
 
 
 F_KINDS = {"sigmoid": 0, "relu": 1, "leaky_relu": 2, "exp": 3, "celu": 4}
@@ -218,7 +223,10 @@ class Solver:
     """One rank's DGR solver over a forest (any object with forestgen.Forest's fields)."""
 
     def __init__(self, forest, rank: int = 0, world: int = 1, nccl_id: bytes | None = None, device=None,
-                 stream=None):
+                 stream=None, allreduce=None):
+        """allreduce: optional Python callable (buf_ptr, count, dtype, stream_ptr) -> int replacing NCCL
+        (dgr_dist.allreduce): sums `count` int64 (dtype 0) / int32 (dtype 1) elements at device address
+        buf_ptr over the ranks in place, after the work on stream_ptr."""
         import torch
         if not torch.cuda.is_available():
             raise DgrError("libdgr needs a CUDA device (no CPU fallback)")
@@ -232,7 +240,11 @@ class Solver:
         self.n_subnets, self.n_paths = self._d.n_subnets, self._d.n_paths
         self._idbuf = None
         dist = None
-        if world > 1:
+        self._ar = None
+        if world > 1 and allreduce is not None:
+            self._ar = ALLREDUCE_FN(lambda _u, buf, n, dt, st: int(allreduce(buf, n, dt, st)))
+            dist = _Dist(rank, world, None, self._ar, None)
+        elif world > 1:
             if nccl_id is None or len(nccl_id) != 128:
                 raise DgrError("world > 1 needs the 128-byte NCCL unique id from rank 0")
             self._idbuf = ctypes.create_string_buffer(nccl_id, 128)

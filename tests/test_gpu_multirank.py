@@ -1,0 +1,147 @@
+"""The sharded (world > 1) device path on one GPU: R ranks in one process, one thread per rank, the
+demand exchange done by a caller-supplied allreduce (dgr_dist.allreduce) instead of NCCL.
+
+SURVEY §8(e) / DESIGN.md §7: nets are sharded over the ranks (dgr_partition), Gumbel noise is keyed
+on global indices and the exchanged demand is exact fixed point, so every rank count must reproduce
+the single-rank run BIT-EXACTLY: demand grids, loss, every logit (each from the rank that owns it),
+induced tree choices / routes / integer grids / metrics.  This exercises everything of the NCCL path
+except NCCL itself (which needs one process per GPU).
+"""
+import threading
+
+import numpy as np
+import pytest
+
+import forestgen
+import paper_conf_dac_0159layhrr24_b200 as dgr
+
+pytestmark = pytest.mark.gpu
+
+
+class _DevArray:
+    """A device buffer of the library as a torch tensor (CUDA array interface, no copy)."""
+
+    def __init__(self, ptr: int, n: int, dtype: int):
+        self.__cuda_array_interface__ = {"shape": (int(n),), "typestr": "<i8" if dtype == 0 else "<i4",
+                                         "data": (int(ptr), False), "version": 3}
+
+
+class ThreadAllreduce:
+    """In-place sum over R threads' device buffers: every rank synchronises the device, rank 0 sums
+    the R buffers in rank order and writes the sum back into all of them."""
+
+    def __init__(self, world: int):
+        import torch
+        self.torch = torch
+        self.world = world
+        self.bufs = [None] * world
+        self.barrier = threading.Barrier(world)
+        self.calls = 0
+
+    def for_rank(self, rank: int):
+        def fn(buf, n, dtype, stream):
+            torch = self.torch
+            try:
+                torch.cuda.synchronize()
+                self.bufs[rank] = torch.as_tensor(_DevArray(buf, n, dtype), device="cuda")
+                self.barrier.wait()
+                if rank == 0:
+                    tot = self.bufs[0].clone()
+                    for t in self.bufs[1:]:
+                        tot += t
+                    for t in self.bufs:
+                        t.copy_(tot)
+                    torch.cuda.synchronize()
+                    self.calls += 1
+                self.barrier.wait()
+                return 0
+            except Exception:   # a failing exchange must fail the dgr_* call, not pass silently
+                self.barrier.abort()
+                return 1
+        return fn
+
+
+def _run(solvers, body):
+    out, errs = [None] * len(solvers), []
+
+    def work(r):
+        try:
+            out[r] = body(solvers[r])
+        except Exception as e:   # pragma: no cover - surfaced below
+            errs.append(e)
+
+    th = [threading.Thread(target=work, args=(r,)) for r in range(len(solvers))]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    if errs:
+        raise errs[0]
+    return out
+
+
+def _schedule(s):
+    losses = [s.step(6, 1.0, 0.3), s.step(4, 0.9, 0.3)]
+    return losses, s.demand(), s.logits(), s.induce(0.9)
+
+
+@pytest.mark.parametrize("name,world", [("c1e4", 2), ("c1e4", 3), ("ispd18", 4), ("ispd19", 8)])
+def test_sharded_ranks_reproduce_one_rank_bit_exactly(name, world):
+    f = forestgen.generate(name)
+    ref = dgr.Solver(f)
+    ref_losses, (rdh, rdv), (rwt, rwp), rind = _schedule(ref)
+    ref.close()
+
+    ex = ThreadAllreduce(world)
+    solvers = [dgr.Solver(f, rank=r, world=world, allreduce=ex.for_rank(r)) for r in range(world)]
+    res = _run(solvers, _schedule)
+    assert ex.calls >= 10 + 2, "the exchange ran once per iteration and twice in induction"
+
+    part = dgr.partition(f, world)
+    tree_off, sub_off, path_off = (np.asarray(f.net_tree_off), np.asarray(f.tree_sub_off),
+                                   np.asarray(f.sub_path_off))
+    for r, (losses, (dh, dv), (wt, wp), ind) in enumerate(res):
+        # replicated: the global demand, the loss and the induced grids / metrics of every rank
+        for a, b in zip(losses, ref_losses):
+            assert np.array_equal(a, b), (r, a, b)
+        assert np.array_equal(dh, rdh) and np.array_equal(dv, rdv)
+        assert np.array_equal(ind.D_h, rind.D_h) and np.array_equal(ind.D_v, rind.D_v)
+        assert np.array_equal(ind.metrics, rind.metrics)
+        # rank-local: its nets' tree logits, path logits, tree choices and routes
+        n0, n1 = part[r], part[r + 1]
+        t0, t1 = tree_off[n0], tree_off[n1]
+        s0, s1 = sub_off[t0], sub_off[t1]
+        p0, p1 = path_off[s0], path_off[s1]
+        assert np.array_equal(wt[t0:t1], rwt[t0:t1])
+        assert np.array_equal(wp[p0:p1], rwp[p0:p1])
+        assert np.array_equal(ind.tree_choice[n0:n1], rind.tree_choice[n0:n1])
+        assert np.array_equal(ind.route[s0:s1], rind.route[s0:s1])
+    for s in solvers:
+        s.close()
+
+
+def test_failing_exchange_is_reported():
+    f = forestgen.generate("tiny")
+    solvers = [dgr.Solver(f, rank=r, world=2, allreduce=lambda *a: 7) for r in range(2)]
+    with pytest.raises(dgr.DgrError, match="allreduce callback returned 7"):
+        solvers[0].step(1, 1.0, 0.3)
+    for s in solvers:
+        s.close()
+
+
+def test_slow_tiles_equal_pipelined_tiles(monkeypatch):
+    """A net gives bit-identical results whichever tile kind it lands in (the kind can depend on the
+    tile's composition, hence on the rank count): every tile on the slow / global-memory path
+    (DGR_ALL_SLOW, read at plan time) against the normal plan."""
+    f = forestgen.generate("c1e4")
+    a = dgr.Solver(f)
+    monkeypatch.setenv("DGR_ALL_SLOW", "1")
+    b = dgr.Solver(f)
+    monkeypatch.delenv("DGR_ALL_SLOW")
+    assert b.info()["n_pipe_tiles"] == 0 and a.info()["n_pipe_tiles"] > 0
+    for t in (1.0, 1.0, 0.9):
+        assert np.array_equal(a.step(2, t, 0.3), b.step(2, t, 0.3))
+    assert all(np.array_equal(x, y) for x, y in zip(a.demand(), b.demand()))
+    assert all(np.array_equal(x, y) for x, y in zip(a.logits(), b.logits()))
+    a.close()
+    b.close()
