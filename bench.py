@@ -425,7 +425,7 @@ def main():
                 "d2h_bytes_per_step": d2h / e2e_iters,
                 "note": f"one solve from host CSR arrays through the C ABI: dgr_forest_plan + dgr_bind_workspace "
                         f"(reads {h2d} B of host CSR arrays, validation + encoding + H2D) + {e2e_iters} x dgr_step_async(1) with the loss of each iteration copied to pinned host memory "
-                        f"iteration + dgr_get_demand; wall clock, max over ranks (after one untimed warm-up solve)",
+                        f"+ dgr_get_demand; wall clock, max over ranks (after one untimed warm-up solve)",
                 "split": e2e_split},
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

@@ -588,10 +588,17 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
         }
       }
       int ks = T.sub0;   // next kernel-order sub-net
+      // trees of nets with >= 2 trees (their candidates carry kMultiTree)
+      auto multi_tree = [&](int64_t j) {
+        const int64_t n = std::upper_bound(d->net_tree_off + starts[t], d->net_tree_off + starts[t + 1] + 1, j) -
+                          d->net_tree_off - 1;
+        return d->net_tree_off[n + 1] - d->net_tree_off[n] > 1;
+      };
       // group bundles
       int fill = 32, b = T.b0 - 1, prev_tree = -1;
       for (int64_t j = j0; j < j1; ++j) {
         const int toff = (int)(j - pl.tree_lo) - T.tree0;
+        const uint32_t mt = multi_tree(j) ? kMultiTree : 0u;
         for (int64_t sn = d->tree_sub_off[j]; sn < d->tree_sub_off[j + 1]; ++sn) {
           const int64_t ls = sn - pl.sub_lo;
           if (single[ls]) continue;
@@ -607,7 +614,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
           pl.ksub_csr[ks] = (int32_t)ls;
           pl.sub_first_slot[ls] = (int64_t)b * 32 + fill;
           for (int64_t i = p0; i < p1; ++i) {
-            uint32_t pw = pw_path[i - pl.path_lo] | ((uint32_t)toff << kTreeShift);
+            uint32_t pw = pw_path[i - pl.path_lo] | ((uint32_t)toff << kTreeShift) | mt;
             if (i == p0) {
               pw |= kSubHead;
               if (toff != prev_tree) pw |= kTreeHead;
@@ -622,10 +629,16 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
           ++ks;
         }
       }
-      // singleton bundles
+      // singleton bundles: the lone straight sub-nets of multi-tree nets first, then those of
+      // single-tree nets, so that most singleton bundles have no dq to accumulate (their reverse is
+      // skipped)
       int lane = 32;
       b = T.b0 + T.nbg - 1;
+      for (int pass = 0; pass < 2; ++pass)
       for (int64_t j = j0; j < j1; ++j) {
+        const bool mj = multi_tree(j);
+        if (mj != (pass == 0)) continue;
+        const uint32_t mt = mj ? kMultiTree : 0u;
         const int toff = (int)(j - pl.tree_lo) - T.tree0;
         for (int64_t sn = d->tree_sub_off[j]; sn < d->tree_sub_off[j + 1]; ++sn) {
           const int64_t ls = sn - pl.sub_lo;
@@ -641,7 +654,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
           const int64_t p0 = d->sub_path_off[sn];
           const size_t slot = (size_t)b * 32 + lane;
           pl.sub_first_slot[ls] = (int64_t)slot;
-          pl.pword[slot] = pw_path[p0 - pl.path_lo] | ((uint32_t)toff << kTreeShift) | kSubHead |
+          pl.pword[slot] = pw_path[p0 - pl.path_lo] | ((uint32_t)toff << kTreeShift) | kSubHead | mt |
                            (toff != prev_tree ? kTreeHead : 0u);
           pl.slot_path[slot] = (int32_t)(p0 - pl.path_lo);
           prev_tree = toff;

@@ -69,6 +69,8 @@ constexpr uint32_t kSubHead = 8u;    // lane starts a sub-net group
 constexpr uint32_t kTreeHead = 16u;  // group head whose tree differs from the previous group's in the bundle
 constexpr int kTreeShift = 5;        // bits 5..13: tree of the lane relative to the bundle's tree base
 constexpr uint32_t kTreeMask = 511u;
+constexpr uint32_t kMultiTree = 1u << 15; // the candidate's net has >= 2 trees: its tree's dq is used
+                                           // (a lone tree has du = 0, so its dq is never needed)
 constexpr uint32_t kOutside = 1u << 14;   // Z-HVH / Z-VHV shape whose x_m / y_m lies outside the
                                            // sub-net's span: a C-shape detour (row f4, reading Q14b)
 // bits 16..31: x_m (Z-HVH) or y_m (Z-VHV)

@@ -913,15 +913,16 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         float sa = seg_reduce(p * dd, L.lane, L.end, Sum());
         sa = __shfl_sync(kFull, sa, L.head);
         const float dw = L.valid ? p * A.inv_t * q * (dd - sa) : 0.f;
-        if (L.valid && L.lane == L.head)
+        if (L.valid && L.lane == L.head && (L.pw & kMultiTree))
           dq_add(dq3, L.tree - T.tree0, __double2ll_rn((c + (double)sa) * kDqScale));
         if (L.valid) {
           adam_update(w, m, v, dw, A);
           St.w[sl] = w;
           st_stream2(&P.mv[gsl], make_float2(m, v), pol);
         }
-      } else {
-        // singleton bundle: c of a straight path (one segment, no turning point); p = 1
+      } else if (__any_sync(kFull, pw & kMultiTree)) {
+        // singleton bundle: c of a straight path (one segment, no turning point); p = 1.  Only dq
+        // comes out of it, and only a multi-tree net's dq is used: bundles without one are skipped
         const bool valid = (pw & 7u) != kPad;
         const bool isv = (pw & 7u) == kStraightV;
         const int tree = bi.z + (int)((pw >> kTreeShift) & kTreeMask);
