@@ -67,6 +67,21 @@ def test_workspace_size_of_valid_forest(tiny):
     assert n > 0 and err == ""
 
 
+def test_dist_needs_nccl_id_or_allreduce_callback(tiny):
+    """dgr_dist: world > 1 needs an NCCL id or a caller-supplied allreduce (host-only check)."""
+    lib = dgr.load_library()
+    d = binding._DescHolder(tiny)
+    none = binding._Dist(0, 2, None)
+    assert lib.dgr_workspace_size(ctypes.byref(d.desc), ctypes.byref(none)) == 0   # 0 on error
+    assert "allreduce callback" in lib.dgr_last_error().decode()
+    cb = binding.ALLREDUCE_FN(lambda *a: 0)
+    for r in range(2):
+        ok = binding._Dist(r, 2, None, cb, None)
+        assert lib.dgr_workspace_size(ctypes.byref(d.desc), ctypes.byref(ok)) > 0, lib.dgr_last_error()
+    bad = binding._Dist(2, 2, None, cb, None)
+    assert lib.dgr_workspace_size(ctypes.byref(d.desc), ctypes.byref(bad)) == 0
+
+
 @pytest.mark.parametrize("mutate,msg", [
     (lambda f: f.sub_path_off.__setitem__(3, f.sub_path_off[2]), "empty group"),
     (lambda f: f.net_tree_off.__setitem__(1, 0), "empty group"),
