@@ -8,6 +8,9 @@
 // identical data and the result does not depend on the number of ranks.
 #include <cuda_runtime.h>
 #include <nccl.h>
+#include <cuda.h>
+#include <cudaTypedefs.h>
+#include <map>
 
 #include <algorithm>
 #include <chrono>
@@ -247,6 +250,7 @@ struct Plan {
   std::vector<TileDesc> tiles;          // pipelined tiles first (see make_plan)
   int64_t n_global_tiles = 0;
   int64_t n_pipe_tiles = 0;
+  std::vector<std::pair<int, int>> tmap_shapes;   // (ww, wh) of each tensor-map pair (TileDesc::tmap)
 };
 
 // (cell, field) pairs of one candidate's demand events in the pipelined tile kernel (field 0 dH,
@@ -734,14 +738,74 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       return 4 * a.nbg + (a.nb - a.nbg) > 4 * b.nbg + (b.nb - b.nbg);
     });
   }
+  // one (S_H, S_V) tensor-map pair per distinct window shape of the pipelined tiles (TMA box
+  // extents <= 256); other tiles take their window by cp.async
+  {
+    std::map<std::pair<int, int>, int> idx;
+    const bool no_tma = getenv("DGR_NO_TMA_WINDOW") != nullptr;
+    for (int64_t t = 0; t < (int64_t)pl.tiles.size(); ++t) {
+      TileDesc& T = pl.tiles[t];
+      T.tmap = -1;
+      if (no_tma || t >= pl.n_pipe_tiles || T.ww <= 0 || T.wh <= 0 || T.ww > 256 || T.wh > 256) continue;
+      auto it = idx.find({T.ww, T.wh});
+      if (it == idx.end()) {
+        it = idx.emplace(std::make_pair(T.ww, T.wh), (int)pl.tmap_shapes.size()).first;
+        pl.tmap_shapes.push_back({T.ww, T.wh});
+      }
+      T.tmap = it->second;
+    }
+  }
   return DGR_OK;
+}
+
+// ---------------------------------------------------------------------------------------
+// TMA tensor maps of the tile windows: 2-D views of S_H ([Y][XP] fp64) and S_V^T ([X][YP] fp64)
+// with the window's shape as the box, so one copy per field lands in the kernel's row-major
+// (column-major) window layout.  cuTensorMapEncodeTiled comes from the driver through the runtime's
+// entry-point query (no link against libcuda).
+// ---------------------------------------------------------------------------------------
+int encode_window_maps(const std::vector<std::pair<int, int>>& shapes, const void* SH, const void* SVT, int X, int Y,
+                       unsigned char* out) {
+  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+  if (!encode) {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !fn)
+      return -1;
+    encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  }
+  const cuuint64_t XP = (cuuint64_t)(X + (X & 1)), YP = (cuuint64_t)(Y + (Y & 1));
+  for (size_t i = 0; i < shapes.size(); ++i) {
+    const cuuint32_t ww = (cuuint32_t)shapes[i].first, wh = (cuuint32_t)shapes[i].second;
+    const cuuint32_t es[2] = {1, 1};
+    {   // H field: inner dimension x
+      const cuuint64_t dims[2] = {XP, (cuuint64_t)Y};
+      const cuuint64_t strides[1] = {XP * 8};
+      const cuuint32_t box[2] = {ww, wh};
+      CUresult r = encode(reinterpret_cast<CUtensorMap*>(out + 256 * i), CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2,
+                          const_cast<void*>(SH), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                          CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      if (r != CUDA_SUCCESS) return (int)r;
+    }
+    {   // V field: inner dimension y
+      const cuuint64_t dims[2] = {YP, (cuuint64_t)X};
+      const cuuint64_t strides[1] = {YP * 8};
+      const cuuint32_t box[2] = {wh, ww};
+      CUresult r = encode(reinterpret_cast<CUtensorMap*>(out + 256 * i + 128), CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2,
+                          const_cast<void*>(SVT), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                          CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      if (r != CUDA_SUCCESS) return (int)r;
+    }
+  }
+  return 0;
 }
 
 // ---------------------------------------------------------------------------------------
 // workspace layout
 // ---------------------------------------------------------------------------------------
 struct Layout {
-  size_t tiles, mnets, binfo, pword, sxy, slot_path, wp, mv, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
+  size_t tiles, mnets, tmaps, binfo, pword, sxy, slot_path, wp, mv, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
       partial, lpart, loss, chosen, tree_choice, route, nsize, nucleus_tmp, DHVC, iscal, ipartial, metrics, total;
   size_t xcount;   // int64 elements in the exchange buffer
 };
@@ -754,6 +818,7 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
                nn = (size_t)(pl.net_hi - pl.net_lo), G = (size_t)X * Y;
   L.tiles = take(sizeof(TileDesc) * pl.tiles.size());
   L.mnets = take(4 * pl.mnets.size() + 16);   // +16 B: 16-byte aligned bulk reads may run past the end
+  L.tmaps = take(256 * pl.tmap_shapes.size() + 256);   // 128-byte CUtensorMaps, (S_H, S_V) per window shape
   L.binfo = take(sizeof(int4) * pl.nb);
   L.pword = take(4 * slots);
   L.sxy = take(8 * ns + 16);
@@ -982,6 +1047,7 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   P.nid_base = pl.nid_base;
   P.seed = desc->seed;
   P.mnets = (const int32_t*)(ws + L.mnets);
+  P.tmaps = (const unsigned char*)(ws + L.tmaps);
   for (int r = 0; r < 10; ++r) {   // Philox4x32-10 round keys of the seed
     P.rk[2 * r] = (uint32_t)desc->seed + (uint32_t)r * 0x9E3779B9u;
     P.rk[2 * r + 1] = (uint32_t)(desc->seed >> 32) + (uint32_t)r * 0xBB67AE85u;
@@ -1046,7 +1112,8 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
       {L.wt, 4 * nt, desc->w_tree0 + pl.tree_lo},
       {L.q, 4 * nt, nullptr},
       {L.capH, 4 * G, desc->cap_h},
-      {L.capVT, 4 * G, nullptr}};
+      {L.capVT, 4 * G, nullptr},
+      {L.tmaps, 256 * pl.tmap_shapes.size(), nullptr}};
   std::vector<size_t> at(regs.size() + 1, 0);
   for (size_t i = 0; i < regs.size(); ++i) at[i + 1] = at[i] + ((regs[i].bytes + 255) & ~(size_t)255);
   std::lock_guard<std::mutex> lock(g_pin.m);
@@ -1063,6 +1130,12 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
     pslots[sl] = v ? 1.f : 0.f;   // p of a lone straight candidate (never rewritten by the pipelined kernel)
   }
   for (size_t j = 0; j < nt; ++j) qs[j] = 1.f;   // q of a net's lone tree stays 1 (never rewritten)
+  // tensor maps of the tile windows over this workspace's S_H ([Y][XP]) and S_V ([X][YP]) (fp64)
+  if (!pl.tmap_shapes.empty()) {
+    unsigned char* tm = reinterpret_cast<unsigned char*>(pin + at[13]);
+    const int rc = encode_window_maps(pl.tmap_shapes, (const void*)P.SH, (const void*)P.SVT, desc->X, desc->Y, tm);
+    if (rc) return cleanup(fail(DGR_ECUDA, "cuTensorMapEncodeTiled failed (%d)", rc));
+  }
 #pragma omp parallel for schedule(static)
   for (int y = 0; y < desc->Y; ++y)
     for (int x = 0; x < desc->X; ++x) capVT[(size_t)x * desc->Y + y] = desc->cap_v[(size_t)y * desc->X + x];

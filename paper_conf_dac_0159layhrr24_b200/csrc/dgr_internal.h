@@ -84,7 +84,14 @@ struct TileDesc {
   int32_t global, nbg;     // nbg: group bundles (the first nbg of the tile; the rest are singleton bundles)
   int32_t sub0, nsub;      // local sub-nets (kernel order within the tile)
   int32_t mn0, nmn;        // the tile's nets with >= 2 trees: mnets[mn0 .. mn0 + nmn) (net offsets in the tile)
+  int32_t tmap;            // pipelined tiles: index of the (S_H, S_V) tensor-map pair of the window's shape
+                           // (one 2-D TMA copy per field), -1: the window comes by cp.async
 };
+
+// Shared-memory offset (elements) of a pipelined tile's V field: the H field rounded up to 128 bytes
+// of doubles (TMA destinations are 128-byte aligned).
+inline __host__ __device__ int win_hv(int ww, int wh) { return (ww * wh + 15) & ~15; }
+constexpr int kWinPad = 16;   // the S / event windows hold up to 2 (kWinMax + kWinPad) elements
 
 struct KParams {
   // sizes
@@ -112,6 +119,7 @@ struct KParams {
   float* pp;                // p_i of the last forward (the reverse of that iteration reads it)
   const int32_t* net_tree_off;    // local, n_nets_l + 1
   const int32_t* mnets;     // per tile: offsets (in the tile) of its nets with >= 2 trees
+  const unsigned char* tmaps;   // CUtensorMap pairs (S_H window, S_V window), 128 B each, per window shape
   float *wt, *mt, *vt, *q;
   // grids (the exchange buffer, in this order: dH | dVT | VD | VDT)
   long long* dH;            // [Y][X]

@@ -640,7 +640,7 @@ struct StageLayout {
   static constexpr size_t q = (mn + 4 * kPMnMax + 15) / 16 * 16;
   static constexpr size_t wt = q + 4 * kPTreeMax;
   static constexpr size_t S = (wt + 4 * kPTreeMax + 127) / 128 * 128;
-  static constexpr size_t bytes = S + 2 * 8 * kWinMax;
+  static constexpr size_t bytes = S + 2 * 8 * (kWinMax + kWinPad);
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -747,6 +747,14 @@ __device__ __forceinline__ void tile_ranges(const TileDesc& T, int& s_lo, int& s
 }
 
 // warp 0 issues the bulk copies of tile T into stage `st`, completing on `bar`
+__device__ __forceinline__ void tma_2d(void* dst, const void* tmap, int c0, int c1, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
+          smem_u32(dst)),
+      "l"(tmap), "r"(c0), "r"(c1), "r"(smem_u32(bar))
+      : "memory");
+}
+
 template <bool REV>
 __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDesc& T, unsigned char* st, uint64_t* bar,
                                                  bool window = true) {
@@ -758,12 +766,20 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
   const uint32_t slot_bytes = (uint32_t)T.nb * 128u, gslot_bytes = (uint32_t)T.nbg * 128u;
   const bool sw = REV && window && !(KO(32));   // knock-out 32: no S window (timing only)
   const uint32_t nrow = sw ? (uint32_t)T.wh : 0u, ncol = sw ? (uint32_t)T.ww : 0u;
+  // REV && !window && tmap >= 0: the S window by two 2-D tensor copies (H field, V field)
+  const bool tw = REV && !window && T.tmap >= 0 && !(KO(32));
   const uint32_t bytes = slot_bytes + gslot_bytes + 16u * T.nb + 8u * (s_hi - s_lo) + 4u * (n_hi - n_lo) +
-                         4u * (mn_hi - mn_lo) + 8u * (t_hi - t_lo) + 8u * (nrow * T.ww + ncol * T.wh);
+                         4u * (mn_hi - mn_lo) + 8u * (t_hi - t_lo) + 8u * (nrow * T.ww + ncol * T.wh) +
+                         (tw ? 16u * (uint32_t)(T.ww * T.wh) : 0u);
   if (lane == 0) mbar_expect_tx(bar, bytes);
   __syncwarp();
   const size_t s0 = (size_t)T.b0 * 32;
   const uint64_t pol = policy_stream();
+  if (tw && lane == 8) {
+    const unsigned char* tm = P.tmaps + 256 * (size_t)T.tmap;
+    tma_2d(S.S, tm, T.wx0, T.wy0, bar);
+    tma_2d(S.S + win_hv(T.ww, T.wh), tm + 128, T.wy0, T.wx0, bar);
+  }
   // work items: 0..7 the 1-D arrays, then window rows, then window columns
   const int nitems = 8 + (int)nrow + (int)ncol;
   for (int it = lane; it < nitems; it += 32) {
@@ -783,7 +799,7 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
       bulk_g2s(S.S + (size_t)yi * T.ww, P.SH + (size_t)(T.wy0 + yi) * P.XP + T.wx0, 8u * T.ww, bar);
     } else {
       const int xi = it - 8 - (int)nrow;
-      bulk_g2s(S.S + (size_t)T.ww * T.wh + (size_t)xi * T.wh, P.SVT + (size_t)(T.wx0 + xi) * P.YP + T.wy0, 8u * T.wh, bar);
+      bulk_g2s(S.S + win_hv(T.ww, T.wh) + (size_t)xi * T.wh, P.SVT + (size_t)(T.wx0 + xi) * P.YP + T.wy0, 8u * T.wh, bar);
     }
   }
 }
@@ -819,7 +835,7 @@ __device__ __forceinline__ void lsu_tile_loads(const KParams& P, const TileDesc&
     case 6: cp_copy(S.wt, P.wt + t_lo, 4u * (t_hi - t_lo), lane); break;
     default: cp_copy(S.q, P.q + t_lo, 4u * (t_hi - t_lo), lane); break;
   }
-  if (REV && !(KO(32))) {
+  if (REV && !(KO(32)) && !(arrays == false && T.tmap >= 0)) {
     // S_H window rows (ww doubles = ww/2 chunks each), then S_V window columns (wh/2 chunks each);
     // row = floor((i + 1/2) / half) in fp32 is exact for i < 2^12 (see the flush)
     const int hw = T.ww >> 1, hh = T.wh >> 1, n = hw * T.wh;
@@ -828,7 +844,7 @@ __device__ __forceinline__ void lsu_tile_loads(const KParams& P, const TileDesc&
       const int r = (int)(((float)i + 0.5f) * inv_hw), c = i - r * hw;
       cp16(S.S + (size_t)r * T.ww + 2 * c, P.SH + (size_t)(T.wy0 + r) * P.XP + T.wx0 + 2 * c);
     }
-    double* SV = S.S + (size_t)T.ww * T.wh;
+    double* SV = S.S + win_hv(T.ww, T.wh);
     for (int i = tid; i < n; i += NT) {
       const int r = (int)(((float)i + 0.5f) * inv_hh), c = i - r * hh;
       cp16(SV + (size_t)r * T.wh + 2 * c, P.SVT + (size_t)(T.wx0 + r) * P.YP + T.wy0 + 2 * c);
@@ -866,7 +882,7 @@ __device__ long long g_tile_prof[kProfTiles * 8];
 __device__ __forceinline__ void stamp(const KParams& P, int tile, int k) {
   if ((KO(256)) && threadIdx.x == 0 && tile < kProfTiles) g_tile_prof[tile * 8 + k] = clock64();
 }
-constexpr size_t kGpOffset = 3 * 4 * kWinMax;   // tile path noise, after the event window in St.S
+constexpr size_t kGpOffset = 3 * 4 * (kWinMax + kWinPad);   // tile path noise, after the event window in St.S
 template <bool REV, bool FWD, int NT>
 __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A, const TileDesc& T, Stage St,
                                              int* ev_s, float* gp, int* dq3) {
@@ -878,10 +894,10 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
   const int mn_lo = T.mn0 & ~3;
   const uint64_t pol = policy_stream();   // L2 evict-first for the streamed slot state
-  const int ncell = T.ww * T.wh;
-  const Win W{T.wx0, T.wy0, T.ww, T.wh, ncell};
-  const int wB0 = -(T.wy0 * T.ww + T.wx0), wB1 = ncell - T.wx0 * T.wh - T.wy0;   // orientation bases
-  const int hv2 = 2 * ncell;                                                    // VD part of the window
+  const int ncell = T.ww * T.wh, hv = win_hv(T.ww, T.wh);   // V field at hv (128-byte aligned)
+  const Win W{T.wx0, T.wy0, T.ww, T.wh, hv};
+  const int wB0 = -(T.wy0 * T.ww + T.wx0), wB1 = hv - T.wx0 * T.wh - T.wy0;   // orientation bases
+  const int hv2 = 2 * hv;                                                     // VD part of the window
   const int nbg = T.nbg;
 
   // ---------------- reverse of iteration k ----------------
@@ -950,7 +966,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   // ---------------- net level (one thread per net), event window cleared alongside ----------------
   if (FWD) {
     int4* z = reinterpret_cast<int4*>(ev_s);   // the S window is free after the reverse
-    for (int i = tid; i < (3 * ncell + 3) / 4; i += NT) z[i] = make_int4(0, 0, 0, 0);
+    for (int i = tid; i < (3 * hv) / 4; i += NT) z[i] = make_int4(0, 0, 0, 0);
   }
   // the tile's nets with >= 2 trees (a lone tree has q = 1 and du = 0 always: its logit and Adam
   // state never change, and its q = 1 arrives with the stage)
@@ -1097,8 +1113,8 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     const int hw = T.ww >> 1, hh = T.wh >> 1;
     const float inv_hw = 1.f / (float)hw, inv_hh = 1.f / (float)hh;
     const int2* evH = reinterpret_cast<const int2*>(ev_s);
-    const int2* evV = reinterpret_cast<const int2*>(ev_s + ncell);
-    const int2* evD = reinterpret_cast<const int2*>(ev_s + 2 * ncell);
+    const int2* evV = reinterpret_cast<const int2*>(ev_s + hv);
+    const int2* evD = reinterpret_cast<const int2*>(ev_s + 2 * hv);
     const int npair = ncell >> 1;
     for (int i = tid; i < npair; i += NT) {
       const int2 h = evH[i], d = evD[i], v = evV[i];
@@ -1137,7 +1153,7 @@ constexpr int kBThreads = DGR_BTHREADS;
 constexpr int kBPerSM = DGR_BPERSM;
 constexpr size_t kTailBytes = 12 * kPipeTrees + 16;   // dq limbs, mbarrier
 constexpr size_t kBSmemBytes = (StageLayout::bytes + kTailBytes) > kSmemBytes ? (StageLayout::bytes + kTailBytes) : kSmemBytes;
-static_assert(kGpOffset + 4 * 32 * kTargetBundles <= 2 * 8 * kWinMax, "event window + path noise must fit the S window");
+static_assert(kGpOffset + 4 * 32 * kTargetBundles <= 2 * 8 * (kWinMax + kWinPad), "event window + path noise must fit the S window");
 
 template <bool REV, bool FWD>
 __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepArgs A) {
