@@ -102,7 +102,7 @@ struct KParams {
   int32_t ntiles_slow;      // global / oversized tiles (one CTA each)
   int32_t XP, YP;           // even pitches of S_H rows and S_V columns
   int32_t skip;             // DGR_DEBUG_SKIP: timing knock-outs (results invalid), 0 in production
-  int32_t pf;               // bit 0: L2 prefetch of the state a tile reads directly (DGR_PF, default 0)
+  int32_t pf;               // L2 prefetch at tile start (DGR_PF): bit 1 the trees' Adam moments (default), bit 0 also the slots' m, v, p
   int64_t path_base, tree_base;   // global index of the first local path / tree
   int64_t nid_base;         // global noise index of the rank's first noisy candidate
   uint64_t seed;

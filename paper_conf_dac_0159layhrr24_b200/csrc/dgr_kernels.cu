@@ -856,11 +856,11 @@ __device__ __forceinline__ void lsu_tile_loads(const KParams& P, const TileDesc&
 // L2 prefetch of what a tile reads directly (not through the stage): the group slots' Adam moments
 // and stored p, the trees' Adam moments; issued next to the stage's bulk copies, so the direct loads
 // of the reverse and net-level phases hit L2.
-__device__ __forceinline__ void prefetch_tile(const KParams& P, const TileDesc& T) {
+__device__ __forceinline__ void prefetch_tile(const KParams& P, const TileDesc& T, bool slots = true) {
   const int lane = threadIdx.x & 31;
   const size_t s0 = (size_t)T.b0 * 32;
   const int t_lo = T.tree0 & ~3, t_hi = (T.tree0 + T.ntree + 3) & ~3;
-  const uint32_t gs = (uint32_t)T.nbg * 32u;
+  const uint32_t gs = slots ? (uint32_t)T.nbg * 32u : 0u;
   switch (lane) {
     case 0: if (gs) prefetch_l2(P.mv + s0, 8u * gs); break;
     case 1: if (gs) prefetch_l2(P.pp + s0, 4u * gs); break;
@@ -1190,7 +1190,12 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
   griddep_wait();   // S, logits, q and the event grids come from the previous kernels
 #if DGR_LSU_STAGE == 2
   // the eight 1-D arrays by bulk copies (8 per tile: few and large), the S window by cp.async
-  if (threadIdx.x < 32) issue_tile_loads<REV>(P, T, smem, bar, false);
+  if (threadIdx.x < 32) {
+    issue_tile_loads<REV>(P, T, smem, bar, false);
+    // the trees' Adam moments are read by the net level (one dependent chain per net, the
+    // phase's critical path): bring them to L2 with the stage (DGR_PF bit 1; bit 0 also the slots')
+    if (REV && (P.pf & 3)) prefetch_tile(P, T, (P.pf & 1) != 0);
+  }
   lsu_tile_loads<REV, kBThreads>(P, T, smem, false);
   asm volatile("cp.async.wait_group 0;" ::: "memory");
   mbar_wait(bar, 0u);
