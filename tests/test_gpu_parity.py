@@ -67,7 +67,7 @@ def scaled_err(a, b):
     return np.abs(a - b) / np.maximum(np.abs(b), 1.0)
 
 
-def compare_state(s, o, what, probe=None, max_ill=0.01):
+def compare_state(s, o, what, probe=None, max_ill=0.01, exempt=None):
     """Element-wise parity of demand and logits.  Without a probe: every element within TOL.
     With the fp32 probe (multi-iteration runs, DESIGN.md §3 Q21b): every element within TOL, or, where
     an fp32 evaluation of the same formulation is itself further than TOL from fp64 (Adam turns a
@@ -86,12 +86,15 @@ def compare_state(s, o, what, probe=None, max_ill=0.01):
         return
     pdh, pdv = probe.demand()
     pwt, pwp = probe.logits()
-    for g, r, pr, nm in ((gdh, odh, pdh, "d_h"), (gdv, odv, pdv, "d_v"), (gwp, owp, pwp, "w_path"),
-                         (gwt, owt, pwt, "w_tree")):
+    ex_t, ex_p = exempt if exempt is not None else (None, None)
+    for g, r, pr, nm, ex in ((gdh, odh, pdh, "d_h", None), (gdv, odv, pdv, "d_v", None),
+                             (gwp, owp, pwp, "w_path", ex_p), (gwt, owt, pwt, "w_tree", ex_t)):
         eg, e32 = scaled_err(g, r), scaled_err(pr, r)
         strict = eg <= TOL
         relaxed = ~strict & (eg <= 10.0 * e32)
         bad = ~strict & ~relaxed
+        if ex is not None:   # checked by the caller (ill-conditioned first Adam step, Q21b)
+            bad &= ~ex.reshape(bad.shape)
         i = int(np.argmax(np.where(bad, eg, -1))) if bad.any() else 0
         assert not bad.any(), (f"{what} {nm}: {bad.sum()} elements beyond TOL and beyond 10x the fp32 probe; "
                                f"worst {i}: gpu {g.flat[i]} fp64 {r.flat[i]} fp32 {pr.flat[i]}")
@@ -279,10 +282,12 @@ def test_empty_and_degenerate_forests():
     compare_state(s, o, "2x2", probe=probes(f, [(20, 1.0)]))
 
 
-def test_full_size_sampled_parity():
-    """BASELINE.json configs[3] (ispd19, ~1e6 nets, the bench workload) in the bench's launch
-    configuration: full demand / loss of the first forward and every logit after one iteration."""
-    f = forestgen.generate("ispd19")
+@pytest.mark.parametrize("name", ["ispd19", "sweep4e6"])
+def test_full_size_sampled_parity(name):
+    """BASELINE.json configs[3] (ispd19, ~1e6 nets, the bench workload) and the largest sweep point
+    of configs[4] (sweep4e6: 3.8e6 nets on 2000x2000) in the bench's launch configuration: full
+    demand / loss of the first forward and every logit after one iteration."""
+    f = forestgen.generate(name)
     s = dgr.Solver(f)
     o = oracle.Oracle(f)
     gl = s.step(0, 1.0, 0.3)
@@ -293,7 +298,21 @@ def test_full_size_sampled_parity():
     assert_close(gdh, odh, what="d_h"); assert_close(gdv, odv, what="d_v")
     s.step(1, 1.0, 0.3)
     o.step(1, 1.0, 0.3, ow(dgr.Weights()))
-    compare_state(s, o, "ispd19", probe=probes(f, [(0, 1.0), (1, 1.0)]), max_ill=1e-4)
+    # reading Q21b at full size: Adam's first step is lr * g / (|g| + eps), so a coordinate whose
+    # fp64 gradient is below what fp32 resolves (|g| < 1e-5: fp32 sums of per-candidate cost
+    # differences of O(100)) may take any step in [-lr, lr]; those must be rare.  Every other logit
+    # follows compare_state (TOL, or the fp32-probe clause).
+    o0 = oracle.Oracle(f)
+    o0.forward(1.0, ow(dgr.Weights()))
+    dw0, du0 = o0.backward(1.0, ow(dgr.Weights()))
+    gwt, gwp = s.logits()
+    owt, owp = o.logits()
+    for g, r, d0, nm in ((gwp, owp, dw0, "w_path"), (gwt, owt, du0, "w_tree")):
+        ill = np.abs(d0) < 1e-5
+        assert np.abs(g - r)[ill].max(initial=0) <= 2 * 0.3 + 1e-6, nm
+        assert (ill & (np.abs(g - r) > TOL * np.maximum(np.abs(r), 1))).mean() <= 1e-5, nm
+    compare_state(s, o, name, probe=probes(f, [(0, 1.0), (1, 1.0)]), max_ill=1e-4,
+                  exempt=(np.abs(du0) < 1e-5, np.abs(dw0) < 1e-5))
 
 
 def test_table1_workload_relu_parity_and_optimum():
