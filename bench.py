@@ -222,6 +222,16 @@ def cpu_baseline(f, seconds_target=12.0):
             "path_cand_per_s": n / dt * f.n_paths}
 
 
+METRIC = "DAG-forest solver iters/sec (path-cand/s, overflow, WL alongside)"
+
+
+def workload_name(config: str) -> str:
+    """The workload string both arms report (BASELINE.json configs[3] by default)."""
+    if config == "ispd19":
+        return "ispd19 (BASELINE.json configs[3]: ISPD'19-shaped congested synthetic)"
+    return config
+
+
 def run_reference(args):
     rank, world, _ = dist_env()
     if rank != 0:
@@ -251,10 +261,11 @@ def run_reference(args):
         o.step(1, 1.0, 0.3, W)
     dt = time.perf_counter() - t0
     value = args.steps / dt * frac
-    line = {"metric": "DAG-forest solver iters/sec", "value": value, "unit": "iters/s", "impl": "reference",
+    line = {"metric": METRIC, "value": value, "unit": "iters/s", "impl": "reference",
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
-            "data": "synthetic", "config": {"workload": args.config, "nets": f.n_nets, "paths": f.n_paths},
+            "data": "synthetic", "config": {"workload": workload_name(args.config), "grid": f"{f.X}x{f.Y}",
+                                            "nets": f.n_nets, "paths": f.n_paths},
             "path_cand_per_s": value * f.n_paths,
             "cpu_baseline": {"value": value, "unit": "iters/s", "cores": 1, "kind": "oracle", "sample": sample},
             "e2e": {"value": value, "unit": "iters/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -386,11 +397,11 @@ def main():
     alg_iter = sv["KG"] + sv["KBF"]
     alg_iter_strict = sb["KG"] + sb["KBF"]
     line = {
-        "metric": "DAG-forest solver iters/sec (path-cand/s, overflow, WL alongside)",
+        "metric": METRIC,
         "value": iters_per_s, "unit": "iters/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
         "dtype": "f32", "data": "synthetic",
-        "config": {"workload": f"{args.config} (BASELINE.json configs[3]: ISPD'19-shaped congested synthetic)",
+        "config": {"workload": workload_name(args.config),
                    "grid": f"{f.X}x{f.Y}", "nets": f.n_nets, "trees": f.n_trees, "subnets": f.n_subnets,
                    "paths": f.n_paths, "segments": f.n_segs, "turning_points": f.n_tps,
                    "step": "one solver iteration (softmax, scatter, loss/gradient map, reverse, Adam) = KG + KBF; induction timed separately",
