@@ -1139,14 +1139,16 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
 #pragma omp parallel for schedule(static)
   for (int y = 0; y < desc->Y; ++y)
     for (int x = 0; x < desc->X; ++x) capVT[(size_t)x * desc->Y + y] = desc->cap_v[(size_t)y * desc->X + x];
-  for (size_t i = 0; i < regs.size(); ++i)
-    if (regs[i].src && regs[i].bytes) par_copy(pin + at[i], regs[i].src, regs[i].bytes);
-  tm.mark("bind: host staging");
+  tm.mark("bind: host staging (in place)");
+  // stage region i and start its upload, so that the DMA of region i overlaps the staging of i+1
   cudaError_t e = cudaSuccess;
-  for (size_t i = 0; i < regs.size() && e == cudaSuccess; ++i)
-    if (regs[i].bytes) e = cudaMemcpyAsync(ws + regs[i].off, pin + at[i], regs[i].bytes, cudaMemcpyHostToDevice, s);
+  for (size_t i = 0; i < regs.size() && e == cudaSuccess; ++i) {
+    if (!regs[i].bytes) continue;
+    if (regs[i].src) par_copy(pin + at[i], regs[i].src, regs[i].bytes);
+    e = cudaMemcpyAsync(ws + regs[i].off, pin + at[i], regs[i].bytes, cudaMemcpyHostToDevice, s);
+  }
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
-  tm.mark("bind: upload");
+  tm.mark("bind: staging + upload");
   if (e != cudaSuccess) return cleanup(fail(DGR_ECUDA, "upload: %s", cudaGetErrorString(e)));
   if (cudaMallocHost(&h->pinned, 16 * sizeof(double)) != cudaSuccess) return cleanup(fail(DGR_ECUDA, "cudaMallocHost failed"));
   if (world > 1 && dist->allreduce) {
