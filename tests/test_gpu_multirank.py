@@ -145,3 +145,19 @@ def test_slow_tiles_equal_pipelined_tiles(monkeypatch):
     assert all(np.array_equal(x, y) for x, y in zip(a.logits(), b.logits()))
     a.close()
     b.close()
+
+
+def test_tma_window_equals_cp_async_window(monkeypatch):
+    """The S window of a pipelined tile arrives by two 2-D TMA tensor copies, or (windows wider or
+    taller than 256 cells, or DGR_NO_TMA_WINDOW at plan time) by cp.async: bit-identical results."""
+    f = forestgen.generate("c1e4_c")
+    a = dgr.Solver(f)
+    monkeypatch.setenv("DGR_NO_TMA_WINDOW", "1")
+    b = dgr.Solver(f)
+    monkeypatch.delenv("DGR_NO_TMA_WINDOW")
+    for t in (1.0, 0.9):
+        assert np.array_equal(a.step(3, t, 0.3), b.step(3, t, 0.3))
+    assert all(np.array_equal(x, y) for x, y in zip(a.demand(), b.demand()))
+    assert all(np.array_equal(x, y) for x, y in zip(a.logits(), b.logits()))
+    a.close()
+    b.close()
