@@ -145,7 +145,8 @@ int dgr_bind_workspace(struct dgr_handle* h, const dgr_forest_desc* desc, const 
  * Validates desc, keeps this rank's nets (dgr_partition), encodes them for the device, copies
  * them into dev_workspace (>= dgr_workspace_size bytes, 256-byte aligned) on cuda_stream
  * (a cudaStream_t; NULL = legacy default stream), zeroes Adam state and the iteration counter k.
- * With world > 1 this also creates the NCCL communicator (collective).  Synchronises. */
+ * With world > 1 this also creates the NCCL communicator (collective), unless dist->allreduce
+ * supplies the exchange.  Synchronises. */
 int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev_workspace,
                     int64_t workspace_bytes, void* cuda_stream, struct dgr_handle** out);
 
@@ -159,7 +160,8 @@ int dgr_forest_load(const dgr_forest_desc* desc, const dgr_dist* dist, void* dev
 int dgr_step(struct dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w,
              dgr_loss* last);
 
-/* dgr_step without host synchronisation: the same iterations, then a stream-ordered copy of the
+/* dgr_step without host synchronisation (the same iterations of PAPER.md §4.3-4.4, P:803-847,
+ * P:913-914), then a stream-ordered copy of the
  * loss of the last forward (4 doubles: total, wl, via, overflow, as dgr_loss) into loss_out
  * (host memory, caller-owned; pinned memory keeps the call asynchronous).  loss_out is valid
  * after dgr_sync or any synchronising call on the handle.  NULL loss_out: DGR_EINVAL. */
