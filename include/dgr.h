@@ -108,7 +108,8 @@ typedef struct {
 } dgr_weights;
 
 /* Loss of a forward pass: total = a_wl*wl + a_via*via + a_of*overflow, with
- * wl = E[WL] (Eq. 11), via = sqrt(L) E[TP] (Eq. 12), overflow = sum_e f(cap_e - d_e) (Eq. 9). */
+ * wl = E[WL] (Eq. 11), via = sqrt(L) E[TP] (Eq. 12), overflow = sum_e f(d_e - cap_e) (Eq. 9), f of
+ * the overflow x = d - cap (reading Q2: the paper's f(cap - d) with f decreasing). */
 typedef struct { double total, wl, via, overflow; } dgr_loss;
 
 struct dgr_handle;
@@ -193,7 +194,7 @@ int dgr_induce(struct dgr_handle* h, float top_p, int32_t* tree_choice, int32_t*
 
 /* Introspection: iteration counter k, this rank's net range, encoded sizes.  info[12] =
  * {k, net_lo, net_hi, n_bundles, n_path_slots, workspace_bytes, world, rank, n_tiles,
- *  n_global_tiles, 0, 0}. */
+ *  n_global_tiles, n_pipelined_tiles, 0}. */
 int dgr_get_info(struct dgr_handle* h, int64_t info[12]);
 
 /* Host-only view of the rank's encoding plan (no GPU needed): out[8] = {n_tiles, n_global_tiles,
@@ -207,7 +208,8 @@ int dgr_plan_info(const dgr_forest_desc* desc, const dgr_dist* dist, int64_t out
  * dgr_profile_read synchronises and returns, per stage, the summed milliseconds and the number of
  * launches: 0 KF (forward-only tile kernel, once per dgr_step call), 1 demand allreduce (NCCL;
  * world > 1), 2 KG (scan / loss / gradient map; 1 kernel), 3 KBF (reverse of k fused with the
- * forward of k+1), 4 KB (reverse only; not launched since every call ends with KBF), 5..7 unused. */
+ * forward of k+1), 4 KB (reverse only; not launched since every call ends with KBF), 5 KL (the loss reduction,
+ * once per call after its last KG), 6..7 unused. */
 int dgr_profile(struct dgr_handle* h, int32_t enable);
 int dgr_profile_read(struct dgr_handle* h, double ms[8], int64_t launches[8]);
 

@@ -169,6 +169,7 @@ bool classify(const dgr_forest_desc* d, int64_t i, int x0, int y0, int x1, int y
   if (ax == bx && ((ay == y0 && by == y1) || (ay == y1 && by == y0))) {   // Z-HVH (or C-HVH) at x_m = ax
     const int xm = ax;
     if (xm == x0 || xm == x1) return false;
+    if (xm < 0 || xm >= d->X) return false;   // a C-shape detour must stay inside the grid
     if (!has({0, y0, std::min(x0, xm), std::max(x0, xm)}) || !has({1, xm, ylo, yhi}) ||
         !has({0, y1, std::min(xm, x1), std::max(xm, x1)}))
       return false;
@@ -177,6 +178,7 @@ bool classify(const dgr_forest_desc* d, int64_t i, int x0, int y0, int x1, int y
   if (ay == by && ((ax == x0 && bx == x1) || (ax == x1 && bx == x0))) {   // Z-VHV (or C-VHV) at y_m = ay
     const int ym = ay;
     if (ym == y0 || ym == y1) return false;
+    if (ym < 0 || ym >= d->Y) return false;   // a C-shape detour must stay inside the grid
     *outside = ym < ylo || ym > yhi;
     if (!has({1, x0, std::min(y0, ym), std::max(y0, ym)}) || !has({0, ym, x0, x1}) ||
         !has({1, x1, std::min(ym, y1), std::max(ym, y1)}))
@@ -886,7 +888,12 @@ struct dgr_handle {
   // last iteration of the previous dgr_step call ran it), so the next call can start from them
   bool fwd_valid = false;
   float t_fwd = 0.f;
+  // the exchange grids may hold demand events no KG has consumed yet (set before every forward
+  // launch, cleared after the KG that reads them): a call that failed part-way leaves it set, and
+  // the next call clears the grids instead of adding its events on top of the stale ones
+  bool grids_dirty = false;
   double* pinned = nullptr;   // 16 doubles of pinned host memory
+  int dev = -1;               // device of the workspace (set at bind); every later call runs on it
   // profiling: a CUDA event after every stage, attributed to that stage
   bool prof = false;
   std::vector<cudaEvent_t> ev;
@@ -895,6 +902,17 @@ struct dgr_handle {
 };
 
 namespace {
+// Makes the handle's device current for the duration of an entry point (the caller's current
+// device may differ: launches and stream work must go to the workspace's device) and restores it.
+struct DevGuard {
+  int prev = -1;
+  explicit DevGuard(const dgr_handle* h) {
+    if (!h || h->dev < 0) return;
+    if (cudaGetDevice(&prev) != cudaSuccess) { prev = -1; return; }
+    if (prev != h->dev) cudaSetDevice(h->dev); else prev = -1;
+  }
+  ~DevGuard() { if (prev >= 0) cudaSetDevice(prev); }
+};
 // stage -1 opens an interval; stage >= 0 closes the interval since the previous event
 int prof_mark(dgr_handle* h, int stage) {
   if (!h->prof) return DGR_OK;
@@ -1030,6 +1048,15 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   if (!dev_workspace || workspace_bytes < (int64_t)L.total)
     return fail(DGR_ENOMEM, "workspace of %lld bytes < %zu needed", (long long)workspace_bytes, L.total);
   if (((uintptr_t)dev_workspace) & 255) return fail(DGR_EINVAL, "workspace not 256-byte aligned");
+  {
+    cudaPointerAttributes pa{};
+    if (cudaPointerGetAttributes(&pa, dev_workspace) != cudaSuccess || pa.type != cudaMemoryTypeDevice) {
+      cudaGetLastError();
+      return fail(DGR_EINVAL, "workspace is not device memory");
+    }
+    h->dev = pa.device;
+  }
+  DevGuard dg(h);
   char* ws = (char*)dev_workspace;
   P.nb = pl.nb;
   P.ntiles = (int32_t)pl.n_pipe_tiles;
@@ -1181,6 +1208,7 @@ int dgr_step_async(dgr_handle* h, int32_t iters, float temperature, float lr, co
 
 int dgr_sync(dgr_handle* h) {
   g_err.clear();
+  DevGuard dg(h);
   if (!h) return fail(DGR_EINVAL, "NULL handle");
   CUDA_TRY(cudaStreamSynchronize(h->stream));
   return DGR_OK;
@@ -1189,6 +1217,7 @@ int dgr_sync(dgr_handle* h) {
 static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w, dgr_loss* last,
                      double* loss_async) {
   g_err.clear();
+  DevGuard dg(h);
   if (!h || !w) return fail(DGR_EINVAL, "NULL handle or weights");
   if (!h->ws) return fail(DGR_ESTATE, "no workspace bound (dgr_bind_workspace)");
   if (iters < 0) return fail(DGR_EINVAL, "iters < 0");
@@ -1222,7 +1251,8 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
   if (!(h->fwd_valid && h->t_fwd == temperature)) {
     // KG clears the event grids in place after reading them; stale events of a forward at another
     // temperature are cleared here
-    if (h->fwd_valid) CUDA_TRY(cudaMemsetAsync(P.dH, 0, 4 * grid_bytes, s));   // dH | dV^T | VD | VD^T
+    if (h->grids_dirty) CUDA_TRY(cudaMemsetAsync(P.dH, 0, 4 * grid_bytes, s));   // dH | dV^T | VD | VD^T
+    h->grids_dirty = true;
     launch_tiles(P, a, kForwardOnly, s);
     if ((rc = prof_mark(h, 0))) return rc;
   }
@@ -1239,6 +1269,7 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
       if ((rc = prof_mark(h, 1))) return rc;
     }
     launch_kg(P, a, s);
+    h->grids_dirty = false;
     if ((rc = prof_mark(h, 2))) return rc;
     if (last) {   // the reported loss of this call's last forward
       launch_kg_loss(P, a, s);
@@ -1247,6 +1278,7 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
     if (iters > 0) {
       // reverse of iteration k + forward of k+1 (also after the last iteration: the next call
       // at the same temperature starts from it)
+      h->grids_dirty = true;
       launch_tiles(P, a, kReverseForward, s);
       h->k += 1;
       if ((rc = prof_mark(h, 3))) return rc;
@@ -1284,6 +1316,7 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
 
 int dgr_get_demand(dgr_handle* h, float* d_h, float* d_v) {
   g_err.clear();
+  DevGuard dg(h);
   if (!h || !d_h || !d_v) return fail(DGR_EINVAL, "NULL argument");
   if (!h->ws) return fail(DGR_ESTATE, "no workspace bound (dgr_bind_workspace)");
   if (!h->have_forward) return fail(DGR_ESTATE, "no forward has run yet");
@@ -1299,6 +1332,7 @@ int dgr_get_demand(dgr_handle* h, float* d_h, float* d_v) {
 
 int dgr_get_logits(dgr_handle* h, float* w_tree, float* w_path) {
   g_err.clear();
+  DevGuard dg(h);
   if (!h) return fail(DGR_EINVAL, "NULL handle");
   if (!h->ws) return fail(DGR_ESTATE, "no workspace bound (dgr_bind_workspace)");
   const Plan& pl = h->plan;
@@ -1320,6 +1354,7 @@ int dgr_get_logits(dgr_handle* h, float* w_tree, float* w_path) {
 int dgr_induce(dgr_handle* h, float top_p, int32_t* tree_choice, int32_t* route, int64_t* nucleus_off,
                int32_t* nucleus, int32_t* D_h, int32_t* D_v, double metrics[5]) {
   g_err.clear();
+  DevGuard dg(h);
   if (!h || !tree_choice || !route || !nucleus_off || !nucleus || !D_h || !D_v || !metrics)
     return fail(DGR_EINVAL, "NULL argument");
   if (!h->ws) return fail(DGR_ESTATE, "no workspace bound (dgr_bind_workspace)");
@@ -1406,6 +1441,7 @@ int dgr_plan_info(const dgr_forest_desc* desc, const dgr_dist* dist, int64_t out
 
 int dgr_profile(dgr_handle* h, int32_t enable) {
   g_err.clear();
+  DevGuard dg(h);
   if (!h) return fail(DGR_EINVAL, "NULL handle");
   h->prof = enable != 0;
   h->ev_used = 0;
@@ -1414,6 +1450,7 @@ int dgr_profile(dgr_handle* h, int32_t enable) {
 
 int dgr_profile_read(dgr_handle* h, double ms[8], int64_t launches[8]) {
   g_err.clear();
+  DevGuard dg(h);
   if (!h || !ms || !launches) return fail(DGR_EINVAL, "NULL argument");
   CUDA_TRY(cudaStreamSynchronize(h->stream));
   for (int i = 0; i < 8; ++i) { ms[i] = 0.0; launches[i] = 0; }
@@ -1430,6 +1467,7 @@ int dgr_profile_read(dgr_handle* h, double ms[8], int64_t launches[8]) {
 
 int dgr_free(dgr_handle* h) {
   g_err.clear();
+  DevGuard dg(h);
   if (!h) return DGR_OK;
   if (h->stream) cudaStreamSynchronize(h->stream);
   for (auto e : h->ev) cudaEventDestroy(e);

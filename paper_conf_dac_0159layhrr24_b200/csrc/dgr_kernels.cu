@@ -3,7 +3,7 @@
 // One iteration k is two kernels (plus the NCCL allreduce of the demand when world > 1):
 //
 //   KG   per G-cell line (CTA / line): scan of the difference arrays -> demand d (Eq. (10),
-//        P:556-564), overflow cost f(cap - d) (Eq. (9)), gradient map G = -a3 f'(cap - d), and
+//        P:556-564), overflow cost f(d - cap) (Eq. (9), reading Q2), gradient map G = a3 f'(d - cap), and
 //        the exclusive prefix S of G along the line; clears the difference arrays.
 //   KBF  per tile (CTA / tile of whole nets, see dgr_internal.h):
 //          reverse of iteration k:  p(k) recomputed (same Gumbel noise), c_i = dcost/dpi_i from
@@ -1222,7 +1222,7 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
 // ------------------------------------------------------------------------------------------
 // KG: one CTA per line (Y H-rows, then X V-columns).  Scan of the difference array gives the
 // wire demand W; d = (W + beta (VD_a + VD_b)) 2^-24 (Eq. (10), reading Q3); overflow cost
-// f(cap - d) (Eq. (9)); G = dcost/dd = -a3 f'(cap - d); S = exclusive prefix of G (fp64).
+// f(d - cap) (Eq. (9), reading Q2); G = dcost/dd = a3 f'(d - cap); S = exclusive prefix of G (fp64).
 // The line's difference and turning-point entries are cleared for the next forward.
 // ------------------------------------------------------------------------------------------
 constexpr int kGThreads = 32 * kKgWarps;

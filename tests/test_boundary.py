@@ -162,3 +162,33 @@ def test_candidate_order_contract(tiny):
     s2 = int(np.nonzero(n == 2)[0][0]) if (n == 2).any() else None
     if s2 is not None:
         assert _ws(_permute_candidates(tiny, s2, [0, 1]))[0] > 0
+
+
+@pytest.mark.parametrize("xm", [-3, -1, "X", "X+2"])
+def test_c_shape_detour_outside_grid_rejected(xm):
+    """A C-shape detour (reading Q14b) whose x_m lies outside the grid is DGR_EINVAL: its demand
+    events and S reads would otherwise index outside the grid."""
+    import copy
+    f = copy.deepcopy(forestgen.generate("tiny_c"))
+    xm = {"X": f.X, "X+2": f.X + 2}.get(xm, xm)
+    for i in range(f.n_paths):
+        t0, t1 = f.path_tp_off[i], f.path_tp_off[i + 1]
+        if t1 - t0 != 2 or f.tp_xy[t0, 0] != f.tp_xy[t0 + 1, 0]:
+            continue
+        s = int(np.searchsorted(f.sub_path_off, i, side="right") - 1)
+        x0, y0, x1, y1 = f.sub_xy[s]
+        if min(x0, x1) <= f.tp_xy[t0, 0] <= max(x0, x1):
+            continue                                          # a Z, not a C-HVH
+        f.tp_xy[t0:t1, 0] = xm
+        for g in range(f.path_seg_off[i], f.path_seg_off[i + 1]):
+            d, line, lo, hi = f.seg[g]
+            if d == 1:
+                f.seg[g, 1] = xm
+            else:
+                xe = x0 if line == y0 else x1
+                f.seg[g, 2], f.seg[g, 3] = min(xe, xm), max(xe, xm)
+        break
+    else:
+        pytest.fail("tiny_c has no C-HVH candidate")
+    n, err = _ws(f)
+    assert n == 0 and "pattern" in err, err

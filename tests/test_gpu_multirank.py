@@ -129,6 +129,29 @@ def test_failing_exchange_is_reported():
         s.close()
 
 
+def test_failed_step_leaves_no_stale_events():
+    """A dgr_step that fails after its forward (here: the exchange) must not leave that forward's
+    demand events behind for the next call to add onto (dgr.h: an error leaves no partial state).
+    Rank 0 of 2 with an exchange that adds nothing (the other rank's share is zero): after one
+    failed call, the next call equals the same call on a fresh handle."""
+    f = forestgen.generate("tiny")
+    calls = {"n": 0}
+
+    def flaky(*a):
+        calls["n"] += 1
+        return 7 if calls["n"] == 1 else 0
+
+    a = dgr.Solver(f, rank=0, world=2, allreduce=flaky)
+    b = dgr.Solver(f, rank=0, world=2, allreduce=lambda *a: 0)
+    with pytest.raises(dgr.DgrError, match="allreduce callback returned 7"):
+        a.step(1, 1.0, 0.3)
+    assert np.array_equal(a.step(2, 1.0, 0.3), b.step(2, 1.0, 0.3))
+    assert all(np.array_equal(x, y) for x, y in zip(a.demand(), b.demand()))
+    assert all(np.array_equal(x, y) for x, y in zip(a.logits(), b.logits()))
+    a.close()
+    b.close()
+
+
 def test_slow_tiles_equal_pipelined_tiles(monkeypatch):
     """A net gives bit-identical results whichever tile kind it lands in (the kind can depend on the
     tile's composition, hence on the rank count): every tile on the slow / global-memory path
