@@ -67,37 +67,62 @@ def scaled_err(a, b):
     return np.abs(a - b) / np.maximum(np.abs(b), 1.0)
 
 
-def compare_state(s, o, what, probe=None, max_ill=0.01, exempt=None):
+# Relaxed clause of the parity contract (reading Q21b), for elements beyond TOL:
+#   |gpu - fp64| <= K_PROBE * |fp32 probe - fp64|  (both scaled by max(|fp64|, 1))   and
+#   |gpu - fp64| <= 2 lr                             (never more than two Adam steps apart)
+# where the fp32 probe (the oracle's own source built with real = float) is itself beyond TOL.
+K_PROBE = float(__import__("os").environ.get("DGR_K_PROBE", "2.0"))   # env: data-gathering runs only
+LR = 0.3
+PARITY_COUNTS = {}   # test -> field -> clause counts (printed in the session summary, tests/conftest.py)
+
+
+def _record(what, nm, **kv):
+    PARITY_COUNTS.setdefault(what, {})[nm] = kv
+
+
+def compare_state(s, o, what, probe=None, max_ill=0.01, exempt=None, k_probe=K_PROBE):
     """Element-wise parity of demand and logits.  Without a probe: every element within TOL.
     With the fp32 probe (multi-iteration runs, DESIGN.md §3 Q21b): every element within TOL, or, where
     an fp32 evaluation of the same formulation is itself further than TOL from fp64 (Adam turns a
-    near-zero gradient's rounding into an lr-sized step), no further from fp64 than 10x that fp32
-    evaluation (one sample of fp32 rounding; the kernel rounds elsewhere); such elements must stay
-    below `max_ill` of the total."""
+    near-zero gradient's rounding into an lr-sized step), no further from fp64 than k_probe times that
+    fp32 evaluation and never more than 2 lr; such elements must stay below `max_ill` of the total.
+    `exempt` (per logit field) marks coordinates the caller checks itself (the first Adam step of a
+    coordinate whose fp64 gradient is below fp32 resolution).  Every clause's count is recorded."""
     gdh, gdv = s.demand()
     odh, odv = o.demand()
     gwt, gwp = s.logits()
     owt, owp = o.logits()
-    if probe is None:
-        assert_close(gdh, odh, what=what + " d_h")
-        assert_close(gdv, odv, what=what + " d_v")
-        assert_close(gwp, owp, what=what + " w_path")
-        assert_close(gwt, owt, what=what + " w_tree")
-        return
-    pdh, pdv = probe.demand()
-    pwt, pwp = probe.logits()
+    pr = None
+    if probe is not None:
+        pdh, pdv = probe.demand()
+        pwt, pwp = probe.logits()
+        pr = (pdh, pdv, pwp, pwt)
     ex_t, ex_p = exempt if exempt is not None else (None, None)
-    for g, r, pr, nm, ex in ((gdh, odh, pdh, "d_h", None), (gdv, odv, pdv, "d_v", None),
-                             (gwp, owp, pwp, "w_path", ex_p), (gwt, owt, pwt, "w_tree", ex_t)):
-        eg, e32 = scaled_err(g, r), scaled_err(pr, r)
+    fields = ((gdh, odh, "d_h", None), (gdv, odv, "d_v", None), (gwp, owp, "w_path", ex_p), (gwt, owt, "w_tree", ex_t))
+    for fi, (g, r, nm, ex) in enumerate(fields):
+        g = np.asarray(g, np.float64); r = np.asarray(r, np.float64)
+        eg = scaled_err(g, r)
         strict = eg <= TOL
-        relaxed = ~strict & (eg <= 10.0 * e32)
+        if pr is None:
+            relaxed = np.zeros_like(strict)
+            e32 = np.zeros_like(eg)
+        else:
+            e32 = scaled_err(pr[fi], r)
+            relaxed = ~strict & (e32 > TOL) & (eg <= k_probe * e32) & (np.abs(g - r) <= 2 * LR + 1e-6)
         bad = ~strict & ~relaxed
+        exempted = np.zeros_like(bad)
         if ex is not None:   # checked by the caller (ill-conditioned first Adam step, Q21b)
-            bad &= ~ex.reshape(bad.shape)
+            exempted = bad & ex.reshape(bad.shape)
+            bad &= ~exempted
+        ratio = (eg / np.maximum(e32, 1e-300))[relaxed]
+        _record(what, nm, n=int(eg.size), strict=int(strict.sum()), probe=int(relaxed.sum()),
+                exempt=int(exempted.sum()), bad=int(bad.sum()), max_err=float(eg.max(initial=0.0)),
+                max_err_strict_excl=float(eg[~strict].max(initial=0.0)),
+                max_probe_ratio=float(ratio.max(initial=0.0)))
         i = int(np.argmax(np.where(bad, eg, -1))) if bad.any() else 0
-        assert not bad.any(), (f"{what} {nm}: {bad.sum()} elements beyond TOL and beyond 10x the fp32 probe; "
-                               f"worst {i}: gpu {g.flat[i]} fp64 {r.flat[i]} fp32 {pr.flat[i]}")
+        assert not bad.any(), (f"{what} {nm}: {bad.sum()} elements beyond TOL and outside the fp32-probe clause; "
+                               f"worst {i}: gpu {g.flat[i]} fp64 {r.flat[i]}"
+                               + (f" fp32 {pr[fi].flat[i]}" if pr is not None else ""))
         assert relaxed.mean() <= max_ill, f"{what} {nm}: {relaxed.sum()} of {relaxed.size} need the fp32 clause"
 
 
@@ -164,6 +189,21 @@ def test_trajectory_parity(forests, name, schedule):
         assert_rel(gl[-1][i], ol[-1][i], what=nm)
 
 
+@pytest.mark.parametrize("name", ["ispd18", "ispd19"])
+def test_trajectory_parity_100_iterations_full_size(name):
+    """BASELINE.json north_star: "the logits after 100 iterations in fp32 within 1e-4", at configs[2]
+    (ispd18, ~1e5 nets) and configs[3] (ispd19, ~1e6 nets, the bench workload), in the bench's launch
+    configuration: 100 iterations at t = 1 with Adam at lr 0.3, then every demand element
+    and every logit against the fp64 oracle, and the loss of the 100th forward (reading Q11)."""
+    f = forestgen.generate(name)
+    sched = [(100, 1.0)]
+    s, o, gl, ol = run_both(f, sched)
+    compare_state(s, o, name + " 100 it", probe=probes(f, sched), max_ill=1e-3)
+    for i, nm in enumerate(("total", "wl", "via", "overflow")):
+        assert_rel(gl[-1][i], ol[-1][i], what=nm)
+    assert s.iteration == 100
+
+
 @pytest.mark.parametrize("f_kind", [2, 3, 4])
 def test_alternative_activations_one_iteration(forests, f_kind):
     """Piecewise-linear f (LeakyReLU, CELU's linear branch) make exact cost ties common: the two L
@@ -180,12 +220,19 @@ def test_alternative_activations_one_iteration(forests, f_kind):
     tie_p, tie_t = np.abs(dw0) < 1e-10, np.abs(du0) < 1e-10
     gwt, gwp = s.logits()
     owt, owp = o.logits()
+    _record(f"alt_f{f_kind} ties", "w_path", n=int(tie_p.size), tie=int(tie_p.sum()),
+            max_abs_tie=float(np.abs(gwp - owp)[tie_p].max(initial=0)))
+    _record(f"alt_f{f_kind} ties", "w_tree", n=int(tie_t.size), tie=int(tie_t.sum()),
+            max_abs_tie=float(np.abs(gwt - owt)[tie_t].max(initial=0)))
     assert np.abs(gwp - owp)[tie_p].max(initial=0) <= 1e-3 and np.abs(gwt - owt)[tie_t].max(initial=0) <= 1e-3
     pr = probes(f, [(1, 1.0)], W)
     pwt, pwp = pr.logits()
     for g, r, p32, tie, nm in ((gwp, owp, pwp, tie_p, "w_path"), (gwt, owt, pwt, tie_t, "w_tree")):
         eg, e32 = scaled_err(g, r), scaled_err(p32, r)
-        bad = ~tie & (eg > TOL) & (eg > 10.0 * e32)
+        relaxed = ~tie & (eg > TOL) & (e32 > TOL) & (eg <= K_PROBE * e32) & (np.abs(g - r) <= 2 * LR + 1e-6)
+        bad = ~tie & (eg > TOL) & ~relaxed
+        PARITY_COUNTS[f"alt_f{f_kind} ties"][nm].update(probe=int(relaxed.sum()), bad=int(bad.sum()),
+                                                         strict=int((~tie & (eg <= TOL)).sum()))
         assert not bad.any(), f"f{f_kind} {nm}: {bad.sum()} bad"
     assert tie_p.mean() < 0.2
     gdh, gdv = s.demand(); odh, odv = o.demand()
@@ -309,6 +356,9 @@ def test_full_size_sampled_parity(name):
     owt, owp = o.logits()
     for g, r, d0, nm in ((gwp, owp, dw0, "w_path"), (gwt, owt, du0, "w_tree")):
         ill = np.abs(d0) < 1e-5
+        _record(name + " first-step |g|<1e-5", nm, n=int(ill.size), ill=int(ill.sum()),
+                ill_beyond_tol=int((ill & (np.abs(g - r) > TOL * np.maximum(np.abs(r), 1))).sum()),
+                max_abs_ill=float(np.abs(g - r)[ill].max(initial=0)))
         assert np.abs(g - r)[ill].max(initial=0) <= 2 * 0.3 + 1e-6, nm
         assert (ill & (np.abs(g - r) > TOL * np.maximum(np.abs(r), 1))).mean() <= 1e-5, nm
     compare_state(s, o, name, probe=probes(f, [(0, 1.0), (1, 1.0)]), max_ill=1e-4,
