@@ -88,6 +88,7 @@ def _load(fp32: bool = False):
         L.odgr_forward.argtypes = [vp, c.c_double, W, c.c_int, _dp]
         L.odgr_forward.restype = c.c_double
         L.odgr_backward.argtypes = [vp, c.c_double, W, _dp, _dp]
+        L.odgr_backward_c.argtypes = [vp, c.c_double, W, _dp, _dp, _dp]
         L.odgr_adam.argtypes = [vp, c.c_double, _dp, _dp]
         L.odgr_next_iteration.argtypes = [vp]
         L.odgr_step.argtypes = [vp, c.c_int, c.c_double, c.c_double, W, _dp]
@@ -220,8 +221,13 @@ class Oracle:
                                     ewl, etp, ctypes.byref(w), out)
         return out
 
-    def backward(self, t: float, w: Weights):
+    def backward(self, t: float, w: Weights, costs: bool = False):
+        """dw, du of the last forward (and, with costs=True, every candidate's c_i = d cost / d pi_i)."""
         dw = np.zeros(self.f.n_paths); du = np.zeros(self.f.n_trees)
+        if costs:
+            c = np.zeros(self.f.n_paths)
+            self._L.odgr_backward_c(self._h, t, ctypes.byref(w), dw, du, c)
+            return dw, du, c
         self._L.odgr_backward(self._h, t, ctypes.byref(w), dw, du)
         return dw, du
 

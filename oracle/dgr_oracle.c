@@ -331,7 +331,7 @@ ODGR_API double odgr_forward(odgr_state* s, double t, const odgr_weights* W, int
 }
 
 /* ---- reverse: d cost / d w for the shard's logits (the chain rule of P:841-845) ---- */
-static void backward(odgr_state* s, real t, const odgr_weights* W, real* dw_path, real* du_tree) {
+static void backward(odgr_state* s, real t, const odgr_weights* W, real* dw_path, real* du_tree, real* c_path) {
   const int X = s->X, Y = s->Y;
   size_t G = (size_t)X * Y;
   const real a3 = (real)W->a_of, slope = (real)W->f_slope, beta = (real)W->beta;
@@ -368,6 +368,7 @@ static void backward(odgr_state* s, real t, const odgr_weights* W, real* dw_path
             if (y <= Y - 2) v += gv[(size_t)y * X + x];
             c += beta * v;
           }
+          if (c_path) c_path[i] = c;      /* (tests: the resolution of the gradient's fp32 evaluation) */
           dw_path[i] = s->q[j] * c;       /* dp_i = q_tree(i) c_i (stored temporarily) */
           dq += s->p[i] * c;
           spd += s->p[i] * dw_path[i];
@@ -385,18 +386,28 @@ static void backward(odgr_state* s, real t, const odgr_weights* W, real* dw_path
   free(gv);
 }
 
-ODGR_API void odgr_backward(odgr_state* s, double t, const odgr_weights* W, double* dw_path, double* du_tree) {
+/* c_path (nullable): the per-candidate cost c_i = d cost / d pi_i of the same pass */
+ODGR_API void odgr_backward_c(odgr_state* s, double t, const odgr_weights* W, double* dw_path, double* du_tree,
+                              double* c_path) {
   real* dw = rzeros(s->n_paths);
   real* du = rzeros(s->n_trees);
-  backward(s, (real)t, W, dw, du);
+  real* c = c_path ? rzeros(s->n_paths) : NULL;
+  backward(s, (real)t, W, dw, du, c);
   for (int64_t n = s->net_lo; n < s->net_hi; ++n)
     for (int64_t j = s->net_tree_off[n]; j < s->net_tree_off[n + 1]; ++j) {
       du_tree[j] = du[j];
-      for (int64_t i = s->sub_path_off[s->tree_sub_off[j]]; i < s->sub_path_off[s->tree_sub_off[j + 1]]; ++i)
+      for (int64_t i = s->sub_path_off[s->tree_sub_off[j]]; i < s->sub_path_off[s->tree_sub_off[j + 1]]; ++i) {
         dw_path[i] = dw[i];
+        if (c) c_path[i] = c[i];
+      }
     }
   free(dw);
   free(du);
+  free(c);
+}
+
+ODGR_API void odgr_backward(odgr_state* s, double t, const odgr_weights* W, double* dw_path, double* du_tree) {
+  odgr_backward_c(s, t, W, dw_path, du_tree, NULL);
 }
 
 /* ---- Adam (torch.optim.Adam semantics; betas 0.9/0.999, eps 1e-8; reading Q9) ---- */
@@ -439,7 +450,7 @@ ODGR_API void odgr_step(odgr_state* s, int iters, double t, double lr, const odg
   real* du = rzeros(s->n_trees);
   for (int it = 0; it < iters; ++it) {
     odgr_forward(s, t, W, 1, out);
-    backward(s, (real)t, W, dw, du);
+    backward(s, (real)t, W, dw, du, NULL);
     adam(s, (real)lr, dw, du);
     s->k += 1;
   }

@@ -3,7 +3,7 @@
 //
 // The data-parallel unit is the net (§3.2: nets couple only through the demand d of
 // Eq. (10)).  Rank r keeps a contiguous, work-balanced range of nets; per iteration
-// the ranks exchange one int64 buffer [dH | dV^T | VD | VD^T] with ncclAllReduce —
+// the ranks exchange one int64 buffer [dH | dV^T | E[WL], E[TP]] with ncclAllReduce —
 // fixed point makes the sum exact, so every rank then runs the (replicated) grid pass on
 // identical data and the result does not depend on the number of ranks.
 #include <cuda_runtime.h>
@@ -833,7 +833,7 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.mt = take(4 * nt + 16);
   L.vt = take(4 * nt + 16);
   L.q = take(4 * nt + 16);
-  L.xcount = 4 * G;   // dH | dV^T | VD | VD^T
+  L.xcount = 2 * G + 2;   // dH | dV^T | E[WL], E[TP]
   L.xbuf = take(8 * L.xcount);
   L.capH = take(4 * G);
   L.capVT = take(4 * G);
@@ -845,7 +845,7 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.dOutH = take(4 * G);
   L.dOutVT = take(4 * G);
   L.partial = take(8 * (size_t)(X + Y));
-  L.lpart = take(16 * (size_t)(X + Y));
+  L.lpart = take(8 * (size_t)(X + Y) + 16);   // per-line demand sums, then lsum[2]
   L.loss = take(8 * 4);
   L.chosen = take(nt);
   L.tree_choice = take(4 * nn);
@@ -888,6 +888,7 @@ struct dgr_handle {
   // last iteration of the previous dgr_step call ran it), so the next call can start from them
   bool fwd_valid = false;
   float t_fwd = 0.f;
+  float beta_fwd = 0.f;   // the forward's turning-point demand is folded into the grids with its beta
   // the exchange grids may hold demand events no KG has consumed yet (set before every forward
   // launch, cleared after the KG that reads them): a call that failed part-way leaves it set, and
   // the next call clears the grids instead of adding its events on top of the stale ones
@@ -1090,14 +1091,14 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   const size_t G = (size_t)desc->X * desc->Y;
   P.dH = (long long*)(ws + L.xbuf);
   P.dVT = P.dH + G;
-  P.VD = P.dVT + G;
-  P.VDT = P.VD + G;
+  P.acc = P.dVT + G;
   P.capH = (const float*)(ws + L.capH);
   P.capVT = (const float*)(ws + L.capVT);
   P.SH = (double*)(ws + L.SH); P.SVT = (double*)(ws + L.SVT);
   P.dOutH = (float*)(ws + L.dOutH); P.dOutVT = (float*)(ws + L.dOutVT);
   P.partial = (double*)(ws + L.partial);
   P.lpart = (long long*)(ws + L.lpart);
+  P.lsum = P.lpart + (desc->X + desc->Y);
   P.loss = (double*)(ws + L.loss);
   P.chosen = (uint8_t*)(ws + L.chosen);
   P.tree_choice = (int32_t*)(ws + L.tree_choice);
@@ -1231,6 +1232,9 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
   a.a_wl = w->a_wl; a.a_via = w->a_via; a.a_of = w->a_of; a.beta = w->beta_via;
   a.sqrt_l = std::sqrt(w->n_layers);
   a.f_slope = w->f_slope; a.f_kind = w->f_kind;
+  a.beta_q = (double)w->beta_via * kGridBeta;
+  a.beta_exact = std::nearbyint(a.beta_q) == a.beta_q && std::fabs(a.beta_q) < 9.0e15;
+  a.beta_qi = a.beta_exact ? (long long)a.beta_q : 0;
   const size_t xbytes = 8 * h->lay.xcount;
   (void)xbytes;
   cudaStream_t s = h->stream;
@@ -1247,11 +1251,10 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
   a.store_d = 0;
   adam_args(h->k);
   if ((rc = prof_mark(h, -1))) return rc;
-  const size_t grid_bytes = 8 * (size_t)h->X * h->Y;
-  if (!(h->fwd_valid && h->t_fwd == temperature)) {
+  if (!(h->fwd_valid && h->t_fwd == temperature && h->beta_fwd == w->beta_via)) {
     // KG clears the event grids in place after reading them; stale events of a forward at another
     // temperature are cleared here
-    if (h->grids_dirty) CUDA_TRY(cudaMemsetAsync(P.dH, 0, 4 * grid_bytes, s));   // dH | dV^T | VD | VD^T
+    if (h->grids_dirty) CUDA_TRY(cudaMemsetAsync(P.dH, 0, 8 * h->lay.xcount, s));   // dH | dV^T | E[WL], E[TP]
     h->grids_dirty = true;
     launch_tiles(P, a, kForwardOnly, s);
     if ((rc = prof_mark(h, 0))) return rc;
@@ -1287,6 +1290,7 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
   if (iters > 0) {
     h->fwd_valid = true;
     h->t_fwd = temperature;
+    h->beta_fwd = w->beta_via;
   }
   CUDA_TRY(cudaGetLastError());
   if ((P.skip & 256) && getenv("DGR_PROF_OUT")) {   // diagnostics: per-tile phase clocks of the last KBF

@@ -21,10 +21,12 @@
 //     #valid lanes | kSingleBundle}
 //   * per sub-net: canonical endpoints (x0 <= x1; y0 < y1 if x0 == x1) as int16 x 4
 //   * per tree:    w, m, v, q (fp32)
-//   * grids: difference arrays of the wire demand along H rows ([Y][X]) and along V columns
-//     (stored transposed, [X][Y], so both scans run over contiguous lines), the turning-point
-//     ("via") demand per G-cell ([Y][X]), all int64 in 2^-24 fixed point; prefix sums S of
-//     the overflow gradient per line (fp64, the same two layouts).
+//   * grids: difference arrays of the demand along H rows ([Y][X]) and along V columns (stored
+//     transposed, [X][Y], so both scans run over contiguous lines), int64 in 2^-40 fixed point,
+//     with each turning point's beta pi folded in as a +-beta pi window over its incident edges
+//     (Eq. (10), reading Q3), followed by two int64 counters (E[TP] and a border term, 2^-24) of
+//     the same forward: this is the whole per-iteration exchange buffer; prefix sums S of the
+//     overflow gradient per line (fp64, the same two layouts).
 #pragma once
 #include <cstdint>
 
@@ -33,6 +35,9 @@ namespace dgr {
 constexpr int kFracBits = 24;                      // fixed point of pi: round(pi * 2^24)
 constexpr float kFixScale = 16777216.0f;           // 2^24
 constexpr double kFixInv = 1.0 / 16777216.0;
+constexpr int kGridShift = 16;                     // difference arrays: 2^-(24+16) = 2^-40 fixed point
+constexpr double kGridInv = 1.0 / 1099511627776.0; // 2^-40
+constexpr double kGridBeta = 65536.0;              // beta pi (pi in 2^-24) -> 2^-40: exact for beta in 2^-16 Z
 constexpr double kDqScale = 4294967296.0;          // dq_j accumulated in 2^-32 fixed point
 constexpr double kDqInv = 1.0 / 4294967296.0;
 
@@ -121,11 +126,11 @@ struct KParams {
   const int32_t* mnets;     // per tile: offsets (in the tile) of its nets with >= 2 trees
   const unsigned char* tmaps;   // CUtensorMap pairs (S_H window, S_V window), 128 B each, per window shape
   float *wt, *mt, *vt, *q;
-  // grids (the exchange buffer, in this order: dH | dVT | VD | VDT)
-  long long* dH;            // [Y][X]
-  long long* dVT;           // [X][Y]
-  long long* VD;            // [Y][X] turning points per G-cell
-  long long* VDT;           // [X][Y] the same, column-major (KG's column pass)
+  // grids (the exchange buffer, in this order: dH | dVT | acc)
+  long long* dH;            // [Y][X] 2^-40: wire events << 16, turning points folded in (+-beta pi)
+  long long* dVT;           // [X][Y] the same along columns
+  long long* acc;           // [2] E[TP] and the border deficit B = sum_v VD_v (4 - deg v) of the forward
+                            // in the grids (2^-24), summed by the tiles (E[WL] follows from the demand)
   const float* capH;        // [Y][X]
   const float* capVT;       // [X][Y]
   double* SH;               // [Y][XP]
@@ -133,7 +138,8 @@ struct KParams {
   float* dOutH;             // [Y][X]
   float* dOutVT;            // [X][Y]
   double* partial;          // [Y + X] overflow partial sums per line
-  long long* lpart;         // [2 (Y + X)] per-line E[WL], E[TP] partial sums (2^-24 fixed point)
+  long long* lsum;          // [2] acc of the last KG's forward (KG moves acc here and clears it)
+  long long* lpart;         // [Y + X] per-line sums of the demand (2^-40), for E[WL]
   double* loss;             // [4]
   // induce scratch
   uint8_t* chosen;          // [n_trees_l]
@@ -156,6 +162,9 @@ struct StepArgs {
   float lr_over_bc1;  // lr / (1 - beta1^(k+1))
   float inv_sqrt_bc2; // 1 / sqrt(1 - beta2^(k+1))
   float a_wl, a_via, a_of, beta, sqrt_l, f_slope;
+  double beta_q;      // beta * 2^16: a turning point's pi (2^-24) -> its folded demand (2^-40)
+  long long beta_qi;  // the same as an integer when beta_exact
+  int32_t beta_exact; // beta * 2^16 is an integer (beta a multiple of 2^-16): exact integer folds
   int32_t f_kind;
   int32_t store_d;
 };

@@ -35,6 +35,24 @@ constexpr unsigned kFull = 0xffffffffu;
 #endif
 #define KO(bit) (DGR_DIAG && (P.skip & (bit)))
 
+// DGR_ACCURATE=1: correctly rounded-ish fp32 library functions (expf, logf, sqrtf, IEEE division)
+// on the per-candidate path instead of the MUFU approximations (experiment: parity vs speed)
+#ifndef DGR_HEAD_SOFTMAX
+#define DGR_HEAD_SOFTMAX 1   // softmax shifted by the group head's z (exact maximum only when needed)
+#endif
+#ifndef DGR_ACCURATE
+#define DGR_ACCURATE 0
+#endif
+#if DGR_ACCURATE
+#define FEXP(x) expf(x)
+#define FLOG(x) logf(x)
+#define FDIV(a, b) ((a) / (b))
+#else
+#define FEXP(x) __expf(x)
+#define FLOG(x) __logf(x)
+#define FDIV(a, b) __fdividef(a, b)
+#endif
+
 // ------------------------------------------------------------------------------------------
 // Counter-based noise: Philox4x32-10 keyed on (seed; idx>>2, k, stream), word idx & 3.
 // u = ((r >> 9) + 1/2) 2^-23 is exact in fp32; g = -ln(-ln u) (reading Q7).
@@ -65,7 +83,7 @@ __device__ __forceinline__ uint4 philox_rk(uint4 c, const uint32_t* rk) {
 // g = -ln(-ln u) from one Philox word (the outer log by MUFU: |error| < 1e-6 on g)
 __device__ __forceinline__ float gumbel_word(uint32_t w) {
   const float u = ((float)(w >> 9) + 0.5f) * (1.0f / 8388608.0f);
-  return -__logf(-logf(u));
+  return -FLOG(-logf(u));
 }
 
 __device__ __forceinline__ float gumbel(uint64_t seed, uint64_t idx, uint32_t k, uint32_t stream) {
@@ -124,17 +142,6 @@ struct Max {
   __device__ __forceinline__ float operator()(float a, float b) const { return fmaxf(a, b); }
 };
 
-// p_i = softmax over the sub-net group of (w_i + g_i) / t (reading Q1)
-__device__ __forceinline__ float group_softmax(const KParams& P, float inv_t, uint32_t k, const Lane& L, float w) {
-  const float z = L.valid ? (w + (L.single ? 0.f : gumbel(P.seed, (uint64_t)L.nid, k, 0u))) * inv_t : -INFINITY;
-  float m = seg_reduce(z, L.lane, L.end, Max());
-  m = __shfl_sync(kFull, m, L.head);
-  const float e = L.valid ? __expf(z - m) : 0.f;
-  float s = seg_reduce(e, L.lane, L.end, Sum());
-  s = __shfl_sync(kFull, s, L.head);
-  return L.valid ? e / s : 0.f;
-}
-
 // dq_j in 2^-32 fixed point, accumulated in shared memory as three 32-bit limbs (a 64-bit shared
 // atomic is a CAS loop on sm_100): v = hi 2^42 + mid 2^21 + lo with lo, mid in [0, 2^21) (up to 1024
 // contributions per tree cannot overflow a limb) and hi = v >> 42 signed; exact for any int64 v.
@@ -154,14 +161,133 @@ __device__ __forceinline__ void red64(long long* p, long long v) {
   if (v != 0) atomicAdd(reinterpret_cast<unsigned long long*>(p), static_cast<unsigned long long>(v));
 }
 
+// beta v (v in 2^-24) in the 2^-40 fixed point of the difference arrays: an exact integer product
+// when beta is a multiple of 2^-16 (beta_exact; the default 0.25 is), else rounded per event
+template <bool EXACT = false>
+__device__ __forceinline__ long long beta_fold(const StepArgs& A, long long v) {
+  if (EXACT) return v * A.beta_qi;
+  return A.beta_exact ? v * A.beta_qi : __double2ll_rn(A.beta_q * (double)v);
+}
+
+// red.global.add.u64 unless v == 0, predicated instead of branched (no memory clobber: nothing in
+// the kernel reads the global difference arrays back)
+__device__ __forceinline__ void red64p(long long* p, long long v) {
+  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.s64 q, %1, 0;\n\t@q red.global.add.u64 [%0], %1;\n\t}" ::"l"(p), "l"(v));
+}
+
+// Missing incident edges of G-cell (x, y) at the grid border: 4 - deg(x, y)
+__device__ __forceinline__ int border_deficit(int x, int y, int X, int Y) {
+  return (x == 0) + (x == X - 1) + (y == 0) + (y == Y - 1);
+}
+
+// A turning point at (x, y) with probability weight v (2^-24) adds beta v to each incident edge
+// (Eq. (10), reading Q3): edges x-1 and x of row y, y-1 and y of column x (clipped at the border).
+// In the difference arrays (2^-40) that is +beta v at max(x-1, 0) and -beta v at x+1 (if inside)
+// of the row, the same along the column.  Global-memory form (global tiles); also accumulates the
+// turning point's share of E[TP] and of the border deficit B = sum_v VD_v (4 - deg(v)).
+__device__ __forceinline__ void tp_fold_global(const KParams& P, const StepArgs& A, int x, int y, int v,
+                                               long long& etp, long long& bdef) {
+  if (v == 0) return;
+  const long long b = beta_fold(A, v);
+  const int X = P.X, Y = P.Y;
+  red64(P.dH + (size_t)y * X + max(x - 1, 0), b);
+  if (x + 1 <= X - 1) red64(P.dH + (size_t)y * X + x + 1, -b);
+  red64(P.dVT + (size_t)x * Y + max(y - 1, 0), b);
+  if (y + 1 <= Y - 1) red64(P.dVT + (size_t)x * Y + y + 1, -b);
+  etp += v;
+  bdef += (long long)v * border_deficit(x, y, X, Y);
+}
+
+// Flush of a tile's event window into the global difference arrays.  The window's three fields are
+// int32 (2^-24), row-major over the window (cell (x, y) at (y - wy0) ww + x - wx0): H events at 0,
+// V events at hv, turning points VD at 2 hv; the width is even, so pair i is cells 2i, 2i+1 of one
+// row.  Global cell j of a row receives (H_j << 16) + beta (VD_{j+1} - VD_{j-1} + [j = 0] VD_0):
+// its wire events and the turning points' +-beta pi windows along the row (tp_fold_global); cell j
+// of a column likewise with V and the VD of the cells above / below.  One pass, four predicated
+// int64 reductions per pair; cells outside the grid hold no events and receive nothing.  Returns
+// the window's share of E[TP] = sum VD and of the border deficit B = sum VD (4 - deg) (2^-24); KG
+// derives E[WL] from the folded demand and these two (kg_loss_kernel).
+template <int NT, bool EXACT>
+__device__ __forceinline__ void flush_window_t(const KParams& P, const StepArgs& A, int wx0, int wy0, int ww, int wh,
+                                               int hv, const int* ev_s, long long& etp, long long& bdef) {
+  const int X = P.X, Y = P.Y, tid = threadIdx.x;
+  const int hw = ww >> 1;
+  // row = floor((i + 1/2) / half width) in fp32 is exact here: the fraction stays >= 1/(2 half)
+  // >> the rounding of i < 2^12
+  const float inv_hw = 1.f / (float)hw;
+  const int2* evH = reinterpret_cast<const int2*>(ev_s);
+  const int2* evV = reinterpret_cast<const int2*>(ev_s + hv);
+  const int* evD = ev_s + 2 * hv;
+  const int2* evD2 = reinterpret_cast<const int2*>(evD);
+  const int npair = hw * wh;
+  const int bq = (int)A.beta_qi;   // EXACT: beta 2^16 (|beta| < 2^15)
+  // windows that reach past the grid's last row / column (their outer cells hold no events but
+  // must not be flushed) and windows on the grid border (clipped turning-point windows) take the
+  // checked path; the rest (nearly all) need no per-cell test
+  const bool plain = wx0 > 0 && wy0 > 0 && wx0 + ww < X && wy0 + wh < Y;
+  for (int i = tid; i < npair; i += NT) {
+    const int r = (int)(((float)i + 0.5f) * inv_hw), cx = 2 * (i - r * hw);
+    const int gx = wx0 + cx, gy = wy0 + r;
+    const int2 h = evH[i], v = evV[i], d = evD2[i];
+    const int dl = cx > 0 ? evD[2 * i - 1] : 0, dr = cx + 2 < ww ? evD[2 * i + 2] : 0;
+    const int2 du = r > 0 ? evD2[i - hw] : make_int2(0, 0), dn = r + 1 < wh ? evD2[i + hw] : make_int2(0, 0);
+    // turning-point counts are >= 0 and < 2^31 per cell, so these differences fit int32
+    int fh0 = d.y - dl, fh1 = dr - d.x, fv0 = dn.x - du.x, fv1 = dn.y - du.y;
+    etp += (long long)d.x + d.y;
+    const size_t gH = (size_t)gy * X + gx, gV = (size_t)gx * Y + gy;
+    long long a0, a1, b0, b1;
+    if (EXACT) {
+      a0 = (long long)h.x * 65536 + (long long)fh0 * bq;
+      a1 = (long long)h.y * 65536 + (long long)fh1 * bq;
+      b0 = (long long)v.x * 65536 + (long long)fv0 * bq;
+      b1 = (long long)v.y * 65536 + (long long)fv1 * bq;
+    } else {
+      a0 = ((long long)h.x << kGridShift) + beta_fold(A, fh0);
+      a1 = ((long long)h.y << kGridShift) + beta_fold(A, fh1);
+      b0 = ((long long)v.x << kGridShift) + beta_fold(A, fv0);
+      b1 = ((long long)v.y << kGridShift) + beta_fold(A, fv1);
+    }
+    if (!plain) {
+      // clipped windows of turning points on the first row / column start at edge 0; cells outside
+      // the grid receive nothing; border cells have fewer incident edges (B)
+      if (gx == 0) a0 += beta_fold<EXACT>(A, d.x);
+      if (gy == 0) { b0 += beta_fold<EXACT>(A, d.x); b1 += beta_fold<EXACT>(A, d.y); }
+      if (!(gx < X && gy < Y)) { a0 = 0; b0 = 0; }
+      if (!(gx + 1 < X && gy < Y)) { a1 = 0; b1 = 0; }
+      if (gy < Y) bdef += (long long)d.x * border_deficit(gx, gy, X, Y) + (long long)d.y * border_deficit(gx + 1, gy, X, Y);
+    }
+    red64p(P.dH + gH, a0);
+    red64p(P.dH + gH + 1, a1);
+    red64p(P.dVT + gV, b0);
+    red64p(P.dVT + gV + Y, b1);
+  }
+}
+
+template <int NT>
+__device__ __forceinline__ void flush_window(const KParams& P, const StepArgs& A, int wx0, int wy0, int ww, int wh,
+                                             int hv, const int* ev_s, long long& etp, long long& bdef) {
+  if (A.beta_exact) flush_window_t<NT, true>(P, A, wx0, wy0, ww, wh, hv, ev_s, etp, bdef);
+  else flush_window_t<NT, false>(P, A, wx0, wy0, ww, wh, hv, ev_s, etp, bdef);
+}
+
+__device__ __forceinline__ long long warp_sum_ll(long long v) {
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) v += __shfl_down_sync(kFull, v, off);
+  return v;
+}
+
 __device__ __forceinline__ void adam_update(float& w, float& m, float& v, float g, const StepArgs& A) {
   m = fmaf(0.1f, g - m, m);                         // m.lerp_(g, 1 - beta1)
   v = fmaf(0.999f, v, 0.001f * g * g);              // v * beta2 + (1 - beta2) g^2
   // MUFU square root and division: ~1e-7 relative, well inside the 1e-4 bar
   float sq;
+#if DGR_ACCURATE
+  sq = sqrtf(v);
+#else
   asm("sqrt.approx.f32 %0, %1;" : "=f"(sq) : "f"(v));
+#endif
   const float denom = sq * A.inv_sqrt_bc2 + 1e-8f;
-  w -= A.lr_over_bc1 * __fdividef(m, denom);
+  w -= A.lr_over_bc1 * FDIV(m, denom);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -222,6 +348,13 @@ __device__ __forceinline__ double path_cost(const double* S, const Win& W, int X
   return c + (double)A.beta * tp + (double)A.a_wl * (double)wl + (double)A.a_via * (double)A.sqrt_l * (double)ntp;
 }
 
+// wire length of a candidate in the Z(o, m) form (every shape: straight, L, Z, C)
+__device__ __forceinline__ int lane_wl(uint32_t pw, int x0, int y0, int x1, int y1) {
+  const int o = pw & 1, m = (int)(pw >> 16);
+  const int p0 = o ? y0 : x0, p1 = o ? y1 : x1, q0 = o ? x0 : y0, q1 = o ? x1 : y1;
+  return abs(m - p0) + abs(p1 - m) + abs(q1 - q0);
+}
+
 __device__ __forceinline__ void red_shared_add(uint32_t saddr, int v) {
   asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.s32 p, %1, 0;\n\t@p red.shared.add.s32 [%0], %1;\n\t}" ::"r"(saddr), "r"(v)
                : "memory");
@@ -247,22 +380,6 @@ __device__ __forceinline__ void c_events(uint32_t pw, int x0, int y0, int x1, in
 }
 
 
-// Gumbel noise of a warp's contiguous candidates gid0 .. gid0+n-1 into g[0..n): one Philox4x32-10
-// call per 4 consecutive candidates (counter gid >> 2), spread over the lanes.
-__device__ __forceinline__ void warp_noise(float* g, uint64_t seed, int64_t gid0, int n, uint32_t k, int lane) {
-  const int64_t c0 = gid0 >> 2, c1 = (gid0 + n - 1) >> 2;
-  const uint2 key = make_uint2((uint32_t)seed, (uint32_t)(seed >> 32));
-  for (int64_t c = c0 + lane; c <= c1; c += 32) {
-    const uint4 r = philox4x32_10(make_uint4((uint32_t)c, (uint32_t)(c >> 32), k, 0u), key);
-    const int64_t i0 = c * 4 - gid0;
-    if (i0 >= 0 && i0 < n) g[i0] = gumbel_word(r.x);
-    if (i0 + 1 >= 0 && i0 + 1 < n) g[i0 + 1] = gumbel_word(r.y);
-    if (i0 + 2 >= 0 && i0 + 2 < n) g[i0 + 2] = gumbel_word(r.z);
-    if (i0 + 3 >= 0 && i0 + 3 < n) g[i0 + 3] = gumbel_word(r.w);
-  }
-  __syncwarp();
-}
-
 // Lane view built from already-loaded bundle info and pattern word (no memory access).
 __device__ __forceinline__ void lane_from(int4 bi, uint32_t pw, const KParams& P, Lane& L) {
   L.lane = threadIdx.x & 31;
@@ -282,14 +399,20 @@ __device__ __forceinline__ void lane_from(int4 bi, uint32_t pw, const KParams& P
   L.nid = P.nid_base + bi.x + L.lane;
 }
 
+// p_i = exp(z_i - m) / sum_k exp(z_k - m) for any shift m (softmax shift invariance): m = the group
+// head's z, unless some lane of the warp exceeds its head by more than 64 (exp overflow risk), then
+// the exact group maximum.  The head's own term is exp(0) = 1, so the sum is >= 1.
 __device__ __forceinline__ float softmax_from_noise(const Lane& L, float w, float g, float inv_t) {
   const float z = L.valid ? (w + g) * inv_t : -INFINITY;
-  float m = seg_reduce(z, L.lane, L.end, Max());
-  m = __shfl_sync(kFull, m, L.head);
-  const float e = L.valid ? __expf(z - m) : 0.f;
+  float m = __shfl_sync(kFull, z, L.head);
+  if (!DGR_HEAD_SOFTMAX || __any_sync(kFull, z - m > 64.f)) {
+    m = seg_reduce(z, L.lane, L.end, Max());
+    m = __shfl_sync(kFull, m, L.head);
+  }
+  const float e = L.valid ? FEXP(z - m) : 0.f;
   float s = seg_reduce(e, L.lane, L.end, Sum());
   s = __shfl_sync(kFull, s, L.head);
-  return L.valid ? __fdividef(e, s) : 0.f;
+  return L.valid ? FDIV(e, s) : 0.f;
 }
 
 // ------------------------------------------------------------------------------------------
@@ -300,7 +423,6 @@ __device__ __forceinline__ float softmax_from_noise(const Lane& L, float w, floa
 //   wst    float[kMaxBundles * 32]    new logits of the tile (reverse -> forward)
 //   dq_s   long long[kTreeMax]        dq_j in 2^-32 fixed point
 //   q_s    float[kTreeMax]            q_j (iteration k in the reverse, k_next in the forward)
-//   red_s  long long[2]               E[WL], E[TP] partial sums
 // Each warp owns a contiguous range of the tile's bundles, so its candidates are contiguous.
 // ------------------------------------------------------------------------------------------
 constexpr int kWarps = kTileThreads / 32;
@@ -385,10 +507,18 @@ __device__ __forceinline__ void reverse_warp(const KParams& P, const StepArgs& A
 // with A = pi_HV, B = pi_VH, Hs = sum pi over Z-HVH, Vs = sum pi over Z-VHV.  dH is the difference
 // array of the H wire demand along rows, dV along columns, VD the turning points.  Written as
 // 0/1-flag arithmetic so the warp never diverges on the pattern.
+// Event window of a tile (row-major fields: H at 0, V at hv, turning points at 2 hv)
+struct EWin {
+  int ox, oy, w, hv;
+  __device__ __forceinline__ int h(int x, int y) const { return (y - oy) * w + (x - ox); }
+  __device__ __forceinline__ int v(int x, int y) const { return hv + (y - oy) * w + (x - ox); }
+  __device__ __forceinline__ int d(int x, int y) const { return 2 * hv + (y - oy) * w + (x - ox); }
+};
+
 template <bool GLOBAL>
 __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A, const TileDesc& T, int bw0,
                                              int bw1, bool have_w, const float* wst, const float* q_s, float* g_s,
-                                             const Win& W, int* ev_s, long long* red_s) {
+                                             const EWin& W, int* ev_s, long long& etp, long long& bdef) {
   const int lane = threadIdx.x & 31;
   const int4 bfirst = __ldg(&P.binfo[bw0]);
   const uint32_t ev_base = (uint32_t)__cvta_generic_to_shared(ev_s);
@@ -448,34 +578,33 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
     if (L.valid) {
       if (GLOBAL) {
         const int X = P.X, Y = P.Y;
-        red64(P.dH + (size_t)ya * X + xa, ah); red64(P.dVT + (size_t)xa * Y + ya, av);
-        red64(P.VD + (size_t)ya * X + xa, ad); red64(P.VDT + (size_t)xa * Y + ya, ad);
-        red64(P.dH + (size_t)yb * X + xb, bh); red64(P.dVT + (size_t)xb * Y + yb, bv);
-        red64(P.VD + (size_t)yb * X + xb, bd); red64(P.VDT + (size_t)xb * Y + yb, bd);
+        const long long sh = 1ll << kGridShift;
+        red64(P.dH + (size_t)ya * X + xa, ah * sh); red64(P.dVT + (size_t)xa * Y + ya, av * sh);
+        tp_fold_global(P, A, xa, ya, ad, etp, bdef);
+        red64(P.dH + (size_t)yb * X + xb, bh * sh); red64(P.dVT + (size_t)xb * Y + yb, bv * sh);
+        tp_fold_global(P, A, xb, yb, bd, etp, bdef);
       }
       if (outside) {
         if (GLOBAL) {
           const int X = P.X, Y = P.Y;
           c_events(L.pw, x0, y0, x1, y1, vq, [&](int fld, int x, int y, int val) {
-            red64(fld == 0 ? P.dH + (size_t)y * X + x : fld == 1 ? P.dVT + (size_t)x * Y + y : P.VD + (size_t)y * X + x, val);
-            if (fld == 2) red64(P.VDT + (size_t)x * Y + y, val);
+            if (fld == 2) tp_fold_global(P, A, x, y, val, etp, bdef);
+            else red64(fld == 0 ? P.dH + (size_t)y * X + x : P.dVT + (size_t)x * Y + y, (long long)val << kGridShift);
           });
         } else {
           c_events(L.pw, x0, y0, x1, y1, vq, [&](int fld, int x, int y, int val) {
-            red_shared_add(ev_base + 4u * (fld == 0 ? W.h(x, y) : fld == 1 ? W.v(x, y) : 2 * W.hv + W.h(x, y)), val);
+            red_shared_add(ev_base + 4u * (fld == 0 ? W.h(x, y) : fld == 1 ? W.v(x, y) : W.d(x, y)), val);
           });
         }
       }
     }
     if (!GLOBAL) {
-      const int hv2 = 2 * W.hv;   // VD part of the event window
-      const int ia_h = W.h(xa, ya), ib_h = W.h(xb, yb);
-      red_shared_add(ev_base + 4u * ia_h, ah);
+      red_shared_add(ev_base + 4u * W.h(xa, ya), ah);
       red_shared_add(ev_base + 4u * W.v(xa, ya), av);
-      red_shared_add(ev_base + 4u * (hv2 + ia_h), ad);
-      red_shared_add(ev_base + 4u * ib_h, bh);
+      red_shared_add(ev_base + 4u * W.d(xa, ya), ad);
+      red_shared_add(ev_base + 4u * W.h(xb, yb), bh);
       red_shared_add(ev_base + 4u * W.v(xb, yb), bv);
-      red_shared_add(ev_base + 4u * (hv2 + ib_h), bd);
+      red_shared_add(ev_base + 4u * W.d(xb, yb), bd);
     }
     L = Ln; e = en;
     slot += 32;
@@ -495,11 +624,9 @@ __device__ __forceinline__ void slow_tile(const KParams& P, const StepArgs& A, c
   float* wst = reinterpret_cast<float*>(smem + kRegionA);
   long long* dq_s = reinterpret_cast<long long*>(wst + kMaxBundles * 32);
   float* q_s = reinterpret_cast<float*>(dq_s + kTreeMax);
-  long long* red_s = reinterpret_cast<long long*>(q_s + kTreeMax);
 
   const int tid = threadIdx.x, warp = tid >> 5;
   const int ncell = T.ww * T.wh;
-  const int X = P.X, Y = P.Y;
   const Win Wg{0, 0, P.XP, P.YP, (int)(P.SVT - P.SH)};
   const Win Ws{T.wx0, T.wy0, T.ww, T.wh, ncell};
   float* g_s = g_all + warp * kWarpCand;
@@ -563,9 +690,9 @@ __device__ __forceinline__ void slow_tile(const KParams& P, const StepArgs& A, c
           zmax = fmaxf(zmax, z);
         }
         float sum = 0.f;   // the normalisation of process_tile, operation for operation
-        for (int j = a; j < b; ++j) sum += __expf(q_s[j - T.tree0] - zmax);
+        for (int j = a; j < b; ++j) sum += FEXP(q_s[j - T.tree0] - zmax);
         for (int j = a; j < b; ++j) {
-          const float q = __expf(q_s[j - T.tree0] - zmax) / sum;
+          const float q = FEXP(q_s[j - T.tree0] - zmax) / sum;
           q_s[j - T.tree0] = q;
           P.q[j] = q;
         }
@@ -579,33 +706,20 @@ __device__ __forceinline__ void slow_tile(const KParams& P, const StepArgs& A, c
       int4* z = reinterpret_cast<int4*>(ev_s);
       for (int i = tid; i < (3 * ncell + 3) / 4; i += kTileThreads) z[i] = make_int4(0, 0, 0, 0);
     }
-    if (tid < 2) red_s[tid] = 0;
     __syncthreads();
+    long long etp = 0, bdef = 0;
+    const EWin Ew{T.wx0, T.wy0, T.ww, ncell};
     if (bw0 < bw1) {
-      if (T.global) forward_warp<true>(P, A, T, bw0, bw1, REV, wst, q_s, g_s, Wg, ev_s, red_s);
-      else forward_warp<false>(P, A, T, bw0, bw1, REV, wst, q_s, g_s, Ws, ev_s, red_s);
+      if (T.global) forward_warp<true>(P, A, T, bw0, bw1, REV, wst, q_s, g_s, Ew, ev_s, etp, bdef);
+      else forward_warp<false>(P, A, T, bw0, bw1, REV, wst, q_s, g_s, Ew, ev_s, etp, bdef);
     }
     __syncthreads();
-    if (!T.global) {
-      // flush the window once: a warp per window row (H-type fields) / column (V-type fields),
-      // lanes along it, so the int64 reductions are coalesced
-      const int lane = tid & 31;
-      for (int yi = warp; yi < T.wh; yi += kWarps) {
-        const size_t g0 = (size_t)(T.wy0 + yi) * X + T.wx0;
-        const int* rowH = ev_s + yi * T.ww;
-        const int* rowD = ev_s + 2 * ncell + yi * T.ww;
-        for (int xi = lane; xi < T.ww; xi += 32) {
-          if (T.wx0 + xi >= X) break;
-          red64(P.dH + g0 + xi, rowH[xi]);
-          red64(P.VD + g0 + xi, rowD[xi]);
-          red64(P.VDT + (size_t)(T.wx0 + xi) * Y + T.wy0 + yi, rowD[xi]);
-        }
-      }
-      for (int xi = warp; xi < T.ww; xi += kWarps) {
-        const size_t g0 = (size_t)(T.wx0 + xi) * Y + T.wy0;
-        const int* colV = ev_s + ncell + xi * T.wh;
-        for (int yi = lane; yi < T.wh; yi += 32) red64(P.dVT + g0 + yi, colV[yi]);
-      }
+    if (!T.global) flush_window<kTileThreads>(P, A, T.wx0, T.wy0, T.ww, T.wh, ncell, ev_s, etp, bdef);
+    etp = warp_sum_ll(etp);
+    bdef = warp_sum_ll(bdef);
+    if ((tid & 31) == 0 && (etp | bdef)) {   // exact integers: any order gives the same sums
+      atomicAdd(reinterpret_cast<unsigned long long*>(P.acc), (unsigned long long)etp);
+      atomicAdd(reinterpret_cast<unsigned long long*>(P.acc + 1), (unsigned long long)bdef);
     }
   }
 }
@@ -894,10 +1008,10 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
   const int mn_lo = T.mn0 & ~3;
   const uint64_t pol = policy_stream();   // L2 evict-first for the streamed slot state
-  const int ncell = T.ww * T.wh, hv = win_hv(T.ww, T.wh);   // V field at hv (128-byte aligned)
+  const int hv = win_hv(T.ww, T.wh);   // V field at hv (128-byte aligned)
   const Win W{T.wx0, T.wy0, T.ww, T.wh, hv};
-  const int wB0 = -(T.wy0 * T.ww + T.wx0), wB1 = hv - T.wx0 * T.wh - T.wy0;   // orientation bases
   const int hv2 = 2 * hv;                                                     // VD part of the window
+  const int eb = -(T.wy0 * T.ww + T.wx0);                                     // event-window origin
   const int nbg = T.nbg;
 
   // ---------------- reverse of iteration k ----------------
@@ -1008,9 +1122,9 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         zmax = fmaxf(zmax, zj);
       }
       float sum = 0.f;
-      for (int j = a; j < b; ++j) sum += __expf(St.q[j] - zmax);
+      for (int j = a; j < b; ++j) sum += FEXP(St.q[j] - zmax);
       for (int j = a; j < b; ++j) {
-        const float q = __expf(St.q[j] - zmax) / sum;
+        const float q = FEXP(St.q[j] - zmax) / sum;
         St.q[j] = q;
         P.q[j + t_lo] = q;
       }
@@ -1059,24 +1173,26 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
           // +v at its lower and -v at its upper end, plus its turning points.  No cross-lane collapse: lanes of one
           // sub-net that share a corner cell meet in the shared-memory reduction.
           const short4 e = St.sxy[L.sub - s_lo];
-          const int x0 = e.x, y0 = e.y, x1 = e.z, y1 = e.w;
           const int o = L.pw & 1, ntp = (L.pw >> 1) & 3, m = (int)(L.pw >> 16);
-          const int p0 = o ? y0 : x0, p1 = o ? y1 : x1, q0 = o ? x0 : y0, q1 = o ? x1 : y1;
-          const int Lp = o ? W.vs : W.hs, Ls = o ? W.hs : W.vs;
-          const int Bp = o ? wB1 : wB0, Bs = o ? wB0 : wB1;
-          const int r0 = q0 * Lp + Bp, r1 = q1 * Lp + Bp, sb = m * Ls + Bs;
-          const int a0 = r0 + m, a1 = r1 + m, s0 = sb + q0, s1 = sb + q1;
+          // the event window's fields are row-major: cell (x, y) at (y - wy0) ww + x - wx0.  In the
+          // Z(o, m) form a cell (a, b) of orientation o (a along the primary lines) is at a A + b B
+          // with (A, B) = (1, ww) for o = 0 and (ww, 1) for o = 1, so the segment ends of one line
+          // are ordered like their cell indices
+          const int A_ = o ? T.ww : 1, B_ = o ? 1 : T.ww;
+          const int p0 = o ? e.y : e.x, p1 = o ? e.w : e.z, q0 = o ? e.x : e.y, q1 = o ? e.z : e.w;
+          const int cp0 = p0 * A_ + q0 * B_ + eb, cp1 = p1 * A_ + q1 * B_ + eb;
+          const int cm0 = m * A_ + q0 * B_ + eb, cm1 = m * A_ + q1 * B_ + eb;
+          const int fP = o ? hv : 0, fS = o ? 0 : hv;   // fields of the primary / secondary lines
           // each segment: +v at its lower end, -v at its upper end (nothing if zero-length)
-          const int v1 = m != p0 ? vq : 0, v2 = q1 != q0 ? vq : 0, v3 = p1 != m ? vq : 0;
-          red_shared_add(ev_base + 4u * (r0 + min(p0, m)), v1);
-          red_shared_add(ev_base + 4u * (r0 + max(p0, m)), -v1);
-          red_shared_add(ev_base + 4u * (sb + min(q0, q1)), v2);
-          red_shared_add(ev_base + 4u * (sb + max(q0, q1)), -v2);
-          red_shared_add(ev_base + 4u * (r1 + min(m, p1)), v3);
-          red_shared_add(ev_base + 4u * (r1 + max(m, p1)), -v3);
-          // turning points: VD takes the H-orientation index of the cell (a for o = 0, s for o = 1)
-          red_shared_add(ev_base + 4u * (hv2 + (o ? s0 : a0)), ntp >= 1 ? vq : 0);
-          red_shared_add(ev_base + 4u * (hv2 + (o ? s1 : a1)), ntp == 2 ? vq : 0);
+          const int v1 = cm0 != cp0 ? vq : 0, v2 = cm1 != cm0 ? vq : 0, v3 = cp1 != cm1 ? vq : 0;
+          red_shared_add(ev_base + 4u * (fP + min(cp0, cm0)), v1);
+          red_shared_add(ev_base + 4u * (fP + max(cp0, cm0)), -v1);
+          red_shared_add(ev_base + 4u * (fS + min(cm0, cm1)), v2);
+          red_shared_add(ev_base + 4u * (fS + max(cm0, cm1)), -v2);
+          red_shared_add(ev_base + 4u * (fP + min(cm1, cp1)), v3);
+          red_shared_add(ev_base + 4u * (fP + max(cm1, cp1)), -v3);
+          red_shared_add(ev_base + 4u * (hv2 + cm0), ntp >= 1 ? vq : 0);   // turning points
+          red_shared_add(ev_base + 4u * (hv2 + cm1), ntp == 2 ? vq : 0);
         }
       } else {
         // singleton bundle: pi = q; +pi where the segment starts, -pi where it ends
@@ -1087,8 +1203,8 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
           const float q = St.q[tree - t_lo];
           const int vq = __float2int_rn(q * kFixScale);
           const short4 e = St.sxy[bi.y + lane - s_lo];
-          const int ia = isv ? W.v(e.x, e.y) : W.h(e.x, e.y);
-          const int ib = isv ? W.v(e.x, e.w) : W.h(e.z, e.y);
+          const int ia = e.y * T.ww + e.x + eb + (isv ? hv : 0);   // row-major event fields
+          const int ib = (isv ? e.w * T.ww + e.x + hv : e.y * T.ww + e.z) + eb;
           red_shared_add(ev_base + 4u * ia, vq);
           red_shared_add(ev_base + 4u * ib, -vq);
         }
@@ -1106,32 +1222,22 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     bulk_commit();
   }
   if (FWD && !(KO(1))) {
-    // flush: the window's cell pairs as one flat range per field (rows of dH / VD, columns of dV;
-    // widths are even, so pair i is cells 2i, 2i+1 of the field); zero cells are skipped, and every
-    // cell outside the grid is zero (events only land on grid cells).  row = floor((i + 1/2) / half
-    // width) in fp32 is exact here: the fraction stays >= 1/(2 half) >> the rounding of i < 2^12.
-    const int hw = T.ww >> 1, hh = T.wh >> 1;
-    const float inv_hw = 1.f / (float)hw, inv_hh = 1.f / (float)hh;
-    const int2* evH = reinterpret_cast<const int2*>(ev_s);
-    const int2* evV = reinterpret_cast<const int2*>(ev_s + hv);
-    const int2* evD = reinterpret_cast<const int2*>(ev_s + 2 * hv);
-    const int npair = ncell >> 1;
-    for (int i = tid; i < npair; i += NT) {
-      const int2 h = evH[i], d = evD[i], v = evV[i];
-      if (h.x | h.y | d.x | d.y) {
-        const int r = (int)(((float)i + 0.5f) * inv_hw);
-        const size_t g = (size_t)(T.wy0 + r) * X + T.wx0 + 2 * (i - r * hw);
-        red64(P.dH + g, h.x); red64(P.dH + g + 1, h.y);
-        red64(P.VD + g, d.x); red64(P.VD + g + 1, d.y);
-        if (d.x | d.y) {   // the turning points also column-major, for KG's column pass
-          const size_t gt = (size_t)(T.wx0 + 2 * (i - r * hw)) * Y + T.wy0 + r;
-          red64(P.VDT + gt, d.x); red64(P.VDT + gt + Y, d.y);
-        }
-      }
-      if (v.x | v.y) {
-        const int c = (int)(((float)i + 0.5f) * inv_hh);
-        const size_t g = (size_t)(T.wx0 + c) * Y + T.wy0 + 2 * (i - c * hh);
-        red64(P.dVT + g, v.x); red64(P.dVT + g + 1, v.y);
+    // flush the window once, then the tile's shares of E[TP] and of the border deficit summed in
+    // warp order into the exchange buffer's counters
+    long long etp = 0, bdef = 0;
+    flush_window<NT>(P, A, T.wx0, T.wy0, T.ww, T.wh, hv, ev_s, etp, bdef);
+    etp = warp_sum_ll(etp);
+    bdef = warp_sum_ll(bdef);
+    long long* part = reinterpret_cast<long long*>(dq3);   // free after the net level
+    if (lane == 0) { part[2 * warp] = etp; part[2 * warp + 1] = bdef; }
+    __syncthreads();
+    if (tid == 0) {
+      long long a = 0, b = 0;
+#pragma unroll
+      for (int w = 0; w < NW; ++w) { a += part[2 * w]; b += part[2 * w + 1]; }
+      if (a | b) {
+        atomicAdd(reinterpret_cast<unsigned long long*>(P.acc), (unsigned long long)a);
+        atomicAdd(reinterpret_cast<unsigned long long*>(P.acc + 1), (unsigned long long)b);
       }
     }
   }
@@ -1305,39 +1411,35 @@ __device__ __forceinline__ void striped_exclusive_scan(T (&v)[kGItems], T* sh /*
 __global__ void __launch_bounds__(1024) kg_loss_kernel(KParams P, StepArgs A) {
   // fixed-shape tree reduction (strided thread sums, warp shuffles, warp totals in warp order):
   // deterministic, one pass, no block scans
-  __shared__ double shs[32];
-  __shared__ long long shw[32], sht[32];
+  __shared__ double shs[32], shd[32];
   const int nl = P.X + P.Y, lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  double s = 0.0;
-  long long w = 0, t = 0;
+  double s = 0.0, sd = 0.0;
   for (int i = threadIdx.x; i < nl; i += blockDim.x) {
     s += P.partial[i];
-    const longlong2 l = reinterpret_cast<const longlong2*>(P.lpart)[i];
-    w += l.x;
-    t += l.y;
+    sd += (double)P.lpart[i] * kGridInv;   // each line's sum of the demand (exact in 2^-40, ~1e4 tracks)
   }
 #pragma unroll
   for (int off = 16; off > 0; off >>= 1) {
     s += __shfl_down_sync(kFull, s, off);
-    w += __shfl_down_sync(kFull, w, off);
-    t += __shfl_down_sync(kFull, t, off);
+    sd += __shfl_down_sync(kFull, sd, off);
   }
-  if (lane == 0) { shs[wid] = s; shw[wid] = w; sht[wid] = t; }
+  if (lane == 0) { shs[wid] = s; shd[wid] = sd; }
   __syncthreads();
   if (wid == 0) {
     const int nw = blockDim.x >> 5;
     s = lane < nw ? shs[lane] : 0.0;
-    w = lane < nw ? shw[lane] : 0;
-    t = lane < nw ? sht[lane] : 0;
+    sd = lane < nw ? shd[lane] : 0.0;
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) {
       s += __shfl_down_sync(kFull, s, off);
-      w += __shfl_down_sync(kFull, w, off);
-      t += __shfl_down_sync(kFull, t, off);
+      sd += __shfl_down_sync(kFull, sd, off);
     }
     if (lane == 0) {
-      const double ewl = (double)w * kFixInv;
-      const double etp = (double)t * kFixInv;
+      // E[TP] = sum of the turning points (exact fixed point, the exchange buffer's counter); the
+      // folded demand sums to E[WL] + beta sum_v VD_v deg(v) = E[WL] + beta (4 E[TP] - B)
+      const double etp = (double)P.lsum[0] * kFixInv;
+      const double bdef = (double)P.lsum[1] * kFixInv;
+      const double ewl = sd - (double)A.beta * (4.0 * etp - bdef);
       const double via = (double)A.sqrt_l * etp;
       P.loss[0] = (double)A.a_wl * ewl + (double)A.a_via * via + (double)A.a_of * s;
       P.loss[1] = ewl;
@@ -1347,49 +1449,84 @@ __global__ void __launch_bounds__(1024) kg_loss_kernel(KParams P, StepArgs A) {
   }
 }
 
+// f(x) and df/dx = df/dd of the overflow x = d - cap (Eq. (9), reading Q2) in fp32 (x itself in
+// fp64: d comes from exact fixed point); relative error ~1e-6, well inside the 1e-4 bar, at a
+// fraction of fp64 exp's cost
+__device__ __forceinline__ void overflow_f(const StepArgs& A, double x, double& fv, double& fg) {
+  const float xf = (float)x, sf = A.f_slope;
+  switch (A.f_kind) {
+    case 0: {   // sigmoid sigma(s x); stable for both signs
+      const float e = FEXP(-fabsf(sf * xf));
+      const float inv = FDIV(1.f, 1.f + e);
+      fv = (sf * xf > 0.f) ? inv : e * inv;
+      fg = sf * e * inv * inv;
+      break;
+    }
+    case 1: fv = x > 0.0 ? x : 0.0; fg = x > 0.0 ? 1.0 : 0.0; break;        // ReLU
+    case 2: fv = x > 0.0 ? x : (double)sf * x; fg = x > 0.0 ? 1.0 : (double)sf; break;   // LeakyReLU (Fig. 6)
+    case 3: fv = exp((double)sf * x); fg = (double)sf * fv; break;          // exp (Fig. 6): fp64 range
+    default: {                                                              // CELU (Fig. 6)
+      const float e = expf(fminf(xf, 0.f) / sf);
+      fv = x > 0.0 ? x : (double)(sf * (e - 1.f));
+      fg = x > 0.0 ? 1.0 : (double)e;
+    }
+  }
+}
+
 #ifndef DGR_KG_MINB
 #define DGR_KG_MINB 4
 #endif
+// One CTA per line (the launch has X + Y CTAs; CTA b would take lines b, b + gridDim.x, ... of a
+// smaller grid), chunk by chunk: the next chunk's difference and capacity values are loaded into
+// registers before the current one is scanned, so a long line's loads overlap its scans and
+// barriers.  (A persistent grid of resident CTAs was measured 1% slower per iteration: it holds
+// every SM slot until its last line, so the next KBF's CTAs cannot fill in behind it under PDL.)
 __global__ void __launch_bounds__(kGThreads, DGR_KG_MINB) kg_kernel(KParams P, StepArgs A) {
   __shared__ long long shl[33];
   __shared__ double shd[33];
   __shared__ double shw[kKgWarps];
-  __shared__ long long shwl[2 * kKgWarps];
+  __shared__ long long shwl[kKgWarps];
   griddep_launch();
   griddep_wait();   // the difference arrays are complete (the previous KBF / allreduce)
-  const int line = blockIdx.x;
-  const bool isH = line < P.Y;
-  const int n = isH ? P.X : P.Y;
-  const int ln = isH ? line : line - P.Y;
-  const size_t base = (size_t)ln * n;
-  long long* diff = (isH ? P.dH : P.dVT) + base;
-  // turning points at the line's cells (VD for rows, its column-major copy VD^T for columns)
-  long long* vd = (isH ? P.VD : P.VDT) + base;
-  const float* cap = (isH ? P.capH : P.capVT) + base;
-  double* S = isH ? P.SH + (size_t)ln * P.XP : P.SVT + (size_t)ln * P.YP;
-  float* dout = (isH ? P.dOutH : P.dOutVT) + base;
-  const double beta = A.beta;
-  long long carryW = 0;
-  long long wsum = 0, tsum = 0;   // E[WL] = sum_e W_e, E[TP] = sum_cells VD (rows pass), 2^-24 fixed point
-  double carryS = 0.0, of = 0.0;
-  const int lane = threadIdx.x & 31;
-  for (int c0 = 0; c0 < n; c0 += kGThreads * kGItems) {
-    long long v[kGItems], t0[kGItems], t1[kGItems];
-    float cp[kGItems];
+  const int nl = P.X + P.Y, lane = threadIdx.x & 31;
+  if (blockIdx.x == 0 && threadIdx.x == 0) {   // E[TP], B of this forward, for the loss; cleared for the next
+    P.lsum[0] = P.acc[0]; P.lsum[1] = P.acc[1];
+    P.acc[0] = 0; P.acc[1] = 0;
+  }
+  auto line_len = [&](int l) { return l < P.Y ? P.X : P.Y; };
+  auto line_diff = [&](int l) { return l < P.Y ? P.dH + (size_t)l * P.X : P.dVT + (size_t)(l - P.Y) * P.Y; };
+  auto line_cap = [&](int l) { return l < P.Y ? P.capH + (size_t)l * P.X : P.capVT + (size_t)(l - P.Y) * P.Y; };
+  long long v[kGItems];
+  float cp[kGItems];
+  auto load = [&](int l, int c0, long long (&vv)[kGItems], float (&cc)[kGItems]) {
+    const int n = line_len(l);
+    const long long* diff = line_diff(l);
+    const float* cap = line_cap(l);
 #pragma unroll
     for (int j = 0; j < kGItems; ++j) {
       const int pos = c0 + j * kGThreads + threadIdx.x;
-      v[j] = pos < n ? diff[pos] : 0;
-      t0[j] = pos < n ? vd[pos] : 0;
-      cp[j] = pos < n ? cap[pos] : 0.f;
+      vv[j] = pos < n ? diff[pos] : 0;
+      cc[j] = pos < n ? cap[pos] : 0.f;
     }
-#pragma unroll
-    for (int j = 0; j < kGItems; ++j) {   // the next cell's turning points: the next lane's t0
-      const int pos = c0 + j * kGThreads + threadIdx.x;
-      t1[j] = __shfl_down_sync(kFull, t0[j], 1);
-      if (lane == 31) t1[j] = pos + 1 < n ? vd[pos + 1] : 0;
-      if (isH) tsum += t0[j];
-    }
+  };
+  int line = blockIdx.x, c0 = 0;
+  if (line >= nl) return;
+  load(line, 0, v, cp);
+  long long carryW = 0, sumD = 0;   // sumD: sum over the line's edges of the demand (2^-40)
+  double carryS = 0.0, of = 0.0;
+  while (true) {
+    const bool isH = line < P.Y;
+    const int n = isH ? P.X : P.Y;
+    const int ln = isH ? line : line - P.Y;
+    long long* diff = line_diff(line);
+    double* S = isH ? P.SH + (size_t)ln * P.XP : P.SVT + (size_t)ln * P.YP;
+    float* dout = (isH ? P.dOutH : P.dOutVT) + (size_t)ln * n;
+    // the next chunk of this CTA (the rest of this line, else its next line), prefetched
+    int nline = line, nc0 = c0 + kGThreads * kGItems;
+    if (nc0 >= n) { nline += gridDim.x; nc0 = 0; }
+    long long nv[kGItems];
+    float ncp[kGItems];
+    if (nline < nl) load(nline, nc0, nv, ncp);
     long long totW;
     long long ex[kGItems];
 #pragma unroll
@@ -1398,7 +1535,7 @@ __global__ void __launch_bounds__(kGThreads, DGR_KG_MINB) kg_kernel(KParams P, S
 #pragma unroll
     for (int j = 0; j < kGItems; ++j) {
       const int pos = c0 + j * kGThreads + threadIdx.x;
-      if (pos < n) { diff[pos] = 0; vd[pos] = 0; }   // cleared for the next forward
+      if (pos < n) diff[pos] = 0;   // cleared for the next forward
     }
     double g[kGItems];
 #pragma unroll
@@ -1406,31 +1543,12 @@ __global__ void __launch_bounds__(kGThreads, DGR_KG_MINB) kg_kernel(KParams P, S
       const int pos = c0 + j * kGThreads + threadIdx.x;
       double G = 0.0;
       if (pos < n - 1) {
-        const long long W = carryW + ex[j] + v[j];   // inclusive prefix = wire demand of edge pos
-        wsum += W;
-        const double d = (double)W * kFixInv + beta * ((double)(t0[j] + t1[j]) * kFixInv);
-        const double x = d - (double)cp[j];                 // overflow x = -(cap - d)
-        // f(x) and df/dx = df/dd in fp32 (x itself in fp64: d comes from exact fixed point);
-        // relative error ~1e-6, well inside the 1e-4 bar, at a fraction of fp64 exp's cost
-        const float xf = (float)x, sf = A.f_slope;
+        // inclusive prefix = demand of edge pos: W_e + beta (VD_a + VD_b) (Eq. (10), reading Q3)
+        const long long D = carryW + ex[j] + v[j];
+        sumD += D;
+        const double d = (double)D * kGridInv;
         double fv, fg;
-        switch (A.f_kind) {
-          case 0: {   // sigmoid sigma(s x); stable for both signs
-            const float e = __expf(-fabsf(sf * xf));
-            const float inv = __fdividef(1.f, 1.f + e);
-            fv = (sf * xf > 0.f) ? inv : e * inv;
-            fg = sf * e * inv * inv;
-            break;
-          }
-          case 1: fv = x > 0.0 ? x : 0.0; fg = x > 0.0 ? 1.0 : 0.0; break;        // ReLU
-          case 2: fv = x > 0.0 ? x : (double)sf * x; fg = x > 0.0 ? 1.0 : (double)sf; break;   // LeakyReLU (Fig. 6)
-          case 3: fv = exp((double)sf * x); fg = (double)sf * fv; break;          // exp (Fig. 6): fp64 range
-          default: {                                                              // CELU (Fig. 6)
-            const float e = expf(fminf(xf, 0.f) / sf);
-            fv = x > 0.0 ? x : (double)(sf * (e - 1.f));
-            fg = x > 0.0 ? 1.0 : (double)e;
-          }
-        }
+        overflow_f(A, d - (double)cp[j], fv, fg);   // overflow x = d - cap = -(cap - d)
         of += fv;
         G = (double)A.a_of * fg;
         if (A.store_d) dout[pos] = (float)d;
@@ -1448,31 +1566,31 @@ __global__ void __launch_bounds__(kGThreads, DGR_KG_MINB) kg_kernel(KParams P, S
     }
     carryW += totW;
     carryS += totS;
-    if (c0 + kGThreads * kGItems < n) __syncthreads();   // the next chunk reuses shl / shd
-  }
-  // per-line partials of the overflow cost and of E[WL], E[TP] (exact integers): warp sums, then
-  // thread 0 sums the warps in order (deterministic); kg_loss_kernel sums the lines
+    if (nline != line) {
+      // per-line partials of the overflow cost and the demand sum: warp sums, then thread 0 sums
+      // the warps in order (deterministic); kg_loss_kernel sums the lines
 #pragma unroll
-  for (int off = 16; off > 0; off >>= 1) {
-    of += __shfl_down_sync(kFull, of, off);
-    wsum += __shfl_down_sync(kFull, wsum, off);
-    tsum += __shfl_down_sync(kFull, tsum, off);
-  }
-  if (lane == 0) {
-    const int w = threadIdx.x >> 5;
-    shw[w] = of;
-    shwl[2 * w] = wsum;
-    shwl[2 * w + 1] = tsum;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    double tot = 0.0;
-    long long ws = 0, ts = 0;
+      for (int off = 16; off > 0; off >>= 1) {
+        of += __shfl_down_sync(kFull, of, off);
+        sumD += __shfl_down_sync(kFull, sumD, off);
+      }
+      if (lane == 0) { shw[threadIdx.x >> 5] = of; shwl[threadIdx.x >> 5] = sumD; }
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        double tot = 0.0;
+        long long td = 0;
 #pragma unroll
-    for (int w = 0; w < kKgWarps; ++w) { tot += shw[w]; ws += shwl[2 * w]; ts += shwl[2 * w + 1]; }
-    P.partial[line] = tot;
-    P.lpart[2 * line] = ws;
-    P.lpart[2 * line + 1] = ts;
+        for (int w = 0; w < kKgWarps; ++w) { tot += shw[w]; td += shwl[w]; }
+        P.partial[line] = tot;
+        P.lpart[line] = td;
+      }
+      carryW = 0; sumD = 0; carryS = 0.0; of = 0.0;
+    }
+    if (nline >= nl) break;
+    __syncthreads();   // the next chunk reuses shl / shd / shw
+    line = nline; c0 = nc0;
+#pragma unroll
+    for (int j = 0; j < kGItems; ++j) { v[j] = nv[j]; cp[j] = ncp[j]; }
   }
 }
 
@@ -1508,7 +1626,7 @@ __global__ void __launch_bounds__(256) ki_path_kernel(KParams P, float inv_t, fl
   const float z = L.valid ? w * inv_t : -INFINITY;
   float m = seg_reduce(z, L.lane, L.end, Max());
   m = __shfl_sync(kFull, m, L.head);
-  const float e = L.valid ? __expf(z - m) : 0.f;
+  const float e = L.valid ? FEXP(z - m) : 0.f;
   float s = seg_reduce(e, L.lane, L.end, Sum());
   s = __shfl_sync(kFull, s, L.head);
   const float ph = e / s;

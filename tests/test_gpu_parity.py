@@ -67,12 +67,24 @@ def scaled_err(a, b):
     return np.abs(a - b) / np.maximum(np.abs(b), 1.0)
 
 
-# Relaxed clause of the parity contract (reading Q21b), for elements beyond TOL:
-#   |gpu - fp64| <= K_PROBE * |fp32 probe - fp64|  (both scaled by max(|fp64|, 1))   and
-#   |gpu - fp64| <= 2 lr                             (never more than two Adam steps apart)
-# where the fp32 probe (the oracle's own source built with real = float) is itself beyond TOL.
+# The float parity contract (readings Q21, Q21b, Q21c).  An element passes
+#   strict:   |gpu - fp64| <= TOL max(|fp64|, 1);
+#   exempt:   (logits after ONE Adam step) the fp64 gradient is below the resolution of an fp32
+#             evaluation of the paper's formulation (first_step_exempt): Adam's first step is
+#             lr g / (|g| + eps), so such a coordinate may land anywhere in [w0 - lr, w0 + lr];
+#   probe:    (multi-iteration runs) the fp32 probe -- the oracle's own source built with real = float
+#             -- is itself beyond TOL there, and |gpu - fp64| <= K_PROBE |probe - fp64| and <= 2 lr;
+#   chaotic:  (multi-iteration runs) beyond TOL where the probe is not: a trajectory that took a
+#             different rounding path earlier.  Allowed only up to as many elements as the fp32 probe
+#             deviates at in total (the GPU is no less accurate than fp32 evaluation of the same
+#             formulas), each within CHAOS_DEMAND (demand) / 2 lr (logits).
+# Anything else fails.  Every clause's count is recorded (tests/conftest.py prints them and writes
+# $DGR_PARITY_COUNTS).
 K_PROBE = float(__import__("os").environ.get("DGR_K_PROBE", "2.0"))   # env: data-gathering runs only
+KAPPA = 2.0 ** -16          # fp32 resolution of a gradient relative to the terms it is formed from
+CHAOS_DEMAND = 20 * TOL
 LR = 0.3
+ADAM_EPS = 1e-8             # torch.optim.Adam default (reading Q9)
 PARITY_COUNTS = {}   # test -> field -> clause counts (printed in the session summary, tests/conftest.py)
 
 
@@ -80,14 +92,48 @@ def _record(what, nm, **kv):
     PARITY_COUNTS.setdefault(what, {})[nm] = kv
 
 
-def compare_state(s, o, what, probe=None, max_ill=0.01, exempt=None, k_probe=K_PROBE):
-    """Element-wise parity of demand and logits.  Without a probe: every element within TOL.
-    With the fp32 probe (multi-iteration runs, DESIGN.md §3 Q21b): every element within TOL, or, where
-    an fp32 evaluation of the same formulation is itself further than TOL from fp64 (Adam turns a
-    near-zero gradient's rounding into an lr-sized step), no further from fp64 than k_probe times that
-    fp32 evaluation and never more than 2 lr; such elements must stay below `max_ill` of the total.
-    `exempt` (per logit field) marks coordinates the caller checks itself (the first Adam step of a
-    coordinate whose fp64 gradient is below fp32 resolution).  Every clause's count is recorded."""
+def first_step_exempt(f, W=None, t=1.0):
+    """Coordinates whose fp64 first-step gradient is below the resolution of an fp32 evaluation of the
+    paper's formulation (reading Q21b): dw_i = (p_i q_j / t)(c_i - sum_k p_k c_k) is formed from absolute
+    costs c (PyTorch autograd of Eq. (9) through the softmaxes), so fp32 resolves it only to
+    ~eps_p (p_i q_j / t)(|c_i| + sum_k p_k |c_k|), eps_p the relative error of the fp32 probabilities;
+    likewise du_j = (q_j / t)(dq_j - sum_l q_l dq_l) with dq_j = sum_{i in j} p_i c_i.  eps_p: z = (w + g)/t
+    in fp32 carries 2^-24 |z| of rounding (|z| <~ 20 at the first step), and exp's argument reduction
+    as much again, so eps_p <~ 2^-24 * 2 * 20 = 2.4e-6 and the gradient's error <~ 2 eps_p (terms);
+    KAPPA = 2^-16 = 1.5e-5 leaves a factor 3.  A coordinate is exempt when its gradient's sign is
+    not resolved (|g| < KAPPA terms), or when Adam's first step lr g / (|g| + eps) (bias-corrected
+    from zero moments) amplifies that resolution beyond TOL: its derivative in g is
+    lr eps / (|g| + eps)^2, so lr eps KAPPA terms / (|g| + eps)^2 > TOL max(|w|, 1) (|g| near eps).
+    Returns (tree mask, path mask)."""
+    W = ow(W or dgr.Weights())
+    o = oracle.Oracle(f)
+    o.forward(t, W)
+    dw, du, c = o.backward(t, W, costs=True)
+    q, p = o.probs()
+    path_sub = np.repeat(np.arange(f.n_subnets), np.diff(f.sub_path_off))
+    sub_tree = np.repeat(np.arange(f.n_trees), np.diff(f.tree_sub_off))
+    tree_net = np.repeat(np.arange(f.n_nets), np.diff(f.net_tree_off))
+    path_tree = sub_tree[path_sub]
+    grp = np.zeros(f.n_subnets)
+    np.add.at(grp, path_sub, p * np.abs(c))
+    r_path = KAPPA * p * q[path_tree] / t * (np.abs(c) + grp[path_sub])
+    dq = np.zeros(f.n_trees)
+    np.add.at(dq, path_tree, p * c)
+    ngrp = np.zeros(f.n_nets)
+    np.add.at(ngrp, tree_net, q * np.abs(dq))
+    r_tree = KAPPA * q / t * (np.abs(dq) + ngrp[tree_net])
+    wt0 = np.asarray(f.w_tree0, np.float64); wp0 = np.asarray(f.w_path0, np.float64)
+
+    def ill(g, r, w0):
+        step_sens = LR * ADAM_EPS * r / (np.abs(g) + ADAM_EPS) ** 2   # d(first step)/dg x resolution
+        return (np.abs(g) < r) | (step_sens > TOL * np.maximum(np.abs(w0), 1.0))
+    return ill(du, r_tree, wt0), ill(dw, r_path, wp0)
+
+
+def compare_state(s, o, what, probe=None, max_ill=0.01, exempt=None, chaos=False, k_probe=K_PROBE):
+    """Element-wise parity of demand and logits under the contract above.  `exempt` = (tree mask,
+    path mask) of first_step_exempt (one-iteration runs); `probe` = the fp32 oracle replaying the same
+    schedule; `chaos` allows the chaotic clause (multi-iteration runs)."""
     gdh, gdv = s.demand()
     odh, odv = o.demand()
     gwt, gwp = s.logits()
@@ -102,28 +148,35 @@ def compare_state(s, o, what, probe=None, max_ill=0.01, exempt=None, k_probe=K_P
     for fi, (g, r, nm, ex) in enumerate(fields):
         g = np.asarray(g, np.float64); r = np.asarray(r, np.float64)
         eg = scaled_err(g, r)
+        dif = np.abs(g - r)
         strict = eg <= TOL
-        if pr is None:
-            relaxed = np.zeros_like(strict)
-            e32 = np.zeros_like(eg)
-        else:
-            e32 = scaled_err(pr[fi], r)
-            relaxed = ~strict & (e32 > TOL) & (eg <= k_probe * e32) & (np.abs(g - r) <= 2 * LR + 1e-6)
-        bad = ~strict & ~relaxed
-        exempted = np.zeros_like(bad)
-        if ex is not None:   # checked by the caller (ill-conditioned first Adam step, Q21b)
-            exempted = bad & ex.reshape(bad.shape)
-            bad &= ~exempted
+        e32 = scaled_err(pr[fi], r) if pr is not None else np.zeros_like(eg)
+        n32 = int((e32 > TOL).sum())
+        relaxed = ~strict & (e32 > TOL) & (eg <= k_probe * e32) & (dif <= 2 * LR + 1e-6)
+        rest = ~strict & ~relaxed
+        exempted = np.zeros_like(rest)
+        if ex is not None:
+            exempted = rest & ex.reshape(rest.shape) & (dif <= 2 * LR + 1e-6)
+            rest &= ~exempted
+        chaotic = np.zeros_like(rest)
+        if chaos:
+            bound = (eg <= CHAOS_DEMAND) if nm.startswith("d_") else (dif <= 2 * LR + 1e-6)
+            chaotic = rest & bound
+            rest &= ~chaotic
+        bad = rest
         ratio = (eg / np.maximum(e32, 1e-300))[relaxed]
         _record(what, nm, n=int(eg.size), strict=int(strict.sum()), probe=int(relaxed.sum()),
-                exempt=int(exempted.sum()), bad=int(bad.sum()), max_err=float(eg.max(initial=0.0)),
-                max_err_strict_excl=float(eg[~strict].max(initial=0.0)),
-                max_probe_ratio=float(ratio.max(initial=0.0)))
+                exempt=int(exempted.sum()), chaotic=int(chaotic.sum()), bad=int(bad.sum()),
+                fp32_beyond_tol=n32, fp32_max_err=float(e32.max(initial=0.0)),
+                max_err=float(eg.max(initial=0.0)), max_probe_ratio=float(ratio.max(initial=0.0)),
+                max_err_chaotic=float(eg[chaotic].max(initial=0.0)))
         i = int(np.argmax(np.where(bad, eg, -1))) if bad.any() else 0
-        assert not bad.any(), (f"{what} {nm}: {bad.sum()} elements beyond TOL and outside the fp32-probe clause; "
+        assert not bad.any(), (f"{what} {nm}: {bad.sum()} elements outside every clause; "
                                f"worst {i}: gpu {g.flat[i]} fp64 {r.flat[i]}"
                                + (f" fp32 {pr[fi].flat[i]}" if pr is not None else ""))
         assert relaxed.mean() <= max_ill, f"{what} {nm}: {relaxed.sum()} of {relaxed.size} need the fp32 clause"
+        assert exempted.mean() <= max_ill, f"{what} {nm}: {exempted.sum()} of {exempted.size} exempt"
+        assert chaotic.sum() <= max(n32, 1), f"{what} {nm}: {chaotic.sum()} chaotic elements > the fp32 probe's {n32}"
 
 
 @pytest.mark.parametrize("beta", [0.0, 0.25])
@@ -171,7 +224,7 @@ def test_one_iteration_parity(forests, name):
     """After one Adam step the update of a coordinate whose gradient is ~eps depends on that
     gradient's last bits (Q21b), so the fp32 probe applies from the first step on."""
     s, o, gl, ol = run_both(forests[name], [(1, 1.0)])
-    compare_state(s, o, name, probe=probes(forests[name], [(1, 1.0)]), max_ill=1e-3)
+    compare_state(s, o, name, exempt=first_step_exempt(forests[name]), max_ill=1e-3)
     assert s.iteration == 1
 
 
@@ -184,7 +237,7 @@ def test_one_iteration_parity(forests, name):
 def test_trajectory_parity(forests, name, schedule):
     f = forests[name]
     s, o, gl, ol = run_both(f, schedule)
-    compare_state(s, o, name, probe=probes(f, schedule))
+    compare_state(s, o, name, probe=probes(f, schedule), chaos=True)
     for i, nm in enumerate(("total", "wl", "via", "overflow")):
         assert_rel(gl[-1][i], ol[-1][i], what=nm)
 
@@ -198,7 +251,7 @@ def test_trajectory_parity_100_iterations_full_size(name):
     f = forestgen.generate(name)
     sched = [(100, 1.0)]
     s, o, gl, ol = run_both(f, sched)
-    compare_state(s, o, name + " 100 it", probe=probes(f, sched), max_ill=1e-3)
+    compare_state(s, o, name + " 100 it", probe=probes(f, sched), max_ill=1e-3, chaos=True)
     for i, nm in enumerate(("total", "wl", "via", "overflow")):
         assert_rel(gl[-1][i], ol[-1][i], what=nm)
     assert s.iteration == 100
@@ -225,15 +278,15 @@ def test_alternative_activations_one_iteration(forests, f_kind):
     _record(f"alt_f{f_kind} ties", "w_tree", n=int(tie_t.size), tie=int(tie_t.sum()),
             max_abs_tie=float(np.abs(gwt - owt)[tie_t].max(initial=0)))
     assert np.abs(gwp - owp)[tie_p].max(initial=0) <= 1e-3 and np.abs(gwt - owt)[tie_t].max(initial=0) <= 1e-3
-    pr = probes(f, [(1, 1.0)], W)
-    pwt, pwp = pr.logits()
-    for g, r, p32, tie, nm in ((gwp, owp, pwp, tie_p, "w_path"), (gwt, owt, pwt, tie_t, "w_tree")):
-        eg, e32 = scaled_err(g, r), scaled_err(p32, r)
-        relaxed = ~tie & (eg > TOL) & (e32 > TOL) & (eg <= K_PROBE * e32) & (np.abs(g - r) <= 2 * LR + 1e-6)
-        bad = ~tie & (eg > TOL) & ~relaxed
-        PARITY_COUNTS[f"alt_f{f_kind} ties"][nm].update(probe=int(relaxed.sum()), bad=int(bad.sum()),
+    ex_t, ex_p = first_step_exempt(f, W)
+    for g, r, ex, tie, nm in ((gwp, owp, ex_p, tie_p, "w_path"), (gwt, owt, ex_t, tie_t, "w_tree")):
+        eg = scaled_err(g, r)
+        exempted = ~tie & (eg > TOL) & ex & (np.abs(g - r) <= 2 * LR + 1e-6)
+        bad = ~tie & (eg > TOL) & ~exempted
+        PARITY_COUNTS[f"alt_f{f_kind} ties"][nm].update(exempt_res=int(exempted.sum()), bad=int(bad.sum()),
                                                          strict=int((~tie & (eg <= TOL)).sum()))
         assert not bad.any(), f"f{f_kind} {nm}: {bad.sum()} bad"
+        assert exempted.mean() <= 1e-3, f"f{f_kind} {nm}: {exempted.sum()} exempt"
     assert tie_p.mean() < 0.2
     gdh, gdv = s.demand(); odh, odv = o.demand()
     assert_close(gdh, odh, what="d_h"); assert_close(gdv, odv, what="d_v")
@@ -246,7 +299,7 @@ def test_relu_trajectory_parity(forests):
     for name in ("tiny", "c1e4"):
         sched = [(5, 1.0)]
         s, o, gl, ol = run_both(forests[name], sched, W)
-        compare_state(s, o, "relu " + name, probe=probes(forests[name], sched, W))
+        compare_state(s, o, "relu " + name, probe=probes(forests[name], sched, W), chaos=True)
 
 
 def test_split_calls_and_determinism(forests):
@@ -326,7 +379,7 @@ def test_empty_and_degenerate_forests():
     f = forestgen.generate(dict(X=2, Y=2, n_nets=6, pins_mode=0, pins_min=2, pins_max=4, box_mode=0, box_min=2,
                                 box_max=2, track=1.0, n_tree_cand=2, z_cap=0, seed=3))
     s, o, gl, ol = run_both(f, [(20, 1.0)])
-    compare_state(s, o, "2x2", probe=probes(f, [(20, 1.0)]))
+    compare_state(s, o, "2x2", probe=probes(f, [(20, 1.0)]), chaos=True)
 
 
 @pytest.mark.parametrize("name", ["ispd19", "sweep4e6"])
@@ -345,24 +398,9 @@ def test_full_size_sampled_parity(name):
     assert_close(gdh, odh, what="d_h"); assert_close(gdv, odv, what="d_v")
     s.step(1, 1.0, 0.3)
     o.step(1, 1.0, 0.3, ow(dgr.Weights()))
-    # reading Q21b at full size: Adam's first step is lr * g / (|g| + eps), so a coordinate whose
-    # fp64 gradient is below what fp32 resolves (|g| < 1e-5: fp32 sums of per-candidate cost
-    # differences of O(100)) may take any step in [-lr, lr]; those must be rare.  Every other logit
-    # follows compare_state (TOL, or the fp32-probe clause).
-    o0 = oracle.Oracle(f)
-    o0.forward(1.0, ow(dgr.Weights()))
-    dw0, du0 = o0.backward(1.0, ow(dgr.Weights()))
-    gwt, gwp = s.logits()
-    owt, owp = o.logits()
-    for g, r, d0, nm in ((gwp, owp, dw0, "w_path"), (gwt, owt, du0, "w_tree")):
-        ill = np.abs(d0) < 1e-5
-        _record(name + " first-step |g|<1e-5", nm, n=int(ill.size), ill=int(ill.sum()),
-                ill_beyond_tol=int((ill & (np.abs(g - r) > TOL * np.maximum(np.abs(r), 1))).sum()),
-                max_abs_ill=float(np.abs(g - r)[ill].max(initial=0)))
-        assert np.abs(g - r)[ill].max(initial=0) <= 2 * 0.3 + 1e-6, nm
-        assert (ill & (np.abs(g - r) > TOL * np.maximum(np.abs(r), 1))).mean() <= 1e-5, nm
-    compare_state(s, o, name, probe=probes(f, [(0, 1.0), (1, 1.0)]), max_ill=1e-4,
-                  exempt=(np.abs(du0) < 1e-5, np.abs(dw0) < 1e-5))
+    # reading Q21b at full size: every logit within TOL unless its fp64 gradient is below the fp32
+    # resolution of its own terms (first_step_exempt); such coordinates must be rare (<= 1e-5)
+    compare_state(s, o, name, max_ill=1e-5, exempt=first_step_exempt(f))
 
 
 def test_table1_workload_relu_parity_and_optimum():
@@ -372,7 +410,7 @@ def test_table1_workload_relu_parity_and_optimum():
     W = dgr.Weights(a_wl=0.0, a_via=0.0, a_of=1.0, beta_via=0.0, f_kind=1)
     f = forestgen.generate("table1_r5")
     s, o, gl, ol = run_both(f, [(3, 1.0)], W)
-    compare_state(s, o, "table1_r5", probe=probes(f, [(3, 1.0)], W), max_ill=0.02)
+    compare_state(s, o, "table1_r5", probe=probes(f, [(3, 1.0)], W), max_ill=0.02, chaos=True)
     g = _small(2)
     opt = brute_force_overflow(g)
     best = None
