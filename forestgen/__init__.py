@@ -37,7 +37,7 @@ class _Config(ctypes.Structure):
         ("box_mu", ctypes.c_double), ("cluster_frac", ctypes.c_double), ("n_hotspots", ctypes.c_int32),
         ("track", ctypes.c_double), ("beta_pin", ctypes.c_double), ("n_tree_cand", ctypes.c_int32),
         ("z_cap", ctypes.c_int32), ("seed", ctypes.c_uint64), ("local_weight", ctypes.c_double),
-        ("c_cap", ctypes.c_int32),
+        ("c_cap", ctypes.c_int32), ("m_cap", ctypes.c_int32),
     ]
 
 
@@ -135,6 +135,14 @@ CONFIGS: dict[str, dict] = {
                    z_cap=0, c_cap=2, seed=3),
     "c1e4_c": dict(X=256, Y=256, n_nets=10_000, pins_mode=1, box_mode=1, box_mu=8.0, cluster_frac=0.0,
                    n_hotspots=0, track=1.0, beta_pin=0.25, n_tree_cand=2, z_cap=11, c_cap=2, seed=1),
+    # row f4' (reading Q14c): monotone staircases (4 turning points) and groups > 32 (uncapped Z)
+    "tiny_m": dict(X=32, Y=32, n_nets=40, pins_mode=0, pins_min=2, pins_max=4, box_mode=0, box_min=14,
+                   box_max=24, cluster_frac=0.0, n_hotspots=0, track=1.0, beta_pin=0.0, n_tree_cand=2,
+                   z_cap=0, c_cap=1, m_cap=2, seed=7),
+    "c1e4_m": dict(X=256, Y=256, n_nets=10_000, pins_mode=1, box_mode=1, box_mu=8.0, cluster_frac=0.0,
+                   n_hotspots=0, track=1.0, beta_pin=0.25, n_tree_cand=2, z_cap=24, c_cap=1, m_cap=2, seed=1),
+    "ispd18_m": dict(X=600, Y=600, n_nets=100_000, pins_mode=1, box_mode=1, box_mu=6.0, cluster_frac=0.3,
+                     n_hotspots=8, track=2.0, beta_pin=0.25, n_tree_cand=2, z_cap=24, c_cap=1, m_cap=2, seed=1),
     "ispd19_c": dict(X=1000, Y=1000, n_nets=1_000_000, pins_mode=1, box_mode=1, box_mu=5.0,
                      cluster_frac=0.3, n_hotspots=32, track=4.0, beta_pin=0.25, n_tree_cand=2, z_cap=11,
                      c_cap=2, seed=1),
@@ -212,7 +220,7 @@ def generate(config: str | dict, seed: int | None = None, gumbel_seed: int = GUM
     c = _Config()
     defaults = dict(pins_min=2, pins_max=4, box_min=2, box_max=8, box_mu=5.0, cluster_frac=0.0,
                     n_hotspots=0, track=1.0, beta_pin=0.0, n_tree_cand=2, z_cap=15, seed=1,
-                    pins_mode=0, box_mode=0, local_weight=1.0, c_cap=0)
+                    pins_mode=0, box_mode=0, local_weight=1.0, c_cap=0, m_cap=0)
     for k, v in {**defaults, **cfg}.items():
         setattr(c, k, v)
     lib = _load()
@@ -315,3 +323,44 @@ def subset(f: Forest, net_lo: int, net_hi: int) -> Forest:
         cap_h=f.cap_h, cap_v=f.cap_v,
         w_tree0=f.w_tree0[t0:t1].copy(), w_path0=f.w_path0[p0:p1].copy(), seed=f.seed,
     )
+
+
+def _gather_paths(f: Forest, order: np.ndarray) -> dict:
+    """CSR path arrays (segments, turning points, initial logits) with the paths in `order`."""
+    nseg = np.diff(f.path_seg_off)[order]
+    ntp = np.diff(f.path_tp_off)[order]
+    seg_idx = np.concatenate([np.arange(f.path_seg_off[p], f.path_seg_off[p + 1]) for p in order]) if len(order) else np.zeros(0, np.int64)
+    tp_idx = np.concatenate([np.arange(f.path_tp_off[p], f.path_tp_off[p + 1]) for p in order]) if len(order) else np.zeros(0, np.int64)
+    return dict(path_seg_off=np.concatenate([[0], np.cumsum(nseg)]).astype(np.int64),
+                path_tp_off=np.concatenate([[0], np.cumsum(ntp)]).astype(np.int64),
+                seg=f.seg[seg_idx].copy(), tp_xy=f.tp_xy[tp_idx].copy(), w_path0=f.w_path0[order].copy())
+
+
+def shuffle_candidates(f: Forest, seed: int = 0) -> Forest:
+    """The same forest with every sub-net's path candidates in a random order (a valid forest the
+    tile kernel's canonical order does not cover: it runs on the general path, row f4')."""
+    rng = np.random.default_rng(seed)
+    order = np.concatenate([f.sub_path_off[s] + rng.permutation(int(f.sub_path_off[s + 1] - f.sub_path_off[s]))
+                            for s in range(f.n_subnets)]).astype(np.int64) if f.n_subnets else np.zeros(0, np.int64)
+    g = Forest(X=f.X, Y=f.Y, net_tree_off=f.net_tree_off.copy(), tree_sub_off=f.tree_sub_off.copy(),
+               sub_path_off=f.sub_path_off.copy(), sub_xy=f.sub_xy.copy(), cap_h=f.cap_h, cap_v=f.cap_v,
+               w_tree0=f.w_tree0.copy(), seed=f.seed, **_gather_paths(f, order))
+    g.meta = dict(f.meta, shuffled_candidates=seed)
+    return g
+
+
+def shuffle_nets(f: Forest, seed: int = 0) -> Forest:
+    """The same forest with its nets in a random order (trees, sub-nets and paths follow their net)."""
+    rng = np.random.default_rng(seed)
+    nets = rng.permutation(f.n_nets)
+    trees = np.concatenate([np.arange(f.net_tree_off[n], f.net_tree_off[n + 1]) for n in nets]).astype(np.int64)
+    subs = np.concatenate([np.arange(f.tree_sub_off[t], f.tree_sub_off[t + 1]) for t in trees]).astype(np.int64)
+    paths = np.concatenate([np.arange(f.sub_path_off[s], f.sub_path_off[s + 1]) for s in subs]).astype(np.int64)
+    g = Forest(X=f.X, Y=f.Y,
+               net_tree_off=np.concatenate([[0], np.cumsum(np.diff(f.net_tree_off)[nets])]).astype(np.int64),
+               tree_sub_off=np.concatenate([[0], np.cumsum(np.diff(f.tree_sub_off)[trees])]).astype(np.int64),
+               sub_path_off=np.concatenate([[0], np.cumsum(np.diff(f.sub_path_off)[subs])]).astype(np.int64),
+               sub_xy=f.sub_xy[subs].copy(), cap_h=f.cap_h, cap_v=f.cap_v, w_tree0=f.w_tree0[trees].copy(),
+               seed=f.seed, **_gather_paths(f, paths))
+    g.meta = dict(f.meta, shuffled_nets=seed)
+    return g

@@ -15,6 +15,7 @@
 #include "forestgen.h"
 
 #include <algorithm>
+#include <array>
 #include <cmath>
 #include <cstdio>
 #include <cstring>
@@ -167,7 +168,25 @@ void c_positions(int lo, int hi, int c_cap, int n, std::vector<int>* pos) {
   for (int d = 1; d <= c_cap; ++d) if (hi + d < n) pos->push_back(hi + d);
 }
 
-void enumerate_paths(const Sub& s, int z_cap, int c_cap, int X, int Y, NetOut& o) {
+// Monotone staircase corners (row f4', reading Q14c) along a span [lo, hi] of length a >= 3 and
+// a cross span of length b >= 2: for k = 1..m_cap, first corner lo + max(1, floor(k a / (2 (m_cap + 1)))),
+// second corner half-way from it to hi (strictly inside), cross line lo' + floor(k b / (m_cap + 1))
+// clamped strictly inside; duplicates dropped
+void stair_corners(int lo, int a, int clo, int b, int m_cap, std::vector<std::array<int, 3>>* out) {
+  out->clear();
+  if (m_cap <= 0 || a < 3 || b < 2) return;
+  for (int k = 1; k <= m_cap; ++k) {
+    int p1 = lo + std::max(1, (k * a) / (2 * (m_cap + 1)));
+    p1 = std::min(p1, lo + a - 2);
+    const int p2 = p1 + std::max(1, (lo + a - p1) / 2);
+    int q = clo + (k * b) / (m_cap + 1);
+    q = std::min(std::max(q, clo + 1), clo + b - 1);
+    const std::array<int, 3> c{p1, std::min(p2, lo + a - 1), q};
+    if (std::find(out->begin(), out->end(), c) == out->end()) out->push_back(c);
+  }
+}
+
+void enumerate_paths(const Sub& s, int z_cap, int c_cap, int m_cap, int X, int Y, NetOut& o) {
   const int x0 = s.x0, y0 = s.y0, x1 = s.x1, y1 = s.y1;
   int np = 0;
   if (y0 == y1) {                       // straight H
@@ -209,6 +228,26 @@ void enumerate_paths(const Sub& s, int z_cap, int c_cap, int X, int Y, NetOut& o
       add_seg(o, 1, x0, y0, ym); add_seg(o, 0, ym, x0, x1); add_seg(o, 1, x1, ym, y1);
       add_tp(o, x0, ym); add_tp(o, x1, ym);
       o.path_nseg.push_back(3); o.path_ntp.push_back(2); ++np;
+    }
+    // monotone staircases (Q14c): HVHVH turning at x_a, x_b on an intermediate row y_m, then
+    // VHVHV turning at y_a, y_b (from y0 towards y1) on an intermediate column x_m
+    std::vector<std::array<int, 3>> st;
+    const int b = std::abs(y1 - y0), sy = y1 > y0 ? 1 : -1;
+    stair_corners(x0, x1 - x0, 0, b, m_cap, &st);
+    for (auto& c : st) {
+      const int xa = c[0], xb = c[1], ym = y0 + sy * c[2];
+      add_seg(o, 0, y0, x0, xa); add_seg(o, 1, xa, y0, ym); add_seg(o, 0, ym, xa, xb);
+      add_seg(o, 1, xb, ym, y1); add_seg(o, 0, y1, xb, x1);
+      add_tp(o, xa, y0); add_tp(o, xa, ym); add_tp(o, xb, ym); add_tp(o, xb, y1);
+      o.path_nseg.push_back(5); o.path_ntp.push_back(4); ++np;
+    }
+    stair_corners(0, b, x0, x1 - x0, m_cap, &st);
+    for (auto& c : st) {
+      const int ya = y0 + sy * c[0], yb = y0 + sy * c[1], xm = c[2];
+      add_seg(o, 1, x0, y0, ya); add_seg(o, 0, ya, x0, xm); add_seg(o, 1, xm, ya, yb);
+      add_seg(o, 0, yb, xm, x1); add_seg(o, 1, x1, yb, y1);
+      add_tp(o, x0, ya); add_tp(o, xm, ya); add_tp(o, xm, yb); add_tp(o, x1, yb);
+      o.path_nseg.push_back(5); o.path_ntp.push_back(4); ++np;
     }
   }
   o.sub_npath.push_back(np);
@@ -269,7 +308,7 @@ void build_trees(const forestgen_config& c, NetOut& o) {
     o.tree_nsub.push_back((int)t.size());
     for (auto& s : t) {
       o.subs.push_back(s);
-      enumerate_paths(s, c.z_cap, c.c_cap, c.X, c.Y, o);
+      enumerate_paths(s, c.z_cap, c.c_cap, c.m_cap, c.X, c.Y, o);
     }
   }
 }
@@ -303,6 +342,7 @@ extern "C" int forestgen_generate(const forestgen_config* cp, forestgen_forest**
   if (c.box_mode == 0 && (c.box_min < 1 || c.box_max < c.box_min)) { g_err = "bad box range"; return -1; }
   if (c.n_tree_cand < 1 || c.n_tree_cand > 2) { g_err = "n_tree_cand must be 1 or 2"; return -1; }
   if (c.c_cap < 0) { g_err = "c_cap < 0"; return -1; }
+  if (c.m_cap < 0) { g_err = "m_cap < 0"; return -1; }
   const int X = c.X, Y = c.Y;
 
   // hotspots (global stream)

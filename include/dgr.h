@@ -27,9 +27,8 @@
  *   G-cell grid X x Y.  H edge (x,y)-(x+1,y), x in [0,X-2]; V edge (x,y)-(x,y+1), y in [0,Y-2].
  *   Grids are row-major [Y][X]; the last column (H) / last row (V) is padding.
  *   Segment {dir (0 = H, 1 = V), line (y for H, x for V), lo, hi}: the edges [lo,hi) of the line.
- *   Every path candidate must be one of the patterns of its sub-net (x0,y0)-(x1,y1): the
- *   straight path, HV / VH L-shapes, Z-HVH (interior x_m) or Z-VHV (interior y_m) (§3.1,
- *   P:313-315; §4.2); each sub-net has 1..32 candidates.
+ *   A path candidate is any rectilinear path given as its segments and turning points (§3.1,
+ *   L-, Z-, C-shape patterns and monotonic routes); each sub-net has 1..1024.
  */
 #ifndef DGR_H
 #define DGR_H
@@ -52,11 +51,13 @@ const char* dgr_last_error(void);
 
 /* The routing DAG forest F = {T, S, P} of §3.2 as flat CSR arrays, in GLOBAL order.
  * Offsets have length n+1, start at 0 and are non-decreasing; every group is non-empty.
- * Path candidates are the straight / L / Z patterns of §3.1: every path must be one of
- * them for its sub-net (its segments and turning points are checked).  A sub-net whose endpoints
- * share a row or column has straight candidates only; any other sub-net lists exactly one HV
- * (horizontal first) and one VH candidate, in that order, then its Z-HVH candidates, then its
- * Z-VHV candidates (the order forestgen emits); anything else is DGR_EINVAL.
+ * Path candidates (§3.1) are rectilinear paths: every segment a non-empty edge range of
+ * a grid line, every turning point a G-cell on one of the path's segments (else DGR_EINVAL).  A
+ * sub-net whose candidates are its straight path, or HV, VH, Z-HVH..., Z-VHV..., C-shapes in that
+ * order (the order forestgen emits), 32 at most, runs in the tile kernels; any other sub-net
+ * (monotone staircases, other orders, up to 1024 candidates) makes its net run on the general
+ * path (row f4': one warp per net over the explicit segment lists).  Same results
+ * either way; the order of a sub-net's candidates is its tie-break order (induction).
  * Gumbel noise (Q7): a sub-net whose only candidate is a straight path draws none (its
  * softmax is identically 1); every other candidate, in global path order, takes the next noise
  * index n (0, 1, 2, ...) and draws g from Philox4x32-10(key = seed, counter = {n >> 2 (64 bit),
@@ -194,7 +195,7 @@ int dgr_induce(struct dgr_handle* h, float top_p, int32_t* tree_choice, int32_t*
 
 /* Introspection: iteration counter k, this rank's net range, encoded sizes.  info[12] =
  * {k, net_lo, net_hi, n_bundles, n_path_slots, workspace_bytes, world, rank, n_tiles,
- *  n_global_tiles, n_pipelined_tiles, 0}. */
+ *  n_global_tiles, n_pipelined_tiles, n_general_paths} (candidates on the general path). */
 int dgr_get_info(struct dgr_handle* h, int64_t info[12]);
 
 /* Host-only view of the rank's encoding plan (no GPU needed): out[8] = {n_tiles, n_global_tiles,

@@ -21,7 +21,8 @@
  *   Sub-net endpoints are emitted canonically: x0 <= x1 and, if x0 == x1,
  *   y0 < y1.  Path candidate order per sub-net: the straight path if the
  *   sub-net is aligned, else [HV, VH, Z-HVH by x_m ascending, Z-VHV by y_m
- *   ascending, C-HVH by x_m ascending, C-VHV by y_m ascending] (
+ *   ascending, C-HVH by x_m ascending, C-VHV by y_m ascending, staircases HVHVH then VHVHV]
+ *   (
  *   C-shapes, Q14b: x_m in [x0-c_cap, x0-1] then [x1+1, x1+c_cap], y_m in
  *   [ylo-c_cap, ylo-1] then [yhi+1, yhi+c_cap], inside the grid).
  *   Nets are emitted in Morton order of their pin bounding-box centre.
@@ -50,6 +51,8 @@ typedef struct {
   uint64_t seed;
   double  local_weight;    /* weight of the local-net term of Eq. (1) (1 = as written; 0 for Table 1's uniform cap) */
   int32_t c_cap;           /* C-shape detours per side of a non-aligned sub-net (0 = none; reading Q14b) */
+  int32_t m_cap;           /* monotone staircases per orientation (0 = none; row f4, reading Q14c): HVHVH
+                              and VHVHV paths with four turning points, after the C-shapes */
 } forestgen_config;
 
 typedef struct forestgen_forest forestgen_forest;

@@ -88,10 +88,10 @@ int validate_structure(const dgr_forest_desc* d) {
   int64_t big = d->n_subnets;
 #pragma omp parallel for schedule(static) reduction(min : big)
   for (int64_t s = 0; s < d->n_subnets; ++s)
-    if (d->sub_path_off[s + 1] - d->sub_path_off[s] > 32) big = std::min(big, s);
+    if (d->sub_path_off[s + 1] - d->sub_path_off[s] > kGenMaxGroup) big = std::min(big, s);
   if (big < d->n_subnets)
-    return fail(DGR_EINVAL, "sub-net %lld has %lld > 32 candidates", (long long)big,
-                (long long)(d->sub_path_off[big + 1] - d->sub_path_off[big]));
+    return fail(DGR_EINVAL, "sub-net %lld has %lld > %d candidates", (long long)big,
+                (long long)(d->sub_path_off[big + 1] - d->sub_path_off[big]), kGenMaxGroup);
   if ((d->n_segs && !d->seg) || (d->n_tps && !d->tp_xy) || (d->n_subnets && !d->sub_xy) || !d->cap_h ||
       !d->cap_v || (d->n_trees && !d->w_tree0) || (d->n_paths && !d->w_path0))
     return fail(DGR_EINVAL, "NULL array");
@@ -188,6 +188,29 @@ bool classify(const dgr_forest_desc* d, int64_t i, int x0, int y0, int x1, int y
   return false;
 }
 
+// A candidate outside the Z(o, m) patterns (row f4', reading Q14c) runs on the general path from
+// its explicit segments and turning points: each segment must be a non-empty edge range of a grid
+// line, each turning point a grid cell on one of the path's segments.
+bool valid_path(const dgr_forest_desc* d, int64_t i) {
+  const int64_t g0 = d->path_seg_off[i], g1 = d->path_seg_off[i + 1];
+  for (int64_t g = g0; g < g1; ++g) {
+    const int32_t* s = d->seg + 4 * g;
+    const int n = s[0] == 0 ? d->X : d->Y, m = s[0] == 0 ? d->Y : d->X;   // line length, lines
+    if ((s[0] != 0 && s[0] != 1) || s[1] < 0 || s[1] >= m || s[2] < 0 || s[2] >= s[3] || s[3] > n - 1) return false;
+  }
+  for (int64_t t = d->path_tp_off[i]; t < d->path_tp_off[i + 1]; ++t) {
+    const int x = d->tp_xy[2 * t], y = d->tp_xy[2 * t + 1];
+    if (x < 0 || x >= d->X || y < 0 || y >= d->Y) return false;
+    bool on = false;
+    for (int64_t g = g0; g < g1 && !on; ++g) {
+      const int32_t* s = d->seg + 4 * g;
+      on = s[0] == 0 ? (s[1] == y && s[2] <= x && x <= s[3]) : (s[1] == x && s[2] <= y && y <= s[3]);
+    }
+    if (!on) return false;
+  }
+  return true;
+}
+
 // ---------------------------------------------------------------------------------------
 // the rank's encoded shard
 // ---------------------------------------------------------------------------------------
@@ -253,6 +276,14 @@ struct Plan {
   int64_t n_global_tiles = 0;
   int64_t n_pipe_tiles = 0;
   std::vector<std::pair<int, int>> tmap_shapes;   // (ww, wh) of each tensor-map pair (TileDesc::tmap)
+  // general nets (row f4'): their candidates take virtual slots [nb * 32, nb * 32 + n_gpath)
+  int64_t n_gpath = 0;
+  std::vector<int2> gnet;
+  std::vector<int4> gtree;
+  std::vector<GSub> gsub;
+  std::vector<int32_t> gp_seg_off, gp_tp_off;
+  std::vector<short4> gseg;
+  std::vector<short2> gtp;
 };
 
 // (cell, field) pairs of one candidate's demand events in the pipelined tile kernel (field 0 dH,
@@ -337,11 +368,12 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   //    sub-nets; the first failing sub-net, in index order, is reported)
   PodBuf<short4> sxy_csr, sub_ext;
   PodBuf<uint32_t> pw_path;
-  PodBuf<char> single;
+  PodBuf<char> single, gen;   // gen: the sub-net runs on the general path (row f4')
   sxy_csr.alloc(ns);
   sub_ext.alloc(ns);
   pw_path.alloc((size_t)(pl.path_hi - pl.path_lo));
   single.alloc(ns);
+  gen.alloc(ns);
   int64_t bad_sub = ns;   // smallest failing local sub-net
 #pragma omp parallel for schedule(dynamic, 4096) reduction(min : bad_sub)
   for (int64_t ls = 0; ls < ns; ++ls) {
@@ -349,6 +381,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     const int32_t* e = d->sub_xy + 4 * s;
     int x0 = e[0], y0 = e[1], x1 = e[2], y1 = e[3];
     single[ls] = 0;
+    gen[ls] = 0;
     if (x0 > x1 || (x0 == x1 && y0 > y1)) { std::swap(x0, x1); std::swap(y0, y1); }
     if (x0 < 0 || x1 >= X || std::min(y0, y1) < 0 || std::max(y0, y1) >= Y || (x0 == x1 && y0 == y1)) {
       bad_sub = std::min(bad_sub, ls);
@@ -357,7 +390,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     sxy_csr[ls] = make_short4((short)x0, (short)y0, (short)x1, (short)y1);
     const int64_t p0 = d->sub_path_off[s], p1 = d->sub_path_off[s + 1];
     uint32_t shapes[32];
-    bool ok = true;
+    bool ok = p1 - p0 <= 32;
     int ex0 = x0, ex1 = x1, ey0 = std::min(y0, y1), ey1 = std::max(y0, y1);   // extent incl. detours
     for (int64_t i = p0; i < p1 && ok; ++i) {
       uint32_t shape;
@@ -373,7 +406,12 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     }
     sub_ext[ls] = make_short4((short)ex0, (short)ey0, (short)ex1, (short)ey1);
     if (!ok || !canonical_group(shapes, (int)(p1 - p0), x0 == x1 || y0 == y1)) {
-      bad_sub = std::min(bad_sub, ls);
+      // not all Z(o, m) patterns in the tile kernel's order, or more than 32: the general path
+      // (explicit segments), provided every candidate is a well-formed rectilinear path
+      for (int64_t i = p0; i < p1; ++i)
+        if (!valid_path(d, i)) { bad_sub = std::min(bad_sub, ls); break; }
+      gen[ls] = 1;
+      single[ls] = (p1 - p0 == 1) && (d->path_seg_off[p0 + 1] - d->path_seg_off[p0] == 1);
       continue;
     }
     single[ls] = (p1 - p0 == 1) && (shapes[0] == kStraightH || shapes[0] == kStraightV);
@@ -386,17 +424,30 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     if (x0 < 0 || x1 >= X || std::min(y0, y1) < 0 || std::max(y0, y1) >= Y)
       return fail(DGR_EINVAL, "sub-net %lld endpoints outside the grid", (long long)s);
     if (x0 == x1 && y0 == y1) return fail(DGR_EINVAL, "sub-net %lld has zero length", (long long)s);
-    for (int64_t i = d->sub_path_off[s]; i < d->sub_path_off[s + 1]; ++i) {
-      uint32_t shape;
-      int mid;
-      bool outside;
-      if (!classify(d, i, x0, y0, x1, y1, &shape, &mid, &outside))
-        return fail(DGR_EINVAL, "path %lld is not a straight/L/Z pattern of sub-net %lld (or its turning points are wrong)",
+    for (int64_t i = d->sub_path_off[s]; i < d->sub_path_off[s + 1]; ++i)
+      if (!valid_path(d, i))
+        return fail(DGR_EINVAL, "path %lld of sub-net %lld is malformed (a segment outside the grid or empty, or a turning point off the path)",
                     (long long)i, (long long)s);
-    }
-    return fail(DGR_EINVAL, "sub-net %lld: candidates must be straight (aligned sub-net) or HV, VH, Z-HVH..., Z-VHV..., C... in this order",
-                (long long)s);
+    return fail(DGR_EINVAL, "sub-net %lld is malformed", (long long)s);
   }
+  // a net with any general sub-net runs entirely on the general path (its trees' softmax and dq
+  // stay in one warp)
+  PodBuf<char> gen_net;
+  gen_net.alloc(nn);
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t ln = 0; ln < nn; ++ln) {
+    const int64_t n = pl.net_lo + ln;
+    const int64_t s0 = d->tree_sub_off[d->net_tree_off[n]], s1 = d->tree_sub_off[d->net_tree_off[n + 1]];
+    bool g = false;
+    for (int64_t sn = s0; sn < s1 && !g; ++sn) g = gen[sn - pl.sub_lo];
+    gen_net[ln] = g;
+    if (g) for (int64_t sn = s0; sn < s1; ++sn) gen[sn - pl.sub_lo] = 1;
+  }
+  int64_t n_gpath = 0;
+#pragma omp parallel for schedule(static) reduction(+ : n_gpath)
+  for (int64_t ls = 0; ls < ns; ++ls)
+    if (gen[ls]) n_gpath += d->sub_path_off[pl.sub_lo + ls + 1] - d->sub_path_off[pl.sub_lo + ls];
+  pl.n_gpath = n_gpath;
   tm.mark("classify");
   // local noise index of every sub-net's first candidate (-1 for lone straight paths)
   PodBuf<int64_t> nid_sub;
@@ -455,6 +506,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   auto pack_net = [&](int64_t n, Pack& pk) {   // bundle packing of one net's sub-nets
     const int64_t s0 = d->tree_sub_off[d->net_tree_off[n]], s1 = d->tree_sub_off[d->net_tree_off[n + 1]];
     for (int64_t s = s0; s < s1; ++s) {
+      if (gen[s - pl.sub_lo]) continue;   // general path: virtual slots
       if (single[s - pl.sub_lo]) { ++pk.nsing; continue; }
       const int g = (int)(d->sub_path_off[s + 1] - d->sub_path_off[s]);
       if (pk.fill + g > 32) { ++pk.nbg; pk.fill = 0; }
@@ -480,6 +532,12 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     const int64_t na = pl.net_lo + ch * kChunkNets, nb_ = std::min(pl.net_hi, na + kChunkNets);
     Cur cur;
     for (int64_t n = na; n < nb_; ++n) {
+      if (gen_net[n - pl.net_lo]) {   // a general net: a "tile" of its own (global = 2, no bundles)
+        cstarts[ch].push_back(n);
+        cglobs[ch].push_back(2);
+        cur = Cur();
+        continue;
+      }
       int bx0, by0, bx1, by1;
       net_box(n, bx0, by0, bx1, by1);
       const bool big = aligned_area(bx0, by0, bx1, by1) > kWinMax;
@@ -549,7 +607,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   // every element is written by the parallel fill below (padding slots included)
   pl.binfo.alloc(tb0[ntile]);
   pl.pword.alloc(nslot);
-  pl.slot_path.alloc(nslot);
+  pl.slot_path.alloc(nslot + (size_t)pl.n_gpath);   // bundle slots, then the general paths' virtual slots
   pl.sxy.alloc(ns);
   pl.ksub_csr.alloc(ns);
   pl.sub_first_slot.alloc(ns);
@@ -594,6 +652,14 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
         }
       }
       int ks = T.sub0;   // next kernel-order sub-net
+      if (T.global == 2) {   // a general net: kernel order = CSR order; virtual slots assigned below
+        for (int64_t sn = d->tree_sub_off[j0]; sn < d->tree_sub_off[j1]; ++sn, ++ks) {
+          pl.sxy[ks] = sxy_csr[sn - pl.sub_lo];
+          pl.ksub_csr[ks] = (int32_t)(sn - pl.sub_lo);
+        }
+        pl.tiles[t] = T;
+        continue;
+      }
       // trees of nets with >= 2 trees (their candidates carry kMultiTree)
       auto multi_tree = [&](int64_t j) {
         const int64_t n = std::upper_bound(d->net_tree_off + starts[t], d->net_tree_off + starts[t + 1] + 1, j) -
@@ -723,9 +789,48 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     }
   }
   tm.mark("bundles + event check");
+  pl.nb = (int)pl.binfo.size();
+  // general nets (row f4'): out of the tile list into their own arrays, candidates on virtual slots
+  {
+    int64_t vslot = (int64_t)pl.nb * 32, gp = 0;
+    pl.gp_seg_off.assign(1, 0);
+    pl.gp_tp_off.assign(1, 0);
+    for (const TileDesc& T : pl.tiles) {
+      if (T.global != 2) continue;
+      const int64_t n = pl.net_lo + T.net0;
+      const int64_t j0 = d->net_tree_off[n], j1 = d->net_tree_off[n + 1];
+      pl.gnet.push_back(make_int2((int)pl.gtree.size(), (int)(j1 - j0)));
+      int ks = T.sub0;
+      for (int64_t j = j0; j < j1; ++j) {
+        pl.gtree.push_back(make_int4((int)(j - pl.tree_lo), (int)pl.gsub.size(),
+                                     (int)(d->tree_sub_off[j + 1] - d->tree_sub_off[j]), j1 - j0 > 1));
+        for (int64_t sn = d->tree_sub_off[j]; sn < d->tree_sub_off[j + 1]; ++sn, ++ks) {
+          const int64_t ls = sn - pl.sub_lo, p0 = d->sub_path_off[sn], p1 = d->sub_path_off[sn + 1];
+          GSub g{};
+          g.slot = (int32_t)vslot; g.n = (int32_t)(p1 - p0); g.nid = single[ls] ? -1 : (int32_t)nid_sub[ls];
+          g.ksub = ks; g.tree = (int32_t)(j - pl.tree_lo); g.gp = (int32_t)gp;
+          pl.gsub.push_back(g);
+          pl.sub_first_slot[ls] = vslot;
+          for (int64_t i = p0; i < p1; ++i, ++vslot, ++gp) {
+            pl.slot_path[vslot] = (int32_t)(i - pl.path_lo);
+            for (int64_t q = d->path_seg_off[i]; q < d->path_seg_off[i + 1]; ++q) {
+              const int32_t* sg = d->seg + 4 * q;
+              pl.gseg.push_back(make_short4((short)sg[0], (short)sg[1], (short)sg[2], (short)sg[3]));
+            }
+            for (int64_t q = d->path_tp_off[i]; q < d->path_tp_off[i + 1]; ++q)
+              pl.gtp.push_back(make_short2((short)d->tp_xy[2 * q], (short)d->tp_xy[2 * q + 1]));
+            pl.gp_seg_off.push_back((int32_t)pl.gseg.size());
+            pl.gp_tp_off.push_back((int32_t)pl.gtp.size());
+          }
+        }
+      }
+    }
+    pl.tiles.erase(std::remove_if(pl.tiles.begin(), pl.tiles.end(), [](const TileDesc& T) { return T.global == 2; }),
+                   pl.tiles.end());
+  }
+  tm.mark("general nets");
   pl.n_global_tiles = 0;
   for (const auto& T : pl.tiles) pl.n_global_tiles += T.global;
-  pl.nb = (int)pl.binfo.size();
   // pipelined tiles (shared-memory window and stage) first, then the rest
   const bool all_slow = getenv("DGR_ALL_SLOW") != nullptr;   // diagnostics: every tile on the slow path
   auto pipelined = [all_slow](const TileDesc& T) {
@@ -807,7 +912,7 @@ int encode_window_maps(const std::vector<std::pair<int, int>>& shapes, const voi
 // workspace layout
 // ---------------------------------------------------------------------------------------
 struct Layout {
-  size_t tiles, mnets, tmaps, binfo, pword, sxy, slot_path, wp, mv, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
+  size_t tiles, gnet, gtree, gsub, gp_seg_off, gp_tp_off, gseg, gtp, gdq, mnets, tmaps, binfo, pword, sxy, slot_path, wp, mv, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
       partial, lpart, loss, chosen, tree_choice, route, nsize, nucleus_tmp, DHVC, iscal, ipartial, metrics, total;
   size_t xcount;   // int64 elements in the exchange buffer
 };
@@ -816,13 +921,22 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   Layout L{};
   size_t o = 0;
   auto take = [&](size_t bytes) { size_t r = o; o += (bytes + 255) & ~(size_t)255; return r; };
-  const size_t slots = (size_t)pl.nb * 32, ns = pl.sxy.size(), nt = (size_t)(pl.tree_hi - pl.tree_lo),
-               nn = (size_t)(pl.net_hi - pl.net_lo), G = (size_t)X * Y;
+  // slots: the bundles' 32 per bundle, then the general paths' virtual slots (row f4')
+  const size_t bslots = (size_t)pl.nb * 32, slots = bslots + (size_t)pl.n_gpath, ns = pl.sxy.size(),
+               nt = (size_t)(pl.tree_hi - pl.tree_lo), nn = (size_t)(pl.net_hi - pl.net_lo), G = (size_t)X * Y;
   L.tiles = take(sizeof(TileDesc) * pl.tiles.size());
+  L.gnet = take(sizeof(int2) * pl.gnet.size() + 16);
+  L.gtree = take(sizeof(int4) * pl.gtree.size() + 16);
+  L.gsub = take(sizeof(GSub) * pl.gsub.size() + 16);
+  L.gp_seg_off = take(4 * pl.gp_seg_off.size() + 16);
+  L.gp_tp_off = take(4 * pl.gp_tp_off.size() + 16);
+  L.gseg = take(8 * pl.gseg.size() + 16);
+  L.gtp = take(4 * pl.gtp.size() + 16);
+  L.gdq = take(8 * pl.gtree.size() + 16);
   L.mnets = take(4 * pl.mnets.size() + 16);   // +16 B: 16-byte aligned bulk reads may run past the end
   L.tmaps = take(256 * pl.tmap_shapes.size() + 256);   // 128-byte CUtensorMaps, (S_H, S_V) per window shape
   L.binfo = take(sizeof(int4) * pl.nb);
-  L.pword = take(4 * slots);
+  L.pword = take(4 * bslots);
   L.sxy = take(8 * ns + 16);
   L.slot_path = take(4 * slots);
   L.wp = take(4 * slots);
@@ -1075,6 +1189,17 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   P.nid_base = pl.nid_base;
   P.seed = desc->seed;
   P.mnets = (const int32_t*)(ws + L.mnets);
+  P.ngen = (int32_t)pl.gnet.size();
+  P.ngen_blocks = (P.ngen + kGenWarps - 1) / kGenWarps;
+  P.ngsub = (int32_t)pl.gsub.size();
+  P.gnet = (const int2*)(ws + L.gnet);
+  P.gtree = (const int4*)(ws + L.gtree);
+  P.gsub = (const GSub*)(ws + L.gsub);
+  P.gp_seg_off = (const int32_t*)(ws + L.gp_seg_off);
+  P.gp_tp_off = (const int32_t*)(ws + L.gp_tp_off);
+  P.gseg = (const short4*)(ws + L.gseg);
+  P.gtp = (const short2*)(ws + L.gtp);
+  P.gdq = (long long*)(ws + L.gdq);
   P.tmaps = (const unsigned char*)(ws + L.tmaps);
   for (int r = 0; r < 10; ++r) {   // Philox4x32-10 round keys of the seed
     P.rk[2 * r] = (uint32_t)desc->seed + (uint32_t)r * 0x9E3779B9u;
@@ -1124,14 +1249,14 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   tm.mark("bind: prepare kernels");
   if (cudaMemsetAsync(ws, 0, L.total, s) != cudaSuccess) return cleanup(fail(DGR_ECUDA, "memset workspace failed"));
   // host-side staging of the encoded shard, packed into pinned memory, then one copy per region
-  const size_t slots = (size_t)pl.nb * 32;
+  const size_t slots = (size_t)pl.nb * 32 + (size_t)pl.n_gpath;   // bundle slots, then general (virtual) slots
   const size_t nt = (size_t)(pl.tree_hi - pl.tree_lo);
   struct Region { size_t off, bytes; const void* src; };   // src == nullptr: filled in place below
   std::vector<Region> regs = {
       {L.tiles, sizeof(TileDesc) * pl.tiles.size(), pl.tiles.data()},
       {L.mnets, 4 * pl.mnets.size(), pl.mnets.data()},
       {L.binfo, sizeof(int4) * pl.nb, pl.binfo.data()},
-      {L.pword, 4 * slots, pl.pword.data()},
+      {L.pword, 4 * (size_t)pl.nb * 32, pl.pword.data()},
       {L.sxy, 8 * pl.sxy.size(), pl.sxy.data()},
       {L.wp, 4 * slots, nullptr},
       {L.pp, 4 * slots, nullptr},
@@ -1141,7 +1266,14 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
       {L.q, 4 * nt, nullptr},
       {L.capH, 4 * G, desc->cap_h},
       {L.capVT, 4 * G, nullptr},
-      {L.tmaps, 256 * pl.tmap_shapes.size(), nullptr}};
+      {L.tmaps, 256 * pl.tmap_shapes.size(), nullptr},
+      {L.gnet, sizeof(int2) * pl.gnet.size(), pl.gnet.data()},
+      {L.gtree, sizeof(int4) * pl.gtree.size(), pl.gtree.data()},
+      {L.gsub, sizeof(GSub) * pl.gsub.size(), pl.gsub.data()},
+      {L.gp_seg_off, 4 * pl.gp_seg_off.size(), pl.gp_seg_off.data()},
+      {L.gp_tp_off, 4 * pl.gp_tp_off.size(), pl.gp_tp_off.data()},
+      {L.gseg, 8 * pl.gseg.size(), pl.gseg.data()},
+      {L.gtp, 4 * pl.gtp.size(), pl.gtp.data()}};
   std::vector<size_t> at(regs.size() + 1, 0);
   for (size_t i = 0; i < regs.size(); ++i) at[i + 1] = at[i] + ((regs[i].bytes + 255) & ~(size_t)255);
   std::lock_guard<std::mutex> lock(g_pin.m);
@@ -1341,7 +1473,7 @@ int dgr_get_logits(dgr_handle* h, float* w_tree, float* w_path) {
   if (!h->ws) return fail(DGR_ESTATE, "no workspace bound (dgr_bind_workspace)");
   const Plan& pl = h->plan;
   if (w_path) {
-    std::vector<float> slots((size_t)pl.nb * 32);
+    std::vector<float> slots((size_t)pl.nb * 32 + (size_t)pl.n_gpath);
     CUDA_TRY(cudaMemcpyAsync(slots.data(), h->P.wp, 4 * slots.size(), cudaMemcpyDeviceToHost, h->stream));
     CUDA_TRY(cudaStreamSynchronize(h->stream));
     for (size_t sl = 0; sl < slots.size(); ++sl)
@@ -1378,7 +1510,7 @@ int dgr_induce(dgr_handle* h, float top_p, int32_t* tree_choice, int32_t* route,
   launch_induce_metrics(P, h->beta_last, s);
   CUDA_TRY(cudaGetLastError());
   const int64_t nn = pl.net_hi - pl.net_lo, ns = pl.sub_hi - pl.sub_lo;
-  std::vector<int32_t> tc(nn), rt(ns), nsz(ns), nuc((size_t)pl.nb * 32);
+  std::vector<int32_t> tc(nn), rt(ns), nsz(ns), nuc((size_t)pl.nb * 32 + (size_t)pl.n_gpath);
   CUDA_TRY(cudaMemcpyAsync(tc.data(), P.tree_choice, 4 * nn, cudaMemcpyDeviceToHost, s));
   CUDA_TRY(cudaMemcpyAsync(rt.data(), P.route, 4 * ns, cudaMemcpyDeviceToHost, s));
   CUDA_TRY(cudaMemcpyAsync(nsz.data(), P.nsize, 4 * ns, cudaMemcpyDeviceToHost, s));
@@ -1417,7 +1549,8 @@ int dgr_get_info(dgr_handle* h, int64_t info[12]) {
   if (!h || !info) return fail(DGR_EINVAL, "NULL argument");
   info[0] = h->k; info[1] = h->plan.net_lo; info[2] = h->plan.net_hi; info[3] = h->plan.nb;
   info[4] = (int64_t)h->plan.nb * 32; info[5] = (int64_t)h->lay.total; info[6] = h->world; info[7] = h->rank;
-  info[8] = (int64_t)h->plan.tiles.size(); info[9] = h->plan.n_global_tiles; info[10] = h->plan.n_pipe_tiles; info[11] = 0;
+  info[8] = (int64_t)h->plan.tiles.size(); info[9] = h->plan.n_global_tiles; info[10] = h->plan.n_pipe_tiles;
+  info[11] = h->plan.n_gpath;
   return DGR_OK;
 }
 

@@ -66,6 +66,8 @@ constexpr int kPipeSubs = DGR_PIPE_SUBS;           // sub-nets per pipelined til
 #endif
 constexpr int kKgWarps = DGR_KG_WARPS;             // warps per KG CTA (one line per CTA)
 constexpr int kEventMax = 127;                     // events per window cell-field (int32 safety)
+constexpr int kGenMaxGroup = 1024;                 // candidates per sub-net (general path, row f4')
+constexpr int kGenWarps = 8;                       // general nets per CTA (one warp each)
 
 enum Shape : uint32_t {
   kStraightH = 0, kStraightV = 1, kHV = 2, kVH = 3, kZHVH = 4, kZVHV = 5, kPad = 7
@@ -93,6 +95,20 @@ struct TileDesc {
                            // (one 2-D TMA copy per field), -1: the window comes by cp.async
 };
 
+// "General" nets (row f4'): nets with a sub-net whose candidates are not all Z(o, m)
+// patterns (monotone staircases, any rectilinear path), exceed 32 candidates or come in another
+// order.  They run one warp per net against global memory from explicit segment lists; their
+// candidates take "virtual" slots after the bundles' (same w, m, v, p arrays).
+struct GSub {
+  int32_t slot;            // virtual slot of the first candidate
+  int32_t n;               // candidates
+  int32_t nid;             // local noise index of the first candidate, -1: a lone straight path (p = 1)
+  int32_t ksub;            // kernel-order sub-net (induction outputs)
+  int32_t tree;            // local tree
+  int32_t gp;              // general path index of the first candidate (segment / turning-point lists)
+  int32_t pad[2];
+};
+
 // Shared-memory offset (elements) of a pipelined tile's V field: the H field rounded up to 128 bytes
 // of doubles (TMA destinations are 128-byte aligned).
 inline __host__ __device__ int win_hv(int ww, int wh) { return (ww * wh + 15) & ~15; }
@@ -108,6 +124,9 @@ struct KParams {
   int32_t XP, YP;           // even pitches of S_H rows and S_V columns
   int32_t skip;             // DGR_DEBUG_SKIP: timing knock-outs (results invalid), 0 in production
   int32_t pf;               // L2 prefetch at tile start (DGR_PF): bit 1 the trees' Adam moments (default), bit 0 also the slots' m, v, p
+  int32_t ngen;             // general nets (row f4'), run by CTAs [ntiles_slow, ntiles_slow + ngen_blocks)
+  int32_t ngen_blocks;
+  int32_t ngsub;            // their sub-nets
   int64_t path_base, tree_base;   // global index of the first local path / tree
   int64_t nid_base;         // global noise index of the rank's first noisy candidate
   uint64_t seed;
@@ -125,6 +144,16 @@ struct KParams {
   const int32_t* net_tree_off;    // local, n_nets_l + 1
   const int32_t* mnets;     // per tile: offsets (in the tile) of its nets with >= 2 trees
   const unsigned char* tmaps;   // CUtensorMap pairs (S_H window, S_V window), 128 B each, per window shape
+  // general nets (row f4'): per net {first gtree, trees}; per tree {local tree, first gsub, sub-nets,
+  // multi-tree flag}; per sub-net a GSub; per general path its segment / turning-point ranges
+  const int2* gnet;
+  const int4* gtree;
+  const GSub* gsub;
+  const int32_t* gp_seg_off;    // [n_gpath + 1] into gseg
+  const int32_t* gp_tp_off;     // [n_gpath + 1] into gtp
+  const short4* gseg;           // {dir, line, lo, hi}
+  const short2* gtp;            // {x, y}
+  long long* gdq;               // [gtrees] dq_j in 2^-32 fixed point (reverse -> net level)
   float *wt, *mt, *vt, *q;
   // grids (the exchange buffer, in this order: dH | dVT | acc)
   long long* dH;            // [Y][X] 2^-40: wire events << 16, turning points folded in (+-beta pi)

@@ -1075,7 +1075,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     }
     __syncthreads();
   }
-  stamp(P, (int)blockIdx.x - P.ntiles_slow, 2);
+  stamp(P, (int)blockIdx.x - P.ntiles_slow - P.ngen_blocks, 2);
 
   // ---------------- net level (one thread per net), event window cleared alongside ----------------
   if (FWD) {
@@ -1148,7 +1148,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     }
   }
   __syncthreads();
-  stamp(P, (int)blockIdx.x - P.ntiles_slow, 3);
+  stamp(P, (int)blockIdx.x - P.ntiles_slow - P.ngen_blocks, 3);
 
   // ---------------- forward of iteration k_next ----------------
   if (FWD) {
@@ -1212,7 +1212,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     }
   }
   __syncthreads();
-  stamp(P, (int)blockIdx.x - P.ntiles_slow, 4);
+  stamp(P, (int)blockIdx.x - P.ntiles_slow - P.ngen_blocks, 4);
   // write back the tile's group slot state with bulk stores (asynchronous; readers wait on the group)
   if (tid == 0 && nbg > 0) {
     fence_proxy_async();
@@ -1239,6 +1239,198 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         atomicAdd(reinterpret_cast<unsigned long long*>(P.acc), (unsigned long long)a);
         atomicAdd(reinterpret_cast<unsigned long long*>(P.acc + 1), (unsigned long long)b);
       }
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// General nets (row f4', reading Q14c): any rectilinear candidates (monotone staircases ...), groups
+// of up to kGenMaxGroup, any candidate order.  One warp per net, from explicit segment and
+// turning-point lists, against S and the difference arrays in global memory; a group is processed
+// in chunks of 32 lanes.  Same formulas as the tile path: c_i (Eqs. (9)-(12) chain rule, reading
+// Q3), softmax backward with differences to the group's first candidate, Adam, tree level, noise
+// keyed on the global noise / tree index (Q7), +-pi segment events and folded turning points.
+// ------------------------------------------------------------------------------------------
+__device__ __forceinline__ double gen_cost(const KParams& P, const StepArgs& A, int gp) {
+  const int X = P.X, Y = P.Y;
+  double c = 0.0, tp = 0.0;
+  int wl = 0;
+  for (int q = P.gp_seg_off[gp]; q < P.gp_seg_off[gp + 1]; ++q) {
+    const short4 g = P.gseg[q];   // {dir, line, lo, hi}: edges [lo, hi) of the line
+    const double* S = g.x == 0 ? P.SH + (size_t)g.y * P.XP : P.SVT + (size_t)g.y * P.YP;
+    c += S[g.w] - S[g.z];
+    wl += g.w - g.z;
+  }
+  const int t0 = P.gp_tp_off[gp], t1 = P.gp_tp_off[gp + 1];
+  for (int q = t0; q < t1; ++q) {   // the (clipped) edges left / right and below / above the cell
+    const short2 v = P.gtp[q];
+    const double* SH = P.SH + (size_t)v.y * P.XP;
+    const double* SV = P.SVT + (size_t)v.x * P.YP;
+    tp += (SH[v.x + (v.x < X - 1)] - SH[v.x - (v.x > 0)]) + (SV[v.y + (v.y < Y - 1)] - SV[v.y - (v.y > 0)]);
+  }
+  return c + (double)A.beta * tp + (double)A.a_wl * (double)wl + (double)A.a_via * (double)A.sqrt_l * (double)(t1 - t0);
+}
+
+// demand events of general path gp with weight v (2^-24): +-v at each segment's ends, folded turning points
+__device__ __forceinline__ void gen_events(const KParams& P, const StepArgs& A, int gp, int v, long long& etp, long long& bdef) {
+  if (v == 0) return;
+  const long long vs = (long long)v << kGridShift;
+  for (int q = P.gp_seg_off[gp]; q < P.gp_seg_off[gp + 1]; ++q) {
+    const short4 g = P.gseg[q];
+    long long* diff = g.x == 0 ? P.dH + (size_t)g.y * P.X : P.dVT + (size_t)g.y * P.Y;
+    red64(diff + g.z, vs);
+    red64(diff + g.w, -vs);
+  }
+  for (int q = P.gp_tp_off[gp]; q < P.gp_tp_off[gp + 1]; ++q) {
+    const short2 t = P.gtp[q];
+    tp_fold_global(P, A, t.x, t.y, v, etp, bdef);
+  }
+}
+
+__device__ __forceinline__ float warp_sum_f(float v) {
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(kFull, v, off);
+  return v;
+}
+__device__ __forceinline__ float warp_max_f(float v) {
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) v = fmaxf(v, __shfl_xor_sync(kFull, v, off));
+  return v;
+}
+
+template <bool REV, bool FWD>
+__device__ __forceinline__ void gen_net(const KParams& P, const StepArgs& A, int gn, long long& etp, long long& bdef) {
+  const int lane = threadIdx.x & 31;
+  const int2 nd = P.gnet[gn];   // {first gtree, trees}
+  if (REV) {   // reverse of iteration k
+    for (int g = nd.x; g < nd.x + nd.y; ++g) {
+      const int4 gt = P.gtree[g];   // {local tree, first gsub, sub-nets, multi-tree}
+      const float q = P.q[gt.x];
+      long long dq = 0;             // dq_j = sum over the tree's sub-nets of sum_k p_k c_k (2^-32)
+      for (int s = gt.y; s < gt.y + gt.z; ++s) {
+        const GSub G = P.gsub[s];
+        if (G.nid < 0) {            // a lone straight path: p = 1, its c goes to dq
+          if (lane == 0) dq += __double2ll_rn(gen_cost(P, A, G.gp) * kDqScale);
+          continue;
+        }
+        double c0 = 0.0, cl = 0.0;  // the group's first c; this lane's c of the first chunk
+        float sa = 0.f;             // sum_k p_k (c_k - c_0)
+        for (int b = 0; b < G.n; b += 32) {
+          const int i = b + lane;
+          const bool v = i < G.n;
+          const double c = v ? gen_cost(P, A, G.gp + i) : 0.0;
+          if (b == 0) { c0 = __shfl_sync(kFull, c, 0); cl = c; }
+          sa += v ? P.pp[G.slot + i] * (float)(c - c0) : 0.f;
+        }
+        sa = warp_sum_f(sa);
+        for (int b = 0; b < G.n; b += 32) {
+          const int i = b + lane;
+          if (i < G.n) {
+            const double c = b == 0 ? cl : gen_cost(P, A, G.gp + i);
+            const int sl = G.slot + i;
+            const float p = P.pp[sl];
+            const float dw = p * A.inv_t * q * ((float)(c - c0) - sa);   // (p_i/t) q (dd_i - sum_k p_k dd_k)
+            float w = P.wp[sl];
+            float2 mv = P.mv[sl];
+            adam_update(w, mv.x, mv.y, dw, A);
+            P.wp[sl] = w;
+            P.mv[sl] = mv;
+          }
+        }
+        if (lane == 0) dq += __double2ll_rn((c0 + (double)sa) * kDqScale);
+      }
+      if (lane == 0) P.gdq[g] = dq;
+    }
+    __syncwarp();
+  }
+  if (lane == 0) {   // tree level: du_j, Adam on w_tree (k); q_j of k+1 (noise stream 1)
+    const int g0 = nd.x, g1 = nd.x + nd.y;
+    if (REV && nd.y > 1) {
+      double sq = 0.0, sw = 0.0;
+      for (int g = g0; g < g1; ++g) {
+        const double ql = (double)P.q[P.gtree[g].x];
+        sq += ql * ((double)P.gdq[g] * kDqInv);
+        sw += ql;
+      }
+      sq /= sw;
+      for (int g = g0; g < g1; ++g) {
+        const int j = P.gtree[g].x;
+        const double du = (double)P.q[j] * (double)A.inv_t * ((double)P.gdq[g] * kDqInv - sq);
+        float w = P.wt[j], m = P.mt[j], v = P.vt[j];
+        adam_update(w, m, v, (float)du, A);
+        P.wt[j] = w; P.mt[j] = m; P.vt[j] = v;
+      }
+    }
+    if (FWD && nd.y > 1) {   // a lone tree keeps q = 1
+      float zmax = -INFINITY;
+      for (int g = g0; g < g1; ++g) {
+        const int j = P.gtree[g].x;
+        zmax = fmaxf(zmax, (P.wt[j] + gumbel(P.seed, (uint64_t)(P.tree_base + j), (uint32_t)A.k_next, 1u)) * A.inv_t);
+      }
+      float sum = 0.f;
+      for (int g = g0; g < g1; ++g) {
+        const int j = P.gtree[g].x;
+        sum += FEXP((P.wt[j] + gumbel(P.seed, (uint64_t)(P.tree_base + j), (uint32_t)A.k_next, 1u)) * A.inv_t - zmax);
+      }
+      for (int g = g0; g < g1; ++g) {
+        const int j = P.gtree[g].x;
+        P.q[j] = FEXP((P.wt[j] + gumbel(P.seed, (uint64_t)(P.tree_base + j), (uint32_t)A.k_next, 1u)) * A.inv_t - zmax) / sum;
+      }
+    }
+  }
+  __syncwarp();
+  if (FWD) {   // forward of iteration k+1
+    for (int g = nd.x; g < nd.x + nd.y; ++g) {
+      const int4 gt = P.gtree[g];
+      const float q = P.q[gt.x];
+      for (int s = gt.y; s < gt.y + gt.z; ++s) {
+        const GSub G = P.gsub[s];
+        if (G.nid < 0) {            // lone straight path: pi = q
+          if (lane == 0) gen_events(P, A, G.gp, __float2int_rn(q * kFixScale), etp, bdef);
+          continue;
+        }
+        // p_i = softmax over the group of (w_i + g_i) / t: the maximum, then the sum, then p
+        float zl = -INFINITY, zmax = -INFINITY;
+        for (int b = 0; b < G.n; b += 32) {
+          const int i = b + lane;
+          const float z = i < G.n ? (P.wp[G.slot + i] + gumbel(P.seed, (uint64_t)(P.nid_base + G.nid + i), (uint32_t)A.k_next, 0u)) * A.inv_t
+                                  : -INFINITY;
+          if (b == 0) zl = z;
+          zmax = fmaxf(zmax, z);
+        }
+        zmax = warp_max_f(zmax);
+        float sum = 0.f;
+        for (int b = 0; b < G.n; b += 32) {
+          const int i = b + lane;
+          const float z = b == 0 ? zl : (i < G.n ? (P.wp[G.slot + i] + gumbel(P.seed, (uint64_t)(P.nid_base + G.nid + i), (uint32_t)A.k_next, 0u)) * A.inv_t : -INFINITY);
+          sum += i < G.n ? FEXP(z - zmax) : 0.f;
+        }
+        sum = warp_sum_f(sum);
+        for (int b = 0; b < G.n; b += 32) {
+          const int i = b + lane;
+          if (i < G.n) {
+            const float z = b == 0 ? zl : (P.wp[G.slot + i] + gumbel(P.seed, (uint64_t)(P.nid_base + G.nid + i), (uint32_t)A.k_next, 0u)) * A.inv_t;
+            const float p = FDIV(FEXP(z - zmax), sum);
+            P.pp[G.slot + i] = p;
+            gen_events(P, A, G.gp + i, __float2int_rn(q * p * kFixScale), etp, bdef);
+          }
+        }
+      }
+    }
+  }
+}
+
+template <bool REV, bool FWD>
+__device__ __forceinline__ void gen_block(const KParams& P, const StepArgs& A, int gb) {
+  const int warp = threadIdx.x >> 5;
+  long long etp = 0, bdef = 0;
+  for (int gn = gb * kGenWarps + warp; gn < P.ngen; gn += P.ngen_blocks * kGenWarps) gen_net<REV, FWD>(P, A, gn, etp, bdef);
+  if (FWD) {
+    etp = warp_sum_ll(etp);
+    bdef = warp_sum_ll(bdef);
+    if ((threadIdx.x & 31) == 0 && (etp | bdef)) {   // exact integers: any order gives the same sums
+      atomicAdd(reinterpret_cast<unsigned long long*>(P.acc), (unsigned long long)etp);
+      atomicAdd(reinterpret_cast<unsigned long long*>(P.acc + 1), (unsigned long long)bdef);
     }
   }
 }
@@ -1273,10 +1465,15 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
     slow_tile<REV, FWD>(P, A, P.tiles_slow[blockIdx.x], smem);
     return;
   }
+  if ((int)blockIdx.x < P.ntiles_slow + P.ngen_blocks) {   // general nets (row f4'): a warp per net
+    griddep_wait();
+    gen_block<REV, FWD>(P, A, (int)blockIdx.x - P.ntiles_slow);
+    return;
+  }
   int* ev_s = reinterpret_cast<int*>(St.S);
   float* gp = reinterpret_cast<float*>(reinterpret_cast<unsigned char*>(St.S) + kGpOffset);
-  const TileDesc T = P.tiles[blockIdx.x - P.ntiles_slow];
-  const int tix = (int)blockIdx.x - P.ntiles_slow;
+  const int tix = (int)blockIdx.x - P.ntiles_slow - P.ngen_blocks;
+  const TileDesc T = P.tiles[tix];
   stamp(P, tix, 0);
   if ((KO(256)) && threadIdx.x == 0 && tix < kProfTiles) {
     unsigned sm, gt_lo;
@@ -1669,6 +1866,59 @@ __global__ void __launch_bounds__(256) ki_path_kernel(KParams P, float inv_t, fl
   }
 }
 
+// KI2 for the general nets' sub-nets (row f4'): a warp per sub-net of any size; the same rules
+// (rank by (w desc, index asc), noise-free p_hat = softmax(w / t), nucleus = smallest prefix with
+// cumulative p_hat >= top_p, route = its first) over explicit segment lists.
+__global__ void __launch_bounds__(256) ki_gen_kernel(KParams P, float inv_t, float top_p) {
+  const int s = blockIdx.x * 8 + (threadIdx.x >> 5), lane = threadIdx.x & 31;
+  if (s >= P.ngsub) return;
+  const GSub G = P.gsub[s];
+  if (!P.chosen[G.tree]) {
+    if (lane == 0) { P.nsize[G.ksub] = 0; P.route[G.ksub] = -1; }
+    return;
+  }
+  float zmax = -INFINITY;
+  for (int i = lane; i < G.n; i += 32) zmax = fmaxf(zmax, P.wp[G.slot + i] * inv_t);
+  zmax = warp_max_f(zmax);
+  float sum = 0.f;
+  for (int i = lane; i < G.n; i += 32) sum += FEXP(P.wp[G.slot + i] * inv_t - zmax);
+  sum = warp_sum_f(sum);
+  int cnt = 0;
+  for (int b = 0; b < G.n; b += 32) {
+    const int i = b + lane;
+    bool in = false;
+    if (i < G.n) {
+      const float w = P.wp[G.slot + i];
+      int rank = 0;
+      float before = 0.f;   // p_hat of the better-ranked candidates
+      for (int k = 0; k < G.n; ++k) {
+        const float wk = P.wp[G.slot + k];
+        if (wk > w || (wk == w && k < i)) { ++rank; before += FDIV(FEXP(wk * inv_t - zmax), sum); }
+      }
+      in = rank == 0 || before < top_p;
+      const int32_t gid = (int32_t)(P.path_base + P.slot_path[G.slot + i]);
+      if (in) P.nucleus_tmp[G.slot + rank] = gid;
+      if (rank == 0) {
+        P.route[G.ksub] = gid;
+        const int X = P.X;
+        int wl = 0;
+        for (int q = P.gp_seg_off[G.gp + i]; q < P.gp_seg_off[G.gp + i + 1]; ++q) {
+          const short4 g = P.gseg[q];
+          for (int e = g.z; e < g.w; ++e)
+            atomicAdd(g.x == 0 ? &P.DH[(size_t)g.y * X + e] : &P.DV[(size_t)e * X + g.y], 1);
+          wl += g.w - g.z;
+        }
+        const int t0 = P.gp_tp_off[G.gp + i], t1 = P.gp_tp_off[G.gp + i + 1];
+        for (int q = t0; q < t1; ++q) atomicAdd(&P.VC[(size_t)P.gtp[q].y * X + P.gtp[q].x], 1);
+        atomicAdd(reinterpret_cast<unsigned long long*>(P.iscal), (unsigned long long)wl);
+        atomicAdd(reinterpret_cast<unsigned long long*>(P.iscal + 1), (unsigned long long)(t1 - t0));
+      }
+    }
+    cnt += __popc(__ballot_sync(kFull, in));
+  }
+  if (lane == 0) P.nsize[G.ksub] = cnt;
+}
+
 __global__ void __launch_bounds__(256) ki_metrics_kernel(KParams P, float beta) {
   __shared__ double sh[32];
   const int X = P.X, Y = P.Y;
@@ -1754,7 +2004,7 @@ static cudaLaunchConfig_t pdl_config(int grid, int block, size_t smem, cudaStrea
 }
 void launch_tiles(const KParams& p, const StepArgs& a, TileMode mode, cudaStream_t s) {
   // one launch: global tiles in the first CTAs (the longest start earliest), then the pipelined tiles
-  const int grid = p.ntiles + p.ntiles_slow;
+  const int grid = p.ntiles + p.ntiles_slow + p.ngen_blocks;
   if (grid == 0) return;
   cudaLaunchAttribute attr;
   cudaLaunchConfig_t cfg = pdl_config(grid, kBThreads, kBSmemBytes, s, &attr);
@@ -1776,6 +2026,7 @@ int induce_metric_blocks(const KParams& p) {
 void launch_induce(const KParams& p, float t_final, float top_p, float /*beta*/, cudaStream_t s) {
   if (p.n_nets_l > 0) ki_tree_kernel<<<cdiv(p.n_nets_l, 256), 256, 0, s>>>(p);
   if (p.nb > 0) ki_path_kernel<<<cdiv(p.nb, 8), 256, 0, s>>>(p, 1.0f / t_final, top_p);
+  if (p.ngsub > 0) ki_gen_kernel<<<cdiv(p.ngsub, 8), 256, 0, s>>>(p, 1.0f / t_final, top_p);
 }
 void launch_induce_metrics(const KParams& p, float beta, cudaStream_t s) {
   const int nb = induce_metric_blocks(p);

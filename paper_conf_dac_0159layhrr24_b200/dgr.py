@@ -313,7 +313,7 @@ class Solver:
         _check(load_library().dgr_get_info(self._h, _ptr(a, ctypes.c_int64)))
         return dict(k=int(a[0]), net_lo=int(a[1]), net_hi=int(a[2]), n_bundles=int(a[3]), n_slots=int(a[4]),
                     workspace_bytes=int(a[5]), world=int(a[6]), rank=int(a[7]), n_tiles=int(a[8]),
-                    n_global_tiles=int(a[9]), n_pipe_tiles=int(a[10]))
+                    n_global_tiles=int(a[9]), n_pipe_tiles=int(a[10]), n_general_paths=int(a[11]))
 
     STAGES = ("KF", "allreduce", "KG", "KBF", "KB", "KL")   # KL: the loss kernel, once per call
 

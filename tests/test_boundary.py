@@ -85,8 +85,9 @@ def test_dist_needs_nccl_id_or_allreduce_callback(tiny):
 @pytest.mark.parametrize("mutate,msg", [
     (lambda f: f.sub_path_off.__setitem__(3, f.sub_path_off[2]), "empty group"),
     (lambda f: f.net_tree_off.__setitem__(1, 0), "empty group"),
-    (lambda f: f.seg.__setitem__((0, 3), f.seg[0, 2]), "pattern"),
-    (lambda f: f.tp_xy.__setitem__((0, 0), (f.tp_xy[0, 0] + 1) % f.X), "pattern"),
+    (lambda f: f.seg.__setitem__((0, 3), f.seg[0, 2]), "malformed"),                 # empty segment
+    (lambda f: f.tp_xy.__setitem__((0, 0), (f.tp_xy[0, 0] + 1) % f.X), "malformed"),  # turning point off the path
+    (lambda f: f.seg.__setitem__((0, 1), f.Y + 3), "malformed"),                      # segment line outside the grid
     (lambda f: f.sub_xy.__setitem__((0, 2), 99), "outside the grid"),
     (lambda f: f.path_seg_off.__setitem__(2, f.path_seg_off[3] + 1), "monotone"),
 ])
@@ -98,11 +99,39 @@ def test_invalid_forest_rejected(tiny, mutate, msg):
     assert n == 0 and msg in err, err
 
 
-def test_group_of_33_rejected(tiny):
+def _info(f):
+    lib = dgr.load_library()
+    d = binding._DescHolder(f)
+    out = (ctypes.c_int64 * 8)()
+    rc = lib.dgr_plan_info(ctypes.byref(d.desc), None, out)
+    return rc, lib.dgr_last_error().decode()
+
+
+def test_general_nets_accepted():
+    """Row f4' (reading Q14c): groups above 32 (uncapped Z), monotone staircases (4 turning points)
+    and candidates in any order are planned onto the general path, not rejected."""
     f = forestgen.generate("c1e4", z_cap=0)          # uncapped Z: groups above 32 exist
     assert np.diff(f.sub_path_off).max() > 32
     n, err = _ws(f)
-    assert n == 0 and "> 32 candidates" in err
+    assert n > 0 and err == "", err
+    g = forestgen.generate("tiny_m")
+    assert (np.diff(g.path_seg_off) == 5).any()
+    assert _info(g)[0] == 0
+    # a shuffled candidate order (reverse the candidates of every sub-net: CSR arrays rebuilt)
+    h = forestgen.shuffle_candidates(forestgen.generate("tiny"), seed=3)
+    assert _info(h)[0] == 0, _info(h)[1]
+
+
+def test_group_above_limit_rejected():
+    """More than kGenMaxGroup = 1024 candidates in one sub-net is DGR_EINVAL."""
+    for seed in range(1, 200):
+        f = forestgen.generate(dict(X=1200, Y=1200, n_nets=1, pins_mode=0, pins_min=2, pins_max=2, box_mode=0,
+                                    box_min=1190, box_max=1190, track=1.0, n_tree_cand=1, z_cap=0, seed=seed))
+        if f.n_subnets and np.diff(f.sub_path_off).max() > 1024:
+            break
+    assert np.diff(f.sub_path_off).max() > 1024
+    n, err = _ws(f)
+    assert n == 0 and "> 1024 candidates" in err, err
 
 
 def test_gpu_required_without_cuda(tiny):
@@ -149,19 +178,19 @@ def _permute_candidates(f, s, order):
 
 
 def test_candidate_order_contract(tiny):
-    """dgr.h: a non-aligned sub-net lists HV, VH, then Z-HVH, then Z-VHV candidates (the forward's
-    event collapse relies on it); any other order is rejected, never silently mis-summed."""
+    """dgr.h: any order of a sub-net's candidates is accepted.  The canonical order (HV, VH, Z-HVH...,
+    Z-VHV..., C...) runs in the tile kernels, any other on the general path (row f4'); the plan
+    reports the general candidates (dgr_get_info info[11] on a bound handle)."""
     n = np.diff(tiny.sub_path_off)
     s = int(np.nonzero(n >= 4)[0][0])
     ok, err = _ws(_permute_candidates(tiny, s, list(range(n[s]))))
     assert ok > 0 and err == ""
     for order in ([1, 0] + list(range(2, n[s])), [2, 0, 1] + list(range(3, n[s]))):
         ws, err = _ws(_permute_candidates(tiny, s, order))
-        assert ws == 0 and "in this order" in err, err
-    # an L pair alone is fine; a lone L candidate is not
+        assert ws > 0 and err == "", err
     s2 = int(np.nonzero(n == 2)[0][0]) if (n == 2).any() else None
     if s2 is not None:
-        assert _ws(_permute_candidates(tiny, s2, [0, 1]))[0] > 0
+        assert _ws(_permute_candidates(tiny, s2, [1, 0]))[0] > 0
 
 
 @pytest.mark.parametrize("xm", [-3, -1, "X", "X+2"])
@@ -191,4 +220,4 @@ def test_c_shape_detour_outside_grid_rejected(xm):
     else:
         pytest.fail("tiny_c has no C-HVH candidate")
     n, err = _ws(f)
-    assert n == 0 and "pattern" in err, err
+    assert n == 0 and "malformed" in err, err

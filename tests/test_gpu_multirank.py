@@ -85,7 +85,7 @@ def _schedule(s):
     return losses, s.demand(), s.logits(), s.induce(0.9)
 
 
-@pytest.mark.parametrize("name,world", [("c1e4", 2), ("c1e4", 3), ("ispd18", 4), ("ispd19", 8)])
+@pytest.mark.parametrize("name,world", [("c1e4", 2), ("c1e4", 3), ("ispd18", 4), ("ispd19", 8), ("c1e4_m", 3)])
 def test_sharded_ranks_reproduce_one_rank_bit_exactly(name, world):
     f = forestgen.generate(name)
     ref = dgr.Solver(f)

@@ -37,7 +37,10 @@ def ow(w: dgr.Weights):
 
 @pytest.fixture(scope="module")
 def forests():
-    return {n: forestgen.generate(n) for n in ("tiny", "c1e4", "ispd18", "tiny_c", "c1e4_c")}
+    fs = {n: forestgen.generate(n) for n in ("tiny", "c1e4", "ispd18", "tiny_c", "c1e4_c", "tiny_m", "c1e4_m")}
+    # row f4': candidates in a random order per sub-net (the general path, like the staircases)
+    fs["c1e4_shuf"] = forestgen.shuffle_candidates(fs["c1e4"], seed=7)
+    return fs
 
 
 def run_both(f, schedule, W=None, lr=0.3):
@@ -180,7 +183,7 @@ def compare_state(s, o, what, probe=None, max_ill=0.01, exempt=None, chaos=False
 
 
 @pytest.mark.parametrize("beta", [0.0, 0.25])
-@pytest.mark.parametrize("name", ["c1e4", "c1e4_c"])
+@pytest.mark.parametrize("name", ["c1e4", "c1e4_c", "c1e4_m", "c1e4_shuf"])
 def test_one_hot_demand_is_bit_exact(forests, beta, name):
     f = copy.deepcopy(forests[name])
     rng = np.random.default_rng(0)
@@ -204,7 +207,7 @@ def test_one_hot_demand_is_bit_exact(forests, beta, name):
     assert np.array_equal(gdh.astype(np.float64), odh) and np.array_equal(gdv.astype(np.float64), odv)
 
 
-@pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18", "tiny_c", "c1e4_c"])
+@pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18", "tiny_c", "c1e4_c", "tiny_m", "c1e4_m"])
 @pytest.mark.parametrize("f_kind", [0, 1, 2, 3, 4])
 def test_forward_parity(forests, name, f_kind):
     """sigmoid, ReLU and the LeakyReLU / exp / CELU of Fig. 6."""
@@ -219,7 +222,7 @@ def test_forward_parity(forests, name, f_kind):
     assert s.iteration == 0
 
 
-@pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18", "tiny_c", "c1e4_c"])
+@pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18", "tiny_c", "c1e4_c", "tiny_m", "c1e4_m", "c1e4_shuf"])
 def test_one_iteration_parity(forests, name):
     """After one Adam step the update of a coordinate whose gradient is ~eps depends on that
     gradient's last bits (Q21b), so the fp32 probe applies from the first step on."""
@@ -233,6 +236,9 @@ def test_one_iteration_parity(forests, name):
     ("c1e4", [(100, 1.0)]),
     ("tiny_c", [(100, 1.0), (100, 0.9)]),                # row f4: C-shape detours
     ("c1e4_c", [(100, 1.0)]),
+    ("tiny_m", [(100, 1.0), (100, 0.9)]),                # row f4': staircases, groups > 32
+    ("c1e4_m", [(100, 1.0)]),
+    ("c1e4_shuf", [(100, 1.0)]),                         # any candidate order
 ])
 def test_trajectory_parity(forests, name, schedule):
     f = forests[name]
@@ -325,7 +331,7 @@ def test_step_async_equals_step(forests):
     assert np.array_equal(a.logits()[1], b.logits()[1]) and np.array_equal(a.logits()[0], b.logits()[0])
 
 
-@pytest.mark.parametrize("name", ["tiny", "c1e4", "c1e4_c"])
+@pytest.mark.parametrize("name", ["tiny", "c1e4", "c1e4_c", "tiny_m", "c1e4_m", "c1e4_shuf"])
 def test_induce_parity(forests, name):
     f = forests[name]
     s, o, _, _ = run_both(f, [(60, 1.0), (40, 0.9)])
@@ -426,3 +432,20 @@ def test_table1_workload_relu_parity_and_optimum():
         best = m if best is None else min(best, m)
     assert best == opt
     assert W_T1["f_kind"] == 1
+
+
+def test_general_path_is_used(forests):
+    """Row f4': the staircase / large-group / shuffled configs do run candidates on the general path
+    (dgr_get_info info[11] = general candidates) and the plain configs do not."""
+    for name, want in (("c1e4", False), ("c1e4_m", True), ("c1e4_shuf", True), ("tiny_m", True)):
+        s = dgr.Solver(forests[name])
+        assert (s.info()["n_general_paths"] > 0) == want, name
+
+
+def test_ispd18_staircases_one_iteration():
+    """Row f4' at ISPD'18 scale (configs[2] shape with staircases and groups up to 58)."""
+    f = forestgen.generate("ispd18_m")
+    s, o, gl, ol = run_both(f, [(1, 1.0)])
+    for i in range(4):
+        assert_rel(gl[0][i], ol[0][i], what="loss")
+    compare_state(s, o, "ispd18_m", exempt=first_step_exempt(f), max_ill=1e-3)

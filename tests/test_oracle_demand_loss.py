@@ -86,7 +86,12 @@ def _small_subforest(f, max_space=20000):
 
 @pytest.mark.parametrize("which", [0, 1, 2])
 def test_brute_force_expectation(tinyx, which):
-    """E[D_e], E[WL], E[TP] of Eq. (10)-(12) equal the enumeration of every discrete selection."""
+    """E[D_e], E[WL], E[TP] of Eq. (10)-(12) equal the enumeration of every discrete selection.
+    For the staircase recipe (row f4') the enumerable sub-forests come from the same recipe with
+    small boxes and one staircase per orientation (its large groups are not enumerable)."""
+    if tinyx.meta["config"].get("m_cap", 0):
+        tinyx = forestgen.generate(dict(tinyx.meta["config"], box_min=4, box_max=7, z_cap=1, c_cap=0, m_cap=1))
+        assert any(np.diff(tinyx.path_seg_off) == 5)
     los = _small_subforest(tinyx)
     assert len(los) > which
     lo = los[which * (len(los) // 3)]
