@@ -41,6 +41,9 @@ def parse():
     ap.add_argument("--impl", default="dgr", choices=["dgr", "reference"])
     ap.add_argument("--config", default="ispd19")
     ap.add_argument("--no-quality", action="store_true", help="skip the full 1000-iteration solve")
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "torch"],
+                    help="N > 1: the demand exchange over NCCL (default) or through torch.distributed (gloo) via "
+                         "dgr_dist.allreduce (plumbing test: several ranks may share one GPU)")
     ap.add_argument("--e2e-iters", type=int, default=1000,
                     help="iterations of the end-to-end solve (default: the paper's 1000, P:915-917)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -287,10 +290,16 @@ def main():
     rank, world, local = dist_env()
     if world != args.gpus:
         print(f"warning: --gpus {args.gpus} but WORLD_SIZE {world}; using WORLD_SIZE", file=sys.stderr)
+    local = local % max(1, torch.cuda.device_count())   # (--exchange torch: ranks may share a GPU)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     nccl_id = None
-    if world > 1:
+    ar = None
+    gloo = world > 1 and args.exchange == "torch"
+    if gloo:
+        tdist.init_process_group("gloo")
+        ar = dgr.torch_allreduce()
+    elif world > 1:
         tdist.init_process_group("nccl", device_id=dev)
         buf = torch.zeros(128, dtype=torch.uint8, device=dev)
         if rank == 0:
@@ -300,12 +309,15 @@ def main():
 
     def barrier():
         if world > 1:
-            tdist.barrier(device_ids=[local])
+            if gloo:
+                tdist.barrier()
+            else:
+                tdist.barrier(device_ids=[local])
 
     def max_over_ranks(x: float) -> float:
         if world == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        t = torch.tensor([x], dtype=torch.float64, device="cpu" if gloo else dev)
         tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
         return float(t.item())
 
@@ -318,7 +330,7 @@ def main():
     # (e2e_iters iterations, t x 0.9 every 100), each iteration's loss read back to the host, then the
     # demand grids.  Untimed warm-up solve first (one-time costs: CUDA module loading, allocator,
     # host thread pool); the pinned loss buffer is allocated before the timed region.
-    s = dgr.Solver(f, rank=rank, world=world, nccl_id=nccl_id, device=dev, stream=stream)
+    s = dgr.Solver(f, rank=rank, world=world, nccl_id=nccl_id, device=dev, stream=stream, allreduce=ar)
     for _ in range(3):
         s.step(1, 1.0, 0.3, W, want_loss=True)
     s.demand()
@@ -328,7 +340,7 @@ def main():
     losses = torch.empty((n_e2e, 4), dtype=torch.float64).pin_memory().numpy()
     barrier(); torch.cuda.synchronize()
     t0 = time.perf_counter()
-    s = dgr.Solver(f, rank=rank, world=world, nccl_id=nccl_id, device=dev, stream=stream)  # H2D of the forest
+    s = dgr.Solver(f, rank=rank, world=world, nccl_id=nccl_id, device=dev, stream=stream, allreduce=ar)  # H2D of the forest
     t_load = time.perf_counter()
     h2d = s.host_input_bytes()
     d2h = 0
@@ -351,7 +363,7 @@ def main():
     del s
 
     # ---------------- device-timed region: K iterations, inputs resident in HBM ----------------
-    s = dgr.Solver(f, rank=rank, world=world, nccl_id=nccl_id, device=dev, stream=stream)
+    s = dgr.Solver(f, rank=rank, world=world, nccl_id=nccl_id, device=dev, stream=stream, allreduce=ar)
     info = s.info()
     s.step(max(3, args.warmup), 1.0, 0.3, W, want_loss=False)
     ev0 = torch.cuda.Event(enable_timing=True); ev1 = torch.cuda.Event(enable_timing=True)
@@ -411,7 +423,8 @@ def main():
                    "paths": f.n_paths, "segments": f.n_segs, "turning_points": f.n_tps,
                    "step": "one solver iteration (softmax, scatter, loss/gradient map, reverse, Adam) = KG + KBF; induction timed separately",
                    "l2": f"inputs larger than L2: {info['workspace_bytes'] / 1e6:.0f} MB resident state per rank touched every iteration > 126 MB L2",
-                   "parallelism": f"dp{world} (nets sharded, demand allreduce)" if world > 1 else "single GPU"},
+                   "parallelism": (f"dp{world} (nets sharded; demand reduce-scatter, band-local KG, S all-gather"
+                                   f" over {'torch.distributed gloo (plumbing test)' if gloo else 'NCCL'})") if world > 1 else "single GPU"},
         "path_cand_per_s": iters_per_s * f.n_paths,
         "iteration_roofline": {"alg_bytes": alg_iter, "achieved_gbs": alg_iter * iters_per_s / 1e9, "peak": peak,
                                "frac": alg_iter * iters_per_s / 1e9 / peak,
@@ -451,7 +464,7 @@ def main():
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:
-        tdist.barrier(device_ids=[local])
+        barrier()
         tdist.destroy_process_group()
 
 

@@ -325,15 +325,26 @@ def subset(f: Forest, net_lo: int, net_hi: int) -> Forest:
     )
 
 
+def _ranges(off: np.ndarray, sel: np.ndarray) -> np.ndarray:
+    """Concatenation of the index ranges [off[i], off[i+1]) for i in sel (vectorised)."""
+    off = np.asarray(off, np.int64)
+    lo, hi = off[sel], off[np.asarray(sel) + 1]
+    n = hi - lo
+    if n.sum() == 0:
+        return np.zeros(0, np.int64)
+    start = np.repeat(lo - np.concatenate([[0], np.cumsum(n)[:-1]]), n)
+    return start + np.arange(int(n.sum()), dtype=np.int64)
+
+
 def _gather_paths(f: Forest, order: np.ndarray) -> dict:
     """CSR path arrays (segments, turning points, initial logits) with the paths in `order`."""
+    order = np.asarray(order, np.int64)
     nseg = np.diff(f.path_seg_off)[order]
     ntp = np.diff(f.path_tp_off)[order]
-    seg_idx = np.concatenate([np.arange(f.path_seg_off[p], f.path_seg_off[p + 1]) for p in order]) if len(order) else np.zeros(0, np.int64)
-    tp_idx = np.concatenate([np.arange(f.path_tp_off[p], f.path_tp_off[p + 1]) for p in order]) if len(order) else np.zeros(0, np.int64)
     return dict(path_seg_off=np.concatenate([[0], np.cumsum(nseg)]).astype(np.int64),
                 path_tp_off=np.concatenate([[0], np.cumsum(ntp)]).astype(np.int64),
-                seg=f.seg[seg_idx].copy(), tp_xy=f.tp_xy[tp_idx].copy(), w_path0=f.w_path0[order].copy())
+                seg=f.seg[_ranges(f.path_seg_off, order)].copy(), tp_xy=f.tp_xy[_ranges(f.path_tp_off, order)].copy(),
+                w_path0=f.w_path0[order].copy())
 
 
 def shuffle_candidates(f: Forest, seed: int = 0) -> Forest:
@@ -353,9 +364,9 @@ def shuffle_nets(f: Forest, seed: int = 0) -> Forest:
     """The same forest with its nets in a random order (trees, sub-nets and paths follow their net)."""
     rng = np.random.default_rng(seed)
     nets = rng.permutation(f.n_nets)
-    trees = np.concatenate([np.arange(f.net_tree_off[n], f.net_tree_off[n + 1]) for n in nets]).astype(np.int64)
-    subs = np.concatenate([np.arange(f.tree_sub_off[t], f.tree_sub_off[t + 1]) for t in trees]).astype(np.int64)
-    paths = np.concatenate([np.arange(f.sub_path_off[s], f.sub_path_off[s + 1]) for s in subs]).astype(np.int64)
+    trees = _ranges(f.net_tree_off, nets)
+    subs = _ranges(f.tree_sub_off, trees)
+    paths = _ranges(f.sub_path_off, subs)
     g = Forest(X=f.X, Y=f.Y,
                net_tree_off=np.concatenate([[0], np.cumsum(np.diff(f.net_tree_off)[nets])]).astype(np.int64),
                tree_sub_off=np.concatenate([[0], np.cumsum(np.diff(f.tree_sub_off)[trees])]).astype(np.int64),

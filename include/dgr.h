@@ -81,7 +81,9 @@ typedef struct {
 } dgr_forest_desc;
 
 /* Caller-supplied exchange (optional, replaces NCCL): an in-place sum over the ranks of `count`
- * elements at device pointer `buf` (dtype 0 = int64, 1 = int32), ordered after the work already
+ * elements at device pointer `buf` (dtype 0 = int64, 1 = int32, 2 = fp64, 3 = fp32; the library
+ * expresses its reduce-scatter / all-gather steps through it: all-gather zeroes the other ranks'
+ * chunks first, so fp64 / fp32 sums are exact), ordered after the work already
  * enqueued on `cuda_stream` and visible to the work enqueued after the call returns.  Returns 0 on
  * success; any other value makes the calling dgr_* function fail with DGR_ENCCL.  Used to run
  * several ranks in one process (e.g. on one GPU, for testing the sharded path without NCCL). */

@@ -6,7 +6,7 @@ solver iteration runs in the CUDA kernels.  There is no CPU fallback: without th
 extension or a GPU the binding raises.
 """
 from .dgr import (BuiltForest, DgrError, Loss, Solver, Weights, build_forest, lib_path, load_library,  # noqa: F401
-                  nccl_unique_id, partition, plan_info)
+                  nccl_unique_id, partition, plan_info, torch_allreduce)
 
 __all__ = ["Solver", "Weights", "Loss", "DgrError", "partition", "nccl_unique_id", "load_library", "lib_path", "plan_info",
-           "build_forest", "BuiltForest"]
+           "build_forest", "BuiltForest", "torch_allreduce"]

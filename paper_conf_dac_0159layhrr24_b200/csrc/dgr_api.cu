@@ -22,6 +22,7 @@
 #include <memory>
 #include <mutex>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "dgr.h"
@@ -263,11 +264,16 @@ void par_copy(char* dst, const void* src, size_t bytes) {
 struct Plan {
   int64_t net_lo = 0, net_hi = 0, tree_lo = 0, tree_hi = 0, sub_lo = 0, sub_hi = 0, path_lo = 0, path_hi = 0;
   int64_t nid_base = 0;                 // global noise index of the rank's first noisy candidate
+  int rank = 0, world = 1;
   int nb = 0;
   PodBuf<int4> binfo;
   PodBuf<uint32_t> pword;
   PodBuf<short4> sxy;                   // kernel order
-  std::vector<int32_t> net_tree_off;
+  std::vector<int32_t> net_tree_off;   // over the nets in plan order: tree offsets in plan (tile) order
+  std::vector<int64_t> perm;           // plan position -> local CSR net (spatial order, see make_plan 1c)
+  std::vector<int32_t> tperm;          // plan-ordered local tree -> local CSR tree
+  std::vector<int32_t> net_gtree;      // plan position -> local CSR index of the net's first tree
+  std::vector<NoiseRun> runs;          // per tile (TileDesc run0 / nrun)
   std::vector<int32_t> mnets;           // per tile: offsets of its nets with >= 2 trees (TileDesc mn0 / nmn)
   PodBuf<int32_t> ksub_csr;             // kernel-order sub-net -> local CSR sub-net
   PodBuf<int64_t> sub_first_slot;       // local CSR sub-net -> slot of its first candidate
@@ -338,6 +344,8 @@ struct PhaseTimer {   // DGR_PLAN_TIMING=1: host planning phases to stderr (deve
 
 int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   PhaseTimer tm;
+  pl.rank = rank;
+  pl.world = world;
   int rc = validate_structure(d);
   tm.mark("validate");
   if (rc) return rc;
@@ -354,8 +362,6 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   pl.path_hi = d->sub_path_off[pl.sub_hi];
   const int64_t nn = pl.net_hi - pl.net_lo, ns = pl.sub_hi - pl.sub_lo;
   const int X = d->X, Y = d->Y;
-  pl.net_tree_off.resize(nn + 1);
-  for (int64_t n = 0; n <= nn; ++n) pl.net_tree_off[n] = (int32_t)(d->net_tree_off[pl.net_lo + n] - pl.tree_lo);
   // noise indices: the candidates of earlier ranks' nets that draw noise
   {
     int64_t cnt = 0;
@@ -499,6 +505,58 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     nbox[ln] = make_int4(std::max(0, bx0 - 1), std::max(0, by0 - 1), std::min(X - 1, bx1 + 1), std::min(Y - 1, by1 + 1));
   }
   tm.mark("net boxes");
+  // 1c. spatial order of the nets: tiles are runs of consecutive nets, so nets
+  //     are taken in Morton order of their box centres, unless the caller's order is already
+  //     spatially coherent (>= 80% of consecutive nets within 32 cells; forestgen emits Morton
+  //     order) -- then that order.  Only the planning order changes: noise keys and every output
+  //     stay in global (CSR) indices.
+  std::vector<int64_t>& perm = pl.perm;
+  perm.resize(nn);
+  for (int64_t i = 0; i < nn; ++i) perm[i] = i;
+  {
+    int64_t near = 0;
+#pragma omp parallel for schedule(static) reduction(+ : near)
+    for (int64_t ln = 0; ln < nn - 1; ++ln) {
+      const int4 a = nbox[ln], b = nbox[ln + 1];
+      const int dx = std::abs((a.x + a.z) - (b.x + b.z)), dy = std::abs((a.y + a.w) - (b.y + b.w));   // 2 x centre distance
+      near += std::max(dx, dy) <= 64;
+    }
+    const bool coherent = nn < 2 || near * 10 >= (nn - 1) * 8;
+    if (!coherent || getenv("DGR_PLAN_SORT")) {
+      auto spread = [](uint32_t v) {   // bit i -> bit 2i (16 bits)
+        v &= 0xFFFF;
+        v = (v | (v << 8)) & 0x00FF00FF; v = (v | (v << 4)) & 0x0F0F0F0F;
+        v = (v | (v << 2)) & 0x33333333; v = (v | (v << 1)) & 0x55555555;
+        return v;
+      };
+      std::vector<std::pair<uint32_t, int64_t>> key(nn);
+#pragma omp parallel for schedule(static)
+      for (int64_t ln = 0; ln < nn; ++ln) {
+        const int4 b = nbox[ln];
+        key[ln] = {spread((uint32_t)((b.x + b.z) >> 1)) | (spread((uint32_t)((b.y + b.w) >> 1)) << 1), ln};
+      }
+      std::sort(key.begin(), key.end());
+      for (int64_t i = 0; i < nn; ++i) perm[i] = key[i].second;
+    }
+  }
+  // trees and sub-nets renumbered in plan order (a tile's trees / sub-nets stay contiguous)
+  std::vector<int32_t> ptree_off(nn + 1, 0), psub_off(nn + 1, 0);
+  for (int64_t pn = 0; pn < nn; ++pn) {
+    const int64_t n = pl.net_lo + perm[pn];
+    ptree_off[pn + 1] = ptree_off[pn] + (int32_t)(d->net_tree_off[n + 1] - d->net_tree_off[n]);
+    psub_off[pn + 1] = psub_off[pn] + (int32_t)(d->tree_sub_off[d->net_tree_off[n + 1]] - d->tree_sub_off[d->net_tree_off[n]]);
+  }
+  pl.net_tree_off = ptree_off;
+  pl.tperm.resize((size_t)(pl.tree_hi - pl.tree_lo));
+  pl.net_gtree.resize(nn);
+#pragma omp parallel for schedule(static)
+  for (int64_t pn = 0; pn < nn; ++pn) {
+    const int64_t n = pl.net_lo + perm[pn];
+    pl.net_gtree[pn] = (int32_t)(d->net_tree_off[n] - pl.tree_lo);
+    for (int64_t j = d->net_tree_off[n]; j < d->net_tree_off[n + 1]; ++j)
+      pl.tperm[ptree_off[pn] + (j - d->net_tree_off[n])] = (int32_t)(j - pl.tree_lo);
+  }
+  tm.mark("spatial order");
   auto net_box = [&](int64_t n, int& bx0, int& by0, int& bx1, int& by1) {
     const int4 b = nbox[n - pl.net_lo];
     bx0 = b.x; by0 = b.y; bx1 = b.z; by1 = b.w;
@@ -529,11 +587,12 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   std::vector<int64_t> cbad(nchunk, -1);
 #pragma omp parallel for schedule(dynamic, 1)
   for (int64_t ch = 0; ch < nchunk; ++ch) {
-    const int64_t na = pl.net_lo + ch * kChunkNets, nb_ = std::min(pl.net_hi, na + kChunkNets);
+    const int64_t pa = ch * kChunkNets, pb = std::min(nn, pa + kChunkNets);
     Cur cur;
-    for (int64_t n = na; n < nb_; ++n) {
+    for (int64_t pn = pa; pn < pb; ++pn) {
+      const int64_t n = pl.net_lo + perm[pn];
       if (gen_net[n - pl.net_lo]) {   // a general net: a "tile" of its own (global = 2, no bundles)
-        cstarts[ch].push_back(n);
+        cstarts[ch].push_back(pn);
         cglobs[ch].push_back(2);
         cur = Cur();
         continue;
@@ -561,10 +620,10 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
         continue;
       }
       // close the open tile, open a new one at net n
-      cstarts[ch].push_back(n);
+      cstarts[ch].push_back(pn);
       cglobs[ch].push_back(big);
       cur = Cur();
-      cur.open = true; cur.global = big; cur.net0 = n; cur.ntree = ntree; cur.nsub = nsub;
+      cur.open = true; cur.global = big; cur.net0 = pn; cur.ntree = ntree; cur.nsub = nsub;
       cur.bx0 = bx0; cur.by0 = by0; cur.bx1 = bx1; cur.by1 = by1;
       pack_net(n, cur.pk);
       if ((cur.pk.total() > kMaxBundles || ntree > kTreeMax) && cbad[ch] < 0) cbad[ch] = n;
@@ -584,7 +643,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     starts.insert(starts.end(), cstarts[ch].begin(), cstarts[ch].end());
     globs.insert(globs.end(), cglobs[ch].begin(), cglobs[ch].end());
   }
-  starts.push_back(pl.net_hi);
+  starts.push_back(nn);   // plan positions
   tm.mark("tiles (greedy)");
   // 3. bundles, tile by tile: the tile's group bundles (packing restarts at each tile), then its
   //    singleton bundles; sub-nets renumbered in that order ("kernel order").  Count per tile,
@@ -594,7 +653,8 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
 #pragma omp parallel for schedule(dynamic, 64)
   for (int64_t t = 0; t < ntile; ++t) {
     Pack pk;
-    for (int64_t n = starts[t]; n < starts[t + 1]; ++n) {
+    for (int64_t pn = starts[t]; pn < starts[t + 1]; ++pn) {
+      const int64_t n = pl.net_lo + perm[pn];
       pack_net(n, pk);
       tmn[t + 1] += d->net_tree_off[n + 1] - d->net_tree_off[n] > 1;
     }
@@ -612,6 +672,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   pl.ksub_csr.alloc(ns);
   pl.sub_first_slot.alloc(ns);
   pl.tiles.assign(ntile, TileDesc{});
+  std::vector<std::vector<NoiseRun>> tile_runs(ntile);
   tm.mark("bundle counts + alloc");
 #pragma omp parallel
   {
@@ -620,30 +681,39 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
 #pragma omp for schedule(dynamic, 16)
     for (int64_t t = 0; t < ntile; ++t) {
       TileDesc T{};
-      T.net0 = (int32_t)(starts[t] - pl.net_lo);
+      T.net0 = (int32_t)starts[t];
       T.nnet = (int32_t)(starts[t + 1] - starts[t]);
-      T.tree0 = (int32_t)(d->net_tree_off[starts[t]] - pl.tree_lo);
-      T.ntree = (int32_t)(d->net_tree_off[starts[t + 1]] - d->net_tree_off[starts[t]]);
+      T.tree0 = ptree_off[starts[t]];
+      T.ntree = ptree_off[starts[t + 1]] - T.tree0;
+      // the tile's trees in plan order: CSR tree, plan-ordered local tree, net has >= 2 trees
+      struct TT { int64_t j; int32_t pt; bool multi; };
+      std::vector<TT> tts;
+      for (int64_t pn = starts[t]; pn < starts[t + 1]; ++pn) {
+        const int64_t n = pl.net_lo + perm[pn];
+        const int64_t a = d->net_tree_off[n], b = d->net_tree_off[n + 1];
+        for (int64_t j = a; j < b; ++j) tts.push_back({j, (int32_t)(ptree_off[pn] + (j - a)), b - a > 1});
+      }
       T.b0 = tb0[t];
       T.nb = tb0[t + 1] - tb0[t];
       T.mn0 = tmn[t];
       T.nmn = tmn[t + 1] - tmn[t];
-      for (int64_t n = starts[t], k = T.mn0; n < starts[t + 1]; ++n)
-        if (d->net_tree_off[n + 1] - d->net_tree_off[n] > 1) pl.mnets[k++] = (int32_t)(n - starts[t]);
+      for (int64_t pn = starts[t], k = T.mn0; pn < starts[t + 1]; ++pn) {
+        const int64_t n = pl.net_lo + perm[pn];
+        if (d->net_tree_off[n + 1] - d->net_tree_off[n] > 1) pl.mnets[k++] = (int32_t)(pn - starts[t]);
+      }
       T.nbg = tbg[t];
       T.global = globs[t];
       int bx0 = X, by0 = Y, bx1 = -1, by1 = -1;
-      for (int64_t n = starts[t]; n < starts[t + 1]; ++n) {
+      for (int64_t pn = starts[t]; pn < starts[t + 1]; ++pn) {
         int a0, b0_, a1, b1_;
-        net_box(n, a0, b0_, a1, b1_);
+        net_box(pl.net_lo + perm[pn], a0, b0_, a1, b1_);
         bx0 = std::min(bx0, a0); by0 = std::min(by0, b0_); bx1 = std::max(bx1, a1); by1 = std::max(by1, b1_);
       }
       T.wx0 = bx0 & ~1; T.wy0 = by0 & ~1;
       T.ww = (bx1 + 1 - T.wx0 + 1) & ~1; T.wh = (by1 + 1 - T.wy0 + 1) & ~1;
       if (T.global) { T.wx0 = 0; T.wy0 = 0; T.ww = 0; T.wh = 0; }
-      T.sub0 = (int32_t)(d->tree_sub_off[d->net_tree_off[starts[t]]] - pl.sub_lo);
-      T.nsub = (int32_t)(d->tree_sub_off[d->net_tree_off[starts[t + 1]]] - pl.sub_lo) - T.sub0;
-      const int64_t j0 = d->net_tree_off[starts[t]], j1 = d->net_tree_off[starts[t + 1]];
+      T.sub0 = psub_off[starts[t]];
+      T.nsub = psub_off[starts[t + 1]] - T.sub0;
       for (int b = T.b0; b < T.b0 + T.nb; ++b) {
         pl.binfo[b] = make_int4(0, 0, 0, 0);
         for (int l = 0; l < 32; ++l) {
@@ -653,24 +723,22 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       }
       int ks = T.sub0;   // next kernel-order sub-net
       if (T.global == 2) {   // a general net: kernel order = CSR order; virtual slots assigned below
-        for (int64_t sn = d->tree_sub_off[j0]; sn < d->tree_sub_off[j1]; ++sn, ++ks) {
-          pl.sxy[ks] = sxy_csr[sn - pl.sub_lo];
-          pl.ksub_csr[ks] = (int32_t)(sn - pl.sub_lo);
-        }
+        for (const TT& tt : tts)
+          for (int64_t sn = d->tree_sub_off[tt.j]; sn < d->tree_sub_off[tt.j + 1]; ++sn, ++ks) {
+            pl.sxy[ks] = sxy_csr[sn - pl.sub_lo];
+            pl.ksub_csr[ks] = (int32_t)(sn - pl.sub_lo);
+          }
         pl.tiles[t] = T;
         continue;
       }
-      // trees of nets with >= 2 trees (their candidates carry kMultiTree)
-      auto multi_tree = [&](int64_t j) {
-        const int64_t n = std::upper_bound(d->net_tree_off + starts[t], d->net_tree_off + starts[t + 1] + 1, j) -
-                          d->net_tree_off - 1;
-        return d->net_tree_off[n + 1] - d->net_tree_off[n] > 1;
-      };
-      // group bundles
-      int fill = 32, b = T.b0 - 1, prev_tree = -1;
-      for (int64_t j = j0; j < j1; ++j) {
-        const int toff = (int)(j - pl.tree_lo) - T.tree0;
-        const uint32_t mt = multi_tree(j) ? kMultiTree : 0u;
+      // group bundles; binfo.x = the tile noise offset of lane 0 (noisy candidates before it), and
+      // the tile's noisy candidates in this order form runs of consecutive noise indices
+      int fill = 32, b = T.b0 - 1, prev_tree = -1, noff = 0;
+      std::vector<NoiseRun> truns;
+      for (const TT& tt : tts) {
+        const int64_t j = tt.j;
+        const int toff = tt.pt - T.tree0;
+        const uint32_t mt = tt.multi ? kMultiTree : 0u;
         for (int64_t sn = d->tree_sub_off[j]; sn < d->tree_sub_off[j + 1]; ++sn) {
           const int64_t ls = sn - pl.sub_lo;
           if (single[ls]) continue;
@@ -678,10 +746,13 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
           const int g = (int)(p1 - p0);
           if (fill + g > 32) {
             ++b;
-            pl.binfo[b] = make_int4((int)nid_sub[ls], ks, T.tree0, 0);
+            pl.binfo[b] = make_int4(noff, ks, T.tree0, 0);
             fill = 0;
             prev_tree = -1;
           }
+          if (!truns.empty() && truns.back().nid + truns.back().len == (int32_t)nid_sub[ls]) truns.back().len += g;
+          else truns.push_back({noff, g, (int32_t)nid_sub[ls], 0});
+          noff += g;
           pl.sxy[ks] = sxy_csr[ls];
           pl.ksub_csr[ks] = (int32_t)ls;
           pl.sub_first_slot[ls] = (int64_t)b * 32 + fill;
@@ -707,11 +778,12 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       int lane = 32;
       b = T.b0 + T.nbg - 1;
       for (int pass = 0; pass < 2; ++pass)
-      for (int64_t j = j0; j < j1; ++j) {
-        const bool mj = multi_tree(j);
+      for (const TT& tt : tts) {
+        const int64_t j = tt.j;
+        const bool mj = tt.multi;
         if (mj != (pass == 0)) continue;
         const uint32_t mt = mj ? kMultiTree : 0u;
-        const int toff = (int)(j - pl.tree_lo) - T.tree0;
+        const int toff = tt.pt - T.tree0;
         for (int64_t sn = d->tree_sub_off[j]; sn < d->tree_sub_off[j + 1]; ++sn) {
           const int64_t ls = sn - pl.sub_lo;
           if (!single[ls]) continue;
@@ -745,7 +817,8 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       if (!T.global) {
         const int W1 = T.ww + 1;
         cov.assign((size_t)W1 * (T.wh + 1), 0);
-        for (int64_t sn = d->tree_sub_off[j0]; sn < d->tree_sub_off[j1]; ++sn) {
+        for (const TT& tt : tts)
+        for (int64_t sn = d->tree_sub_off[tt.j]; sn < d->tree_sub_off[tt.j + 1]; ++sn) {
           const short4 b = sub_ext[sn - pl.sub_lo];
           const int bx0 = b.x - T.wx0, by0 = b.y - T.wy0, bx1 = b.z - T.wx0 + 1, by1 = b.w - T.wy0 + 1;
           cov[(size_t)by0 * W1 + bx0] += 1; cov[(size_t)by0 * W1 + bx1] -= 1;
@@ -765,9 +838,11 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
         cnt.assign((size_t)3 * T.ww * T.wh, 0);
         stamp.assign((size_t)3 * T.ww * T.wh, -1);   // last sub-net counted at a cell-field
         bool ok = true;
-        for (int64_t sn = d->tree_sub_off[j0]; sn < d->tree_sub_off[j1] && ok; ++sn) {
+        int id = -1;
+        for (const TT& tt : tts)
+        for (int64_t sn = d->tree_sub_off[tt.j]; sn < d->tree_sub_off[tt.j + 1] && ok; ++sn) {
           const short4 e = sxy_csr[sn - pl.sub_lo];
-          const int id = (int)(sn - d->tree_sub_off[j0]);
+          ++id;
           for (int64_t i = d->sub_path_off[sn]; i < d->sub_path_off[sn + 1] && ok; ++i) {
             const uint32_t pw = pw_path[i - pl.path_lo];
             int ex[8], ey[8], ef[8];
@@ -785,8 +860,27 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
         }
         if (!ok) { T.global = 1; T.wx0 = T.wy0 = T.ww = T.wh = 0; }
       }
+      tile_runs[t] = std::move(truns);
       pl.tiles[t] = T;
     }
+  }
+  // the tiles' noise runs, with the Philox quads (4 consecutive global noise indices) each spans
+  pl.runs.clear();
+  for (int64_t t = 0; t < ntile; ++t) {
+    TileDesc& T = pl.tiles[t];
+    T.run0 = (int32_t)pl.runs.size();
+    T.nrun = (int32_t)tile_runs[t].size();
+    int32_t q = 0;
+    for (NoiseRun r : tile_runs[t]) {
+      r.quad0 = q;
+      const int64_t g0 = pl.nid_base + r.nid;
+      q += (int32_t)(((g0 + r.len - 1) >> 2) - (g0 >> 2) + 1);
+      pl.runs.push_back(r);
+    }
+    T.nquad = q;
+    T.nid0 = T.nrun > 0 ? tile_runs[t][0].nid : 0;
+    T.nnoisy = 0;
+    for (const NoiseRun& r : tile_runs[t]) T.nnoisy += r.len;
   }
   tm.mark("bundles + event check");
   pl.nb = (int)pl.binfo.size();
@@ -797,18 +891,19 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     pl.gp_tp_off.assign(1, 0);
     for (const TileDesc& T : pl.tiles) {
       if (T.global != 2) continue;
-      const int64_t n = pl.net_lo + T.net0;
+      const int64_t n = pl.net_lo + perm[T.net0];
       const int64_t j0 = d->net_tree_off[n], j1 = d->net_tree_off[n + 1];
       pl.gnet.push_back(make_int2((int)pl.gtree.size(), (int)(j1 - j0)));
       int ks = T.sub0;
       for (int64_t j = j0; j < j1; ++j) {
-        pl.gtree.push_back(make_int4((int)(j - pl.tree_lo), (int)pl.gsub.size(),
-                                     (int)(d->tree_sub_off[j + 1] - d->tree_sub_off[j]), j1 - j0 > 1));
+        // {plan-ordered local tree, first gsub, sub-nets, local CSR tree (the tree's noise key)}
+        pl.gtree.push_back(make_int4(T.tree0 + (int)(j - j0), (int)pl.gsub.size(),
+                                     (int)(d->tree_sub_off[j + 1] - d->tree_sub_off[j]), (int)(j - pl.tree_lo)));
         for (int64_t sn = d->tree_sub_off[j]; sn < d->tree_sub_off[j + 1]; ++sn, ++ks) {
           const int64_t ls = sn - pl.sub_lo, p0 = d->sub_path_off[sn], p1 = d->sub_path_off[sn + 1];
           GSub g{};
           g.slot = (int32_t)vslot; g.n = (int32_t)(p1 - p0); g.nid = single[ls] ? -1 : (int32_t)nid_sub[ls];
-          g.ksub = ks; g.tree = (int32_t)(j - pl.tree_lo); g.gp = (int32_t)gp;
+          g.ksub = ks; g.tree = T.tree0 + (int32_t)(j - j0); g.gp = (int32_t)gp;
           pl.gsub.push_back(g);
           pl.sub_first_slot[ls] = vslot;
           for (int64_t i = p0; i < p1; ++i, ++vslot, ++gp) {
@@ -912,9 +1007,14 @@ int encode_window_maps(const std::vector<std::pair<int, int>>& shapes, const voi
 // workspace layout
 // ---------------------------------------------------------------------------------------
 struct Layout {
-  size_t tiles, gnet, gtree, gsub, gp_seg_off, gp_tp_off, gseg, gtp, gdq, mnets, tmaps, binfo, pword, sxy, slot_path, wp, mv, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
+  size_t tiles, net_gtree, runs, gnet, gtree, gsub, gp_seg_off, gp_tp_off, gseg, gtp, gdq, mnets, tmaps, binfo, pword, sxy, slot_path, wp, mv, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
       partial, lpart, loss, chosen, tree_choice, route, nsize, nucleus_tmp, DHVC, iscal, ipartial, metrics, total;
   size_t xcount;   // int64 elements in the exchange buffer
+  // grid bands (SURVEY §8(e) refinement 2): rank r reduces and scans H rows [r yb, (r+1) yb) and V
+  // columns [r xb, (r+1) xb); the row-major H arrays have world * yb rows, the V arrays world * xb
+  // columns (padding beyond Y / X), so every rank's band is one contiguous chunk
+  int yb = 0, xb = 0;
+  size_t gh = 0, gv = 0;   // cells of the H arrays ([world yb][X]) and of the V arrays ([world xb][Y])
 };
 
 Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
@@ -943,21 +1043,27 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.mv = take(8 * slots);
   L.pp = take(4 * slots);   // p of the last forward (read by the next reverse)
   L.nto = take(4 * (nn + 1) + 16);   // +16 B: 16-byte aligned bulk reads may run past the end
+  L.net_gtree = take(4 * nn + 16);
+  L.runs = take(sizeof(NoiseRun) * pl.runs.size() + 16);
   L.wt = take(4 * nt + 16);
   L.mt = take(4 * nt + 16);
   L.vt = take(4 * nt + 16);
   L.q = take(4 * nt + 16);
-  L.xcount = 2 * G + 2;   // dH | dV^T | E[WL], E[TP]
+  L.yb = (Y + pl.world - 1) / pl.world;
+  L.xb = (X + pl.world - 1) / pl.world;
+  L.gh = (size_t)pl.world * L.yb * X;
+  L.gv = (size_t)pl.world * L.xb * Y;
+  L.xcount = L.gh + L.gv + 2;   // dH | dV^T | E[TP], B
   L.xbuf = take(8 * L.xcount);
   L.capH = take(4 * G);
   L.capVT = take(4 * G);
   // S_H [Y][XP] then S_V^T [X][YP] (even pitches, contiguous: one base pointer in the kernels),
   // plus padding for window rows / columns that run one cell past the grid
   const size_t XP = (size_t)(X + (X & 1)), YP = (size_t)(Y + (Y & 1));
-  L.SH = take(8 * (Y * XP + X * YP) + 256);
-  L.SVT = L.SH + 8 * Y * XP;
-  L.dOutH = take(4 * G);
-  L.dOutVT = take(4 * G);
+  L.SH = take(8 * ((size_t)pl.world * L.yb * XP + (size_t)pl.world * L.xb * YP) + 256);
+  L.SVT = L.SH + 8 * (size_t)pl.world * L.yb * XP;
+  L.dOutH = take(4 * L.gh);
+  L.dOutVT = take(4 * L.gv);
   L.partial = take(8 * (size_t)(X + Y));
   L.lpart = take(8 * (size_t)(X + Y) + 16);   // per-line demand sums, then lsum[2]
   L.loss = take(8 * 4);
@@ -1069,14 +1175,73 @@ int dgr_partition(const dgr_forest_desc* desc, int32_t world, int64_t* out) {
   return DGR_OK;
 }
 
-// in-place sum over the ranks on the handle's stream: NCCL, or the caller's exchange
+// Collectives on the handle's stream, NCCL or the caller's exchange (dgr_dist.allreduce; reduce-scatter
+// and all-gather are then expressed through it).  dtype: 0 int64, 1 int32, 2 fp64, 3 fp32.
+enum { kI64 = 0, kI32 = 1, kF64 = 2, kF32 = 3 };
+static ncclDataType_t nccl_type(int dt) {
+  return dt == kI64 ? ncclInt64 : dt == kI32 ? ncclInt32 : dt == kF64 ? ncclFloat64 : ncclFloat32;
+}
+static size_t dt_bytes(int dt) { return (dt == kI32 || dt == kF32) ? 4 : 8; }
+static int live_comm(dgr_handle* h) {
+  if (h->world > 1 && !h->ar_fn && !h->comm) return fail(DGR_ESTATE, "the NCCL communicator was aborted after an error or timeout");
+  return DGR_OK;
+}
+// in-place sum over the ranks
 static int allreduce(dgr_handle* h, void* buf, int64_t count, int dtype) {
   if (h->ar_fn) {
     const int r = h->ar_fn(h->ar_user, buf, count, dtype, (void*)h->stream);
     return r ? fail(DGR_ENCCL, "allreduce callback returned %d", r) : DGR_OK;
   }
-  NCCL_TRY(ncclAllReduce(buf, buf, (size_t)count, dtype ? ncclInt32 : ncclInt64, ncclSum, h->comm, h->stream));
+  NCCL_TRY(ncclAllReduce(buf, buf, (size_t)count, nccl_type(dtype), ncclSum, h->comm, h->stream));
   return DGR_OK;
+}
+// in place over world chunks of `chunk` elements: this rank's chunk gets the sum of every rank's
+// copy of it (the other chunks are left undefined)
+static int reduce_scatter(dgr_handle* h, void* buf, int64_t chunk, int dtype) {
+  if (h->ar_fn) return allreduce(h, buf, chunk * h->world, dtype);
+  NCCL_TRY(ncclReduceScatter(buf, (char*)buf + (size_t)h->rank * chunk * dt_bytes(dtype), (size_t)chunk, nccl_type(dtype),
+                             ncclSum, h->comm, h->stream));
+  return DGR_OK;
+}
+// in place over world chunks: every rank's own chunk copied into every rank's buffer
+static int all_gather(dgr_handle* h, void* buf, int64_t chunk, int dtype) {
+  const size_t cb = (size_t)chunk * dt_bytes(dtype);
+  if (h->ar_fn) {   // the other chunks zeroed, then summed: x + 0 + ... + 0 = x exactly
+    char* b = (char*)buf;
+    if (h->rank > 0) CUDA_TRY(cudaMemsetAsync(b, 0, cb * h->rank, h->stream));
+    if (h->rank + 1 < h->world) CUDA_TRY(cudaMemsetAsync(b + cb * (h->rank + 1), 0, cb * (h->world - h->rank - 1), h->stream));
+    return allreduce(h, buf, chunk * h->world, dtype);
+  }
+  NCCL_TRY(ncclAllGather((char*)buf + (size_t)h->rank * cb, buf, (size_t)chunk, nccl_type(dtype), h->comm, h->stream));
+  return DGR_OK;
+}
+static int group_start(dgr_handle* h) { if (!h->ar_fn) NCCL_TRY(ncclGroupStart()); return DGR_OK; }
+static int group_end(dgr_handle* h) { if (!h->ar_fn) NCCL_TRY(ncclGroupEnd()); return DGR_OK; }
+
+// Waits for the handle's stream.  With an NCCL communicator: polls, and aborts the communicator
+// (ncclCommAbort) on an asynchronous NCCL error or after DGR_NCCL_TIMEOUT_MS (default 300000 ms)
+// without completion, so a rank whose peer died returns DGR_ENCCL instead of hanging.
+static int wait_stream(dgr_handle* h) {
+  if (!h->comm) { CUDA_TRY(cudaStreamSynchronize(h->stream)); return DGR_OK; }
+  const char* to = getenv("DGR_NCCL_TIMEOUT_MS");
+  const double limit_ms = to ? atof(to) : 300000.0;
+  const auto t0 = std::chrono::steady_clock::now();
+  for (;;) {
+    const cudaError_t e = cudaStreamQuery(h->stream);
+    if (e == cudaSuccess) return DGR_OK;
+    if (e != cudaErrorNotReady) return fail(DGR_ECUDA, "stream: %s", cudaGetErrorString(e));
+    ncclResult_t ar = ncclSuccess;
+    ncclCommGetAsyncError(h->comm, &ar);
+    const double ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    if ((ar != ncclSuccess && ar != ncclInProgress) || ms > limit_ms) {
+      ncclCommAbort(h->comm);
+      h->comm = nullptr;
+      if (ar != ncclSuccess && ar != ncclInProgress)
+        return fail(DGR_ENCCL, "NCCL error %s (communicator aborted)", ncclGetErrorString(ar));
+      return fail(DGR_ENCCL, "NCCL exchange not complete after %.0f ms (communicator aborted)", ms);
+    }
+    std::this_thread::sleep_for(std::chrono::microseconds(50));
+  }
 }
 
 static int dist_args(const dgr_dist* dist, int* rank, int* world) {
@@ -1212,11 +1377,18 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   P.wp = (float*)(ws + L.wp); P.mv = (float2*)(ws + L.mv);
   P.pp = (float*)(ws + L.pp);
   P.net_tree_off = (const int32_t*)(ws + L.nto);
+  P.net_gtree = (const int32_t*)(ws + L.net_gtree);
+  P.perm_id = 1;
+  for (size_t i = 0; i < pl.perm.size() && P.perm_id; ++i) P.perm_id = pl.perm[i] == (int64_t)i;
+  P.runs = (const NoiseRun*)(ws + L.runs);
   P.wt = (float*)(ws + L.wt); P.mt = (float*)(ws + L.mt); P.vt = (float*)(ws + L.vt); P.q = (float*)(ws + L.q);
   const size_t G = (size_t)desc->X * desc->Y;
   P.dH = (long long*)(ws + L.xbuf);
-  P.dVT = P.dH + G;
-  P.acc = P.dVT + G;
+  P.dVT = P.dH + L.gh;
+  P.acc = P.dVT + L.gv;
+  // the rank's KG lines (its grid bands; all lines on one GPU)
+  P.kg_h0 = std::min(desc->Y, rank * L.yb); P.kg_h1 = std::min(desc->Y, (rank + 1) * L.yb);
+  P.kg_v0 = std::min(desc->X, rank * L.xb); P.kg_v1 = std::min(desc->X, (rank + 1) * L.xb);
   P.capH = (const float*)(ws + L.capH);
   P.capVT = (const float*)(ws + L.capVT);
   P.SH = (double*)(ws + L.SH); P.SVT = (double*)(ws + L.SVT);
@@ -1262,7 +1434,7 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
       {L.pp, 4 * slots, nullptr},
       {L.slot_path, 4 * slots, pl.slot_path.data()},
       {L.nto, 4 * pl.net_tree_off.size(), pl.net_tree_off.data()},
-      {L.wt, 4 * nt, desc->w_tree0 + pl.tree_lo},
+      {L.wt, 4 * nt, nullptr},   // plan (tile) order of the trees
       {L.q, 4 * nt, nullptr},
       {L.capH, 4 * G, desc->cap_h},
       {L.capVT, 4 * G, nullptr},
@@ -1273,7 +1445,9 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
       {L.gp_seg_off, 4 * pl.gp_seg_off.size(), pl.gp_seg_off.data()},
       {L.gp_tp_off, 4 * pl.gp_tp_off.size(), pl.gp_tp_off.data()},
       {L.gseg, 8 * pl.gseg.size(), pl.gseg.data()},
-      {L.gtp, 4 * pl.gtp.size(), pl.gtp.data()}};
+      {L.gtp, 4 * pl.gtp.size(), pl.gtp.data()},
+      {L.net_gtree, 4 * pl.net_gtree.size(), pl.net_gtree.data()},
+      {L.runs, sizeof(NoiseRun) * pl.runs.size(), pl.runs.data()}};
   std::vector<size_t> at(regs.size() + 1, 0);
   for (size_t i = 0; i < regs.size(); ++i) at[i + 1] = at[i] + ((regs[i].bytes + 255) & ~(size_t)255);
   std::lock_guard<std::mutex> lock(g_pin.m);
@@ -1282,6 +1456,8 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   float* wslots = reinterpret_cast<float*>(pin + at[5]);
   float* pslots = reinterpret_cast<float*>(pin + at[6]);
   float* qs = reinterpret_cast<float*>(pin + at[10]);
+  float* wts = reinterpret_cast<float*>(pin + at[9]);
+  for (size_t j = 0; j < nt; ++j) wts[j] = desc->w_tree0[pl.tree_lo + pl.tperm[j]];
   float* capVT = reinterpret_cast<float*>(pin + at[12]);
 #pragma omp parallel for schedule(static)
   for (size_t sl = 0; sl < slots; ++sl) {
@@ -1343,8 +1519,7 @@ int dgr_sync(dgr_handle* h) {
   g_err.clear();
   DevGuard dg(h);
   if (!h) return fail(DGR_EINVAL, "NULL handle");
-  CUDA_TRY(cudaStreamSynchronize(h->stream));
-  return DGR_OK;
+  return wait_stream(h);
 }
 
 static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w, dgr_loss* last,
@@ -1358,6 +1533,7 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
   if (w->f_kind < 0 || w->f_kind > 4) return fail(DGR_EINVAL, "f_kind must be 0..4 (sigmoid, ReLU, LeakyReLU, exp, CELU)");
   if ((w->f_kind == 0 || w->f_kind == 3 || w->f_kind == 4) && !(w->f_slope > 0.f))
     return fail(DGR_EINVAL, "f_slope must be > 0 for sigmoid / exp / CELU");
+  if (int rc0 = live_comm(h)) return rc0;
   KParams& P = h->P;
   StepArgs a{};
   a.inv_t = 1.f / temperature;
@@ -1365,6 +1541,9 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
   a.sqrt_l = std::sqrt(w->n_layers);
   a.f_slope = w->f_slope; a.f_kind = w->f_kind;
   a.beta_q = (double)w->beta_via * kGridBeta;
+  a.beta_d = (double)a.beta;
+  a.a_wl_d = (double)a.a_wl;
+  a.via_d = (double)a.a_via * (double)a.sqrt_l;
   a.beta_exact = std::nearbyint(a.beta_q) == a.beta_q && std::fabs(a.beta_q) < 9.0e15;
   a.beta_qi = a.beta_exact ? (long long)a.beta_q : 0;
   const size_t xbytes = 8 * h->lay.xcount;
@@ -1399,13 +1578,42 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
     a.k_next = h->k + 1;
     a.store_d = last;
     adam_args(h->k);
+    const Layout& Lay = h->lay;
     if (h->world > 1) {
-      if ((rc = allreduce(h, P.dH, (int64_t)h->lay.xcount, 0))) return rc;
+      // the forward's events reduced into each rank's grid bands (SURVEY §8(e) refinement 2), the
+      // counters summed; the other ranks' bands cleared for the next forward (KG clears its own)
+      const int r = h->rank;
+      const size_t hb = (size_t)Lay.yb * h->X, vb = (size_t)Lay.xb * h->Y;
+      if ((rc = group_start(h)) || (rc = reduce_scatter(h, P.dH, (int64_t)hb, kI64)) ||
+          (rc = reduce_scatter(h, P.dVT, (int64_t)vb, kI64)) || (rc = allreduce(h, P.acc, 2, kI64)) || (rc = group_end(h)))
+        return rc;
+      if (r > 0) CUDA_TRY(cudaMemsetAsync(P.dH, 0, 8 * hb * r, s));
+      if (r + 1 < h->world) CUDA_TRY(cudaMemsetAsync(P.dH + hb * (r + 1), 0, 8 * hb * (h->world - r - 1), s));
+      if (r > 0) CUDA_TRY(cudaMemsetAsync(P.dVT, 0, 8 * vb * r, s));
+      if (r + 1 < h->world) CUDA_TRY(cudaMemsetAsync(P.dVT + vb * (r + 1), 0, 8 * vb * (h->world - r - 1), s));
+      if (last) {   // the loss sums every line's partial: the other bands' lines enter as zeros
+        CUDA_TRY(cudaMemsetAsync(P.partial, 0, 8 * (size_t)(h->X + h->Y), s));
+        CUDA_TRY(cudaMemsetAsync(P.lpart, 0, 8 * (size_t)(h->X + h->Y), s));
+      }
       if ((rc = prof_mark(h, 1))) return rc;
     }
-    launch_kg(P, a, s);
+    launch_kg(P, a, s);   // this rank's bands (every line on one GPU)
     h->grids_dirty = false;
     if ((rc = prof_mark(h, 2))) return rc;
+    if (h->world > 1) {
+      // the prefix sums S of every band to every rank (each rank's tiles read any of them); in the
+      // last iteration also the loss partials and the demand of get_demand
+      const size_t XP = (size_t)P.XP, YP = (size_t)P.YP;
+      if ((rc = group_start(h)) || (rc = all_gather(h, P.SH, (int64_t)(Lay.yb * XP), kF64)) ||
+          (rc = all_gather(h, P.SVT, (int64_t)(Lay.xb * YP), kF64)))
+        return rc;
+      if (last && ((rc = allreduce(h, P.partial, h->X + h->Y, kF64)) || (rc = allreduce(h, P.lpart, h->X + h->Y, kI64)) ||
+                   (rc = all_gather(h, P.dOutH, (int64_t)Lay.yb * h->X, kF32)) ||
+                   (rc = all_gather(h, P.dOutVT, (int64_t)Lay.xb * h->Y, kF32))))
+        return rc;
+      if ((rc = group_end(h))) return rc;
+      if ((rc = prof_mark(h, 1))) return rc;
+    }
     if (last) {   // the reported loss of this call's last forward
       launch_kg_loss(P, a, s);
       if ((rc = prof_mark(h, 5))) return rc;
@@ -1441,7 +1649,7 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
     CUDA_TRY(cudaMemcpyAsync(loss_async, P.loss, 4 * sizeof(double), cudaMemcpyDeviceToHost, s));
   if (last) {
     CUDA_TRY(cudaMemcpyAsync(h->pinned, P.loss, 4 * sizeof(double), cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(cudaStreamSynchronize(s));
+    if (int rc_ = wait_stream(h)) return rc_;
     last->total = h->pinned[0];
     last->wl = h->pinned[1];
     last->via = h->pinned[2];
@@ -1460,7 +1668,7 @@ int dgr_get_demand(dgr_handle* h, float* d_h, float* d_v) {
   std::vector<float> vt(G);
   CUDA_TRY(cudaMemcpyAsync(d_h, h->P.dOutH, 4 * G, cudaMemcpyDeviceToHost, h->stream));
   CUDA_TRY(cudaMemcpyAsync(vt.data(), h->P.dOutVT, 4 * G, cudaMemcpyDeviceToHost, h->stream));
-  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  if (int rc_ = wait_stream(h)) return rc_;
   for (int x = 0; x < h->X; ++x)
     for (int y = 0; y < h->Y; ++y) d_v[(size_t)y * h->X + x] = vt[(size_t)x * h->Y + y];
   return DGR_OK;
@@ -1475,14 +1683,15 @@ int dgr_get_logits(dgr_handle* h, float* w_tree, float* w_path) {
   if (w_path) {
     std::vector<float> slots((size_t)pl.nb * 32 + (size_t)pl.n_gpath);
     CUDA_TRY(cudaMemcpyAsync(slots.data(), h->P.wp, 4 * slots.size(), cudaMemcpyDeviceToHost, h->stream));
-    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    if (int rc_ = wait_stream(h)) return rc_;
     for (size_t sl = 0; sl < slots.size(); ++sl)
       if (pl.slot_path[sl] >= 0) w_path[pl.path_lo + pl.slot_path[sl]] = slots[sl];
   }
-  if (w_tree) {
-    CUDA_TRY(cudaMemcpyAsync(w_tree + pl.tree_lo, h->P.wt, 4 * (size_t)(pl.tree_hi - pl.tree_lo),
-                             cudaMemcpyDeviceToHost, h->stream));
-    CUDA_TRY(cudaStreamSynchronize(h->stream));
+  if (w_tree) {   // the device holds the trees in plan order (tperm: plan order -> local CSR)
+    std::vector<float> wt((size_t)(pl.tree_hi - pl.tree_lo));
+    CUDA_TRY(cudaMemcpyAsync(wt.data(), h->P.wt, 4 * wt.size(), cudaMemcpyDeviceToHost, h->stream));
+    if (int rc_ = wait_stream(h)) return rc_;
+    for (size_t j = 0; j < wt.size(); ++j) w_tree[pl.tree_lo + pl.tperm[j]] = wt[j];
   }
   return DGR_OK;
 }
@@ -1518,13 +1727,13 @@ int dgr_induce(dgr_handle* h, float top_p, int32_t* tree_choice, int32_t* route,
   CUDA_TRY(cudaMemcpyAsync(D_h, P.DH, 4 * G, cudaMemcpyDeviceToHost, s));
   CUDA_TRY(cudaMemcpyAsync(D_v, P.DV, 4 * G, cudaMemcpyDeviceToHost, s));
   CUDA_TRY(cudaMemcpyAsync(h->pinned, P.metrics, 5 * sizeof(double), cudaMemcpyDeviceToHost, s));
-  CUDA_TRY(cudaStreamSynchronize(s));
+  if (int rc_ = wait_stream(h)) return rc_;
   for (int i = 0; i < 5; ++i) metrics[i] = h->pinned[i];
   if (h->world > 1) {
     std::fill(tree_choice, tree_choice + h->n_nets, -1);
     std::fill(route, route + h->n_subnets, -1);
   }
-  std::copy(tc.begin(), tc.end(), tree_choice + pl.net_lo);
+  for (int64_t pn = 0; pn < nn; ++pn) tree_choice[pl.net_lo + pl.perm[pn]] = tc[pn];   // plan order -> CSR
   // route / nsize come in kernel sub-net order; nucleus_tmp holds each sub-net's nucleus in rank
   // order from its first candidate's slot on
   std::vector<int32_t> nsz_csr(ns);

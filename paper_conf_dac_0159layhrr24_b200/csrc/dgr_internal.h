@@ -17,8 +17,8 @@
 //     in that "kernel order" too (a permutation of the tile's sub-net range).
 //   * per slot:    pword (shape | flags | tree offset | mid), w, m, v (fp32), p of the last
 //     forward (fp32)
-//   * per bundle:  {noise index of lane 0, first kernel-order sub-net, the tile's first tree,
-//     #valid lanes | kSingleBundle}
+//   * per bundle:  {tile noise offset of lane 0 (its noisy candidates before this bundle), first
+//     kernel-order sub-net, the tile's first tree, #valid lanes | kSingleBundle}
 //   * per sub-net: canonical endpoints (x0 <= x1; y0 < y1 if x0 == x1) as int16 x 4
 //   * per tree:    w, m, v, q (fp32)
 //   * grids: difference arrays of the demand along H rows ([Y][X]) and along V columns (stored
@@ -93,6 +93,15 @@ struct TileDesc {
   int32_t mn0, nmn;        // the tile's nets with >= 2 trees: mnets[mn0 .. mn0 + nmn) (net offsets in the tile)
   int32_t tmap;            // pipelined tiles: index of the (S_H, S_V) tensor-map pair of the window's shape
                            // (one 2-D TMA copy per field), -1: the window comes by cp.async
+  int32_t run0, nrun;      // noise runs[run0 .. run0 + nrun): the tile's noisy candidates in bundle order as
+  int32_t nquad;           // runs of consecutive global noise indices; Philox quads they span in total
+  int32_t nid0, nnoisy;    // the first run's local noise index; the tile's noisy candidates (one run: all)
+};
+
+// A run of a tile's noisy candidates (group-bundle lanes in order, padding skipped) whose global noise
+// indices are consecutive: tile noise offsets [off, off + len) draw noise indices nid_base + nid ..
+struct NoiseRun {
+  int32_t off, len, nid, quad0;   // quad0: Philox quads of the tile's earlier runs
 };
 
 // "General" nets (row f4'): nets with a sub-net whose candidates are not all Z(o, m)
@@ -127,6 +136,7 @@ struct KParams {
   int32_t ngen;             // general nets (row f4'), run by CTAs [ntiles_slow, ntiles_slow + ngen_blocks)
   int32_t ngen_blocks;
   int32_t ngsub;            // their sub-nets
+  int32_t kg_h0, kg_h1, kg_v0, kg_v1;   // the rank's KG lines: H rows [kg_h0, kg_h1), V columns [kg_v0, kg_v1)
   int64_t path_base, tree_base;   // global index of the first local path / tree
   int64_t nid_base;         // global noise index of the rank's first noisy candidate
   uint64_t seed;
@@ -143,6 +153,9 @@ struct KParams {
   float* pp;                // p_i of the last forward (the reverse of that iteration reads it)
   const int32_t* net_tree_off;    // local, n_nets_l + 1
   const int32_t* mnets;     // per tile: offsets (in the tile) of its nets with >= 2 trees
+  const int32_t* net_gtree; // per (plan-ordered) local net: local CSR index of its first tree (tree noise key, Q7)
+  int32_t perm_id;          // the plan keeps the caller's net order (plan-ordered trees = CSR trees)
+  const NoiseRun* runs;     // per tile: noise runs (TileDesc run0 / nrun)
   const unsigned char* tmaps;   // CUtensorMap pairs (S_H window, S_V window), 128 B each, per window shape
   // general nets (row f4'): per net {first gtree, trees}; per tree {local tree, first gsub, sub-nets,
   // multi-tree flag}; per sub-net a GSub; per general path its segment / turning-point ranges
@@ -192,6 +205,7 @@ struct StepArgs {
   float inv_sqrt_bc2; // 1 / sqrt(1 - beta2^(k+1))
   float a_wl, a_via, a_of, beta, sqrt_l, f_slope;
   double beta_q;      // beta * 2^16: a turning point's pi (2^-24) -> its folded demand (2^-40)
+  double beta_d, a_wl_d, via_d;   // beta, a1, a2 sqrt(L) in fp64 (the path cost's constants)
   long long beta_qi;  // the same as an integer when beta_exact
   int32_t beta_exact; // beta * 2^16 is an integer (beta a multiple of 2^-16): exact integer folds
   int32_t f_kind;

@@ -93,6 +93,47 @@ __device__ __forceinline__ float gumbel(uint64_t seed, uint64_t idx, uint32_t k,
   return gumbel_word(s == 0 ? r.x : (s == 1 ? r.y : (s == 2 ? r.z : r.w)));
 }
 
+// Gumbel noise (stream 0) of a tile's noisy candidates into gp[tile noise offset]: the tile's runs of
+// consecutive global noise indices (NoiseRun), one Philox call per aligned quad of indices, spread
+// over the CTA's threads (a quad's run found by binary search over the runs' quad offsets).
+template <int NT>
+__device__ __forceinline__ void tile_noise(const KParams& P, const TileDesc& T, uint32_t k, float* gp) {
+  if (T.nrun == 1) {   // one run (nets in the caller's order): its quads spread over the threads
+    const int64_t g0 = P.nid_base + T.nid0;
+    for (int q = threadIdx.x; q < T.nquad; q += NT) {
+      const int64_t c = (g0 >> 2) + q;
+      const uint4 w = philox_rk(make_uint4((uint32_t)c, (uint32_t)(c >> 32), k, 0u), P.rk);
+      const uint32_t wd[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int64_t o = c * 4 + i - g0;
+        if (o >= 0 && o < T.nnoisy) gp[o] = gumbel_word(wd[i]);
+      }
+    }
+    return;
+  }
+  // several runs (nets re-ordered by the plan): the quads spread over the threads, a quad's run found
+  // by binary search over the runs' quad offsets (a thread per run would serialise a large net's quads)
+  const int4* R = reinterpret_cast<const int4*>(P.runs) + T.run0;   // {off, len, nid, quad0}
+  for (int q = threadIdx.x; q < T.nquad; q += NT) {
+    int lo = 0, hi = T.nrun - 1;
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (__ldg(&R[mid].w) <= q) lo = mid; else hi = mid - 1;
+    }
+    const int4 r = __ldg(&R[lo]);
+    const int64_t g0 = P.nid_base + r.z;
+    const int64_t c = (g0 >> 2) + (q - r.w);
+    const uint4 w = philox_rk(make_uint4((uint32_t)c, (uint32_t)(c >> 32), k, 0u), P.rk);
+    const uint32_t wd[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int64_t o = c * 4 + i - g0;
+      if (o >= 0 && o < r.y) gp[r.x + o] = gumbel_word(wd[i]);
+    }
+  }
+}
+
 // ------------------------------------------------------------------------------------------
 // Per-lane view of a bundle: which sub-net group / tree / global candidate this lane is.
 // ------------------------------------------------------------------------------------------
@@ -102,7 +143,6 @@ struct Lane {
   bool valid;
   int sub, tree;
   bool single;     // lane of a singleton bundle (lone straight sub-nets: p = 1, no noise)
-  int64_t nid;     // global noise index (group bundles; reading Q7)
 };
 
 __device__ __forceinline__ void lane_setup(const KParams& P, int b, Lane& L) {
@@ -121,7 +161,6 @@ __device__ __forceinline__ void lane_setup(const KParams& P, int b, Lane& L) {
   L.sub = bi.y + __popc(L.hm & L.le) - 1;
   L.tree = bi.z + (int)((L.pw >> kTreeShift) & kTreeMask);
   L.single = (bi.w & kSingleBundle) != 0;
-  L.nid = P.nid_base + bi.x + L.lane;
 }
 
 // reduction over the lane's group [head, end]; the result is valid at the head lane
@@ -345,7 +384,7 @@ __device__ __forceinline__ double path_cost(const double* S, const Win& W, int X
   if (ntp >= 1) tp = (S[a0 + mp] - S[a0 - mn]) + (S[s0 + (q0 < qmax)] - S[s0 - (q0 > 0)]);
   if (ntp == 2) tp += (S[a1 + mp] - S[a1 - mn]) + (S[s1 + (q1 < qmax)] - S[s1 - (q1 > 0)]);
   const int wl = abs(m - p0) + abs(p1 - m) + abs(q1 - q0);
-  return c + (double)A.beta * tp + (double)A.a_wl * (double)wl + (double)A.a_via * (double)A.sqrt_l * (double)ntp;
+  return c + A.beta_d * tp + A.a_wl_d * (double)wl + A.via_d * (double)ntp;
 }
 
 // wire length of a candidate in the Z(o, m) form (every shape: straight, L, Z, C)
@@ -396,7 +435,6 @@ __device__ __forceinline__ void lane_from(int4 bi, uint32_t pw, const KParams& P
   L.sub = bi.y + __popc(L.hm & L.le) - 1;
   L.tree = bi.z + (int)((pw >> kTreeShift) & kTreeMask);
   L.single = (bi.w & kSingleBundle) != 0;
-  L.nid = P.nid_base + bi.x + L.lane;
 }
 
 // p_i = exp(z_i - m) / sum_k exp(z_k - m) for any shift m (softmax shift invariance): m = the group
@@ -517,7 +555,7 @@ struct EWin {
 
 template <bool GLOBAL>
 __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A, const TileDesc& T, int bw0,
-                                             int bw1, bool have_w, const float* wst, const float* q_s, float* g_s,
+                                             int bw1, bool have_w, const float* wst, const float* q_s, const float* gt,
                                              const EWin& W, int* ev_s, long long& etp, long long& bdef) {
   const int lane = threadIdx.x & 31;
   const int4 bfirst = __ldg(&P.binfo[bw0]);
@@ -529,16 +567,18 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
   int4 bi1 = make_int4(0, 0, 0, 0);
   uint32_t pw1 = kPad | kSubHead;
   if (bw0 + 1 < bw1) { bi1 = __ldg(&P.binfo[bw0 + 1]); pw1 = __ldg(&P.pword[slot + 32]); }
+  int boff = bfirst.x, boffn = 0;   // the bundles' tile noise offsets
   for (int b = bw0; b < bw1; ++b) {
     Lane Ln = L;
     short4 en = e;
     if (b + 1 < bw1) {
+      boffn = bi1.x;
       lane_from(bi1, pw1, P, Ln);
       if (Ln.valid) en = __ldg(&P.sxy[Ln.sub]);
       if (b + 2 < bw1) { bi1 = __ldg(&P.binfo[b + 2]); pw1 = __ldg(&P.pword[slot + 64]); }
     }
     const float w = have_w ? wst[(b - T.b0) * 32 + lane] : P.wp[slot];
-    const float g = (L.valid && !L.single) ? gumbel(P.seed, (uint64_t)L.nid, (uint32_t)A.k_next, 0u) : 0.f;
+    const float g = (L.valid && !L.single) ? gt[boff + L.lane] : 0.f;   // the tile's noise, by offset
     const float p = softmax_from_noise(L, w, g, A.inv_t);
     P.pp[slot] = p;
     const float q = L.valid ? q_s[L.tree - T.tree0] : 0.f;
@@ -606,7 +646,7 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
       red_shared_add(ev_base + 4u * W.v(xb, yb), bv);
       red_shared_add(ev_base + 4u * W.d(xb, yb), bd);
     }
-    L = Ln; e = en;
+    L = Ln; e = en; boff = boffn;
     slot += 32;
   }
 
@@ -629,7 +669,6 @@ __device__ __forceinline__ void slow_tile(const KParams& P, const StepArgs& A, c
   const int ncell = T.ww * T.wh;
   const Win Wg{0, 0, P.XP, P.YP, (int)(P.SVT - P.SH)};
   const Win Ws{T.wx0, T.wy0, T.ww, T.wh, ncell};
-  float* g_s = g_all + warp * kWarpCand;
   // this warp's contiguous bundle range
   const int per = (T.nb + kWarps - 1) / kWarps;
   const int bw0 = T.b0 + min(warp * per, T.nb), bw1 = T.b0 + min((warp + 1) * per, T.nb);
@@ -685,7 +724,7 @@ __device__ __forceinline__ void slow_tile(const KParams& P, const StepArgs& A, c
       } else {
         float zmax = -INFINITY;
         for (int j = a; j < b; ++j) {
-          const float z = (P.wt[j] + gumbel(P.seed, (uint64_t)(P.tree_base + j), (uint32_t)A.k_next, 1u)) * A.inv_t;
+          const float z = (P.wt[j] + gumbel(P.seed, (uint64_t)(P.tree_base + P.net_gtree[net] + (j - a)), (uint32_t)A.k_next, 1u)) * A.inv_t;
           q_s[j - T.tree0] = z;
           zmax = fmaxf(zmax, z);
         }
@@ -706,12 +745,13 @@ __device__ __forceinline__ void slow_tile(const KParams& P, const StepArgs& A, c
       int4* z = reinterpret_cast<int4*>(ev_s);
       for (int i = tid; i < (3 * ncell + 3) / 4; i += kTileThreads) z[i] = make_int4(0, 0, 0, 0);
     }
+    if (T.nbg > 0) tile_noise<kTileThreads>(P, T, (uint32_t)A.k_next, g_all);   // path noise by tile noise offset
     __syncthreads();
     long long etp = 0, bdef = 0;
     const EWin Ew{T.wx0, T.wy0, T.ww, ncell};
     if (bw0 < bw1) {
-      if (T.global) forward_warp<true>(P, A, T, bw0, bw1, REV, wst, q_s, g_s, Ew, ev_s, etp, bdef);
-      else forward_warp<false>(P, A, T, bw0, bw1, REV, wst, q_s, g_s, Ew, ev_s, etp, bdef);
+      if (T.global) forward_warp<true>(P, A, T, bw0, bw1, REV, wst, q_s, g_all, Ew, ev_s, etp, bdef);
+      else forward_warp<false>(P, A, T, bw0, bw1, REV, wst, q_s, g_all, Ew, ev_s, etp, bdef);
     }
     __syncthreads();
     if (!T.global) flush_window<kTileThreads>(P, A, T.wx0, T.wy0, T.ww, T.wh, ncell, ev_s, etp, bdef);
@@ -1061,7 +1101,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
           const short4 e = St.sxy[bi.y + lane - s_lo];
           const int ia = isv ? W.v(e.x, e.y) : W.h(e.x, e.y);
           const int ib = isv ? W.v(e.x, e.w) : W.h(e.z, e.y);
-          c = (St.S[ib] - St.S[ia]) + (double)A.a_wl * (double)((e.z - e.x) + (e.w - e.y));
+          c = (St.S[ib] - St.S[ia]) + A.a_wl_d * (double)((e.z - e.x) + (e.w - e.y));
         }
         const uint32_t th = __ballot_sync(kFull, (pw & kTreeHead) || !valid) | 1u;
         const uint32_t le = kFull >> (31 - lane);
@@ -1111,7 +1151,8 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
       int64_t cq = -1;   // one Philox call per aligned quad of tree indices
       uint4 r = make_uint4(0u, 0u, 0u, 0u);
       for (int j = a; j < b; ++j) {
-        const int64_t gj = P.tree_base + t_lo + j;
+        // global tree id (plan order = CSR order unless the plan re-ordered the nets)
+        const int64_t gj = P.tree_base + (P.perm_id ? t_lo + j : __ldg(&P.net_gtree[T.net0 + n]) + (j - a));
         if ((gj >> 2) != cq) {
           cq = gj >> 2;
           r = philox_rk(make_uint4((uint32_t)cq, (uint32_t)(cq >> 32), (uint32_t)A.k_next, 1u), P.rk);
@@ -1130,30 +1171,13 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
       }
     }
   }
-  if (FWD && nbg > 0 && !(KO(2))) {
-    // Gumbel noise of the tile's noisy candidates (stream 0): contiguous noise indices
-    // [bi[0].x, bi[nbg-1].x + #valid), one Philox call per 4 consecutive indices
-    const int64_t n0 = P.nid_base + St.bi[0].x;
-    const int4 bl = St.bi[nbg - 1];
-    const int nn = bl.x + (bl.w & 0xff) - St.bi[0].x;
-    const int64_t c0 = n0 >> 2, c1 = (n0 + nn - 1) >> 2;
-    for (int64_t c = c0 + tid; c <= c1; c += NT) {
-      const uint4 r = philox_rk(make_uint4((uint32_t)c, (uint32_t)(c >> 32), (uint32_t)A.k_next, 0u), P.rk);
-      const uint32_t wd[4] = {r.x, r.y, r.z, r.w};
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const int64_t i = c * 4 + q - n0;
-        if (i >= 0 && i < nn) gp[i] = gumbel_word(wd[q]);
-      }
-    }
-  }
+  if (FWD && nbg > 0 && !(KO(2))) tile_noise<NT>(P, T, (uint32_t)A.k_next, gp);   // path noise (stream 0)
   __syncthreads();
   stamp(P, (int)blockIdx.x - P.ntiles_slow - P.ngen_blocks, 3);
 
   // ---------------- forward of iteration k_next ----------------
   if (FWD) {
     const uint32_t ev_base = smem_u32(ev_s);
-    const int nid0 = nbg > 0 ? St.bi[0].x : 0;
     for (int lb = warp; lb < T.nb; lb += NW) {
       const int4 bi = St.bi[lb];
       const uint32_t pw = St.pw[lb * 32 + lane];
@@ -1162,7 +1186,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         lane_from(bi, pw, P, L);
         const int sl = lb * 32 + lane;
         const float w = St.w[sl];
-        const float g = L.valid ? gp[bi.x + lane - nid0] : 0.f;
+        const float g = L.valid ? gp[bi.x + lane] : 0.f;   // bi.x: the bundle's tile noise offset
         const float p = softmax_from_noise(L, w, g, A.inv_t);
         st_stream(&P.pp[(size_t)T.b0 * 32 + sl], p, pol);
         const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
@@ -1268,7 +1292,7 @@ __device__ __forceinline__ double gen_cost(const KParams& P, const StepArgs& A, 
     const double* SV = P.SVT + (size_t)v.x * P.YP;
     tp += (SH[v.x + (v.x < X - 1)] - SH[v.x - (v.x > 0)]) + (SV[v.y + (v.y < Y - 1)] - SV[v.y - (v.y > 0)]);
   }
-  return c + (double)A.beta * tp + (double)A.a_wl * (double)wl + (double)A.a_via * (double)A.sqrt_l * (double)(t1 - t0);
+  return c + A.beta_d * tp + A.a_wl_d * (double)wl + A.via_d * (double)(t1 - t0);
 }
 
 // demand events of general path gp with weight v (2^-24): +-v at each segment's ends, folded turning points
@@ -1365,16 +1389,16 @@ __device__ __forceinline__ void gen_net(const KParams& P, const StepArgs& A, int
       float zmax = -INFINITY;
       for (int g = g0; g < g1; ++g) {
         const int j = P.gtree[g].x;
-        zmax = fmaxf(zmax, (P.wt[j] + gumbel(P.seed, (uint64_t)(P.tree_base + j), (uint32_t)A.k_next, 1u)) * A.inv_t);
+        zmax = fmaxf(zmax, (P.wt[j] + gumbel(P.seed, (uint64_t)(P.tree_base + P.gtree[g].w), (uint32_t)A.k_next, 1u)) * A.inv_t);
       }
       float sum = 0.f;
       for (int g = g0; g < g1; ++g) {
         const int j = P.gtree[g].x;
-        sum += FEXP((P.wt[j] + gumbel(P.seed, (uint64_t)(P.tree_base + j), (uint32_t)A.k_next, 1u)) * A.inv_t - zmax);
+        sum += FEXP((P.wt[j] + gumbel(P.seed, (uint64_t)(P.tree_base + P.gtree[g].w), (uint32_t)A.k_next, 1u)) * A.inv_t - zmax);
       }
       for (int g = g0; g < g1; ++g) {
         const int j = P.gtree[g].x;
-        P.q[j] = FEXP((P.wt[j] + gumbel(P.seed, (uint64_t)(P.tree_base + j), (uint32_t)A.k_next, 1u)) * A.inv_t - zmax) / sum;
+        P.q[j] = FEXP((P.wt[j] + gumbel(P.seed, (uint64_t)(P.tree_base + P.gtree[g].w), (uint32_t)A.k_next, 1u)) * A.inv_t - zmax) / sum;
       }
     }
   }
@@ -1685,7 +1709,10 @@ __global__ void __launch_bounds__(kGThreads, DGR_KG_MINB) kg_kernel(KParams P, S
   __shared__ long long shwl[kKgWarps];
   griddep_launch();
   griddep_wait();   // the difference arrays are complete (the previous KBF / allreduce)
-  const int nl = P.X + P.Y, lane = threadIdx.x & 31;
+  // the rank's lines (SURVEY §8(e) refinement 2): H rows [kg_h0, kg_h1), then V columns [kg_v0, kg_v1)
+  // (all of them on one GPU); slot b is line slot_line(b) (line ids: rows 0..Y-1, columns Y..Y+X-1)
+  const int nhs = P.kg_h1 - P.kg_h0, nl = nhs + (P.kg_v1 - P.kg_v0), lane = threadIdx.x & 31;
+  auto slot_line = [&](int b) { return b < nhs ? P.kg_h0 + b : P.Y + P.kg_v0 + (b - nhs); };
   if (blockIdx.x == 0 && threadIdx.x == 0) {   // E[TP], B of this forward, for the loss; cleared for the next
     P.lsum[0] = P.acc[0]; P.lsum[1] = P.acc[1];
     P.acc[0] = 0; P.acc[1] = 0;
@@ -1706,8 +1733,9 @@ __global__ void __launch_bounds__(kGThreads, DGR_KG_MINB) kg_kernel(KParams P, S
       cc[j] = pos < n ? cap[pos] : 0.f;
     }
   };
-  int line = blockIdx.x, c0 = 0;
-  if (line >= nl) return;
+  int slot = blockIdx.x, c0 = 0;
+  if (slot >= nl) return;
+  int line = slot_line(slot);
   load(line, 0, v, cp);
   long long carryW = 0, sumD = 0;   // sumD: sum over the line's edges of the demand (2^-40)
   double carryS = 0.0, of = 0.0;
@@ -1719,11 +1747,12 @@ __global__ void __launch_bounds__(kGThreads, DGR_KG_MINB) kg_kernel(KParams P, S
     double* S = isH ? P.SH + (size_t)ln * P.XP : P.SVT + (size_t)ln * P.YP;
     float* dout = (isH ? P.dOutH : P.dOutVT) + (size_t)ln * n;
     // the next chunk of this CTA (the rest of this line, else its next line), prefetched
-    int nline = line, nc0 = c0 + kGThreads * kGItems;
-    if (nc0 >= n) { nline += gridDim.x; nc0 = 0; }
+    int nslot = slot, nc0 = c0 + kGThreads * kGItems;
+    if (nc0 >= n) { nslot += gridDim.x; nc0 = 0; }
+    const int nline = nslot < nl ? slot_line(nslot) : -1;
     long long nv[kGItems];
     float ncp[kGItems];
-    if (nline < nl) load(nline, nc0, nv, ncp);
+    if (nslot < nl) load(nline, nc0, nv, ncp);
     long long totW;
     long long ex[kGItems];
 #pragma unroll
@@ -1783,9 +1812,9 @@ __global__ void __launch_bounds__(kGThreads, DGR_KG_MINB) kg_kernel(KParams P, S
       }
       carryW = 0; sumD = 0; carryS = 0.0; of = 0.0;
     }
-    if (nline >= nl) break;
+    if (nslot >= nl) break;
     __syncthreads();   // the next chunk reuses shl / shd / shw
-    line = nline; c0 = nc0;
+    slot = nslot; line = nline; c0 = nc0;
 #pragma unroll
     for (int j = 0; j < kGItems; ++j) { v[j] = nv[j]; cp[j] = ncp[j]; }
   }
@@ -1803,7 +1832,7 @@ __global__ void __launch_bounds__(256) ki_tree_kernel(KParams P) {
   int best = a;
   for (int j = a + 1; j < b; ++j) if (P.wt[j] > P.wt[best]) best = j;   // q_hat monotone in w
   for (int j = a; j < b; ++j) P.chosen[j] = (j == best);
-  P.tree_choice[n] = (int32_t)(P.tree_base + best);
+  P.tree_choice[n] = (int32_t)(P.tree_base + P.net_gtree[n] + (best - a));   // global (CSR) tree id
 }
 
 __global__ void __launch_bounds__(256) ki_path_kernel(KParams P, float inv_t, float top_p) {
@@ -2015,7 +2044,9 @@ void launch_tiles(const KParams& p, const StepArgs& a, TileMode mode, cudaStream
 void launch_kg_loss(const KParams& p, const StepArgs& a, cudaStream_t s) { kg_loss_kernel<<<1, 1024, 0, s>>>(p, a); }
 void launch_kg(const KParams& p, const StepArgs& a, cudaStream_t s) {
   cudaLaunchAttribute attr;
-  cudaLaunchConfig_t cfg = pdl_config(p.X + p.Y, kGThreads, 0, s, &attr);
+  const int nl = (p.kg_h1 - p.kg_h0) + (p.kg_v1 - p.kg_v0);
+  if (nl <= 0) return;
+  cudaLaunchConfig_t cfg = pdl_config(nl, kGThreads, 0, s, &attr);
   cudaLaunchKernelEx(&cfg, kg_kernel, p, a);
 }
 int induce_metric_blocks(const KParams& p) {

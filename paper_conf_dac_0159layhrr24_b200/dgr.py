@@ -219,14 +219,45 @@ class InduceResult:
     metrics: np.ndarray
 
 
+class _DevBuf:
+    """A library device buffer as a CUDA array (no copy)."""
+
+    def __init__(self, ptr: int, n: int, dtype: int):
+        self.__cuda_array_interface__ = {"shape": (int(n),), "typestr": ("<i8", "<i4", "<f8", "<f4")[dtype],
+                                         "data": (int(ptr), False), "version": 3}
+
+
+def torch_allreduce(group=None):
+    """A dgr_dist.allreduce callback over a torch.distributed process group (e.g. gloo: the ranks'
+    exchange without NCCL, so that several ranks can share one GPU).  Plumbing only: the buffer goes
+    to the host, torch.distributed sums it, and it comes back."""
+    import torch
+    import torch.distributed as tdist
+
+    def fn(buf, n, dtype, stream):
+        try:
+            st = torch.cuda.ExternalStream(stream) if stream else torch.cuda.current_stream()
+            st.synchronize()
+            dev = torch.as_tensor(_DevBuf(buf, n, dtype), device="cuda")
+            host = dev.cpu()
+            tdist.all_reduce(host, group=group)
+            dev.copy_(host)
+            torch.cuda.synchronize()
+            return 0
+        except Exception:   # the failing dgr_* call reports DGR_ENCCL
+            return 1
+    return fn
+
+
 class Solver:
     """One rank's DGR solver over a forest (any object with forestgen.Forest's fields)."""
 
     def __init__(self, forest, rank: int = 0, world: int = 1, nccl_id: bytes | None = None, device=None,
                  stream=None, allreduce=None):
         """allreduce: optional Python callable (buf_ptr, count, dtype, stream_ptr) -> int replacing NCCL
-        (dgr_dist.allreduce): sums `count` int64 (dtype 0) / int32 (dtype 1) elements at device address
-        buf_ptr over the ranks in place, after the work on stream_ptr."""
+        (dgr_dist.allreduce): sums `count` int64 / int32 / fp64 / fp32 (dtype 0 / 1 / 2 / 3) elements at
+        device address buf_ptr over the ranks in place, after the work on stream_ptr (e.g.
+        torch_allreduce() over a torch.distributed process group)."""
         import torch
         if not torch.cuda.is_available():
             raise DgrError("libdgr needs a CUDA device (no CPU fallback)")

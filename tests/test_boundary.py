@@ -221,3 +221,13 @@ def test_c_shape_detour_outside_grid_rejected(xm):
         pytest.fail("tiny_c has no C-HVH candidate")
     n, err = _ws(f)
     assert n == 0 and "malformed" in err, err
+
+
+def test_plan_restores_a_spatial_net_order():
+    """the plan takes nets in a spatial (Morton) order when the caller's order is
+    not spatially coherent, so a net-shuffled forest tiles like the sorted one (dgr_plan_info)."""
+    f = forestgen.generate("c1e4")
+    g = forestgen.shuffle_nets(f, seed=5)
+    a, b = dgr.plan_info(f), dgr.plan_info(g)
+    assert b["n_paths"] == a["n_paths"]
+    assert b["n_tiles"] <= 1.1 * a["n_tiles"] and b["n_global_tiles"] <= a["n_global_tiles"] + 2, (a, b)

@@ -22,7 +22,7 @@ class _DevArray:
     """A device buffer of the library as a torch tensor (CUDA array interface, no copy)."""
 
     def __init__(self, ptr: int, n: int, dtype: int):
-        self.__cuda_array_interface__ = {"shape": (int(n),), "typestr": "<i8" if dtype == 0 else "<i4",
+        self.__cuda_array_interface__ = {"shape": (int(n),), "typestr": ("<i8", "<i4", "<f8", "<f4")[dtype],
                                          "data": (int(ptr), False), "version": 3}
 
 
@@ -85,9 +85,9 @@ def _schedule(s):
     return losses, s.demand(), s.logits(), s.induce(0.9)
 
 
-@pytest.mark.parametrize("name,world", [("c1e4", 2), ("c1e4", 3), ("ispd18", 4), ("ispd19", 8), ("c1e4_m", 3)])
+@pytest.mark.parametrize("name,world", [("c1e4", 2), ("c1e4", 3), ("ispd18", 4), ("ispd19", 8), ("c1e4_m", 3), ("c1e4_nshuf", 2)])
 def test_sharded_ranks_reproduce_one_rank_bit_exactly(name, world):
-    f = forestgen.generate(name)
+    f = forestgen.shuffle_nets(forestgen.generate("c1e4"), seed=5) if name == "c1e4_nshuf" else forestgen.generate(name)
     ref = dgr.Solver(f)
     ref_losses, (rdh, rdv), (rwt, rwp), rind = _schedule(ref)
     ref.close()

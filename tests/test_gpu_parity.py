@@ -40,6 +40,8 @@ def forests():
     fs = {n: forestgen.generate(n) for n in ("tiny", "c1e4", "ispd18", "tiny_c", "c1e4_c", "tiny_m", "c1e4_m")}
     # row f4': candidates in a random order per sub-net (the general path, like the staircases)
     fs["c1e4_shuf"] = forestgen.shuffle_candidates(fs["c1e4"], seed=7)
+    # nets in a random order: the plan restores a spatial order (Morton)
+    fs["c1e4_nshuf"] = forestgen.shuffle_nets(fs["c1e4"], seed=5)
     return fs
 
 
@@ -222,7 +224,8 @@ def test_forward_parity(forests, name, f_kind):
     assert s.iteration == 0
 
 
-@pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18", "tiny_c", "c1e4_c", "tiny_m", "c1e4_m", "c1e4_shuf"])
+@pytest.mark.parametrize("name", ["tiny", "c1e4", "ispd18", "tiny_c", "c1e4_c", "tiny_m", "c1e4_m", "c1e4_shuf",
+                                  "c1e4_nshuf"])
 def test_one_iteration_parity(forests, name):
     """After one Adam step the update of a coordinate whose gradient is ~eps depends on that
     gradient's last bits (Q21b), so the fp32 probe applies from the first step on."""
@@ -239,6 +242,7 @@ def test_one_iteration_parity(forests, name):
     ("tiny_m", [(100, 1.0), (100, 0.9)]),                # row f4': staircases, groups > 32
     ("c1e4_m", [(100, 1.0)]),
     ("c1e4_shuf", [(100, 1.0)]),                         # any candidate order
+    ("c1e4_nshuf", [(100, 1.0)]),                        # any net order
 ])
 def test_trajectory_parity(forests, name, schedule):
     f = forests[name]
@@ -331,7 +335,7 @@ def test_step_async_equals_step(forests):
     assert np.array_equal(a.logits()[1], b.logits()[1]) and np.array_equal(a.logits()[0], b.logits()[0])
 
 
-@pytest.mark.parametrize("name", ["tiny", "c1e4", "c1e4_c", "tiny_m", "c1e4_m", "c1e4_shuf"])
+@pytest.mark.parametrize("name", ["tiny", "c1e4", "c1e4_c", "tiny_m", "c1e4_m", "c1e4_shuf", "c1e4_nshuf"])
 def test_induce_parity(forests, name):
     f = forests[name]
     s, o, _, _ = run_both(f, [(60, 1.0), (40, 0.9)])
@@ -449,3 +453,15 @@ def test_ispd18_staircases_one_iteration():
     for i in range(4):
         assert_rel(gl[0][i], ol[0][i], what="loss")
     compare_state(s, o, "ispd18_m", exempt=first_step_exempt(f), max_ill=1e-3)
+
+
+def test_dgr_star_search_reaches_the_optimum():
+    """Row f2, DGR* (P:880-885): on an enumerable Table-1-style instance the hyper-parameter search
+    (sampled lr in [1e-4, 1], gamma in {0.8, ..., 0.95}) reaches the brute-force optimum."""
+    import tools.dgr_star as ds
+    from tests.test_table1 import _small, brute_force_overflow
+    g = _small(3)
+    opt = brute_force_overflow(g)
+    default, sampled, best = ds.search(g, runs=12)
+    assert min(min(default), best[0]) == opt
+    assert all(o >= opt for o, _, _ in sampled)

@@ -14,7 +14,9 @@ import paper_conf_dac_0159layhrr24_b200 as dgr  # noqa: E402
 name = sys.argv[1] if len(sys.argv) > 1 else "ispd19"
 iters = int(sys.argv[2]) if len(sys.argv) > 2 else 200
 reps = int(sys.argv[3]) if len(sys.argv) > 3 else 3
-f = forestgen.generate(name)
+f = forestgen.generate(name.replace("+nshuf", ""))
+if name.endswith("+nshuf"):   # the same forest with its nets in a random order (the plan restores a spatial one)
+    f = forestgen.shuffle_nets(f, seed=5)
 s = dgr.Solver(f)
 s.step(20, 1.0, 0.3, want_loss=False)
 st = torch.cuda.current_stream()
