@@ -398,7 +398,7 @@ def main():
     sb = stage_bytes(st)        # this design's own minimum, stricter
     sv = survey_bytes(st, f.X, f.Y)   # SURVEY.md §8(d) per-unit figures (contract)
     per_launch_ms = {k: stage_ms[k] / n_prof[k] for k in stage_ms if n_prof[k]}
-    mine = {k: stage_ms[k] for k in stage_ms if k != "allreduce" and n_prof[k]}
+    mine = {k: stage_ms[k] for k in stage_ms if k in sb and n_prof[k]}   # the iteration's kernels (not the exchange / loss)
     dom = max(mine, key=mine.get)
     peak, peak_src = measured_peak()
     alg_dom = sv.get(dom, sb[dom])
@@ -461,10 +461,11 @@ def main():
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(f)
     s.close()
+    if world > 1:
+        barrier()   # every rank is done before rank 0 reports
     if rank == 0:
         print(json.dumps(line), flush=True)
-    if world > 1:
-        barrier()
+    if world > 1 and not gloo:   # (gloo: no teardown collective after the report; process exit closes it)
         tdist.destroy_process_group()
 
 

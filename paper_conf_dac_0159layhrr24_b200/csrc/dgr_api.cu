@@ -274,10 +274,12 @@ struct Plan {
   std::vector<int32_t> tperm;          // plan-ordered local tree -> local CSR tree
   std::vector<int32_t> net_gtree;      // plan position -> local CSR index of the net's first tree
   std::vector<NoiseRun> runs;          // per tile (TileDesc run0 / nrun)
-  std::vector<int32_t> mnets;           // per tile: offsets of its nets with >= 2 trees (TileDesc mn0 / nmn)
+  std::vector<uint32_t> mnets;          // per tile: the trees of its nets with >= 2 trees, one per lane (tree_lane),
+                                        // a net's trees never straddle a warp; padded to warps (TileDesc mn0 / nmn)
   PodBuf<int32_t> ksub_csr;             // kernel-order sub-net -> local CSR sub-net
   PodBuf<int64_t> sub_first_slot;       // local CSR sub-net -> slot of its first candidate
   PodBuf<int32_t> slot_path;            // slot -> local CSR path (-1: padding)
+  PodBuf<uint32_t> ldesc;               // per bundle slot: lane descriptor (lane_desc)
   std::vector<TileDesc> tiles;          // pipelined tiles first (see make_plan)
   int64_t n_global_tiles = 0;
   int64_t n_pipe_tiles = 0;
@@ -487,7 +489,22 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   pl.tiles.clear();
   pl.binfo.clear();
   pl.pword.clear();
-  struct Pack { int nbg = 0, fill = 32, nsing = 0; int total() const { return nbg + (nsing + 31) / 32; } };
+  // group bundles counted first-fit online (bin fills), singletons 32 to a bundle; the fill's packing
+  // (pack_groups) never needs more bundles than this count
+  struct Pack {
+    int nbg = 0, nsing = 0;
+    uint8_t fills[kMaxBundles];
+    int total() const { return nbg + (nsing + 31) / 32; }
+    void add(int g) {
+      int k = 0;
+      while (k < nbg && fills[k] + g > 32) ++k;
+      if (k == nbg) {
+        if (nbg == kMaxBundles) { ++nbg; return; }   // over the limit: the caller rejects the tile
+        fills[nbg++] = 0;
+      }
+      fills[k] = (uint8_t)(fills[k] + g);
+    }
+  };
   struct Cur { bool open = false; int64_t net0 = 0; Pack pk; int ntree = 0, nsub = 0; int bx0 = 0, by0 = 0, bx1 = -1, by1 = -1; bool global = false; };
   // bounding box of each net's sub-nets plus a 1-cell halo (parallel over nets)
   PodBuf<int4> nbox;
@@ -566,9 +583,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     for (int64_t s = s0; s < s1; ++s) {
       if (gen[s - pl.sub_lo]) continue;   // general path: virtual slots
       if (single[s - pl.sub_lo]) { ++pk.nsing; continue; }
-      const int g = (int)(d->sub_path_off[s + 1] - d->sub_path_off[s]);
-      if (pk.fill + g > 32) { ++pk.nbg; pk.fill = 0; }
-      pk.fill += g;
+      pk.add((int)(d->sub_path_off[s + 1] - d->sub_path_off[s]));
     }
   };
   // windows start on even cells and have even extents so their S rows / columns are 16-byte
@@ -645,6 +660,45 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   }
   starts.push_back(nn);   // plan positions
   tm.mark("tiles (greedy)");
+  // Group bundles of a tile: its noisy sub-nets (groups of g <= 32 candidates, never split) packed
+  // first-fit decreasing (ties in plan order), or first-fit in plan order when that needs fewer
+  // bundles (so never more than the tile greedy's first-fit count).  Returns the bins as lists of indices into the tile's groups in plan order.
+  auto pack_groups = [](const std::vector<int>& gs) {
+    std::vector<std::vector<int>> nf, ff;   // nf: first-fit online in plan order (the greedy's count)
+    {
+      std::vector<int> fills;
+      for (int i = 0; i < (int)gs.size(); ++i) {
+        size_t k = 0;
+        while (k < fills.size() && fills[k] + gs[i] > 32) ++k;
+        if (k == fills.size()) { fills.push_back(0); nf.emplace_back(); }
+        fills[k] += gs[i];
+        nf[k].push_back(i);
+      }
+    }
+    std::vector<int> order(gs.size());
+    for (int i = 0; i < (int)gs.size(); ++i) order[i] = i;
+    std::stable_sort(order.begin(), order.end(), [&](int a, int b) { return gs[a] > gs[b]; });
+    std::vector<int> fills;
+    for (int i : order) {
+      size_t k = 0;
+      while (k < fills.size() && fills[k] + gs[i] > 32) ++k;
+      if (k == fills.size()) { fills.push_back(0); ff.emplace_back(); }
+      fills[k] += gs[i];
+      ff[k].push_back(i);
+    }
+    for (auto& bin : ff) std::sort(bin.begin(), bin.end());   // plan order within a bundle
+    return ff.size() <= nf.size() ? ff : nf;
+  };
+  auto tile_groups = [&](int64_t pa, int64_t pb) {   // group sizes of the tile's noisy sub-nets, plan order
+    std::vector<int> gs;
+    for (int64_t pn = pa; pn < pb; ++pn) {
+      const int64_t n = pl.net_lo + perm[pn];
+      const int64_t s0 = d->tree_sub_off[d->net_tree_off[n]], s1 = d->tree_sub_off[d->net_tree_off[n + 1]];
+      for (int64_t sn = s0; sn < s1; ++sn)
+        if (!gen[sn - pl.sub_lo] && !single[sn - pl.sub_lo]) gs.push_back((int)(d->sub_path_off[sn + 1] - d->sub_path_off[sn]));
+    }
+    return gs;
+  };
   // 3. bundles, tile by tile: the tile's group bundles (packing restarts at each tile), then its
   //    singleton bundles; sub-nets renumbered in that order ("kernel order").  Count per tile,
   //    prefix, then fill the tiles in parallel (each owns a contiguous bundle and sub-net range).
@@ -653,13 +707,19 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
 #pragma omp parallel for schedule(dynamic, 64)
   for (int64_t t = 0; t < ntile; ++t) {
     Pack pk;
+    int lanes = 0;   // tree lanes of the tile's multi-tree nets (a net's trees within one warp)
     for (int64_t pn = starts[t]; pn < starts[t + 1]; ++pn) {
       const int64_t n = pl.net_lo + perm[pn];
       pack_net(n, pk);
-      tmn[t + 1] += d->net_tree_off[n + 1] - d->net_tree_off[n] > 1;
+      const int nt = (int)(d->net_tree_off[n + 1] - d->net_tree_off[n]);
+      if (nt > 1) {
+        if ((lanes & 31) + nt > 32) lanes = (lanes + 31) & ~31;
+        lanes += nt;
+      }
     }
-    tbg[t] = pk.nbg;
-    tb0[t + 1] = pk.total();
+    tmn[t + 1] = (lanes + 31) & ~31;
+    tbg[t] = (int32_t)pack_groups(tile_groups(starts[t], starts[t + 1])).size();
+    tb0[t + 1] = tbg[t] + (pk.nsing + 31) / 32;
   }
   for (int64_t t = 0; t < ntile; ++t) { tb0[t + 1] += tb0[t]; tmn[t + 1] += tmn[t]; }
   pl.mnets.assign(tmn[ntile], 0);
@@ -668,6 +728,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   pl.binfo.alloc(tb0[ntile]);
   pl.pword.alloc(nslot);
   pl.slot_path.alloc(nslot + (size_t)pl.n_gpath);   // bundle slots, then the general paths' virtual slots
+  pl.ldesc.alloc(nslot);
   pl.sxy.alloc(ns);
   pl.ksub_csr.alloc(ns);
   pl.sub_first_slot.alloc(ns);
@@ -697,9 +758,18 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       T.nb = tb0[t + 1] - tb0[t];
       T.mn0 = tmn[t];
       T.nmn = tmn[t + 1] - tmn[t];
-      for (int64_t pn = starts[t], k = T.mn0; pn < starts[t + 1]; ++pn) {
-        const int64_t n = pl.net_lo + perm[pn];
-        if (d->net_tree_off[n + 1] - d->net_tree_off[n] > 1) pl.mnets[k++] = (int32_t)(pn - starts[t]);
+      {
+        int64_t k = T.mn0;
+        for (int64_t pn = starts[t]; pn < starts[t + 1]; ++pn) {
+          const int64_t n = pl.net_lo + perm[pn];
+          const int nt = (int)(d->net_tree_off[n + 1] - d->net_tree_off[n]);
+          if (nt < 2) continue;
+          if (((k - T.mn0) & 31) + nt > 32)
+            while ((k - T.mn0) & 31) pl.mnets[k++] = kNoTreeLane;
+          for (int q = 0; q < nt; ++q)
+            pl.mnets[k++] = tree_lane(ptree_off[pn] + q - T.tree0, (int)(pn - starts[t]), q == 0);
+        }
+        while (k < T.mn0 + T.nmn) pl.mnets[k++] = kNoTreeLane;
       }
       T.nbg = tbg[t];
       T.global = globs[t];
@@ -719,6 +789,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
         for (int l = 0; l < 32; ++l) {
           pl.pword[(size_t)b * 32 + l] = kPad | kSubHead;
           pl.slot_path[(size_t)b * 32 + l] = -1;
+          pl.ldesc[(size_t)b * 32 + l] = lane_desc(0, l, l, l);   // padding: a group of its own
         }
       }
       int ks = T.sub0;   // next kernel-order sub-net
@@ -731,45 +802,57 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
         pl.tiles[t] = T;
         continue;
       }
-      // group bundles; binfo.x = the tile noise offset of lane 0 (noisy candidates before it), and
-      // the tile's noisy candidates in this order form runs of consecutive noise indices
-      int fill = 32, b = T.b0 - 1, prev_tree = -1, noff = 0;
+      // group bundles.  The tile's noisy sub-nets in plan order define the tile noise offsets, whose
+      // global noise indices form runs (tile_noise fills gp by offset); the groups are then packed
+      // (pack_groups), and each slot's lane descriptor carries its noise offset, group head and end
+      // lane and its sub-net's index in the bundle (kernel order follows the bundles' slot order)
+      struct Grp { int64_t ls; int g, noff, toff; uint32_t mt; };
+      std::vector<Grp> grps;
+      std::vector<int> gsz;
       std::vector<NoiseRun> truns;
+      int noff = 0;
       for (const TT& tt : tts) {
-        const int64_t j = tt.j;
-        const int toff = tt.pt - T.tree0;
-        const uint32_t mt = tt.multi ? kMultiTree : 0u;
-        for (int64_t sn = d->tree_sub_off[j]; sn < d->tree_sub_off[j + 1]; ++sn) {
+        for (int64_t sn = d->tree_sub_off[tt.j]; sn < d->tree_sub_off[tt.j + 1]; ++sn) {
           const int64_t ls = sn - pl.sub_lo;
           if (single[ls]) continue;
-          const int64_t p0 = d->sub_path_off[sn], p1 = d->sub_path_off[sn + 1];
-          const int g = (int)(p1 - p0);
-          if (fill + g > 32) {
-            ++b;
-            pl.binfo[b] = make_int4(noff, ks, T.tree0, 0);
-            fill = 0;
-            prev_tree = -1;
-          }
+          const int g = (int)(d->sub_path_off[sn + 1] - d->sub_path_off[sn]);
           if (!truns.empty() && truns.back().nid + truns.back().len == (int32_t)nid_sub[ls]) truns.back().len += g;
           else truns.push_back({noff, g, (int32_t)nid_sub[ls], 0});
+          grps.push_back({ls, g, noff, tt.pt - T.tree0, tt.multi ? kMultiTree : 0u});
+          gsz.push_back(g);
           noff += g;
-          pl.sxy[ks] = sxy_csr[ls];
-          pl.ksub_csr[ks] = (int32_t)ls;
-          pl.sub_first_slot[ls] = (int64_t)b * 32 + fill;
+        }
+      }
+      const auto bins = pack_groups(gsz);
+      int b = T.b0 - 1, prev_tree = -1;
+      for (const auto& bin : bins) {
+        ++b;
+        pl.binfo[b] = make_int4(0, ks, T.tree0, 0);
+        int fill = 0, gi = 0;
+        prev_tree = -1;
+        for (int idx : bin) {
+          const Grp& G = grps[idx];
+          const int64_t sn = pl.sub_lo + G.ls;
+          const int64_t p0 = d->sub_path_off[sn], p1 = d->sub_path_off[sn + 1];
+          pl.sxy[ks] = sxy_csr[G.ls];
+          pl.ksub_csr[ks] = (int32_t)G.ls;
+          pl.sub_first_slot[G.ls] = (int64_t)b * 32 + fill;
           for (int64_t i = p0; i < p1; ++i) {
-            uint32_t pw = pw_path[i - pl.path_lo] | ((uint32_t)toff << kTreeShift) | mt;
+            uint32_t pw = pw_path[i - pl.path_lo] | ((uint32_t)G.toff << kTreeShift) | G.mt;
             if (i == p0) {
               pw |= kSubHead;
-              if (toff != prev_tree) pw |= kTreeHead;
+              if (G.toff != prev_tree) pw |= kTreeHead;
             }
             const size_t slot = (size_t)b * 32 + fill + (i - p0);
             pl.pword[slot] = pw;
             pl.slot_path[slot] = (int32_t)(i - pl.path_lo);
+            pl.ldesc[slot] = lane_desc(G.noff + (int)(i - p0), fill, fill + G.g - 1, gi);
           }
-          prev_tree = toff;
-          fill += g;
-          pl.binfo[b].w += g;
+          prev_tree = G.toff;
+          fill += G.g;
+          pl.binfo[b].w += G.g;
           ++ks;
+          ++gi;
         }
       }
       // singleton bundles: the lone straight sub-nets of multi-tree nets first, then those of
@@ -800,6 +883,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
           pl.sub_first_slot[ls] = (int64_t)slot;
           pl.pword[slot] = pw_path[p0 - pl.path_lo] | ((uint32_t)toff << kTreeShift) | kSubHead | mt |
                            (toff != prev_tree ? kTreeHead : 0u);
+          pl.ldesc[slot] = lane_desc(0, lane, lane, lane);
           pl.slot_path[slot] = (int32_t)(p0 - pl.path_lo);
           prev_tree = toff;
           ++lane;
@@ -864,23 +948,36 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       pl.tiles[t] = T;
     }
   }
-  // the tiles' noise runs, with the Philox quads (4 consecutive global noise indices) each spans
+  // the tiles' noise runs.  A tile with one run (the caller's order kept) draws its quads in
+  // parallel from TileDesc alone; a tile with several (re-ordered nets: about one per net) gets its
+  // runs cut at global noise indices that are multiples of 16, so each piece spans at most 4 Philox
+  // quads and one thread draws it (no search for a quad's run)
   pl.runs.clear();
   for (int64_t t = 0; t < ntile; ++t) {
     TileDesc& T = pl.tiles[t];
+    const auto& tr = tile_runs[t];
     T.run0 = (int32_t)pl.runs.size();
-    T.nrun = (int32_t)tile_runs[t].size();
-    int32_t q = 0;
-    for (NoiseRun r : tile_runs[t]) {
-      r.quad0 = q;
-      const int64_t g0 = pl.nid_base + r.nid;
-      q += (int32_t)(((g0 + r.len - 1) >> 2) - (g0 >> 2) + 1);
-      pl.runs.push_back(r);
-    }
-    T.nquad = q;
-    T.nid0 = T.nrun > 0 ? tile_runs[t][0].nid : 0;
+    T.nid0 = tr.empty() ? 0 : tr[0].nid;
     T.nnoisy = 0;
-    for (const NoiseRun& r : tile_runs[t]) T.nnoisy += r.len;
+    for (const NoiseRun& r : tr) T.nnoisy += r.len;
+    if (tr.size() <= 1) {
+      T.nrun = (int32_t)tr.size();
+      const int64_t g0 = pl.nid_base + T.nid0;
+      T.nquad = tr.empty() ? 0 : (int32_t)(((g0 + T.nnoisy - 1) >> 2) - (g0 >> 2) + 1);
+      for (const NoiseRun& r : tr) pl.runs.push_back(r);
+      continue;
+    }
+    for (const NoiseRun& r : tr) {
+      int off = r.off, nid = r.nid, len = r.len;
+      while (len > 0) {
+        const int64_t g = pl.nid_base + nid;
+        const int piece = (int)std::min<int64_t>(len, 16 - (g & 15));
+        pl.runs.push_back({off, piece, nid, 0});
+        off += piece; nid += piece; len -= piece;
+      }
+    }
+    T.nrun = (int32_t)(pl.runs.size() - T.run0);
+    T.nquad = 0;
   }
   tm.mark("bundles + event check");
   pl.nb = (int)pl.binfo.size();
@@ -930,7 +1027,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   const bool all_slow = getenv("DGR_ALL_SLOW") != nullptr;   // diagnostics: every tile on the slow path
   auto pipelined = [all_slow](const TileDesc& T) {
     return !all_slow && !T.global && T.nbg <= kTargetBundles && T.nb <= kTileBundles && T.ntree <= kPipeTrees &&
-           T.nsub <= kPipeSubs;
+           T.nsub <= kPipeSubs && T.nmn <= kTileThreads;
   };
   std::stable_partition(pl.tiles.begin(), pl.tiles.end(), pipelined);
   pl.n_pipe_tiles = 0;
@@ -1007,7 +1104,7 @@ int encode_window_maps(const std::vector<std::pair<int, int>>& shapes, const voi
 // workspace layout
 // ---------------------------------------------------------------------------------------
 struct Layout {
-  size_t tiles, net_gtree, runs, gnet, gtree, gsub, gp_seg_off, gp_tp_off, gseg, gtp, gdq, mnets, tmaps, binfo, pword, sxy, slot_path, wp, mv, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
+  size_t ldesc, tiles, net_gtree, runs, gnet, gtree, gsub, gp_seg_off, gp_tp_off, gseg, gtp, gdq, mnets, tmaps, binfo, pword, sxy, slot_path, wp, mv, pp, nto, wt, mt, vt, q, xbuf, capH, capVT, SH, SVT, dOutH, dOutVT,
       partial, lpart, loss, chosen, tree_choice, route, nsize, nucleus_tmp, DHVC, iscal, ipartial, metrics, total;
   size_t xcount;   // int64 elements in the exchange buffer
   // grid bands (SURVEY §8(e) refinement 2): rank r reduces and scans H rows [r yb, (r+1) yb) and V
@@ -1033,10 +1130,11 @@ Layout make_layout(const Plan& pl, int X, int Y, int metric_blocks) {
   L.gseg = take(8 * pl.gseg.size() + 16);
   L.gtp = take(4 * pl.gtp.size() + 16);
   L.gdq = take(8 * pl.gtree.size() + 16);
-  L.mnets = take(4 * pl.mnets.size() + 16);   // +16 B: 16-byte aligned bulk reads may run past the end
+  L.mnets = take(4 * pl.mnets.size() + 16);
   L.tmaps = take(256 * pl.tmap_shapes.size() + 256);   // 128-byte CUtensorMaps, (S_H, S_V) per window shape
   L.binfo = take(sizeof(int4) * pl.nb);
   L.pword = take(4 * bslots);
+  L.ldesc = take(4 * bslots);
   L.sxy = take(8 * ns + 16);
   L.slot_path = take(4 * slots);
   L.wp = take(4 * slots);
@@ -1353,7 +1451,7 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   P.tree_base = pl.tree_lo;
   P.nid_base = pl.nid_base;
   P.seed = desc->seed;
-  P.mnets = (const int32_t*)(ws + L.mnets);
+  P.mnets = (const uint32_t*)(ws + L.mnets);
   P.ngen = (int32_t)pl.gnet.size();
   P.ngen_blocks = (P.ngen + kGenWarps - 1) / kGenWarps;
   P.ngsub = (int32_t)pl.gsub.size();
@@ -1372,6 +1470,7 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   }
   P.binfo = (const int4*)(ws + L.binfo);
   P.pword = (const uint32_t*)(ws + L.pword);
+  P.ldesc = (const uint32_t*)(ws + L.ldesc);
   P.sxy = (const short4*)(ws + L.sxy);
   P.slot_path = (const int32_t*)(ws + L.slot_path);
   P.wp = (float*)(ws + L.wp); P.mv = (float2*)(ws + L.mv);
@@ -1447,7 +1546,8 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
       {L.gseg, 8 * pl.gseg.size(), pl.gseg.data()},
       {L.gtp, 4 * pl.gtp.size(), pl.gtp.data()},
       {L.net_gtree, 4 * pl.net_gtree.size(), pl.net_gtree.data()},
-      {L.runs, sizeof(NoiseRun) * pl.runs.size(), pl.runs.data()}};
+      {L.runs, sizeof(NoiseRun) * pl.runs.size(), pl.runs.data()},
+      {L.ldesc, 4 * (size_t)pl.nb * 32, pl.ldesc.data()}};   // (regions 5, 6, 9, 10, 12, 13 are filled in place below)
   std::vector<size_t> at(regs.size() + 1, 0);
   for (size_t i = 0; i < regs.size(); ++i) at[i + 1] = at[i] + ((regs[i].bytes + 255) & ~(size_t)255);
   std::lock_guard<std::mutex> lock(g_pin.m);

@@ -90,7 +90,7 @@ struct TileDesc {
   int32_t wx0, wy0, ww, wh;  // window (cells; even origin and extents), unused for global tiles
   int32_t global, nbg;     // nbg: group bundles (the first nbg of the tile; the rest are singleton bundles)
   int32_t sub0, nsub;      // local sub-nets (kernel order within the tile)
-  int32_t mn0, nmn;        // the tile's nets with >= 2 trees: mnets[mn0 .. mn0 + nmn) (net offsets in the tile)
+  int32_t mn0, nmn;        // the trees of the tile's nets with >= 2 trees: mnets[mn0 .. mn0 + nmn) (tree_lane)
   int32_t tmap;            // pipelined tiles: index of the (S_H, S_V) tensor-map pair of the window's shape
                            // (one 2-D TMA copy per field), -1: the window comes by cp.async
   int32_t run0, nrun;      // noise runs[run0 .. run0 + nrun): the tile's noisy candidates in bundle order as
@@ -101,7 +101,7 @@ struct TileDesc {
 // A run of a tile's noisy candidates (group-bundle lanes in order, padding skipped) whose global noise
 // indices are consecutive: tile noise offsets [off, off + len) draw noise indices nid_base + nid ..
 struct NoiseRun {
-  int32_t off, len, nid, quad0;   // quad0: Philox quads of the tile's earlier runs
+  int32_t off, len, nid, unused;   // multi-run tiles: pieces within one aligned block of 16 noise indices
 };
 
 // "General" nets (row f4'): nets with a sub-net whose candidates are not all Z(o, m)
@@ -117,6 +117,21 @@ struct GSub {
   int32_t gp;              // general path index of the first candidate (segment / turning-point lists)
   int32_t pad[2];
 };
+
+// Lane descriptor of a bundle slot (plan-time decode of the bundle's group structure): the lane's
+// tile noise offset (bits 0-10), its group's head and end lane (11-15, 16-20) and the index of its
+// sub-net within the bundle (21-25).  Padding and singleton lanes are groups of their own.
+inline __host__ __device__ uint32_t lane_desc(int noff, int head, int end, int sub) {
+  return (uint32_t)noff | ((uint32_t)head << 11) | ((uint32_t)end << 16) | ((uint32_t)sub << 21);
+}
+
+// A tree lane of a tile's net level: the tree (relative to the tile's first tree, bits 0-9), its net
+// (offset in the tile, bits 10-20) and whether it is the net's first tree (bit 31); a net's trees
+// occupy consecutive lanes of one warp.  kNoTreeLane pads.
+constexpr uint32_t kNoTreeLane = 0xFFFFFFFFu;
+inline __host__ __device__ uint32_t tree_lane(int tree_rel, int net_rel, bool head) {
+  return (uint32_t)tree_rel | ((uint32_t)net_rel << 10) | (head ? 0x80000000u : 0u);
+}
 
 // Shared-memory offset (elements) of a pipelined tile's V field: the H field rounded up to 128 bytes
 // of doubles (TMA destinations are 128-byte aligned).
@@ -146,13 +161,14 @@ struct KParams {
   const TileDesc* tiles_slow;
   const int4* binfo;
   const uint32_t* pword;
+  const uint32_t* ldesc;    // lane descriptors (lane_desc), per bundle slot
   const short4* sxy;        // kernel order
   const int32_t* slot_path; // local CSR path of each slot (-1 for padding); induction only
   float* wp;
   float2* mv;               // Adam moments (m, v) of each slot, interleaved (one 8-byte access)
   float* pp;                // p_i of the last forward (the reverse of that iteration reads it)
   const int32_t* net_tree_off;    // local, n_nets_l + 1
-  const int32_t* mnets;     // per tile: offsets (in the tile) of its nets with >= 2 trees
+  const uint32_t* mnets;    // per tile: the trees of its nets with >= 2 trees, a lane each (tree_lane)
   const int32_t* net_gtree; // per (plan-ordered) local net: local CSR index of its first tree (tree noise key, Q7)
   int32_t perm_id;          // the plan keeps the caller's net order (plan-ordered trees = CSR trees)
   const NoiseRun* runs;     // per tile: noise runs (TileDesc run0 / nrun)

@@ -93,9 +93,11 @@ __device__ __forceinline__ float gumbel(uint64_t seed, uint64_t idx, uint32_t k,
   return gumbel_word(s == 0 ? r.x : (s == 1 ? r.y : (s == 2 ? r.z : r.w)));
 }
 
-// Gumbel noise (stream 0) of a tile's noisy candidates into gp[tile noise offset]: the tile's runs of
-// consecutive global noise indices (NoiseRun), one Philox call per aligned quad of indices, spread
-// over the CTA's threads (a quad's run found by binary search over the runs' quad offsets).
+// Gumbel noise (stream 0) of a tile's noisy candidates: the raw Philox word of each into gp[tile noise
+// offset] (each lane turns its own word into g = -ln(-ln u) where it uses it: no conversion is spent
+// on the words of a quad that no candidate draws); the tile's runs of
+// consecutive global noise indices (NoiseRun), one Philox call per aligned quad of indices (one run:
+// the quads spread over the CTA's threads; several: a thread per run piece of at most 4 quads).
 template <int NT>
 __device__ __forceinline__ void tile_noise(const KParams& P, const TileDesc& T, uint32_t k, float* gp) {
   if (T.nrun == 1) {   // one run (nets in the caller's order): its quads spread over the threads
@@ -107,29 +109,25 @@ __device__ __forceinline__ void tile_noise(const KParams& P, const TileDesc& T, 
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
         const int64_t o = c * 4 + i - g0;
-        if (o >= 0 && o < T.nnoisy) gp[o] = gumbel_word(wd[i]);
+        if (o >= 0 && o < T.nnoisy) gp[o] = __uint_as_float(wd[i]);
       }
     }
     return;
   }
-  // several runs (nets re-ordered by the plan): the quads spread over the threads, a quad's run found
-  // by binary search over the runs' quad offsets (a thread per run would serialise a large net's quads)
-  const int4* R = reinterpret_cast<const int4*>(P.runs) + T.run0;   // {off, len, nid, quad0}
-  for (int q = threadIdx.x; q < T.nquad; q += NT) {
-    int lo = 0, hi = T.nrun - 1;
-    while (lo < hi) {
-      const int mid = (lo + hi + 1) >> 1;
-      if (__ldg(&R[mid].w) <= q) lo = mid; else hi = mid - 1;
-    }
-    const int4 r = __ldg(&R[lo]);
+  // several runs (nets re-ordered by the plan), cut into pieces within one aligned block of 16 noise
+  // indices (at most 4 Philox quads each): a thread per piece
+  const int4* R = reinterpret_cast<const int4*>(P.runs) + T.run0;   // {off, len, nid, -}
+  for (int ri = threadIdx.x; ri < T.nrun; ri += NT) {
+    const int4 r = __ldg(&R[ri]);
     const int64_t g0 = P.nid_base + r.z;
-    const int64_t c = (g0 >> 2) + (q - r.w);
-    const uint4 w = philox_rk(make_uint4((uint32_t)c, (uint32_t)(c >> 32), k, 0u), P.rk);
-    const uint32_t wd[4] = {w.x, w.y, w.z, w.w};
+    for (int64_t c = g0 >> 2; c <= (g0 + r.y - 1) >> 2; ++c) {
+      const uint4 w = philox_rk(make_uint4((uint32_t)c, (uint32_t)(c >> 32), k, 0u), P.rk);
+      const uint32_t wd[4] = {w.x, w.y, w.z, w.w};
 #pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const int64_t o = c * 4 + i - g0;
-      if (o >= 0 && o < r.y) gp[r.x + o] = gumbel_word(wd[i]);
+      for (int i = 0; i < 4; ++i) {
+        const int64_t o = c * 4 + i - g0;
+        if (o >= 0 && o < r.y) gp[r.x + o] = __uint_as_float(wd[i]);
+      }
     }
   }
 }
@@ -270,6 +268,7 @@ __device__ __forceinline__ void flush_window_t(const KParams& P, const StepArgs&
     const int2 h = evH[i], v = evV[i], d = evD2[i];
     const int dl = cx > 0 ? evD[2 * i - 1] : 0, dr = cx + 2 < ww ? evD[2 * i + 2] : 0;
     const int2 du = r > 0 ? evD2[i - hw] : make_int2(0, 0), dn = r + 1 < wh ? evD2[i + hw] : make_int2(0, 0);
+    if (((h.x | h.y | v.x | v.y | d.x | d.y | dl | dr) | (du.x | du.y | dn.x | dn.y)) == 0) continue;   // nothing to flush
     // turning-point counts are >= 0 and < 2^31 per cell, so these differences fit int32
     int fh0 = d.y - dl, fh1 = dr - d.x, fv0 = dn.x - du.x, fv1 = dn.y - du.y;
     etp += (long long)d.x + d.y;
@@ -440,6 +439,20 @@ __device__ __forceinline__ void lane_from(int4 bi, uint32_t pw, const KParams& P
 // p_i = exp(z_i - m) / sum_k exp(z_k - m) for any shift m (softmax shift invariance): m = the group
 // head's z, unless some lane of the warp exceeds its head by more than 64 (exp overflow risk), then
 // the exact group maximum.  The head's own term is exp(0) = 1, so the sum is >= 1.
+// Lane view of a group-bundle slot from its plan-time lane descriptor (no ballots): head / end lane
+// of its group, its sub-net (bundle's first + index), tree; the fields a group lane needs.
+__device__ __forceinline__ void lane_from_desc(int4 bi, uint32_t pw, uint32_t ld, Lane& L) {
+  L.lane = threadIdx.x & 31;
+  L.pw = pw;
+  L.shape = pw & 7u;
+  L.valid = L.shape != kPad;
+  L.head = (int)((ld >> 11) & 31u);
+  L.end = (int)((ld >> 16) & 31u);
+  L.sub = bi.y + (int)((ld >> 21) & 31u);
+  L.tree = bi.z + (int)((pw >> kTreeShift) & kTreeMask);
+  L.single = false;
+}
+
 __device__ __forceinline__ float softmax_from_noise(const Lane& L, float w, float g, float inv_t) {
   const float z = L.valid ? (w + g) * inv_t : -INFINITY;
   float m = __shfl_sync(kFull, z, L.head);
@@ -567,18 +580,16 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
   int4 bi1 = make_int4(0, 0, 0, 0);
   uint32_t pw1 = kPad | kSubHead;
   if (bw0 + 1 < bw1) { bi1 = __ldg(&P.binfo[bw0 + 1]); pw1 = __ldg(&P.pword[slot + 32]); }
-  int boff = bfirst.x, boffn = 0;   // the bundles' tile noise offsets
   for (int b = bw0; b < bw1; ++b) {
     Lane Ln = L;
     short4 en = e;
     if (b + 1 < bw1) {
-      boffn = bi1.x;
       lane_from(bi1, pw1, P, Ln);
       if (Ln.valid) en = __ldg(&P.sxy[Ln.sub]);
       if (b + 2 < bw1) { bi1 = __ldg(&P.binfo[b + 2]); pw1 = __ldg(&P.pword[slot + 64]); }
     }
     const float w = have_w ? wst[(b - T.b0) * 32 + lane] : P.wp[slot];
-    const float g = (L.valid && !L.single) ? gt[boff + L.lane] : 0.f;   // the tile's noise, by offset
+    const float g = (L.valid && !L.single) ? gumbel_word(__float_as_uint(gt[__ldg(&P.ldesc[slot]) & 0x7FFu])) : 0.f;
     const float p = softmax_from_noise(L, w, g, A.inv_t);
     P.pp[slot] = p;
     const float q = L.valid ? q_s[L.tree - T.tree0] : 0.f;
@@ -646,7 +657,7 @@ __device__ __forceinline__ void forward_warp(const KParams& P, const StepArgs& A
       red_shared_add(ev_base + 4u * W.v(xb, yb), bv);
       red_shared_add(ev_base + 4u * W.d(xb, yb), bd);
     }
-    L = Ln; e = en; boff = boffn;
+    L = Ln; e = en;
     slot += 32;
   }
 
@@ -783,7 +794,7 @@ constexpr int kPNetMax = kPipeTrees + 8;
 // info, sub-net endpoints, net->tree offsets, the multi-tree net list, tree logits and q, and the S
 // window.  Adam moments and the stored p of the paths, and m, v of the trees, are read / written
 // directly (each warp its bundle's 128-byte rows), so the stage fits 5 CTAs per SM.
-constexpr int kPMnMax = kPipeTrees / 2 + 4;                 // nets with >= 2 trees per tile (+ slack)
+constexpr int kPMnMax = 0;   // (the net level's tree lanes are read straight from mnets, not staged)
 struct StageLayout {
   static constexpr size_t pw = 0;
   static constexpr size_t w = pw + 4 * 32 * kTileBundles;
@@ -916,14 +927,13 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
   Stage S(st);
   int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
-  const int mn_lo = T.mn0 & ~3, mn_hi = (T.mn0 + T.nmn + 3) & ~3;
   const uint32_t slot_bytes = (uint32_t)T.nb * 128u, gslot_bytes = (uint32_t)T.nbg * 128u;
   const bool sw = REV && window && !(KO(32));   // knock-out 32: no S window (timing only)
   const uint32_t nrow = sw ? (uint32_t)T.wh : 0u, ncol = sw ? (uint32_t)T.ww : 0u;
   // REV && !window && tmap >= 0: the S window by two 2-D tensor copies (H field, V field)
   const bool tw = REV && !window && T.tmap >= 0 && !(KO(32));
   const uint32_t bytes = slot_bytes + gslot_bytes + 16u * T.nb + 8u * (s_hi - s_lo) + 4u * (n_hi - n_lo) +
-                         4u * (mn_hi - mn_lo) + 8u * (t_hi - t_lo) + 8u * (nrow * T.ww + ncol * T.wh) +
+                         8u * (t_hi - t_lo) + 8u * (nrow * T.ww + ncol * T.wh) +
                          (tw ? 16u * (uint32_t)(T.ww * T.wh) : 0u);
   if (lane == 0) mbar_expect_tx(bar, bytes);
   __syncwarp();
@@ -944,7 +954,7 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
         case 2: bulk_g2s_stream(S.bi, P.binfo + T.b0, 16u * T.nb, bar, pol); break;
         case 3: bulk_g2s_stream(S.sxy, P.sxy + s_lo, 8u * (s_hi - s_lo), bar, pol); break;
         case 4: bulk_g2s_stream(S.nto, P.net_tree_off + n_lo, 4u * (n_hi - n_lo), bar, pol); break;
-        case 5: if (mn_hi > mn_lo) bulk_g2s(S.mn, P.mnets + mn_lo, 4u * (mn_hi - mn_lo), bar); break;
+        case 5: break;
         case 6: bulk_g2s(S.wt, P.wt + t_lo, 4u * (t_hi - t_lo), bar); break;
         default: bulk_g2s(S.q, P.q + t_lo, 4u * (t_hi - t_lo), bar); break;   // also a lone tree's q = 1
       }
@@ -977,7 +987,6 @@ __device__ __forceinline__ void lsu_tile_loads(const KParams& P, const TileDesc&
   Stage S(st);
   int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
-  const int mn_lo = T.mn0 & ~3, mn_hi = (T.mn0 + T.nmn + 3) & ~3;
   const size_t s0 = (size_t)T.b0 * 32;
   if (arrays) switch (warp & 7) {
     case 0: cp_copy(S.pw, P.pword + s0, (uint32_t)T.nb * 128u, lane); break;
@@ -985,7 +994,7 @@ __device__ __forceinline__ void lsu_tile_loads(const KParams& P, const TileDesc&
     case 2: cp_copy(S.bi, P.binfo + T.b0, 16u * T.nb, lane); break;
     case 3: cp_copy(S.sxy, P.sxy + s_lo, 8u * (s_hi - s_lo), lane); break;
     case 4: cp_copy(S.nto, P.net_tree_off + n_lo, 4u * (n_hi - n_lo), lane); break;
-    case 5: cp_copy(S.mn, P.mnets + mn_lo, 4u * (mn_hi - mn_lo), lane); break;
+    case 5: break;
     case 6: cp_copy(S.wt, P.wt + t_lo, 4u * (t_hi - t_lo), lane); break;
     default: cp_copy(S.q, P.q + t_lo, 4u * (t_hi - t_lo), lane); break;
   }
@@ -1039,14 +1048,13 @@ __device__ __forceinline__ void stamp(const KParams& P, int tile, int k) {
 constexpr size_t kGpOffset = 3 * 4 * (kWinMax + kWinPad);   // tile path noise, after the event window in St.S
 template <bool REV, bool FWD, int NT>
 __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A, const TileDesc& T, Stage St,
-                                             int* ev_s, float* gp, int* dq3) {
+                                             int* ev_s, float* gp, int* dq3, uint32_t ld_first, uint32_t mte) {
   // dq3[0..3 ntree) arrives zeroed (the caller clears it before its first barrier)
   constexpr int NW = NT / 32;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int X = P.X, Y = P.Y;
   int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
-  const int mn_lo = T.mn0 & ~3;
   const uint64_t pol = policy_stream();   // L2 evict-first for the streamed slot state
   const int hv = win_hv(T.ww, T.wh);   // V field at hv (128-byte aligned)
   const Win W{T.wx0, T.wy0, T.ww, T.wh, hv};
@@ -1056,12 +1064,16 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
 
   // ---------------- reverse of iteration k ----------------
   if (REV && !(KO(64))) {   // dq3 was zeroed before the stage arrived
+    const uint32_t* LD = P.ldesc + (size_t)T.b0 * 32 + lane;   // lane descriptors, prefetched a bundle ahead
+    uint32_t ldn = ld_first;   // the first one was loaded before the stage wait
     for (int lb = warp; lb < T.nb; lb += NW) {
       const int4 bi = St.bi[lb];
       const uint32_t pw = St.pw[lb * 32 + lane];
+      const uint32_t ld = ldn;
+      if (lb + NW < nbg) ldn = __ldg(LD + (lb + NW) * 32);
       if (lb < nbg) {
         Lane L;
-        lane_from(bi, pw, P, L);
+        lane_from_desc(bi, pw, ld, L);
         const int sl = lb * 32 + lane;
         const size_t gsl = (size_t)T.b0 * 32 + sl;
         float w = St.w[sl];
@@ -1117,27 +1129,41 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   }
   stamp(P, (int)blockIdx.x - P.ntiles_slow - P.ngen_blocks, 2);
 
+  // the forward's first lane descriptor, loaded before the net level (its latency hides there)
+  const uint32_t ld_fwd = (FWD && warp < nbg) ? __ldg(P.ldesc + (size_t)T.b0 * 32 + warp * 32 + lane) : 0u;
   // ---------------- net level (one thread per net), event window cleared alongside ----------------
   if (FWD) {
     int4* z = reinterpret_cast<int4*>(ev_s);   // the S window is free after the reverse
     for (int i = tid; i < (3 * hv) / 4; i += NT) z[i] = make_int4(0, 0, 0, 0);
   }
-  // the tile's nets with >= 2 trees (a lone tree has q = 1 and du = 0 always: its logit and Adam
-  // state never change, and its q = 1 arrives with the stage)
-  for (int i = tid; i < ((KO(128)) ? 0 : T.nmn); i += NT) {
-    const int n = St.mn[T.mn0 + i - mn_lo];
-    const int a = St.nto[T.net0 + n - n_lo] - t_lo, b = St.nto[T.net0 + n + 1 - n_lo] - t_lo;   // stage indices
+  // the tile's nets with >= 2 trees, a lane per tree (a lone tree has q = 1 and du = 0 always: its
+  // logit and Adam state never change, and its q = 1 arrives with the stage).  A net's trees are
+  // consecutive lanes of one warp; its sums run over them in tree order (shuffles), the arithmetic of
+  // the per-net loops of the slow path, so a net computes the same whichever tile it lands in.
+  if (tid < ((KO(128)) ? 0 : T.nmn)) {   // whole warps (nmn is a multiple of 32)
+    const uint32_t e = mte;
+    const bool tv = e != kNoTreeLane;
+    const int jr = (int)(e & 1023u);                    // tree, relative to the tile's first
+    const int j = T.tree0 + jr - t_lo;                  // stage index
+    const int nrel = (int)((e >> 10) & 2047u);           // net, relative to the tile's first
+    const uint32_t hm = __ballot_sync(kFull, !tv || (e >> 31));
+    const uint32_t le = kFull >> (31 - lane);
+    const int head = 31 - __clz(hm & le);
+    const uint32_t rest = hm & ~le;
+    const int end = rest ? (__ffs(rest) - 2) : 31;
     if (REV) {
       // du_j = (q_j/t)(dq_j - sum_l q_l dq_l / sum_l q_l); Adam on w_tree (iteration k)
+      const double ql = tv ? (double)St.q[j] : 0.0;
+      const double qd = tv ? ql * dq_get(dq3, jr) : 0.0;
       double sq = 0.0, sw = 0.0;
-      for (int l = a; l < b; ++l) {
-        const double ql = (double)St.q[l];
-        sq += ql * dq_get(dq3, l + t_lo - T.tree0);
-        sw += ql;
+      for (int k = 0; __any_sync(kFull, head + k <= end); ++k) {
+        const int src = min(head + k, 31);
+        const double a = __shfl_sync(kFull, qd, src), b = __shfl_sync(kFull, ql, src);
+        if (head + k <= end) { sq += a; sw += b; }
       }
       sq /= sw;
-      for (int j = a; j < b; ++j) {
-        const double du = (double)St.q[j] * (double)A.inv_t * (dq_get(dq3, j + t_lo - T.tree0) - sq);
+      if (tv) {
+        const double du = (double)St.q[j] * (double)A.inv_t * (dq_get(dq3, jr) - sq);
         const int jg = j + t_lo;
         float w = St.wt[j], m = P.mt[jg], v = P.vt[jg];
         adam_update(w, m, v, (float)du, A);
@@ -1146,26 +1172,29 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
       }
     }
     if (FWD) {
-      // q_j = softmax over the net's trees of (w_j + g_j)/t, iteration k_next (noise stream 1)
-      float zmax = -INFINITY;
-      int64_t cq = -1;   // one Philox call per aligned quad of tree indices
-      uint4 r = make_uint4(0u, 0u, 0u, 0u);
-      for (int j = a; j < b; ++j) {
-        // global tree id (plan order = CSR order unless the plan re-ordered the nets)
-        const int64_t gj = P.tree_base + (P.perm_id ? t_lo + j : __ldg(&P.net_gtree[T.net0 + n]) + (j - a));
-        if ((gj >> 2) != cq) {
-          cq = gj >> 2;
-          r = philox_rk(make_uint4((uint32_t)cq, (uint32_t)(cq >> 32), (uint32_t)A.k_next, 1u), P.rk);
-        }
+      // q_j = softmax over the net's trees of (w_j + g_j)/t, iteration k_next (noise stream 1, keyed on
+      // the global tree id: plan order = CSR order, else from net_gtree)
+      const int jh = __shfl_sync(kFull, j, head);
+      float z = -INFINITY;
+      if (tv) {
+        const int64_t gj = P.tree_base + (P.perm_id ? (int64_t)(t_lo + j) : (int64_t)__ldg(&P.net_gtree[T.net0 + nrel]) + (j - jh));
+        const uint4 r = philox_rk(make_uint4((uint32_t)(gj >> 2), (uint32_t)(gj >> 34), (uint32_t)A.k_next, 1u), P.rk);
         const uint32_t wd = (gj & 3) == 0 ? r.x : (gj & 3) == 1 ? r.y : (gj & 3) == 2 ? r.z : r.w;
-        const float zj = (St.wt[j] + gumbel_word(wd)) * A.inv_t;
-        St.q[j] = zj;
-        zmax = fmaxf(zmax, zj);
+        z = (St.wt[j] + gumbel_word(wd)) * A.inv_t;
       }
+      float zmax = -INFINITY;
+      for (int k = 0; __any_sync(kFull, head + k <= end); ++k) {
+        const float a = __shfl_sync(kFull, z, min(head + k, 31));
+        if (head + k <= end) zmax = fmaxf(zmax, a);
+      }
+      const float ez = tv ? FEXP(z - zmax) : 0.f;
       float sum = 0.f;
-      for (int j = a; j < b; ++j) sum += FEXP(St.q[j] - zmax);
-      for (int j = a; j < b; ++j) {
-        const float q = FEXP(St.q[j] - zmax) / sum;
+      for (int k = 0; __any_sync(kFull, head + k <= end); ++k) {
+        const float a = __shfl_sync(kFull, ez, min(head + k, 31));
+        if (head + k <= end) sum += a;
+      }
+      if (tv) {
+        const float q = ez / sum;
         St.q[j] = q;
         P.q[j + t_lo] = q;
       }
@@ -1178,15 +1207,19 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   // ---------------- forward of iteration k_next ----------------
   if (FWD) {
     const uint32_t ev_base = smem_u32(ev_s);
+    const uint32_t* LD = P.ldesc + (size_t)T.b0 * 32 + lane;   // lane descriptors, prefetched a bundle ahead
+    uint32_t ldn = ld_fwd;
     for (int lb = warp; lb < T.nb; lb += NW) {
       const int4 bi = St.bi[lb];
       const uint32_t pw = St.pw[lb * 32 + lane];
+      const uint32_t ld = ldn;
+      if (lb + NW < nbg) ldn = __ldg(LD + (lb + NW) * 32);
       if (lb < nbg) {
         Lane L;
-        lane_from(bi, pw, P, L);
+        lane_from_desc(bi, pw, ld, L);
         const int sl = lb * 32 + lane;
         const float w = St.w[sl];
-        const float g = L.valid ? gp[bi.x + lane] : 0.f;   // bi.x: the bundle's tile noise offset
+        const float g = L.valid ? gumbel_word(__float_as_uint(gp[ld & 0x7FFu])) : 0.f;   // the lane's word, by its tile noise offset
         const float p = softmax_from_noise(L, w, g, A.inv_t);
         st_stream(&P.pp[(size_t)T.b0 * 32 + sl], p, pol);
         const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
@@ -1209,14 +1242,22 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
           const int fP = o ? hv : 0, fS = o ? 0 : hv;   // fields of the primary / secondary lines
           // each segment: +v at its lower end, -v at its upper end (nothing if zero-length)
           const int v1 = cm0 != cp0 ? vq : 0, v2 = cm1 != cm0 ? vq : 0, v3 = cp1 != cm1 ? vq : 0;
+#if !defined(DGR_EXP_SKIP_EVENTS)   // (timing experiments only: results invalid when defined)
+#if !defined(DGR_EXP_SKIP_CORNERS)
           red_shared_add(ev_base + 4u * (fP + min(cp0, cm0)), v1);
+#endif
           red_shared_add(ev_base + 4u * (fP + max(cp0, cm0)), -v1);
           red_shared_add(ev_base + 4u * (fS + min(cm0, cm1)), v2);
           red_shared_add(ev_base + 4u * (fS + max(cm0, cm1)), -v2);
           red_shared_add(ev_base + 4u * (fP + min(cm1, cp1)), v3);
+#if !defined(DGR_EXP_SKIP_CORNERS)
           red_shared_add(ev_base + 4u * (fP + max(cm1, cp1)), -v3);
+#endif
           red_shared_add(ev_base + 4u * (hv2 + cm0), ntp >= 1 ? vq : 0);   // turning points
           red_shared_add(ev_base + 4u * (hv2 + cm1), ntp == 2 ? vq : 0);
+#else
+          if (vq == 123456789) red_shared_add(ev_base + 4u * (fP + cp0 + cm0 + cm1 + cp1 + fS + v1 + v2 + v3), 1);
+#endif
         }
       } else {
         // singleton bundle: pi = q; +pi where the segment starts, -pi where it ends
@@ -1513,6 +1554,12 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   for (int i = threadIdx.x; i < 3 * kPipeTrees; i += kBThreads) dq3[i] = 0;
+  // the reverse's first lane descriptor (plan data: no dependence on the previous kernels), loaded
+  // now so that its latency hides behind the stage
+  const int wid = threadIdx.x >> 5;
+  const uint32_t ld_first = (REV && wid < T.nbg) ? __ldg(P.ldesc + (size_t)T.b0 * 32 + wid * 32 + (threadIdx.x & 31)) : 0u;
+  // this thread's tree lane of the net level (plan data), likewise
+  const uint32_t mte = (int)threadIdx.x < T.nmn ? __ldg(P.mnets + T.mn0 + threadIdx.x) : kNoTreeLane;
   __syncthreads();
   griddep_wait();   // S, logits, q and the event grids come from the previous kernels
 #if DGR_LSU_STAGE == 2
@@ -1540,7 +1587,7 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
   mbar_wait(bar, 0u);
 #endif
   stamp(P, tix, 1);
-  if (!(KO(16))) process_tile<REV, FWD, kBThreads>(P, A, T, St, ev_s, gp, dq3);
+  if (!(KO(16))) process_tile<REV, FWD, kBThreads>(P, A, T, St, ev_s, gp, dq3, ld_first, mte);
   if (KO(256)) __syncthreads();   // (diagnostics: the flush of every warp is done)
   stamp(P, tix, 5);
   if (threadIdx.x == 0) bulk_wait_read();   // the stage must outlive the bulk stores' reads

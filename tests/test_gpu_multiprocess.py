@@ -25,7 +25,8 @@ def _torchrun(nproc, *args, timeout=900):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
            "--master-addr", "127.0.0.1", f"--master-port={_port()}", *args]
     r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=timeout)
-    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
+    ranks = "\n".join(ln for ln in (r.stdout + r.stderr).splitlines() if "[rank" in ln)
+    assert r.returncode == 0, ranks[-4000:] + r.stderr[-2000:]
     lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
     assert len(lines) == 1, r.stdout[-3000:] + r.stderr[-3000:]
     return json.loads(lines[0])

@@ -57,8 +57,7 @@ def main():
         ok["tree_choice"] = bool(np.array_equal(tc, ref["tree_choice"]))
         ok["route"] = bool(np.array_equal(rt, ref["route"]))
         print(json.dumps({"ok": all(ok.values()), "checks": ok, "world": world, "forest": name}), flush=True)
-    tdist.barrier()
-    tdist.destroy_process_group()
+    tdist.barrier()   # rank 0 has reported; process exit closes the gloo group
 
 
 if __name__ == "__main__":
