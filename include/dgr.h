@@ -90,7 +90,10 @@ typedef struct {
 typedef int (*dgr_allreduce_fn)(void* user, void* buf, int64_t count, int32_t dtype, void* cuda_stream);
 
 /* Multi-GPU: one process per GPU.  rank 0 calls dgr_nccl_unique_id and broadcasts the 128
- * bytes (e.g. over torch.distributed); every rank passes them here. NULL or world == 1: single GPU.
+ * bytes (e.g. over torch.distributed); every rank passes them here. NULL, or world == 1 with
+ * neither an id nor a callback: single GPU, no exchange.  world == 1 WITH an NCCL id (or a
+ * callback) runs the band exchange of world > 1 through a one-rank communicator (or the callback):
+ * the same results, the NCCL path exercised on one GPU (tests).
  * With `allreduce` non-NULL the ranks exchange through it instead (nccl_unique_id unused). */
 typedef struct {
   int32_t rank, world;
@@ -165,10 +168,12 @@ int dgr_step(struct dgr_handle* h, int32_t iters, float temperature, float lr, c
              dgr_loss* last);
 
 /* dgr_step without host synchronisation (the same iterations of PAPER.md §4.3-4.4, P:803-847,
- * P:913-914), then a stream-ordered copy of the
+ * P:913-914), then a stream-ordered write of the
  * loss of the last forward (4 doubles: total, wl, via, overflow, as dgr_loss) into loss_out
- * (host memory, caller-owned; pinned memory keeps the call asynchronous).  loss_out is valid
- * after dgr_sync or any synchronising call on the handle.  NULL loss_out: DGR_EINVAL. */
+ * (host memory, caller-owned): pinned (page-locked, device-accessible) memory is written by the
+ * loss kernel itself, with no copy on the stream; pageable memory gets a cudaMemcpyAsync after it.
+ * loss_out is valid after dgr_sync or any synchronising call on the handle.  NULL loss_out:
+ * DGR_EINVAL. */
 int dgr_step_async(struct dgr_handle* h, int32_t iters, float temperature, float lr, const dgr_weights* w,
                    double* loss_out);
 

@@ -597,6 +597,16 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   // run in parallel; each boundary costs at most one extra tile.
   constexpr int64_t kChunkNets = 1 << 15;
   const int64_t nchunk = std::max<int64_t>(1, (nn + kChunkNets - 1) / kChunkNets);
+  // group bundles per tile: kTargetBundles, fewer for a forest too small to fill one wave of
+  // resident tiles (148 SMs x 5 CTAs): there a tile's lifetime IS the kernel's time, and smaller
+  // tiles cut it.  DGR_TILE_BUNDLES overrides (experiments).
+  int tgt = kTargetBundles;
+  {
+    const int64_t est = (pl.path_hi - pl.path_lo + 31) / 32;   // ~ bundles of the rank's forest
+    const int64_t slots = 148 * 5;
+    if (est < (int64_t)kTargetBundles * slots) tgt = (int)std::max<int64_t>(4, (est + slots - 1) / slots);
+    if (const char* e = getenv("DGR_TILE_BUNDLES")) tgt = std::min(kTargetBundles, std::max(1, atoi(e)));
+  }
   std::vector<std::vector<int64_t>> cstarts(nchunk);
   std::vector<std::vector<char>> cglobs(nchunk);
   std::vector<int64_t> cbad(nchunk, -1);
@@ -623,7 +633,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
         const int ux0 = std::min(cur.bx0, bx0), uy0 = std::min(cur.by0, by0);
         const int ux1 = std::max(cur.bx1, bx1), uy1 = std::max(cur.by1, by1);
         pack_net(n, pk2);
-        fits = aligned_area(ux0, uy0, ux1, uy1) <= kWinMax && pk2.nbg <= kTargetBundles && pk2.total() <= kTileBundles &&
+        fits = aligned_area(ux0, uy0, ux1, uy1) <= kWinMax && pk2.nbg <= tgt && pk2.total() <= tgt + (kTileBundles - kTargetBundles) &&
                cur.ntree + ntree <= kPipeTrees && cur.nsub + nsub <= kPipeSubs;
         if (fits) { cur.bx0 = ux0; cur.by0 = uy0; cur.bx1 = ux1; cur.by1 = uy1; }
       } else if (cur.open && cur.global && big) {
@@ -1193,6 +1203,9 @@ struct dgr_handle {
   KParams P{};
   cudaStream_t stream = nullptr;
   int rank = 0, world = 1;
+  // the band exchange runs (world > 1, or a one-rank dgr_dist with an NCCL id or a callback: the
+  // exchange path exercised on one GPU)
+  bool xchg = false;
   ncclComm_t comm = nullptr;
   dgr_allreduce_fn ar_fn = nullptr;   // caller-supplied exchange instead of NCCL (dgr_dist.allreduce)
   void* ar_user = nullptr;
@@ -1281,7 +1294,7 @@ static ncclDataType_t nccl_type(int dt) {
 }
 static size_t dt_bytes(int dt) { return (dt == kI32 || dt == kF32) ? 4 : 8; }
 static int live_comm(dgr_handle* h) {
-  if (h->world > 1 && !h->ar_fn && !h->comm) return fail(DGR_ESTATE, "the NCCL communicator was aborted after an error or timeout");
+  if (h->xchg && !h->ar_fn && !h->comm) return fail(DGR_ESTATE, "the NCCL communicator was aborted after an error or timeout");
   return DGR_OK;
 }
 // in-place sum over the ranks
@@ -1587,10 +1600,11 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   tm.mark("bind: staging + upload");
   if (e != cudaSuccess) return cleanup(fail(DGR_ECUDA, "upload: %s", cudaGetErrorString(e)));
   if (cudaMallocHost(&h->pinned, 16 * sizeof(double)) != cudaSuccess) return cleanup(fail(DGR_ECUDA, "cudaMallocHost failed"));
-  if (world > 1 && dist->allreduce) {
+  h->xchg = dist && (world > 1 || dist->nccl_unique_id || dist->allreduce);
+  if (h->xchg && dist->allreduce) {
     h->ar_fn = dist->allreduce;
     h->ar_user = dist->allreduce_user;
-  } else if (world > 1) {
+  } else if (h->xchg) {
     ncclUniqueId id;
     memcpy(&id, dist->nccl_unique_id, sizeof(id));
     ncclResult_t r = ncclCommInitRank(&h->comm, world, id, rank);
@@ -1635,6 +1649,16 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
     return fail(DGR_EINVAL, "f_slope must be > 0 for sigmoid / exp / CELU");
   if (int rc0 = live_comm(h)) return rc0;
   KParams& P = h->P;
+  // the loss goes straight from kg_loss_kernel into a pinned (device-accessible) host buffer: the
+  // caller's (dgr_step_async) or the handle's (dgr_step); a pageable buffer gets a copy after it
+  double* loss_dev = nullptr;
+  {
+    double* want = loss_async ? loss_async : (last ? h->pinned : nullptr);
+    cudaPointerAttributes at{};
+    if (want && cudaPointerGetAttributes(&at, want) == cudaSuccess && at.type == cudaMemoryTypeHost && at.devicePointer)
+      loss_dev = static_cast<double*>(at.devicePointer);
+    cudaGetLastError();   // a pageable pointer may leave an error code behind
+  }
   StepArgs a{};
   a.inv_t = 1.f / temperature;
   a.a_wl = w->a_wl; a.a_via = w->a_via; a.a_of = w->a_of; a.beta = w->beta_via;
@@ -1679,7 +1703,7 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
     a.store_d = last;
     adam_args(h->k);
     const Layout& Lay = h->lay;
-    if (h->world > 1) {
+    if (h->xchg) {
       // the forward's events reduced into each rank's grid bands (SURVEY §8(e) refinement 2), the
       // counters summed; the other ranks' bands cleared for the next forward (KG clears its own)
       const int r = h->rank;
@@ -1700,7 +1724,7 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
     launch_kg(P, a, s);   // this rank's bands (every line on one GPU)
     h->grids_dirty = false;
     if ((rc = prof_mark(h, 2))) return rc;
-    if (h->world > 1) {
+    if (h->xchg) {
       // the prefix sums S of every band to every rank (each rank's tiles read any of them); in the
       // last iteration also the loss partials and the demand of get_demand
       const size_t XP = (size_t)P.XP, YP = (size_t)P.YP;
@@ -1715,7 +1739,9 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
       if ((rc = prof_mark(h, 1))) return rc;
     }
     if (last) {   // the reported loss of this call's last forward
-      launch_kg_loss(P, a, s);
+      KParams PL = P;
+      PL.loss_host = loss_dev;
+      launch_kg_loss(PL, a, s);
       if ((rc = prof_mark(h, 5))) return rc;
     }
     if (iters > 0) {
@@ -1745,10 +1771,10 @@ static int step_impl(dgr_handle* h, int32_t iters, float temperature, float lr, 
   h->t_last = temperature;
   h->beta_last = w->beta_via;
   h->have_forward = true;
-  if (loss_async)   // stream-ordered read of this call's loss; no host synchronisation
+  if (loss_async && !loss_dev)   // stream-ordered read of this call's loss; no host synchronisation
     CUDA_TRY(cudaMemcpyAsync(loss_async, P.loss, 4 * sizeof(double), cudaMemcpyDeviceToHost, s));
   if (last) {
-    CUDA_TRY(cudaMemcpyAsync(h->pinned, P.loss, 4 * sizeof(double), cudaMemcpyDeviceToHost, s));
+    if (!loss_dev) CUDA_TRY(cudaMemcpyAsync(h->pinned, P.loss, 4 * sizeof(double), cudaMemcpyDeviceToHost, s));
     if (int rc_ = wait_stream(h)) return rc_;
     last->total = h->pinned[0];
     last->wl = h->pinned[1];
@@ -1811,7 +1837,7 @@ int dgr_induce(dgr_handle* h, float top_p, int32_t* tree_choice, int32_t* route,
   CUDA_TRY(cudaMemsetAsync(P.DH, 0, 4 * 3 * G, s));
   CUDA_TRY(cudaMemsetAsync(P.iscal, 0, 16, s));
   launch_induce(P, h->t_last, top_p, h->beta_last, s);
-  if (h->world > 1) {
+  if (h->xchg) {
     int rc;
     if ((rc = allreduce(h, P.DH, (int64_t)(3 * G), 1))) return rc;
     if ((rc = allreduce(h, P.iscal, 2, 0))) return rc;

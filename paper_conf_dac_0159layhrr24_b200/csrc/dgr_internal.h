@@ -199,6 +199,8 @@ struct KParams {
   long long* lsum;          // [2] acc of the last KG's forward (KG moves acc here and clears it)
   long long* lpart;         // [Y + X] per-line sums of the demand (2^-40), for E[WL]
   double* loss;             // [4]
+  double* loss_host;        // [4] or null: the caller's pinned host buffer (device alias), written by
+                            // kg_loss_kernel directly instead of a copy after it (dgr_step_async)
   // induce scratch
   uint8_t* chosen;          // [n_trees_l]
   int32_t* tree_choice;     // [n_nets_l] (global tree index)

@@ -1681,6 +1681,7 @@ __global__ void __launch_bounds__(1024) kg_loss_kernel(KParams P, StepArgs A) {
   // deterministic, one pass, no block scans
   __shared__ double shs[32], shd[32];
   const int nl = P.X + P.Y, lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  griddep_wait();   // launched with PDL behind the last KG: its partials
   double s = 0.0, sd = 0.0;
   for (int i = threadIdx.x; i < nl; i += blockDim.x) {
     s += P.partial[i];
@@ -1713,6 +1714,9 @@ __global__ void __launch_bounds__(1024) kg_loss_kernel(KParams P, StepArgs A) {
       P.loss[1] = ewl;
       P.loss[2] = via;
       P.loss[3] = s;
+      if (P.loss_host) {   // straight into the caller's pinned buffer (visible after the stream syncs)
+        P.loss_host[0] = P.loss[0]; P.loss_host[1] = ewl; P.loss_host[2] = via; P.loss_host[3] = s;
+      }
     }
   }
 }
@@ -2088,7 +2092,11 @@ void launch_tiles(const KParams& p, const StepArgs& a, TileMode mode, cudaStream
   else if (mode == kReverseForward) cudaLaunchKernelEx(&cfg, tile_bulk<true, true>, p, a);
   else cudaLaunchKernelEx(&cfg, tile_bulk<true, false>, p, a);
 }
-void launch_kg_loss(const KParams& p, const StepArgs& a, cudaStream_t s) { kg_loss_kernel<<<1, 1024, 0, s>>>(p, a); }
+void launch_kg_loss(const KParams& p, const StepArgs& a, cudaStream_t s) {
+  cudaLaunchAttribute attr;
+  cudaLaunchConfig_t cfg = pdl_config(1, 1024, 0, s, &attr);
+  cudaLaunchKernelEx(&cfg, kg_loss_kernel, p, a);
+}
 void launch_kg(const KParams& p, const StepArgs& a, cudaStream_t s) {
   cudaLaunchAttribute attr;
   const int nl = (p.kg_h1 - p.kg_h0) + (p.kg_v1 - p.kg_v0);

@@ -272,10 +272,12 @@ class Solver:
         self._idbuf = None
         dist = None
         self._ar = None
-        if world > 1 and allreduce is not None:
+        # world == 1 with an NCCL id or a callback: the band exchange runs anyway (one-rank
+        # communicator / the callback), the sharded path exercised on one GPU
+        if allreduce is not None:
             self._ar = ALLREDUCE_FN(lambda _u, buf, n, dt, st: int(allreduce(buf, n, dt, st)))
             dist = _Dist(rank, world, None, self._ar, None)
-        elif world > 1:
+        elif world > 1 or nccl_id is not None:
             if nccl_id is None or len(nccl_id) != 128:
                 raise DgrError("world > 1 needs the 128-byte NCCL unique id from rank 0")
             self._idbuf = ctypes.create_string_buffer(nccl_id, 128)

@@ -184,3 +184,87 @@ def test_tma_window_equals_cp_async_window(monkeypatch):
     assert all(np.array_equal(x, y) for x, y in zip(a.logits(), b.logits()))
     a.close()
     b.close()
+
+
+@pytest.mark.parametrize("name", ["c1e4", "c1e4_m", "ispd18"])
+def test_one_rank_nccl_exchange_reproduces_single_gpu(name):
+    """The band exchange through a real NCCL communicator (one rank: dgr_dist with world 1 and an NCCL
+    id, include/dgr.h): ncclReduceScatter / ncclAllGather / ncclAllReduce in groups on the handle's
+    stream, the band clears and the polling wait, bit-identical to the plain single-GPU path."""
+    f = forestgen.generate(name)
+    ref = dgr.Solver(f)
+    r_losses, (rdh, rdv), (rwt, rwp), rind = _schedule(ref)
+    ref.close()
+    s = dgr.Solver(f, nccl_id=dgr.nccl_unique_id())
+    losses, (dh, dv), (wt, wp), ind = _schedule(s)
+    s.close()
+    for a, b in zip(losses, r_losses):
+        assert np.array_equal(a, b)
+    assert np.array_equal(dh, rdh) and np.array_equal(dv, rdv)
+    assert np.array_equal(wt, rwt) and np.array_equal(wp, rwp)
+    assert np.array_equal(ind.tree_choice, rind.tree_choice) and np.array_equal(ind.route, rind.route)
+    assert np.array_equal(ind.D_h, rind.D_h) and np.array_equal(ind.metrics, rind.metrics)
+
+
+_ABORT_SCRIPT = r"""
+import os, sys
+import numpy as np
+import forestgen
+import paper_conf_dac_0159layhrr24_b200 as dgr
+s = dgr.Solver(forestgen.generate("ispd19"), nccl_id=dgr.nccl_unique_id())
+s.step(2, 1.0, 0.3)
+os.environ["DGR_NCCL_TIMEOUT_MS"] = "0"
+try:
+    s.step(100, 1.0, 0.3)
+    sys.exit("no timeout")
+except dgr.DgrError as e:
+    assert "communicator aborted" in str(e), e
+del os.environ["DGR_NCCL_TIMEOUT_MS"]
+try:
+    s.step(1, 1.0, 0.3)
+    sys.exit("step after abort succeeded")
+except dgr.DgrError as e:
+    assert "aborted" in str(e), e
+s.close()
+t = dgr.Solver(forestgen.generate("tiny"))
+assert np.isfinite(t.step(2, 1.0, 0.3)).all()
+t.close()
+print("ABORT-OK")
+"""
+
+
+def test_nccl_timeout_aborts_the_communicator():
+    """A synchronising call that finds the NCCL exchange unfinished after DGR_NCCL_TIMEOUT_MS aborts
+    the communicator (ncclCommAbort) and fails with DGR_ENCCL instead of hanging; later calls fail
+    with DGR_ESTATE; the device stays usable.  A timeout of 0 ms trips on the first poll of a long
+    call (100 ispd19 iterations, ~20 ms).  In a subprocess: an abort with work in flight must not
+    take this test process's CUDA context with it if it goes wrong."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", _ABORT_SCRIPT], cwd=root, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0 and "ABORT-OK" in r.stdout, (r.returncode, r.stdout[-2000:], r.stderr[-2000:])
+
+
+def test_tile_bundle_target_does_not_change_results(monkeypatch):
+    """Small forests get tiles of fewer bundles (a full wave of resident tiles, make_plan); the tile
+    composition never changes a result: auto against 32 and 4 group bundles per tile, bit-identical."""
+    f = forestgen.generate("c1e4")
+    outs = []
+    for tb in (None, "32", "4"):
+        if tb is None:
+            monkeypatch.delenv("DGR_TILE_BUNDLES", raising=False)
+        else:
+            monkeypatch.setenv("DGR_TILE_BUNDLES", tb)
+        s = dgr.Solver(f)
+        monkeypatch.delenv("DGR_TILE_BUNDLES", raising=False)
+        outs.append((s.info()["n_tiles"], _schedule(s)))
+        s.close()
+    assert outs[0][0] != outs[1][0] and outs[2][0] > outs[1][0]
+    for _, (losses, (dh, dv), (wt, wp), ind) in outs[1:]:
+        r_losses, (rdh, rdv), (rwt, rwp), rind = outs[0][1]
+        assert all(np.array_equal(a, b) for a, b in zip(losses, r_losses))
+        assert np.array_equal(dh, rdh) and np.array_equal(dv, rdv)
+        assert np.array_equal(wt, rwt) and np.array_equal(wp, rwp)
+        assert np.array_equal(ind.tree_choice, rind.tree_choice) and np.array_equal(ind.metrics, rind.metrics)

@@ -322,12 +322,15 @@ def test_split_calls_and_determinism(forests):
     assert all(np.array_equal(x, y) for x, y in zip(a.demand(), b.demand()))
 
 
-def test_step_async_equals_step(forests):
-    """dgr_step_async (no host sync, loss copied stream-ordered) is dgr_step: same losses, same state."""
+@pytest.mark.parametrize("pinned", [False, True])
+def test_step_async_equals_step(forests, pinned):
+    """dgr_step_async (no host sync) is dgr_step: same losses, same state.  A pageable loss buffer gets
+    a stream-ordered copy; a pinned one is written by the loss kernel itself (no copy in the chain)."""
+    import torch
     f = forests["c1e4"]
     a = dgr.Solver(f); b = dgr.Solver(f)
     la = np.array([a.step(1, 0.9, 0.3) for _ in range(5)])
-    lb = np.zeros((5, 4))
+    lb = torch.zeros((5, 4), dtype=torch.float64).pin_memory().numpy() if pinned else np.zeros((5, 4))
     for i in range(5):
         b.step_async(1, 0.9, 0.3, None, lb[i])
     b.sync()

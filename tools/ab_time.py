@@ -29,10 +29,19 @@ for _ in range(reps):
     e1.record(st)
     torch.cuda.synchronize()
     best = max(best, iters / (e0.elapsed_time(e1) * 1e-3))
+# host enqueue time of the same call (dgr_step without a loss read does not synchronise): if it is
+# below the device time per iteration, launches are not what bounds the loop
+import time  # noqa: E402
+torch.cuda.synchronize()
+h0 = time.perf_counter()
+s.step(iters, 1.0, 0.3, want_loss=False)
+host_us = (time.perf_counter() - h0) / iters * 1e6
+torch.cuda.synchronize()
 s.profile(True)
 s.step(iters, 1.0, 0.3, want_loss=False)
 ms, n = s.profile_read()
 s.profile(False)
 print(json.dumps({"lib": os.path.basename(os.environ.get("DGR_LIB", "libdgr.so")), "kg_cta": bool(os.environ.get("DGR_KG_CTA")),
-                  "config": name, "iters_per_s": best,
+                  "config": name, "tile_bundles": os.environ.get("DGR_TILE_BUNDLES", "auto"),
+                  "tiles": s.info()["n_tiles"], "iters_per_s": best, "host_enqueue_us_per_iter": host_us,
                   "stage_ms": {k: ms[k] / n[k] for k in ms if n[k]}}))
