@@ -591,7 +591,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   auto aligned_area = [](int bx0, int by0, int bx1, int by1) -> int64_t {
     const int x0 = bx0 & ~1, y0 = by0 & ~1;
     const int w = (bx1 + 1 - x0 + 1) & ~1, h = (by1 + 1 - y0 + 1) & ~1;
-    return (int64_t)w * h;
+    return std::max((int64_t)h * win_pitch(w), (int64_t)w * win_pitch(h));   // the padded fields (win_pitch)
   };
   // The greedy restarts at fixed chunk boundaries (independent of the thread count) so the chunks
   // run in parallel; each boundary costs at most one extra tile.
@@ -1055,7 +1055,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
     for (int64_t t = 0; t < (int64_t)pl.tiles.size(); ++t) {
       TileDesc& T = pl.tiles[t];
       T.tmap = -1;
-      if (no_tma || t >= pl.n_pipe_tiles || T.ww <= 0 || T.wh <= 0 || T.ww > 256 || T.wh > 256) continue;
+      if (no_tma || t >= pl.n_pipe_tiles || T.ww <= 0 || T.wh <= 0 || win_pitch(T.ww) > 256 || win_pitch(T.wh) > 256) continue;
       auto it = idx.find({T.ww, T.wh});
       if (it == idx.end()) {
         it = idx.emplace(std::make_pair(T.ww, T.wh), (int)pl.tmap_shapes.size()).first;
@@ -1069,8 +1069,8 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
 
 // ---------------------------------------------------------------------------------------
 // TMA tensor maps of the tile windows: 2-D views of S_H ([Y][XP] fp64) and S_V^T ([X][YP] fp64)
-// with the window's shape as the box, so one copy per field lands in the kernel's row-major
-// (column-major) window layout.  cuTensorMapEncodeTiled comes from the driver through the runtime's
+// with the window's shape as the box (rows / columns padded to win_pitch), so one copy per field
+// lands in the kernel's row-major (column-major) window layout.  cuTensorMapEncodeTiled comes from the driver through the runtime's
 // entry-point query (no link against libcuda).
 // ---------------------------------------------------------------------------------------
 int encode_window_maps(const std::vector<std::pair<int, int>>& shapes, const void* SH, const void* SVT, int X, int Y,
@@ -1091,7 +1091,7 @@ int encode_window_maps(const std::vector<std::pair<int, int>>& shapes, const voi
     {   // H field: inner dimension x
       const cuuint64_t dims[2] = {XP, (cuuint64_t)Y};
       const cuuint64_t strides[1] = {XP * 8};
-      const cuuint32_t box[2] = {ww, wh};
+      const cuuint32_t box[2] = {(cuuint32_t)win_pitch((int)ww), wh};   // padded rows (columns past X: zeros)
       CUresult r = encode(reinterpret_cast<CUtensorMap*>(out + 256 * i), CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2,
                           const_cast<void*>(SH), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
                           CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
@@ -1100,7 +1100,7 @@ int encode_window_maps(const std::vector<std::pair<int, int>>& shapes, const voi
     {   // V field: inner dimension y
       const cuuint64_t dims[2] = {YP, (cuuint64_t)X};
       const cuuint64_t strides[1] = {YP * 8};
-      const cuuint32_t box[2] = {wh, ww};
+      const cuuint32_t box[2] = {(cuuint32_t)win_pitch((int)wh), ww};
       CUresult r = encode(reinterpret_cast<CUtensorMap*>(out + 256 * i + 128), CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2,
                           const_cast<void*>(SVT), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
                           CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);

@@ -136,6 +136,15 @@ inline __host__ __device__ uint32_t tree_lane(int tree_rel, int net_rel, bool he
 // Shared-memory offset (elements) of a pipelined tile's V field: the H field rounded up to 128 bytes
 // of doubles (TMA destinations are 128-byte aligned).
 inline __host__ __device__ int win_hv(int ww, int wh) { return (ww * wh + 15) & ~15; }
+// Shared-memory pitch of an (even) window dimension n: n when n = 2 mod 4, else n + 2.  Lanes that
+// walk across the rows of a field (one Z candidate per lane: stride = pitch) then spread over 16
+// banks instead of colliding in a few (a pitch that is a multiple of 16 cells put every lane of a
+// fp64 gather, or of an int32 event add, in one bank).  TMA boxes need 16-byte rows, so the pitch
+// stays even.  The S window: H rows of pitch win_pitch(ww) at 0, V columns of pitch win_pitch(wh)
+// at win_s_hv; the event window: three row-major fields of pitch win_pitch(ww), win_hv(pitch, wh)
+// apart.
+inline __host__ __device__ int win_pitch(int n) { return (n & 3) ? n : n + 2; }
+inline __host__ __device__ int win_s_hv(int ww, int wh) { return win_hv(win_pitch(ww), wh); }
 constexpr int kWinPad = 16;   // the S / event windows hold up to 2 (kWinMax + kWinPad) elements
 
 struct KParams {

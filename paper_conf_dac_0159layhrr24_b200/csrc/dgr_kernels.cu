@@ -236,9 +236,9 @@ __device__ __forceinline__ void tp_fold_global(const KParams& P, const StepArgs&
 }
 
 // Flush of a tile's event window into the global difference arrays.  The window's three fields are
-// int32 (2^-24), row-major over the window (cell (x, y) at (y - wy0) ww + x - wx0): H events at 0,
-// V events at hv, turning points VD at 2 hv; the width is even, so pair i is cells 2i, 2i+1 of one
-// row.  Global cell j of a row receives (H_j << 16) + beta (VD_{j+1} - VD_{j-1} + [j = 0] VD_0):
+// int32 (2^-24), row-major over the window with row pitch ep >= ww (cell (x, y) at (y - wy0) ep +
+// x - wx0): H events at 0, V events at hv, turning points VD at 2 hv; width and pitch are even, so
+// pair i of row r is cells 2i, 2i+1 of that row.  Global cell j of a row receives (H_j << 16) + beta (VD_{j+1} - VD_{j-1} + [j = 0] VD_0):
 // its wire events and the turning points' +-beta pi windows along the row (tp_fold_global); cell j
 // of a column likewise with V and the VD of the cells above / below.  One pass, four predicated
 // int64 reductions per pair; cells outside the grid hold no events and receive nothing.  Returns
@@ -246,9 +246,9 @@ __device__ __forceinline__ void tp_fold_global(const KParams& P, const StepArgs&
 // derives E[WL] from the folded demand and these two (kg_loss_kernel).
 template <int NT, bool EXACT>
 __device__ __forceinline__ void flush_window_t(const KParams& P, const StepArgs& A, int wx0, int wy0, int ww, int wh,
-                                               int hv, const int* ev_s, long long& etp, long long& bdef) {
+                                               int ep, int hv, const int* ev_s, long long& etp, long long& bdef) {
   const int X = P.X, Y = P.Y, tid = threadIdx.x;
-  const int hw = ww >> 1;
+  const int hw = ww >> 1, hp = ep >> 1;   // pairs per row: of the window, of the (even) pitch
   // row = floor((i + 1/2) / half width) in fp32 is exact here: the fraction stays >= 1/(2 half)
   // >> the rounding of i < 2^12
   const float inv_hw = 1.f / (float)hw;
@@ -265,9 +265,10 @@ __device__ __forceinline__ void flush_window_t(const KParams& P, const StepArgs&
   for (int i = tid; i < npair; i += NT) {
     const int r = (int)(((float)i + 0.5f) * inv_hw), cx = 2 * (i - r * hw);
     const int gx = wx0 + cx, gy = wy0 + r;
-    const int2 h = evH[i], v = evV[i], d = evD2[i];
-    const int dl = cx > 0 ? evD[2 * i - 1] : 0, dr = cx + 2 < ww ? evD[2 * i + 2] : 0;
-    const int2 du = r > 0 ? evD2[i - hw] : make_int2(0, 0), dn = r + 1 < wh ? evD2[i + hw] : make_int2(0, 0);
+    const int pi = r * hp + (cx >> 1);   // the pair in the pitched fields
+    const int2 h = evH[pi], v = evV[pi], d = evD2[pi];
+    const int dl = cx > 0 ? evD[2 * pi - 1] : 0, dr = cx + 2 < ww ? evD[2 * pi + 2] : 0;
+    const int2 du = r > 0 ? evD2[pi - hp] : make_int2(0, 0), dn = r + 1 < wh ? evD2[pi + hp] : make_int2(0, 0);
     if (((h.x | h.y | v.x | v.y | d.x | d.y | dl | dr) | (du.x | du.y | dn.x | dn.y)) == 0) continue;   // nothing to flush
     // turning-point counts are >= 0 and < 2^31 per cell, so these differences fit int32
     int fh0 = d.y - dl, fh1 = dr - d.x, fv0 = dn.x - du.x, fv1 = dn.y - du.y;
@@ -303,9 +304,9 @@ __device__ __forceinline__ void flush_window_t(const KParams& P, const StepArgs&
 
 template <int NT>
 __device__ __forceinline__ void flush_window(const KParams& P, const StepArgs& A, int wx0, int wy0, int ww, int wh,
-                                             int hv, const int* ev_s, long long& etp, long long& bdef) {
-  if (A.beta_exact) flush_window_t<NT, true>(P, A, wx0, wy0, ww, wh, hv, ev_s, etp, bdef);
-  else flush_window_t<NT, false>(P, A, wx0, wy0, ww, wh, hv, ev_s, etp, bdef);
+                                             int ep, int hv, const int* ev_s, long long& etp, long long& bdef) {
+  if (A.beta_exact) flush_window_t<NT, true>(P, A, wx0, wy0, ww, wh, ep, hv, ev_s, etp, bdef);
+  else flush_window_t<NT, false>(P, A, wx0, wy0, ww, wh, ep, hv, ev_s, etp, bdef);
 }
 
 __device__ __forceinline__ long long warp_sum_ll(long long v) {
@@ -765,7 +766,7 @@ __device__ __forceinline__ void slow_tile(const KParams& P, const StepArgs& A, c
       else forward_warp<false>(P, A, T, bw0, bw1, REV, wst, q_s, g_all, Ew, ev_s, etp, bdef);
     }
     __syncthreads();
-    if (!T.global) flush_window<kTileThreads>(P, A, T.wx0, T.wy0, T.ww, T.wh, ncell, ev_s, etp, bdef);
+    if (!T.global) flush_window<kTileThreads>(P, A, T.wx0, T.wy0, T.ww, T.wh, T.ww, ncell, ev_s, etp, bdef);
     etp = warp_sum_ll(etp);
     bdef = warp_sum_ll(bdef);
     if ((tid & 31) == 0 && (etp | bdef)) {   // exact integers: any order gives the same sums
@@ -934,7 +935,7 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
   const bool tw = REV && !window && T.tmap >= 0 && !(KO(32));
   const uint32_t bytes = slot_bytes + gslot_bytes + 16u * T.nb + 8u * (s_hi - s_lo) + 4u * (n_hi - n_lo) +
                          8u * (t_hi - t_lo) + 8u * (nrow * T.ww + ncol * T.wh) +
-                         (tw ? 16u * (uint32_t)(T.ww * T.wh) : 0u);
+                         (tw ? 8u * (uint32_t)(T.wh * win_pitch(T.ww) + T.ww * win_pitch(T.wh)) : 0u);
   if (lane == 0) mbar_expect_tx(bar, bytes);
   __syncwarp();
   const size_t s0 = (size_t)T.b0 * 32;
@@ -942,7 +943,7 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
   if (tw && lane == 8) {
     const unsigned char* tm = P.tmaps + 256 * (size_t)T.tmap;
     tma_2d(S.S, tm, T.wx0, T.wy0, bar);
-    tma_2d(S.S + win_hv(T.ww, T.wh), tm + 128, T.wy0, T.wx0, bar);
+    tma_2d(S.S + win_s_hv(T.ww, T.wh), tm + 128, T.wy0, T.wx0, bar);
   }
   // work items: 0..7 the 1-D arrays, then window rows, then window columns
   const int nitems = 8 + (int)nrow + (int)ncol;
@@ -960,10 +961,10 @@ __device__ __forceinline__ void issue_tile_loads(const KParams& P, const TileDes
       }
     } else if (it < 8 + (int)nrow) {
       const int yi = it - 8;
-      bulk_g2s(S.S + (size_t)yi * T.ww, P.SH + (size_t)(T.wy0 + yi) * P.XP + T.wx0, 8u * T.ww, bar);
+      bulk_g2s(S.S + (size_t)yi * win_pitch(T.ww), P.SH + (size_t)(T.wy0 + yi) * P.XP + T.wx0, 8u * T.ww, bar);
     } else {
       const int xi = it - 8 - (int)nrow;
-      bulk_g2s(S.S + win_hv(T.ww, T.wh) + (size_t)xi * T.wh, P.SVT + (size_t)(T.wx0 + xi) * P.YP + T.wy0, 8u * T.wh, bar);
+      bulk_g2s(S.S + win_s_hv(T.ww, T.wh) + (size_t)xi * win_pitch(T.wh), P.SVT + (size_t)(T.wx0 + xi) * P.YP + T.wy0, 8u * T.wh, bar);
     }
   }
 }
@@ -1005,12 +1006,12 @@ __device__ __forceinline__ void lsu_tile_loads(const KParams& P, const TileDesc&
     const float inv_hw = 1.f / (float)hw, inv_hh = 1.f / (float)hh;
     for (int i = tid; i < n; i += NT) {
       const int r = (int)(((float)i + 0.5f) * inv_hw), c = i - r * hw;
-      cp16(S.S + (size_t)r * T.ww + 2 * c, P.SH + (size_t)(T.wy0 + r) * P.XP + T.wx0 + 2 * c);
+      cp16(S.S + (size_t)r * win_pitch(T.ww) + 2 * c, P.SH + (size_t)(T.wy0 + r) * P.XP + T.wx0 + 2 * c);
     }
-    double* SV = S.S + win_hv(T.ww, T.wh);
+    double* SV = S.S + win_s_hv(T.ww, T.wh);
     for (int i = tid; i < n; i += NT) {
       const int r = (int)(((float)i + 0.5f) * inv_hh), c = i - r * hh;
-      cp16(SV + (size_t)r * T.wh + 2 * c, P.SVT + (size_t)(T.wx0 + r) * P.YP + T.wy0 + 2 * c);
+      cp16(SV + (size_t)r * win_pitch(T.wh) + 2 * c, P.SVT + (size_t)(T.wx0 + r) * P.YP + T.wy0 + 2 * c);
     }
   }
   asm volatile("cp.async.commit_group;" ::: "memory");
@@ -1056,10 +1057,13 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   int s_lo, s_hi, n_lo, n_hi, t_lo, t_hi;
   tile_ranges(T, s_lo, s_hi, n_lo, n_hi, t_lo, t_hi);
   const uint64_t pol = policy_stream();   // L2 evict-first for the streamed slot state
-  const int hv = win_hv(T.ww, T.wh);   // V field at hv (128-byte aligned)
-  const Win W{T.wx0, T.wy0, T.ww, T.wh, hv};
+  // S window: H rows of pitch win_pitch(ww), V columns of pitch win_pitch(wh) from win_s_hv;
+  // event window: row-major fields of pitch ep, hv apart (128-byte aligned)
+  const Win W{T.wx0, T.wy0, win_pitch(T.ww), win_pitch(T.wh), win_s_hv(T.ww, T.wh)};
+  const int ep = win_pitch(T.ww);
+  const int hv = win_hv(ep, T.wh);
   const int hv2 = 2 * hv;                                                     // VD part of the window
-  const int eb = -(T.wy0 * T.ww + T.wx0);                                     // event-window origin
+  const int eb = -(T.wy0 * ep + T.wx0);                                       // event-window origin
   const int nbg = T.nbg;
 
   // ---------------- reverse of iteration k ----------------
@@ -1235,7 +1239,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
           // Z(o, m) form a cell (a, b) of orientation o (a along the primary lines) is at a A + b B
           // with (A, B) = (1, ww) for o = 0 and (ww, 1) for o = 1, so the segment ends of one line
           // are ordered like their cell indices
-          const int A_ = o ? T.ww : 1, B_ = o ? 1 : T.ww;
+          const int A_ = o ? ep : 1, B_ = o ? 1 : ep;
           const int p0 = o ? e.y : e.x, p1 = o ? e.w : e.z, q0 = o ? e.x : e.y, q1 = o ? e.z : e.w;
           const int cp0 = p0 * A_ + q0 * B_ + eb, cp1 = p1 * A_ + q1 * B_ + eb;
           const int cm0 = m * A_ + q0 * B_ + eb, cm1 = m * A_ + q1 * B_ + eb;
@@ -1268,8 +1272,8 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
           const float q = St.q[tree - t_lo];
           const int vq = __float2int_rn(q * kFixScale);
           const short4 e = St.sxy[bi.y + lane - s_lo];
-          const int ia = e.y * T.ww + e.x + eb + (isv ? hv : 0);   // row-major event fields
-          const int ib = (isv ? e.w * T.ww + e.x + hv : e.y * T.ww + e.z) + eb;
+          const int ia = e.y * ep + e.x + eb + (isv ? hv : 0);   // row-major event fields
+          const int ib = (isv ? e.w * ep + e.x + hv : e.y * ep + e.z) + eb;
           red_shared_add(ev_base + 4u * ia, vq);
           red_shared_add(ev_base + 4u * ib, -vq);
         }
@@ -1290,7 +1294,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     // flush the window once, then the tile's shares of E[TP] and of the border deficit summed in
     // warp order into the exchange buffer's counters
     long long etp = 0, bdef = 0;
-    flush_window<NT>(P, A, T.wx0, T.wy0, T.ww, T.wh, hv, ev_s, etp, bdef);
+    flush_window<NT>(P, A, T.wx0, T.wy0, T.ww, T.wh, ep, hv, ev_s, etp, bdef);
     etp = warp_sum_ll(etp);
     bdef = warp_sum_ll(bdef);
     long long* part = reinterpret_cast<long long*>(dq3);   // free after the net level
