@@ -673,48 +673,59 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   // Group bundles of a tile: its noisy sub-nets (groups of g <= 32 candidates, never split) packed
   // first-fit decreasing (ties in plan order), or first-fit in plan order when that needs fewer
   // bundles (so never more than the tile greedy's first-fit count).  Returns the bins as lists of indices into the tile's groups in plan order.
-  auto pack_groups = [](const std::vector<int>& gs) {
-    std::vector<std::vector<int>> nf, ff;   // nf: first-fit online in plan order (the greedy's count)
-    {
-      std::vector<int> fills;
-      for (int i = 0; i < (int)gs.size(); ++i) {
-        size_t k = 0;
-        while (k < fills.size() && fills[k] + gs[i] > 32) ++k;
-        if (k == fills.size()) { fills.push_back(0); nf.emplace_back(); }
-        fills[k] += gs[i];
-        nf[k].push_back(i);
-      }
+  // (no per-call allocations once warm: sizes bucketed 32..0 for the decreasing order, which keeps
+  // plan order among equal sizes like a stable sort; the result is each group's bin, and the
+  // members listed bin by bin in plan order)
+  struct GroupPack {
+    std::vector<int> bin_nf, bin_ff, fills, members, start, cursor;
+    std::vector<int> bucket[33];
+    int nbins = 0;
+    void run(const std::vector<int>& gs) {
+      const int n = (int)gs.size();
+      fills.resize(n + 1);
+      auto first_fit = [&](int g, int& nb) {
+        int k = 0;
+        while (k < nb && fills[k] + g > 32) ++k;
+        if (k == nb) fills[nb++] = 0;
+        fills[k] += g;
+        return k;
+      };
+      bin_nf.resize(n); bin_ff.resize(n);
+      int nnf = 0, nff = 0;
+      for (int i = 0; i < n; ++i) bin_nf[i] = first_fit(gs[i], nnf);   // online, plan order (the greedy's count)
+      for (auto& b : bucket) b.clear();
+      for (int i = 0; i < n; ++i) bucket[std::min(gs[i], 32)].push_back(i);
+      for (int g = 32; g >= 0; --g)
+        for (int i : bucket[g]) bin_ff[i] = first_fit(gs[i], nff);
+      const std::vector<int>& bin = nff <= nnf ? bin_ff : bin_nf;
+      nbins = std::min(nff, nnf);
+      start.assign(nbins + 1, 0);
+      for (int i = 0; i < n; ++i) ++start[bin[i] + 1];
+      for (int b = 0; b < nbins; ++b) start[b + 1] += start[b];
+      cursor.assign(start.begin(), start.end() - 1);
+      members.resize(n);
+      for (int i = 0; i < n; ++i) members[cursor[bin[i]]++] = i;
     }
-    std::vector<int> order(gs.size());
-    for (int i = 0; i < (int)gs.size(); ++i) order[i] = i;
-    std::stable_sort(order.begin(), order.end(), [&](int a, int b) { return gs[a] > gs[b]; });
-    std::vector<int> fills;
-    for (int i : order) {
-      size_t k = 0;
-      while (k < fills.size() && fills[k] + gs[i] > 32) ++k;
-      if (k == fills.size()) { fills.push_back(0); ff.emplace_back(); }
-      fills[k] += gs[i];
-      ff[k].push_back(i);
-    }
-    for (auto& bin : ff) std::sort(bin.begin(), bin.end());   // plan order within a bundle
-    return ff.size() <= nf.size() ? ff : nf;
   };
-  auto tile_groups = [&](int64_t pa, int64_t pb) {   // group sizes of the tile's noisy sub-nets, plan order
-    std::vector<int> gs;
+  auto tile_groups = [&](int64_t pa, int64_t pb, std::vector<int>& gs) {   // group sizes of the tile's noisy sub-nets, plan order
+    gs.clear();
     for (int64_t pn = pa; pn < pb; ++pn) {
       const int64_t n = pl.net_lo + perm[pn];
       const int64_t s0 = d->tree_sub_off[d->net_tree_off[n]], s1 = d->tree_sub_off[d->net_tree_off[n + 1]];
       for (int64_t sn = s0; sn < s1; ++sn)
         if (!gen[sn - pl.sub_lo] && !single[sn - pl.sub_lo]) gs.push_back((int)(d->sub_path_off[sn + 1] - d->sub_path_off[sn]));
     }
-    return gs;
   };
   // 3. bundles, tile by tile: the tile's group bundles (packing restarts at each tile), then its
   //    singleton bundles; sub-nets renumbered in that order ("kernel order").  Count per tile,
   //    prefix, then fill the tiles in parallel (each owns a contiguous bundle and sub-net range).
   const int64_t ntile = (int64_t)starts.size() - 1;
   std::vector<int32_t> tb0(ntile + 1, 0), tbg(ntile, 0), tmn(ntile + 1, 0);
-#pragma omp parallel for schedule(dynamic, 64)
+#pragma omp parallel
+  {
+  GroupPack gp;
+  std::vector<int> gsz;
+#pragma omp for schedule(dynamic, 64)
   for (int64_t t = 0; t < ntile; ++t) {
     Pack pk;
     int lanes = 0;   // tree lanes of the tile's multi-tree nets (a net's trees within one warp)
@@ -728,8 +739,11 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       }
     }
     tmn[t + 1] = (lanes + 31) & ~31;
-    tbg[t] = (int32_t)pack_groups(tile_groups(starts[t], starts[t + 1])).size();
+    tile_groups(starts[t], starts[t + 1], gsz);
+    gp.run(gsz);
+    tbg[t] = (int32_t)gp.nbins;
     tb0[t + 1] = tbg[t] + (pk.nsing + 31) / 32;
+  }
   }
   for (int64_t t = 0; t < ntile; ++t) { tb0[t + 1] += tb0[t]; tmn[t + 1] += tmn[t]; }
   pl.mnets.assign(tmn[ntile], 0);
@@ -749,6 +763,12 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   {
     std::vector<uint16_t> cnt;
     std::vector<int> stamp, cov;
+    GroupPack gp;
+    struct TT { int64_t j; int32_t pt; bool multi; };
+    struct Grp { int64_t ls; int g, noff, toff; uint32_t mt; };
+    std::vector<TT> tts;   // (per-thread buffers, reused across tiles)
+    std::vector<Grp> grps;
+    std::vector<int> gsz;
 #pragma omp for schedule(dynamic, 16)
     for (int64_t t = 0; t < ntile; ++t) {
       TileDesc T{};
@@ -757,8 +777,7 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       T.tree0 = ptree_off[starts[t]];
       T.ntree = ptree_off[starts[t + 1]] - T.tree0;
       // the tile's trees in plan order: CSR tree, plan-ordered local tree, net has >= 2 trees
-      struct TT { int64_t j; int32_t pt; bool multi; };
-      std::vector<TT> tts;
+      tts.clear();
       for (int64_t pn = starts[t]; pn < starts[t + 1]; ++pn) {
         const int64_t n = pl.net_lo + perm[pn];
         const int64_t a = d->net_tree_off[n], b = d->net_tree_off[n + 1];
@@ -816,9 +835,8 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       // global noise indices form runs (tile_noise fills gp by offset); the groups are then packed
       // (pack_groups), and each slot's lane descriptor carries its noise offset, group head and end
       // lane and its sub-net's index in the bundle (kernel order follows the bundles' slot order)
-      struct Grp { int64_t ls; int g, noff, toff; uint32_t mt; };
-      std::vector<Grp> grps;
-      std::vector<int> gsz;
+      grps.clear();
+      gsz.clear();
       std::vector<NoiseRun> truns;
       int noff = 0;
       for (const TT& tt : tts) {
@@ -833,14 +851,15 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
           noff += g;
         }
       }
-      const auto bins = pack_groups(gsz);
+      gp.run(gsz);
       int b = T.b0 - 1, prev_tree = -1;
-      for (const auto& bin : bins) {
+      for (int bn = 0; bn < gp.nbins; ++bn) {
         ++b;
         pl.binfo[b] = make_int4(0, ks, T.tree0, 0);
         int fill = 0, gi = 0;
         prev_tree = -1;
-        for (int idx : bin) {
+        for (int mi = gp.start[bn]; mi < gp.start[bn + 1]; ++mi) {
+          const int idx = gp.members[mi];
           const Grp& G = grps[idx];
           const int64_t sn = pl.sub_lo + G.ls;
           const int64_t p0 = d->sub_path_off[sn], p1 = d->sub_path_off[sn + 1];
@@ -1570,7 +1589,11 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
   float* pslots = reinterpret_cast<float*>(pin + at[6]);
   float* qs = reinterpret_cast<float*>(pin + at[10]);
   float* wts = reinterpret_cast<float*>(pin + at[9]);
-  for (size_t j = 0; j < nt; ++j) wts[j] = desc->w_tree0[pl.tree_lo + pl.tperm[j]];
+#pragma omp parallel for schedule(static)
+  for (size_t j = 0; j < nt; ++j) {
+    wts[j] = desc->w_tree0[pl.tree_lo + pl.tperm[j]];
+    qs[j] = 1.f;   // q of a net's lone tree stays 1 (never rewritten)
+  }
   float* capVT = reinterpret_cast<float*>(pin + at[12]);
 #pragma omp parallel for schedule(static)
   for (size_t sl = 0; sl < slots; ++sl) {
@@ -1578,7 +1601,6 @@ int dgr_bind_workspace(dgr_handle* h, const dgr_forest_desc* desc, const dgr_dis
     wslots[sl] = v ? desc->w_path0[pl.path_lo + pl.slot_path[sl]] : 0.f;
     pslots[sl] = v ? 1.f : 0.f;   // p of a lone straight candidate (never rewritten by the pipelined kernel)
   }
-  for (size_t j = 0; j < nt; ++j) qs[j] = 1.f;   // q of a net's lone tree stays 1 (never rewritten)
   // tensor maps of the tile windows over this workspace's S_H ([Y][XP]) and S_V ([X][YP]) (fp64)
   if (!pl.tmap_shapes.empty()) {
     unsigned char* tm = reinterpret_cast<unsigned char*>(pin + at[13]);

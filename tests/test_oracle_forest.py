@@ -102,6 +102,39 @@ def test_candidate1_is_a_steiner_tree_no_longer_than_the_mst(c1e4, c1e4_built):
     assert checked3 > 50
 
 
+def test_candidate1_is_a_local_optimum_of_the_1_steiner_step(c1e4, c1e4_built):
+    """Candidate 1 against the definition of iterated 1-Steiner (reading Q17, Kahng-Robins), checked
+    with scipy's MST rather than the oracle's Prim: (a) its edges form a minimum spanning tree of
+    pins + Steiner points; (b) it is a fixed point of the 1-Steiner step: adding any further Hanan
+    grid point of the pins does not shorten that point set's MST (the loop stops only then).  Nets
+    of 3..6 pins (Hanan grids of <= 36 points)."""
+    o = c1e4_built
+    checked = 0
+    for n in range(c1e4.n_nets):
+        pins = c1e4.pin_xy[c1e4.net_pin_off[n]:c1e4.net_pin_off[n + 1]].astype(np.int64)
+        if not 3 <= len(pins) <= 6:
+            continue
+        trees = _tree_subs(o, n)
+        if len(trees) < 2:
+            continue
+        t1 = trees[1]
+        pset = {tuple(p) for p in pins}
+        ends = {(s[0], s[1]) for s in t1} | {(s[2], s[3]) for s in t1}
+        pts = np.array([tuple(p) for p in pins] + sorted(ends - pset), np.int64)
+        l1 = np.abs(t1[:, 2] - t1[:, 0]).sum() + np.abs(t1[:, 3] - t1[:, 1]).sum()
+        mst = _manhattan_mst(pts)
+        assert abs(l1 - mst) < 1e-6, (n, l1, mst)                                     # (a)
+        have = {tuple(p) for p in pts}
+        for hx in np.unique(pins[:, 0]):
+            for hy in np.unique(pins[:, 1]):
+                if (hx, hy) in have:
+                    continue
+                grown = _manhattan_mst(np.vstack([pts, [[hx, hy]]]))
+                assert grown >= mst - 1e-6, (n, (hx, hy), grown, mst)                   # (b)
+        checked += 1
+    assert checked > 100
+
+
 def test_path_candidates_are_the_patterns(tiny):
     """Every candidate is a monotone route between its sub-net's endpoints (length |dx| + |dy|,
     turning points = segments - 1), groups are straight / HV, VH, Z... (Q14, all Z on tiny)."""
