@@ -558,10 +558,32 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   }
   // trees and sub-nets renumbered in plan order (a tile's trees / sub-nets stay contiguous)
   std::vector<int32_t> ptree_off(nn + 1, 0), psub_off(nn + 1, 0);
-  for (int64_t pn = 0; pn < nn; ++pn) {
-    const int64_t n = pl.net_lo + perm[pn];
-    ptree_off[pn + 1] = ptree_off[pn] + (int32_t)(d->net_tree_off[n + 1] - d->net_tree_off[n]);
-    psub_off[pn + 1] = psub_off[pn] + (int32_t)(d->tree_sub_off[d->net_tree_off[n + 1]] - d->tree_sub_off[d->net_tree_off[n]]);
+  {   // counts, then a two-pass prefix over fixed chunks
+#pragma omp parallel for schedule(static)
+    for (int64_t pn = 0; pn < nn; ++pn) {
+      const int64_t n = pl.net_lo + perm[pn];
+      ptree_off[pn + 1] = (int32_t)(d->net_tree_off[n + 1] - d->net_tree_off[n]);
+      psub_off[pn + 1] = (int32_t)(d->tree_sub_off[d->net_tree_off[n + 1]] - d->tree_sub_off[d->net_tree_off[n]]);
+    }
+    constexpr int64_t kChunk = 1 << 15;
+    const int64_t nch = (nn + kChunk - 1) / kChunk;
+    std::vector<int32_t> bt(nch + 1, 0), bs(nch + 1, 0);
+#pragma omp parallel for schedule(static)
+    for (int64_t ch = 0; ch < nch; ++ch) {
+      int32_t a = 0, b = 0;
+      for (int64_t pn = ch * kChunk + 1; pn <= std::min(nn, (ch + 1) * kChunk); ++pn) {
+        a += ptree_off[pn]; ptree_off[pn] = a;
+        b += psub_off[pn]; psub_off[pn] = b;
+      }
+      bt[ch + 1] = a; bs[ch + 1] = b;
+    }
+    for (int64_t ch = 0; ch < nch; ++ch) { bt[ch + 1] += bt[ch]; bs[ch + 1] += bs[ch]; }
+#pragma omp parallel for schedule(static)
+    for (int64_t ch = 1; ch < nch; ++ch)
+      for (int64_t pn = ch * kChunk + 1; pn <= std::min(nn, (ch + 1) * kChunk); ++pn) {
+        ptree_off[pn] += bt[ch];
+        psub_off[pn] += bs[ch];
+      }
   }
   pl.net_tree_off = ptree_off;
   pl.tperm.resize((size_t)(pl.tree_hi - pl.tree_lo));
