@@ -533,7 +533,7 @@ def main():
                 "d2h_bytes_per_step": d2h / e2e_iters,
                 "note": f"one solve of the paper's schedule from host CSR arrays through the C ABI: dgr_forest_plan + dgr_bind_workspace "
                         f"(reads {h2d} B of host CSR arrays, validation + encoding + H2D) + {e2e_iters} x dgr_step_async(1) "
-                        f"(t = 0.9^floor(k/100), lr 0.3) with the loss of each iteration copied to pinned host memory "
+                        f"(t = 0.9^floor(k/100), lr 0.3) with the loss of each iteration written stream-ordered into pinned host memory (by the loss kernel) "
                         f"+ dgr_get_demand; wall clock, max over ranks (after one untimed warm-up solve)",
                 "split": e2e_split},
     }
