@@ -1324,6 +1324,9 @@ __device__ __forceinline__ double gen_cost(const KParams& P, const StepArgs& A, 
   const int X = P.X, Y = P.Y;
   double c = 0.0, tp = 0.0;
   int wl = 0;
+  // (unrolled: the segment records and then their S values load in parallel, not one dependent
+  // pair of L2 round trips per segment)
+#pragma unroll 4
   for (int q = P.gp_seg_off[gp]; q < P.gp_seg_off[gp + 1]; ++q) {
     const short4 g = P.gseg[q];   // {dir, line, lo, hi}: edges [lo, hi) of the line
     const double* S = g.x == 0 ? P.SH + (size_t)g.y * P.XP : P.SVT + (size_t)g.y * P.YP;
@@ -1331,6 +1334,7 @@ __device__ __forceinline__ double gen_cost(const KParams& P, const StepArgs& A, 
     wl += g.w - g.z;
   }
   const int t0 = P.gp_tp_off[gp], t1 = P.gp_tp_off[gp + 1];
+#pragma unroll 4
   for (int q = t0; q < t1; ++q) {   // the (clipped) edges left / right and below / above the cell
     const short2 v = P.gtp[q];
     const double* SH = P.SH + (size_t)v.y * P.XP;
@@ -1344,12 +1348,14 @@ __device__ __forceinline__ double gen_cost(const KParams& P, const StepArgs& A, 
 __device__ __forceinline__ void gen_events(const KParams& P, const StepArgs& A, int gp, int v, long long& etp, long long& bdef) {
   if (v == 0) return;
   const long long vs = (long long)v << kGridShift;
+#pragma unroll 4
   for (int q = P.gp_seg_off[gp]; q < P.gp_seg_off[gp + 1]; ++q) {
     const short4 g = P.gseg[q];
     long long* diff = g.x == 0 ? P.dH + (size_t)g.y * P.X : P.dVT + (size_t)g.y * P.Y;
     red64(diff + g.z, vs);
     red64(diff + g.w, -vs);
   }
+#pragma unroll 4
   for (int q = P.gp_tp_off[gp]; q < P.gp_tp_off[gp + 1]; ++q) {
     const short2 t = P.gtp[q];
     tp_fold_global(P, A, t.x, t.y, v, etp, bdef);
@@ -1375,13 +1381,17 @@ __device__ __forceinline__ void gen_net(const KParams& P, const StepArgs& A, int
     for (int g = nd.x; g < nd.x + nd.y; ++g) {
       const int4 gt = P.gtree[g];   // {local tree, first gsub, sub-nets, multi-tree}
       const float q = P.q[gt.x];
-      long long dq = 0;             // dq_j = sum over the tree's sub-nets of sum_k p_k c_k (2^-32)
+      // dq_j = sum over the tree's sub-nets of sum_k p_k c_k (2^-32 fixed point: exact, any order).
+      // Lone straight paths (p = 1: their c goes to dq as is) a lane each, then the groups
+      long long dq = 0;
+      for (int s = gt.y + lane; s < gt.y + gt.z; s += 32) {
+        const GSub G = P.gsub[s];
+        if (G.nid < 0) dq += __double2ll_rn(gen_cost(P, A, G.gp) * kDqScale);
+      }
+      dq = warp_sum_ll(dq);         // (lane 0 holds the total)
       for (int s = gt.y; s < gt.y + gt.z; ++s) {
         const GSub G = P.gsub[s];
-        if (G.nid < 0) {            // a lone straight path: p = 1, its c goes to dq
-          if (lane == 0) dq += __double2ll_rn(gen_cost(P, A, G.gp) * kDqScale);
-          continue;
-        }
+        if (G.nid < 0) continue;
         double c0 = 0.0, cl = 0.0;  // the group's first c; this lane's c of the first chunk
         float sa = 0.f;             // sum_k p_k (c_k - c_0)
         for (int b = 0; b < G.n; b += 32) {
@@ -1452,12 +1462,13 @@ __device__ __forceinline__ void gen_net(const KParams& P, const StepArgs& A, int
     for (int g = nd.x; g < nd.x + nd.y; ++g) {
       const int4 gt = P.gtree[g];
       const float q = P.q[gt.x];
+      for (int s = gt.y + lane; s < gt.y + gt.z; s += 32) {   // lone straight paths (pi = q), a lane each
+        const GSub G = P.gsub[s];
+        if (G.nid < 0) gen_events(P, A, G.gp, __float2int_rn(q * kFixScale), etp, bdef);
+      }
       for (int s = gt.y; s < gt.y + gt.z; ++s) {
         const GSub G = P.gsub[s];
-        if (G.nid < 0) {            // lone straight path: pi = q
-          if (lane == 0) gen_events(P, A, G.gp, __float2int_rn(q * kFixScale), etp, bdef);
-          continue;
-        }
+        if (G.nid < 0) continue;
         // p_i = softmax over the group of (w_i + g_i) / t: the maximum, then the sum, then p
         float zl = -INFINITY, zmax = -INFINITY;
         for (int b = 0; b < G.n; b += 32) {
