@@ -37,6 +37,9 @@ constexpr unsigned kFull = 0xffffffffu;
 
 // DGR_ACCURATE=1: correctly rounded-ish fp32 library functions (expf, logf, sqrtf, IEEE division)
 // on the per-candidate path instead of the MUFU approximations (experiment: parity vs speed)
+#ifndef DGR_NL_EARLY
+#define DGR_NL_EARLY 1   // net level: tree moments loaded before its barrier, tree noise before the Adam chain
+#endif
 #ifndef DGR_HEAD_SOFTMAX
 #define DGR_HEAD_SOFTMAX 1   // softmax shifted by the group head's z (exact maximum only when needed)
 #endif
@@ -98,18 +101,30 @@ __device__ __forceinline__ float gumbel(uint64_t seed, uint64_t idx, uint32_t k,
 // on the words of a quad that no candidate draws); the tile's runs of
 // consecutive global noise indices (NoiseRun), one Philox call per aligned quad of indices (one run:
 // the quads spread over the CTA's threads; several: a thread per run piece of at most 4 quads).
-template <int NT>
+// VEC (pipelined tiles, one run): quad q goes whole to gp[4q .. 4q + 3] (one 16-byte store per thread,
+// no bank conflicts), so the word of tile noise offset o sits at gp[o + noise_shift(P, T)].
+__device__ __forceinline__ int noise_shift(const KParams& P, const TileDesc& T) {
+  return T.nrun == 1 ? (int)((P.nid_base + T.nid0) & 3) : 0;
+}
+template <int NT, bool VEC = false>
 __device__ __forceinline__ void tile_noise(const KParams& P, const TileDesc& T, uint32_t k, float* gp) {
   if (T.nrun == 1) {   // one run (nets in the caller's order): its quads spread over the threads
     const int64_t g0 = P.nid_base + T.nid0;
-    for (int q = threadIdx.x; q < T.nquad; q += NT) {
-      const int64_t c = (g0 >> 2) + q;
-      const uint4 w = philox_rk(make_uint4((uint32_t)c, (uint32_t)(c >> 32), k, 0u), P.rk);
-      const uint32_t wd[4] = {w.x, w.y, w.z, w.w};
+    if (VEC) {
+      for (int q = threadIdx.x; q < T.nquad; q += NT) {
+        const int64_t c = (g0 >> 2) + q;
+        reinterpret_cast<uint4*>(gp)[q] = philox_rk(make_uint4((uint32_t)c, (uint32_t)(c >> 32), k, 0u), P.rk);
+      }
+    } else {
+      for (int q = threadIdx.x; q < T.nquad; q += NT) {
+        const int64_t c = (g0 >> 2) + q;
+        const uint4 w = philox_rk(make_uint4((uint32_t)c, (uint32_t)(c >> 32), k, 0u), P.rk);
+        const uint32_t wd[4] = {w.x, w.y, w.z, w.w};
 #pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const int64_t o = c * 4 + i - g0;
-        if (o >= 0 && o < T.nnoisy) gp[o] = __uint_as_float(wd[i]);
+        for (int i = 0; i < 4; ++i) {
+          const int64_t o = c * 4 + i - g0;
+          if (o >= 0 && o < T.nnoisy) gp[o] = __uint_as_float(wd[i]);
+        }
       }
     }
     return;
@@ -1049,7 +1064,8 @@ __device__ __forceinline__ void stamp(const KParams& P, int tile, int k) {
 constexpr size_t kGpOffset = 3 * 4 * (kWinMax + kWinPad);   // tile path noise, after the event window in St.S
 template <bool REV, bool FWD, int NT>
 __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A, const TileDesc& T, Stage St,
-                                             int* ev_s, float* gp, int* dq3, uint32_t ld_first, uint32_t mte) {
+                                             int* ev_s, float* gp, int* dq3, uint32_t ld_first, uint32_t mte,
+                                             const uint32_t* twd) {
   // dq3[0..3 ntree) arrives zeroed (the caller clears it before its first barrier)
   constexpr int NW = NT / 32;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -1129,6 +1145,20 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         if (valid && ((th >> lane) & 1u)) dq_add(dq3, tree - T.tree0, pc);
       }
     }
+  }
+  // the net level's tree Adam moments (one dependent global round trip on that phase's critical
+  // path), loaded now: their latency hides behind the barrier and the dq reductions, and the
+  // reverse's registers are dead here
+  float mt_pre = 0.f, vt_pre = 0.f;
+  (void)mt_pre; (void)vt_pre;
+#if DGR_NL_EARLY
+  if (REV && tid < T.nmn && mte != kNoTreeLane) {
+    const int jg = T.tree0 + (int)(mte & 1023u);
+    mt_pre = __ldcg(P.mt + jg);
+    vt_pre = __ldcg(P.vt + jg);
+  }
+#endif
+  if (REV && !(KO(64))) {
     __syncthreads();
   }
   stamp(P, (int)blockIdx.x - P.ntiles_slow - P.ngen_blocks, 2);
@@ -1155,6 +1185,11 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     const int head = 31 - __clz(hm & le);
     const uint32_t rest = hm & ~le;
     const int end = rest ? (__ffs(rest) - 2) : 31;
+#if DGR_NL_EARLY
+    // the tree's Gumbel noise first: independent of the reverse, it overlaps the Adam chain
+    const uint32_t wd = (FWD && tv) ? twd[tid] : 0u;   // drawn at the tile's entry
+    (void)nrel;
+#endif
     if (REV) {
       // du_j = (q_j/t)(dq_j - sum_l q_l dq_l / sum_l q_l); Adam on w_tree (iteration k)
       const double ql = tv ? (double)St.q[j] : 0.0;
@@ -1169,7 +1204,11 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
       if (tv) {
         const double du = (double)St.q[j] * (double)A.inv_t * (dq_get(dq3, jr) - sq);
         const int jg = j + t_lo;
+#if DGR_NL_EARLY
+        float w = St.wt[j], m = mt_pre, v = vt_pre;
+#else
         float w = St.wt[j], m = P.mt[jg], v = P.vt[jg];
+#endif
         adam_update(w, m, v, (float)du, A);
         St.wt[j] = w;
         P.wt[jg] = w; P.mt[jg] = m; P.vt[jg] = v;
@@ -1178,14 +1217,18 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
     if (FWD) {
       // q_j = softmax over the net's trees of (w_j + g_j)/t, iteration k_next (noise stream 1, keyed on
       // the global tree id: plan order = CSR order, else from net_gtree)
-      const int jh = __shfl_sync(kFull, j, head);
       float z = -INFINITY;
+#if DGR_NL_EARLY
+      if (tv) z = (St.wt[j] + gumbel_word(wd)) * A.inv_t;
+#else
+      const int jh = __shfl_sync(kFull, j, head);
       if (tv) {
         const int64_t gj = P.tree_base + (P.perm_id ? (int64_t)(t_lo + j) : (int64_t)__ldg(&P.net_gtree[T.net0 + nrel]) + (j - jh));
         const uint4 r = philox_rk(make_uint4((uint32_t)(gj >> 2), (uint32_t)(gj >> 34), (uint32_t)A.k_next, 1u), P.rk);
         const uint32_t wd = (gj & 3) == 0 ? r.x : (gj & 3) == 1 ? r.y : (gj & 3) == 2 ? r.z : r.w;
         z = (St.wt[j] + gumbel_word(wd)) * A.inv_t;
       }
+#endif
       float zmax = -INFINITY;
       for (int k = 0; __any_sync(kFull, head + k <= end); ++k) {
         const float a = __shfl_sync(kFull, z, min(head + k, 31));
@@ -1204,13 +1247,14 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
       }
     }
   }
-  if (FWD && nbg > 0 && !(KO(2))) tile_noise<NT>(P, T, (uint32_t)A.k_next, gp);   // path noise (stream 0)
+  if (FWD && nbg > 0 && !(KO(2))) tile_noise<NT, true>(P, T, (uint32_t)A.k_next, gp);   // path noise (stream 0)
   __syncthreads();
   stamp(P, (int)blockIdx.x - P.ntiles_slow - P.ngen_blocks, 3);
 
   // ---------------- forward of iteration k_next ----------------
   if (FWD) {
     const uint32_t ev_base = smem_u32(ev_s);
+    const int gsh = noise_shift(P, T);
     const uint32_t* LD = P.ldesc + (size_t)T.b0 * 32 + lane;   // lane descriptors, prefetched a bundle ahead
     uint32_t ldn = ld_fwd;
     for (int lb = warp; lb < T.nb; lb += NW) {
@@ -1223,7 +1267,7 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
         lane_from_desc(bi, pw, ld, L);
         const int sl = lb * 32 + lane;
         const float w = St.w[sl];
-        const float g = L.valid ? gumbel_word(__float_as_uint(gp[ld & 0x7FFu])) : 0.f;   // the lane's word, by its tile noise offset
+        const float g = L.valid ? gumbel_word(__float_as_uint(gp[(ld & 0x7FFu) + gsh])) : 0.f;   // the lane's word, by its tile noise offset
         const float p = softmax_from_noise(L, w, g, A.inv_t);
         st_stream(&P.pp[(size_t)T.b0 * 32 + sl], p, pol);
         const float q = L.valid ? St.q[L.tree - t_lo] : 0.f;
@@ -1529,9 +1573,9 @@ constexpr int kBThreads = DGR_BTHREADS;
 #define DGR_BPERSM 5
 #endif
 constexpr int kBPerSM = DGR_BPERSM;
-constexpr size_t kTailBytes = 12 * kPipeTrees + 16;   // dq limbs, mbarrier
+constexpr size_t kTailBytes = 12 * kPipeTrees + 16 + 4 * kBThreads;   // dq limbs, mbarrier, tree noise words
 constexpr size_t kBSmemBytes = (StageLayout::bytes + kTailBytes) > kSmemBytes ? (StageLayout::bytes + kTailBytes) : kSmemBytes;
-static_assert(kGpOffset + 4 * 32 * kTargetBundles <= 2 * 8 * (kWinMax + kWinPad), "event window + path noise must fit the S window");
+static_assert(kGpOffset + 4 * 32 * kTargetBundles + 32 <= 2 * 8 * (kWinMax + kWinPad), "event window + path noise must fit the S window");
 
 template <bool REV, bool FWD>
 __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepArgs A) {
@@ -1577,6 +1621,7 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
   const uint32_t mte = (int)threadIdx.x < T.nmn ? __ldg(P.mnets + T.mn0 + threadIdx.x) : kNoTreeLane;
   __syncthreads();
   griddep_wait();   // S, logits, q and the event grids come from the previous kernels
+  uint32_t* twd = reinterpret_cast<uint32_t*>(bar + 2);   // the net level's tree noise words
 #if DGR_LSU_STAGE == 2
   // the eight 1-D arrays by bulk copies (8 per tile: few and large), the S window by cp.async
   if (threadIdx.x < 32) {
@@ -1586,6 +1631,24 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
     if (REV && (P.pf & 3)) prefetch_tile(P, T, (P.pf & 1) != 0);
   }
   lsu_tile_loads<REV, kBThreads>(P, T, smem, false);
+  // the net level's tree noise (stream 1, keyed on the global tree id: plan data and the iteration
+  // only), drawn while the stage is in flight: off that phase's critical path.  Raw
+  // Philox words, one per tree lane, read back by the same thread.
+  if (FWD && (int)threadIdx.x < T.nmn) {   // whole warps (nmn is a multiple of 32)
+    const int lane = threadIdx.x & 31;
+    const bool tv = mte != kNoTreeLane;
+    const int j = T.tree0 + (int)(mte & 1023u) - (T.tree0 & ~3);   // stage index, as in the net level
+    const uint32_t hm = __ballot_sync(kFull, !tv || (mte >> 31));
+    const int head = 31 - __clz(hm & (kFull >> (31 - lane)));
+    const int jh = __shfl_sync(kFull, j, head);
+    if (tv) {
+      const int nrel = (int)((mte >> 10) & 2047u);
+      const int64_t gj = P.tree_base + (P.perm_id ? (int64_t)(T.tree0 + (int)(mte & 1023u))
+                                                  : (int64_t)__ldg(&P.net_gtree[T.net0 + nrel]) + (j - jh));
+      const uint4 r = philox_rk(make_uint4((uint32_t)(gj >> 2), (uint32_t)(gj >> 34), (uint32_t)A.k_next, 1u), P.rk);
+      twd[threadIdx.x] = (gj & 3) == 0 ? r.x : (gj & 3) == 1 ? r.y : (gj & 3) == 2 ? r.z : r.w;
+    }
+  }
   asm volatile("cp.async.wait_group 0;" ::: "memory");
   mbar_wait(bar, 0u);
   __syncthreads();
@@ -1602,7 +1665,7 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
   mbar_wait(bar, 0u);
 #endif
   stamp(P, tix, 1);
-  if (!(KO(16))) process_tile<REV, FWD, kBThreads>(P, A, T, St, ev_s, gp, dq3, ld_first, mte);
+  if (!(KO(16))) process_tile<REV, FWD, kBThreads>(P, A, T, St, ev_s, gp, dq3, ld_first, mte, twd);
   if (KO(256)) __syncthreads();   // (diagnostics: the flush of every warp is done)
   stamp(P, tix, 5);
   if (threadIdx.x == 0) bulk_wait_read();   // the stage must outlive the bulk stores' reads
