@@ -1084,13 +1084,15 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
 
   // ---------------- reverse of iteration k ----------------
   if (REV && !(KO(64))) {   // dq3 was zeroed before the stage arrived
-    const uint32_t* LD = P.ldesc + (size_t)T.b0 * 32 + lane;   // lane descriptors, prefetched a bundle ahead
+    // lane descriptors, prefetched a bundle ahead (LDn: this warp's next bundle's)
+    const uint32_t* LDn = P.ldesc + ((size_t)T.b0 + warp + NW) * 32 + lane;
     uint32_t ldn = ld_first;   // the first one was loaded before the stage wait
     for (int lb = warp; lb < T.nb; lb += NW) {
       const int4 bi = St.bi[lb];
       const uint32_t pw = St.pw[lb * 32 + lane];
       const uint32_t ld = ldn;
-      if (lb + NW < nbg) ldn = __ldg(LD + (lb + NW) * 32);
+      if (lb + NW < nbg) ldn = __ldg(LDn);
+      LDn += NW * 32;
       if (lb < nbg) {
         Lane L;
         lane_from_desc(bi, pw, ld, L);
@@ -1255,13 +1257,15 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
   if (FWD) {
     const uint32_t ev_base = smem_u32(ev_s);
     const int gsh = noise_shift(P, T);
-    const uint32_t* LD = P.ldesc + (size_t)T.b0 * 32 + lane;   // lane descriptors, prefetched a bundle ahead
+    // lane descriptors, prefetched a bundle ahead (LDn: this warp's next bundle's)
+    const uint32_t* LDn = P.ldesc + ((size_t)T.b0 + warp + NW) * 32 + lane;
     uint32_t ldn = ld_fwd;
     for (int lb = warp; lb < T.nb; lb += NW) {
       const int4 bi = St.bi[lb];
       const uint32_t pw = St.pw[lb * 32 + lane];
       const uint32_t ld = ldn;
-      if (lb + NW < nbg) ldn = __ldg(LD + (lb + NW) * 32);
+      if (lb + NW < nbg) ldn = __ldg(LDn);
+      LDn += NW * 32;
       if (lb < nbg) {
         Lane L;
         lane_from_desc(bi, pw, ld, L);
@@ -1283,11 +1287,12 @@ __device__ __forceinline__ void process_tile(const KParams& P, const StepArgs& A
           // Z(o, m) form a cell (a, b) of orientation o (a along the primary lines) is at a A + b B
           // with (A, B) = (1, ww) for o = 0 and (ww, 1) for o = 1, so the segment ends of one line
           // are ordered like their cell indices
-          const int A_ = o ? ep : 1, B_ = o ? 1 : ep;
-          const int p0 = o ? e.y : e.x, p1 = o ? e.w : e.z, q0 = o ? e.x : e.y, q1 = o ? e.z : e.w;
-          const int cp0 = p0 * A_ + q0 * B_ + eb, cp1 = p1 * A_ + q1 * B_ + eb;
-          const int cm0 = m * A_ + q0 * B_ + eb, cm1 = m * A_ + q1 * B_ + eb;
-          const int fP = o ? hv : 0, fS = o ? 0 : hv;   // fields of the primary / secondary lines
+          // (the sub-net's end cells need no orientation; a step along the primary lines is A_)
+          const int A_ = o ? ep : 1;
+          const int p0 = o ? e.y : e.x, p1 = o ? e.w : e.z;
+          const int cp0 = e.y * ep + e.x + eb, cp1 = e.w * ep + e.z + eb;
+          const int cm0 = cp0 + (m - p0) * A_, cm1 = cp1 + (m - p1) * A_;
+          const int fP = o ? hv : 0, fS = hv - fP;   // fields of the primary / secondary lines
           // each segment: +v at its lower end, -v at its upper end (nothing if zero-length)
           const int v1 = cm0 != cp0 ? vq : 0, v2 = cm1 != cm0 ? vq : 0, v3 = cp1 != cm1 ? vq : 0;
 #if !defined(DGR_EXP_SKIP_EVENTS)   // (timing experiments only: results invalid when defined)
@@ -1586,7 +1591,7 @@ __global__ void __launch_bounds__(kBThreads, kBPerSM) tile_bulk(KParams P, StepA
   griddep_launch();
   if ((int)blockIdx.x < P.ntiles_slow) {   // global tiles first: the longest CTAs start earliest
     griddep_wait();
-    slow_tile<REV, FWD>(P, A, P.tiles_slow[blockIdx.x], smem);
+    if (!(KO(512))) slow_tile<REV, FWD>(P, A, P.tiles_slow[blockIdx.x], smem);   // (knock-out 512: timing only)
     return;
   }
   if ((int)blockIdx.x < P.ntiles_slow + P.ngen_blocks) {   // general nets (row f4'): a warp per net

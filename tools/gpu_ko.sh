@@ -1,6 +1,6 @@
 #!/bin/bash
 # KBF knock-out table (timing only, results invalid): a -DDGR_DIAG=1 build timed with each phase of the
-# tile kernel switched off (DGR_DEBUG_SKIP bits: 1 flush, 2 path noise, 4 forward events, 8 path cost,
+# tile kernel switched off (DGR_DEBUG_SKIP bits: 1 flush, 2 path noise, 4 forward events, 8 path cost, 512 global tiles,
 # 16 whole tile body, 32 S window, 64 reverse, 128 net level); the marginal cost of each phase.
 # usage: tools/gpu_ko.sh TAG [CONFIG] [skip values...]
 TAG=${1:-ko}; CFG=${2:-ispd19}; shift; shift
