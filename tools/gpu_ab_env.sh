@@ -8,7 +8,7 @@ for round in 1 2; do
   for cfg in $CFGS; do
     for e in "$@"; do
       if [ "$e" = - ]; then python tools/ab_time.py $cfg 200 3 | sed 's/^/{"env": "-", "d": /; s/$/}/'
-      else env $e python tools/ab_time.py $cfg 200 3 | sed "s/^/{\"env\": \"$e\", \"d\": /; s/\$/}/"; fi
+      else env $e python tools/ab_time.py $cfg 200 3 | sed "s|^|{\"env\": \"$e\", \"d\": |; s|\$|}|"; fi
     done
   done
 done 2>&1 | grep -v Warning | tee $O/ab.jsonl | python -c "
