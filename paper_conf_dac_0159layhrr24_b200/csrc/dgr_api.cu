@@ -632,8 +632,12 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
   std::vector<std::vector<int64_t>> cstarts(nchunk);
   std::vector<std::vector<char>> cglobs(nchunk);
   std::vector<int64_t> cbad(nchunk, -1);
+  auto greedy = [&](const int tgt) {
 #pragma omp parallel for schedule(dynamic, 1)
   for (int64_t ch = 0; ch < nchunk; ++ch) {
+    cstarts[ch].clear();
+    cglobs[ch].clear();
+    cbad[ch] = -1;
     const int64_t pa = ch * kChunkNets, pb = std::min(nn, pa + kChunkNets);
     Cur cur;
     for (int64_t pn = pa; pn < pb; ++pn) {
@@ -674,6 +678,21 @@ int make_plan(const dgr_forest_desc* d, int rank, int world, Plan& pl) {
       cur.bx0 = bx0; cur.by0 = by0; cur.bx1 = bx1; cur.by1 = by1;
       pack_net(n, cur.pk);
       if ((cur.pk.total() > kMaxBundles || ntree > kTreeMax) && cbad[ch] < 0) cbad[ch] = n;
+    }
+  }
+  };
+  greedy(tgt);
+  // Between one and three waves of resident tiles the last wave runs part-empty: shrink the tiles
+  // so the pipelined tiles fill whole waves (ispd18-sized forests: 1.45 waves of 32-bundle tiles ->
+  // 24-bundle tiles, +3% same-box, profiles/r02_ab_tile_target_waves.jsonl)
+  if (tgt == kTargetBundles && !getenv("DGR_TILE_BUNDLES")) {
+    int64_t npipe = 0;
+    for (int64_t ch = 0; ch < nchunk; ++ch)
+      for (char g : cglobs[ch]) npipe += (g == 0);
+    const double waves = (double)npipe / (148.0 * 5.0);
+    if (waves > 1.0 && waves < 3.0) {
+      const int t2 = std::max(16, (int)std::ceil(kTargetBundles * waves / std::ceil(waves)));
+      if (t2 < tgt) greedy(t2);
     }
   }
   std::vector<int64_t> starts;
